@@ -1,0 +1,215 @@
+/*
+ * photon.h — C ABI of libphoton, the B200 (sm_100a) hot path of Photon's online analysis.
+ *
+ * Source of the method: Liu, Sun, Carlson, "Photon: A Fine-grained Sampled Simulation Methodology for GPU
+ * Workloads", MICRO '23 (text at PAPER.md; "L<n>" below = a line of that text plus its section/figure/equation).
+ * Readings of passages the paper leaves silent or garbled are tagged [P-n]; the register is DESIGN.md §3.
+ *
+ * Conventions (apply to every entry point):
+ *  - Every array pointer is a DEVICE pointer unless its comment says HOST.  The caller owns all inputs, outputs
+ *    and workspaces; the library never allocates or frees device memory.
+ *  - `stream` is a cudaStream_t passed as void* (NULL = legacy default stream).  Calls only ENQUEUE work on it and
+ *    never synchronise, except photon_check (documented below) and the *_count helpers that say "syncs".
+ *  - Return value: PHOTON_OK or a negative photon_status.  Host-detectable errors (NULL pointers, sizes, params,
+ *    workspace too small) return immediately and enqueue nothing.  Errors only the device can see (a BB id out of
+ *    range, non-monotone offsets, a full hash table, an exactness bound exceeded, ...) are LATCHED in the call's
+ *    workspace (first error wins: code + element index) and reported by photon_check().
+ *  - Outputs are bit-identical across runs, devices, shard counts, and to the CPU oracle (oracle/).
+ *  - A photon_ctx is owned by one host thread and one CUDA device.  No C++ exception crosses this ABI.
+ */
+#ifndef PHOTON_H
+#define PHOTON_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define PHOTON_ABI_VERSION 1
+#define PHOTON_BINS 16 /* "project these BBVs into fixed-size BBVs (We use 16)" — L178 §3 Obs. 5 */
+
+typedef enum {
+  PHOTON_OK = 0,
+  PHOTON_EINVAL = -1,    /* bad host-side argument: NULL pointer, size or parameter out of range             */
+  PHOTON_ECUDA = -2,     /* CUDA runtime / launch error; text via photon_last_error                             */
+  PHOTON_ERANGE = -3,    /* device-detected bad input: bb >= n_bb, offsets not monotone, retire < issue,
+                            records not retire-sorted, time >= 2^40, per-warp insts >= 2^32, N_k >= 2^50       */
+  PHOTON_ECAPACITY = -4, /* a workspace table (warp types, candidate pairs) is full: retry with a larger one    */
+  PHOTON_EWORKSPACE = -5 /* ws_bytes smaller than the matching photon_*_workspace_bytes()                       */
+} photon_status;
+
+typedef struct photon_ctx photon_ctx; /* opaque host object; owns no device memory */
+
+int photon_abi_version(void);
+/* Creates a context bound to `cuda_device` (reads its SM count).  Returns PHOTON_ECUDA without a usable device. */
+int photon_create(photon_ctx **out, int cuda_device);
+void photon_destroy(photon_ctx *ctx);
+/* Host string describing the most recent error of this ctx; valid until the next call on it. */
+const char *photon_last_error(const photon_ctx *ctx);
+/* SYNCHRONISES `stream`, then reads the device error latch of the most recent call that used a workspace.
+ * Returns that call's device status (PHOTON_OK if none); *bad_index (may be NULL) receives the offending element
+ * index (event, warp, record, kernel or slot, per the code) or -1. */
+int photon_check(photon_ctx *ctx, void *stream, int64_t *bad_index);
+
+/* ------------------------------------------------------------------------------------------------------------
+ * Input 1: the functional basic-block trace of the analysed (sampled) warps, CSR by kernel then by warp.
+ * Paper: the online analysis functionally simulates a sample of warps (1%, L208/L258) and records, per warp, the
+ * sequence of executed basic blocks; a BB is identified by its start PC (L105, L161) and has a length in
+ * instructions.  The trace IS that sample [P-21]: W counts the traced warps.
+ * ---------------------------------------------------------------------------------------------------------- */
+typedef struct {
+  uint32_t n_kernels;              /* K >= 1, kernels in launch order                                              */
+  uint32_t n_bb;                   /* B, 1 <= B <= 65536 (global BB-id space)                                      */
+  uint64_t n_warps;                /* W  (< 2^40)                                                                  */
+  uint64_t n_events;               /* E  (< 2^48)                                                                  */
+  const uint64_t *kernel_warp_off; /* [K+1] non-decreasing, [0]=0, [K]=W: kernel k owns warps [off[k],off[k+1])    */
+  const uint64_t *warp_event_off;  /* [W+1] non-decreasing, [0]=0, [W]=E: warp w owns events [off[w],off[w+1])     */
+  const uint16_t *bb;              /* [E] BB id per event, execution order within a warp; 16-byte aligned          */
+  const uint32_t *bb_len;          /* [B] instructions per BB, 1 <= len < 2^18                                     */
+  const uint8_t *bb_bin;           /* [B] projection bin (< 16) of each BB [P-2]; NULL => bin(b) = b & 15          */
+} photon_trace;
+
+/* Canonical warp-type tables (output of photon_warp_group / photon_types_merge).  Capacity is `capacity` rows
+ * (types), at most n_warps are ever needed.  Row order: kernel-major (CSR by kernel_type_off), within a kernel by
+ * (count descending, key lexicographically ascending) [P-4]; row 0 of a kernel is its dominant type. */
+typedef struct {
+  uint64_t capacity;          /* rows allocated in type_key/type_count/type_first_warp                          */
+  uint32_t *warp_type;        /* [W] kernel-local canonical type id of each warp (0 = dominant); may be NULL for
+                                 photon_types_merge                                                             */
+  uint64_t *kernel_type_off;  /* [K+1] CSR: kernel k owns rows [off[k], off[k+1]); off[K] = total types T       */
+  uint32_t *type_key;         /* [capacity][16] projected 16-bin BBV of the type (L178) [P-3]                   */
+  uint64_t *type_count;       /* [capacity] warps of the type, c_t (L178 "portion of warps")                   */
+  uint64_t *type_first_warp;  /* [capacity] lowest (global) warp index with this type                          */
+  uint8_t *warp_sampling_ok;  /* [K] 1 iff 100*c_0 > 95*W_k: dominant type holds MORE than 95% (L249) [P-15]   */
+} photon_types;
+
+/* ---- A1: per-warp BBV projected to 16 bins (L154, L161, L178) [P-1][P-2] -------------------------------------
+ * p_w[j] = sum over events e of warp w with bin(bb[e]) == j of bb_len[bb[e]]    (u32; warp_insts I_w = sum_j p_w[j])
+ * kernel_bb_insts[k][b] = sum over warps w of kernel k of count_w(b) * bb_len[b]  (the BB distribution, L208-210)
+ * Any output may be NULL (not computed).  Device errors: ERANGE (bb >= n_bb: index = event; non-monotone
+ * warp_event_off / kernel_warp_off: index = warp / kernel; I_w >= 2^32: index = warp). */
+size_t photon_bbv_workspace_bytes(const photon_trace *trace);
+int photon_bbv_build(photon_ctx *ctx, const photon_trace *trace, void *ws, size_t ws_bytes,
+                     uint32_t *warp_bbv16 /*[W][16] or NULL*/, uint64_t *warp_insts /*[W] or NULL*/,
+                     uint64_t *kernel_bb_insts /*[K][B] or NULL*/, void *stream);
+
+/* ---- A2: warp-type grouping + dominance decision (L154, L178, L249) ------------------------------------------
+ * Warps of one kernel with equal projected keys form one type [P-3]; canonical order [P-4]; weight_t = c_t / W_k
+ * (L178); warp_sampling_ok per L249 [P-15].  warp_bbv16 == NULL runs the fused single-pass path (A1+A2 in one
+ * streaming kernel); otherwise keys are read from warp_bbv16 (the unfused path).  The workspace holds an
+ * open-addressing hash table sized from `type_capacity_hint` (expected total types; 0 => a default of
+ * min(W, 2^20)); if it fills, the call latches PHOTON_ECAPACITY and the caller retries with a larger hint.
+ * out->capacity must be >= the number of types found (ECAPACITY otherwise). */
+size_t photon_group_workspace_bytes(const photon_trace *trace, uint64_t type_capacity_hint);
+int photon_warp_group(photon_ctx *ctx, const photon_trace *trace, const uint32_t *warp_bbv16 /*or NULL*/, void *ws,
+                      size_t ws_bytes, photon_types *out, void *stream);
+/* SYNCS the stream and returns kernel_type_off[K] (total types) in *total_types (HOST). */
+int photon_types_total(photon_ctx *ctx, const photon_types *types, uint32_t n_kernels, uint64_t *total_types,
+                       void *stream);
+
+/* ---- A3 + A4: GPU-BBV signature and kernel matching (L159 Fig 5, L178, L271 Fig 12) ---------------
+ * Signature of kernel k [P-4][P-5]: g_k = concat over its types r = 0..T_k-1 (canonical order) of c_r*key_r[0..15]
+ * (u64); mass N_k = sum g_k.  The normalised GPU BBV is g_k / N_k.
+ * Distance [P-6]: D(k,r) = sum_i |g_k[i]/N_k - g_r[i]/N_r| over position-aligned, zero-padded signatures.
+ * Close: D < theta = theta_num/theta_den [P-7][P-15], decided exactly as
+ *        theta_den * sum_i |g_k[i]*N_r - g_r[i]*N_k| < theta_num * N_k * N_r   (u128; N = 0 never matches [P-19]).
+ * Warp rule [P-10] (L271 Fig 12 note, L277): (W_k == W_r) or min(W_k, W_r) >= n_cores, with W = warps_total.
+ * For k in launch order: cand = { r < k : r in pool, close, warp rule } where pool = representatives (kernels
+ * that were not themselves matched) [P-8] or all prior kernels when pool_all_prior = 1.  cand empty => k is a
+ * representative, match[k] = -1; else match[k] = argmin over cand of (|W_k - W_r|, r) [P-9] ("closest warp
+ * count", L271 Step 3).  match_dist[k] = D(k, match[k]) in fp64 (rel. err < 1e-6), +inf for representatives.
+ * Device errors: ERANGE (N_k >= 2^50, index = kernel); ECAPACITY (candidate-pair table full). */
+typedef struct {
+  uint32_t theta_num, theta_den; /* theta = num/den; default 1/20; 1 <= den <= 2^20, num <= 2*den               */
+  uint64_t n_cores;              /* equal-warp rule below this count; default 64 (R9 Nano CUs, Table 1)    */
+  uint32_t pool_all_prior;       /* 0 = representatives only (default) [P-8]; 1 = every prior kernel           */
+} photon_match_params;
+
+/* Workspace for K kernels, T total types and room for `pair_capacity` close pairs (0 => default 16*K + 65536). */
+size_t photon_match_workspace_bytes(uint32_t n_kernels, uint64_t total_types, uint64_t pair_capacity);
+int photon_kernel_match(photon_ctx *ctx, uint32_t n_kernels, const photon_types *types,
+                        const uint64_t *warps_total /*[K]*/, photon_match_params params, void *ws, size_t ws_bytes,
+                        int64_t *match /*[K]*/, double *match_dist /*[K] or NULL*/, void *stream);
+
+/* Split form of photon_kernel_match, used by the multi-GPU driver (signatures all-reduced, pair lists
+ * all-gathered between the steps).  sig_build writes g and N only for kernels [k_lo, k_hi) (others untouched).
+ * match_scan appends the close pairs (k, r) with k in [k_lo, k_hi) to pairs[] (u64: k << 32 | r), count in
+ * *n_pairs (DEVICE u64, zeroed by the call); `pair_capacity` entries fit.  match_resolve takes the union of all
+ * pair lists (any order) and runs the launch-order resolution; its result does not depend on pair order. */
+int photon_sig_build(photon_ctx *ctx, uint32_t n_kernels, const uint64_t *kernel_type_off, const uint32_t *type_key,
+                     const uint64_t *type_count, uint32_t k_lo, uint32_t k_hi, uint64_t *sig /*[16*T]*/,
+                     uint64_t *mass /*[K]*/, void *stream);
+int photon_match_scan(photon_ctx *ctx, uint32_t n_kernels, const uint64_t *kernel_type_off, const uint64_t *sig,
+                      const uint64_t *mass, const uint64_t *warps_total, photon_match_params params, uint32_t k_lo,
+                      uint32_t k_hi, void *ws, size_t ws_bytes, uint64_t *pairs, uint64_t pair_capacity,
+                      uint64_t *n_pairs, void *stream);
+int photon_match_resolve(photon_ctx *ctx, uint32_t n_kernels, const uint64_t *kernel_type_off, const uint64_t *sig,
+                         const uint64_t *mass, const uint64_t *warps_total, photon_match_params params,
+                         const uint64_t *pairs, uint64_t n_pairs, void *ws, size_t ws_bytes, int64_t *match,
+                         double *match_dist, void *stream);
+
+/* ---- A5: per-BB stability test + BB-sampling switch (L208-210 Fig 7, L220-229 Eq. 1) -------------------
+ * Timing stream: one record per retired BB execution of the detailed simulation, CSR by kernel, each kernel's
+ * records sorted by retire time (ties keep input order) [P-18]; times are integer ticks < 2^40 [P-16].
+ * For each kernel k and BB type b, walk b's executions in stream order.  At its j-th execution (1-based) with
+ * j >= 2n (n = window_n, L229) [P-11], over the last n executions (x = issue, y = retire):
+ *   cond1 (Eq. 1; |1-a| < delta, L229):  den > 0 and delta_den*|den - num| < delta_num*den,
+ *          num = n*Sxy - Sx*Sy, den = n*Sxx - Sx^2   (exact i128)                                  [P-16]
+ *   cond2 (mean check, L229) [P-12][P-17]:  S_2n > 0 and delta_den*|2*S_n - S_2n| < delta_num*S_2n,
+ *          S_m = sum of (retire - issue) over the last m executions.
+ * The first such execution latches b stable [P-13]: first_stable[k][b] = its position in kernel k's stream
+ * (0-based record index relative to kernel_rec_off[k]) and stable_dur_sum[k][b] = S_n; else -1 / 0.
+ * Switch (L208, Fig 7) [P-14][P-15]: order k's stable BBs by position; switch_at[k] = the first position at
+ * which 100 * sum of their weights > 95 * (total weight), weights = kernel_bb_insts[k][*]; -1 if never or if
+ * the total is 0.  rate_num/rate_den replaces 95/100.
+ * Device errors: ERANGE (bb >= n_bb, retire < issue, retire decreasing within a kernel, time >= 2^40,
+ * non-monotone kernel_rec_off; index = record or kernel). */
+typedef struct {
+  uint32_t n_kernels, n_bb;        /* K, B as in the trace                                                      */
+  uint64_t n_records;              /* R (< 2^32)                                                                */
+  const uint64_t *kernel_rec_off;  /* [K+1]                                                                     */
+  const uint16_t *bb;              /* [R]                                                                       */
+  const uint64_t *issue, *retire;  /* [R] ticks                                                                 */
+} photon_timing;
+typedef struct {
+  uint32_t window_n;             /* n, default 2048 (L229); 2 <= n <= 8192                                     */
+  uint32_t delta_num, delta_den; /* delta, default 3/100 (L229); 1 <= den <= 2^16, num <= den                  */
+  uint32_t rate_num, rate_den;   /* switch rate, default 95/100 (L208); 1 <= den <= 2^16, num <= den           */
+} photon_stable_params;
+
+size_t photon_stable_workspace_bytes(const photon_timing *timing);
+int photon_bb_stable(photon_ctx *ctx, const photon_timing *timing, const uint64_t *kernel_bb_insts /*[K][B]*/,
+                     photon_stable_params params, void *ws, size_t ws_bytes, int64_t *first_stable /*[K][B]*/,
+                     uint64_t *stable_dur_sum /*[K][B] or NULL*/, int64_t *switch_at /*[K]*/, void *stream);
+
+/* ---- Multi-GPU merge helpers ------------------------------------------------------------------
+ * A shard is a contiguous warp range of the global trace; its local kernel l is global kernel kernel_base + l and
+ * its local warp v is global warp warp_base + v.  Rows exchanged between ranks (88 bytes each):       */
+typedef struct {
+  uint32_t kernel;     /* global kernel id */
+  uint32_t pad;
+  uint32_t key[16];
+  uint64_t count;
+  uint64_t first_warp; /* global warp index */
+} photon_type_row;
+/* Writes the local types as rows (global ids) to rows[0..T_local); T_local = local->kernel_type_off[K_local]. */
+int photon_types_export(photon_ctx *ctx, uint32_t n_kernels_local, const photon_types *local, uint32_t kernel_base,
+                        uint64_t warp_base, photon_type_row *rows, void *stream);
+/* Merges rows of all shards (any order; rows with equal (kernel, key) add counts and take the min first_warp)
+ * into canonical global tables for K kernels; `kernel_warps` [K] = analysed warps per kernel (for the dominance
+ * decision).  global->warp_type is ignored. */
+size_t photon_merge_workspace_bytes(uint64_t n_rows, uint32_t n_kernels);
+int photon_types_merge(photon_ctx *ctx, const photon_type_row *rows, uint64_t n_rows, uint32_t n_kernels,
+                       const uint64_t *kernel_warps, void *ws, size_t ws_bytes, photon_types *global, void *stream);
+/* warp_type_global[v] = global canonical id of local warp v's type.  ws from photon_merge_workspace_bytes of the
+ * same merge (its lookup table is reused; pass the same ws that the merge used, unmodified). */
+int photon_types_remap(photon_ctx *ctx, uint32_t n_kernels_local, uint64_t n_warps_local,
+                       const photon_types *local, const photon_types *global, uint32_t kernel_base, const void *ws,
+                       size_t ws_bytes, uint32_t *warp_type_global, void *stream);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* PHOTON_H */

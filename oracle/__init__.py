@@ -1,0 +1,160 @@
+"""CPU oracle for the Photon online-analysis hot path — TEST INFRASTRUCTURE ONLY.
+
+Only tests/, __graft_entry__.smoke() and bench.py (cpu_baseline leg, --impl reference) may import this package.
+The product path (paper_conf_micro_liusc23_b200) never imports it and shares no code with it.
+
+The arithmetic lives in photon_oracle.cpp (plain single-threaded C++17, each function citing PAPER.md); this
+module only marshals numpy arrays.  Pins: tests/test_oracle_pins.py.  Parity unpinned by the paper (no paper
+number exists for them): theta [P-7] and the readings [P-2], [P-5], [P-6], [P-8] — DESIGN.md §3.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+import subprocess
+from typing import Optional
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+_SO = os.path.join(_HERE, "liboracle.so")
+_SRC = os.path.join(_HERE, "photon_oracle.cpp")
+
+OK, EINVAL, ERANGE, ECAPACITY = 0, -1, -3, -4
+
+
+class OracleError(RuntimeError):
+    def __init__(self, code: int, index: int):
+        super().__init__(f"oracle error {code} at index {index}")
+        self.code = code
+        self.index = index
+
+
+def build(force: bool = False) -> str:
+    if force or not os.path.exists(_SO) or os.path.getmtime(_SO) < os.path.getmtime(_SRC):
+        subprocess.check_call(["g++", "-O2", "-std=c++17", "-shared", "-fPIC", "-o", _SO, _SRC])
+    return _SO
+
+
+_lib = None
+
+
+def _L():
+    global _lib
+    if _lib is None:
+        build()
+        L = ctypes.CDLL(_SO)
+        vp, u32, u64, i32 = ctypes.c_void_p, ctypes.c_uint32, ctypes.c_uint64, ctypes.c_int
+        L.or_bbv.restype = i32
+        L.or_bbv.argtypes = [u32, u32, u64, u64, vp, vp, vp, vp, vp, vp, vp, vp, vp]
+        L.or_group.restype = i32
+        L.or_group.argtypes = [u32, u64, vp, vp, u64, vp, vp, vp, vp, vp, vp]
+        L.or_signature.restype = i32
+        L.or_signature.argtypes = [u32, vp, vp, vp, vp, vp, vp]
+        L.or_match.restype = i32
+        L.or_match.argtypes = [u32, vp, vp, vp, vp, u32, u32, u64, u32, vp, vp]
+        L.or_stable.restype = i32
+        L.or_stable.argtypes = [u32, u32, u64, vp, vp, vp, vp, vp, u32, u32, u32, u32, u32, i32, vp, vp, vp, vp]
+        _lib = L
+    return _lib
+
+
+def _p(a: Optional[np.ndarray]):
+    return None if a is None else a.ctypes.data
+
+
+def _c(a, dt):
+    return np.ascontiguousarray(a, dtype=dt)
+
+
+def bbv(trace, want_kbb: bool = True):
+    """A1: (warp_bbv16 [W,16] u32, warp_insts [W] u64, kernel_bb_insts [K,B] u64 or None)."""
+    K, B, W, E = trace.n_kernels, trace.n_bb, trace.n_warps, trace.n_events
+    p16 = np.zeros((W, 16), np.uint32)
+    ins = np.zeros(W, np.uint64)
+    kbb = np.zeros((K, B), np.uint64) if want_kbb else None
+    bad = ctypes.c_int64(-1)
+    bbin = None if trace.bb_bin is None else _c(trace.bb_bin, np.uint8)
+    kwo, weo = _c(trace.kernel_warp_off, np.uint64), _c(trace.warp_event_off, np.uint64)
+    bbs, bl = _c(trace.bb, np.uint16), _c(trace.bb_len, np.uint32)
+    rc = _L().or_bbv(K, B, W, E, _p(kwo), _p(weo), _p(bbs), _p(bl), _p(bbin), _p(p16), _p(ins), _p(kbb),
+                     ctypes.byref(bad))
+    if rc != OK:
+        raise OracleError(rc, bad.value)
+    return p16, ins, kbb
+
+
+def group(trace, warp_bbv16: np.ndarray):
+    """A2: canonical type tables (dict of numpy arrays, names as photon_types)."""
+    K, W = trace.n_kernels, trace.n_warps
+    cap = max(W, 1)
+    out = dict(warp_type=np.zeros(W, np.uint32), kernel_type_off=np.zeros(K + 1, np.uint64),
+               type_key=np.zeros((cap, 16), np.uint32), type_count=np.zeros(cap, np.uint64),
+               type_first_warp=np.zeros(cap, np.uint64), warp_sampling_ok=np.zeros(K, np.uint8))
+    kwo = _c(trace.kernel_warp_off, np.uint64)
+    p16 = _c(warp_bbv16, np.uint32)
+    rc = _L().or_group(K, W, _p(kwo), _p(p16), cap, _p(out["warp_type"]), _p(out["kernel_type_off"]),
+                       _p(out["type_key"]), _p(out["type_count"]), _p(out["type_first_warp"]),
+                       _p(out["warp_sampling_ok"]))
+    if rc != OK:
+        raise OracleError(rc, -1)
+    T = int(out["kernel_type_off"][-1])
+    for k in ("type_key", "type_count", "type_first_warp"):
+        out[k] = out[k][:T].copy()
+    return out
+
+
+def signature(kernel_type_off, type_key, type_count):
+    """A3: (sig [16T] u64, mass [K] u64)."""
+    kto = _c(kernel_type_off, np.uint64)
+    K = len(kto) - 1
+    T = int(kto[-1])
+    sig = np.zeros(max(16 * T, 1), np.uint64)
+    mass = np.zeros(max(K, 1), np.uint64)
+    bad = ctypes.c_int64(-1)
+    rc = _L().or_signature(K, _p(kto), _p(_c(type_key, np.uint32)), _p(_c(type_count, np.uint64)), _p(sig),
+                           _p(mass), ctypes.byref(bad))
+    if rc != OK:
+        raise OracleError(rc, bad.value)
+    return sig[:16 * T], mass[:K]
+
+
+def match(kernel_type_off, sig, mass, warps_total, theta=(1, 20), n_cores=64, pool_all_prior=0):
+    """A4: (match [K] i64, match_dist [K] f64)."""
+    kto = _c(kernel_type_off, np.uint64)
+    K = len(kto) - 1
+    m = np.zeros(max(K, 1), np.int64)
+    d = np.zeros(max(K, 1), np.float64)
+    sg = _c(sig, np.uint64) if len(sig) else np.zeros(1, np.uint64)
+    rc = _L().or_match(K, _p(kto), _p(sg), _p(_c(mass, np.uint64)), _p(_c(warps_total, np.uint64)),
+                       int(theta[0]), int(theta[1]), int(n_cores), int(pool_all_prior), _p(m), _p(d))
+    if rc != OK:
+        raise OracleError(rc, -1)
+    return m[:K], d[:K]
+
+
+def stable(timing, kernel_bb_insts, n=2048, delta=(3, 100), rate=(95, 100), brute=False):
+    """A5: (first_stable [K,B] i64, stable_dur_sum [K,B] u64, switch_at [K] i64)."""
+    K, B, R = timing.n_kernels, int(timing.n_bb), timing.n_records
+    fs = np.zeros((K, B), np.int64)
+    ds = np.zeros((K, B), np.uint64)
+    sw = np.zeros(max(K, 1), np.int64)
+    bad = ctypes.c_int64(-1)
+    kbb = _c(kernel_bb_insts, np.uint64)
+    rc = _L().or_stable(K, B, R, _p(_c(timing.kernel_rec_off, np.uint64)), _p(_c(timing.bb, np.uint16)),
+                        _p(_c(timing.issue, np.uint64)), _p(_c(timing.retire, np.uint64)), _p(kbb), int(n),
+                        int(delta[0]), int(delta[1]), int(rate[0]), int(rate[1]), 1 if brute else 0, _p(fs),
+                        _p(ds), _p(sw), ctypes.byref(bad))
+    if rc != OK:
+        raise OracleError(rc, bad.value)
+    return fs, ds, sw[:K]
+
+
+def analyse(trace, theta=(1, 20), n_cores=64, pool_all_prior=0):
+    """The benchmarked chain A1 -> A2 -> A3 -> A4 on one trace; returns a dict of every output."""
+    p16, ins, kbb = bbv(trace, want_kbb=False)
+    t = group(trace, p16)
+    sig, mass = signature(t["kernel_type_off"], t["type_key"], t["type_count"])
+    m, d = match(t["kernel_type_off"], sig, mass, trace.warps_total, theta, n_cores, pool_all_prior)
+    t.update(warp_bbv16=p16, warp_insts=ins, sig=sig, mass=mass, match=m, match_dist=d)
+    return t

@@ -1,0 +1,505 @@
+"""Pins of the CPU oracle against things other than itself (CPU only, -m "not gpu").
+
+Each pin names the PAPER.md passage (L<n>) or the mathematical fact it rests on.  None of them re-calls the
+oracle's own formula: the references are the paper's printed numbers, a hand-worked example, exact Fraction
+arithmetic written independently here, numpy's least squares / bincount, brute force on tiny inputs, and
+invariants (so a dropped term, a wrong sign or index, or a transposed operand fails one of them).
+"""
+import itertools
+import json
+import os
+from fractions import Fraction
+
+import numpy as np
+import pytest
+
+import oracle
+import tracegen as tg
+
+GOLD = os.path.join(os.path.dirname(__file__), "golden")
+
+
+def _gold(name):
+    with open(os.path.join(GOLD, name)) as f:
+        return json.load(f)
+
+
+# ---------------------------------------------------------------------------------------------------------------
+# Worked GPU-BBV example (tests/golden/worked_example.json, derived by hand from L178 + readings)
+def test_worked_example_full_chain():
+    g = _gold("worked_example.json")
+    e = g["expect"]
+    tr = tg.trace_from_warps(g["kernels"], g["bb_len"])
+    p16, ins, kbb = oracle.bbv(tr)
+    assert p16[:, :3].tolist() == e["warp_bbv16_nonzero"] and not p16[:, 3:].any()
+    assert ins.tolist() == e["warp_insts"]
+    assert kbb.tolist() == e["kernel_bb_insts"]
+    t = oracle.group(tr, p16)
+    assert t["warp_type"].tolist() == e["warp_type"]
+    assert t["kernel_type_off"].tolist() == e["kernel_type_off"]
+    assert t["type_key"][:, :3].tolist() == e["type_key_nonzero"]
+    assert t["type_count"].tolist() == e["type_count"]
+    assert t["type_first_warp"].tolist() == e["type_first_warp"]
+    assert t["warp_sampling_ok"].tolist() == e["warp_sampling_ok"]
+    sig, mass = oracle.signature(t["kernel_type_off"], t["type_key"], t["type_count"])
+    assert mass.tolist() == e["mass"]
+    a = {str(i): int(v) for i, v in enumerate(sig[:32]) if v}
+    b = {str(i): int(v) for i, v in enumerate(sig[32:48]) if v}
+    assert a == e["sig_nonzero_A"] and b == e["sig_nonzero_B"]
+    for key, theta, cores in [("match_theta_1_20_cores_64", (1, 20), 64), ("match_theta_1_2_cores_64", (1, 2), 64),
+                              ("match_theta_1_2_cores_2", (1, 2), 2), ("match_theta_4_11_cores_2", (4, 11), 2),
+                              ("match_theta_2_5_cores_2", (2, 5), 2)]:
+        m, d = oracle.match(t["kernel_type_off"], sig, mass, tr.warps_total, theta, cores)
+        assert m.tolist() == e[key], key
+        if m[1] == 0:
+            assert d[1] == pytest.approx(e["D_AB_num"] / e["D_AB_den"], rel=1e-12)
+        assert np.isinf(d[0])
+
+
+# ---------------------------------------------------------------------------------------------------------------
+# A1: BBV.  Pins: invariant sum_j p_w[j] = I_w = sum_e len(bb_e); identity fold for B <= 16 equals the full BBV
+# computed with numpy.bincount; brute-force recount; single-BB warp p = count x len.
+def _brute_bbv(tr):
+    bins = (np.arange(tr.n_bb) & 15) if tr.bb_bin is None else tr.bb_bin
+    out = np.zeros((tr.n_warps, 16), np.int64)
+    for w in range(tr.n_warps):
+        for e in range(int(tr.warp_event_off[w]), int(tr.warp_event_off[w + 1])):
+            b = int(tr.bb[e])
+            out[w, int(bins[b])] += int(tr.bb_len[b])
+    return out
+
+
+@pytest.mark.parametrize("seed,custom", [(1, False), (2, True), (3, True), (4, False)])
+def test_bbv_bruteforce_and_invariants(seed, custom):
+    tr = tg.random_trace(seed, n_kernels=4, max_warps=12, max_events=40, n_bb=40, custom_bins=custom)
+    p16, ins, kbb = oracle.bbv(tr)
+    assert np.array_equal(p16.astype(np.int64), _brute_bbv(tr))
+    for w in range(tr.n_warps):
+        ev = tr.bb[int(tr.warp_event_off[w]):int(tr.warp_event_off[w + 1])]
+        assert int(ins[w]) == int(tr.bb_len[ev.astype(np.int64)].astype(np.int64).sum())
+        assert int(p16[w].astype(np.int64).sum()) == int(ins[w])
+    # BB distribution: rows sum to the kernel's instructions
+    for k in range(tr.n_kernels):
+        w0, w1 = int(tr.kernel_warp_off[k]), int(tr.kernel_warp_off[k + 1])
+        assert int(kbb[k].sum()) == int(ins[w0:w1].sum())
+
+
+def test_bbv_identity_fold_equals_full_bbv():
+    # B <= 16 with the default fold: the projection is the identity, so p_w = full BBV = bincount x len
+    tr = tg.random_trace(7, n_kernels=3, max_warps=10, max_events=60, n_bb=16)
+    p16, _, _ = oracle.bbv(tr)
+    for w in range(tr.n_warps):
+        ev = tr.bb[int(tr.warp_event_off[w]):int(tr.warp_event_off[w + 1])].astype(np.int64)
+        full = np.bincount(ev, minlength=16) * tr.bb_len.astype(np.int64)
+        assert np.array_equal(p16[w].astype(np.int64), full)
+
+
+def test_bbv_single_bb_warp_and_empty_warp():
+    # single-BB warp: p = count x len; empty warp (L231 empty-task warps execute almost nothing): key all zeros
+    tr = tg.trace_from_warps([[[5] * 7, [], [5]]], bb_len=[1] * 5 + [13])
+    p16, ins, _ = oracle.bbv(tr)
+    assert p16[0, 5] == 7 * 13 and p16[0].sum() == 7 * 13
+    assert not p16[1].any() and ins[1] == 0
+    assert p16[2, 5] == 13
+
+
+def test_bbv_range_errors():
+    tr = tg.trace_from_warps([[[0, 1, 9]]], bb_len=[1, 2, 3])  # bb 9 >= B
+    with pytest.raises(oracle.OracleError) as ei:
+        oracle.bbv(tr)
+    assert ei.value.code == oracle.ERANGE and ei.value.index == 2
+    tr = tg.trace_from_warps([[[0], [1]]], bb_len=[1, 2])
+    tr.warp_event_off = np.array([0, 1, 0], np.uint64)  # non-monotone (and [W] != E)
+    with pytest.raises(oracle.OracleError):
+        oracle.bbv(tr)
+    tr = tg.trace_from_warps([[[0] * 3]], bb_len=[(1 << 31) + 5])  # I_w >= 2^32
+    with pytest.raises(oracle.OracleError) as ei:
+        oracle.bbv(tr)
+    assert ei.value.code == oracle.ERANGE and ei.value.index == 0
+
+
+# ---------------------------------------------------------------------------------------------------------------
+# A2: grouping.  Pins: partition (each warp exactly one type, counts sum to W_k); brute-force O(W^2): same type
+# <=> equal key; canonical ids invariant under warp permutation; order = count desc then key asc (checked against
+# Python's sorted on tuples); dominance boundary exactly 95% -> 0, above -> 1 (L249 strict).
+@pytest.mark.parametrize("seed", [11, 12, 13])
+def test_group_partition_bruteforce(seed):
+    tr = tg.random_trace(seed, n_kernels=5, max_warps=30, max_events=20, n_bb=20, custom_bins=True)
+    p16, _, _ = oracle.bbv(tr)
+    t = oracle.group(tr, p16)
+    kto = t["kernel_type_off"]
+    for k in range(tr.n_kernels):
+        w0, w1 = int(tr.kernel_warp_off[k]), int(tr.kernel_warp_off[k + 1])
+        rows = range(int(kto[k]), int(kto[k + 1]))
+        assert sum(int(t["type_count"][r]) for r in rows) == w1 - w0
+        for a, b in itertools.product(range(w0, w1), repeat=2):
+            assert (t["warp_type"][a] == t["warp_type"][b]) == bool(np.array_equal(p16[a], p16[b]))
+        for w in range(w0, w1):
+            assert np.array_equal(t["type_key"][int(kto[k]) + int(t["warp_type"][w])], p16[w])
+        # canonical order by Python's own tuple sort
+        keyed = sorted(((-int(t["type_count"][r]), tuple(int(x) for x in t["type_key"][r])) for r in rows))
+        assert [(-c, key) for c, key in keyed] == [(int(t["type_count"][r]), tuple(int(x) for x in t["type_key"][r]))
+                                                   for r in rows]
+        for r in rows:
+            members = [w for w in range(w0, w1) if np.array_equal(p16[w], t["type_key"][r])]
+            assert t["type_first_warp"][r] == min(members)
+        Wk = w1 - w0
+        dom = int(t["type_count"][int(kto[k])]) if Wk else 0
+        assert t["warp_sampling_ok"][k] == (1 if Wk and Fraction(dom, Wk) > Fraction(95, 100) else 0)
+
+
+def test_group_permutation_invariance():
+    tr = tg.random_trace(21, n_kernels=1, max_warps=40, max_events=15, n_bb=10)
+    p16, _, _ = oracle.bbv(tr)
+    t = oracle.group(tr, p16)
+    perm = np.random.default_rng(5).permutation(tr.n_warps)
+    tr2 = tg.trace_from_warps([[tr.bb[int(tr.warp_event_off[w]):int(tr.warp_event_off[w + 1])].tolist()
+                                for w in perm]], tr.bb_len)
+    p2, _, _ = oracle.bbv(tr2)
+    t2 = oracle.group(tr2, p2)
+    assert np.array_equal(t["type_key"], t2["type_key"]) and np.array_equal(t["type_count"], t2["type_count"])
+    assert np.array_equal(t2["warp_type"], t["warp_type"][perm])
+
+
+@pytest.mark.parametrize("n_dom,n_all,ok", [(19, 20, 0), (95, 100, 0), (96, 100, 1), (20, 20, 1), (1, 1, 1),
+                                            (190, 201, 0), (191, 201, 1)])
+def test_dominance_boundary(n_dom, n_all, ok):
+    # L249 "accounts for more than 95%": strict; 19/20 = 95% exactly -> no warp sampling
+    warps = [[0, 1]] * n_dom + [[0]] * (n_all - n_dom)
+    tr = tg.trace_from_warps([warps], bb_len=[3, 4])
+    p16, _, _ = oracle.bbv(tr)
+    assert oracle.group(tr, p16)["warp_sampling_ok"][0] == ok
+
+
+# ---------------------------------------------------------------------------------------------------------------
+# A3 / A4: signature, distance, matching.  Pins: sum g = N; Fraction distance of the normalised weighted BBVs
+# built here from the type table (independent code); metric properties; strict threshold boundary; brute-force
+# launch-order resolution on random tiny lists; scenario pins.
+def _frac_gpu_bbv(t, k):
+    """GPU BBV of kernel k as Fractions, built the L178 way: weights c_t/W, weighted BBVs listed, then [P-5]
+    scaled to unit mass.  Written independently of the oracle (which works on integers g, N)."""
+    kto = t["kernel_type_off"]
+    rows = range(int(kto[k]), int(kto[k + 1]))
+    W = sum(int(t["type_count"][r]) for r in rows)
+    vec = []
+    for r in rows:
+        wgt = Fraction(int(t["type_count"][r]), W)
+        vec.extend(wgt * int(x) for x in t["type_key"][r])
+    s = sum(vec)
+    return [v / s for v in vec] if s else vec
+
+
+def _frac_dist(a, b):
+    L = max(len(a), len(b))
+    a = a + [Fraction(0)] * (L - len(a))
+    b = b + [Fraction(0)] * (L - len(b))
+    return sum(abs(x - y) for x, y in zip(a, b))
+
+
+def _pipeline(tr):
+    p16, _, _ = oracle.bbv(tr)
+    t = oracle.group(tr, p16)
+    sig, mass = oracle.signature(t["kernel_type_off"], t["type_key"], t["type_count"])
+    return t, sig, mass
+
+
+def test_signature_mass_and_distance_metric_properties():
+    tr = tg.random_trace(31, n_kernels=6, max_warps=12, max_events=12, n_bb=12, dup_p=0.8)
+    t, sig, mass = _pipeline(tr)
+    kto = t["kernel_type_off"]
+    for k in range(tr.n_kernels):
+        assert int(sig[16 * int(kto[k]):16 * int(kto[k + 1])].astype(object).sum()) == int(mass[k])
+    vecs = [_frac_gpu_bbv(t, k) for k in range(tr.n_kernels)]
+    nz = [k for k in range(tr.n_kernels) if mass[k] > 0]
+    for a in nz:
+        assert _frac_dist(vecs[a], vecs[a]) == 0
+        for b in nz:
+            dab = _frac_dist(vecs[a], vecs[b])
+            assert dab == _frac_dist(vecs[b], vecs[a]) and 0 <= dab <= 2
+            for c in nz:
+                assert _frac_dist(vecs[a], vecs[c]) <= dab + _frac_dist(vecs[b], vecs[c])
+    # oracle's reported distance for a forced match (theta = 2 + pool_all_prior) equals the Fraction value
+    for a, b in itertools.combinations(nz, 2):
+        sub = tg.trace_from_warps([_warps_of(tr, a), _warps_of(tr, b)], tr.bb_len)
+        t2, s2, m2 = _pipeline(sub)
+        d_exact = _frac_dist(_frac_gpu_bbv(t2, 0), _frac_gpu_bbv(t2, 1))
+        if d_exact < 2:
+            mm, dd = oracle.match(t2["kernel_type_off"], s2, m2, [1000, 1000], theta=(2, 1), n_cores=64)
+            assert mm[1] == 0 and dd[1] == pytest.approx(float(d_exact), rel=1e-12, abs=0)
+
+
+def _warps_of(tr, k):
+    return [tr.bb[int(tr.warp_event_off[w]):int(tr.warp_event_off[w + 1])].tolist()
+            for w in range(int(tr.kernel_warp_off[k]), int(tr.kernel_warp_off[k + 1]))]
+
+
+def _brute_resolve(vecs, masses, wt, theta, cores, pool_all):
+    """Launch-order leader clustering (L271 Fig 12 Steps 2-3, [P-8][P-9][P-10]) on Fraction distances."""
+    K = len(vecs)
+    rep, match = [False] * K, [-1] * K
+    for k in range(K):
+        best = None
+        for r in range(k):
+            if not (pool_all or rep[r]) or masses[k] == 0 or masses[r] == 0:
+                continue
+            if not (wt[k] == wt[r] or min(wt[k], wt[r]) >= cores):
+                continue
+            if _frac_dist(vecs[k], vecs[r]) < theta:
+                cand = (abs(wt[k] - wt[r]), r)
+                best = cand if best is None or cand < best else best
+        if best is None:
+            rep[k] = True
+        else:
+            match[k] = best[1]
+    return match
+
+
+@pytest.mark.parametrize("seed", range(6))
+@pytest.mark.parametrize("theta", [(1, 100), (1, 20), (1, 10), (1, 5), (1, 2)])
+def test_match_bruteforce_random(seed, theta):
+    rs = np.random.default_rng(100 + seed)
+    # few prototypes with small perturbations so many pairs are near the threshold
+    protos = [[int(x) for x in rs.integers(0, 6, int(rs.integers(1, 8)))] for _ in range(3)]
+    kernels = []
+    for _ in range(9):
+        p = protos[int(rs.integers(0, 3))]
+        warps = [list(p) for _ in range(int(rs.integers(1, 8)))]
+        if rs.random() < 0.5:
+            warps.append(p + [int(rs.integers(0, 6))])
+        kernels.append(warps)
+    wt = [int(x) for x in rs.choice([16, 32, 64, 100, 128, 128], size=len(kernels))]
+    tr = tg.trace_from_warps(kernels, bb_len=[1, 2, 3, 5, 8, 13], warps_total=wt)
+    t, sig, mass = _pipeline(tr)
+    vecs = [_frac_gpu_bbv(t, k) for k in range(len(kernels))]
+    for pool_all in (0, 1):
+        m, d = oracle.match(t["kernel_type_off"], sig, mass, wt, theta, 64, pool_all)
+        assert m.tolist() == _brute_resolve(vecs, [int(x) for x in mass], wt, Fraction(*theta), 64, pool_all)
+        for k in range(len(kernels)):
+            if m[k] >= 0:
+                assert d[k] == pytest.approx(float(_frac_dist(vecs[k], vecs[int(m[k])])), rel=1e-12)
+
+
+def test_match_scenarios():
+    a, b = [0, 1, 1, 2], [0, 2, 2, 2, 1]
+    # identical repeat matches its first occurrence; chain: k2 matches k0 (representative), not k1 (matched)
+    tr = tg.trace_from_warps([[a] * 4, [a] * 4, [a] * 4, [b] * 4], [2, 3, 1], warps_total=[100, 100, 100, 100])
+    t, sig, mass = _pipeline(tr)
+    m, d = oracle.match(t["kernel_type_off"], sig, mass, tr.warps_total)
+    assert m.tolist() == [-1, 0, 0, -1] and d[1] == 0.0 and np.isinf(d[0])
+    # fewer warps than GPU cores (64): unequal counts never match; equal counts do (L271 Fig 12 note, L277)
+    m, _ = oracle.match(t["kernel_type_off"], sig, mass, np.array([32, 33, 32, 32], np.uint64))
+    assert m.tolist() == [-1, -1, 0, -1]
+    # closest warp count wins; a tie goes to the earliest representative (pool = all prior so 0 and 1 compete)
+    m, _ = oracle.match(t["kernel_type_off"], sig, mass, np.array([100, 140, 120, 100], np.uint64),
+                        pool_all_prior=1)
+    assert m[2] == 0  # |120-100| = |120-140| = 20: tie -> earliest
+    m, _ = oracle.match(t["kernel_type_off"], sig, mass, np.array([100, 130, 120, 100], np.uint64),
+                        pool_all_prior=1)
+    assert m[2] == 1
+    # empty signature never matches [P-19]
+    tr = tg.trace_from_warps([[[]], [[]]], [1])
+    t, sig, mass = _pipeline(tr)
+    m, d = oracle.match(t["kernel_type_off"], sig, mass, [64, 64], theta=(2, 1))
+    assert m.tolist() == [-1, -1] and np.isinf(d).all()
+
+
+def test_match_theta_exact_boundary():
+    # D = 4/11 exactly (worked example): theta = 4/11 -> not close (strict); 4/11 + tiny -> close
+    g = _gold("worked_example.json")
+    tr = tg.trace_from_warps(g["kernels"], g["bb_len"], warps_total=[100, 100])
+    t, sig, mass = _pipeline(tr)
+    assert oracle.match(t["kernel_type_off"], sig, mass, tr.warps_total, (4, 11))[0].tolist() == [-1, -1]
+    assert oracle.match(t["kernel_type_off"], sig, mass, tr.warps_total, (400001, 1100000))[0].tolist() == [-1, 0]
+    assert oracle.match(t["kernel_type_off"], sig, mass, tr.warps_total, (399999, 1100000))[0].tolist() == [-1, -1]
+
+
+# ---------------------------------------------------------------------------------------------------------------
+# A5: Eq. 1 slope and the stability detector.
+def _exact_slope(xs, ys):
+    """Eq. 1 (L222-225) in exact rationals, written from the textbook normal equations."""
+    n = len(xs)
+    xm = Fraction(sum(xs), n)
+    ym = Fraction(sum(ys), n)
+    sxy = sum((x - xm) * (y - ym) for x, y in zip(xs, ys))
+    sxx = sum((x - xm) ** 2 for x in xs)
+    return sxy / sxx
+
+
+def _timing_one_kernel(xs, ys, bbs=None):
+    R = len(xs)
+    return tg.Timing(kernel_rec_off=np.array([0, R], np.uint64),
+                     bb=np.array(bbs if bbs is not None else [0] * R, np.uint16),
+                     issue=np.array(xs, np.uint64), retire=np.array(ys, np.uint64), n_bb=1 if bbs is None else max(bbs) + 1)
+
+
+def _line_stream(a: Fraction, b: Fraction, n: int, count: int, x0=10_000, dx=10_000, offset=10 ** 9):
+    xs = [x0 + dx * i for i in range(count)]
+    ys = [int(a * x + b + offset) for x in xs]  # a*x integral for the chosen a and dx
+    return xs, ys
+
+
+@pytest.mark.parametrize("entry", _gold("paper_lines.json")["lines"] + _gold("paper_lines.json")["boundary"])
+def test_eq1_paper_lines_and_boundary(entry):
+    a = Fraction(entry["a"])
+    b = Fraction(entry.get("b", "0")) * 100  # microseconds -> ticks, keeps the line (slope is unit-free)
+    n = 8
+    xs, ys = _line_stream(a, b, n, 2 * n)
+    # the closed form agrees with numpy's least squares and with the exact rational slope
+    assert _exact_slope(xs, ys) == a
+    assert np.polyfit(np.array(xs, float), np.array(ys, float), 1)[0] == pytest.approx(float(a), rel=1e-9)
+    fs, ds, sw = oracle.stable(_timing_one_kernel(xs, ys), np.array([[1]], np.uint64), n=n)
+    assert (fs[0, 0] == 2 * n - 1) == entry["stable"], entry
+    if entry["stable"]:
+        assert int(ds[0, 0]) == sum(y - x for x, y in zip(xs[n:], ys[n:]))  # S_n of the last n
+        assert sw[0] == 2 * n - 1
+
+
+def test_eq1_float_hazard_at_boundary():
+    # a = 0.97 exactly (|1-a| = delta): numpy.polyfit's float slope lands on the wrong side of |1-a| < 0.03 and a
+    # float detector would call it stable; the exact integer test (the oracle's) does not [P-15][P-16]
+    xs, ys = _line_stream(Fraction(97, 100), Fraction(0), 8, 16, x0=0, dx=1000, offset=10 ** 6)
+    fa = np.polyfit(np.array(xs, float), np.array(ys, float), 1)[0]
+    assert _exact_slope(xs, ys) == Fraction(97, 100)
+    assert abs(1 - fa) < 0.03  # the float hazard is real on this stream
+    fs, _, _ = oracle.stable(_timing_one_kernel(xs, ys), np.array([[1]], np.uint64), n=8)
+    assert fs[0, 0] == -1
+
+
+@pytest.mark.parametrize("seed", range(8))
+def test_stability_bruteforce_fraction(seed):
+    """Random small streams of 3 BB types: first-stable positions equal a from-scratch Fraction recomputation
+    of cond1 (Eq. 1, |1-a| < delta) and cond2 (mean check) at every execution, in both oracle modes."""
+    rs = np.random.default_rng(seed)
+    n = int(rs.choice([2, 3, 5, 8]))
+    R = 120
+    types = rs.integers(0, 3, R)
+    t = 0
+    xs, ys = [], []
+    for i in range(R):
+        t += int(rs.integers(0, 4))
+        d = int(rs.choice([5, 5, 5, 6])) if rs.random() < 0.8 else int(rs.integers(0, 12))
+        xs.append(t)
+        ys.append(t + d)
+    order = sorted(range(R), key=lambda i: (ys[i], i))
+    xs = [xs[i] for i in order]
+    ys = [ys[i] for i in order]
+    bbs = [int(types[i]) for i in range(R)]
+    tm = _timing_one_kernel(xs, ys, bbs)
+    tm.n_bb = 3
+    kbb = np.array([[50, 30, 20]], np.uint64)
+    delta = Fraction(3, 100) if seed % 2 else Fraction(1, 5)
+    expect = [-1, -1, -1]
+    for b in range(3):
+        idx = [i for i in range(R) if bbs[i] == b]
+        for j in range(2 * n, len(idx) + 1):
+            win = idx[j - n:j]
+            win2 = idx[j - 2 * n:j]
+            wx = [xs[i] for i in win]
+            wy = [ys[i] for i in win]
+            if len(set(wx)) < 2:
+                c1 = False
+            else:
+                c1 = abs(1 - _exact_slope(wx, wy)) < delta
+            sn = sum(ys[i] - xs[i] for i in win)
+            s2n = sum(ys[i] - xs[i] for i in win2)
+            c2 = s2n > 0 and abs(Fraction(sn, n) - Fraction(s2n, 2 * n)) < delta * Fraction(s2n, 2 * n)
+            if c1 and c2:
+                expect[b] = idx[j - 1]
+                break
+    for brute in (True, False):
+        fs, ds, sw = oracle.stable(tm, kbb, n=n, delta=(delta.numerator, delta.denominator), brute=brute)
+        assert fs[0].tolist() == expect
+    # switch [P-14]: order stable BBs by position, first point where the weight share exceeds 95%
+    st = sorted((p, b) for b, p in enumerate(expect) if p >= 0)
+    acc, want = 0, -1
+    for p, b in st:
+        acc += int(kbb[0, b])
+        if Fraction(acc, 100) > Fraction(95, 100):
+            want = p
+            break
+    assert sw[0] == want
+
+
+def test_detector_constructed_streams():
+    n = 2048
+    # L227 MM line scaled x100: y = x + 423, single type -> stable at exactly its 2n-th execution (position 4095)
+    xs = [100 * i for i in range(3 * n)]
+    ys = [x + 423 for x in xs]
+    fs, ds, sw = oracle.stable(_timing_one_kernel(xs, ys), np.array([[7]], np.uint64), n=n)
+    assert fs[0, 0] == 2 * n - 1 and int(ds[0, 0]) == 423 * n and sw[0] == 2 * n - 1
+    # SpMV-like mix (L210): a stable 99.4%-weight BB + a 0.6% BB executed once (rare, never stable) -> switches
+    xs2 = xs + [xs[-1] + 50]
+    ys2 = ys + [ys[-1] + 60]
+    tm = _timing_one_kernel(xs2, ys2, [0] * len(xs) + [1])
+    fs, _, sw = oracle.stable(tm, np.array([[994, 6]], np.uint64), n=n)
+    assert fs[0].tolist() == [2 * n - 1, -1] and sw[0] == 2 * n - 1
+    # exactly 95% weight stable -> no switch (strict, L208 "larger than"); 95.1% -> switch
+    fs, _, sw = oracle.stable(tm, np.array([[950, 50]], np.uint64), n=n)
+    assert sw[0] == -1
+    fs, _, sw = oracle.stable(tm, np.array([[951, 49]], np.uint64), n=n)
+    assert sw[0] == 2 * n - 1
+    # all issue times equal: den = 0 -> not stable [P-16]
+    xs3 = [1000] * (2 * n)
+    ys3 = [1000 + 5 + (i % 3) for i in range(2 * n)]
+    ys3.sort()
+    fs, _, _ = oracle.stable(_timing_one_kernel(xs3, ys3), np.array([[1]], np.uint64), n=n)
+    assert fs[0, 0] == -1
+    # zero durations: S_2n = 0 -> not stable [P-17]
+    xs4 = list(range(2 * n))
+    fs, _, _ = oracle.stable(_timing_one_kernel(xs4, xs4), np.array([[1]], np.uint64), n=n)
+    assert fs[0, 0] == -1
+
+
+def test_detector_ramp_then_flat_bruteforce():
+    # durations ramp down then flatten (the warm-up of L227): compare both oracle modes with a direct recomputation
+    n = 16
+    xs, ys = [], []
+    t = 0
+    for i in range(12 * n):
+        d = 200 - 4 * i if i < 40 else 40
+        xs.append(t)
+        ys.append(t + d)
+        t += 7
+    order = sorted(range(len(xs)), key=lambda i: (ys[i], i))
+    xs = [xs[i] for i in order]
+    ys = [ys[i] for i in order]
+    want = -1
+    for j in range(2 * n, len(xs) + 1):
+        wx, wy = xs[j - n:j], ys[j - n:j]
+        c1 = abs(1 - _exact_slope(wx, wy)) < Fraction(3, 100)
+        sn = sum(y - x for x, y in zip(wx, wy))
+        s2n = sum(y - x for x, y in zip(xs[j - 2 * n:j], ys[j - 2 * n:j]))
+        c2 = s2n > 0 and abs(2 * sn - s2n) * 100 < 3 * s2n
+        if c1 and c2:
+            want = j - 1
+            break
+    assert want > 2 * n  # the ramp delays stability past the first evaluable window
+    for brute in (True, False):
+        fs, _, _ = oracle.stable(_timing_one_kernel(xs, ys), np.array([[1]], np.uint64), n=n, brute=brute)
+        assert fs[0, 0] == want
+
+
+def test_stable_range_errors():
+    tm = _timing_one_kernel([5, 6], [4, 9])  # retire < issue
+    with pytest.raises(oracle.OracleError) as ei:
+        oracle.stable(tm, np.array([[1]], np.uint64), n=2)
+    assert ei.value.index == 0
+    tm = _timing_one_kernel([1, 2], [9, 8])  # not retire-sorted
+    with pytest.raises(oracle.OracleError) as ei:
+        oracle.stable(tm, np.array([[1]], np.uint64), n=2)
+    assert ei.value.index == 1
+    tm = _timing_one_kernel([1, 1 << 40], [9, (1 << 40) + 1])  # time >= 2^40
+    with pytest.raises(oracle.OracleError):
+        oracle.stable(tm, np.array([[1]], np.uint64), n=2)
+
+
+def test_oracle_modes_agree_on_generated_timing():
+    g = tg.Generator(6)
+    tm = g.timing(0, 6)
+    tr = g.kernels_trace(0, 6)
+    _, _, kbb = oracle.bbv(tr)
+    a = oracle.stable(tm, kbb, n=32, brute=True)
+    b = oracle.stable(tm, kbb, n=32, brute=False)
+    for x, y in zip(a, b):
+        assert np.array_equal(x, y)
+    assert (a[0] >= 0).any()  # something stabilises
