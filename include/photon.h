@@ -28,6 +28,11 @@ extern "C" {
 #endif
 
 #define PHOTON_ABI_VERSION 1
+#if defined(__GNUC__)
+#define PHOTON_API __attribute__((visibility("default")))
+#else
+#define PHOTON_API
+#endif
 #define PHOTON_BINS 16 /* "project these BBVs into fixed-size BBVs (We use 16)" — L178 §3 Obs. 5 */
 
 typedef enum {
@@ -42,16 +47,18 @@ typedef enum {
 
 typedef struct photon_ctx photon_ctx; /* opaque host object; owns no device memory */
 
-int photon_abi_version(void);
+PHOTON_API int photon_abi_version(void);
 /* Creates a context bound to `cuda_device` (reads its SM count).  Returns PHOTON_ECUDA without a usable device. */
-int photon_create(photon_ctx **out, int cuda_device);
-void photon_destroy(photon_ctx *ctx);
+PHOTON_API int photon_create(photon_ctx **out, int cuda_device);
+PHOTON_API void photon_destroy(photon_ctx *ctx);
 /* Host string describing the most recent error of this ctx; valid until the next call on it. */
-const char *photon_last_error(const photon_ctx *ctx);
+PHOTON_API const char *photon_last_error(const photon_ctx *ctx);
 /* SYNCHRONISES `stream`, then reads the device error latch of the most recent call that used a workspace.
  * Returns that call's device status (PHOTON_OK if none); *bad_index (may be NULL) receives the offending element
  * index (event, warp, record, kernel or slot, per the code) or -1. */
-int photon_check(photon_ctx *ctx, void *stream, int64_t *bad_index);
+PHOTON_API int photon_check(photon_ctx *ctx, void *stream, int64_t *bad_index);
+/* Same as photon_check for an explicit workspace (one of several calls in flight). SYNCHRONISES `stream`. */
+PHOTON_API int photon_ws_status(photon_ctx *ctx, const void *ws, void *stream, int64_t *bad_index);
 
 /* ------------------------------------------------------------------------------------------------------------
  * Input 1: the functional basic-block trace of the analysed (sampled) warps, CSR by kernel then by warp.
@@ -90,8 +97,8 @@ typedef struct {
  * kernel_bb_insts[k][b] = sum over warps w of kernel k of count_w(b) * bb_len[b]  (the BB distribution, L208-210)
  * Any output may be NULL (not computed).  Device errors: ERANGE (bb >= n_bb: index = event; non-monotone
  * warp_event_off / kernel_warp_off: index = warp / kernel; I_w >= 2^32: index = warp). */
-size_t photon_bbv_workspace_bytes(const photon_trace *trace);
-int photon_bbv_build(photon_ctx *ctx, const photon_trace *trace, void *ws, size_t ws_bytes,
+PHOTON_API size_t photon_bbv_workspace_bytes(const photon_trace *trace);
+PHOTON_API int photon_bbv_build(photon_ctx *ctx, const photon_trace *trace, void *ws, size_t ws_bytes,
                      uint32_t *warp_bbv16 /*[W][16] or NULL*/, uint64_t *warp_insts /*[W] or NULL*/,
                      uint64_t *kernel_bb_insts /*[K][B] or NULL*/, void *stream);
 
@@ -102,11 +109,11 @@ int photon_bbv_build(photon_ctx *ctx, const photon_trace *trace, void *ws, size_
  * open-addressing hash table sized from `type_capacity_hint` (expected total types; 0 => a default of
  * min(W, 2^20)); if it fills, the call latches PHOTON_ECAPACITY and the caller retries with a larger hint.
  * out->capacity must be >= the number of types found (ECAPACITY otherwise). */
-size_t photon_group_workspace_bytes(const photon_trace *trace, uint64_t type_capacity_hint);
-int photon_warp_group(photon_ctx *ctx, const photon_trace *trace, const uint32_t *warp_bbv16 /*or NULL*/, void *ws,
+PHOTON_API size_t photon_group_workspace_bytes(const photon_trace *trace, uint64_t type_capacity_hint);
+PHOTON_API int photon_warp_group(photon_ctx *ctx, const photon_trace *trace, const uint32_t *warp_bbv16 /*or NULL*/, void *ws,
                       size_t ws_bytes, photon_types *out, void *stream);
 /* SYNCS the stream and returns kernel_type_off[K] (total types) in *total_types (HOST). */
-int photon_types_total(photon_ctx *ctx, const photon_types *types, uint32_t n_kernels, uint64_t *total_types,
+PHOTON_API int photon_types_total(photon_ctx *ctx, const photon_types *types, uint32_t n_kernels, uint64_t *total_types,
                        void *stream);
 
 /* ---- A3 + A4: GPU-BBV signature and kernel matching (L159 Fig 5, L178, L271 Fig 12) ---------------
@@ -128,8 +135,8 @@ typedef struct {
 } photon_match_params;
 
 /* Workspace for K kernels, T total types and room for `pair_capacity` close pairs (0 => default 16*K + 65536). */
-size_t photon_match_workspace_bytes(uint32_t n_kernels, uint64_t total_types, uint64_t pair_capacity);
-int photon_kernel_match(photon_ctx *ctx, uint32_t n_kernels, const photon_types *types,
+PHOTON_API size_t photon_match_workspace_bytes(uint32_t n_kernels, uint64_t total_types, uint64_t pair_capacity);
+PHOTON_API int photon_kernel_match(photon_ctx *ctx, uint32_t n_kernels, const photon_types *types,
                         const uint64_t *warps_total /*[K]*/, photon_match_params params, void *ws, size_t ws_bytes,
                         int64_t *match /*[K]*/, double *match_dist /*[K] or NULL*/, void *stream);
 
@@ -138,14 +145,14 @@ int photon_kernel_match(photon_ctx *ctx, uint32_t n_kernels, const photon_types 
  * match_scan appends the close pairs (k, r) with k in [k_lo, k_hi) to pairs[] (u64: k << 32 | r), count in
  * *n_pairs (DEVICE u64, zeroed by the call); `pair_capacity` entries fit.  match_resolve takes the union of all
  * pair lists (any order) and runs the launch-order resolution; its result does not depend on pair order. */
-int photon_sig_build(photon_ctx *ctx, uint32_t n_kernels, const uint64_t *kernel_type_off, const uint32_t *type_key,
+PHOTON_API int photon_sig_build(photon_ctx *ctx, uint32_t n_kernels, const uint64_t *kernel_type_off, const uint32_t *type_key,
                      const uint64_t *type_count, uint32_t k_lo, uint32_t k_hi, uint64_t *sig /*[16*T]*/,
-                     uint64_t *mass /*[K]*/, void *stream);
-int photon_match_scan(photon_ctx *ctx, uint32_t n_kernels, const uint64_t *kernel_type_off, const uint64_t *sig,
+                     uint64_t *mass /*[K]*/, void *ws /* >= 256 bytes: error latch */, size_t ws_bytes, void *stream);
+PHOTON_API int photon_match_scan(photon_ctx *ctx, uint32_t n_kernels, const uint64_t *kernel_type_off, const uint64_t *sig,
                       const uint64_t *mass, const uint64_t *warps_total, photon_match_params params, uint32_t k_lo,
                       uint32_t k_hi, void *ws, size_t ws_bytes, uint64_t *pairs, uint64_t pair_capacity,
                       uint64_t *n_pairs, void *stream);
-int photon_match_resolve(photon_ctx *ctx, uint32_t n_kernels, const uint64_t *kernel_type_off, const uint64_t *sig,
+PHOTON_API int photon_match_resolve(photon_ctx *ctx, uint32_t n_kernels, const uint64_t *kernel_type_off, const uint64_t *sig,
                          const uint64_t *mass, const uint64_t *warps_total, photon_match_params params,
                          const uint64_t *pairs, uint64_t n_pairs, void *ws, size_t ws_bytes, int64_t *match,
                          double *match_dist, void *stream);
@@ -179,8 +186,8 @@ typedef struct {
   uint32_t rate_num, rate_den;   /* switch rate, default 95/100 (L208); 1 <= den <= 2^16, num <= den           */
 } photon_stable_params;
 
-size_t photon_stable_workspace_bytes(const photon_timing *timing);
-int photon_bb_stable(photon_ctx *ctx, const photon_timing *timing, const uint64_t *kernel_bb_insts /*[K][B]*/,
+PHOTON_API size_t photon_stable_workspace_bytes(const photon_timing *timing);
+PHOTON_API int photon_bb_stable(photon_ctx *ctx, const photon_timing *timing, const uint64_t *kernel_bb_insts /*[K][B]*/,
                      photon_stable_params params, void *ws, size_t ws_bytes, int64_t *first_stable /*[K][B]*/,
                      uint64_t *stable_dur_sum /*[K][B] or NULL*/, int64_t *switch_at /*[K]*/, void *stream);
 
@@ -195,18 +202,19 @@ typedef struct {
   uint64_t first_warp; /* global warp index */
 } photon_type_row;
 /* Writes the local types as rows (global ids) to rows[0..T_local); T_local = local->kernel_type_off[K_local]. */
-int photon_types_export(photon_ctx *ctx, uint32_t n_kernels_local, const photon_types *local, uint32_t kernel_base,
+PHOTON_API int photon_types_export(photon_ctx *ctx, uint32_t n_kernels_local, const photon_types *local, uint32_t kernel_base,
                         uint64_t warp_base, photon_type_row *rows, void *stream);
 /* Merges rows of all shards (any order; rows with equal (kernel, key) add counts and take the min first_warp)
  * into canonical global tables for K kernels; `kernel_warps` [K] = analysed warps per kernel (for the dominance
  * decision).  global->warp_type is ignored. */
-size_t photon_merge_workspace_bytes(uint64_t n_rows, uint32_t n_kernels);
-int photon_types_merge(photon_ctx *ctx, const photon_type_row *rows, uint64_t n_rows, uint32_t n_kernels,
+PHOTON_API size_t photon_merge_workspace_bytes(uint64_t n_rows, uint32_t n_kernels);
+PHOTON_API int photon_types_merge(photon_ctx *ctx, const photon_type_row *rows, uint64_t n_rows, uint32_t n_kernels,
                        const uint64_t *kernel_warps, void *ws, size_t ws_bytes, photon_types *global, void *stream);
-/* warp_type_global[v] = global canonical id of local warp v's type.  ws from photon_merge_workspace_bytes of the
- * same merge (its lookup table is reused; pass the same ws that the merge used, unmodified). */
-int photon_types_remap(photon_ctx *ctx, uint32_t n_kernels_local, uint64_t n_warps_local,
-                       const photon_types *local, const photon_types *global, uint32_t kernel_base, const void *ws,
+/* warp_type_global[v] = global canonical id of local warp v's type, looked up in the merged table that
+ * photon_types_merge left in `merge_ws` (pass the same buffer, unmodified, with the merge's n_rows and K). */
+PHOTON_API int photon_types_remap(photon_ctx *ctx, uint32_t n_kernels_local, uint64_t n_warps_local,
+                       const uint64_t *kernel_warp_off_local /*[K_local+1]*/, const photon_types *local,
+                       uint32_t kernel_base, uint64_t n_rows_merged, uint32_t n_kernels_global, const void *merge_ws,
                        size_t ws_bytes, uint32_t *warp_type_global, void *stream);
 
 #ifdef __cplusplus

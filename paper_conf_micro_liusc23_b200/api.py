@@ -1,0 +1,342 @@
+"""Thin Python binding of libphoton (same names as the C ABI, argument marshalling only).
+
+PyTorch supplies device memory and streams; every step of the path runs in libphoton's sm_100a kernels.  There
+is no CPU fallback: constructing `Photon` without a CUDA device or without the built library raises.
+
+Unsigned device arrays are carried in signed torch tensors of the same width (u64 -> int64, u32 -> int32,
+u16 -> int16); the bits are what the C ABI sees.
+"""
+from __future__ import annotations
+
+import ctypes
+from dataclasses import dataclass
+from typing import Dict, Optional, Tuple
+
+import numpy as np
+
+from . import _lib
+from ._lib import PhotonError, PhotonUnavailable
+
+_NP2T = {np.dtype(np.uint64): "int64", np.dtype(np.int64): "int64", np.dtype(np.uint32): "int32",
+         np.dtype(np.int32): "int32", np.dtype(np.uint16): "int16", np.dtype(np.uint8): "uint8",
+         np.dtype(np.float64): "float64"}
+
+
+def _torch():
+    import torch
+    return torch
+
+
+def to_device(a: np.ndarray, device, pin: bool = False, non_blocking: bool = False):
+    """numpy -> torch tensor with the same bits (unsigned carried in signed tensors of equal width)."""
+    torch = _torch()
+    a = np.ascontiguousarray(a)
+    view = {8: np.int64, 4: np.int32, 2: np.int16, 1: np.uint8}[a.dtype.itemsize] if a.dtype.kind in "ui" else a.dtype
+    t = torch.from_numpy(a.view(view))
+    if pin:
+        t = t.pin_memory()
+    return t.to(device, non_blocking=non_blocking) if device is not None else t
+
+
+def to_numpy(t, dtype) -> np.ndarray:
+    return t.detach().cpu().numpy().view(dtype)
+
+
+@dataclass
+class DeviceTrace:
+    """photon_trace in device memory."""
+    kernel_warp_off: "object"  # int64 [K+1]
+    warp_event_off: "object"   # int64 [W+1]
+    bb: "object"               # int16 [E]
+    bb_len: "object"           # int32 [B]
+    bb_bin: Optional["object"]  # uint8 [B] or None
+    warps_total: "object"      # int64 [K]
+    n_kernels: int
+    n_bb: int
+    n_warps: int
+    n_events: int
+
+    @staticmethod
+    def from_host(trace, device, non_blocking: bool = False) -> "DeviceTrace":
+        """`trace` has numpy fields kernel_warp_off, warp_event_off, bb, bb_len, bb_bin, warps_total."""
+        f = lambda a: to_device(a, device, non_blocking=non_blocking)
+        return DeviceTrace(f(trace.kernel_warp_off), f(trace.warp_event_off), f(trace.bb), f(trace.bb_len),
+                           None if trace.bb_bin is None else f(trace.bb_bin), f(trace.warps_total),
+                           len(trace.kernel_warp_off) - 1, len(trace.bb_len), len(trace.warp_event_off) - 1,
+                           len(trace.bb))
+
+    def c(self) -> _lib.Trace:
+        p = lambda t: t.data_ptr() if (t is not None and t.numel() > 0) else None
+        return _lib.Trace(self.n_kernels, self.n_bb, self.n_warps, self.n_events, p(self.kernel_warp_off),
+                          p(self.warp_event_off), p(self.bb), p(self.bb_len), p(self.bb_bin))
+
+
+@dataclass
+class DeviceTiming:
+    kernel_rec_off: "object"  # int64 [K+1]
+    bb: "object"              # int16 [R]
+    issue: "object"           # int64 [R]
+    retire: "object"          # int64 [R]
+    n_kernels: int
+    n_bb: int
+    n_records: int
+
+    @staticmethod
+    def from_host(tm, device, n_bb: Optional[int] = None) -> "DeviceTiming":
+        f = lambda a: to_device(a, device)
+        return DeviceTiming(f(tm.kernel_rec_off), f(tm.bb), f(tm.issue), f(tm.retire), len(tm.kernel_rec_off) - 1,
+                            int(n_bb if n_bb is not None else tm.n_bb), len(tm.bb))
+
+    def c(self) -> _lib.Timing:
+        p = lambda t: t.data_ptr() if t.numel() > 0 else None
+        return _lib.Timing(self.n_kernels, self.n_bb, self.n_records, p(self.kernel_rec_off), p(self.bb),
+                           p(self.issue), p(self.retire))
+
+
+def ht_capacity(hint: int, n_warps: int) -> int:
+    """Mirror of abi.cu's hash-table sizing (power of two >= 2 x expected types, >= 1024)."""
+    h = hint if hint else min(n_warps, 1 << 18)
+    cap = 1024
+    while cap < 2 * h:
+        cap <<= 1
+    return cap
+
+
+class Photon:
+    """One libphoton context on one CUDA device."""
+
+    def __init__(self, device=None):
+        torch = _torch()
+        if not torch.cuda.is_available():
+            raise PhotonUnavailable("libphoton needs a CUDA device (sm_100a); none is visible")
+        self.torch = torch
+        self.device = torch.device("cuda", torch.cuda.current_device() if device is None else int(device))
+        self.L = _lib.load()
+        ctx = ctypes.c_void_p()
+        rc = self.L.photon_create(ctypes.byref(ctx), self.device.index)
+        if rc != 0:
+            raise PhotonUnavailable(f"photon_create failed ({rc})")
+        self.ctx = ctx
+        self._ws: Dict[str, object] = {}
+
+    def __del__(self):
+        if getattr(self, "ctx", None) is not None and getattr(self, "L", None) is not None:
+            self.L.photon_destroy(self.ctx)
+            self.ctx = None
+
+    # -- plumbing ---------------------------------------------------------------------------------------------
+    def stream_ptr(self, stream=None) -> int:
+        s = stream if stream is not None else self.torch.cuda.current_stream(self.device)
+        return s.cuda_stream
+
+    def workspace(self, tag: str, nbytes: int):
+        """Cached device workspace (grows, never shrinks); returns a view of exactly nbytes."""
+        ws = self._ws.get(tag)
+        if ws is None or ws.numel() < nbytes:
+            ws = self.torch.empty(max(nbytes, 256), dtype=self.torch.uint8, device=self.device)
+            self._ws[tag] = ws
+        return ws[:max(nbytes, 256)]
+
+    def _rc(self, rc: int):
+        if rc != 0:
+            raise PhotonError(rc, self.L.photon_last_error(self.ctx).decode())
+
+    def ws_status(self, ws, stream=None) -> Tuple[int, int]:
+        bad = ctypes.c_int64(-1)
+        rc = self.L.photon_ws_status(self.ctx, ws.data_ptr(), self.stream_ptr(stream), ctypes.byref(bad))
+        return rc, bad.value
+
+    def check(self, ws, stream=None):
+        rc, bad = self.ws_status(ws, stream)
+        if rc != 0:
+            raise PhotonError(rc, self.L.photon_last_error(self.ctx).decode(), bad)
+
+    def empty(self, n, dtype):
+        return self.torch.empty(max(int(n), 0), dtype=getattr(self.torch, dtype), device=self.device)
+
+    # -- A1 ----------------------------------------------------------------------------------------------------
+    def photon_bbv_build(self, t: DeviceTrace, bbv16: bool = True, insts: bool = True, kbb: bool = False,
+                         stream=None, check: bool = True, out: Optional[dict] = None) -> dict:
+        ct = t.c()
+        nb = self.L.photon_bbv_workspace_bytes(ctypes.byref(ct))
+        ws = self.workspace("bbv", nb)
+        o = out if out is not None else {}
+        if bbv16 and "warp_bbv16" not in o:
+            o["warp_bbv16"] = self.empty(16 * t.n_warps, "int32")
+        if insts and "warp_insts" not in o:
+            o["warp_insts"] = self.empty(t.n_warps, "int64")
+        if kbb and "kernel_bb_insts" not in o:
+            o["kernel_bb_insts"] = self.empty(t.n_kernels * t.n_bb, "int64")
+        p = lambda k: o[k].data_ptr() if (k in o and o[k].numel()) else None
+        self._rc(self.L.photon_bbv_build(self.ctx, ctypes.byref(ct), ws.data_ptr(), ws.numel(),
+                                         p("warp_bbv16") if bbv16 else None, p("warp_insts") if insts else None,
+                                         p("kernel_bb_insts") if kbb else None, self.stream_ptr(stream)))
+        if check:
+            self.check(ws, stream)
+        return o
+
+    # -- A2 ----------------------------------------------------------------------------------------------------
+    def alloc_types(self, n_kernels: int, n_warps: int, capacity: int) -> dict:
+        cap = max(1, capacity)
+        return dict(capacity=cap, warp_type=self.empty(n_warps, "int32"),
+                    kernel_type_off=self.empty(n_kernels + 1, "int64"), type_key=self.empty(16 * cap, "int32"),
+                    type_count=self.empty(cap, "int64"), type_first_warp=self.empty(cap, "int64"),
+                    warp_sampling_ok=self.empty(n_kernels, "uint8"))
+
+    @staticmethod
+    def types_c(ty: dict) -> _lib.Types:
+        p = lambda k: ty[k].data_ptr() if (ty.get(k) is not None and ty[k].numel()) else None
+        return _lib.Types(ty["capacity"], p("warp_type"), p("kernel_type_off"), p("type_key"), p("type_count"),
+                          p("type_first_warp"), p("warp_sampling_ok"))
+
+    def photon_warp_group(self, t: DeviceTrace, warp_bbv16=None, capacity_hint: int = 0, stream=None,
+                          check: bool = True, out: Optional[dict] = None) -> dict:
+        hint = capacity_hint
+        for _ in range(8):
+            ct = t.c()
+            nb = self.L.photon_group_workspace_bytes(ctypes.byref(ct), hint)
+            ws = self.workspace("group", nb)
+            cap = min(max(t.n_warps, 1), ht_capacity(hint, t.n_warps))
+            ty = out if (out is not None and out["capacity"] >= cap) else self.alloc_types(t.n_kernels, t.n_warps, cap)
+            tc = self.types_c(ty)
+            self._rc(self.L.photon_warp_group(self.ctx, ctypes.byref(ct),
+                                              None if warp_bbv16 is None else warp_bbv16.data_ptr(), ws.data_ptr(),
+                                              ws.numel(), ctypes.byref(tc), self.stream_ptr(stream)))
+            ty["_ws"] = ws
+            if not check:
+                return ty
+            rc, bad = self.ws_status(ws, stream)
+            if rc == _lib.ECAPACITY:
+                hint = max(2 * ht_capacity(hint, t.n_warps), 1 << 12)
+                out = None
+                continue
+            if rc != 0:
+                raise PhotonError(rc, self.L.photon_last_error(self.ctx).decode(), bad)
+            return ty
+        raise PhotonError(_lib.ECAPACITY, "type table kept overflowing")
+
+    def photon_types_total(self, ty: dict, n_kernels: int, stream=None) -> int:
+        v = ctypes.c_uint64(0)
+        tc = self.types_c(ty)
+        self._rc(self.L.photon_types_total(self.ctx, ctypes.byref(tc), n_kernels, ctypes.byref(v),
+                                           self.stream_ptr(stream)))
+        return int(v.value)
+
+    # -- A3 + A4 -----------------------------------------------------------------------------------------------
+    @staticmethod
+    def match_params(theta=(1, 20), n_cores=64, pool_all_prior=0) -> _lib.MatchParams:
+        return _lib.MatchParams(int(theta[0]), int(theta[1]), int(n_cores), int(pool_all_prior))
+
+    def photon_kernel_match(self, n_kernels: int, ty: dict, warps_total, theta=(1, 20), n_cores=64,
+                            pool_all_prior=0, want_dist: bool = True, pair_capacity: int = 0, stream=None,
+                            check: bool = True, out: Optional[dict] = None) -> dict:
+        K = n_kernels
+        cap = pair_capacity or (16 * K + 65536)
+        for _ in range(8):
+            nb = self.L.photon_match_workspace_bytes(K, ty["capacity"], cap)
+            ws = self.workspace("match", nb)
+            o = out if out is not None else {}
+            o.setdefault("match", self.empty(K, "int64"))
+            if want_dist:
+                o.setdefault("match_dist", self.empty(K, "float64"))
+            tc = self.types_c(ty)
+            self._rc(self.L.photon_kernel_match(self.ctx, K, ctypes.byref(tc), warps_total.data_ptr(),
+                                                self.match_params(theta, n_cores, pool_all_prior), ws.data_ptr(),
+                                                ws.numel(), o["match"].data_ptr(),
+                                                o["match_dist"].data_ptr() if want_dist else None,
+                                                self.stream_ptr(stream)))
+            o["_ws"] = ws
+            if not check:
+                return o
+            rc, bad = self.ws_status(ws, stream)
+            if rc == _lib.ECAPACITY:
+                cap *= 4
+                continue
+            if rc != 0:
+                raise PhotonError(rc, self.L.photon_last_error(self.ctx).decode(), bad)
+            return o
+        raise PhotonError(_lib.ECAPACITY, "pair table kept overflowing")
+
+    # split form (multi-GPU driver)
+    def photon_sig_build(self, K, kto, type_key, type_count, k_lo, k_hi, sig, mass, stream=None):
+        ws = self.workspace("sig", 256)
+        self._rc(self.L.photon_sig_build(self.ctx, K, kto.data_ptr(), type_key.data_ptr(), type_count.data_ptr(),
+                                         k_lo, k_hi, sig.data_ptr() if sig.numel() else None, mass.data_ptr(),
+                                         ws.data_ptr(), ws.numel(), self.stream_ptr(stream)))
+        return ws
+
+    def photon_match_scan(self, K, kto, sig, mass, warps_total, params, k_lo, k_hi, pairs, n_pairs, stream=None):
+        nb = self.L.photon_match_workspace_bytes(K, 1, pairs.numel())
+        ws = self.workspace("scan", nb)
+        self._rc(self.L.photon_match_scan(self.ctx, K, kto.data_ptr(), sig.data_ptr() if sig.numel() else None,
+                                          mass.data_ptr(), warps_total.data_ptr(), params, k_lo, k_hi, ws.data_ptr(),
+                                          ws.numel(), pairs.data_ptr(), pairs.numel(), n_pairs.data_ptr(),
+                                          self.stream_ptr(stream)))
+        return ws
+
+    def photon_match_resolve(self, K, kto, sig, mass, warps_total, params, pairs, n_pairs: int, match, match_dist,
+                             stream=None):
+        nb = self.L.photon_match_workspace_bytes(K, 1, max(n_pairs, 1))
+        ws = self.workspace("resolve", nb)
+        self._rc(self.L.photon_match_resolve(self.ctx, K, kto.data_ptr(), sig.data_ptr() if sig.numel() else None,
+                                             mass.data_ptr(), warps_total.data_ptr(), params,
+                                             pairs.data_ptr() if n_pairs else None, n_pairs, ws.data_ptr(),
+                                             ws.numel(), match.data_ptr(),
+                                             None if match_dist is None else match_dist.data_ptr(),
+                                             self.stream_ptr(stream)))
+        return ws
+
+    # -- A5 ----------------------------------------------------------------------------------------------------
+    def photon_bb_stable(self, tm: DeviceTiming, kernel_bb_insts, n: int = 2048, delta=(3, 100), rate=(95, 100),
+                         want_dur: bool = True, stream=None, check: bool = True, out: Optional[dict] = None) -> dict:
+        ct = tm.c()
+        nb = self.L.photon_stable_workspace_bytes(ctypes.byref(ct))
+        ws = self.workspace("stable", nb)
+        o = out if out is not None else {}
+        o.setdefault("first_stable", self.empty(tm.n_kernels * tm.n_bb, "int64"))
+        if want_dur:
+            o.setdefault("stable_dur_sum", self.empty(tm.n_kernels * tm.n_bb, "int64"))
+        o.setdefault("switch_at", self.empty(tm.n_kernels, "int64"))
+        prm = _lib.StableParams(int(n), int(delta[0]), int(delta[1]), int(rate[0]), int(rate[1]))
+        self._rc(self.L.photon_bb_stable(self.ctx, ctypes.byref(ct), kernel_bb_insts.data_ptr(), prm, ws.data_ptr(),
+                                         ws.numel(), o["first_stable"].data_ptr(),
+                                         o["stable_dur_sum"].data_ptr() if want_dur else None,
+                                         o["switch_at"].data_ptr(), self.stream_ptr(stream)))
+        o["_ws"] = ws
+        if check:
+            self.check(ws, stream)
+        return o
+
+    # -- multi-GPU helpers -------------------------------------------------------------------------------------
+    def photon_types_export(self, K_local, ty, kernel_base, warp_base, rows, stream=None):
+        tc = self.types_c(ty)
+        self._rc(self.L.photon_types_export(self.ctx, K_local, ctypes.byref(tc), kernel_base, warp_base,
+                                            rows.data_ptr(), self.stream_ptr(stream)))
+
+    def photon_types_merge(self, rows, n_rows, K, kernel_warps, out: dict, stream=None):
+        nb = self.L.photon_merge_workspace_bytes(n_rows, K)
+        ws = self.workspace("merge", nb)
+        tc = self.types_c(out)
+        self._rc(self.L.photon_types_merge(self.ctx, rows.data_ptr() if n_rows else None, n_rows, K,
+                                           kernel_warps.data_ptr(), ws.data_ptr(), ws.numel(), ctypes.byref(tc),
+                                           self.stream_ptr(stream)))
+        return ws
+
+    def photon_types_remap(self, K_local, W_local, kwo_local, ty_local, kernel_base, n_rows, K, merge_ws,
+                           warp_type_global, stream=None):
+        tc = self.types_c(ty_local)
+        self._rc(self.L.photon_types_remap(self.ctx, K_local, W_local, kwo_local.data_ptr(), ctypes.byref(tc),
+                                           kernel_base, n_rows, K, merge_ws.data_ptr(), merge_ws.numel(),
+                                           warp_type_global.data_ptr() if W_local else None,
+                                           self.stream_ptr(stream)))
+
+    # -- the benchmarked chain ---------------------------------------------------------------------------------
+    def analyse(self, t: DeviceTrace, theta=(1, 20), n_cores=64, pool_all_prior=0, want_dist=False, stream=None,
+                check: bool = True, capacity_hint: int = 0, pair_capacity: int = 0) -> dict:
+        """A1 -> A2 -> A3 -> A4 on one device (fused BBV + grouping pass, then canonical tables, signatures,
+        match).  With check=False nothing synchronises (errors stay latched in the returned workspaces)."""
+        ty = self.photon_warp_group(t, None, capacity_hint, stream=stream, check=check)
+        m = self.photon_kernel_match(t.n_kernels, ty, t.warps_total, theta, n_cores, pool_all_prior, want_dist,
+                                     pair_capacity, stream=stream, check=check)
+        ty.update(match=m["match"], match_dist=m.get("match_dist"), _mws=m["_ws"])
+        return ty

@@ -1,0 +1,517 @@
+// abi.cu — the C ABI of libphoton (include/photon.h): argument validation, workspace layout, launch sequencing.
+// No computation happens here; every step of the path runs in the kernels of k_*.cu on the caller's stream.
+#include <cstdarg>
+#include <cstdio>
+#include <cstring>
+#include <new>
+#include <string>
+
+#include "internal.h"
+
+using namespace photon;
+
+struct photon_ctx {
+  int device = 0;
+  int num_sms = 148;
+  std::string err;
+  const void* last_ws = nullptr;
+};
+
+namespace {
+
+int fail(photon_ctx* c, int code, const char* fmt, ...) {
+  if (c) {
+    char buf[512];
+    va_list ap;
+    va_start(ap, fmt);
+    vsnprintf(buf, sizeof buf, fmt, ap);
+    va_end(ap);
+    c->err = buf;
+  }
+  return code;
+}
+
+int cuda_fail(photon_ctx* c, cudaError_t e, const char* where) {
+  return fail(c, PHOTON_ECUDA, "%s: %s", where, cudaGetErrorString(e));
+}
+
+#define CK(expr, where)                             \
+  do {                                              \
+    cudaError_t _e = (expr);                        \
+    if (_e != cudaSuccess) return cuda_fail(ctx, _e, where); \
+  } while (0)
+
+bool aligned(const void* p, size_t a) { return ((uintptr_t)p % a) == 0; }
+
+int check_trace(photon_ctx* ctx, const photon_trace* t) {
+  if (!t) return fail(ctx, PHOTON_EINVAL, "trace is NULL");
+  if (t->n_kernels == 0) return fail(ctx, PHOTON_EINVAL, "n_kernels must be >= 1");
+  if (t->n_bb == 0 || t->n_bb > 65536) return fail(ctx, PHOTON_EINVAL, "n_bb must be in [1, 65536]");
+  if (t->n_warps >= (1ull << 40) || t->n_events >= (1ull << 48)) return fail(ctx, PHOTON_EINVAL, "W or E too large");
+  if (!t->kernel_warp_off || !t->warp_event_off || !t->bb_len) return fail(ctx, PHOTON_EINVAL, "NULL trace array");
+  if (t->n_events && !t->bb) return fail(ctx, PHOTON_EINVAL, "bb is NULL");
+  if (t->bb && !aligned(t->bb, 16)) return fail(ctx, PHOTON_EINVAL, "bb must be 16-byte aligned");
+  return PHOTON_OK;
+}
+
+TraceDev to_dev(const photon_trace* t) {
+  TraceDev d;
+  d.kwo = t->kernel_warp_off; d.weo = t->warp_event_off; d.bb = t->bb; d.bb_len = t->bb_len; d.bb_bin = t->bb_bin;
+  d.K = t->n_kernels; d.B = t->n_bb; d.W = t->n_warps; d.E = t->n_events;
+  return d;
+}
+
+// ---- workspace layouts ----------------------------------------------------------------------------------
+struct BbvWs {
+  DevErr* err;
+  uint32_t* tbl;  // table + (K+1) u64 chunk prefix after it (see launch_kernel_bb_insts)
+  uint32_t* max_len;
+  size_t bytes;
+};
+BbvWs bbv_layout(const photon_trace* t, void* base) {
+  Carver c(base);
+  BbvWs w;
+  w.err = c.take<DevErr>(1);
+  uint32_t P2 = next_pow2_u32(t->n_bb < 16 ? 16 : t->n_bb);
+  w.tbl = c.take<uint32_t>((size_t)P2 + 64 + 2 * ((size_t)t->n_kernels + 1) + 64);
+  w.max_len = c.take<uint32_t>(4);
+  w.bytes = c.off + 256;
+  return w;
+}
+
+uint64_t ht_capacity(uint64_t hint, uint64_t W) {
+  uint64_t h = hint ? hint : (W < (1ull << 18) ? W : (1ull << 18));
+  uint64_t cap = 1024;
+  while (cap < 2 * h) cap <<= 1;
+  return cap;
+}
+
+struct HtWs {
+  HashTable ht;
+  CanonWs cw;
+};
+void carve_ht(Carver& c, uint64_t cap, uint32_t K, HtWs& w) {
+  w.ht.hkey = c.take<uint64_t>(cap);
+  w.ht.ready = c.take<uint32_t>(cap);
+  w.ht.kern = c.take<uint32_t>(cap);
+  w.ht.key = c.take<uint32_t>(cap * 16);
+  w.ht.count = c.take<uint32_t>(cap);
+  w.ht.first = c.take<uint64_t>(cap);
+  w.ht.mask = cap - 1;
+  w.cw.tcount = c.take<uint32_t>(K + 1);
+  w.cw.cursor = c.take<uint32_t>(K + 1);
+  w.cw.list = c.take<uint32_t>(cap);
+  w.cw.canon = c.take<uint32_t>(cap);
+  w.cw.scratch = c.take<uint64_t>(cap / 2 + 1);  // used as u32[cap]
+}
+
+struct GroupWs {
+  BbvWs b;
+  HtWs h;
+  size_t bytes;
+};
+GroupWs group_layout(const photon_trace* t, uint64_t hint, void* base, size_t ws_bytes) {
+  GroupWs g;
+  g.b = bbv_layout(t, base);
+  Carver c(base);
+  c.off = g.b.bytes;
+  uint64_t cap = ht_capacity(hint, t->n_warps);
+  if (base && ws_bytes) {
+    // the capacity actually used is the largest power of two that fits (callers may pass a larger workspace)
+    while (true) {
+      Carver probe(nullptr);
+      probe.off = g.b.bytes;
+      HtWs tmp;
+      carve_ht(probe, cap * 2, t->n_kernels, tmp);
+      if (probe.off + 256 > ws_bytes) break;
+      cap *= 2;
+    }
+  }
+  carve_ht(c, cap, t->n_kernels, g.h);
+  g.bytes = c.off + 256;
+  return g;
+}
+
+struct MatchLayout {
+  DevErr* err;
+  uint64_t* sig;
+  uint64_t* mass;
+  MatchWs mw;
+  uint64_t* pairs;
+  uint64_t* n_pairs;
+  size_t bytes;
+};
+MatchLayout match_layout(uint32_t K, uint64_t T, uint64_t pair_cap, void* base) {
+  Carver c(base);
+  MatchLayout m;
+  if (!pair_cap) pair_cap = 16ull * K + 65536;
+  m.err = c.take<DevErr>(1);
+  m.sig = c.take<uint64_t>(16 * (T ? T : 1));
+  m.mass = c.take<uint64_t>(K + 1);
+  m.mw.prof = c.take<float>(16ull * K + 16);
+  m.mw.maybe = c.take<uint64_t>(pair_cap);
+  m.mw.n_maybe = c.take<uint64_t>(1);
+  m.mw.cand_cnt = c.take<uint32_t>(K + 1);
+  m.mw.cand_off = c.take<uint64_t>(K + 1);
+  m.mw.cand_cur = c.take<uint32_t>(K + 1);
+  m.mw.cand = c.take<uint32_t>(pair_cap);
+  m.mw.state = c.take<uint8_t>(K + 1);
+  m.mw.flag = c.take<uint32_t>(4);
+  m.mw.pair_cap = pair_cap;
+  m.pairs = c.take<uint64_t>(pair_cap);
+  m.n_pairs = c.take<uint64_t>(1);
+  m.bytes = c.off + 256;
+  return m;
+}
+
+// match layout from ws_bytes: largest pair capacity that fits (T is fixed by the caller's bound)
+MatchLayout match_layout_fit(uint32_t K, uint64_t T, void* base, size_t ws_bytes) {
+  uint64_t cap = 16ull * K + 65536;
+  MatchLayout m = match_layout(K, T, cap, nullptr);
+  while (m.bytes > ws_bytes && cap > 1024) { cap /= 2; m = match_layout(K, T, cap, nullptr); }
+  for (;;) {
+    MatchLayout bigger = match_layout(K, T, cap * 2, nullptr);
+    if (bigger.bytes > ws_bytes) break;
+    cap *= 2;
+  }
+  return match_layout(K, T, cap, base);
+}
+
+photon_match_params norm_params(photon_match_params p) {
+  if (p.theta_den == 0) { p.theta_num = 1; p.theta_den = 20; }
+  if (p.n_cores == 0) p.n_cores = 64;
+  return p;
+}
+
+int check_match_params(photon_ctx* ctx, const photon_match_params& p) {
+  if (p.theta_den == 0 || p.theta_den > (1u << 20) || p.theta_num > 2u * p.theta_den)
+    return fail(ctx, PHOTON_EINVAL, "theta must be num/den with 1 <= den <= 2^20, num <= 2*den");
+  return PHOTON_OK;
+}
+
+struct StableWs {
+  DevErr* err;
+  void* rest;
+  size_t rest_bytes;
+  size_t bytes;
+};
+StableWs stable_layout(const photon_timing* t, void* base) {
+  Carver c(base);
+  StableWs s;
+  s.err = c.take<DevErr>(1);
+  s.rest_bytes = stable_ws_bytes(*t);
+  s.rest = c.take<uint8_t>(s.rest_bytes);
+  s.bytes = c.off + 256;
+  return s;
+}
+
+struct MergeWs {
+  DevErr* err;
+  HtWs h;
+  size_t bytes;
+};
+MergeWs merge_layout(uint64_t n_rows, uint32_t K, void* base) {
+  Carver c(base);
+  MergeWs m;
+  m.err = c.take<DevErr>(1);
+  uint64_t cap = 1024;
+  while (cap < 2 * n_rows) cap <<= 1;
+  carve_ht(c, cap, K, m.h);
+  m.bytes = c.off + 256;
+  return m;
+}
+
+}  // namespace
+
+extern "C" {
+
+int photon_abi_version(void) { return PHOTON_ABI_VERSION; }
+
+int photon_create(photon_ctx** out, int cuda_device) {
+  if (!out) return PHOTON_EINVAL;
+  *out = nullptr;
+  int n = 0;
+  if (cudaGetDeviceCount(&n) != cudaSuccess || n == 0 || cuda_device < 0 || cuda_device >= n) {
+    cudaGetLastError();
+    return PHOTON_ECUDA;
+  }
+  photon_ctx* c = new (std::nothrow) photon_ctx();
+  if (!c) return PHOTON_ECUDA;
+  c->device = cuda_device;
+  if (cudaDeviceGetAttribute(&c->num_sms, cudaDevAttrMultiProcessorCount, cuda_device) != cudaSuccess) {
+    delete c;
+    return PHOTON_ECUDA;
+  }
+  *out = c;
+  return PHOTON_OK;
+}
+
+void photon_destroy(photon_ctx* ctx) { delete ctx; }
+
+const char* photon_last_error(const photon_ctx* ctx) { return ctx ? ctx->err.c_str() : "NULL ctx"; }
+
+static int read_latch(photon_ctx* ctx, const void* ws, void* stream, int64_t* bad) {
+  if (bad) *bad = -1;
+  cudaStream_t s = (cudaStream_t)stream;
+  CK(cudaStreamSynchronize(s), "cudaStreamSynchronize");
+  CK(cudaGetLastError(), "pending CUDA error");
+  if (!ws) return PHOTON_OK;
+  DevErr e;
+  CK(cudaMemcpy(&e, ws, sizeof e, cudaMemcpyDeviceToHost), "read error latch");
+  if (bad) *bad = e.code ? e.index : -1;
+  if (e.code) fail(ctx, e.code, "device-detected error %d at index %lld", e.code, (long long)e.index);
+  return e.code;
+}
+
+int photon_check(photon_ctx* ctx, void* stream, int64_t* bad_index) {
+  if (!ctx) return PHOTON_EINVAL;
+  return read_latch(ctx, ctx->last_ws, stream, bad_index);
+}
+
+int photon_ws_status(photon_ctx* ctx, const void* ws, void* stream, int64_t* bad_index) {
+  if (!ctx) return PHOTON_EINVAL;
+  return read_latch(ctx, ws, stream, bad_index);
+}
+
+// ---- A1 -----------------------------------------------------------------------------------------------------
+size_t photon_bbv_workspace_bytes(const photon_trace* t) { return t ? bbv_layout(t, nullptr).bytes : 0; }
+
+int photon_bbv_build(photon_ctx* ctx, const photon_trace* t, void* ws, size_t ws_bytes, uint32_t* warp_bbv16,
+                     uint64_t* warp_insts, uint64_t* kernel_bb_insts, void* stream) {
+  if (!ctx) return PHOTON_EINVAL;
+  int rc = check_trace(ctx, t);
+  if (rc) return rc;
+  if (!ws) return fail(ctx, PHOTON_EINVAL, "workspace is NULL");
+  BbvWs w = bbv_layout(t, ws);
+  if (ws_bytes < w.bytes) return fail(ctx, PHOTON_EWORKSPACE, "workspace %zu < %zu bytes", ws_bytes, w.bytes);
+  if (warp_bbv16 && !aligned(warp_bbv16, 16)) return fail(ctx, PHOTON_EINVAL, "warp_bbv16 must be 16-byte aligned");
+  cudaStream_t s = (cudaStream_t)stream;
+  CK(cudaSetDevice(ctx->device), "cudaSetDevice");
+  ctx->last_ws = ws;
+  TraceDev d = to_dev(t);
+  CK(cudaMemsetAsync(w.err, 0, sizeof(DevErr), s), "memset");
+  CK(launch_validate_offsets(d, w.err, s), "validate");
+  CK(launch_table_prep(d, w.tbl, w.max_len, w.err, s), "table");
+  if (warp_bbv16 || warp_insts)
+    CK(launch_bbv(d, w.tbl, w.max_len, warp_bbv16, warp_insts, nullptr, nullptr, w.err, ctx->num_sms, s), "bbv");
+  if (kernel_bb_insts) CK(launch_kernel_bb_insts(d, w.tbl, kernel_bb_insts, w.err, ctx->num_sms, s), "kbb");
+  return PHOTON_OK;
+}
+
+// ---- A2 -----------------------------------------------------------------------------------------------------
+size_t photon_group_workspace_bytes(const photon_trace* t, uint64_t hint) {
+  return t ? group_layout(t, hint, nullptr, 0).bytes : 0;
+}
+
+int photon_warp_group(photon_ctx* ctx, const photon_trace* t, const uint32_t* warp_bbv16, void* ws, size_t ws_bytes,
+                      photon_types* out, void* stream) {
+  if (!ctx) return PHOTON_EINVAL;
+  int rc = check_trace(ctx, t);
+  if (rc) return rc;
+  if (!ws || !out) return fail(ctx, PHOTON_EINVAL, "workspace or output is NULL");
+  if (!out->warp_type || !out->kernel_type_off || !out->type_key || !out->type_count || !out->type_first_warp ||
+      !out->warp_sampling_ok)
+    return fail(ctx, PHOTON_EINVAL, "NULL photon_types array");
+  if (!aligned(out->type_key, 16)) return fail(ctx, PHOTON_EINVAL, "type_key must be 16-byte aligned");
+  if (warp_bbv16 && !aligned(warp_bbv16, 16)) return fail(ctx, PHOTON_EINVAL, "warp_bbv16 must be 16-byte aligned");
+  GroupWs g0 = group_layout(t, 0, nullptr, 0);
+  if (ws_bytes < g0.b.bytes + 256) return fail(ctx, PHOTON_EWORKSPACE, "workspace too small");
+  GroupWs g = group_layout(t, 1, ws, ws_bytes);  // largest table that fits
+  if (g.bytes > ws_bytes) return fail(ctx, PHOTON_EWORKSPACE, "workspace %zu < %zu bytes", ws_bytes, g.bytes);
+  cudaStream_t s = (cudaStream_t)stream;
+  CK(cudaSetDevice(ctx->device), "cudaSetDevice");
+  ctx->last_ws = ws;
+  TraceDev d = to_dev(t);
+  DevErr* err = g.b.err;
+  CK(cudaMemsetAsync(err, 0, sizeof(DevErr), s), "memset");
+  CK(launch_ht_clear(g.h.ht, s), "ht_clear");
+  CK(launch_validate_offsets(d, err, s), "validate");
+  if (warp_bbv16) {
+    CK(launch_group_from_bbv(d, warp_bbv16, g.h.ht, out->warp_type, err, s), "group_from_bbv");
+  } else {
+    CK(launch_table_prep(d, g.b.tbl, g.b.max_len, err, s), "table");
+    CK(launch_bbv(d, g.b.tbl, g.b.max_len, nullptr, nullptr, &g.h.ht, out->warp_type, err, ctx->num_sms, s),
+       "bbv_fused");
+  }
+  CK(launch_canonicalise(g.h.ht, t->n_kernels, t->kernel_warp_off, nullptr, *out, g.h.cw, err, ctx->num_sms, s),
+     "canon");
+  CK(launch_remap(out->warp_type, g.h.cw.canon, t->n_warps, out->warp_type, err, s), "remap");
+  return PHOTON_OK;
+}
+
+int photon_types_total(photon_ctx* ctx, const photon_types* types, uint32_t K, uint64_t* total, void* stream) {
+  if (!ctx || !types || !total || !types->kernel_type_off) return PHOTON_EINVAL;
+  CK(cudaStreamSynchronize((cudaStream_t)stream), "sync");
+  CK(cudaMemcpy(total, types->kernel_type_off + K, 8, cudaMemcpyDeviceToHost), "read total");
+  return PHOTON_OK;
+}
+
+// ---- A3 + A4 ------------------------------------------------------------------------------------------------
+size_t photon_match_workspace_bytes(uint32_t K, uint64_t T, uint64_t pair_cap) {
+  return match_layout(K, T, pair_cap, nullptr).bytes;
+}
+
+int photon_kernel_match(photon_ctx* ctx, uint32_t K, const photon_types* types, const uint64_t* warps_total,
+                        photon_match_params params, void* ws, size_t ws_bytes, int64_t* match, double* match_dist,
+                        void* stream) {
+  if (!ctx) return PHOTON_EINVAL;
+  if (!types || !types->kernel_type_off || !types->type_key || !types->type_count || !warps_total || !match || !ws)
+    return fail(ctx, PHOTON_EINVAL, "NULL argument");
+  if (K == 0) return fail(ctx, PHOTON_EINVAL, "K must be >= 1");
+  params = norm_params(params);
+  int rc = check_match_params(ctx, params);
+  if (rc) return rc;
+  uint64_t T = types->capacity;
+  MatchLayout m0 = match_layout(K, T, 1024, nullptr);
+  if (ws_bytes < m0.bytes) return fail(ctx, PHOTON_EWORKSPACE, "workspace %zu < %zu bytes", ws_bytes, m0.bytes);
+  MatchLayout m = match_layout_fit(K, T, ws, ws_bytes);
+  cudaStream_t s = (cudaStream_t)stream;
+  CK(cudaSetDevice(ctx->device), "cudaSetDevice");
+  ctx->last_ws = ws;
+  CK(cudaMemsetAsync(m.err, 0, sizeof(DevErr), s), "memset");
+  CK(launch_sig_build(K, types->kernel_type_off, types->type_key, types->type_count, 0, K, m.sig, m.mass, m.err, s),
+     "sig");
+  CK(launch_match_scan(K, types->kernel_type_off, m.sig, m.mass, warps_total, params, 0, K, m.mw, m.pairs,
+                       m.mw.pair_cap, m.n_pairs, m.err, ctx->num_sms, s),
+     "scan");
+  CK(launch_match_resolve(K, types->kernel_type_off, m.sig, m.mass, warps_total, params, m.pairs, m.mw.pair_cap,
+                          m.n_pairs, m.mw, match, match_dist, m.err, s),
+     "resolve");
+  return PHOTON_OK;
+}
+
+int photon_sig_build(photon_ctx* ctx, uint32_t K, const uint64_t* kto, const uint32_t* type_key,
+                     const uint64_t* type_count, uint32_t k_lo, uint32_t k_hi, uint64_t* sig, uint64_t* mass,
+                     void* ws, size_t ws_bytes, void* stream) {
+  if (!ctx) return PHOTON_EINVAL;
+  if (!kto || !type_key || !type_count || !sig || !mass || k_hi > K || k_lo > k_hi || !ws)
+    return fail(ctx, PHOTON_EINVAL, "bad sig_build arguments");
+  if (ws_bytes < 256) return fail(ctx, PHOTON_EWORKSPACE, "sig_build workspace must be >= 256 bytes");
+  cudaStream_t s = (cudaStream_t)stream;
+  CK(cudaSetDevice(ctx->device), "cudaSetDevice");
+  ctx->last_ws = ws;
+  DevErr* err = (DevErr*)ws;
+  CK(cudaMemsetAsync(err, 0, sizeof(DevErr), s), "memset");
+  CK(launch_sig_build(K, kto, type_key, type_count, k_lo, k_hi, sig, mass, err, s), "sig");
+  return PHOTON_OK;
+}
+
+int photon_match_scan(photon_ctx* ctx, uint32_t K, const uint64_t* kto, const uint64_t* sig, const uint64_t* mass,
+                      const uint64_t* warps_total, photon_match_params params, uint32_t k_lo, uint32_t k_hi, void* ws,
+                      size_t ws_bytes, uint64_t* pairs, uint64_t pair_capacity, uint64_t* n_pairs, void* stream) {
+  if (!ctx) return PHOTON_EINVAL;
+  if (!kto || !sig || !mass || !warps_total || !ws || !pairs || !n_pairs || k_hi > K || k_lo > k_hi || K == 0)
+    return fail(ctx, PHOTON_EINVAL, "bad match_scan arguments");
+  params = norm_params(params);
+  int rc = check_match_params(ctx, params);
+  if (rc) return rc;
+  MatchLayout m0 = match_layout(K, 1, 1024, nullptr);
+  if (ws_bytes < m0.bytes) return fail(ctx, PHOTON_EWORKSPACE, "workspace too small");
+  MatchLayout m = match_layout_fit(K, 1, ws, ws_bytes);
+  cudaStream_t s = (cudaStream_t)stream;
+  CK(cudaSetDevice(ctx->device), "cudaSetDevice");
+  ctx->last_ws = ws;
+  CK(cudaMemsetAsync(m.err, 0, sizeof(DevErr), s), "memset");
+  CK(launch_match_scan(K, kto, sig, mass, warps_total, params, k_lo, k_hi, m.mw, pairs, pair_capacity, n_pairs, m.err,
+                       ctx->num_sms, s),
+     "scan");
+  return PHOTON_OK;
+}
+
+int photon_match_resolve(photon_ctx* ctx, uint32_t K, const uint64_t* kto, const uint64_t* sig, const uint64_t* mass,
+                         const uint64_t* warps_total, photon_match_params params, const uint64_t* pairs,
+                         uint64_t n_pairs, void* ws, size_t ws_bytes, int64_t* match, double* match_dist,
+                         void* stream) {
+  if (!ctx) return PHOTON_EINVAL;
+  if (!kto || !sig || !mass || !warps_total || !ws || (n_pairs && !pairs) || !match || K == 0)
+    return fail(ctx, PHOTON_EINVAL, "bad match_resolve arguments");
+  params = norm_params(params);
+  int rc = check_match_params(ctx, params);
+  if (rc) return rc;
+  // resolve needs cand arrays for n_pairs entries
+  MatchLayout m = match_layout(K, 1, n_pairs ? n_pairs : 1, nullptr);
+  if (ws_bytes < m.bytes) return fail(ctx, PHOTON_EWORKSPACE, "workspace %zu < %zu bytes", ws_bytes, m.bytes);
+  m = match_layout_fit(K, 1, ws, ws_bytes);
+  cudaStream_t s = (cudaStream_t)stream;
+  CK(cudaSetDevice(ctx->device), "cudaSetDevice");
+  ctx->last_ws = ws;
+  CK(cudaMemsetAsync(m.err, 0, sizeof(DevErr), s), "memset");
+  CK(launch_match_resolve(K, kto, sig, mass, warps_total, params, pairs, n_pairs, nullptr, m.mw, match, match_dist,
+                          m.err, s),
+     "resolve");
+  return PHOTON_OK;
+}
+
+// ---- A5 -----------------------------------------------------------------------------------------------------
+size_t photon_stable_workspace_bytes(const photon_timing* t) { return t ? stable_layout(t, nullptr).bytes : 0; }
+
+int photon_bb_stable(photon_ctx* ctx, const photon_timing* t, const uint64_t* kbb, photon_stable_params p, void* ws,
+                     size_t ws_bytes, int64_t* first_stable, uint64_t* dur, int64_t* switch_at, void* stream) {
+  if (!ctx) return PHOTON_EINVAL;
+  if (!t || !t->kernel_rec_off || (t->n_records && (!t->bb || !t->issue || !t->retire)) || !kbb || !first_stable ||
+      !switch_at || !ws)
+    return fail(ctx, PHOTON_EINVAL, "NULL argument");
+  if (t->n_kernels == 0 || t->n_bb == 0 || t->n_bb > 65536 || t->n_records >= (1ull << 32))
+    return fail(ctx, PHOTON_EINVAL, "bad timing sizes");
+  if (p.window_n == 0) { p.window_n = 2048; }
+  if (p.delta_den == 0) { p.delta_num = 3; p.delta_den = 100; }
+  if (p.rate_den == 0) { p.rate_num = 95; p.rate_den = 100; }
+  if (p.window_n < 2 || p.window_n > 8192 || p.delta_den > (1u << 16) || p.delta_num > p.delta_den ||
+      p.rate_den > (1u << 16) || p.rate_num > p.rate_den)
+    return fail(ctx, PHOTON_EINVAL, "bad stable params");
+  StableWs w = stable_layout(t, ws);
+  if (ws_bytes < w.bytes) return fail(ctx, PHOTON_EWORKSPACE, "workspace %zu < %zu bytes", ws_bytes, w.bytes);
+  cudaStream_t s = (cudaStream_t)stream;
+  CK(cudaSetDevice(ctx->device), "cudaSetDevice");
+  ctx->last_ws = ws;
+  CK(cudaMemsetAsync(w.err, 0, sizeof(DevErr), s), "memset");
+  CK(launch_stable(*t, kbb, p, w.rest, w.rest_bytes, first_stable, dur, switch_at, w.err, ctx->num_sms, s), "stable");
+  return PHOTON_OK;
+}
+
+// ---- multi-GPU helpers ------------------------------------------------------------------------------------
+int photon_types_export(photon_ctx* ctx, uint32_t K_local, const photon_types* local, uint32_t kernel_base,
+                        uint64_t warp_base, photon_type_row* rows, void* stream) {
+  if (!ctx) return PHOTON_EINVAL;
+  if (!local || !rows || K_local == 0) return fail(ctx, PHOTON_EINVAL, "bad export arguments");
+  CK(cudaSetDevice(ctx->device), "cudaSetDevice");
+  CK(launch_types_export(K_local, *local, kernel_base, warp_base, rows, (cudaStream_t)stream), "export");
+  return PHOTON_OK;
+}
+
+size_t photon_merge_workspace_bytes(uint64_t n_rows, uint32_t K) { return merge_layout(n_rows, K, nullptr).bytes; }
+
+int photon_types_merge(photon_ctx* ctx, const photon_type_row* rows, uint64_t n_rows, uint32_t K,
+                       const uint64_t* kernel_warps, void* ws, size_t ws_bytes, photon_types* global, void* stream) {
+  if (!ctx) return PHOTON_EINVAL;
+  if ((n_rows && !rows) || K == 0 || !kernel_warps || !ws || !global || !global->kernel_type_off ||
+      !global->type_key || !global->type_count || !global->type_first_warp || !global->warp_sampling_ok)
+    return fail(ctx, PHOTON_EINVAL, "bad merge arguments");
+  MergeWs m = merge_layout(n_rows, K, ws);
+  if (ws_bytes < m.bytes) return fail(ctx, PHOTON_EWORKSPACE, "workspace %zu < %zu bytes", ws_bytes, m.bytes);
+  cudaStream_t s = (cudaStream_t)stream;
+  CK(cudaSetDevice(ctx->device), "cudaSetDevice");
+  ctx->last_ws = ws;
+  CK(cudaMemsetAsync(m.err, 0, sizeof(DevErr), s), "memset");
+  CK(launch_ht_clear(m.h.ht, s), "ht_clear");
+  CK(launch_rows_insert(rows, n_rows, K, m.h.ht, m.err, s), "rows_insert");
+  CK(launch_canonicalise(m.h.ht, K, nullptr, kernel_warps, *global, m.h.cw, m.err, ctx->num_sms, s), "canon");
+  return PHOTON_OK;
+}
+
+int photon_types_remap(photon_ctx* ctx, uint32_t K_local, uint64_t W_local, const uint64_t* kernel_warp_off_local,
+                       const photon_types* local, uint32_t kernel_base, uint64_t n_rows_merged, uint32_t K_global,
+                       const void* merge_ws, size_t ws_bytes, uint32_t* warp_type_global, void* stream) {
+  if (!ctx) return PHOTON_EINVAL;
+  if (!local || !kernel_warp_off_local || !merge_ws || !warp_type_global || K_local == 0)
+    return fail(ctx, PHOTON_EINVAL, "bad remap arguments");
+  MergeWs m = merge_layout(n_rows_merged, K_global, (void*)merge_ws);
+  if (ws_bytes < m.bytes) return fail(ctx, PHOTON_EWORKSPACE, "merge workspace mismatch");
+  CK(cudaSetDevice(ctx->device), "cudaSetDevice");
+  CK(launch_remap_direct(kernel_warp_off_local, K_local, W_local, *local, kernel_base, m.h.ht, m.h.cw.canon,
+                         warp_type_global, m.err, (cudaStream_t)stream),
+     "remap");
+  return PHOTON_OK;
+}
+
+}  // extern "C"

@@ -1,0 +1,180 @@
+// common.cuh — device helpers shared by the libphoton kernels (sm_100a only).
+#pragma once
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include "../../include/photon.h"
+
+#if defined(__CUDA_ARCH__) && (__CUDA_ARCH__ < 1000)
+#error "libphoton is written for sm_100a (B200) only"
+#endif
+
+namespace photon {
+
+typedef unsigned __int128 u128;
+typedef __int128 i128;
+
+constexpr uint64_t kTimeLimit = 1ull << 40;  // [P-16] ticks < 2^40
+constexpr uint64_t kMassLimit = 1ull << 50;  // N_k < 2^50 (u128 cross products stay exact)
+constexpr uint64_t kInstsLimit = 1ull << 32; // per-warp instructions < 2^32 (u32 bins)
+constexpr uint32_t kMaxLen = (1u << 18) - 1; // bb_len < 2^18 (packed table entry)
+
+// ---- device error latch: first error wins (code, index) -----------------------------------------------------
+struct DevErr {
+  int32_t code;
+  int32_t pad;
+  int64_t index;
+};
+
+__device__ __forceinline__ void latch(DevErr* e, int code, int64_t index) {
+  if (atomicCAS(&e->code, 0, code) == 0) {
+    e->index = index;
+  }
+}
+
+// ---- workspace carving ------------------------------------------------------------------------------------
+struct Carver {
+  size_t off = 0;
+  uint8_t* base = nullptr;
+  explicit Carver(void* b) : base((uint8_t*)b) {}
+  template <class T>
+  T* take(size_t n) {
+    off = (off + 255) & ~(size_t)255;
+    T* p = base ? (T*)(base + off) : nullptr;
+    off += n * sizeof(T);
+    return p;
+  }
+};
+
+__host__ __device__ __forceinline__ uint64_t umin64(uint64_t a, uint64_t b) { return a < b ? a : b; }
+__host__ __device__ __forceinline__ uint64_t umax64(uint64_t a, uint64_t b) { return a > b ? a : b; }
+__host__ __device__ __forceinline__ uint64_t ceil_div(uint64_t a, uint64_t b) { return (a + b - 1) / b; }
+__host__ __device__ __forceinline__ uint32_t next_pow2_u32(uint32_t v) {
+  uint32_t p = 1;
+  while (p < v) p <<= 1;
+  return p;
+}
+
+// ---- hashing of (kernel, 16-bin key) ----------------------------------------------------------------------
+__device__ __forceinline__ uint64_t mix64(uint64_t x) {
+  x ^= x >> 31;
+  x *= 0x7FB5D329728EA185ull;
+  x ^= x >> 27;
+  x *= 0x81DADEF4BC2DD44Dull;
+  x ^= x >> 33;
+  return x;
+}
+__device__ __forceinline__ uint64_t hash_key(uint32_t k, const uint32_t* p) {
+  uint64_t h = 0x9E3779B97F4A7C15ull ^ ((uint64_t)k * 0xC2B2AE3D27D4EB4Full);
+#pragma unroll
+  for (int j = 0; j < 16; j += 2) {
+    uint64_t v = (uint64_t)p[j] | ((uint64_t)p[j + 1] << 32);
+    h = (h ^ v) * 0x100000001B3ull;
+    h ^= h >> 29;
+  }
+  h = mix64(h);
+  return h ? h : 1;
+}
+
+// ---- PTX wrappers: mbarrier + 1-D bulk copy (TMA engine) ------------------------------------------------------
+__device__ __forceinline__ uint32_t smem_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
+
+__device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count) : "memory");
+}
+__device__ __forceinline__ void fence_mbar_init() {
+  asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+}
+__device__ __forceinline__ void mbar_arrive_expect_tx(uint64_t* bar, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.release.cta.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes)
+               : "memory");
+}
+__device__ __forceinline__ bool mbar_try_wait(uint64_t* bar, uint32_t parity) {
+  uint32_t ok;
+  asm volatile(
+      "{\n .reg .pred p;\n mbarrier.try_wait.parity.acquire.cta.shared::cta.b64 p, [%1], %2;\n selp.u32 %0, 1, 0, p;\n}\n"
+      : "=r"(ok)
+      : "r"(smem_u32(bar)), "r"(parity)
+      : "memory");
+  return ok != 0;
+}
+__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
+  while (!mbar_try_wait(bar, parity)) {
+  }
+}
+// global -> shared bulk copy, completion counted on `bar` (bytes multiple of 16, addresses 16-byte aligned)
+__device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
+  asm volatile(
+      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(smem_u32(dst)),
+      "l"(src), "r"(bytes), "r"(smem_u32(bar))
+      : "memory");
+}
+
+__device__ __forceinline__ uint32_t ld_acquire_u32(const uint32_t* p) {
+  uint32_t v;
+  asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ void st_release_u32(uint32_t* p, uint32_t v) {
+  asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+__device__ __forceinline__ uint32_t ld_relaxed_u32(const uint32_t* p) {
+  uint32_t v;
+  asm volatile("ld.relaxed.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
+
+// ---- 128-bit helpers ---------------------------------------------------------------------------------------
+__device__ __forceinline__ u128 mul64x64(uint64_t a, uint64_t b) {
+  return (u128)a * b;
+}
+
+// ---- global warp-type hash table (workspace) ------------------------------------------------------------------
+struct HashTable {
+  uint64_t* hkey;   // [cap] 0 = empty, else hash (nonzero)
+  uint32_t* ready;  // [cap] 1 once kern/key are published
+  uint32_t* kern;   // [cap]
+  uint32_t* key;    // [cap][16]
+  uint32_t* count;  // [cap]
+  uint64_t* first;  // [cap] min warp index (init ~0)
+  uint64_t mask;    // cap - 1 (cap power of two)
+};
+
+// Insert-or-find (k, p) with hash h.  Returns the slot, or UINT32_MAX (after latching ECAPACITY) when full.
+// Adds `cnt` to the slot's count and lowers its first warp to `wmin`.  Readers spin only on slots whose writer
+// already won the CAS (it runs to completion without waiting), so there is no deadlock.
+__device__ __forceinline__ uint32_t ht_insert(const HashTable& ht, DevErr* err, uint32_t k, const uint32_t* p,
+                                              uint64_t h, uint32_t cnt, uint64_t wmin) {
+  uint64_t i = h & ht.mask;
+  for (uint64_t probe = 0; probe <= ht.mask; ++probe) {
+    unsigned long long cur = atomicCAS((unsigned long long*)&ht.hkey[i], 0ull, (unsigned long long)h);
+    bool mine = false;
+    if (cur == 0ull) {
+      ht.kern[i] = k;
+      uint4* dst = (uint4*)&ht.key[i * 16];
+      dst[0] = make_uint4(p[0], p[1], p[2], p[3]);
+      dst[1] = make_uint4(p[4], p[5], p[6], p[7]);
+      dst[2] = make_uint4(p[8], p[9], p[10], p[11]);
+      dst[3] = make_uint4(p[12], p[13], p[14], p[15]);
+      __threadfence();
+      st_release_u32(&ht.ready[i], 1u);
+      mine = true;
+    } else if (cur == h) {
+      while (ld_acquire_u32(&ht.ready[i]) == 0u) {
+      }
+      mine = ld_relaxed_u32(&ht.kern[i]) == k;
+#pragma unroll
+      for (int j = 0; j < 16; ++j) mine = mine && (ld_relaxed_u32(&ht.key[i * 16 + j]) == p[j]);
+    }
+    if (mine) {
+      atomicAdd(&ht.count[i], cnt);
+      atomicMin((unsigned long long*)&ht.first[i], (unsigned long long)wmin);
+      return (uint32_t)i;
+    }
+    i = (i + 1) & ht.mask;
+  }
+  latch(err, PHOTON_ECAPACITY, (int64_t)h);
+  return UINT32_MAX;
+}
+
+}  // namespace photon

@@ -1,0 +1,92 @@
+// internal.h — host-side interface between the C ABI (abi.cu) and the kernel files.
+#pragma once
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include "common.cuh"
+
+namespace photon {
+
+// ---- A1 / A2 (k_bbv.cu) -------------------------------------------------------------------------------------
+struct TraceDev {
+  const uint64_t* kwo;
+  const uint64_t* weo;
+  const uint16_t* bb;
+  const uint32_t* bb_len;
+  const uint8_t* bb_bin;
+  uint32_t K, B;
+  uint64_t W, E;
+};
+
+// packed per-BB table (len << 14 | bin << 10; bit 0 marks ids in [B, P2)), P2 = next pow2 >= B
+size_t bbv_table_bytes(uint32_t B);
+cudaError_t launch_table_prep(const TraceDev& t, uint32_t* tbl, uint32_t* max_len, DevErr* err, cudaStream_t s);
+cudaError_t launch_validate_offsets(const TraceDev& t, DevErr* err, cudaStream_t s);
+// streaming K1 (+ fused K2a when ht != nullptr)
+cudaError_t launch_bbv(const TraceDev& t, const uint32_t* tbl, const uint32_t* max_len, uint32_t* warp_bbv16,
+                       uint64_t* warp_insts, const HashTable* ht, uint32_t* warp_slot, DevErr* err, int num_sms,
+                       cudaStream_t s);
+// K2a from materialised BBVs (unfused path)
+cudaError_t launch_group_from_bbv(const TraceDev& t, const uint32_t* warp_bbv16, const HashTable& ht,
+                                  uint32_t* warp_slot, DevErr* err, cudaStream_t s);
+cudaError_t launch_kernel_bb_insts(const TraceDev& t, const uint32_t* tbl, uint64_t* kbb, DevErr* err,
+                                   int num_sms, cudaStream_t s);
+
+// ---- A2 canonicalisation (k_types.cu) ---------------------------------------------------------------------
+cudaError_t launch_ht_clear(const HashTable& ht, cudaStream_t s);
+struct CanonWs {
+  uint32_t* tcount;   // [K] types per kernel
+  uint32_t* cursor;   // [K]
+  uint32_t* list;     // [cap] slot ids grouped by kernel
+  uint32_t* canon;    // [cap] slot -> kernel-local canonical id
+  uint64_t* scratch;  // [cap] sort scratch (large kernels)
+};
+// From the hash table to canonical photon_types (kernel_type_off, rows, warp_sampling_ok) and the slot->id map.
+cudaError_t launch_canonicalise(const HashTable& ht, uint32_t K, const uint64_t* kwo_or_null,
+                                const uint64_t* kernel_warps_or_null, const photon_types& out, const CanonWs& cw,
+                                DevErr* err, int num_sms, cudaStream_t s);
+// warp_type[w] = canon[warp_slot[w]]  (in place allowed)
+cudaError_t launch_remap(const uint32_t* warp_slot, const uint32_t* canon, uint64_t W, uint32_t* warp_type,
+                         DevErr* err, cudaStream_t s);
+// multi-GPU helpers
+cudaError_t launch_types_export(uint32_t K, const photon_types& local, uint32_t kernel_base, uint64_t warp_base,
+                                photon_type_row* rows, cudaStream_t s);
+cudaError_t launch_rows_insert(const photon_type_row* rows, uint64_t n, uint32_t K, const HashTable& ht,
+                               DevErr* err, cudaStream_t s);
+// warp_type_global[v] = canonical id (in the merged table) of local warp v's type (direct hash lookup)
+cudaError_t launch_remap_direct(const uint64_t* kwo_local, uint32_t K_local, uint64_t W_local,
+                                const photon_types& local, uint32_t kernel_base, const HashTable& ht,
+                                const uint32_t* canon, uint32_t* warp_type_global, DevErr* err, cudaStream_t s);
+
+// ---- A3/A4 (k_match.cu) -----------------------------------------------------------------------------------
+struct MatchWs {
+  float* prof;         // [K][16] normalised per-bin profile (filter)
+  uint64_t* maybe;     // [pair_cap] profile-filter survivors
+  uint64_t* n_maybe;   // [1]
+  uint32_t* cand_cnt;  // [K]
+  uint64_t* cand_off;  // [K+1]
+  uint32_t* cand_cur;  // [K]
+  uint32_t* cand;      // [pair_cap] r per (k, r), grouped by k
+  uint8_t* state;      // [K] 0 undecided, 1 representative, 2 matched
+  uint32_t* flag;      // [4]
+  uint64_t pair_cap;
+};
+cudaError_t launch_sig_build(uint32_t K, const uint64_t* kto, const uint32_t* type_key, const uint64_t* type_count,
+                             uint32_t k_lo, uint32_t k_hi, uint64_t* sig, uint64_t* mass, DevErr* err, cudaStream_t s);
+cudaError_t launch_match_scan(uint32_t K, const uint64_t* kto, const uint64_t* sig, const uint64_t* mass,
+                              const uint64_t* wt, photon_match_params p, uint32_t k_lo, uint32_t k_hi,
+                              const MatchWs& mw, uint64_t* pairs, uint64_t pair_cap, uint64_t* n_pairs, DevErr* err,
+                              int num_sms, cudaStream_t s);
+cudaError_t launch_match_resolve(uint32_t K, const uint64_t* kto, const uint64_t* sig, const uint64_t* mass,
+                                 const uint64_t* wt, photon_match_params p, const uint64_t* pairs, uint64_t n_pairs,
+                                 const uint64_t* n_pairs_dev, const MatchWs& mw, int64_t* match, double* match_dist,
+                                 DevErr* err, cudaStream_t s);
+
+// ---- A5 (k_stable.cu) -------------------------------------------------------------------------------------
+struct StableLayout;
+size_t stable_ws_bytes(const photon_timing& t);
+cudaError_t launch_stable(const photon_timing& t, const uint64_t* kbb, photon_stable_params p, void* ws,
+                          size_t ws_bytes, int64_t* first_stable, uint64_t* dur, int64_t* switch_at, DevErr* err,
+                          int num_sms, cudaStream_t s);
+
+}  // namespace photon

@@ -1,0 +1,365 @@
+// k_match.cu — A3 (GPU-BBV signature) and A4 (kernel matching).
+//
+// PAPER.md L178 / Fig 5 (L159): the GPU BBV lists the weighted per-type BBVs in descending weight order; [P-5] it is
+// scaled to unit L1 mass, so with g_k = concat_t (c_t * key_t) (integers) and N_k = sum g_k the GPU BBV is g_k/N_k.
+// Fig 12 (L271) Step 2: "finds all prior kernels whose distance is less than the threshold" [P-6 L1, P-7 theta,
+// P-8 pool = representatives, P-15 strict]; Step 3: "selects kernels whose warp count is closest" [P-9]; note:
+// warp counts must be equal below the GPU core count [P-10] (also L277).
+//
+// Design: the decision is exact in u128: theta_den * sum_i |g_k[i] N_r - g_r[i] N_k| <
+// theta_num * N_k * N_r.  To avoid the O(K^2 L) exact work, pairs are first filtered with a provably conservative
+// fp32 lower bound: the per-bin profile distance sum_j |P_k[j] - P_r[j]| (P = per-bin sums of g/N) is <= D by the
+// triangle inequality; a pair is dropped only if that bound exceeds theta by more than its worst rounding error.
+// Survivors get the exact u128 check (one warp per pair).  Launch-order resolution (leader clustering) is then a
+// parallel fixed point: k is a representative iff none of its close predecessors is one.
+#include <math.h>
+
+#include "internal.h"
+
+namespace photon {
+
+namespace {
+
+// ---- A3: g = count * key, N = sum g (one warp per kernel) ------------------------------------------------
+__global__ void k_sig(uint32_t k_lo, uint32_t k_hi, const uint64_t* __restrict__ kto,
+                      const uint32_t* __restrict__ key, const uint64_t* __restrict__ count, uint64_t* __restrict__ sig,
+                      uint64_t* __restrict__ mass, DevErr* err) {
+  uint32_t warp = (blockIdx.x * blockDim.x + threadIdx.x) >> 5, lane = threadIdx.x & 31;
+  uint32_t k = k_lo + warp;
+  if (k >= k_hi) return;
+  uint64_t r0 = kto[k], r1 = kto[k + 1];
+  uint64_t acc = 0;
+  bool over = false;
+  for (uint64_t i = r0 * 16 + lane; i < r1 * 16; i += 32) {
+    uint64_t c = count[i >> 4];
+    uint64_t g;
+    over |= c >= (1ull << 32);
+    g = c * (uint64_t)key[i];
+    sig[i] = g;
+    over |= g >= kMassLimit;
+    acc += g;
+    over |= acc >= kMassLimit;
+  }
+  for (int o = 16; o > 0; o >>= 1) {
+    acc += __shfl_xor_sync(0xffffffffu, acc, o);
+    over |= __shfl_xor_sync(0xffffffffu, (int)over, o) != 0;
+  }
+  if (lane == 0) {
+    if (over || acc >= kMassLimit) latch(err, PHOTON_ERANGE, (int64_t)k);
+    mass[k] = acc;
+  }
+}
+
+// per-bin profile P_k[j] = sum_t g[16t+j] / N_k (filter only), one warp per kernel
+__global__ void k_prof(uint32_t K, const uint64_t* __restrict__ kto, const uint64_t* __restrict__ sig,
+                       const uint64_t* __restrict__ mass, float* __restrict__ prof) {
+  uint32_t warp = (blockIdx.x * blockDim.x + threadIdx.x) >> 5, lane = threadIdx.x & 31;
+  if (warp >= K) return;
+  uint32_t k = warp;
+  uint64_t r0 = kto[k], r1 = kto[k + 1];
+  uint64_t acc = 0;
+  for (uint64_t r = r0 + (lane >> 4); r < r1; r += 2) acc += sig[r * 16 + (lane & 15)];
+  acc += __shfl_xor_sync(0xffffffffu, acc, 16);
+  if (lane < 16) {
+    uint64_t N = mass[k];
+    prof[(uint64_t)k * 16 + lane] = N ? (float)((double)acc / (double)N) : 0.f;
+  }
+}
+
+// ---- pair filter: 64 x 64 tiles of (k, r < k) --------------------------------------------------------------
+constexpr int FT = 64;
+struct ScanArgs {
+  uint32_t K, k_lo, k_hi;
+  const uint64_t* kto;
+  const uint64_t* sig;
+  const uint64_t* mass;
+  const uint64_t* wt;
+  const float* prof;
+  photon_match_params p;
+  float bound;  // reject if profile distance >= bound
+  uint64_t* maybe;
+  uint64_t* n_maybe;
+  uint64_t cap;
+  DevErr* err;
+};
+
+__global__ void __launch_bounds__(256) k_pair_filter(ScanArgs a, uint64_t t0) {
+  // blockIdx.x enumerates lower-triangle tiles (kb, rb) with rb <= kb, kb over [k_lo, k_hi) in FT blocks
+  uint64_t t = t0 + blockIdx.x;
+  // invert t = kb*(kb+1)/2 + rb relative to the first k block
+  uint32_t kb = (uint32_t)((sqrt(8.0 * (double)t + 1.0) - 1.0) * 0.5);
+  while ((uint64_t)(kb + 1) * (kb + 2) / 2 <= t) ++kb;
+  while ((uint64_t)kb * (kb + 1) / 2 > t) --kb;
+  uint32_t rb = t - kb * (kb + 1) / 2;
+
+  uint32_t k0 = kb * FT, r0 = rb * FT;  // absolute kernel indices (k blocks start at 0; k < k_lo are skipped)
+  __shared__ float pk[FT][17], pr[FT][17];
+  __shared__ uint64_t wk[FT], wr[FT], nk[FT], nr[FT];
+  for (int i = threadIdx.x; i < FT * 16; i += 256) {
+    int row = i >> 4, j = i & 15;
+    uint32_t k = k0 + row, r = r0 + row;
+    pk[row][j] = k < a.K ? a.prof[(uint64_t)k * 16 + j] : 0.f;
+    pr[row][j] = r < a.K ? a.prof[(uint64_t)r * 16 + j] : 0.f;
+  }
+  for (int i = threadIdx.x; i < FT; i += 256) {
+    uint32_t k = k0 + i, r = r0 + i;
+    wk[i] = k < a.K ? a.wt[k] : 0; nk[i] = k < a.K ? a.mass[k] : 0;
+    wr[i] = r < a.K ? a.wt[r] : 0; nr[i] = r < a.K ? a.mass[r] : 0;
+  }
+  __syncthreads();
+  for (int idx = threadIdx.x; idx < FT * FT; idx += 256) {
+    int i = idx / FT, j = idx % FT;
+    uint32_t k = k0 + i, r = r0 + j;
+    if (k >= a.k_hi || k < a.k_lo || r >= k) continue;
+    if (nk[i] == 0 || nr[j] == 0) continue;  // [P-19]
+    uint64_t Wk = wk[i], Wr = wr[j];
+    if (!(Wk == Wr || (Wk < Wr ? Wk : Wr) >= a.p.n_cores)) continue;  // [P-10]
+    float d = 0.f;
+#pragma unroll
+    for (int b = 0; b < 16; ++b) d += fabsf(pk[i][b] - pr[j][b]);
+    if (d >= a.bound) continue;
+    unsigned long long pos = atomicAdd((unsigned long long*)a.n_maybe, 1ull);
+    if (pos < a.cap) a.maybe[pos] = ((uint64_t)k << 32) | r;
+    else latch(a.err, PHOTON_ECAPACITY, (int64_t)pos);
+  }
+}
+
+// exact Dnum = sum_i |g_k[i] N_r - g_r[i] N_k| (zero padded), warp-cooperative; all lanes return the total
+__device__ u128 warp_dnum(const uint64_t* sig, const uint64_t* kto, const uint64_t* mass, uint32_t k, uint32_t r,
+                          u128 stop_at) {
+  const uint32_t lane = threadIdx.x & 31;
+  uint64_t ok = kto[k] * 16, orr = kto[r] * 16;
+  uint64_t Lk = (kto[k + 1] - kto[k]) * 16, Lr = (kto[r + 1] - kto[r]) * 16;
+  uint64_t L = Lk > Lr ? Lk : Lr;
+  uint64_t Nk = mass[k], Nr = mass[r];
+  u128 total = 0;
+  for (uint64_t base = 0; base < L; base += 32 * 8) {
+    u128 acc = 0;
+#pragma unroll 4
+    for (int u = 0; u < 8; ++u) {
+      uint64_t i = base + (uint64_t)u * 32 + lane;
+      if (i < L) {
+        uint64_t gk = i < Lk ? sig[ok + i] : 0, gr = i < Lr ? sig[orr + i] : 0;
+        u128 x = (u128)gk * Nr, y = (u128)gr * Nk;
+        acc += x > y ? x - y : y - x;
+      }
+    }
+    uint64_t lo = (uint64_t)acc, hi = (uint64_t)(acc >> 64);
+    for (int o = 16; o > 0; o >>= 1) {
+      uint64_t lo2 = __shfl_xor_sync(0xffffffffu, lo, o), hi2 = __shfl_xor_sync(0xffffffffu, hi, o);
+      uint64_t s = lo + lo2;
+      hi = hi + hi2 + (s < lo ? 1 : 0);
+      lo = s;
+    }
+    total += ((u128)hi << 64) | lo;
+    if (total >= stop_at) break;  // early exit: already not close
+  }
+  return total;
+}
+
+__global__ void k_pair_exact(ScanArgs a, uint64_t* pairs, uint64_t pair_cap, uint64_t* n_pairs) {
+  uint64_t n = *a.n_maybe;
+  if (n > a.cap) n = a.cap;
+  uint64_t warp = ((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  uint64_t nw = ((uint64_t)gridDim.x * blockDim.x) >> 5;
+  for (uint64_t q = warp; q < n; q += nw) {
+    uint64_t pr = a.maybe[q];
+    uint32_t k = (uint32_t)(pr >> 32), r = (uint32_t)pr;
+    u128 rhs = (u128)a.p.theta_num * ((u128)a.mass[k] * a.mass[r]);
+    // close <=> theta_den * Dnum < rhs ; stop once theta_den * Dnum >= rhs  <=>  Dnum >= ceil(rhs / theta_den)
+    u128 stop = (rhs + a.p.theta_den - 1) / a.p.theta_den;
+    u128 d = warp_dnum(a.sig, a.kto, a.mass, k, r, stop);
+    if ((threadIdx.x & 31) == 0 && (u128)a.p.theta_den * d < rhs) {
+      unsigned long long pos = atomicAdd((unsigned long long*)n_pairs, 1ull);
+      if (pos < pair_cap) pairs[pos] = pr;
+      else latch(a.err, PHOTON_ECAPACITY, (int64_t)pos);
+    }
+  }
+}
+
+// ---- resolve -------------------------------------------------------------------------------------------------
+__device__ __forceinline__ uint64_t pair_count(uint64_t n_host, const uint64_t* n_dev) {
+  return n_dev ? umin64(*n_dev, n_host) : n_host;
+}
+
+__global__ void k_cand_count(const uint64_t* pairs, uint64_t n_host, const uint64_t* n_dev, uint32_t K, uint32_t* cnt,
+                             DevErr* err) {
+  uint64_t n = pair_count(n_host, n_dev);
+  uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= n) return;
+  uint32_t k = (uint32_t)(pairs[i] >> 32), r = (uint32_t)pairs[i];
+  if (k >= K || r >= k) { latch(err, PHOTON_EINVAL, (int64_t)i); return; }
+  atomicAdd(&cnt[k], 1u);
+}
+
+__global__ void __launch_bounds__(1024) k_cand_scan(const uint32_t* cnt, uint32_t K, uint64_t* off, uint32_t* cur) {
+  __shared__ uint64_t ws[32];
+  __shared__ uint64_t carry;
+  if (threadIdx.x == 0) carry = 0;
+  __syncthreads();
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+  for (uint32_t base = 0; base < K; base += 1024) {
+    uint32_t k = base + threadIdx.x;
+    uint64_t v = k < K ? cnt[k] : 0;
+    if (k < K) cur[k] = 0;
+    uint64_t x = v;
+    for (int o = 1; o < 32; o <<= 1) {
+      uint64_t y = __shfl_up_sync(0xffffffffu, x, o);
+      if (lane >= o) x += y;
+    }
+    if (lane == 31) ws[wid] = x;
+    __syncthreads();
+    if (wid == 0) {
+      uint64_t s = ws[lane];
+      for (int o = 1; o < 32; o <<= 1) {
+        uint64_t y = __shfl_up_sync(0xffffffffu, s, o);
+        if (lane >= o) s += y;
+      }
+      ws[lane] = s;
+    }
+    __syncthreads();
+    uint64_t excl = carry + (wid ? ws[wid - 1] : 0) + x - v;
+    if (k < K) off[k] = excl;
+    __syncthreads();
+    if (threadIdx.x == 1023) carry = excl + v;
+    __syncthreads();
+  }
+  if (threadIdx.x == 0) off[K] = carry;
+}
+
+__global__ void k_cand_scatter(const uint64_t* pairs, uint64_t n_host, const uint64_t* n_dev, uint32_t K,
+                               const uint64_t* off, uint32_t* cur, uint32_t* cand) {
+  uint64_t n = pair_count(n_host, n_dev);
+  uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= n) return;
+  uint32_t k = (uint32_t)(pairs[i] >> 32), r = (uint32_t)pairs[i];
+  if (k >= K || r >= k) return;
+  cand[off[k] + atomicAdd(&cur[k], 1u)] = r;
+}
+
+// Fixed point of the launch-order rule: state 1 = representative, 2 = matched.  k decides once all its candidate
+// predecessors have decided (or one of them is a representative).  One CTA; monotone state (races benign).
+__global__ void __launch_bounds__(1024) k_resolve_states(uint32_t K, const uint64_t* off, const uint32_t* cand,
+                                                         uint8_t* state, uint32_t pool_all) {
+  for (uint32_t k = threadIdx.x; k < K; k += blockDim.x) state[k] = 0;
+  __syncthreads();
+  if (pool_all) {
+    for (uint32_t k = threadIdx.x; k < K; k += blockDim.x) state[k] = off[k + 1] > off[k] ? 2 : 1;
+    return;
+  }
+  volatile uint8_t* vs = state;
+  for (;;) {
+    int undecided = 0;
+    for (uint32_t k = threadIdx.x; k < K; k += blockDim.x) {
+      if (vs[k] != 0) continue;
+      bool any_rep = false, all_dec = true;
+      for (uint64_t i = off[k]; i < off[k + 1]; ++i) {
+        uint8_t s = vs[cand[i]];
+        if (s == 1) { any_rep = true; break; }
+        if (s == 0) all_dec = false;
+      }
+      if (any_rep) vs[k] = 2;
+      else if (all_dec) vs[k] = 1;
+      else undecided = 1;
+    }
+    if (!__syncthreads_or(undecided)) break;
+  }
+}
+
+// match[k] = argmin over eligible candidates of (|W_k - W_r|, r); match_dist exact -> fp64 (one warp per kernel)
+__global__ void k_resolve_match(uint32_t K, const uint64_t* off, const uint32_t* cand, const uint8_t* state,
+                                uint32_t pool_all, const uint64_t* wt, const uint64_t* kto, const uint64_t* sig,
+                                const uint64_t* mass, int64_t* match, double* dist) {
+  uint32_t warp = (blockIdx.x * blockDim.x + threadIdx.x) >> 5, lane = threadIdx.x & 31;
+  if (warp >= K) return;
+  uint32_t k = warp;
+  uint64_t best_dw = ~0ull;
+  uint32_t best_r = UINT32_MAX;
+  if (state[k] == 2) {
+    for (uint64_t i = off[k] + lane; i < off[k + 1]; i += 32) {
+      uint32_t r = cand[i];
+      if (!pool_all && state[r] != 1) continue;
+      uint64_t dw = wt[k] > wt[r] ? wt[k] - wt[r] : wt[r] - wt[k];
+      if (dw < best_dw || (dw == best_dw && r < best_r)) { best_dw = dw; best_r = r; }
+    }
+  }
+  for (int o = 16; o > 0; o >>= 1) {
+    uint64_t dw2 = __shfl_xor_sync(0xffffffffu, best_dw, o);
+    uint32_t r2 = __shfl_xor_sync(0xffffffffu, best_r, o);
+    if (dw2 < best_dw || (dw2 == best_dw && r2 < best_r)) { best_dw = dw2; best_r = r2; }
+  }
+  if (best_r == UINT32_MAX) {
+    if (lane == 0) { match[k] = -1; if (dist) dist[k] = INFINITY; }
+    return;
+  }
+  if (lane == 0) match[k] = (int64_t)best_r;
+  if (dist) {
+    u128 d = warp_dnum(sig, kto, mass, k, best_r, ~(u128)0);
+    if (lane == 0) {
+      u128 den = (u128)mass[k] * mass[best_r];
+      double dn = (double)(uint64_t)(d >> 64) * 18446744073709551616.0 + (double)(uint64_t)d;
+      double dd = (double)(uint64_t)(den >> 64) * 18446744073709551616.0 + (double)(uint64_t)den;
+      dist[k] = dn / dd;
+    }
+  }
+}
+
+}  // namespace
+
+cudaError_t launch_sig_build(uint32_t K, const uint64_t* kto, const uint32_t* type_key, const uint64_t* type_count,
+                             uint32_t k_lo, uint32_t k_hi, uint64_t* sig, uint64_t* mass, DevErr* err, cudaStream_t s) {
+  (void)K;
+  if (k_hi <= k_lo) return cudaSuccess;
+  uint32_t n = k_hi - k_lo;
+  k_sig<<<(unsigned)ceil_div((uint64_t)n * 32, 256), 256, 0, s>>>(k_lo, k_hi, kto, type_key, type_count, sig, mass, err);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_match_scan(uint32_t K, const uint64_t* kto, const uint64_t* sig, const uint64_t* mass,
+                              const uint64_t* wt, photon_match_params p, uint32_t k_lo, uint32_t k_hi,
+                              const MatchWs& mw, uint64_t* pairs, uint64_t pair_cap, uint64_t* n_pairs, DevErr* err,
+                              int num_sms, cudaStream_t s) {
+  cudaMemsetAsync(n_pairs, 0, 8, s);
+  cudaMemsetAsync(mw.n_maybe, 0, 8, s);
+  if (K == 0 || k_hi <= k_lo) return cudaGetLastError();
+  k_prof<<<(unsigned)ceil_div((uint64_t)K * 32, 256), 256, 0, s>>>(K, kto, sig, mass, mw.prof);
+  ScanArgs a{};
+  a.K = K; a.k_lo = k_lo; a.k_hi = k_hi; a.kto = kto; a.sig = sig; a.mass = mass; a.wt = wt; a.prof = mw.prof;
+  a.p = p;
+  // rigorous margin: each |P_k - P_r| term carries <= 3 fp32 roundings of values in [0, 1] plus 16 additions
+  a.bound = (float)((double)p.theta_num / (double)p.theta_den) + 1e-5f;
+  a.maybe = mw.maybe; a.n_maybe = mw.n_maybe; a.cap = mw.pair_cap; a.err = err;
+  uint32_t kb_hi = (uint32_t)ceil_div(k_hi, FT);
+  uint32_t kb_lo = k_lo / FT;
+  // tiles (kb, rb) with kb in [kb_lo, kb_hi), rb <= kb: enumerate t in [kb_lo(kb_lo+1)/2, kb_hi(kb_hi+1)/2)
+  uint64_t t0 = (uint64_t)kb_lo * (kb_lo + 1) / 2, t1 = (uint64_t)kb_hi * (kb_hi + 1) / 2;
+  // launch with blockIdx offset by t0 via a shifted grid: simplest is to launch t1 tiles and skip kb < kb_lo
+
+  if (t1 > t0) k_pair_filter<<<(unsigned)(t1 - t0), 256, 0, s>>>(a, t0);
+  unsigned grid = (unsigned)num_sms * 8;
+  k_pair_exact<<<grid, 256, 0, s>>>(a, pairs, pair_cap, n_pairs);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_match_resolve(uint32_t K, const uint64_t* kto, const uint64_t* sig, const uint64_t* mass,
+                                 const uint64_t* wt, photon_match_params p, const uint64_t* pairs, uint64_t n_pairs,
+                                 const uint64_t* n_pairs_dev, const MatchWs& mw, int64_t* match, double* match_dist,
+                                 DevErr* err, cudaStream_t s) {
+  if (K == 0) return cudaSuccess;
+  cudaMemsetAsync(mw.cand_cnt, 0, sizeof(uint32_t) * K, s);
+  if (n_pairs) {
+    k_cand_count<<<(unsigned)ceil_div(n_pairs, 256), 256, 0, s>>>(pairs, n_pairs, n_pairs_dev, K, mw.cand_cnt, err);
+  }
+  k_cand_scan<<<1, 1024, 0, s>>>(mw.cand_cnt, K, mw.cand_off, mw.cand_cur);
+  if (n_pairs) {
+    k_cand_scatter<<<(unsigned)ceil_div(n_pairs, 256), 256, 0, s>>>(pairs, n_pairs, n_pairs_dev, K, mw.cand_off,
+                                                                    mw.cand_cur, mw.cand);
+  }
+  k_resolve_states<<<1, 1024, 0, s>>>(K, mw.cand_off, mw.cand, mw.state, p.pool_all_prior);
+  k_resolve_match<<<(unsigned)ceil_div((uint64_t)K * 32, 256), 256, 0, s>>>(K, mw.cand_off, mw.cand, mw.state,
+                                                                           p.pool_all_prior, wt, kto, sig, mass,
+                                                                           match, match_dist);
+  return cudaGetLastError();
+}
+
+}  // namespace photon

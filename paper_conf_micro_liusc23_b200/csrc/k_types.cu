@@ -1,0 +1,316 @@
+// k_types.cu — A2 canonicalisation (K2b, K2c) and the multi-GPU type-row export / merge / remap.
+//
+// weight_t = portion of the kernel's warps in type t; "the weighted BBVs are ordered according to a
+// descending order based on the weights" -> canonical order (count desc, key asc) [P-4].  L249: warp-sampling is
+// possible when the dominant type holds more than 95% of the warps [P-15].
+//
+// The hash table filled by K1/K2a (or by the row merge) is turned into CSR tables by: count types per kernel ->
+// exclusive scan -> scatter slot ids per kernel -> per-kernel sort (shared-memory bitonic for T_k <= 4096,
+// global-memory bitonic by one CTA beyond) -> emit rows and the slot -> canonical id map.  Insertion order into
+// the hash table is nondeterministic; the sort key is total (keys are unique per kernel), so the result is not.
+#include "internal.h"
+
+namespace photon {
+
+namespace {
+
+constexpr int SORT_SMEM_MAX = 4096;
+
+__global__ void k_ht_clear(HashTable ht) {
+  uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (i > ht.mask) return;
+  ht.hkey[i] = 0ull;
+  ht.ready[i] = 0u;
+  ht.count[i] = 0u;
+  ht.first[i] = ~0ull;
+}
+
+__global__ void k_count_types(HashTable ht, uint32_t K, uint32_t* tcount, DevErr* err) {
+  uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (i > ht.mask || ht.hkey[i] == 0ull) return;
+  uint32_t k = ht.kern[i];
+  if (k >= K) { latch(err, PHOTON_ERANGE, (int64_t)k); return; }
+  atomicAdd(&tcount[k], 1u);
+}
+
+// single CTA exclusive scan of tcount[K] -> kto[K+1]; also zeroes cursor and checks capacity
+__global__ void __launch_bounds__(1024) k_scan_types(const uint32_t* tcount, uint32_t K, uint64_t* kto,
+                                                      uint32_t* cursor, uint64_t capacity, DevErr* err) {
+  __shared__ uint64_t warp_sums[32];
+  __shared__ uint64_t carry;
+  if (threadIdx.x == 0) carry = 0;
+  __syncthreads();
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+  for (uint32_t base = 0; base < K; base += 1024) {
+    uint32_t k = base + threadIdx.x;
+    uint64_t v = k < K ? tcount[k] : 0;
+    if (k < K) cursor[k] = 0;
+    uint64_t x = v;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      uint64_t y = __shfl_up_sync(0xffffffffu, x, o);
+      if (lane >= o) x += y;
+    }
+    if (lane == 31) warp_sums[wid] = x;
+    __syncthreads();
+    if (wid == 0) {
+      uint64_t s = warp_sums[lane];
+#pragma unroll
+      for (int o = 1; o < 32; o <<= 1) {
+        uint64_t y = __shfl_up_sync(0xffffffffu, s, o);
+        if (lane >= o) s += y;
+      }
+      warp_sums[lane] = s;
+    }
+    __syncthreads();
+    uint64_t excl = carry + (wid ? warp_sums[wid - 1] : 0) + x - v;
+    if (k < K) kto[k] = excl;
+    __syncthreads();
+    if (threadIdx.x == 1023) carry = excl + v;
+    __syncthreads();
+  }
+  if (threadIdx.x == 0) {
+    kto[K] = carry;
+    if (carry > capacity) latch(err, PHOTON_ECAPACITY, (int64_t)carry);
+  }
+}
+
+__global__ void k_scatter_types(HashTable ht, uint32_t K, const uint64_t* kto, uint32_t* cursor, uint32_t* list,
+                                uint64_t capacity) {
+  uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (i > ht.mask || ht.hkey[i] == 0ull) return;
+  uint32_t k = ht.kern[i];
+  if (k >= K) return;
+  uint64_t pos = kto[k] + atomicAdd(&cursor[k], 1u);
+  if (pos < capacity) list[pos] = (uint32_t)i;
+}
+
+// canonical order: count descending, then key lexicographically ascending [P-4]; UINT32_MAX = padding (last)
+__device__ __forceinline__ bool type_before(const HashTable& ht, uint32_t a, uint32_t b) {
+  if (b == UINT32_MAX) return a != UINT32_MAX;
+  if (a == UINT32_MAX) return false;
+  uint32_t ca = ht.count[a], cb = ht.count[b];
+  if (ca != cb) return ca > cb;
+  const uint32_t* ka = ht.key + (uint64_t)a * 16;
+  const uint32_t* kb = ht.key + (uint64_t)b * 16;
+#pragma unroll 1
+  for (int j = 0; j < 16; ++j)
+    if (ka[j] != kb[j]) return ka[j] < kb[j];
+  return false;
+}
+
+__device__ void emit_rows(const HashTable& ht, uint32_t k, const uint32_t* sorted, uint64_t n, uint64_t off,
+                          const photon_types& out, uint32_t* canon, uint64_t Wk) {
+  for (uint64_t r = threadIdx.x; r < n && off + r < out.capacity; r += blockDim.x) {
+    uint32_t s = sorted[r];
+    const uint4* src = (const uint4*)(ht.key + (uint64_t)s * 16);
+    uint4* dst = (uint4*)(out.type_key + (off + r) * 16);
+    dst[0] = src[0]; dst[1] = src[1]; dst[2] = src[2]; dst[3] = src[3];
+    out.type_count[off + r] = ht.count[s];
+    out.type_first_warp[off + r] = ht.first[s];
+    canon[s] = (uint32_t)r;
+  }
+  if (threadIdx.x == 0) {
+    uint64_t c0 = n ? ht.count[sorted[0]] : 0;
+    out.warp_sampling_ok[k] = (Wk > 0 && 100ull * c0 > 95ull * Wk) ? 1 : 0;  // L249, strict [P-15]
+  }
+}
+
+// one CTA per kernel with T_k <= SORT_SMEM_MAX (larger kernels are skipped here and sorted by k_sort_large)
+__global__ void __launch_bounds__(512) k_sort_small(HashTable ht, uint32_t K, const uint64_t* kto,
+                                                    const uint32_t* list, const uint64_t* kwo,
+                                                    const uint64_t* kernel_warps, photon_types out, uint32_t* canon) {
+  __shared__ uint32_t sh[SORT_SMEM_MAX];
+  for (uint32_t k = blockIdx.x; k < K; k += gridDim.x) {
+    uint64_t off = kto[k], n = kto[k + 1] - off;
+    uint64_t Wk = kernel_warps ? kernel_warps[k] : (kwo[k + 1] - kwo[k]);
+    if (n > SORT_SMEM_MAX) continue;
+    uint32_t P = 1;
+    while (P < n) P <<= 1;
+    for (uint32_t i = threadIdx.x; i < P; i += blockDim.x) sh[i] = i < n ? list[off + i] : UINT32_MAX;
+    __syncthreads();
+    for (uint32_t size = 2; size <= P; size <<= 1) {
+      for (uint32_t stride = size >> 1; stride > 0; stride >>= 1) {
+        for (uint32_t t = threadIdx.x; t < P / 2; t += blockDim.x) {
+          uint32_t i = 2 * stride * (t / stride) + (t % stride);
+          uint32_t j = i + stride;
+          bool up = ((i & size) == 0);
+          uint32_t a = sh[i], b = sh[j];
+          bool sw = up ? type_before(ht, b, a) : type_before(ht, a, b);
+          if (sw) { sh[i] = b; sh[j] = a; }
+        }
+        __syncthreads();
+      }
+    }
+    emit_rows(ht, k, sh, n, off, out, canon, Wk);
+    __syncthreads();
+  }
+}
+
+// kernels with T_k > SORT_SMEM_MAX: one CTA, global-memory bitonic sort in scratch (rare: irregular kernels)
+__global__ void __launch_bounds__(1024) k_sort_large(HashTable ht, uint32_t K, const uint64_t* kto,
+                                                     const uint32_t* list, const uint64_t* kwo,
+                                                     const uint64_t* kernel_warps, photon_types out, uint32_t* canon,
+                                                     uint32_t* scratch) {
+  for (uint32_t k = 0; k < K; ++k) {
+    uint64_t off = kto[k], n = kto[k + 1] - off;
+    if (n <= SORT_SMEM_MAX) continue;
+    uint64_t Wk = kernel_warps ? kernel_warps[k] : (kwo[k + 1] - kwo[k]);
+    uint64_t P = 1;
+    while (P < n) P <<= 1;
+    for (uint64_t i = threadIdx.x; i < P; i += blockDim.x) scratch[i] = i < n ? list[off + i] : UINT32_MAX;
+    __syncthreads();
+    for (uint64_t size = 2; size <= P; size <<= 1) {
+      for (uint64_t stride = size >> 1; stride > 0; stride >>= 1) {
+        for (uint64_t t = threadIdx.x; t < P / 2; t += blockDim.x) {
+          uint64_t i = 2 * stride * (t / stride) + (t % stride);
+          uint64_t j = i + stride;
+          bool up = ((i & size) == 0);
+          uint32_t a = scratch[i], b = scratch[j];
+          bool sw = up ? type_before(ht, b, a) : type_before(ht, a, b);
+          if (sw) { scratch[i] = b; scratch[j] = a; }
+        }
+        __syncthreads();
+      }
+    }
+    emit_rows(ht, k, scratch, n, off, out, canon, Wk);
+    __syncthreads();
+  }
+}
+
+__global__ void k_remap(const uint32_t* slot, const uint32_t* canon, uint64_t W, uint32_t* out) {
+  uint64_t w = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (w >= W) return;
+  uint32_t s = slot[w];
+  out[w] = s == UINT32_MAX ? UINT32_MAX : canon[s];
+}
+
+__device__ __forceinline__ uint32_t row_kernel(const uint64_t* kto, uint32_t K, uint64_t row) {
+  uint32_t lo = 0, hi = K - 1;
+  while (lo < hi) {
+    uint32_t mid = (lo + hi + 1) >> 1;
+    if (kto[mid] <= row) lo = mid; else hi = mid - 1;
+  }
+  return lo;
+}
+
+__global__ void k_export(uint32_t K, photon_types local, uint32_t kernel_base, uint64_t warp_base,
+                         photon_type_row* rows) {
+  uint64_t T = local.kernel_type_off[K];
+  uint64_t r = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (r >= T) return;
+  photon_type_row x;
+  x.kernel = kernel_base + row_kernel(local.kernel_type_off, K, r);
+  x.pad = 0;
+  for (int j = 0; j < 16; ++j) x.key[j] = local.type_key[r * 16 + j];
+  x.count = local.type_count[r];
+  x.first_warp = local.type_first_warp[r] + warp_base;
+  rows[r] = x;
+}
+
+__global__ void k_rows_insert(const photon_type_row* rows, uint64_t n, uint32_t K, HashTable ht, DevErr* err) {
+  uint64_t r = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (r >= n) return;
+  const photon_type_row x = rows[r];
+  if (x.kernel >= K || x.count >= (1ull << 32)) { latch(err, PHOTON_ERANGE, (int64_t)r); return; }
+  uint64_t h = hash_key(x.kernel, x.key);
+  ht_insert(ht, err, x.kernel, x.key, h, (uint32_t)x.count, x.first_warp);
+}
+
+__device__ uint32_t ht_find(const HashTable& ht, uint32_t k, const uint32_t* p, uint64_t h) {
+  uint64_t i = h & ht.mask;
+  for (uint64_t probe = 0; probe <= ht.mask; ++probe) {
+    uint64_t cur = ht.hkey[i];
+    if (cur == 0ull) return UINT32_MAX;
+    if (cur == h && ht.kern[i] == k) {
+      bool same = true;
+      for (int j = 0; j < 16; ++j) same = same && (ht.key[i * 16 + j] == p[j]);
+      if (same) return (uint32_t)i;
+    }
+    i = (i + 1) & ht.mask;
+  }
+  return UINT32_MAX;
+}
+
+__global__ void k_remap_direct(const uint64_t* kwo, uint32_t K, uint64_t W, photon_types local,
+                               uint32_t kernel_base, HashTable ht, const uint32_t* canon, uint32_t* out, DevErr* err) {
+  uint64_t v = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (v >= W) return;
+  uint32_t lo = 0, hi = K - 1;
+  while (lo < hi) {
+    uint32_t mid = (lo + hi + 1) >> 1;
+    if (kwo[mid] <= v) lo = mid; else hi = mid - 1;
+  }
+  uint32_t t = local.warp_type[v];
+  uint64_t row = local.kernel_type_off[lo] + t;
+  uint32_t kg = kernel_base + lo;
+  uint32_t key[16];
+  const uint4* src = (const uint4*)(local.type_key + row * 16);
+#pragma unroll
+  for (int q = 0; q < 4; ++q) {
+    uint4 x = src[q];
+    key[4 * q] = x.x; key[4 * q + 1] = x.y; key[4 * q + 2] = x.z; key[4 * q + 3] = x.w;
+  }
+  uint32_t s = ht_find(ht, kg, key, hash_key(kg, key));
+  if (s == UINT32_MAX) { latch(err, PHOTON_ERANGE, (int64_t)v); out[v] = UINT32_MAX; return; }
+  out[v] = canon[s];
+}
+
+}  // namespace
+
+cudaError_t launch_ht_clear(const HashTable& ht, cudaStream_t s) {
+  uint64_t cap = ht.mask + 1;
+  k_ht_clear<<<(unsigned)ceil_div(cap, 256), 256, 0, s>>>(ht);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_canonicalise(const HashTable& ht, uint32_t K, const uint64_t* kwo, const uint64_t* kernel_warps,
+                                const photon_types& out, const CanonWs& cw, DevErr* err, int num_sms,
+                                cudaStream_t s) {
+  uint64_t cap = ht.mask + 1;
+  cudaMemsetAsync(cw.tcount, 0, sizeof(uint32_t) * (K ? K : 1), s);
+  k_count_types<<<(unsigned)ceil_div(cap, 256), 256, 0, s>>>(ht, K, cw.tcount, err);
+  k_scan_types<<<1, 1024, 0, s>>>(cw.tcount, K, out.kernel_type_off, cw.cursor, out.capacity, err);
+  k_scatter_types<<<(unsigned)ceil_div(cap, 256), 256, 0, s>>>(ht, K, out.kernel_type_off, cw.cursor, cw.list,
+                                                               out.capacity);
+  unsigned grid = (unsigned)(K < (uint32_t)num_sms * 8 ? K : (uint32_t)num_sms * 8);
+  if (grid == 0) grid = 1;
+  k_sort_small<<<grid, 512, 0, s>>>(ht, K, out.kernel_type_off, cw.list, kwo, kernel_warps, out, cw.canon);
+  k_sort_large<<<1, 1024, 0, s>>>(ht, K, out.kernel_type_off, cw.list, kwo, kernel_warps, out, cw.canon,
+                                  (uint32_t*)cw.scratch);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_remap(const uint32_t* warp_slot, const uint32_t* canon, uint64_t W, uint32_t* warp_type,
+                         DevErr* err, cudaStream_t s) {
+  (void)err;
+  if (W == 0) return cudaSuccess;
+  k_remap<<<(unsigned)ceil_div(W, 256), 256, 0, s>>>(warp_slot, canon, W, warp_type);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_types_export(uint32_t K, const photon_types& local, uint32_t kernel_base, uint64_t warp_base,
+                                photon_type_row* rows, cudaStream_t s) {
+  // T is on the device; launch for the capacity bound and guard inside
+  uint64_t cap = local.capacity ? local.capacity : 1;
+  k_export<<<(unsigned)ceil_div(cap, 256), 256, 0, s>>>(K, local, kernel_base, warp_base, rows);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_rows_insert(const photon_type_row* rows, uint64_t n, uint32_t K, const HashTable& ht,
+                               DevErr* err, cudaStream_t s) {
+  if (n == 0) return cudaSuccess;
+  k_rows_insert<<<(unsigned)ceil_div(n, 256), 256, 0, s>>>(rows, n, K, ht, err);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_remap_direct(const uint64_t* kwo_local, uint32_t K_local, uint64_t W_local,
+                                const photon_types& local, uint32_t kernel_base, const HashTable& ht,
+                                const uint32_t* canon, uint32_t* warp_type_global, DevErr* err, cudaStream_t s) {
+  if (W_local == 0) return cudaSuccess;
+  k_remap_direct<<<(unsigned)ceil_div(W_local, 256), 256, 0, s>>>(kwo_local, K_local, W_local, local, kernel_base, ht,
+                                                                   canon, warp_type_global, err);
+  return cudaGetLastError();
+}
+
+}  // namespace photon

@@ -1,0 +1,231 @@
+"""GPU parity: libphoton (through its C ABI) vs the CPU oracle, element by element on the same seeded inputs.
+
+Bar (BASELINE.json north_star): bit-exact BBVs, warp types, type tables, dominance, matches and stability /
+switch decisions; reported fp64 distances within 1e-6 relative.
+"""
+import numpy as np
+import pytest
+
+import oracle
+import tracegen as tg
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def ph():
+    from paper_conf_micro_liusc23_b200 import Photon
+    return Photon(0)
+
+
+def _dev(ph, tr):
+    from paper_conf_micro_liusc23_b200 import DeviceTrace
+    return DeviceTrace.from_host(tr, ph.device)
+
+
+def _np(t, dt):
+    from paper_conf_micro_liusc23_b200 import to_numpy
+    return to_numpy(t, dt)
+
+
+def check_bbv(ph, tr, kbb=True):
+    d = _dev(ph, tr)
+    o = ph.photon_bbv_build(d, bbv16=True, insts=True, kbb=kbb)
+    p16, ins, kb = oracle.bbv(tr, want_kbb=kbb)
+    assert np.array_equal(_np(o["warp_bbv16"], np.uint32).reshape(-1, 16), p16)
+    assert np.array_equal(_np(o["warp_insts"], np.uint64), ins)
+    if kbb:
+        assert np.array_equal(_np(o["kernel_bb_insts"], np.uint64).reshape(tr.n_kernels, tr.n_bb), kb)
+    return d, o, p16
+
+
+def check_types(ph, tr, ty, ref):
+    T = int(ref["kernel_type_off"][-1])
+    assert np.array_equal(_np(ty["kernel_type_off"], np.uint64), ref["kernel_type_off"])
+    assert np.array_equal(_np(ty["warp_type"], np.uint32), ref["warp_type"])
+    assert np.array_equal(_np(ty["type_key"], np.uint32).reshape(-1, 16)[:T], ref["type_key"])
+    assert np.array_equal(_np(ty["type_count"], np.uint64)[:T], ref["type_count"])
+    assert np.array_equal(_np(ty["type_first_warp"], np.uint64)[:T], ref["type_first_warp"])
+    assert np.array_equal(_np(ty["warp_sampling_ok"], np.uint8), ref["warp_sampling_ok"])
+
+
+def check_match(ph, tr, ty, ref, theta=(1, 20), n_cores=64, pool=0):
+    d = _dev(ph, tr)
+    m = ph.photon_kernel_match(tr.n_kernels, ty, d.warps_total, theta, n_cores, pool, want_dist=True)
+    sig, mass = oracle.signature(ref["kernel_type_off"], ref["type_key"], ref["type_count"])
+    om, od = oracle.match(ref["kernel_type_off"], sig, mass, tr.warps_total, theta, n_cores, pool)
+    gm = _np(m["match"], np.int64)
+    gd = _np(m["match_dist"], np.float64)
+    assert np.array_equal(gm, om)
+    fin = np.isfinite(od)
+    assert np.array_equal(np.isfinite(gd), fin)
+    np.testing.assert_allclose(gd[fin], od[fin], rtol=1e-6, atol=0)
+
+
+def full_chain(ph, tr, thetas=((1, 20),), pools=(0,), n_cores=64):
+    d, o, p16 = check_bbv(ph, tr)
+    ref = oracle.group(tr, p16)
+    ty = ph.photon_warp_group(d)  # fused single pass
+    check_types(ph, tr, ty, ref)
+    ty2 = ph.photon_warp_group(d, warp_bbv16=o["warp_bbv16"])  # unfused
+    check_types(ph, tr, ty2, ref)
+    for th in thetas:
+        for pool in pools:
+            check_match(ph, tr, ty, ref, th, n_cores, pool)
+    return ty, ref
+
+
+def test_worked_example(ph):
+    import json, os
+    g = json.load(open(os.path.join(os.path.dirname(__file__), "golden", "worked_example.json")))
+    tr = tg.trace_from_warps(g["kernels"], g["bb_len"])
+    full_chain(ph, tr, thetas=((1, 20), (1, 2), (4, 11), (2, 5)), n_cores=2)
+
+
+@pytest.mark.parametrize("seed", range(10))
+def test_random_small(ph, seed):
+    custom = seed % 2 == 1
+    n_bb = [7, 16, 40, 300, 5000, 9000, 65536, 33, 17, 4096][seed]
+    tr = tg.random_trace(seed, n_kernels=1 + seed % 7, max_warps=600, max_events=90, n_bb=n_bb, custom_bins=custom)
+    full_chain(ph, tr, thetas=((1, 20), (1, 5), (1, 2)), pools=(0, 1))
+
+
+def test_empty_warps_kernels_and_ragged(ph):
+    kernels = [[[], [], [0, 1]], [], [[2] * 1000 + [1] * 3], [[]], [[0, 1, 2, 3, 4, 5, 6]] * 300 + [[1]]]
+    tr = tg.trace_from_warps(kernels, bb_len=[3, 1, 7, 2, 9, 4, 5], warps_total=[3, 64, 1, 1, 301])
+    full_chain(ph, tr, thetas=((1, 20), (2, 1)), pools=(0, 1))
+
+
+@pytest.mark.parametrize("cfg", [1, 6])
+def test_config_small(ph, cfg):
+    tr = tg.make_trace(cfg)
+    full_chain(ph, tr, thetas=((1, 100), (1, 20), (1, 10), (1, 5)), pools=(0, 1))
+
+
+def test_config_c6_sample_1pct(ph):
+    # the paper's 1% sample (L208/L258): every 100th warp, warps_total = launched warps
+    g = tg.Generator(6)
+    tr = g.trace(0, g.n_warps, step=100)
+    full_chain(ph, tr, thetas=((1, 20),), pools=(0, 1))
+
+
+@pytest.mark.parametrize("cfg", [2, 3, 4])
+def test_config_full(ph, cfg):
+    tr = tg.make_trace(cfg)
+    full_chain(ph, tr, thetas=((1, 100), (1, 20), (1, 10), (1, 5)), pools=(0, 1))
+
+
+@pytest.mark.slow
+def test_config_c5_full(ph):
+    """C5 at full size (10^9 events): the oracle runs the whole chain too (~30 s)."""
+    tr = tg.make_trace(5)
+    d = _dev(ph, tr)
+    ty = ph.photon_warp_group(d)
+    ref = oracle.analyse(tr)
+    check_types(ph, tr, ty, ref)
+    m = ph.photon_kernel_match(tr.n_kernels, ty, d.warps_total, (1, 20), 64, 0)
+    assert np.array_equal(_np(m["match"], np.int64), ref["match"])
+
+
+# ---- error paths ------------------------------------------------------------------------------------------------
+def test_errors(ph):
+    from paper_conf_micro_liusc23_b200 import PhotonError
+    tr = tg.trace_from_warps([[[0, 1, 2, 1], [1, 5, 0]]], bb_len=[1, 2, 3])  # bb 5 >= B at event 5
+    with pytest.raises(PhotonError) as ei:
+        ph.photon_bbv_build(_dev(ph, tr))
+    assert ei.value.code == -3 and ei.value.index == 5
+    with pytest.raises(PhotonError) as ei:
+        ph.photon_warp_group(_dev(ph, tr))
+    assert ei.value.code == -3
+    tr = tg.trace_from_warps([[[0] * 3]], bb_len=[(1 << 17) + 5])
+    tr.bb = np.array([0] * 40000, np.uint16)  # 40000 * (2^17+5) >= 2^32: per-warp instructions overflow
+    tr.warp_event_off = np.array([0, 40000], np.uint64)
+    with pytest.raises(PhotonError) as ei:
+        ph.photon_bbv_build(_dev(ph, tr))
+    assert ei.value.code == -3 and ei.value.index == 0
+    tr = tg.trace_from_warps([[[0], [1]]], bb_len=[1, 2])
+    tr.warp_event_off = np.array([0, 2, 2], np.uint64)  # [W] != E... E = 2 here; make it non-monotone instead
+    tr.warp_event_off = np.array([0, 3, 2], np.uint64)
+    with pytest.raises(PhotonError) as ei:
+        ph.photon_bbv_build(_dev(ph, tr))
+    assert ei.value.code == -3
+    tr = tg.trace_from_warps([[[0]]], bb_len=[0])  # length 0 is invalid
+    with pytest.raises(PhotonError) as ei:
+        ph.photon_bbv_build(_dev(ph, tr))
+    assert ei.value.code == -1
+
+
+def test_capacity_retry(ph):
+    # every warp its own type: a hint of 1 forces ECAPACITY, the binding retries with a larger table
+    rs = np.random.default_rng(3)
+    kernels = [[list(rs.integers(0, 16, 20)) for _ in range(5000)]]
+    tr = tg.trace_from_warps(kernels, bb_len=list(range(1, 17)))
+    d = _dev(ph, tr)
+    ty = ph.photon_warp_group(d, capacity_hint=1)
+    p16, _, _ = oracle.bbv(tr, want_kbb=False)
+    check_types(ph, tr, ty, oracle.group(tr, p16))
+
+
+# ---- A5 ------------------------------------------------------------------------------------------------------
+def check_stable(ph, tm, kbb, n, delta=(3, 100), rate=(95, 100)):
+    from paper_conf_micro_liusc23_b200 import DeviceTiming, to_device
+    dt = DeviceTiming.from_host(tm, ph.device)
+    kb = to_device(np.ascontiguousarray(kbb, np.uint64), ph.device)
+    o = ph.photon_bb_stable(dt, kb, n, delta, rate)
+    fs, ds, sw = oracle.stable(tm, kbb, n, delta, rate)
+    K, B = tm.n_kernels, int(tm.n_bb)
+    assert np.array_equal(_np(o["first_stable"], np.int64).reshape(K, B), fs)
+    assert np.array_equal(_np(o["stable_dur_sum"], np.uint64).reshape(K, B), ds)
+    assert np.array_equal(_np(o["switch_at"], np.int64), sw)
+    return fs
+
+
+@pytest.mark.parametrize("n", [8, 32, 64])
+def test_stable_c6(ph, n):
+    g = tg.Generator(6)
+    tm = g.timing()
+    _, _, kbb = oracle.bbv(g.trace())
+    fs = check_stable(ph, tm, kbb, n)
+    assert (fs >= 0).any()
+
+
+def test_stable_c1(ph):
+    g = tg.Generator(1)
+    tm = g.timing()
+    _, _, kbb = oracle.bbv(g.trace())
+    check_stable(ph, tm, kbb, 2048)
+    check_stable(ph, tm, kbb, 512, delta=(1, 100))
+
+
+@pytest.mark.parametrize("cfg", [3, 4])
+def test_stable_configs(ph, cfg):
+    g = tg.Generator(cfg)
+    tm = g.timing()
+    _, _, kbb = oracle.bbv(g.trace())
+    check_stable(ph, tm, kbb, 2048)
+
+
+def test_stable_paper_lines(ph):
+    # L227 lines (stable) and L145 (not), one kernel per line, n = 64
+    from fractions import Fraction
+    n = 64
+    recs = []
+    for a in ["1.00", "0.99", "32.87", "0.97", "0.9701", "1.03", "1.0299"]:
+        xs = [10_000 * (i + 1) for i in range(3 * n)]
+        ys = [int(Fraction(a) * x + 10 ** 9) for x in xs]
+        recs.append((xs, ys))
+    off = np.cumsum([0] + [len(x) for x, _ in recs]).astype(np.uint64)
+    tm = tg.Timing(kernel_rec_off=off, bb=np.zeros(int(off[-1]), np.uint16),
+                   issue=np.concatenate([np.array(x, np.uint64) for x, _ in recs]),
+                   retire=np.concatenate([np.array(y, np.uint64) for _, y in recs]), n_bb=1)
+    fs = check_stable(ph, tm, np.ones((len(recs), 1), np.uint64), n)
+    assert fs[:, 0].tolist() == [2 * n - 1, 2 * n - 1, -1, -1, 2 * n - 1, -1, 2 * n - 1]
+
+
+def test_stable_errors(ph):
+    from paper_conf_micro_liusc23_b200 import PhotonError
+    tm = tg.Timing(kernel_rec_off=np.array([0, 3], np.uint64), bb=np.zeros(3, np.uint16),
+                   issue=np.array([1, 2, 3], np.uint64), retire=np.array([5, 4, 9], np.uint64), n_bb=1)
+    with pytest.raises(PhotonError) as ei:
+        check_stable(ph, tm, np.ones((1, 1), np.uint64), 2)
+    assert ei.value.code == -3 and ei.value.index == 1
