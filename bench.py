@@ -1,0 +1,357 @@
+#!/usr/bin/env python
+"""bench.py — BB-trace events analysed per second (BBV + grouping + match) on 1..8 B200s, with the HBM roofline.
+
+Contract (driver): `python bench.py --gpus N --steps K --warmup W` (torchrun for N > 1, one rank per GPU) prints ONE
+JSON line on rank 0.  A step = one pass of the metric's chain A1 -> A4 (per-warp BBV + warp-type grouping fused in
+one streaming pass, canonical type tables, GPU-BBV signatures, kernel matching) over the whole workload, with the
+trace resident in HBM.  A5 (the BB stability test) is timed in the same run on its own timing stream and reported
+under "a5".  `--impl reference` times the CPU oracle (the only other place this file runs oracle/).
+
+Workload (default): C5 stress — 10^4 kernels, ~10^9 BB events, 4096 BB ids (BASELINE.json configs[4]); it is the
+largest config and fits one GPU (2.0 GB trace).  Inputs (2.0 GB) exceed the 126 MB L2, so no flush is needed.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "BB-trace events analysed/sec (BBV+grouping+match) at 1/2/4/8 B200; % HBM BW"
+CONFIG_DESC = {1: "C1 tiny", 2: "C2 micro mix (10 VADD + 10 GEMM, 64K warps each)", 3: "C3 VGG-16 batch 1",
+               4: "C4 ResNet-152 batch 1", 5: "C5 stress (10^4 kernels, 10^9 events, 4096 BB ids)"}
+
+
+def parse():
+    p = argparse.ArgumentParser()
+    p.add_argument("--gpus", type=int, default=1)
+    p.add_argument("--steps", type=int, default=20)
+    p.add_argument("--warmup", type=int, default=5)
+    p.add_argument("--impl", default="photon", choices=["photon", "reference"])
+    p.add_argument("--config", type=int, default=5)
+    p.add_argument("--seed", type=int, default=None)
+    p.add_argument("--theta", default="1/20")
+    p.add_argument("--e2e-steps", type=int, default=3)
+    p.add_argument("--a5-config", type=int, default=3)
+    p.add_argument("--skip-e2e", action="store_true")
+    p.add_argument("--skip-a5", action="store_true")
+    p.add_argument("--skip-cpu", action="store_true")
+    p.add_argument("--cpu-kernels", type=int, default=3000, help="C5 kernel prefix timed for cpu_baseline")
+    return p.parse_args()
+
+
+def _peaks():
+    try:
+        with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
+            j = json.load(f)
+        return float(j["hbm_gbs"]), "measured (MEASURED_PEAKS.json)"
+    except Exception:
+        return 6650.0, "fallback (B200_PROFILING.md)"
+
+
+def _traffic(cfg):
+    """Per-launch DRAM bytes of the fused K1 from the committed ncu --set full capture (profiles/), else None."""
+    try:
+        with open(os.path.join(ROOT, "profiles", "k1_traffic.json")) as f:
+            j = json.load(f)
+        return j.get(str(cfg))
+    except Exception:
+        return None
+
+
+class Clocks:
+    """nvidia-smi sampler running during the timed region."""
+    Q = ("clocks.sm,clocks.max.sm,clocks_event_reasons.active,clocks_event_reasons.hw_slowdown,"
+         "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+         "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index):
+        self.index = index
+        self.p = None
+
+    def start(self):
+        try:
+            self.p = subprocess.Popen(["nvidia-smi", f"--query-gpu={self.Q}", "--format=csv,noheader,nounits",
+                                       "-lms", "100", "-i", str(self.index)], stdout=subprocess.PIPE,
+                                      stderr=subprocess.DEVNULL, text=True)
+        except Exception:
+            self.p = None
+
+    def stop(self):
+        if self.p is None:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        self.p.terminate()
+        try:
+            out, _ = self.p.communicate(timeout=5)
+        except Exception:
+            self.p.kill()
+            out = ""
+        sms, mx, reasons = [], None, set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for line in out.strip().splitlines():
+            f = [x.strip() for x in line.split(",")]
+            if len(f) < 7:
+                continue
+            try:
+                sms.append(float(f[0]))
+                mx = float(f[1])
+            except ValueError:
+                continue
+            for n, v in zip(names, f[3:7]):
+                if v.lower().startswith("active"):
+                    reasons.add(n)
+        return {"sm_mhz": statistics.median(sms) if sms else None, "sm_max_mhz": mx, "reasons": sorted(reasons),
+                "samples": len(sms)}
+
+
+def dist_env():
+    ws = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    return ws, rank, local
+
+
+def run_reference(args):
+    """The oracle as it stands (plain single-threaded C++), on bounded samples of the same workload."""
+    ws, rank, _ = dist_env()
+    if rank != 0:
+        return
+    import numpy as np
+    import oracle
+    import tracegen as tg
+    g = tg.Generator(args.config, args.seed)
+    k1 = min(g.n_kernels, args.cpu_kernels) if args.config == 5 else g.n_kernels
+    tr = g.kernels_trace(0, k1)
+    num, den = (int(x) for x in args.theta.split("/"))
+    times = []
+    for i in range(args.warmup + args.steps):
+        t0 = time.perf_counter()
+        oracle.analyse(tr, theta=(num, den))
+        dt = time.perf_counter() - t0
+        if i >= args.warmup:
+            times.append(dt)
+    ms = 1000 * statistics.mean(times)
+    value = tr.n_events / (ms / 1000)
+    sample = f"kernels [0,{k1}) of {CONFIG_DESC.get(args.config)}: {tr.n_events} events, {tr.n_warps} warps"
+    line = {"impl": "reference", "metric": METRIC, "value": value, "unit": "events/s", "n_gpus": args.gpus,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True,
+            "scaling": "weak", "vs_baseline": None, "dtype": "u16/u32/u64 integer (u128 exact compares)",
+            "data": "synthetic (tracegen, seeded)",
+            "config": {"workload": CONFIG_DESC.get(args.config), "sample": sample, "theta": args.theta},
+            "cpu_baseline": {"value": value, "unit": "events/s", "cores": 1, "kind": "oracle", "sample": sample},
+            "e2e": {"value": value, "unit": "events/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+def cpu_baseline(args):
+    import oracle
+    import tracegen as tg
+    g = tg.Generator(args.config, args.seed)
+    k1 = min(g.n_kernels, args.cpu_kernels) if args.config == 5 else g.n_kernels
+    tr = g.kernels_trace(0, k1)
+    num, den = (int(x) for x in args.theta.split("/"))
+    t0 = time.perf_counter()
+    oracle.analyse(tr, theta=(num, den))
+    dt = time.perf_counter() - t0
+    return {"value": tr.n_events / dt, "unit": "events/s", "cores": 1, "kind": "oracle",
+            "sample": f"kernels [0,{k1}) of {CONFIG_DESC.get(args.config)}: {tr.n_events} events in {dt:.1f} s "
+                      f"(single-threaded C++ oracle, full chain A1-A4)"}
+
+
+def run_photon(args):
+    import numpy as np
+    import torch
+
+    import tracegen as tg
+    from paper_conf_micro_liusc23_b200 import DeviceTiming, DeviceTrace, Photon, load, to_device
+    from paper_conf_micro_liusc23_b200._lib import PROF_SECTIONS
+
+    ws, rank, local = dist_env()
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    if ws > 1:
+        import torch.distributed as dist
+        dist.init_process_group("nccl", device_id=dev)
+    num, den = (int(x) for x in args.theta.split("/"))
+    g = tg.Generator(args.config, args.seed)
+    if ws > 1:
+        cuts = tg.shard_bounds(g.warp_counts(), ws)
+        tr = g.trace(int(cuts[rank]), int(cuts[rank + 1]))
+    else:
+        tr = g.trace()
+    ph = Photon(local)
+    L = load()
+    d = DeviceTrace.from_host(tr, dev)
+    E_total = int(g.warp_counts().sum()) if ws > 1 else tr.n_events
+    W_total = g.n_warps
+
+    if ws > 1:
+        from paper_conf_micro_liusc23_b200 import dist as pdist
+        runner = pdist.ShardedAnalysis(ph, g.n_kernels, g.kernel_warps, tr, d, theta=(num, den))
+        step = lambda check=False: runner.run(check=check)
+    else:
+        step = lambda check=False: ph.analyse(d, theta=(num, den), check=check)
+
+    # warm-up (the first step checks errors and sizes the tables)
+    res = step(check=True)
+    for _ in range(max(args.warmup - 1, 0)):
+        res = step(check=False)
+    torch.cuda.synchronize()
+    if ws > 1:
+        torch.distributed.barrier()
+
+    clocks = Clocks(local)
+    clocks.start()
+    time.sleep(0.3)
+    L.photon_profile(ph.ctx, 1)
+    launches0 = L.photon_launch_count()
+    s = torch.cuda.current_stream(dev)
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    if ws > 1:
+        torch.distributed.barrier()
+    torch.cuda.synchronize()
+    e0.record(s)
+    for _ in range(args.steps):
+        res = step(check=False)
+    e1.record(s)
+    torch.cuda.synchronize()
+    if ws > 1:
+        torch.distributed.barrier()
+    launches = L.photon_launch_count() - launches0
+    ms = e0.elapsed_time(e1) / args.steps
+    import ctypes
+    pms = (ctypes.c_double * 16)()
+    pcnt = (ctypes.c_uint64 * 16)()
+    L.photon_profile_read(ph.ctx, ph.stream_ptr(), pms, pcnt)
+    L.photon_profile(ph.ctx, 0)
+    clk = clocks.stop()
+    # errors latched during the timed steps?
+    for k in ("_ws", "_mws"):
+        if k in res and res[k] is not None:
+            ph.check(res[k])
+    if ws > 1:
+        t = torch.tensor([ms], device=dev, dtype=torch.float64)
+        torch.distributed.all_reduce(t, op=torch.distributed.ReduceOp.MAX)
+        ms = float(t.item())
+
+    sections = {PROF_SECTIONS[i]: {"ms_per_step": pms[i] / args.steps, "launches": int(pcnt[i])}
+                for i in range(len(PROF_SECTIONS)) if pcnt[i]}
+    hbm_peak, peak_src = _peaks()
+    k1_ms = pms[0] / max(int(pcnt[0]), 1)
+    k1_bytes = 2 * tr.n_events + 8 * (tr.n_warps + 1) + 4 * tr.n_warps  # algorithmic: bb + offsets + warp type
+    achieved = k1_bytes / (k1_ms / 1000) / 1e9
+    roofline = {"bound": "hbm", "kernel": "k_bbv (fused A1+A2 streaming pass)", "achieved": achieved,
+                "peak": hbm_peak, "peak_source": peak_src, "unit": "GB/s", "frac": achieved / hbm_peak,
+                "traffic": _traffic(args.config), "algorithmic_bytes_per_launch": k1_bytes,
+                "k1_ms": k1_ms, "k1_share_of_step": (pms[0] / args.steps) / ms if ms else None,
+                "chain_algorithmic_GBps": (2 * E_total + 12 * W_total) / (ms / 1000) / 1e9}
+    value = E_total / (ms / 1000)
+
+    line = {"metric": METRIC, "value": value, "unit": "events/s", "n_gpus": ws, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True,
+            "scaling": "strong" if ws > 1 else "weak", "vs_baseline": None,
+            "dtype": "u16/u32/u64 integer (u128 exact compares)", "data": "synthetic (tracegen, seeded; no datasets)",
+            "config": {"workload": CONFIG_DESC.get(args.config), "events": E_total, "warps": W_total,
+                       "kernels": g.n_kernels, "bb_ids": g.n_bb, "theta": args.theta,
+                       "parallelism": f"dp{ws} (warp shards)" if ws > 1 else "1 GPU",
+                       "l2": f"inputs ({(2 * E_total + 8 * W_total) / 1e9:.2f} GB) exceed the 126 MB L2; no flush"},
+            "roofline": roofline, "sections": sections, "clocks": clk, "gpu_launches": int(launches)}
+
+    # ---- e2e: the same chain through the API with host (pinned) inputs; H2D + D2H inside the timed region ----
+    if not args.skip_e2e:
+        host = {k: to_device(getattr(tr, k), None).pin_memory() for k in
+                ("kernel_warp_off", "warp_event_off", "bb", "bb_len", "warps_total")}
+        h2d = sum(t.numel() * t.element_size() for t in host.values())
+        dd = DeviceTrace(*[torch.empty_like(host[k], device=dev) for k in
+                           ("kernel_warp_off", "warp_event_off", "bb", "bb_len")], None,
+                         torch.empty_like(host["warps_total"], device=dev), tr.n_kernels, tr.n_bb, tr.n_warps,
+                         tr.n_events)
+        times = []
+        d2h = 0
+        for i in range(args.e2e_steps + 1):
+            torch.cuda.synchronize()
+            a0, a1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            a0.record(s)
+            for k, dst in zip(("kernel_warp_off", "warp_event_off", "bb", "bb_len", "warps_total"),
+                              (dd.kernel_warp_off, dd.warp_event_off, dd.bb, dd.bb_len, dd.warps_total)):
+                dst.copy_(host[k], non_blocking=True)
+            if ws > 1:
+                r = pdist.ShardedAnalysis(ph, g.n_kernels, g.kernel_warps, tr, dd, theta=(num, den)).run(check=False)
+            else:
+                r = ph.analyse(dd, theta=(num, den), check=False)
+            outs = [r["warp_type"], r["kernel_type_off"], r["warp_sampling_ok"], r["match"]]
+            hb = [o.to("cpu", non_blocking=True) for o in outs]
+            a1.record(s)
+            torch.cuda.synchronize()
+            d2h = sum(o.numel() * o.element_size() for o in outs)
+            if i > 0:
+                times.append(a0.elapsed_time(a1))
+        e2e_ms = statistics.mean(times)
+        if ws > 1:
+            t = torch.tensor([e2e_ms], device=dev, dtype=torch.float64)
+            torch.distributed.all_reduce(t, op=torch.distributed.ReduceOp.MAX)
+            e2e_ms = float(t.item())
+        line["e2e"] = {"value": E_total / (e2e_ms / 1000), "unit": "events/s", "h2d_bytes_per_step": int(h2d),
+                       "d2h_bytes_per_step": int(d2h), "ms_per_step": e2e_ms, "steps": args.e2e_steps}
+
+    # ---- A5 on its own timing stream (reported beside the metric) ----
+    if not args.skip_a5 and ws == 1:
+        ga = tg.Generator(args.a5_config)
+        tm = ga.timing()
+        ta = ga.trace()
+        da = DeviceTrace.from_host(ta, dev)
+        kbb = ph.photon_bbv_build(da, bbv16=False, insts=False, kbb=True)["kernel_bb_insts"]
+        dt = DeviceTiming.from_host(tm, dev)
+        o = ph.photon_bb_stable(dt, kbb, 2048)
+        for _ in range(max(args.warmup - 1, 0)):
+            o = ph.photon_bb_stable(dt, kbb, 2048, check=False, out=o)
+        torch.cuda.synchronize()
+        L.photon_profile(ph.ctx, 1)
+        b0, b1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        b0.record(s)
+        n5 = max(args.steps // 4, 3)
+        for _ in range(n5):
+            o = ph.photon_bb_stable(dt, kbb, 2048, check=False, out=o)
+        b1.record(s)
+        torch.cuda.synchronize()
+        ph.check(o["_ws"])
+        L.photon_profile(ph.ctx, 0)
+        ams = b0.elapsed_time(b1) / n5
+        R = tm.n_records
+        abytes = 18 * R
+        line["a5"] = {"metric": "BB timing records tested/sec (stability test + switch)", "value": R / (ams / 1000),
+                      "unit": "records/s", "ms_per_step": ams, "records": R,
+                      "workload": f"{CONFIG_DESC.get(args.a5_config)} timing stream (wave model), n=2048, delta=3/100",
+                      "roofline": {"bound": "hbm", "achieved": abytes / (ams / 1000) / 1e9, "peak": hbm_peak,
+                                   "unit": "GB/s", "frac": abytes / (ams / 1000) / 1e9 / hbm_peak,
+                                   "algorithmic_bytes": abytes, "traffic": None},
+                      "stable_bb_types": int((to_numpy_i64(o["first_stable"]) >= 0).sum())}
+
+    if rank == 0 and ws == 1 and not args.skip_cpu:
+        line["cpu_baseline"] = cpu_baseline(args)
+    if rank == 0:
+        print(json.dumps(line), flush=True)
+    if ws > 1:
+        torch.distributed.destroy_process_group()
+
+
+def to_numpy_i64(t):
+    return t.detach().cpu().numpy()
+
+
+def main():
+    args = parse()
+    if args.impl == "reference":
+        run_reference(args)
+    else:
+        run_photon(args)
+
+
+if __name__ == "__main__":
+    main()

@@ -60,6 +60,27 @@ PHOTON_API int photon_check(photon_ctx *ctx, void *stream, int64_t *bad_index);
 /* Same as photon_check for an explicit workspace (one of several calls in flight). SYNCHRONISES `stream`. */
 PHOTON_API int photon_ws_status(photon_ctx *ctx, const void *ws, void *stream, int64_t *bad_index);
 
+/* Diagnostics.  photon_profile(ctx, 1) resets and enables in-stream CUDA-event timing of each launch section
+ * below (events are recorded on the call's stream around the section's kernels); photon_profile_read SYNCHRONISES
+ * `stream` and writes, per section, the summed milliseconds and the number of timed sections.
+ * photon_launch_count() = libphoton kernel launches since the library was loaded (all contexts). */
+enum {
+  PHOTON_PROF_BBV_FUSED = 0,    /* fused A1+A2 streaming kernel (photon_warp_group, warp_bbv16 == NULL) */
+  PHOTON_PROF_BBV = 1,          /* A1 streaming kernel (photon_bbv_build)                               */
+  PHOTON_PROF_KBB = 2,          /* kernel_bb_insts                                                      */
+  PHOTON_PROF_GROUP_UNFUSED = 3,/* A2 insertion from materialised BBVs                                 */
+  PHOTON_PROF_CANON = 4,        /* canonical type tables + warp remap                                   */
+  PHOTON_PROF_SIG = 5,          /* A3 signatures                                                         */
+  PHOTON_PROF_SCAN = 6,         /* A4 pair filter + exact check                                          */
+  PHOTON_PROF_RESOLVE = 7,      /* A4 launch-order resolution                                            */
+  PHOTON_PROF_STABLE = 8,       /* A5 (all kernels)                                                      */
+  PHOTON_PROF_N = 9
+};
+PHOTON_API int photon_profile(photon_ctx *ctx, int enable);
+PHOTON_API int photon_profile_read(photon_ctx *ctx, void *stream, double *ms /*[PHOTON_PROF_N] HOST*/,
+                                   uint64_t *sections /*[PHOTON_PROF_N] HOST*/);
+PHOTON_API uint64_t photon_launch_count(void);
+
 /* ------------------------------------------------------------------------------------------------------------
  * Input 1: the functional basic-block trace of the analysed (sampled) warps, CSR by kernel then by warp.
  * Paper: the online analysis functionally simulates a sample of warps (1%, L208/L258) and records, per warp, the

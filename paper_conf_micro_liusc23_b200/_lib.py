@@ -55,6 +55,7 @@ class StableParams(ctypes.Structure):
 
 
 TYPE_ROW_BYTES = 88  # photon_type_row
+PROF_SECTIONS = ["bbv_fused", "bbv", "kbb", "group_unfused", "canon", "sig", "scan", "resolve", "stable"]
 
 # (name, restype, argtypes) — mirrors include/photon.h
 _SIGS = [
@@ -64,6 +65,9 @@ _SIGS = [
     ("photon_last_error", c_char_p, [c_void_p]),
     ("photon_check", c_int, [c_void_p, c_void_p, POINTER(c_int64)]),
     ("photon_ws_status", c_int, [c_void_p, c_void_p, c_void_p, POINTER(c_int64)]),
+    ("photon_profile", c_int, [c_void_p, c_int]),
+    ("photon_profile_read", c_int, [c_void_p, c_void_p, POINTER(c_double), POINTER(c_uint64)]),
+    ("photon_launch_count", c_uint64, []),
     ("photon_bbv_workspace_bytes", c_size_t, [POINTER(Trace)]),
     ("photon_bbv_build", c_int, [c_void_p, POINTER(Trace), c_void_p, c_size_t, c_void_p, c_void_p, c_void_p, c_void_p]),
     ("photon_group_workspace_bytes", c_size_t, [POINTER(Trace), c_uint64]),

@@ -118,6 +118,8 @@ class Photon:
             raise PhotonUnavailable(f"photon_create failed ({rc})")
         self.ctx = ctx
         self._ws: Dict[str, object] = {}
+        self._hint: Dict[tuple, int] = {}   # table sizes that worked, reused by later unchecked calls
+        self._pcap: Dict[int, int] = {}
 
     def __del__(self):
         if getattr(self, "ctx", None) is not None and getattr(self, "L", None) is not None:
@@ -191,7 +193,8 @@ class Photon:
 
     def photon_warp_group(self, t: DeviceTrace, warp_bbv16=None, capacity_hint: int = 0, stream=None,
                           check: bool = True, out: Optional[dict] = None) -> dict:
-        hint = capacity_hint
+        key = (t.n_kernels, t.n_warps)
+        hint = max(capacity_hint, self._hint.get(key, 0))
         for _ in range(8):
             ct = t.c()
             nb = self.L.photon_group_workspace_bytes(ctypes.byref(ct), hint)
@@ -212,6 +215,7 @@ class Photon:
                 continue
             if rc != 0:
                 raise PhotonError(rc, self.L.photon_last_error(self.ctx).decode(), bad)
+            self._hint[key] = hint
             return ty
         raise PhotonError(_lib.ECAPACITY, "type table kept overflowing")
 
@@ -231,7 +235,7 @@ class Photon:
                             pool_all_prior=0, want_dist: bool = True, pair_capacity: int = 0, stream=None,
                             check: bool = True, out: Optional[dict] = None) -> dict:
         K = n_kernels
-        cap = pair_capacity or (16 * K + 65536)
+        cap = max(pair_capacity or (16 * K + 65536), self._pcap.get(K, 0))
         for _ in range(8):
             nb = self.L.photon_match_workspace_bytes(K, ty["capacity"], cap)
             ws = self.workspace("match", nb)
@@ -254,6 +258,7 @@ class Photon:
                 continue
             if rc != 0:
                 raise PhotonError(rc, self.L.photon_last_error(self.ctx).decode(), bad)
+            self._pcap[K] = cap
             return o
         raise PhotonError(_lib.ECAPACITY, "pair table kept overflowing")
 

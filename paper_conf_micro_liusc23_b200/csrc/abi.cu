@@ -5,6 +5,8 @@
 #include <cstring>
 #include <new>
 #include <string>
+#include <utility>
+#include <vector>
 
 #include "internal.h"
 
@@ -15,9 +17,36 @@ struct photon_ctx {
   int num_sms = 148;
   std::string err;
   const void* last_ws = nullptr;
+  // optional in-stream timing of each launch section (photon_profile)
+  bool prof = false;
+  std::vector<std::pair<cudaEvent_t, cudaEvent_t>> ev[PHOTON_PROF_N];
+  size_t used[PHOTON_PROF_N] = {0};
 };
 
 namespace {
+
+struct ProfScope {
+  photon_ctx* c;
+  int sec;
+  cudaStream_t s;
+  cudaEvent_t stop = nullptr;
+  ProfScope(photon_ctx* c_, int sec_, cudaStream_t s_) : c(c_), sec(sec_), s(s_) {
+    if (!c->prof) return;
+    auto& v = c->ev[sec];
+    if (c->used[sec] == v.size()) {
+      cudaEvent_t a, b;
+      cudaEventCreate(&a);
+      cudaEventCreate(&b);
+      v.push_back({a, b});
+    }
+    auto& pr = v[c->used[sec]++];
+    cudaEventRecord(pr.first, s);
+    stop = pr.second;
+  }
+  ~ProfScope() {
+    if (stop) cudaEventRecord(stop, s);
+  }
+};
 
 int fail(photon_ctx* c, int code, const char* fmt, ...) {
   if (c) {
@@ -246,7 +275,37 @@ int photon_create(photon_ctx** out, int cuda_device) {
   return PHOTON_OK;
 }
 
-void photon_destroy(photon_ctx* ctx) { delete ctx; }
+void photon_destroy(photon_ctx* ctx) {
+  if (!ctx) return;
+  for (auto& v : ctx->ev)
+    for (auto& pr : v) { cudaEventDestroy(pr.first); cudaEventDestroy(pr.second); }
+  delete ctx;
+}
+
+int photon_profile(photon_ctx* ctx, int enable) {
+  if (!ctx) return PHOTON_EINVAL;
+  ctx->prof = enable != 0;
+  for (auto& u : ctx->used) u = 0;
+  return PHOTON_OK;
+}
+
+int photon_profile_read(photon_ctx* ctx, void* stream, double* ms, uint64_t* launches) {
+  if (!ctx || !ms || !launches) return PHOTON_EINVAL;
+  CK(cudaStreamSynchronize((cudaStream_t)stream), "sync");
+  for (int sec = 0; sec < PHOTON_PROF_N; ++sec) {
+    double tot = 0;
+    for (size_t i = 0; i < ctx->used[sec]; ++i) {
+      float t = 0;
+      CK(cudaEventElapsedTime(&t, ctx->ev[sec][i].first, ctx->ev[sec][i].second), "elapsed");
+      tot += t;
+    }
+    ms[sec] = tot;
+    launches[sec] = ctx->used[sec];
+  }
+  return PHOTON_OK;
+}
+
+uint64_t photon_launch_count(void) { return launch_counter().load(); }
 
 const char* photon_last_error(const photon_ctx* ctx) { return ctx ? ctx->err.c_str() : "NULL ctx"; }
 
@@ -293,8 +352,12 @@ int photon_bbv_build(photon_ctx* ctx, const photon_trace* t, void* ws, size_t ws
   CK(launch_validate_offsets(d, w.err, s), "validate");
   CK(launch_table_prep(d, w.tbl, w.max_len, w.err, s), "table");
   if (warp_bbv16 || warp_insts)
-    CK(launch_bbv(d, w.tbl, w.max_len, warp_bbv16, warp_insts, nullptr, nullptr, w.err, ctx->num_sms, s), "bbv");
-  if (kernel_bb_insts) CK(launch_kernel_bb_insts(d, w.tbl, kernel_bb_insts, w.err, ctx->num_sms, s), "kbb");
+    { ProfScope ps(ctx, PHOTON_PROF_BBV, s);
+      CK(launch_bbv(d, w.tbl, w.max_len, warp_bbv16, warp_insts, nullptr, nullptr, w.err, ctx->num_sms, s), "bbv"); }
+  if (kernel_bb_insts) {
+    ProfScope ps(ctx, PHOTON_PROF_KBB, s);
+    CK(launch_kernel_bb_insts(d, w.tbl, kernel_bb_insts, w.err, ctx->num_sms, s), "kbb");
+  }
   return PHOTON_OK;
 }
 
@@ -327,15 +390,20 @@ int photon_warp_group(photon_ctx* ctx, const photon_trace* t, const uint32_t* wa
   CK(launch_ht_clear(g.h.ht, s), "ht_clear");
   CK(launch_validate_offsets(d, err, s), "validate");
   if (warp_bbv16) {
+    ProfScope ps(ctx, PHOTON_PROF_GROUP_UNFUSED, s);
     CK(launch_group_from_bbv(d, warp_bbv16, g.h.ht, out->warp_type, err, s), "group_from_bbv");
   } else {
     CK(launch_table_prep(d, g.b.tbl, g.b.max_len, err, s), "table");
+    ProfScope ps(ctx, PHOTON_PROF_BBV_FUSED, s);
     CK(launch_bbv(d, g.b.tbl, g.b.max_len, nullptr, nullptr, &g.h.ht, out->warp_type, err, ctx->num_sms, s),
        "bbv_fused");
   }
-  CK(launch_canonicalise(g.h.ht, t->n_kernels, t->kernel_warp_off, nullptr, *out, g.h.cw, err, ctx->num_sms, s),
-     "canon");
-  CK(launch_remap(out->warp_type, g.h.cw.canon, t->n_warps, out->warp_type, err, s), "remap");
+  {
+    ProfScope ps(ctx, PHOTON_PROF_CANON, s);
+    CK(launch_canonicalise(g.h.ht, t->n_kernels, t->kernel_warp_off, nullptr, *out, g.h.cw, err, ctx->num_sms, s),
+       "canon");
+    CK(launch_remap(out->warp_type, g.h.cw.canon, t->n_warps, out->warp_type, err, s), "remap");
+  }
   return PHOTON_OK;
 }
 
@@ -369,14 +437,24 @@ int photon_kernel_match(photon_ctx* ctx, uint32_t K, const photon_types* types, 
   CK(cudaSetDevice(ctx->device), "cudaSetDevice");
   ctx->last_ws = ws;
   CK(cudaMemsetAsync(m.err, 0, sizeof(DevErr), s), "memset");
-  CK(launch_sig_build(K, types->kernel_type_off, types->type_key, types->type_count, 0, K, m.sig, m.mass, m.err, s),
-     "sig");
-  CK(launch_match_scan(K, types->kernel_type_off, m.sig, m.mass, warps_total, params, 0, K, m.mw, m.pairs,
-                       m.mw.pair_cap, m.n_pairs, m.err, ctx->num_sms, s),
-     "scan");
-  CK(launch_match_resolve(K, types->kernel_type_off, m.sig, m.mass, warps_total, params, m.pairs, m.mw.pair_cap,
-                          m.n_pairs, m.mw, match, match_dist, m.err, s),
-     "resolve");
+  {
+    ProfScope ps(ctx, PHOTON_PROF_SIG, s);
+    CK(launch_sig_build(K, types->kernel_type_off, types->type_key, types->type_count, 0, K, m.sig, m.mass, m.err,
+                        s),
+       "sig");
+  }
+  {
+    ProfScope ps(ctx, PHOTON_PROF_SCAN, s);
+    CK(launch_match_scan(K, types->kernel_type_off, m.sig, m.mass, warps_total, params, 0, K, m.mw, m.pairs,
+                         m.mw.pair_cap, m.n_pairs, m.err, ctx->num_sms, s),
+       "scan");
+  }
+  {
+    ProfScope ps(ctx, PHOTON_PROF_RESOLVE, s);
+    CK(launch_match_resolve(K, types->kernel_type_off, m.sig, m.mass, warps_total, params, m.pairs, m.mw.pair_cap,
+                            m.n_pairs, m.mw, match, match_dist, m.err, s),
+       "resolve");
+  }
   return PHOTON_OK;
 }
 
@@ -465,6 +543,7 @@ int photon_bb_stable(photon_ctx* ctx, const photon_timing* t, const uint64_t* kb
   CK(cudaSetDevice(ctx->device), "cudaSetDevice");
   ctx->last_ws = ws;
   CK(cudaMemsetAsync(w.err, 0, sizeof(DevErr), s), "memset");
+  ProfScope ps(ctx, PHOTON_PROF_STABLE, s);
   CK(launch_stable(*t, kbb, p, w.rest, w.rest_bytes, first_stable, dur, switch_at, w.err, ctx->num_sms, s), "stable");
   return PHOTON_OK;
 }

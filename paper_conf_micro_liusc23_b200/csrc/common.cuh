@@ -3,6 +3,8 @@
 #include <cuda_runtime.h>
 #include <stdint.h>
 
+#include <atomic>
+
 #include "../../include/photon.h"
 
 #if defined(__CUDA_ARCH__) && (__CUDA_ARCH__ < 1000)
@@ -10,6 +12,13 @@
 #endif
 
 namespace photon {
+
+// launches of libphoton kernels since load (one counter per process; bench.py reports it as gpu_launches)
+inline std::atomic<uint64_t>& launch_counter() {
+  static std::atomic<uint64_t> n{0};
+  return n;
+}
+inline void note_launch() { launch_counter().fetch_add(1, std::memory_order_relaxed); }
 
 typedef unsigned __int128 u128;
 typedef __int128 i128;

@@ -135,7 +135,10 @@ __device__ void tile_group(const BbvArgs& a, const Smem& m, uint64_t w0, bool va
       for (int j = 0; j < 16; ++j) same = same && (m.hist[j * TPB + o] == p[j]);
       if (!same) bypass = true;
     }
-    if (!bypass) atomicAdd(&m.lcount[slot], cnt);
+    if (!bypass) {
+      atomicAdd(&m.lcount[slot], cnt);
+      atomicMin(&m.lgslot[slot], (uint32_t)tid);  // group leaders are the lowest tid of their group
+    }
   }
   __syncthreads();
   // global insert: one thread per occupied local slot (owner's key) + bypassing leaders
@@ -146,7 +149,7 @@ __device__ void tile_group(const BbvArgs& a, const Smem& m, uint64_t w0, bool va
       uint32_t key[16];
 #pragma unroll
       for (int j = 0; j < 16; ++j) key[j] = m.hist[j * TPB + o];
-      m.lgslot[i] = ht_insert(a.ht, a.err, m.kid[o], key, hh, m.lcount[i], w0 + o);
+      m.lgslot[i] = ht_insert(a.ht, a.err, m.kid[o], key, hh, m.lcount[i], w0 + m.lgslot[i]);
     }
   }
   uint32_t gslot = UINT32_MAX;
@@ -160,7 +163,7 @@ __device__ void tile_group(const BbvArgs& a, const Smem& m, uint64_t w0, bool va
     a.warp_slot[w0 + tid] = mine;
   }
   __syncthreads();
-  for (int i = tid; i < LSLOTS; i += TPB) { m.lhash[i] = 0ull; m.lcount[i] = 0u; }
+  for (int i = tid; i < LSLOTS; i += TPB) { m.lhash[i] = 0ull; m.lcount[i] = 0u; m.lgslot[i] = UINT32_MAX; }
 }
 
 // Slow path (bad input only): locate the first event of [s, e) whose id is >= B.
@@ -181,7 +184,7 @@ __global__ void __launch_bounds__(TPB, 3) k_bbv(BbvArgs a) {
     for (uint32_t i = tid; i < a.P2; i += TPB) m.tbl[i] = a.tbl[i];
 #pragma unroll
   for (int j = 0; j < 16; ++j) m.hist[j * TPB + tid] = 0u;
-  for (int i = tid; i < LSLOTS; i += TPB) { m.lhash[i] = 0ull; m.lcount[i] = 0u; }
+  for (int i = tid; i < LSLOTS; i += TPB) { m.lhash[i] = 0ull; m.lcount[i] = 0u; m.lgslot[i] = UINT32_MAX; }
   if (tid == 0) {
     for (int s = 0; s < NST; ++s) mbar_init(&m.mbar[s], 1);
     fence_mbar_init();
@@ -315,7 +318,7 @@ __global__ void __launch_bounds__(TPB) k_group_from_bbv(BbvArgs a, const uint32_
   const int tid = threadIdx.x;
   const uint64_t w0 = (uint64_t)blockIdx.x * TPB, w1 = umin64(a.W, w0 + TPB), w = w0 + tid;
   const bool valid = w < w1;
-  for (int i = tid; i < LSLOTS; i += TPB) { m.lhash[i] = 0ull; m.lcount[i] = 0u; }
+  for (int i = tid; i < LSLOTS; i += TPB) { m.lhash[i] = 0ull; m.lcount[i] = 0u; m.lgslot[i] = UINT32_MAX; }
   uint32_t p[16];
   if (valid) {
     const uint4* src = (const uint4*)(bbv + w * 16);
@@ -428,13 +431,13 @@ size_t bbv_table_bytes(uint32_t B) { return (size_t)next_pow2_u32(B < 16 ? 16 : 
 cudaError_t launch_table_prep(const TraceDev& t, uint32_t* tbl, uint32_t* max_len, DevErr* err, cudaStream_t s) {
   uint32_t P2 = next_pow2_u32(t.B < 16 ? 16 : t.B);
   cudaMemsetAsync(max_len, 0, 4, s);
-  k_table_prep<<<(P2 + 255) / 256, 256, 0, s>>>(t.bb_len, t.bb_bin, t.B, P2, tbl, max_len, err);
+  note_launch(), k_table_prep<<<(P2 + 255) / 256, 256, 0, s>>>(t.bb_len, t.bb_bin, t.B, P2, tbl, max_len, err);
   return cudaGetLastError();
 }
 
 cudaError_t launch_validate_offsets(const TraceDev& t, DevErr* err, cudaStream_t s) {
   uint64_t n = t.K > 0 ? t.K : 1;
-  k_validate_offsets<<<(unsigned)ceil_div(n, 256), 256, 0, s>>>(t.kwo, t.K, t.weo, t.W, t.E, err);
+  note_launch(), k_validate_offsets<<<(unsigned)ceil_div(n, 256), 256, 0, s>>>(t.kwo, t.K, t.weo, t.W, t.E, err);
   return cudaGetLastError();
 }
 
@@ -450,7 +453,7 @@ static cudaError_t launch_bbv_t(const BbvArgs& a, size_t smem, int num_sms, cuda
   uint64_t grid = (uint64_t)num_sms * per_sm;
   if (grid > a.n_tiles) grid = a.n_tiles;
   if (grid == 0) return cudaSuccess;
-  fn<<<(unsigned)grid, TPB, smem, s>>>(a);
+  note_launch(), fn<<<(unsigned)grid, TPB, smem, s>>>(a);
   return cudaGetLastError();
 }
 
@@ -483,7 +486,7 @@ cudaError_t launch_group_from_bbv(const TraceDev& t, const uint32_t* warp_bbv16,
   size_t smem = bbv_smem_bytes(0);
   cudaError_t e = cudaFuncSetAttribute(k_group_from_bbv, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return e;
-  k_group_from_bbv<<<(unsigned)tiles, TPB, smem, s>>>(a, warp_bbv16);
+  note_launch(), k_group_from_bbv<<<(unsigned)tiles, TPB, smem, s>>>(a, warp_bbv16);
   return cudaGetLastError();
 }
 
@@ -495,7 +498,7 @@ cudaError_t launch_kernel_bb_insts(const TraceDev& t, const uint32_t* tbl, uint6
   // area: the caller reserves K+1 u64 after the table (see abi.cu).
   uint32_t P2 = next_pow2_u32(t.B < 16 ? 16 : t.B);
   uint64_t* kchunk_off = (uint64_t*)(((uintptr_t)(tbl + P2) + 255) & ~(uintptr_t)255);
-  k_kchunks<<<1, 1, 0, s>>>(t.kwo, t.weo, t.K, kchunk_off);
+  note_launch(), k_kchunks<<<1, 1, 0, s>>>(t.kwo, t.weo, t.K, kchunk_off);
   // upper bound on jobs: E/KBB_CHUNK + K
   uint64_t jobs_ub = ceil_div(t.E, KBB_CHUNK) + t.K;
   uint64_t grid = jobs_ub < (uint64_t)num_sms * 4 ? jobs_ub : (uint64_t)num_sms * 4;
@@ -504,7 +507,7 @@ cudaError_t launch_kernel_bb_insts(const TraceDev& t, const uint32_t* tbl, uint6
   cudaFuncSetAttribute(k_kbb, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)(smem < 1024 ? 1024 : smem));
   // exact job count is on the device (kchunk_off[K]); CTAs loop over [0, chunks_total) with chunks_total read
   // from the upper bound and a guard in the kernel via kchunk_off[K].
-  k_kbb<<<(unsigned)grid, 256, smem < 1024 ? 1024 : smem, s>>>(t.kwo, t.weo, t.bb, tbl, t.K, t.B, P2, kbb, jobs_ub,
+  note_launch(), k_kbb<<<(unsigned)grid, 256, smem < 1024 ? 1024 : smem, s>>>(t.kwo, t.weo, t.bb, tbl, t.K, t.B, P2, kbb, jobs_ub,
                                                               kchunk_off);
   return cudaGetLastError();
 }

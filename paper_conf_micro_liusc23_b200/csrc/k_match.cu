@@ -311,7 +311,7 @@ cudaError_t launch_sig_build(uint32_t K, const uint64_t* kto, const uint32_t* ty
   (void)K;
   if (k_hi <= k_lo) return cudaSuccess;
   uint32_t n = k_hi - k_lo;
-  k_sig<<<(unsigned)ceil_div((uint64_t)n * 32, 256), 256, 0, s>>>(k_lo, k_hi, kto, type_key, type_count, sig, mass, err);
+  note_launch(), k_sig<<<(unsigned)ceil_div((uint64_t)n * 32, 256), 256, 0, s>>>(k_lo, k_hi, kto, type_key, type_count, sig, mass, err);
   return cudaGetLastError();
 }
 
@@ -322,7 +322,7 @@ cudaError_t launch_match_scan(uint32_t K, const uint64_t* kto, const uint64_t* s
   cudaMemsetAsync(n_pairs, 0, 8, s);
   cudaMemsetAsync(mw.n_maybe, 0, 8, s);
   if (K == 0 || k_hi <= k_lo) return cudaGetLastError();
-  k_prof<<<(unsigned)ceil_div((uint64_t)K * 32, 256), 256, 0, s>>>(K, kto, sig, mass, mw.prof);
+  note_launch(), k_prof<<<(unsigned)ceil_div((uint64_t)K * 32, 256), 256, 0, s>>>(K, kto, sig, mass, mw.prof);
   ScanArgs a{};
   a.K = K; a.k_lo = k_lo; a.k_hi = k_hi; a.kto = kto; a.sig = sig; a.mass = mass; a.wt = wt; a.prof = mw.prof;
   a.p = p;
@@ -335,9 +335,9 @@ cudaError_t launch_match_scan(uint32_t K, const uint64_t* kto, const uint64_t* s
   uint64_t t0 = (uint64_t)kb_lo * (kb_lo + 1) / 2, t1 = (uint64_t)kb_hi * (kb_hi + 1) / 2;
   // launch with blockIdx offset by t0 via a shifted grid: simplest is to launch t1 tiles and skip kb < kb_lo
 
-  if (t1 > t0) k_pair_filter<<<(unsigned)(t1 - t0), 256, 0, s>>>(a, t0);
+  if (t1 > t0) note_launch(), k_pair_filter<<<(unsigned)(t1 - t0), 256, 0, s>>>(a, t0);
   unsigned grid = (unsigned)num_sms * 8;
-  k_pair_exact<<<grid, 256, 0, s>>>(a, pairs, pair_cap, n_pairs);
+  note_launch(), k_pair_exact<<<grid, 256, 0, s>>>(a, pairs, pair_cap, n_pairs);
   return cudaGetLastError();
 }
 
@@ -348,15 +348,15 @@ cudaError_t launch_match_resolve(uint32_t K, const uint64_t* kto, const uint64_t
   if (K == 0) return cudaSuccess;
   cudaMemsetAsync(mw.cand_cnt, 0, sizeof(uint32_t) * K, s);
   if (n_pairs) {
-    k_cand_count<<<(unsigned)ceil_div(n_pairs, 256), 256, 0, s>>>(pairs, n_pairs, n_pairs_dev, K, mw.cand_cnt, err);
+    note_launch(), k_cand_count<<<(unsigned)ceil_div(n_pairs, 256), 256, 0, s>>>(pairs, n_pairs, n_pairs_dev, K, mw.cand_cnt, err);
   }
-  k_cand_scan<<<1, 1024, 0, s>>>(mw.cand_cnt, K, mw.cand_off, mw.cand_cur);
+  note_launch(), k_cand_scan<<<1, 1024, 0, s>>>(mw.cand_cnt, K, mw.cand_off, mw.cand_cur);
   if (n_pairs) {
-    k_cand_scatter<<<(unsigned)ceil_div(n_pairs, 256), 256, 0, s>>>(pairs, n_pairs, n_pairs_dev, K, mw.cand_off,
+    note_launch(), k_cand_scatter<<<(unsigned)ceil_div(n_pairs, 256), 256, 0, s>>>(pairs, n_pairs, n_pairs_dev, K, mw.cand_off,
                                                                     mw.cand_cur, mw.cand);
   }
-  k_resolve_states<<<1, 1024, 0, s>>>(K, mw.cand_off, mw.cand, mw.state, p.pool_all_prior);
-  k_resolve_match<<<(unsigned)ceil_div((uint64_t)K * 32, 256), 256, 0, s>>>(K, mw.cand_off, mw.cand, mw.state,
+  note_launch(), k_resolve_states<<<1, 1024, 0, s>>>(K, mw.cand_off, mw.cand, mw.state, p.pool_all_prior);
+  note_launch(), k_resolve_match<<<(unsigned)ceil_div((uint64_t)K * 32, 256), 256, 0, s>>>(K, mw.cand_off, mw.cand, mw.state,
                                                                            p.pool_all_prior, wt, kto, sig, mass,
                                                                            match, match_dist);
   return cudaGetLastError();

@@ -111,9 +111,9 @@ __global__ void __launch_bounds__(256) k_scan_apply(const uint32_t* in, uint64_t
 // out may alias in; bsum needs ceil(n/SB) entries; total (device) receives the sum
 void scan_u32(const uint32_t* in, uint32_t* out, uint64_t n, uint32_t* bsum, uint32_t* total, cudaStream_t s) {
   uint64_t nb = ceil_div(n ? n : 1, SB);
-  k_scan_reduce<<<(unsigned)nb, 256, 0, s>>>(in, n, bsum);
-  k_scan_single<<<1, 1024, 0, s>>>(bsum, nb, total);
-  k_scan_apply<<<(unsigned)nb, 256, 0, s>>>(in, n, bsum, out);
+  note_launch(), k_scan_reduce<<<(unsigned)nb, 256, 0, s>>>(in, n, bsum);
+  note_launch(), k_scan_single<<<1, 1024, 0, s>>>(bsum, nb, total);
+  note_launch(), k_scan_apply<<<(unsigned)nb, 256, 0, s>>>(in, n, bsum, out);
 }
 
 // ---- 1. per-kernel record chunks + validation + keys -------------------------------------------------------
@@ -584,42 +584,42 @@ cudaError_t launch_stable(const photon_timing& t, const uint64_t* kbb, photon_st
   cudaMemsetAsync(first_stable, 0xFF, sizeof(int64_t) * (size_t)K * B, s);
   if (dur) cudaMemsetAsync(dur, 0, sizeof(uint64_t) * (size_t)K * B, s);
   cudaMemsetAsync(L.misc, 0, 64, s);
-  k_rec_chunks<<<1, 1024, 0, s>>>(t.kernel_rec_off, K, R, L.coff, err);
+  note_launch(), k_rec_chunks<<<1, 1024, 0, s>>>(t.kernel_rec_off, K, R, L.coff, err);
   if (R > 0) {
     uint64_t jobs_ub = ceil_div(R, REC_CHUNK) + K;
     unsigned grid = (unsigned)umin64(jobs_ub, (uint64_t)num_sms * 8);
-    k_rec_prep<<<grid, 256, 0, s>>>(t, L.coff, bbits, L.key0, err);
+    note_launch(), k_rec_prep<<<grid, 256, 0, s>>>(t, L.coff, bbits, L.key0, err);
     // radix passes over kbits + bbits bits
     uint32_t bits = kbits + bbits;
     uint64_t* kin = L.key0; uint64_t* kout = L.key1;
     uint32_t* vin = L.val0; uint32_t* vout = L.val1;
     int pass = 0;
     for (uint32_t sh = 0; sh < bits; sh += RBITS, ++pass) {
-      k_radix_up<<<(unsigned)L.n_tiles, RT, 0, s>>>(kin, R, sh, L.hist, L.n_tiles);
+      note_launch(), k_radix_up<<<(unsigned)L.n_tiles, RT, 0, s>>>(kin, R, sh, L.hist, L.n_tiles);
       scan_u32(L.hist, L.hist, (uint64_t)RNB * L.n_tiles, L.bsum, L.misc + 4, s);
-      k_radix_down<<<(unsigned)L.n_tiles, RT, 0, s>>>(kin, vin, R, sh, L.hist, L.n_tiles, kout, vout, pass == 0);
+      note_launch(), k_radix_down<<<(unsigned)L.n_tiles, RT, 0, s>>>(kin, vin, R, sh, L.hist, L.n_tiles, kout, vout, pass == 0);
       uint64_t* tk = kin; kin = kout; kout = tk;
       uint32_t* tv = vin; vin = vout; vout = tv;
     }
     // sorted: kin / vin
     unsigned gR = (unsigned)ceil_div(R, 256);
-    k_gather<<<gR, 256, 0, s>>>(vin, R, t.issue, t.retire, L.X, L.Y);
-    k_heads<<<gR, 256, 0, s>>>(kin, R, L.flag);
+    note_launch(), k_gather<<<gR, 256, 0, s>>>(vin, R, t.issue, t.retire, L.X, L.Y);
+    note_launch(), k_heads<<<gR, 256, 0, s>>>(kin, R, L.flag);
     scan_u32(L.flag, L.flag, R, L.bsum, L.misc + 0, s);  // misc[0] = G
-    k_group_start<<<gR, 256, 0, s>>>(kin, R, L.flag, L.gstart);
-    k_group_end<<<1, 1, 0, s>>>(L.gstart, L.misc + 0, R);
-    k_work_count<<<(unsigned)ceil_div(L.gcap, 256), 256, 0, s>>>(L.gstart, L.misc + 0, 2 * p.window_n, L.nwork,
+    note_launch(), k_group_start<<<gR, 256, 0, s>>>(kin, R, L.flag, L.gstart);
+    note_launch(), k_group_end<<<1, 1, 0, s>>>(L.gstart, L.misc + 0, R);
+    note_launch(), k_work_count<<<(unsigned)ceil_div(L.gcap, 256), 256, 0, s>>>(L.gstart, L.misc + 0, 2 * p.window_n, L.nwork,
                                                                  L.gfirst, L.gcap);
     scan_u32(L.nwork, L.nwork, L.gcap, L.bsum, L.misc + 1, s);  // misc[1] = work items
     WinArgs wa{};
     wa.X = L.X; wa.Y = L.Y; wa.gstart = L.gstart; wa.G = L.misc + 0; wa.work_off = L.nwork; wa.n_work = L.misc + 1;
     wa.gcap = L.gcap; wa.n = p.window_n; wa.dnum = p.delta_num; wa.dden = p.delta_den; wa.gfirst = L.gfirst;
-    k_window<<<(unsigned)num_sms * 4, WT, 0, s>>>(wa);
-    k_finish<<<(unsigned)ceil_div(L.gcap * 32, 256), 256, 0, s>>>(kin, vin, L.X, L.Y, L.gstart, L.misc + 0, L.gfirst,
+    note_launch(), k_window<<<(unsigned)num_sms * 4, WT, 0, s>>>(wa);
+    note_launch(), k_finish<<<(unsigned)ceil_div(L.gcap * 32, 256), 256, 0, s>>>(kin, vin, L.X, L.Y, L.gstart, L.misc + 0, L.gfirst,
                                                                  t.kernel_rec_off, bbits, B, p.window_n,
                                                                  first_stable, dur);
     unsigned gk = (unsigned)umin64(K, (uint64_t)num_sms * 8);
-    k_switch<<<gk ? gk : 1, 256, 0, s>>>(kin, L.gstart, L.misc + 0, L.gfirst, first_stable, kbb, K, B, bbits,
+    note_launch(), k_switch<<<gk ? gk : 1, 256, 0, s>>>(kin, L.gstart, L.misc + 0, L.gfirst, first_stable, kbb, K, B, bbits,
                                          p.rate_num, p.rate_den, switch_at);
   } else {
     cudaMemsetAsync(switch_at, 0xFF, sizeof(int64_t) * K, s);

@@ -260,7 +260,7 @@ __global__ void k_remap_direct(const uint64_t* kwo, uint32_t K, uint64_t W, phot
 
 cudaError_t launch_ht_clear(const HashTable& ht, cudaStream_t s) {
   uint64_t cap = ht.mask + 1;
-  k_ht_clear<<<(unsigned)ceil_div(cap, 256), 256, 0, s>>>(ht);
+  note_launch(), k_ht_clear<<<(unsigned)ceil_div(cap, 256), 256, 0, s>>>(ht);
   return cudaGetLastError();
 }
 
@@ -269,14 +269,14 @@ cudaError_t launch_canonicalise(const HashTable& ht, uint32_t K, const uint64_t*
                                 cudaStream_t s) {
   uint64_t cap = ht.mask + 1;
   cudaMemsetAsync(cw.tcount, 0, sizeof(uint32_t) * (K ? K : 1), s);
-  k_count_types<<<(unsigned)ceil_div(cap, 256), 256, 0, s>>>(ht, K, cw.tcount, err);
-  k_scan_types<<<1, 1024, 0, s>>>(cw.tcount, K, out.kernel_type_off, cw.cursor, out.capacity, err);
-  k_scatter_types<<<(unsigned)ceil_div(cap, 256), 256, 0, s>>>(ht, K, out.kernel_type_off, cw.cursor, cw.list,
+  note_launch(), k_count_types<<<(unsigned)ceil_div(cap, 256), 256, 0, s>>>(ht, K, cw.tcount, err);
+  note_launch(), k_scan_types<<<1, 1024, 0, s>>>(cw.tcount, K, out.kernel_type_off, cw.cursor, out.capacity, err);
+  note_launch(), k_scatter_types<<<(unsigned)ceil_div(cap, 256), 256, 0, s>>>(ht, K, out.kernel_type_off, cw.cursor, cw.list,
                                                                out.capacity);
   unsigned grid = (unsigned)(K < (uint32_t)num_sms * 8 ? K : (uint32_t)num_sms * 8);
   if (grid == 0) grid = 1;
-  k_sort_small<<<grid, 512, 0, s>>>(ht, K, out.kernel_type_off, cw.list, kwo, kernel_warps, out, cw.canon);
-  k_sort_large<<<1, 1024, 0, s>>>(ht, K, out.kernel_type_off, cw.list, kwo, kernel_warps, out, cw.canon,
+  note_launch(), k_sort_small<<<grid, 512, 0, s>>>(ht, K, out.kernel_type_off, cw.list, kwo, kernel_warps, out, cw.canon);
+  note_launch(), k_sort_large<<<1, 1024, 0, s>>>(ht, K, out.kernel_type_off, cw.list, kwo, kernel_warps, out, cw.canon,
                                   (uint32_t*)cw.scratch);
   return cudaGetLastError();
 }
@@ -285,7 +285,7 @@ cudaError_t launch_remap(const uint32_t* warp_slot, const uint32_t* canon, uint6
                          DevErr* err, cudaStream_t s) {
   (void)err;
   if (W == 0) return cudaSuccess;
-  k_remap<<<(unsigned)ceil_div(W, 256), 256, 0, s>>>(warp_slot, canon, W, warp_type);
+  note_launch(), k_remap<<<(unsigned)ceil_div(W, 256), 256, 0, s>>>(warp_slot, canon, W, warp_type);
   return cudaGetLastError();
 }
 
@@ -293,14 +293,14 @@ cudaError_t launch_types_export(uint32_t K, const photon_types& local, uint32_t 
                                 photon_type_row* rows, cudaStream_t s) {
   // T is on the device; launch for the capacity bound and guard inside
   uint64_t cap = local.capacity ? local.capacity : 1;
-  k_export<<<(unsigned)ceil_div(cap, 256), 256, 0, s>>>(K, local, kernel_base, warp_base, rows);
+  note_launch(), k_export<<<(unsigned)ceil_div(cap, 256), 256, 0, s>>>(K, local, kernel_base, warp_base, rows);
   return cudaGetLastError();
 }
 
 cudaError_t launch_rows_insert(const photon_type_row* rows, uint64_t n, uint32_t K, const HashTable& ht,
                                DevErr* err, cudaStream_t s) {
   if (n == 0) return cudaSuccess;
-  k_rows_insert<<<(unsigned)ceil_div(n, 256), 256, 0, s>>>(rows, n, K, ht, err);
+  note_launch(), k_rows_insert<<<(unsigned)ceil_div(n, 256), 256, 0, s>>>(rows, n, K, ht, err);
   return cudaGetLastError();
 }
 
@@ -308,7 +308,7 @@ cudaError_t launch_remap_direct(const uint64_t* kwo_local, uint32_t K_local, uin
                                 const photon_types& local, uint32_t kernel_base, const HashTable& ht,
                                 const uint32_t* canon, uint32_t* warp_type_global, DevErr* err, cudaStream_t s) {
   if (W_local == 0) return cudaSuccess;
-  k_remap_direct<<<(unsigned)ceil_div(W_local, 256), 256, 0, s>>>(kwo_local, K_local, W_local, local, kernel_base, ht,
+  note_launch(), k_remap_direct<<<(unsigned)ceil_div(W_local, 256), 256, 0, s>>>(kwo_local, K_local, W_local, local, kernel_base, ht,
                                                                    canon, warp_type_global, err);
   return cudaGetLastError();
 }
