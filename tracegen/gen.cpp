@@ -54,7 +54,7 @@ struct Gen {
   std::vector<Kern> kerns;
   std::vector<uint32_t> bb_len;   // global BB table
   std::vector<uint64_t> kwoff;    // [K+1] prefix of n_warps
-  std::vector<int> drift_class;   // per BB: 0 stable, 1 drift 1/50, 2 drift 1/20
+  std::vector<int> drift_class;   // per BB: 0 stable (ramp + jitter), 1 drift v/8, 2 drift v/2 (v = warp index)
 };
 
 // ---- program tables (local BB lengths) -------------------------------------------------------------------
@@ -544,7 +544,8 @@ static void kernel_timing(const Gen* g, uint32_t k, uint16_t* bb, uint64_t* issu
         double ramp = 4.0 * (double)len * std::max(0.0, 1.0 - (double)t / Tw);
         d = 4 * len + (uint64_t)ramp + (rng(g->seed, P_JIT, k, v, seq) & 7);
       } else {
-        d = 4 * len + (cls == 1 ? t / 50 : t / 20);
+        // drifting BB types: duration grows with the warp's launch order (bounded)
+        d = 4 * len + (cls == 1 ? v / 8 : v / 2);
       }
       recs.push_back(Rec{t + d, t, v, seq, (uint16_t)id});
       t += d;
