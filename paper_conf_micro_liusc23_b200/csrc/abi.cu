@@ -93,8 +93,10 @@ TraceDev to_dev(const photon_trace* t) {
 // ---- workspace layouts ----------------------------------------------------------------------------------
 struct BbvWs {
   DevErr* err;
-  uint32_t* tbl;  // table + (K+1) u64 chunk prefix after it (see launch_kernel_bb_insts)
+  uint32_t* tbl;        // [P2] packed (len, bin) table
   uint32_t* max_len;
+  uint32_t* tile_k0;    // [n_tiles]
+  uint64_t* kchunk;     // [K+1] kernel_bb_insts job prefix
   size_t bytes;
 };
 BbvWs bbv_layout(const photon_trace* t, void* base) {
@@ -102,10 +104,27 @@ BbvWs bbv_layout(const photon_trace* t, void* base) {
   BbvWs w;
   w.err = c.take<DevErr>(1);
   uint32_t P2 = next_pow2_u32(t->n_bb < 16 ? 16 : t->n_bb);
-  w.tbl = c.take<uint32_t>((size_t)P2 + 64 + 2 * ((size_t)t->n_kernels + 1) + 64);
+  w.tbl = c.take<uint32_t>(P2);
   w.max_len = c.take<uint32_t>(4);
+  w.tile_k0 = c.take<uint32_t>(bbv_n_tiles(t->n_warps) + 1);
+  w.kchunk = c.take<uint64_t>((size_t)t->n_kernels + 1);
   w.bytes = c.off + 256;
   return w;
+}
+
+constexpr uint32_t kEntriesPerTile = 8;
+
+void carve_entries(Carver& c, uint64_t n_tiles, uint64_t W, uint64_t ovf_cap, TileEntries& te) {
+  te.per_tile = kEntriesPerTile;
+  te.tile_n = c.take<uint32_t>(n_tiles + 1);
+  te.tile_ovf = c.take<uint64_t>(n_tiles + 1);
+  te.ent = c.take<TileEntry>(n_tiles * kEntriesPerTile + 1);
+  te.tile_slot = c.take<uint32_t>(n_tiles * kEntriesPerTile + 1);
+  te.ovf_cap = ovf_cap;
+  te.ovf = c.take<TileEntry>(ovf_cap);
+  te.ovf_slot = c.take<uint32_t>(ovf_cap);
+  te.ovf_count = c.take<uint64_t>(1);
+  te.lid = c.take<uint16_t>(W + 1);
 }
 
 uint64_t ht_capacity(uint64_t hint, uint64_t W) {
@@ -131,19 +150,21 @@ void carve_ht(Carver& c, uint64_t cap, uint32_t K, HtWs& w) {
   w.cw.cursor = c.take<uint32_t>(K + 1);
   w.cw.list = c.take<uint32_t>(cap);
   w.cw.canon = c.take<uint32_t>(cap);
-  w.cw.scratch = c.take<uint64_t>(cap / 2 + 1);  // used as u32[cap]
+  w.cw.scratch = c.take<uint32_t>(cap);
+  w.cw.big = c.take<uint32_t>(K + 1);
+  w.cw.nbig = c.take<uint32_t>(2);
 }
 
 struct GroupWs {
   BbvWs b;
   HtWs h;
+  TileEntries te;
   size_t bytes;
 };
 GroupWs group_layout(const photon_trace* t, uint64_t hint, void* base, size_t ws_bytes) {
   GroupWs g;
   g.b = bbv_layout(t, base);
-  Carver c(base);
-  c.off = g.b.bytes;
+  const uint64_t nt = bbv_n_tiles(t->n_warps);
   uint64_t cap = ht_capacity(hint, t->n_warps);
   if (base && ws_bytes) {
     // the capacity actually used is the largest power of two that fits (callers may pass a larger workspace)
@@ -151,12 +172,17 @@ GroupWs group_layout(const photon_trace* t, uint64_t hint, void* base, size_t ws
       Carver probe(nullptr);
       probe.off = g.b.bytes;
       HtWs tmp;
+      TileEntries tt;
       carve_ht(probe, cap * 2, t->n_kernels, tmp);
+      carve_entries(probe, nt, t->n_warps, cap * 2, tt);
       if (probe.off + 256 > ws_bytes) break;
       cap *= 2;
     }
   }
+  Carver c(base);
+  c.off = g.b.bytes;
   carve_ht(c, cap, t->n_kernels, g.h);
+  carve_entries(c, nt, t->n_warps, cap, g.te);
   g.bytes = c.off + 256;
   return g;
 }
@@ -350,13 +376,14 @@ int photon_bbv_build(photon_ctx* ctx, const photon_trace* t, void* ws, size_t ws
   TraceDev d = to_dev(t);
   CK(cudaMemsetAsync(w.err, 0, sizeof(DevErr), s), "memset");
   CK(launch_validate_offsets(d, w.err, s), "validate");
-  CK(launch_table_prep(d, w.tbl, w.max_len, w.err, s), "table");
-  if (warp_bbv16 || warp_insts)
-    { ProfScope ps(ctx, PHOTON_PROF_BBV, s);
-      CK(launch_bbv(d, w.tbl, w.max_len, warp_bbv16, warp_insts, nullptr, nullptr, w.err, ctx->num_sms, s), "bbv"); }
+  CK(launch_table_prep(d, w.tbl, w.max_len, nullptr, w.err, s), "table");
+  if (warp_bbv16 || warp_insts) {
+    ProfScope ps(ctx, PHOTON_PROF_BBV, s);
+    CK(launch_bbv(d, w.tbl, w.max_len, nullptr, warp_bbv16, warp_insts, nullptr, w.err, ctx->num_sms, s), "bbv");
+  }
   if (kernel_bb_insts) {
     ProfScope ps(ctx, PHOTON_PROF_KBB, s);
-    CK(launch_kernel_bb_insts(d, w.tbl, kernel_bb_insts, w.err, ctx->num_sms, s), "kbb");
+    CK(launch_kernel_bb_insts(d, w.tbl, kernel_bb_insts, w.kchunk, w.err, ctx->num_sms, s), "kbb");
   }
   return PHOTON_OK;
 }
@@ -388,21 +415,22 @@ int photon_warp_group(photon_ctx* ctx, const photon_trace* t, const uint32_t* wa
   DevErr* err = g.b.err;
   CK(cudaMemsetAsync(err, 0, sizeof(DevErr), s), "memset");
   CK(launch_ht_clear(g.h.ht, s), "ht_clear");
+  CK(cudaMemsetAsync(g.te.ovf_count, 0, 8, s), "memset");
   CK(launch_validate_offsets(d, err, s), "validate");
+  CK(launch_table_prep(d, g.b.tbl, g.b.max_len, g.b.tile_k0, err, s), "table");
   if (warp_bbv16) {
     ProfScope ps(ctx, PHOTON_PROF_GROUP_UNFUSED, s);
-    CK(launch_group_from_bbv(d, warp_bbv16, g.h.ht, out->warp_type, err, s), "group_from_bbv");
+    CK(launch_group_from_bbv(d, warp_bbv16, g.b.tile_k0, g.te, err, s), "group_from_bbv");
   } else {
-    CK(launch_table_prep(d, g.b.tbl, g.b.max_len, err, s), "table");
     ProfScope ps(ctx, PHOTON_PROF_BBV_FUSED, s);
-    CK(launch_bbv(d, g.b.tbl, g.b.max_len, nullptr, nullptr, &g.h.ht, out->warp_type, err, ctx->num_sms, s),
-       "bbv_fused");
+    CK(launch_bbv(d, g.b.tbl, g.b.max_len, g.b.tile_k0, nullptr, nullptr, &g.te, err, ctx->num_sms, s), "bbv_fused");
   }
   {
     ProfScope ps(ctx, PHOTON_PROF_CANON, s);
+    CK(launch_entries_insert(g.te, bbv_n_tiles(t->n_warps), g.h.ht, err, s), "insert");
     CK(launch_canonicalise(g.h.ht, t->n_kernels, t->kernel_warp_off, nullptr, *out, g.h.cw, err, ctx->num_sms, s),
        "canon");
-    CK(launch_remap(out->warp_type, g.h.cw.canon, t->n_warps, out->warp_type, err, s), "remap");
+    CK(launch_remap_entries(g.te, t->n_warps, g.h.cw.canon, out->warp_type, s), "remap");
   }
   return PHOTON_OK;
 }

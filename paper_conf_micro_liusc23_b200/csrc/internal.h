@@ -18,36 +18,64 @@ struct TraceDev {
   uint64_t W, E;
 };
 
-// packed per-BB table (len << 14 | bin << 10; bit 0 marks ids in [B, P2)), P2 = next pow2 >= B
-size_t bbv_table_bytes(uint32_t B);
-cudaError_t launch_table_prep(const TraceDev& t, uint32_t* tbl, uint32_t* max_len, DevErr* err, cudaStream_t s);
-cudaError_t launch_validate_offsets(const TraceDev& t, DevErr* err, cudaStream_t s);
-// streaming K1 (+ fused K2a when ht != nullptr)
-cudaError_t launch_bbv(const TraceDev& t, const uint32_t* tbl, const uint32_t* max_len, uint32_t* warp_bbv16,
-                       uint64_t* warp_insts, const HashTable* ht, uint32_t* warp_slot, DevErr* err, int num_sms,
-                       cudaStream_t s);
-// K2a from materialised BBVs (unfused path)
-cudaError_t launch_group_from_bbv(const TraceDev& t, const uint32_t* warp_bbv16, const HashTable& ht,
-                                  uint32_t* warp_slot, DevErr* err, cudaStream_t s);
-cudaError_t launch_kernel_bb_insts(const TraceDev& t, const uint32_t* tbl, uint64_t* kbb, DevErr* err,
-                                   int num_sms, cudaStream_t s);
+// One distinct (kernel, key) of a tile, with its warp count and lowest warp (written by K1, inserted by K2a).
+struct alignas(16) TileEntry {
+  uint32_t key[16];  // 16-byte aligned (vector stores)
+  uint64_t hash;
+  uint64_t first;
+  uint32_t kernel;
+  uint32_t count;
+  uint32_t pad[2];
+};
+static_assert(sizeof(TileEntry) == 96, "TileEntry layout");
+struct TileEntries {
+  uint32_t* tile_n;      // [n_tiles] distinct keys of the tile
+  uint64_t* tile_ovf;    // [n_tiles] first overflow entry of the tile (when tile_n > per_tile)
+  TileEntry* ent;        // [n_tiles * per_tile]
+  TileEntry* ovf;        // [ovf_cap]
+  uint64_t* ovf_count;   // [1]
+  uint64_t ovf_cap;
+  uint16_t* lid;         // [W] entry id of each warp within its tile
+  uint32_t* tile_slot;   // [n_tiles * per_tile] hash-table slot of each entry
+  uint32_t* ovf_slot;    // [ovf_cap]
+  uint32_t per_tile;
+};
 
-// ---- A2 canonicalisation (k_types.cu) ---------------------------------------------------------------------
+uint64_t bbv_n_tiles(uint64_t W);
+// packed per-BB table (len << 14 | bin << 10; bit 0 marks ids in [B, P2)), P2 = next pow2 >= B; tile -> kernel
+size_t bbv_table_bytes(uint32_t B);
+cudaError_t launch_table_prep(const TraceDev& t, uint32_t* tbl, uint32_t* max_len, uint32_t* tile_k0, DevErr* err,
+                              cudaStream_t s);
+cudaError_t launch_validate_offsets(const TraceDev& t, DevErr* err, cudaStream_t s);
+// streaming K1 (+ fused K2a de-dup when te != nullptr)
+cudaError_t launch_bbv(const TraceDev& t, const uint32_t* tbl, const uint32_t* max_len, const uint32_t* tile_k0,
+                       uint32_t* warp_bbv16, uint64_t* warp_insts, const TileEntries* te, DevErr* err, int num_sms,
+                       cudaStream_t s);
+// K2a de-dup from materialised BBVs (unfused path)
+cudaError_t launch_group_from_bbv(const TraceDev& t, const uint32_t* warp_bbv16, const uint32_t* tile_k0,
+                                  const TileEntries& te, DevErr* err, cudaStream_t s);
+cudaError_t launch_kernel_bb_insts(const TraceDev& t, const uint32_t* tbl, uint64_t* kbb, uint64_t* kchunk_off,
+                                   DevErr* err, int num_sms, cudaStream_t s);
+
+// ---- A2 insertion + canonicalisation (k_types.cu) ------------------------------------------------------------
 cudaError_t launch_ht_clear(const HashTable& ht, cudaStream_t s);
+cudaError_t launch_entries_insert(const TileEntries& te, uint64_t n_tiles, const HashTable& ht, DevErr* err,
+                                  cudaStream_t s);
+cudaError_t launch_remap_entries(const TileEntries& te, uint64_t W, const uint32_t* canon, uint32_t* warp_type,
+                                 cudaStream_t s);
 struct CanonWs {
   uint32_t* tcount;   // [K] types per kernel
   uint32_t* cursor;   // [K]
   uint32_t* list;     // [cap] slot ids grouped by kernel
   uint32_t* canon;    // [cap] slot -> kernel-local canonical id
-  uint64_t* scratch;  // [cap] sort scratch (large kernels)
+  uint32_t* scratch;  // [cap] sort scratch (large kernels)
+  uint32_t* big;      // [K] kernels with > 32 types: mid-size from the front, large ones from the back
+  uint32_t* nbig;     // [2] counters (mid, large)
 };
 // From the hash table to canonical photon_types (kernel_type_off, rows, warp_sampling_ok) and the slot->id map.
 cudaError_t launch_canonicalise(const HashTable& ht, uint32_t K, const uint64_t* kwo_or_null,
                                 const uint64_t* kernel_warps_or_null, const photon_types& out, const CanonWs& cw,
                                 DevErr* err, int num_sms, cudaStream_t s);
-// warp_type[w] = canon[warp_slot[w]]  (in place allowed)
-cudaError_t launch_remap(const uint32_t* warp_slot, const uint32_t* canon, uint64_t W, uint32_t* warp_type,
-                         DevErr* err, cudaStream_t s);
 // multi-GPU helpers
 cudaError_t launch_types_export(uint32_t K, const photon_types& local, uint32_t kernel_base, uint64_t warp_base,
                                 photon_type_row* rows, cudaStream_t s);
@@ -83,7 +111,6 @@ cudaError_t launch_match_resolve(uint32_t K, const uint64_t* kto, const uint64_t
                                  DevErr* err, cudaStream_t s);
 
 // ---- A5 (k_stable.cu) -------------------------------------------------------------------------------------
-struct StableLayout;
 size_t stable_ws_bytes(const photon_timing& t);
 cudaError_t launch_stable(const photon_timing& t, const uint64_t* kbb, photon_stable_params p, void* ws,
                           size_t ws_bytes, int64_t* first_stable, uint64_t* dur, int64_t* switch_at, DevErr* err,

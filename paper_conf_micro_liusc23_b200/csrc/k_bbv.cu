@@ -1,31 +1,34 @@
-// k_bbv.cu — A1 (per-warp BBV projected to 16 bins) fused with A2's insertion step (K1 + K2a).
+// k_bbv.cu — A1 (per-warp BBV projected to 16 bins) fused with A2's de-duplication step (K1 + K2a).
 //
 // PAPER.md: L161 (a BBV lists the basic blocks a warp executed, identified by start PC), L154 (same instruction
 // sequence => same BBV => same warp type), L178 ("project these BBVs into fixed-size BBVs (We use 16) to improve
 // online clustering performance ... we can easily cluster the warps if they have the same BBV").  Readings [P-1]
 // (entry = executions x length) and [P-2] (sum-preserving fold into 16 bins).
 //
-// Design: one persistent CTA per SM slot.  A CTA owns "tiles" of 256 consecutive analysed warps
-// (one warp segment per thread) and streams each tile's contiguous event range from HBM into a 4-stage ring of
-// 8 KB shared-memory chunks with cp.async.bulk (the TMA copy engine) completing on mbarriers; thread 0 keeps the
-// ring full across tile boundaries.  Each thread folds its own segment's events into a private column of a
-// 16 x 256 shared-memory histogram (conflict-free: column = thread), reading 8 events per 128-bit LDS and one
-// packed (len, bin) word per event from a shared-memory BB table.  At the end of a tile each thread holds its
-// warp's 16-bin key: warps of a CUDA warp are de-duplicated with __match_any_sync on a 64-bit hash, then across
-// the CTA in a shared-memory table, and each distinct (kernel, key) is inserted once into the global
-// open-addressing table (exact key verification).  The warp's slot id is written to warp_slot[w]; the
-// canonical type id replaces it later (k_types.cu).
+// Design.  Persistent CTAs of 256 threads; a "tile" is 256 consecutive analysed warps, tile t is
+// handled by CTA t mod grid.  The tile's contiguous event range is streamed through shared memory in chunks of up
+// to 24K events (48 KB), each staged with cp.async.bulk (TMA copy engine, mbarrier completion) while the previous
+// chunk is combined / the previous tile finalised.  Every chunk is split into 256 equal event ranges, one per
+// thread (merge-path balance: independent of how long the warps are), 8 events per 128-bit LDS, two events per
+// dependent step (both bins read before either is written; equal bins merged), one packed (len, bin) word per
+// event from a shared-memory BB table.  A thread adds the events of a warp that STARTS in its range straight into
+// that warp's result column R[w] (16 bins, only writer); events of the warp already open at its range start go to
+// its private HEAD column A[thread].  After a barrier, warp w's owner adds the HEAD columns of the threads its
+// events spilled into (R[w] += sum A[tau]).  Finalise: each thread holds warp w's 16-bin key in R[w].  Warps are
+// de-duplicated with __match_any_sync on a 64-bit hash (exact key check), then across the CTA in a shared-memory
+// table; the tile's distinct (kernel, key, count, first warp) entries go to a per-tile slot area and each warp
+// gets its local entry id (u16).  No global atomics on the streaming path: the entries are inserted into the
+// global type table by k_entries_insert (k_types.cu).
 #include "internal.h"
 
 namespace photon {
 
 namespace {
 
-constexpr int TPB = 256;            // threads per CTA = warp segments per tile
-constexpr int CH = 4096;            // events per ring chunk (8 KB)
-constexpr int NST = 4;              // ring stages
-constexpr int SMEM_TBL_MAX = 8192;  // BB table entries kept in shared memory
-constexpr int LSLOTS = 256;         // CTA-local de-dup slots (>= distinct keys per tile)
+constexpr int TPB = 256;            // threads per CTA = warps per tile
+constexpr int CAPE = 24576;         // staging chunk (events), 48 KB
+constexpr int SMEM_TBL_MAX = 4096;  // BB table entries kept in shared memory
+constexpr int LSLOTS = 256;         // CTA-local de-dup slots
 
 struct BbvArgs {
   const uint64_t* kwo;
@@ -33,115 +36,195 @@ struct BbvArgs {
   const uint16_t* bb;
   const uint32_t* tbl;
   const uint32_t* max_len;
+  const uint32_t* tile_k0;  // [n_tiles] kernel of each tile's first warp
   uint32_t K, B, P2;
   uint64_t W, E;
   uint32_t* warp_bbv16;
   uint64_t* warp_insts;
-  HashTable ht;
-  uint32_t* warp_slot;
-  int fused;
+  TileEntries te;           // fused grouping outputs (te.tile_n == nullptr => not fused)
   DevErr* err;
   uint64_t n_tiles;
 };
 
-constexpr size_t kHistBytes = 16 * TPB * 4;
-constexpr size_t kStageBytes = (size_t)NST * CH * 2;
-constexpr size_t kLocalBytes = LSLOTS * (8 + 4 + 4 + 4);
-constexpr size_t kMiscBytes = 128;
+constexpr size_t kColBytes = 16 * TPB * 4;
+constexpr size_t kStageBytes = (size_t)(CAPE + 16) * 2;  // + alignment slack of the chunk ends
+constexpr size_t kOffsBytes = (TPB + 2) * 8;
+constexpr size_t kLocalBytes = LSLOTS * (8 + 4 + 4 + 4 + 4);
+constexpr size_t kMiscBytes = 256;
 constexpr size_t kKidBytes = TPB * 4;
 
 __host__ __device__ constexpr size_t bbv_smem_bytes(uint32_t tbl_entries) {
-  return kHistBytes + kStageBytes + NST * 8 + kLocalBytes + kMiscBytes + kKidBytes + (size_t)tbl_entries * 4;
+  return 2 * kColBytes + kStageBytes + kOffsBytes + 16 + kLocalBytes + kMiscBytes + kKidBytes +
+         (size_t)tbl_entries * 4;
 }
 
 struct Smem {
-  uint32_t* hist;
-  uint16_t* stage;
-  uint64_t* mbar;
-  uint64_t* lhash;
-  uint32_t* lowner;
-  uint32_t* lcount;
-  uint32_t* lgslot;
-  uint32_t* misc;
-  uint32_t* kid;
-  uint32_t* tbl;
+  uint32_t* hist;    // R: [16][TPB] result column of each warp of the tile (the key at finalise)
+  uint32_t* head;    // A: [16][TPB] HEAD partial of each thread
+  uint16_t* stage;   // [CAPE]
+  uint64_t* offs;    // [TPB+1] absolute event offsets of the tile's warps
+  uint64_t* mbar;    // [1]
+  uint64_t* lhash;   // [LSLOTS]
+  uint32_t* lowner;  // [LSLOTS] thread whose column holds the key
+  uint32_t* lcount;  // [LSLOTS]
+  uint32_t* lminw;   // [LSLOTS] lowest thread (warp) of the entry
+  uint32_t* lent;    // [LSLOTS] dense local entry id
+  uint32_t* misc;    // [64]: 0 n_entries; [2..3] u64 overflow base
+  uint32_t* kid;     // [TPB] kernel of each thread's warp
+  uint32_t* tbl;     // [P2]
 };
 
 __device__ __forceinline__ Smem carve(uint8_t* s) {
   Smem m;
   m.hist = (uint32_t*)s;
-  m.stage = (uint16_t*)(s + kHistBytes);
-  m.mbar = (uint64_t*)(s + kHistBytes + kStageBytes);
-  m.lhash = m.mbar + NST;
+  m.head = (uint32_t*)(s + kColBytes);
+  m.stage = (uint16_t*)(s + 2 * kColBytes);
+  m.offs = (uint64_t*)(s + 2 * kColBytes + kStageBytes);
+  m.mbar = (uint64_t*)(s + 2 * kColBytes + kStageBytes + kOffsBytes);
+  m.lhash = m.mbar + 2;
   m.lowner = (uint32_t*)(m.lhash + LSLOTS);
   m.lcount = m.lowner + LSLOTS;
-  m.lgslot = m.lcount + LSLOTS;
-  m.misc = m.lgslot + LSLOTS;
+  m.lminw = m.lcount + LSLOTS;
+  m.lent = m.lminw + LSLOTS;
+  m.misc = m.lent + LSLOTS;
   m.kid = m.misc + kMiscBytes / 4;
   m.tbl = m.kid + TPB;
   return m;
 }
 
-__device__ __forceinline__ uint32_t kernel_of(const uint64_t* kwo, uint32_t K, uint64_t w) {
-  // last k with kwo[k] <= w (upper_bound - 1): skips empty kernels
-  uint32_t lo = 0, hi = K;  // answer in [0, K-1]
-  while (lo < hi) {
-    uint32_t mid = (lo + hi + 1) >> 1;
-    if (kwo[mid] <= w) lo = mid; else hi = mid - 1;
+// ---- per-event accumulation --------------------------------------------------------------------------------
+// Table entry: len << 14 | bin << 10 (bit 0 = id in [B, P2)); column byte offset of a bin = bin * 1024.
+struct Acc {
+  uint32_t* col;  // column base (byte-addressed by bin << 10)
+  const uint32_t* tbl;
+  uint32_t bmask;
+  uint32_t raw, orr;
+  __device__ __forceinline__ void one(uint32_t b) {
+    raw |= b;
+    uint32_t t = tbl[b & bmask];
+    orr |= t;
+    *(uint32_t*)((uint8_t*)col + (t & 0x3C00u)) += t >> 14;
   }
-  return lo;
+  // two events, both bins read before either is written (equal bins merged) -> two independent chains
+  __device__ __forceinline__ void two(uint32_t w) {
+    uint32_t t0 = tbl[w & bmask], t1 = tbl[(w >> 16) & bmask];
+    orr |= t0 | t1;
+    uint32_t a0 = t0 & 0x3C00u, a1 = t1 & 0x3C00u;
+    uint32_t l0 = t0 >> 14, l1 = t1 >> 14;
+    uint32_t* c0 = (uint32_t*)((uint8_t*)col + a0);
+    uint32_t* c1 = (uint32_t*)((uint8_t*)col + a1);
+    uint32_t h0 = *c0, h1 = *c1;
+    *c1 = h1 + l1;
+    *c0 = h0 + l0 + (a0 == a1 ? l1 : 0u);
+  }
+  __device__ __forceinline__ void eight(uint4 v) {
+    raw |= v.x | v.y | v.z | v.w;
+    two(v.x);
+    two(v.y);
+    two(v.z);
+    two(v.w);
+  }
+  // events [i, end) of the staged chunk (indices relative to the 16-byte aligned stage base)
+  __device__ __forceinline__ void range(const uint16_t* sb, uint32_t i, uint32_t end) {
+    for (; i < end && (i & 7u); ++i) one(sb[i]);
+    const uint4* sb4 = (const uint4*)sb;
+#pragma unroll 2
+    for (; i + 8 <= end; i += 8) eight(sb4[i >> 3]);
+    for (; i < end; ++i) one(sb[i]);
+  }
+};
+
+// Slow path (bad input only): first event of [s, e) whose id is >= B.
+__device__ void report_bad_event(const BbvArgs& a, uint64_t s, uint64_t e) {
+  for (uint64_t i = s; i < e; ++i)
+    if (a.bb[i] >= a.B) { latch(a.err, PHOTON_ERANGE, (int64_t)i); return; }
 }
 
-// ---- tile finalisation: grouping (K2a) -------------------------------------------------------------------
-// Keys live in the hist columns (hist[j*TPB + tid]).  Three CTA barriers: claim local slots, count + verify,
-// global insert; then every thread writes its warp's slot.
-__device__ void tile_group(const BbvArgs& a, const Smem& m, uint64_t w0, bool valid, uint32_t k, const uint32_t* p) {
+// ---- tile finalisation: CTA de-duplication and per-tile entries -----------------------------------------------
+// Keys are in the hist columns; kid[] holds each thread's kernel.
+__device__ void tile_group(const BbvArgs& a, const Smem& m, uint64_t t, uint64_t w0, bool valid, uint32_t k,
+                           const uint32_t* p) {
   const int tid = threadIdx.x, lane = tid & 31;
-  uint64_t h = valid ? hash_key(k, p) : 0;
-  // warp-level de-dup on the hash, then exact verification against the leader's key
-  unsigned active = __ballot_sync(0xffffffffu, valid);
-  unsigned peers = __match_any_sync(0xffffffffu, (unsigned long long)h);
-  int leader = __ffs(peers) - 1;
-  bool eq = true;
-  uint32_t lk = __shfl_sync(0xffffffffu, k, leader);
-  eq = eq && (lk == k);
+  const uint64_t h = valid ? hash_key(k, p) : 0;
+  const unsigned active = __ballot_sync(0xffffffffu, valid);
+  const unsigned peers = __match_any_sync(0xffffffffu, (unsigned long long)h);
+  const int leader = __ffs(peers) - 1;
+  bool eq = (__shfl_sync(0xffffffffu, k, leader) == k);
 #pragma unroll
-  for (int j = 0; j < 16; ++j) {
-    uint32_t v = __shfl_sync(0xffffffffu, p[j], leader);
-    eq = eq && (v == p[j]);
-  }
-  unsigned eqm = __ballot_sync(0xffffffffu, eq);
-  bool is_leader = valid && (lane == leader || !eq);
-  uint32_t cnt = (lane == leader) ? (uint32_t)__popc(peers & eqm & active) : 1u;
-  // claim a local slot (by hash); a different key with the same hash is resolved by exact compare below
+  for (int j = 0; j < 16; ++j) eq = eq && (__shfl_sync(0xffffffffu, p[j], leader) == p[j]);
+  const unsigned eqm = __ballot_sync(0xffffffffu, eq);
+  const bool is_leader = valid && (lane == leader || !eq);
+  const uint32_t cnt = (lane == leader) ? (uint32_t)__popc(peers & eqm & active) : 1u;
+  // claim a local slot by hash; the first claimer owns it and takes a dense entry id
   int slot = -1;
   bool pending = false;
   if (is_leader) {
     uint32_t i = (uint32_t)(h & (LSLOTS - 1));
     for (int probe = 0; probe < LSLOTS; ++probe) {
       unsigned long long cur = atomicCAS((unsigned long long*)&m.lhash[i], 0ull, (unsigned long long)h);
-      if (cur == 0ull) { m.lowner[i] = (uint32_t)tid; slot = (int)i; break; }
+      if (cur == 0ull) {
+        m.lowner[i] = (uint32_t)tid;
+        m.lent[i] = atomicAdd(&m.misc[0], 1u);
+        slot = (int)i;
+        break;
+      }
       if (cur == h) { slot = (int)i; pending = true; break; }
       i = (i + 1) & (LSLOTS - 1);
     }
   }
   __syncthreads();
-  bool bypass = false;  // hash collision inside the tile: insert globally on our own
+  // verify pending claims (equal hash, maybe different key); a mismatch gets its own entry (bypass)
+  uint32_t my_ent = UINT32_MAX;
   if (slot >= 0) {
+    bool own = true;
     if (pending) {
       uint32_t o = m.lowner[slot];
       bool same = (m.kid[o] == k);
 #pragma unroll
       for (int j = 0; j < 16; ++j) same = same && (m.hist[j * TPB + o] == p[j]);
-      if (!same) bypass = true;
+      own = same;
     }
-    if (!bypass) {
+    if (own) {
       atomicAdd(&m.lcount[slot], cnt);
-      atomicMin(&m.lgslot[slot], (uint32_t)tid);  // group leaders are the lowest tid of their group
+      atomicMin(&m.lminw[slot], (uint32_t)tid);  // leaders are the lowest thread of their warp group
+      my_ent = m.lent[slot];
+    } else {
+      my_ent = atomicAdd(&m.misc[0], 1u) | 0x80000000u;
     }
   }
   __syncthreads();
-  // global insert: one thread per occupied local slot (owner's key) + bypassing leaders
+  const uint32_t n_ent = m.misc[0];
+  const uint32_t M = a.te.per_tile;
+  uint64_t* ovf_base = (uint64_t*)(m.misc + 2);
+  if (n_ent > M) {  // rare: more distinct keys than the tile's fixed entry slots
+    if (tid == 0) {
+      unsigned long long pos = atomicAdd((unsigned long long*)a.te.ovf_count, (unsigned long long)(n_ent - M));
+      if (pos + (n_ent - M) > a.te.ovf_cap) latch(a.err, PHOTON_ECAPACITY, (int64_t)pos);
+      a.te.tile_ovf[t] = pos;
+      *ovf_base = pos;
+    }
+    __syncthreads();
+  }
+  if (tid == 0) a.te.tile_n[t] = n_ent;
+  auto put = [&](uint32_t e, uint32_t kern, const uint32_t* key, uint32_t count, uint32_t minw, uint64_t hh) {
+    TileEntry* dst;
+    if (e < M) {
+      dst = a.te.ent + t * M + e;
+    } else {
+      uint64_t pos = *ovf_base + (e - M);
+      if (pos >= a.te.ovf_cap) return;
+      dst = a.te.ovf + pos;
+    }
+    dst->hash = hh;
+    dst->first = w0 + minw;
+    dst->kernel = kern;
+    dst->count = count;
+    uint4* kd = (uint4*)dst->key;
+    kd[0] = make_uint4(key[0], key[1], key[2], key[3]);
+    kd[1] = make_uint4(key[4], key[5], key[6], key[7]);
+    kd[2] = make_uint4(key[8], key[9], key[10], key[11]);
+    kd[3] = make_uint4(key[12], key[13], key[14], key[15]);
+  };
   for (int i = tid; i < LSLOTS; i += TPB) {
     uint64_t hh = m.lhash[i];
     if (hh != 0ull) {
@@ -149,138 +232,198 @@ __device__ void tile_group(const BbvArgs& a, const Smem& m, uint64_t w0, bool va
       uint32_t key[16];
 #pragma unroll
       for (int j = 0; j < 16; ++j) key[j] = m.hist[j * TPB + o];
-      m.lgslot[i] = ht_insert(a.ht, a.err, m.kid[o], key, hh, m.lcount[i], w0 + m.lgslot[i]);
+      put(m.lent[i], m.kid[o], key, m.lcount[i], m.lminw[i], hh);
     }
   }
-  uint32_t gslot = UINT32_MAX;
-  if (bypass) gslot = ht_insert(a.ht, a.err, k, p, h, cnt, w0 + tid);
-  __syncthreads();
-  if (!bypass && slot >= 0) gslot = m.lgslot[slot];
-  // members of a warp group take the leader's slot
-  uint32_t from_leader = __shfl_sync(0xffffffffu, gslot, leader);
+  if (my_ent != UINT32_MAX && (my_ent & 0x80000000u)) put(my_ent & 0x7FFFFFFFu, k, p, cnt, (uint32_t)tid, h);
+  // members of a warp group take the leader's entry
+  const uint32_t from_leader = __shfl_sync(0xffffffffu, my_ent, leader);
   if (valid) {
-    uint32_t mine = (lane == leader || !eq) ? gslot : from_leader;
-    a.warp_slot[w0 + tid] = mine;
+    uint32_t e = (lane == leader || !eq) ? my_ent : from_leader;
+    a.te.lid[w0 + tid] = (uint16_t)(e & 0xFFFFu);
   }
   __syncthreads();
-  for (int i = tid; i < LSLOTS; i += TPB) { m.lhash[i] = 0ull; m.lcount[i] = 0u; m.lgslot[i] = UINT32_MAX; }
+  for (int i = tid; i < LSLOTS; i += TPB) {
+    m.lhash[i] = 0ull;
+    m.lcount[i] = 0u;
+    m.lminw[i] = UINT32_MAX;
+  }
+  if (tid == 0) m.misc[0] = 0u;
 }
 
-// Slow path (bad input only): locate the first event of [s, e) whose id is >= B.
-__device__ void report_bad_event(const BbvArgs& a, uint64_t s, uint64_t e) {
-  for (uint64_t i = s; i < e; ++i)
-    if (a.bb[i] >= a.B) { latch(a.err, PHOTON_ERANGE, (int64_t)i); return; }
+// thread 0: stage events [cs, ce) into shared memory from the 16-byte aligned base cs & ~7 (bulk part on the TMA
+// copy engine + < 8 tail events of the trace with plain loads), completing on the mbarrier
+__device__ __forceinline__ void stage_chunk(const BbvArgs& a, const Smem& m, uint64_t cs, uint64_t ce, uint64_t E8) {
+  const uint64_t A = cs & ~7ull;
+  uint64_t ae = umin64((ce + 7) & ~7ull, E8);
+  uint32_t bytes = ae > A ? (uint32_t)((ae - A) * 2) : 0u;
+  for (uint64_t i = umax64(A, E8); i < ce; ++i) m.stage[i - A] = a.bb[i];
+  mbar_arrive_expect_tx(m.mbar, bytes);
+  for (uint32_t off = 0; off < bytes; off += 16384) {
+    uint32_t n = bytes - off < 16384 ? bytes - off : 16384;
+    bulk_g2s((uint8_t*)m.stage + off, (const uint8_t*)(a.bb + A) + off, n, m.mbar);
+  }
+}
+
+// Chunk sequence of the CTA: tiles blockIdx.x, +gridDim.x, ...; each tile [ts, te) split into CAPE chunks (a tile
+// with no events still has one empty "chunk" so it is finalised).
+struct Cursor {
+  uint64_t t, ts, te, c, nch;
+  bool valid;
+};
+__device__ __forceinline__ void cursor_tile(const BbvArgs& a, Cursor& u, uint64_t t) {
+  u.t = t;
+  u.valid = t < a.n_tiles;
+  u.c = 0;
+  if (!u.valid) { u.ts = u.te = 0; u.nch = 0; return; }
+  uint64_t w0 = t * TPB, w1 = umin64(a.W, w0 + TPB);
+  u.ts = a.weo[w0];
+  u.te = a.weo[w1];
+  u.nch = u.te > u.ts ? ceil_div(u.te - u.ts, CAPE) : 1;
 }
 
 template <bool SMEM_TBL, bool CHECK_MARK>
-__global__ void __launch_bounds__(TPB, 3) k_bbv(BbvArgs a) {
+__global__ void __launch_bounds__(TPB, 2) k_bbv(BbvArgs a) {
   extern __shared__ __align__(128) uint8_t smem_raw[];
   Smem m = carve(smem_raw);
   const int tid = threadIdx.x;
   const uint32_t bmask = a.P2 - 1;
-  const uint32_t* tblp = SMEM_TBL ? m.tbl : a.tbl;
+  const bool fused = a.te.tile_n != nullptr;
 
   if (SMEM_TBL)
     for (uint32_t i = tid; i < a.P2; i += TPB) m.tbl[i] = a.tbl[i];
 #pragma unroll
-  for (int j = 0; j < 16; ++j) m.hist[j * TPB + tid] = 0u;
-  for (int i = tid; i < LSLOTS; i += TPB) { m.lhash[i] = 0ull; m.lcount[i] = 0u; m.lgslot[i] = UINT32_MAX; }
+  for (int j = 0; j < 16; ++j) { m.hist[j * TPB + tid] = 0u; m.head[j * TPB + tid] = 0u; }
+  for (int i = tid; i < LSLOTS; i += TPB) { m.lhash[i] = 0ull; m.lcount[i] = 0u; m.lminw[i] = UINT32_MAX; }
+  if (tid < 64) m.misc[tid] = 0u;
   if (tid == 0) {
-    for (int s = 0; s < NST; ++s) mbar_init(&m.mbar[s], 1);
+    mbar_init(m.mbar, 1);
     fence_mbar_init();
   }
   const uint32_t max_len = *a.max_len;
   const uint64_t E8 = a.E & ~7ull;
+
+  // producer cursor (thread 0): one chunk ahead of the consumers
+  Cursor pc;
+  if (tid == 0) {
+    cursor_tile(a, pc, blockIdx.x);
+    while (pc.valid && pc.te <= pc.ts) cursor_tile(a, pc, pc.t + gridDim.x);  // tiles without events: no chunk
+    if (pc.valid) stage_chunk(a, m, pc.ts, umin64(pc.ts + CAPE, pc.te), E8);
+  }
+  uint32_t phase = 0;
+
+  Acc acc;
+  acc.tbl = SMEM_TBL ? m.tbl : a.tbl;
+  acc.bmask = bmask;
+
+  uint64_t t = blockIdx.x;
+  // offsets of the first tile
+  uint64_t my_off = 0, last_off = 0;
+  if (t < a.n_tiles) {
+    uint64_t w0 = t * TPB, nw = umin64(a.W, w0 + TPB) - w0;
+    my_off = a.weo[w0 + umin64((uint64_t)tid, nw)];
+    if (tid == 0) last_off = a.weo[w0 + nw];
+  }
   __syncthreads();
 
-  // ---- producer (thread 0): walks the same (tile, chunk) sequence as the consumers ----
-  uint64_t p_tile = blockIdx.x, p_A = 0, p_te = 0;
-  uint32_t p_c = 0, p_n = 0;
-  auto p_load = [&]() {
-    if (p_tile < a.n_tiles) {
-      uint64_t w0 = p_tile * TPB, w1 = umin64(a.W, w0 + TPB);
-      uint64_t ts = a.weo[w0], te = a.weo[w1];
-      p_A = ts & ~7ull;
-      p_te = te;
-      p_n = te > p_A ? (uint32_t)ceil_div(te - p_A, CH) : 0u;
-      p_c = 0;
-    }
-  };
-  auto p_issue = [&](uint32_t slot) {
-    while (p_tile < a.n_tiles && p_c >= p_n) { p_tile += gridDim.x; p_load(); }
-    if (p_tile >= a.n_tiles) return;
-    uint64_t cs = p_A + (uint64_t)p_c * CH, ce = umin64(cs + CH, p_te);
-    uint64_t ae = umin64((ce + 7) & ~7ull, E8);  // bulk part [cs, ae)
-    uint16_t* dst = m.stage + (size_t)slot * CH;
-    uint32_t bytes = ae > cs ? (uint32_t)((ae - cs) * 2) : 0u;
-    for (uint64_t i = umax64(cs, E8); i < ce; ++i) dst[i - cs] = a.bb[i];  // < 8 tail events of the trace
-    mbar_arrive_expect_tx(&m.mbar[slot], bytes);
-    if (bytes) bulk_g2s(dst, a.bb + cs, bytes, &m.mbar[slot]);
-    ++p_c;
-  };
-  if (tid == 0) {
-    p_load();
-    for (int s = 0; s < NST; ++s) p_issue((uint32_t)s);
-  }
-
-  uint32_t q = 0;  // chunks consumed by this CTA
-  uint32_t* col = m.hist + tid;
-  for (uint64_t t = blockIdx.x; t < a.n_tiles; t += gridDim.x) {
-    const uint64_t w0 = t * TPB, w1 = umin64(a.W, w0 + TPB);
+  while (t < a.n_tiles) {
+    const uint64_t w0 = t * TPB, w1 = umin64(a.W, w0 + TPB), nw = w1 - w0;
     const uint64_t w = w0 + tid;
     const bool valid = w < w1;
-    uint64_t s = 0, e = 0;
-    if (valid) { s = a.weo[w]; e = a.weo[w + 1]; }
-    const uint64_t ts = a.weo[w0], te = a.weo[w1];
-    const uint64_t A = ts & ~7ull;
-    const uint32_t nch = te > A ? (uint32_t)ceil_div(te - A, CH) : 0u;
-    uint32_t raw = 0, orr = 0;
-    for (uint32_t c = 0; c < nch; ++c, ++q) {
-      const uint32_t slot = q % NST;
-      const uint64_t cs = A + (uint64_t)c * CH, ce = umin64(cs + CH, te);
-      mbar_wait(&m.mbar[slot], (q / NST) & 1u);
-      const uint16_t* sb = m.stage + (size_t)slot * CH;
-      uint64_t lo = umax64(s, cs), hi = umin64(e, ce);
-      if (lo < hi) {
-        uint32_t i = (uint32_t)(lo - cs), end = (uint32_t)(hi - cs);
-        auto acc1 = [&](uint32_t b) {
-          raw |= b;
-          uint32_t tv = tblp[b & bmask];
-          if (CHECK_MARK) orr |= tv;
-          uint32_t* cell = (uint32_t*)((uint8_t*)col + (tv & 0x3C00u));
-          *cell += tv >> 14;
-        };
-        for (; i < end && (i & 7u); ++i) acc1(sb[i]);
-        for (; i + 8 <= end; i += 8) {
-          uint4 v = *(const uint4*)(sb + i);
-          raw |= v.x | v.y | v.z | v.w;
-          uint32_t ws[4] = {v.x, v.y, v.z, v.w};
-#pragma unroll
-          for (int h = 0; h < 4; ++h) {
-            uint32_t t0 = tblp[ws[h] & bmask];
-            uint32_t t1 = tblp[(ws[h] >> 16) & bmask];
-            if (CHECK_MARK) orr |= t0 | t1;
-            uint32_t* c0 = (uint32_t*)((uint8_t*)col + (t0 & 0x3C00u));
-            *c0 += t0 >> 14;
-            uint32_t* c1 = (uint32_t*)((uint8_t*)col + (t1 & 0x3C00u));
-            *c1 += t1 >> 14;
-          }
-        }
-        for (; i < end; ++i) acc1(sb[i]);
-      }
-      __syncthreads();  // everyone is done with this slot
-      if (tid == 0) p_issue(slot);
+    // publish this tile's offsets; prefetch the next tile's (registers)
+    m.offs[tid] = my_off;
+    if (tid == 0) m.offs[nw] = last_off;  // tid < nw covers [0, nw); offs[nw] = tile end
+    const uint64_t tn = t + gridDim.x;
+    uint64_t nx_off = 0, nx_last = 0;
+    if (tn < a.n_tiles) {
+      uint64_t n0 = tn * TPB, nn = umin64(a.W, n0 + TPB) - n0;
+      nx_off = a.weo[n0 + umin64((uint64_t)tid, nn)];
+      if (tid == 0) nx_last = a.weo[n0 + nn];
     }
+    __syncthreads();
+    const uint64_t ts = m.offs[0], te = m.offs[nw];
+    const uint64_t s = valid ? m.offs[tid] : te, e = valid ? m.offs[tid + 1] : te;
+    const uint64_t nch = te > ts ? ceil_div(te - ts, CAPE) : 0;
+    uint32_t raw = 0, orr = 0;
+    for (uint64_t c = 0; c < nch; ++c) {
+      const uint64_t cs = ts + c * CAPE, ce = umin64(cs + CAPE, te), n = ce - cs;
+      const uint64_t A = cs & ~7ull;
+      mbar_wait(m.mbar, phase);
+      phase ^= 1u;
+      // my balanced range [r0, r1) of the chunk
+      const uint64_t r0 = cs + ((uint64_t)tid * n) / TPB, r1 = cs + ((uint64_t)(tid + 1) * n) / TPB;
+      acc.raw = 0;
+      acc.orr = 0;
+      if (r0 < r1) {
+        // warp (segment) containing r0: last s with offs[s] <= r0 (it is non-empty and contains r0)
+        uint32_t lo = 0, hi = (uint32_t)nw - 1;
+        while (lo < hi) {
+          uint32_t mid = (lo + hi + 1) >> 1;
+          if (m.offs[mid] <= r0) lo = mid; else hi = mid - 1;
+        }
+        uint32_t sg = lo;
+        acc.col = m.offs[sg] < r0 ? m.head + tid : m.hist + sg;  // open warp -> HEAD partial; else its result
+        uint64_t i = r0;
+        const uint16_t* sb = m.stage;
+        for (;;) {
+          uint64_t nb = umin64(m.offs[sg + 1], r1);
+          acc.range(sb, (uint32_t)(i - A), (uint32_t)(nb - A));
+          i = nb;
+          if (i >= r1) break;
+          do { ++sg; } while (m.offs[sg + 1] == m.offs[sg]);  // skip empty warps
+          acc.col = m.hist + sg;
+        }
+      }
+      raw |= acc.raw;
+      orr |= acc.orr;
+      __syncthreads();  // accumulation done; the stage is free
+      if (tid == 0) {   // stage the next chunk (this tile's next, or the next tile's first) during the combine
+        ++pc.c;
+        if (pc.c >= pc.nch || pc.te <= pc.ts) {
+          do { cursor_tile(a, pc, pc.t + gridDim.x); } while (pc.valid && pc.te <= pc.ts);
+        }
+        if (pc.valid) {
+          uint64_t ncs = pc.ts + pc.c * CAPE;
+          stage_chunk(a, m, ncs, umin64(ncs + CAPE, pc.te), E8);
+        }
+      }
+      // combine: warp tid (if it has events in this chunk) adds the HEAD partials of the threads it spilled into
+      if (valid && e > s && e > cs && s < ce) {
+        const uint64_t lo_e = umax64(s, cs), hi_e = umin64(e, ce) - 1;
+        const uint32_t ta = (uint32_t)(((lo_e - cs) * TPB + TPB - 1) / n);
+        const uint32_t tb = (uint32_t)(((hi_e - cs) * TPB + TPB - 1) / n);
+        const uint32_t from = ta + (s >= cs ? 1u : 0u);  // a warp starting in ta's range went straight into R
+        if (from <= tb) {
+          uint32_t sum[16];
+#pragma unroll
+          for (int j = 0; j < 16; ++j) sum[j] = 0u;
+          for (uint32_t u = from; u <= tb; ++u) {
+#pragma unroll
+            for (int j = 0; j < 16; ++j) sum[j] += m.head[j * TPB + u];
+          }
+#pragma unroll
+          for (int j = 0; j < 16; ++j) m.hist[j * TPB + tid] += sum[j];
+        }
+      }
+      __syncthreads();  // HEAD columns consumed
+#pragma unroll
+      for (int j = 0; j < 16; ++j) m.head[j * TPB + tid] = 0u;
+    }
+    // tiles without events: keep the producer's cursor in step (it skipped them)
     // ---- finalise the tile ----
-    if (tid == 0) m.misc[0] = kernel_of(a.kwo, a.K, w0);
     uint32_t p[16];
     uint64_t I = 0;
 #pragma unroll
-    for (int j = 0; j < 16; ++j) { p[j] = col[j * TPB]; I += p[j]; }
+    for (int j = 0; j < 16; ++j) {
+      p[j] = m.hist[j * TPB + tid];
+      I += p[j];
+    }
+    // bad ids anywhere in the tile (event ranges != warps): every warp re-scans its own events (bad input only)
+    const int bad_here = ((((raw | (raw >> 16)) & 0xFFFFu) & ~bmask) != 0u || (CHECK_MARK && (orr & 1u))) ? 1 : 0;
+    if (__syncthreads_or(bad_here) && valid) report_bad_event(a, s, e);
+    uint32_t k = a.tile_k0 ? a.tile_k0[t] : 0u;
     if (valid) {
       if (e < s) latch(a.err, PHOTON_ERANGE, (int64_t)w);
-      uint32_t hi_ids = (raw | (raw >> 16)) & 0xFFFFu;
-      if ((hi_ids & ~bmask) != 0u || (CHECK_MARK && (orr & 1u))) report_bad_event(a, s, e);
       if (e > s && (uint64_t)(e - s) * max_len >= kInstsLimit) {
         // bins may have wrapped: recompute the exact total (rare, long warps only)
         uint64_t exact = 0;
@@ -296,18 +439,22 @@ __global__ void __launch_bounds__(TPB, 3) k_bbv(BbvArgs a) {
         dst[3] = make_uint4(p[12], p[13], p[14], p[15]);
       }
       if (a.warp_insts) a.warp_insts[w] = I;
-    }
-    if (a.fused) {
-      __syncthreads();
-      uint32_t k = m.misc[0];
-      if (valid)
+      if (fused)
         while (k + 1 < a.K && a.kwo[k + 1] <= w) ++k;
-      m.kid[tid] = k;  // kernel of each thread's warp, read by tile_group for owners' keys
+    }
+    if (fused) {
+      m.kid[tid] = k;
       __syncthreads();
-      tile_group(a, m, w0, valid, k, p);
+      tile_group(a, m, t, w0, valid, k, p);
+    } else {
+      __syncthreads();
     }
 #pragma unroll
-    for (int j = 0; j < 16; ++j) col[j * TPB] = 0u;
+    for (int j = 0; j < 16; ++j) m.hist[j * TPB + tid] = 0u;
+    my_off = nx_off;
+    last_off = nx_last;
+    t = tn;
+    __syncthreads();  // result columns cleared and offs free before the next tile
   }
 }
 
@@ -316,9 +463,11 @@ __global__ void __launch_bounds__(TPB) k_group_from_bbv(BbvArgs a, const uint32_
   extern __shared__ __align__(128) uint8_t smem_raw[];
   Smem m = carve(smem_raw);
   const int tid = threadIdx.x;
-  const uint64_t w0 = (uint64_t)blockIdx.x * TPB, w1 = umin64(a.W, w0 + TPB), w = w0 + tid;
+  const uint64_t t = blockIdx.x;
+  const uint64_t w0 = t * TPB, w1 = umin64(a.W, w0 + TPB), w = w0 + tid;
   const bool valid = w < w1;
-  for (int i = tid; i < LSLOTS; i += TPB) { m.lhash[i] = 0ull; m.lcount[i] = 0u; m.lgslot[i] = UINT32_MAX; }
+  for (int i = tid; i < LSLOTS; i += TPB) { m.lhash[i] = 0ull; m.lcount[i] = 0u; m.lminw[i] = UINT32_MAX; }
+  if (tid < 64) m.misc[tid] = 0u;
   uint32_t p[16];
   if (valid) {
     const uint4* src = (const uint4*)(bbv + w * 16);
@@ -333,17 +482,15 @@ __global__ void __launch_bounds__(TPB) k_group_from_bbv(BbvArgs a, const uint32_
   }
 #pragma unroll
   for (int j = 0; j < 16; ++j) m.hist[j * TPB + tid] = p[j];
-  if (tid == 0) m.misc[0] = kernel_of(a.kwo, a.K, w0);
-  __syncthreads();
-  uint32_t k = m.misc[0];
+  uint32_t k = a.tile_k0[t];
   if (valid)
     while (k + 1 < a.K && a.kwo[k + 1] <= w) ++k;
   m.kid[tid] = k;
   __syncthreads();
-  tile_group(a, m, w0, valid, k, p);
+  tile_group(a, m, t, w0, valid, k, p);
 }
 
-// ---- per-BB table and input validation -----------------------------------------------------------------
+// ---- per-BB table, tile kernels, input validation ----------------------------------------------------------
 __global__ void k_table_prep(const uint32_t* __restrict__ bb_len, const uint8_t* __restrict__ bb_bin, uint32_t B,
                              uint32_t P2, uint32_t* __restrict__ tbl, uint32_t* max_len, DevErr* err) {
   uint32_t b = blockIdx.x * blockDim.x + threadIdx.x;
@@ -360,6 +507,18 @@ __global__ void k_table_prep(const uint32_t* __restrict__ bb_len, const uint8_t*
   atomicMax(max_len, len);
 }
 
+__global__ void k_tile_k0(const uint64_t* __restrict__ kwo, uint32_t K, uint64_t n_tiles, uint32_t* tile_k0) {
+  uint64_t t = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (t >= n_tiles) return;
+  uint64_t w = t * TPB;
+  uint32_t lo = 0, hi = K - 1;  // last k with kwo[k] <= w
+  while (lo < hi) {
+    uint32_t mid = (lo + hi + 1) >> 1;
+    if (kwo[mid] <= w) lo = mid; else hi = mid - 1;
+  }
+  tile_k0[t] = lo;
+}
+
 __global__ void k_validate_offsets(const uint64_t* __restrict__ kwo, uint32_t K, const uint64_t* __restrict__ weo,
                                    uint64_t W, uint64_t E, DevErr* err) {
   uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
@@ -370,17 +529,22 @@ __global__ void k_validate_offsets(const uint64_t* __restrict__ kwo, uint32_t K,
   if (i < K && kwo[i + 1] < kwo[i]) latch(err, PHOTON_ERANGE, (int64_t)i);
 }
 
+// warp_event_off must be non-decreasing (the streaming kernel relies on it); one thread per warp
+__global__ void k_validate_weo(const uint64_t* __restrict__ weo, uint64_t W, DevErr* err) {
+  uint64_t w = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (w < W && weo[w + 1] < weo[w]) latch(err, PHOTON_ERANGE, (int64_t)w);
+}
+
 // ---- optional BB distribution kernel_bb_insts[k][b] (L208-210) ------------------------------------------------
 // One CTA per (kernel, event chunk); shared-memory counters for B <= 8192 else global atomics.
 constexpr int KBB_CHUNK = 16384;
 __global__ void __launch_bounds__(256) k_kbb(const uint64_t* __restrict__ kwo, const uint64_t* __restrict__ weo,
                                              const uint16_t* __restrict__ bb, const uint32_t* __restrict__ tbl,
-                                             uint32_t K, uint32_t B, uint32_t P2, uint64_t* __restrict__ kbb,
-                                             uint64_t chunks_total, const uint64_t* __restrict__ kchunk_off) {
+                                             uint32_t K, uint32_t B, uint64_t* __restrict__ kbb, uint64_t jobs_ub,
+                                             const uint64_t* __restrict__ kchunk_off) {
   extern __shared__ __align__(16) uint32_t cnt[];
   const uint64_t total = kchunk_off[K];
-  for (uint64_t job = blockIdx.x; job < total && job < chunks_total; job += gridDim.x) {
-    // job -> (kernel, chunk) via binary search over per-kernel chunk prefix
+  for (uint64_t job = blockIdx.x; job < total && job < jobs_ub; job += gridDim.x) {
     uint32_t lo = 0, hi = K - 1;
     while (lo < hi) {
       uint32_t mid = (lo + hi + 1) >> 1;
@@ -390,8 +554,7 @@ __global__ void __launch_bounds__(256) k_kbb(const uint64_t* __restrict__ kwo, c
     uint64_t c = job - kchunk_off[k];
     uint64_t es = weo[kwo[k]], ee = weo[kwo[k + 1]];
     uint64_t cs = es + c * KBB_CHUNK, ce = umin64(cs + KBB_CHUNK, ee);
-    bool smem = B <= 8192;
-    if (smem) {
+    if (B <= 8192) {
       for (uint32_t i = threadIdx.x; i < B; i += blockDim.x) cnt[i] = 0u;
       __syncthreads();
       for (uint64_t i = cs + threadIdx.x; i < ce; i += blockDim.x) {
@@ -400,8 +563,8 @@ __global__ void __launch_bounds__(256) k_kbb(const uint64_t* __restrict__ kwo, c
       }
       __syncthreads();
       for (uint32_t b = threadIdx.x; b < B; b += blockDim.x)
-        if (cnt[b]) atomicAdd((unsigned long long*)&kbb[(uint64_t)k * B + b],
-                              (unsigned long long)cnt[b] * (tbl[b] >> 14));
+        if (cnt[b])
+          atomicAdd((unsigned long long*)&kbb[(uint64_t)k * B + b], (unsigned long long)cnt[b] * (tbl[b] >> 14));
       __syncthreads();
     } else {
       for (uint64_t i = cs + threadIdx.x; i < ce; i += blockDim.x) {
@@ -412,32 +575,65 @@ __global__ void __launch_bounds__(256) k_kbb(const uint64_t* __restrict__ kwo, c
   }
 }
 
-__global__ void k_kchunks(const uint64_t* __restrict__ kwo, const uint64_t* __restrict__ weo, uint32_t K,
-                          uint64_t* kchunk_off) {
-  // single-thread prefix over K (K is small relative to events; launched <<<1,1>>>)
-  uint64_t acc = 0;
-  for (uint32_t k = 0; k < K; ++k) {
-    kchunk_off[k] = acc;
-    uint64_t es = weo[kwo[k]], ee = weo[kwo[k + 1]];
-    acc += ee > es ? ceil_div(ee - es, KBB_CHUNK) : 0;
+// per-kernel chunk prefix (one CTA, block scan over K)
+__global__ void __launch_bounds__(1024) k_kchunks(const uint64_t* __restrict__ kwo, const uint64_t* __restrict__ weo,
+                                                  uint32_t K, uint64_t* kchunk_off) {
+  __shared__ uint64_t ws[32];
+  __shared__ uint64_t carry;
+  if (threadIdx.x == 0) carry = 0;
+  __syncthreads();
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+  for (uint32_t base = 0; base < K; base += 1024) {
+    uint32_t k = base + threadIdx.x;
+    uint64_t v = 0;
+    if (k < K) {
+      uint64_t es = weo[kwo[k]], ee = weo[kwo[k + 1]];
+      v = ee > es ? ceil_div(ee - es, KBB_CHUNK) : 0;
+    }
+    uint64_t x = v;
+    for (int o = 1; o < 32; o <<= 1) {
+      uint64_t y = __shfl_up_sync(0xffffffffu, x, o);
+      if (lane >= o) x += y;
+    }
+    if (lane == 31) ws[wid] = x;
+    __syncthreads();
+    if (wid == 0) {
+      uint64_t sacc = ws[lane];
+      for (int o = 1; o < 32; o <<= 1) {
+        uint64_t y = __shfl_up_sync(0xffffffffu, sacc, o);
+        if (lane >= o) sacc += y;
+      }
+      ws[lane] = sacc;
+    }
+    __syncthreads();
+    uint64_t ex = carry + (wid ? ws[wid - 1] : 0) + x - v;
+    if (k < K) kchunk_off[k] = ex;
+    __syncthreads();
+    if (threadIdx.x == 1023) carry = ex + v;
+    __syncthreads();
   }
-  kchunk_off[K] = acc;
+  if (threadIdx.x == 0) kchunk_off[K] = carry;
 }
 
 }  // namespace
 
 size_t bbv_table_bytes(uint32_t B) { return (size_t)next_pow2_u32(B < 16 ? 16 : B) * 4 + 64; }
+uint64_t bbv_n_tiles(uint64_t W) { return ceil_div(W, TPB); }
 
-cudaError_t launch_table_prep(const TraceDev& t, uint32_t* tbl, uint32_t* max_len, DevErr* err, cudaStream_t s) {
+cudaError_t launch_table_prep(const TraceDev& t, uint32_t* tbl, uint32_t* max_len, uint32_t* tile_k0, DevErr* err,
+                              cudaStream_t s) {
   uint32_t P2 = next_pow2_u32(t.B < 16 ? 16 : t.B);
   cudaMemsetAsync(max_len, 0, 4, s);
   note_launch(), k_table_prep<<<(P2 + 255) / 256, 256, 0, s>>>(t.bb_len, t.bb_bin, t.B, P2, tbl, max_len, err);
+  uint64_t nt = bbv_n_tiles(t.W);
+  if (tile_k0 && nt) note_launch(), k_tile_k0<<<(unsigned)ceil_div(nt, 256), 256, 0, s>>>(t.kwo, t.K, nt, tile_k0);
   return cudaGetLastError();
 }
 
 cudaError_t launch_validate_offsets(const TraceDev& t, DevErr* err, cudaStream_t s) {
   uint64_t n = t.K > 0 ? t.K : 1;
   note_launch(), k_validate_offsets<<<(unsigned)ceil_div(n, 256), 256, 0, s>>>(t.kwo, t.K, t.weo, t.W, t.E, err);
+  if (t.W) note_launch(), k_validate_weo<<<(unsigned)ceil_div(t.W, 256), 256, 0, s>>>(t.weo, t.W, err);
   return cudaGetLastError();
 }
 
@@ -457,18 +653,17 @@ static cudaError_t launch_bbv_t(const BbvArgs& a, size_t smem, int num_sms, cuda
   return cudaGetLastError();
 }
 
-cudaError_t launch_bbv(const TraceDev& t, const uint32_t* tbl, const uint32_t* max_len, uint32_t* warp_bbv16,
-                       uint64_t* warp_insts, const HashTable* ht, uint32_t* warp_slot, DevErr* err, int num_sms,
+cudaError_t launch_bbv(const TraceDev& t, const uint32_t* tbl, const uint32_t* max_len, const uint32_t* tile_k0,
+                       uint32_t* warp_bbv16, uint64_t* warp_insts, const TileEntries* te, DevErr* err, int num_sms,
                        cudaStream_t s) {
   BbvArgs a{};
-  a.kwo = t.kwo; a.weo = t.weo; a.bb = t.bb; a.tbl = tbl; a.max_len = max_len;
+  a.kwo = t.kwo; a.weo = t.weo; a.bb = t.bb; a.tbl = tbl; a.max_len = max_len; a.tile_k0 = tile_k0;
   a.K = t.K; a.B = t.B; a.P2 = next_pow2_u32(t.B < 16 ? 16 : t.B);
   a.W = t.W; a.E = t.E;
   a.warp_bbv16 = warp_bbv16; a.warp_insts = warp_insts;
-  if (ht) { a.ht = *ht; a.fused = 1; }
-  a.warp_slot = warp_slot;
+  if (te) a.te = *te;
   a.err = err;
-  a.n_tiles = ceil_div(t.W, TPB);
+  a.n_tiles = bbv_n_tiles(t.W);
   if (a.n_tiles == 0) return cudaSuccess;
   bool smem_tbl = a.P2 <= SMEM_TBL_MAX;
   bool mark = a.P2 != t.B;
@@ -477,11 +672,12 @@ cudaError_t launch_bbv(const TraceDev& t, const uint32_t* tbl, const uint32_t* m
   return mark ? launch_bbv_t<false, true>(a, smem, num_sms, s) : launch_bbv_t<false, false>(a, smem, num_sms, s);
 }
 
-cudaError_t launch_group_from_bbv(const TraceDev& t, const uint32_t* warp_bbv16, const HashTable& ht,
-                                  uint32_t* warp_slot, DevErr* err, cudaStream_t s) {
+cudaError_t launch_group_from_bbv(const TraceDev& t, const uint32_t* warp_bbv16, const uint32_t* tile_k0,
+                                  const TileEntries& te, DevErr* err, cudaStream_t s) {
   BbvArgs a{};
-  a.kwo = t.kwo; a.K = t.K; a.W = t.W; a.ht = ht; a.fused = 1; a.warp_slot = warp_slot; a.err = err;
-  uint64_t tiles = ceil_div(t.W, TPB);
+  a.kwo = t.kwo; a.K = t.K; a.W = t.W; a.te = te; a.err = err; a.tile_k0 = tile_k0;
+  uint64_t tiles = bbv_n_tiles(t.W);
+  a.n_tiles = tiles;
   if (tiles == 0) return cudaSuccess;
   size_t smem = bbv_smem_bytes(0);
   cudaError_t e = cudaFuncSetAttribute(k_group_from_bbv, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
@@ -490,25 +686,19 @@ cudaError_t launch_group_from_bbv(const TraceDev& t, const uint32_t* warp_bbv16,
   return cudaGetLastError();
 }
 
-cudaError_t launch_kernel_bb_insts(const TraceDev& t, const uint32_t* tbl, uint64_t* kbb, DevErr* err, int num_sms,
-                                   cudaStream_t s) {
+cudaError_t launch_kernel_bb_insts(const TraceDev& t, const uint32_t* tbl, uint64_t* kbb, uint64_t* kchunk_off,
+                                   DevErr* err, int num_sms, cudaStream_t s) {
   (void)err;
   cudaMemsetAsync(kbb, 0, sizeof(uint64_t) * (size_t)t.K * t.B, s);
-  // chunk prefix lives right after the table in the caller's table area? use a small separate allocation in tbl
-  // area: the caller reserves K+1 u64 after the table (see abi.cu).
-  uint32_t P2 = next_pow2_u32(t.B < 16 ? 16 : t.B);
-  uint64_t* kchunk_off = (uint64_t*)(((uintptr_t)(tbl + P2) + 255) & ~(uintptr_t)255);
-  note_launch(), k_kchunks<<<1, 1, 0, s>>>(t.kwo, t.weo, t.K, kchunk_off);
-  // upper bound on jobs: E/KBB_CHUNK + K
+  note_launch(), k_kchunks<<<1, 1024, 0, s>>>(t.kwo, t.weo, t.K, kchunk_off);
   uint64_t jobs_ub = ceil_div(t.E, KBB_CHUNK) + t.K;
   uint64_t grid = jobs_ub < (uint64_t)num_sms * 4 ? jobs_ub : (uint64_t)num_sms * 4;
   if (grid == 0) grid = 1;
   size_t smem = t.B <= 8192 ? (size_t)t.B * 4 : 0;
-  cudaFuncSetAttribute(k_kbb, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)(smem < 1024 ? 1024 : smem));
-  // exact job count is on the device (kchunk_off[K]); CTAs loop over [0, chunks_total) with chunks_total read
-  // from the upper bound and a guard in the kernel via kchunk_off[K].
-  note_launch(), k_kbb<<<(unsigned)grid, 256, smem < 1024 ? 1024 : smem, s>>>(t.kwo, t.weo, t.bb, tbl, t.K, t.B, P2, kbb, jobs_ub,
-                                                              kchunk_off);
+  if (smem < 1024) smem = 1024;
+  cudaFuncSetAttribute(k_kbb, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  note_launch(), k_kbb<<<(unsigned)grid, 256, smem, s>>>(t.kwo, t.weo, t.bb, tbl, t.K, t.B, kbb, jobs_ub,
+                                                           kchunk_off);
   return cudaGetLastError();
 }
 

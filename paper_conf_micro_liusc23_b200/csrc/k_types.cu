@@ -116,15 +116,59 @@ __device__ void emit_rows(const HashTable& ht, uint32_t k, const uint32_t* sorte
   }
 }
 
-// one CTA per kernel with T_k <= SORT_SMEM_MAX (larger kernels are skipped here and sorted by k_sort_large)
-__global__ void __launch_bounds__(512) k_sort_small(HashTable ht, uint32_t K, const uint64_t* kto,
-                                                    const uint32_t* list, const uint64_t* kwo,
-                                                    const uint64_t* kernel_warps, photon_types out, uint32_t* canon) {
+// Kernels with T_k <= 32 (almost all): one warp each, bitonic network over lanes with shuffles.  Larger kernels
+// are queued: 32 < T_k <= SORT_SMEM_MAX at the front of cw.big (k_sort_mid), larger ones at the back (k_sort_large).
+__global__ void __launch_bounds__(256) k_sort_warp(HashTable ht, uint32_t K, const uint64_t* kto,
+                                                   const uint32_t* list, const uint64_t* kwo,
+                                                   const uint64_t* kernel_warps, photon_types out, uint32_t* canon,
+                                                   uint32_t* big, uint32_t* nbig) {
+  const uint32_t lane = threadIdx.x & 31;
+  const uint32_t k = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  if (k >= K) return;
+  const uint64_t off = kto[k], n = kto[k + 1] - off;
+  if (n > 32) {
+    if (lane == 0) {
+      if (n <= SORT_SMEM_MAX) big[atomicAdd(&nbig[0], 1u)] = k;
+      else big[K - 1 - atomicAdd(&nbig[1], 1u)] = k;
+    }
+    return;
+  }
+  const uint64_t Wk = kernel_warps ? kernel_warps[k] : (kwo[k + 1] - kwo[k]);
+  uint32_t mine = lane < n ? list[off + lane] : UINT32_MAX;
+  for (uint32_t size = 2; size <= 32; size <<= 1) {
+    for (uint32_t stride = size >> 1; stride > 0; stride >>= 1) {
+      uint32_t other = __shfl_xor_sync(0xffffffffu, mine, stride);
+      bool up = (lane & size) == 0;
+      bool lower = (lane & stride) == 0;
+      bool mb = type_before(ht, mine, other);
+      bool keep = (lower == up) ? mb : !mb;
+      if (mine == other) keep = true;
+      mine = keep ? mine : other;
+    }
+  }
+  if (lane < n && off + lane < out.capacity) {
+    const uint4* src = (const uint4*)(ht.key + (uint64_t)mine * 16);
+    uint4* dst = (uint4*)(out.type_key + (off + lane) * 16);
+    dst[0] = src[0]; dst[1] = src[1]; dst[2] = src[2]; dst[3] = src[3];
+    out.type_count[off + lane] = ht.count[mine];
+    out.type_first_warp[off + lane] = ht.first[mine];
+    canon[mine] = lane;
+  }
+  uint32_t c0 = __shfl_sync(0xffffffffu, mine != UINT32_MAX ? ht.count[mine] : 0u, 0);
+  if (lane == 0) out.warp_sampling_ok[k] = (Wk > 0 && 100ull * c0 > 95ull * Wk) ? 1 : 0;  // L249 [P-15]
+}
+
+// 32 < T_k <= SORT_SMEM_MAX: one CTA per queued kernel, shared-memory bitonic sort
+__global__ void __launch_bounds__(512) k_sort_mid(HashTable ht, uint32_t K, const uint64_t* kto,
+                                                  const uint32_t* list, const uint64_t* kwo,
+                                                  const uint64_t* kernel_warps, photon_types out, uint32_t* canon,
+                                                  const uint32_t* big, const uint32_t* nbig) {
   __shared__ uint32_t sh[SORT_SMEM_MAX];
-  for (uint32_t k = blockIdx.x; k < K; k += gridDim.x) {
+  const uint32_t nmid = nbig[0];
+  for (uint32_t q = blockIdx.x; q < nmid; q += gridDim.x) {
+    const uint32_t k = big[q];
     uint64_t off = kto[k], n = kto[k + 1] - off;
     uint64_t Wk = kernel_warps ? kernel_warps[k] : (kwo[k + 1] - kwo[k]);
-    if (n > SORT_SMEM_MAX) continue;
     uint32_t P = 1;
     while (P < n) P <<= 1;
     for (uint32_t i = threadIdx.x; i < P; i += blockDim.x) sh[i] = i < n ? list[off + i] : UINT32_MAX;
@@ -147,14 +191,15 @@ __global__ void __launch_bounds__(512) k_sort_small(HashTable ht, uint32_t K, co
   }
 }
 
-// kernels with T_k > SORT_SMEM_MAX: one CTA, global-memory bitonic sort in scratch (rare: irregular kernels)
+// T_k > SORT_SMEM_MAX (rare: highly irregular kernels): one CTA, global-memory bitonic sort in scratch
 __global__ void __launch_bounds__(1024) k_sort_large(HashTable ht, uint32_t K, const uint64_t* kto,
                                                      const uint32_t* list, const uint64_t* kwo,
                                                      const uint64_t* kernel_warps, photon_types out, uint32_t* canon,
-                                                     uint32_t* scratch) {
-  for (uint32_t k = 0; k < K; ++k) {
+                                                     uint32_t* scratch, const uint32_t* big, const uint32_t* nbig) {
+  const uint32_t nlarge = nbig[1];
+  for (uint32_t q = 0; q < nlarge; ++q) {
+    const uint32_t k = big[K - 1 - q];
     uint64_t off = kto[k], n = kto[k + 1] - off;
-    if (n <= SORT_SMEM_MAX) continue;
     uint64_t Wk = kernel_warps ? kernel_warps[k] : (kwo[k + 1] - kwo[k]);
     uint64_t P = 1;
     while (P < n) P <<= 1;
@@ -178,11 +223,42 @@ __global__ void __launch_bounds__(1024) k_sort_large(HashTable ht, uint32_t K, c
   }
 }
 
-__global__ void k_remap(const uint32_t* slot, const uint32_t* canon, uint64_t W, uint32_t* out) {
-  uint64_t w = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+// K2a: insert every tile entry (and overflow entry) into the global table; one thread per entry slot.
+__global__ void k_entries_insert(TileEntries te, uint64_t n_tiles, HashTable ht, DevErr* err) {
+  const uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  const uint64_t nfix = n_tiles * te.per_tile;
+  const TileEntry* x;
+  uint32_t* out;
+  if (i < nfix) {
+    uint64_t t = i / te.per_tile, e = i % te.per_tile;
+    if (e >= te.tile_n[t]) return;
+    x = te.ent + i;
+    out = te.tile_slot + i;
+  } else {
+    uint64_t j = i - nfix;
+    uint64_t n = *te.ovf_count;
+    if (j >= n || j >= te.ovf_cap) return;
+    x = te.ovf + j;
+    out = te.ovf_slot + j;
+  }
+  uint32_t key[16];
+  const uint4* kp = (const uint4*)x->key;
+#pragma unroll
+  for (int q = 0; q < 4; ++q) {
+    uint4 v = kp[q];
+    key[4 * q] = v.x; key[4 * q + 1] = v.y; key[4 * q + 2] = v.z; key[4 * q + 3] = v.w;
+  }
+  *out = ht_insert(ht, err, x->kernel, key, x->hash, x->count, x->first);
+}
+
+// K2c: warp_type[w] = canonical id of the warp's tile entry
+__global__ void k_remap_entries(TileEntries te, uint64_t W, const uint32_t* canon, uint32_t* warp_type) {
+  const uint64_t w = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
   if (w >= W) return;
-  uint32_t s = slot[w];
-  out[w] = s == UINT32_MAX ? UINT32_MAX : canon[s];
+  const uint64_t t = w >> 8;  // 256 warps per tile (k_bbv.cu TPB)
+  const uint32_t e = te.lid[w];
+  uint32_t slot = e < te.per_tile ? te.tile_slot[t * te.per_tile + e] : te.ovf_slot[te.tile_ovf[t] + (e - te.per_tile)];
+  warp_type[w] = slot == UINT32_MAX ? UINT32_MAX : canon[slot];
 }
 
 __device__ __forceinline__ uint32_t row_kernel(const uint64_t* kto, uint32_t K, uint64_t row) {
@@ -273,19 +349,28 @@ cudaError_t launch_canonicalise(const HashTable& ht, uint32_t K, const uint64_t*
   note_launch(), k_scan_types<<<1, 1024, 0, s>>>(cw.tcount, K, out.kernel_type_off, cw.cursor, out.capacity, err);
   note_launch(), k_scatter_types<<<(unsigned)ceil_div(cap, 256), 256, 0, s>>>(ht, K, out.kernel_type_off, cw.cursor, cw.list,
                                                                out.capacity);
-  unsigned grid = (unsigned)(K < (uint32_t)num_sms * 8 ? K : (uint32_t)num_sms * 8);
-  if (grid == 0) grid = 1;
-  note_launch(), k_sort_small<<<grid, 512, 0, s>>>(ht, K, out.kernel_type_off, cw.list, kwo, kernel_warps, out, cw.canon);
+  cudaMemsetAsync(cw.nbig, 0, 8, s);
+  note_launch(), k_sort_warp<<<(unsigned)ceil_div((uint64_t)K * 32, 256), 256, 0, s>>>(
+      ht, K, out.kernel_type_off, cw.list, kwo, kernel_warps, out, cw.canon, cw.big, cw.nbig);
+  note_launch(), k_sort_mid<<<(unsigned)num_sms, 512, 0, s>>>(ht, K, out.kernel_type_off, cw.list, kwo, kernel_warps,
+                                                             out, cw.canon, cw.big, cw.nbig);
   note_launch(), k_sort_large<<<1, 1024, 0, s>>>(ht, K, out.kernel_type_off, cw.list, kwo, kernel_warps, out, cw.canon,
-                                  (uint32_t*)cw.scratch);
+                                                cw.scratch, cw.big, cw.nbig);
   return cudaGetLastError();
 }
 
-cudaError_t launch_remap(const uint32_t* warp_slot, const uint32_t* canon, uint64_t W, uint32_t* warp_type,
-                         DevErr* err, cudaStream_t s) {
-  (void)err;
+cudaError_t launch_entries_insert(const TileEntries& te, uint64_t n_tiles, const HashTable& ht, DevErr* err,
+                                  cudaStream_t s) {
+  uint64_t n = n_tiles * te.per_tile + te.ovf_cap;
+  if (n == 0) return cudaSuccess;
+  note_launch(), k_entries_insert<<<(unsigned)ceil_div(n, 256), 256, 0, s>>>(te, n_tiles, ht, err);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_remap_entries(const TileEntries& te, uint64_t W, const uint32_t* canon, uint32_t* warp_type,
+                                 cudaStream_t s) {
   if (W == 0) return cudaSuccess;
-  note_launch(), k_remap<<<(unsigned)ceil_div(W, 256), 256, 0, s>>>(warp_slot, canon, W, warp_type);
+  note_launch(), k_remap_entries<<<(unsigned)ceil_div(W, 256), 256, 0, s>>>(te, W, canon, warp_type);
   return cudaGetLastError();
 }
 
