@@ -6,19 +6,22 @@
 // (entry = executions x length) and [P-2] (sum-preserving fold into 16 bins).
 //
 // Design.  Persistent CTAs of 256 threads; a "tile" is 256 consecutive analysed warps, tile t is
-// handled by CTA t mod grid.  The tile's contiguous event range is streamed through shared memory in chunks of up
-// to 24K events (48 KB), each staged with cp.async.bulk (TMA copy engine, mbarrier completion) while the previous
-// chunk is combined / the previous tile finalised.  Every chunk is split into 256 equal event ranges, one per
-// thread (merge-path balance: independent of how long the warps are), 8 events per 128-bit LDS, two events per
-// dependent step (both bins read before either is written; equal bins merged), one packed (len, bin) word per
-// event from a shared-memory BB table.  A thread adds the events of a warp that STARTS in its range straight into
-// that warp's result column R[w] (16 bins, only writer); events of the warp already open at its range start go to
-// its private HEAD column A[thread].  After a barrier, warp w's owner adds the HEAD columns of the threads its
-// events spilled into (R[w] += sum A[tau]).  Finalise: each thread holds warp w's 16-bin key in R[w].  Warps are
-// de-duplicated with __match_any_sync on a 64-bit hash (exact key check), then across the CTA in a shared-memory
-// table; the tile's distinct (kernel, key, count, first warp) entries go to a per-tile slot area and each warp
-// gets its local entry id (u16).  No global atomics on the streaming path: the entries are inserted into the
-// global type table by k_entries_insert (k_types.cu).
+// handled by CTA t mod grid.  The tile's events, widened to whole 16-byte words, are streamed through shared
+// memory in chunks of up to 24K events (48 KB), each staged with cp.async.bulk (TMA copy engine, mbarrier
+// completion) while the previous chunk is combined / the previous tile finalised.  Each chunk's words are split
+// into 256 equal runs, one per thread (merge-path balance: independent of how long the warps are), so every lane
+// executes the same word loop: 8 events per 128-bit LDS, two events per dependent step (both bins read before
+// either is written; equal cells merged), one packed (len, bin-offset) word per event from a shared-memory BB
+// table.  A word may contain one warp boundary (events before it go to the current column, after it to the next
+// warp's); words with more boundaries (warps shorter than 8 events) take a per-event path.  A thread adds events
+// of a warp that STARTS in its run straight into that warp's result column R[w] (its only writer); events of the
+// warp already open at its run start go to its private HEAD column.  After a barrier, warp w's owner adds the HEAD
+// columns of the threads its events spilled into.  Events of neighbouring tiles in the first / last word belong to
+// virtual warps whose column is a scratch column.  Finalise: each thread holds warp w's 16-bin key in R[w]; warps
+// are de-duplicated with __match_any_sync on a 64-bit hash (exact key check), then across the CTA in a shared-
+// memory table; the tile's distinct (kernel, key, count, first warp) entries go to a per-tile slot area and each
+// warp gets its local entry id (u16).  No global atomics on the streaming path: k_entries_insert (k_types.cu)
+// inserts the entries into the global type table.
 #include "internal.h"
 
 namespace photon {
@@ -26,9 +29,13 @@ namespace photon {
 namespace {
 
 constexpr int TPB = 256;            // threads per CTA = warps per tile
-constexpr int CAPE = 24576;         // staging chunk (events), 48 KB
+constexpr int COLS = 264;           // column stride (u32) of the 16 x COLS result / HEAD arrays
+constexpr int COLB = COLS * 4;      // bin stride in bytes; table entry = len << 14 | bin * COLB
+constexpr int DUMMY = 256;          // scratch column (events of neighbouring tiles)
+constexpr int CAPE = 24576;         // staging chunk (events, multiple of 8), 48 KB
 constexpr int SMEM_TBL_MAX = 4096;  // BB table entries kept in shared memory
 constexpr int LSLOTS = 256;         // CTA-local de-dup slots
+static_assert(15 * COLB < (1 << 14), "bin offset must fit below the length field");
 
 struct BbvArgs {
   const uint64_t* kwo;
@@ -46,9 +53,9 @@ struct BbvArgs {
   uint64_t n_tiles;
 };
 
-constexpr size_t kColBytes = 16 * TPB * 4;
-constexpr size_t kStageBytes = (size_t)(CAPE + 16) * 2;  // + alignment slack of the chunk ends
-constexpr size_t kOffsBytes = (TPB + 2) * 8;
+constexpr size_t kColBytes = (size_t)16 * COLB;
+constexpr size_t kStageBytes = (size_t)CAPE * 2;
+constexpr size_t kOffsBytes = (TPB + 4) * 8;
 constexpr size_t kLocalBytes = LSLOTS * (8 + 4 + 4 + 4 + 4);
 constexpr size_t kMiscBytes = 256;
 constexpr size_t kKidBytes = TPB * 4;
@@ -59,10 +66,10 @@ __host__ __device__ constexpr size_t bbv_smem_bytes(uint32_t tbl_entries) {
 }
 
 struct Smem {
-  uint32_t* hist;    // R: [16][TPB] result column of each warp of the tile (the key at finalise)
-  uint32_t* head;    // A: [16][TPB] HEAD partial of each thread
+  uint32_t* hist;    // R: [16][COLS] result column of each warp of the tile (the key at finalise) + DUMMY
+  uint32_t* head;    // A: [16][COLS] HEAD partial of each thread
   uint16_t* stage;   // [CAPE]
-  uint64_t* offs;    // [TPB+1] absolute event offsets of the tile's warps
+  uint64_t* offs;    // [TPB+3] o[0] = aligned tile start, o[1+v] = start of warp v, o[nw+1] = end, o[nw+2] = Z
   uint64_t* mbar;    // [1]
   uint64_t* lhash;   // [LSLOTS]
   uint32_t* lowner;  // [LSLOTS] thread whose column holds the key
@@ -93,44 +100,34 @@ __device__ __forceinline__ Smem carve(uint8_t* s) {
 }
 
 // ---- per-event accumulation --------------------------------------------------------------------------------
-// Table entry: len << 14 | bin << 10 (bit 0 = id in [B, P2)); column byte offset of a bin = bin * 1024.
+// Table entry t: len << 14 | bin * COLB (bit 0 = id in [B, P2)); cell address = column + (t & 0x3FFC).
 struct Acc {
-  uint32_t* col;  // column base (byte-addressed by bin << 10)
   const uint32_t* tbl;
   uint32_t bmask;
   uint32_t raw, orr;
-  __device__ __forceinline__ void one(uint32_t b) {
-    raw |= b;
+  __device__ __forceinline__ void one(uint32_t* col, uint32_t b) {
     uint32_t t = tbl[b & bmask];
     orr |= t;
-    *(uint32_t*)((uint8_t*)col + (t & 0x3C00u)) += t >> 14;
+    *(uint32_t*)((uint8_t*)col + (t & 0x3FFCu)) += t >> 14;
   }
-  // two events, both bins read before either is written (equal bins merged) -> two independent chains
-  __device__ __forceinline__ void two(uint32_t w) {
+  // two events into columns c0 / c1: both cells read before either is written (equal cells merged)
+  __device__ __forceinline__ void two(uint32_t w, uint32_t* c0, uint32_t* c1) {
     uint32_t t0 = tbl[w & bmask], t1 = tbl[(w >> 16) & bmask];
     orr |= t0 | t1;
-    uint32_t a0 = t0 & 0x3C00u, a1 = t1 & 0x3C00u;
+    uint32_t* p0 = (uint32_t*)((uint8_t*)c0 + (t0 & 0x3FFCu));
+    uint32_t* p1 = (uint32_t*)((uint8_t*)c1 + (t1 & 0x3FFCu));
     uint32_t l0 = t0 >> 14, l1 = t1 >> 14;
-    uint32_t* c0 = (uint32_t*)((uint8_t*)col + a0);
-    uint32_t* c1 = (uint32_t*)((uint8_t*)col + a1);
-    uint32_t h0 = *c0, h1 = *c1;
-    *c1 = h1 + l1;
-    *c0 = h0 + l0 + (a0 == a1 ? l1 : 0u);
+    uint32_t h0 = *p0, h1 = *p1;
+    *p1 = h1 + l1;
+    *p0 = h0 + l0 + (p0 == p1 ? l1 : 0u);
   }
-  __device__ __forceinline__ void eight(uint4 v) {
+  // one 16-byte word: events j < bo into ca, j >= bo into cb
+  __device__ __forceinline__ void word(uint4 v, uint32_t bo, uint32_t* ca, uint32_t* cb) {
     raw |= v.x | v.y | v.z | v.w;
-    two(v.x);
-    two(v.y);
-    two(v.z);
-    two(v.w);
-  }
-  // events [i, end) of the staged chunk (indices relative to the 16-byte aligned stage base)
-  __device__ __forceinline__ void range(const uint16_t* sb, uint32_t i, uint32_t end) {
-    for (; i < end && (i & 7u); ++i) one(sb[i]);
-    const uint4* sb4 = (const uint4*)sb;
-#pragma unroll 2
-    for (; i + 8 <= end; i += 8) eight(sb4[i >> 3]);
-    for (; i < end; ++i) one(sb[i]);
+    two(v.x, bo > 0 ? ca : cb, bo > 1 ? ca : cb);
+    two(v.y, bo > 2 ? ca : cb, bo > 3 ? ca : cb);
+    two(v.z, bo > 4 ? ca : cb, bo > 5 ? ca : cb);
+    two(v.w, bo > 6 ? ca : cb, bo > 7 ? ca : cb);
   }
 };
 
@@ -141,7 +138,7 @@ __device__ void report_bad_event(const BbvArgs& a, uint64_t s, uint64_t e) {
 }
 
 // ---- tile finalisation: CTA de-duplication and per-tile entries -----------------------------------------------
-// Keys are in the hist columns; kid[] holds each thread's kernel.
+// Keys are in the result columns (hist[j*COLS + tid]); kid[] holds each thread's kernel.
 __device__ void tile_group(const BbvArgs& a, const Smem& m, uint64_t t, uint64_t w0, bool valid, uint32_t k,
                            const uint32_t* p) {
   const int tid = threadIdx.x, lane = tid & 31;
@@ -181,7 +178,7 @@ __device__ void tile_group(const BbvArgs& a, const Smem& m, uint64_t t, uint64_t
       uint32_t o = m.lowner[slot];
       bool same = (m.kid[o] == k);
 #pragma unroll
-      for (int j = 0; j < 16; ++j) same = same && (m.hist[j * TPB + o] == p[j]);
+      for (int j = 0; j < 16; ++j) same = same && (m.hist[j * COLS + o] == p[j]);
       own = same;
     }
     if (own) {
@@ -231,7 +228,7 @@ __device__ void tile_group(const BbvArgs& a, const Smem& m, uint64_t t, uint64_t
       uint32_t o = m.lowner[i];
       uint32_t key[16];
 #pragma unroll
-      for (int j = 0; j < 16; ++j) key[j] = m.hist[j * TPB + o];
+      for (int j = 0; j < 16; ++j) key[j] = m.hist[j * COLS + o];
       put(m.lent[i], m.kid[o], key, m.lcount[i], m.lminw[i], hh);
     }
   }
@@ -251,35 +248,43 @@ __device__ void tile_group(const BbvArgs& a, const Smem& m, uint64_t t, uint64_t
   if (tid == 0) m.misc[0] = 0u;
 }
 
-// thread 0: stage events [cs, ce) into shared memory from the 16-byte aligned base cs & ~7 (bulk part on the TMA
-// copy engine + < 8 tail events of the trace with plain loads), completing on the mbarrier
+// thread 0: stage the word-aligned events [cs, ce) into shared memory (bulk part on the TMA copy engine; events
+// at or past E8 with plain loads, positions past E zero-filled), completing on the mbarrier
 __device__ __forceinline__ void stage_chunk(const BbvArgs& a, const Smem& m, uint64_t cs, uint64_t ce, uint64_t E8) {
-  const uint64_t A = cs & ~7ull;
-  uint64_t ae = umin64((ce + 7) & ~7ull, E8);
-  uint32_t bytes = ae > A ? (uint32_t)((ae - A) * 2) : 0u;
-  for (uint64_t i = umax64(A, E8); i < ce; ++i) m.stage[i - A] = a.bb[i];
+  uint64_t ae = umin64(ce, E8);
+  uint32_t bytes = ae > cs ? (uint32_t)((ae - cs) * 2) : 0u;
+  for (uint64_t i = umax64(cs, E8); i < ce; ++i) m.stage[i - cs] = i < a.E ? a.bb[i] : (uint16_t)0;
   mbar_arrive_expect_tx(m.mbar, bytes);
   for (uint32_t off = 0; off < bytes; off += 16384) {
     uint32_t n = bytes - off < 16384 ? bytes - off : 16384;
-    bulk_g2s((uint8_t*)m.stage + off, (const uint8_t*)(a.bb + A) + off, n, m.mbar);
+    bulk_g2s((uint8_t*)m.stage + off, (const uint8_t*)(a.bb + cs) + off, n, m.mbar);
   }
 }
 
-// Chunk sequence of the CTA: tiles blockIdx.x, +gridDim.x, ...; each tile [ts, te) split into CAPE chunks (a tile
-// with no events still has one empty "chunk" so it is finalised).
+// Chunk sequence of the CTA: tiles blockIdx.x, +gridDim.x, ...; tile events widened to words [A, Z), split into
+// CAPE chunks; tiles without events have no chunk.
 struct Cursor {
-  uint64_t t, ts, te, c, nch;
+  uint64_t t, A, Z, c, nch;
   bool valid;
 };
 __device__ __forceinline__ void cursor_tile(const BbvArgs& a, Cursor& u, uint64_t t) {
   u.t = t;
   u.valid = t < a.n_tiles;
   u.c = 0;
-  if (!u.valid) { u.ts = u.te = 0; u.nch = 0; return; }
+  u.nch = 0;
+  u.A = u.Z = 0;
+  if (!u.valid) return;
   uint64_t w0 = t * TPB, w1 = umin64(a.W, w0 + TPB);
-  u.ts = a.weo[w0];
-  u.te = a.weo[w1];
-  u.nch = u.te > u.ts ? ceil_div(u.te - u.ts, CAPE) : 1;
+  uint64_t ts = a.weo[w0], te = a.weo[w1];
+  if (te <= ts) return;
+  u.A = ts & ~7ull;
+  u.Z = (te + 7) & ~7ull;
+  u.nch = ceil_div(u.Z - u.A, CAPE);
+}
+
+__device__ __forceinline__ uint32_t next_nonempty(const uint64_t* o, uint32_t s, uint32_t last) {
+  do { ++s; } while (s < last && o[s + 1] == o[s]);
+  return s;
 }
 
 template <bool SMEM_TBL, bool CHECK_MARK>
@@ -292,8 +297,7 @@ __global__ void __launch_bounds__(TPB, 2) k_bbv(BbvArgs a) {
 
   if (SMEM_TBL)
     for (uint32_t i = tid; i < a.P2; i += TPB) m.tbl[i] = a.tbl[i];
-#pragma unroll
-  for (int j = 0; j < 16; ++j) { m.hist[j * TPB + tid] = 0u; m.head[j * TPB + tid] = 0u; }
+  for (int i = tid; i < 16 * COLS; i += TPB) { m.hist[i] = 0u; m.head[i] = 0u; }
   for (int i = tid; i < LSLOTS; i += TPB) { m.lhash[i] = 0ull; m.lcount[i] = 0u; m.lminw[i] = UINT32_MAX; }
   if (tid < 64) m.misc[tid] = 0u;
   if (tid == 0) {
@@ -307,8 +311,8 @@ __global__ void __launch_bounds__(TPB, 2) k_bbv(BbvArgs a) {
   Cursor pc;
   if (tid == 0) {
     cursor_tile(a, pc, blockIdx.x);
-    while (pc.valid && pc.te <= pc.ts) cursor_tile(a, pc, pc.t + gridDim.x);  // tiles without events: no chunk
-    if (pc.valid) stage_chunk(a, m, pc.ts, umin64(pc.ts + CAPE, pc.te), E8);
+    while (pc.valid && pc.nch == 0) cursor_tile(a, pc, pc.t + gridDim.x);
+    if (pc.valid) stage_chunk(a, m, pc.A, umin64(pc.A + CAPE, pc.Z), E8);
   }
   uint32_t phase = 0;
 
@@ -317,8 +321,7 @@ __global__ void __launch_bounds__(TPB, 2) k_bbv(BbvArgs a) {
   acc.bmask = bmask;
 
   uint64_t t = blockIdx.x;
-  // offsets of the first tile
-  uint64_t my_off = 0, last_off = 0;
+  uint64_t my_off = 0, last_off = 0;  // weo[w0 + tid] (clamped) and weo[w1] of the current tile
   if (t < a.n_tiles) {
     uint64_t w0 = t * TPB, nw = umin64(a.W, w0 + TPB) - w0;
     my_off = a.weo[w0 + umin64((uint64_t)tid, nw)];
@@ -327,12 +330,15 @@ __global__ void __launch_bounds__(TPB, 2) k_bbv(BbvArgs a) {
   __syncthreads();
 
   while (t < a.n_tiles) {
-    const uint64_t w0 = t * TPB, w1 = umin64(a.W, w0 + TPB), nw = w1 - w0;
+    const uint64_t w0 = t * TPB, w1 = umin64(a.W, w0 + TPB);
+    const uint32_t nw = (uint32_t)(w1 - w0);
     const uint64_t w = w0 + tid;
     const bool valid = w < w1;
-    // publish this tile's offsets; prefetch the next tile's (registers)
-    m.offs[tid] = my_off;
-    if (tid == 0) m.offs[nw] = last_off;  // tid < nw covers [0, nw); offs[nw] = tile end
+    // o[1 + v] = start of warp v, o[nw + 1] = tile end; o[0] / o[nw + 2] = word-aligned bounds (virtual warps)
+    if ((uint32_t)tid <= nw) m.offs[1 + tid] = my_off;
+    if (tid == 0) {
+      m.offs[1 + nw] = last_off;
+    }
     const uint64_t tn = t + gridDim.x;
     uint64_t nx_off = 0, nx_last = 0;
     if (tn < a.n_tiles) {
@@ -341,84 +347,122 @@ __global__ void __launch_bounds__(TPB, 2) k_bbv(BbvArgs a) {
       if (tid == 0) nx_last = a.weo[n0 + nn];
     }
     __syncthreads();
-    const uint64_t ts = m.offs[0], te = m.offs[nw];
-    const uint64_t s = valid ? m.offs[tid] : te, e = valid ? m.offs[tid + 1] : te;
-    const uint64_t nch = te > ts ? ceil_div(te - ts, CAPE) : 0;
-    uint32_t raw = 0, orr = 0;
+    const uint64_t ts = m.offs[1], te = m.offs[1 + nw];
+    const uint64_t At = ts & ~7ull, Zt = (te + 7) & ~7ull;
+    if (tid == 0) {
+      m.offs[0] = At;
+      m.offs[nw + 2] = Zt;
+    }
+    const uint64_t s = valid ? m.offs[1 + tid] : te, e = valid ? m.offs[2 + tid] : te;
+    const uint64_t nch = te > ts ? ceil_div(Zt - At, CAPE) : 0;
+    const uint32_t last = nw + 1;  // index of the virtual tail warp
+    __syncthreads();
+    uint32_t* const headcol = m.head + tid;
+    uint32_t* const dummy = m.hist + DUMMY;
+    auto colof = [&](uint32_t sp) -> uint32_t* { return (sp == 0 || sp == last) ? dummy : m.hist + (sp - 1); };
+    acc.raw = 0;
+    acc.orr = 0;
     for (uint64_t c = 0; c < nch; ++c) {
-      const uint64_t cs = ts + c * CAPE, ce = umin64(cs + CAPE, te), n = ce - cs;
-      const uint64_t A = cs & ~7ull;
+      const uint64_t cs = At + c * CAPE, ce = umin64(cs + CAPE, Zt);
+      const uint64_t nwc = (ce - cs) >> 3;
       mbar_wait(m.mbar, phase);
       phase ^= 1u;
-      // my balanced range [r0, r1) of the chunk
-      const uint64_t r0 = cs + ((uint64_t)tid * n) / TPB, r1 = cs + ((uint64_t)(tid + 1) * n) / TPB;
-      acc.raw = 0;
-      acc.orr = 0;
+      // my run of words [r0, r1) of the chunk
+      const uint64_t r0 = cs + 8 * (((uint64_t)tid * nwc) / TPB), r1 = cs + 8 * (((uint64_t)(tid + 1) * nwc) / TPB);
       if (r0 < r1) {
-        // warp (segment) containing r0: last s with offs[s] <= r0 (it is non-empty and contains r0)
-        uint32_t lo = 0, hi = (uint32_t)nw - 1;
+        // warp (with virtual ones) containing r0: last s' with o[s'] <= r0
+        uint32_t lo = 0, hi = last;
         while (lo < hi) {
           uint32_t mid = (lo + hi + 1) >> 1;
           if (m.offs[mid] <= r0) lo = mid; else hi = mid - 1;
         }
         uint32_t sg = lo;
-        acc.col = m.offs[sg] < r0 ? m.head + tid : m.hist + sg;  // open warp -> HEAD partial; else its result
-        uint64_t i = r0;
-        const uint16_t* sb = m.stage;
-        for (;;) {
-          uint64_t nb = umin64(m.offs[sg + 1], r1);
-          acc.range(sb, (uint32_t)(i - A), (uint32_t)(nb - A));
-          i = nb;
-          if (i >= r1) break;
-          do { ++sg; } while (m.offs[sg + 1] == m.offs[sg]);  // skip empty warps
-          acc.col = m.hist + sg;
+        uint32_t* col = (m.offs[sg] < r0) ? headcol : colof(sg);  // warp open at my run start -> HEAD
+        uint64_t nb = m.offs[sg + 1];
+        uint32_t sgn = sg < last ? next_nonempty(m.offs, sg, last) : sg;
+        uint32_t* coln = colof(sgn);
+        uint64_t nb2 = sgn != sg ? m.offs[sgn + 1] : ~0ull;
+        const uint4* sb4 = (const uint4*)m.stage;
+        for (uint64_t q = r0; q < r1; q += 8) {
+          const uint4 v = sb4[(q - cs) >> 3];
+          if (nb2 < q + 8) {
+            // several warp boundaries inside this word (warps shorter than 8 events): event by event
+            acc.raw |= v.x | v.y | v.z | v.w;
+            const uint32_t wv[4] = {v.x, v.y, v.z, v.w};
+#pragma unroll
+            for (int j = 0; j < 8; ++j) {
+              while (q + j >= nb) {
+                sg = next_nonempty(m.offs, sg, last);
+                col = colof(sg);
+                nb = m.offs[sg + 1];
+              }
+              acc.one(col, (j & 1) ? (wv[j >> 1] >> 16) : (wv[j >> 1] & 0xFFFFu));
+            }
+            while (q + 8 >= nb && sg < last) {  // move to the warp open after this word
+              sg = next_nonempty(m.offs, sg, last);
+              col = colof(sg);
+              nb = m.offs[sg + 1];
+            }
+            sgn = sg < last ? next_nonempty(m.offs, sg, last) : sg;
+            coln = colof(sgn);
+            nb2 = sgn != sg ? m.offs[sgn + 1] : ~0ull;
+            continue;
+          }
+          const uint32_t bo = nb < q + 8 ? (uint32_t)(nb - q) : 8u;  // first event of the next warp
+          acc.word(v, bo, col, coln);
+          if (bo < 8u) {  // crossed one boundary: the next warp is now current
+            sg = sgn;
+            col = coln;
+            nb = nb2;
+            sgn = sg < last ? next_nonempty(m.offs, sg, last) : sg;
+            coln = colof(sgn);
+            nb2 = sgn != sg ? m.offs[sgn + 1] : ~0ull;
+          }
         }
       }
-      raw |= acc.raw;
-      orr |= acc.orr;
       __syncthreads();  // accumulation done; the stage is free
       if (tid == 0) {   // stage the next chunk (this tile's next, or the next tile's first) during the combine
         ++pc.c;
-        if (pc.c >= pc.nch || pc.te <= pc.ts) {
-          do { cursor_tile(a, pc, pc.t + gridDim.x); } while (pc.valid && pc.te <= pc.ts);
+        if (pc.c >= pc.nch) {
+          do { cursor_tile(a, pc, pc.t + gridDim.x); } while (pc.valid && pc.nch == 0);
         }
         if (pc.valid) {
-          uint64_t ncs = pc.ts + pc.c * CAPE;
-          stage_chunk(a, m, ncs, umin64(ncs + CAPE, pc.te), E8);
+          uint64_t ncs = pc.A + pc.c * CAPE;
+          stage_chunk(a, m, ncs, umin64(ncs + CAPE, pc.Z), E8);
         }
       }
       // combine: warp tid (if it has events in this chunk) adds the HEAD partials of the threads it spilled into
       if (valid && e > s && e > cs && s < ce) {
         const uint64_t lo_e = umax64(s, cs), hi_e = umin64(e, ce) - 1;
-        const uint32_t ta = (uint32_t)(((lo_e - cs) * TPB + TPB - 1) / n);
-        const uint32_t tb = (uint32_t)(((hi_e - cs) * TPB + TPB - 1) / n);
-        const uint32_t from = ta + (s >= cs ? 1u : 0u);  // a warp starting in ta's range went straight into R
+        const uint32_t ta = (uint32_t)((((lo_e - cs) >> 3) * TPB + TPB - 1) / nwc);
+        const uint32_t tb = (uint32_t)((((hi_e - cs) >> 3) * TPB + TPB - 1) / nwc);
+        const uint32_t from = ta + (s >= cs ? 1u : 0u);  // a warp starting in ta's run went straight into R
         if (from <= tb) {
           uint32_t sum[16];
 #pragma unroll
           for (int j = 0; j < 16; ++j) sum[j] = 0u;
           for (uint32_t u = from; u <= tb; ++u) {
 #pragma unroll
-            for (int j = 0; j < 16; ++j) sum[j] += m.head[j * TPB + u];
+            for (int j = 0; j < 16; ++j) sum[j] += m.head[j * COLS + u];
           }
 #pragma unroll
-          for (int j = 0; j < 16; ++j) m.hist[j * TPB + tid] += sum[j];
+          for (int j = 0; j < 16; ++j) m.hist[j * COLS + tid] += sum[j];
         }
       }
       __syncthreads();  // HEAD columns consumed
 #pragma unroll
-      for (int j = 0; j < 16; ++j) m.head[j * TPB + tid] = 0u;
+      for (int j = 0; j < 16; ++j) headcol[j * COLS] = 0u;
     }
-    // tiles without events: keep the producer's cursor in step (it skipped them)
     // ---- finalise the tile ----
     uint32_t p[16];
     uint64_t I = 0;
 #pragma unroll
     for (int j = 0; j < 16; ++j) {
-      p[j] = m.hist[j * TPB + tid];
+      p[j] = m.hist[j * COLS + tid];
       I += p[j];
     }
-    // bad ids anywhere in the tile (event ranges != warps): every warp re-scans its own events (bad input only)
+    // bad ids anywhere in the tile (runs != warps): every warp re-scans its own events (bad input only)
+    const uint32_t raw = acc.raw, orr = acc.orr;
     const int bad_here = ((((raw | (raw >> 16)) & 0xFFFFu) & ~bmask) != 0u || (CHECK_MARK && (orr & 1u))) ? 1 : 0;
     if (__syncthreads_or(bad_here) && valid) report_bad_event(a, s, e);
     uint32_t k = a.tile_k0 ? a.tile_k0[t] : 0u;
@@ -450,7 +494,7 @@ __global__ void __launch_bounds__(TPB, 2) k_bbv(BbvArgs a) {
       __syncthreads();
     }
 #pragma unroll
-    for (int j = 0; j < 16; ++j) m.hist[j * TPB + tid] = 0u;
+    for (int j = 0; j < 16; ++j) m.hist[j * COLS + tid] = 0u;
     my_off = nx_off;
     last_off = nx_last;
     t = tn;
@@ -481,7 +525,7 @@ __global__ void __launch_bounds__(TPB) k_group_from_bbv(BbvArgs a, const uint32_
     for (int j = 0; j < 16; ++j) p[j] = 0u;
   }
 #pragma unroll
-  for (int j = 0; j < 16; ++j) m.hist[j * TPB + tid] = p[j];
+  for (int j = 0; j < 16; ++j) m.hist[j * COLS + tid] = p[j];
   uint32_t k = a.tile_k0[t];
   if (valid)
     while (k + 1 < a.K && a.kwo[k + 1] <= w) ++k;
@@ -503,7 +547,7 @@ __global__ void k_table_prep(const uint32_t* __restrict__ bb_len, const uint8_t*
     len = 0;
     bin = 0;
   }
-  tbl[b] = (len << 14) | (bin << 10);
+  tbl[b] = (len << 14) | (bin * (uint32_t)COLB);
   atomicMax(max_len, len);
 }
 
