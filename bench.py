@@ -242,6 +242,9 @@ def run_photon(args):
 
     sections = {PROF_SECTIONS[i]: {"ms_per_step": pms[i] / args.steps, "launches": int(pcnt[i])}
                 for i in range(len(PROF_SECTIONS)) if pcnt[i]}
+    if ws == 1:
+        sections["match_stats"] = ph.match_stats(g.n_kernels, res, {"_ws": res["_mws"]})
+        sections["types"] = ph.photon_types_total(res, g.n_kernels)
     hbm_peak, peak_src = _peaks()
     k1_ms = pms[0] / max(int(pcnt[0]), 1)
     k1_bytes = 2 * tr.n_events + 8 * (tr.n_warps + 1) + 4 * tr.n_warps  # algorithmic: bb + offsets + warp type

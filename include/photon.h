@@ -173,6 +173,10 @@ PHOTON_API int photon_match_scan(photon_ctx *ctx, uint32_t n_kernels, const uint
                       const uint64_t *mass, const uint64_t *warps_total, photon_match_params params, uint32_t k_lo,
                       uint32_t k_hi, void *ws, size_t ws_bytes, uint64_t *pairs, uint64_t pair_capacity,
                       uint64_t *n_pairs, void *stream);
+/* Diagnostics of the most recent photon_kernel_match on `ws` (K and T as passed there; SYNCS): stats[0] = pairs
+ * that passed the conservative fp32 filter, [1] = close pairs (exact), [2] = resolution rounds, [3] = pair capacity. */
+PHOTON_API int photon_match_stats(photon_ctx *ctx, uint32_t n_kernels, uint64_t total_types_bound, const void *ws,
+                                  size_t ws_bytes, uint64_t *stats /*[4] HOST*/, void *stream);
 PHOTON_API int photon_match_resolve(photon_ctx *ctx, uint32_t n_kernels, const uint64_t *kernel_type_off, const uint64_t *sig,
                          const uint64_t *mass, const uint64_t *warps_total, photon_match_params params,
                          const uint64_t *pairs, uint64_t n_pairs, void *ws, size_t ws_bytes, int64_t *match,

@@ -76,6 +76,7 @@ _SIGS = [
     ("photon_match_workspace_bytes", c_size_t, [c_uint32, c_uint64, c_uint64]),
     ("photon_kernel_match", c_int, [c_void_p, c_uint32, POINTER(Types), c_void_p, MatchParams, c_void_p, c_size_t,
                                     c_void_p, c_void_p, c_void_p]),
+    ("photon_match_stats", c_int, [c_void_p, c_uint32, c_uint64, c_void_p, c_size_t, POINTER(c_uint64), c_void_p]),
     ("photon_sig_build", c_int, [c_void_p, c_uint32, c_void_p, c_void_p, c_void_p, c_uint32, c_uint32, c_void_p,
                                  c_void_p, c_void_p, c_size_t, c_void_p]),
     ("photon_match_scan", c_int, [c_void_p, c_uint32, c_void_p, c_void_p, c_void_p, c_void_p, MatchParams, c_uint32,

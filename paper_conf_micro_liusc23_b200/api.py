@@ -262,6 +262,13 @@ class Photon:
             return o
         raise PhotonError(_lib.ECAPACITY, "pair table kept overflowing")
 
+    def match_stats(self, n_kernels: int, ty: dict, m: dict, stream=None) -> dict:
+        st = (ctypes.c_uint64 * 4)()
+        ws = m["_ws"]
+        self._rc(self.L.photon_match_stats(self.ctx, n_kernels, ty["capacity"], ws.data_ptr(), ws.numel(), st,
+                                           self.stream_ptr(stream)))
+        return dict(filter_pairs=int(st[0]), close_pairs=int(st[1]), rounds=int(st[2]), pair_capacity=int(st[3]))
+
     # split form (multi-GPU driver)
     def photon_sig_build(self, K, kto, type_key, type_count, k_lo, k_hi, sig, mass, stream=None):
         ws = self.workspace("sig", 256)

@@ -211,6 +211,7 @@ MatchLayout match_layout(uint32_t K, uint64_t T, uint64_t pair_cap, void* base) 
   m.mw.cand_cur = c.take<uint32_t>(K + 1);
   m.mw.cand = c.take<uint32_t>(pair_cap);
   m.mw.state = c.take<uint8_t>(K + 1);
+  m.mw.ulist = c.take<uint32_t>(2ull * K + 2);
   m.mw.flag = c.take<uint32_t>(4);
   m.mw.pair_cap = pair_cap;
   m.pairs = c.take<uint64_t>(pair_cap);
@@ -483,6 +484,23 @@ int photon_kernel_match(photon_ctx* ctx, uint32_t K, const photon_types* types, 
                             m.n_pairs, m.mw, match, match_dist, m.err, s),
        "resolve");
   }
+  return PHOTON_OK;
+}
+
+int photon_match_stats(photon_ctx* ctx, uint32_t K, uint64_t T, const void* ws, size_t ws_bytes, uint64_t* stats,
+                       void* stream) {
+  if (!ctx || !ws || !stats) return PHOTON_EINVAL;
+  MatchLayout m = match_layout_fit(K, T, (void*)ws, ws_bytes);
+  CK(cudaStreamSynchronize((cudaStream_t)stream), "sync");
+  uint64_t nm = 0, np = 0;
+  uint32_t rounds = 0;
+  CK(cudaMemcpy(&nm, m.mw.n_maybe, 8, cudaMemcpyDeviceToHost), "stats");
+  CK(cudaMemcpy(&np, m.n_pairs, 8, cudaMemcpyDeviceToHost), "stats");
+  CK(cudaMemcpy(&rounds, m.mw.flag, 4, cudaMemcpyDeviceToHost), "stats");
+  stats[0] = nm;
+  stats[1] = np;
+  stats[2] = rounds;
+  stats[3] = m.mw.pair_cap;
   return PHOTON_OK;
 }
 

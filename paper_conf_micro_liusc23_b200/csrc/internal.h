@@ -96,6 +96,7 @@ struct MatchWs {
   uint32_t* cand_cur;  // [K]
   uint32_t* cand;      // [pair_cap] r per (k, r), grouped by k
   uint8_t* state;      // [K] 0 undecided, 1 representative, 2 matched
+  uint32_t* ulist;     // [2K] undecided-kernel lists (resolution rounds)
   uint32_t* flag;      // [4]
   uint64_t pair_cap;
 };

@@ -275,7 +275,7 @@ __device__ __forceinline__ void cursor_tile(const BbvArgs& a, Cursor& u, uint64_
   u.A = u.Z = 0;
   if (!u.valid) return;
   uint64_t w0 = t * TPB, w1 = umin64(a.W, w0 + TPB);
-  uint64_t ts = a.weo[w0], te = a.weo[w1];
+  uint64_t te = umin64(a.weo[w1], a.E), ts = umin64(a.weo[w0], te);  // clamped: bad offsets stay memory-safe
   if (te <= ts) return;
   u.A = ts & ~7ull;
   u.Z = (te + 7) & ~7ull;
@@ -347,7 +347,8 @@ __global__ void __launch_bounds__(TPB, 2) k_bbv(BbvArgs a) {
       if (tid == 0) nx_last = a.weo[n0 + nn];
     }
     __syncthreads();
-    const uint64_t ts = m.offs[1], te = m.offs[1 + nw];
+    // same clamping as cursor_tile (monotone offsets are validated per warp below: e < s latches ERANGE)
+    const uint64_t te = umin64(m.offs[1 + nw], a.E), ts = umin64(m.offs[1], te);
     const uint64_t At = ts & ~7ull, Zt = (te + 7) & ~7ull;
     if (tid == 0) {
       m.offs[0] = At;
@@ -464,14 +465,14 @@ __global__ void __launch_bounds__(TPB, 2) k_bbv(BbvArgs a) {
     // bad ids anywhere in the tile (runs != warps): every warp re-scans its own events (bad input only)
     const uint32_t raw = acc.raw, orr = acc.orr;
     const int bad_here = ((((raw | (raw >> 16)) & 0xFFFFu) & ~bmask) != 0u || (CHECK_MARK && (orr & 1u))) ? 1 : 0;
-    if (__syncthreads_or(bad_here) && valid) report_bad_event(a, s, e);
+    if (__syncthreads_or(bad_here) && valid) report_bad_event(a, umin64(s, a.E), umin64(e, a.E));
     uint32_t k = a.tile_k0 ? a.tile_k0[t] : 0u;
     if (valid) {
       if (e < s) latch(a.err, PHOTON_ERANGE, (int64_t)w);
       if (e > s && (uint64_t)(e - s) * max_len >= kInstsLimit) {
         // bins may have wrapped: recompute the exact total (rare, long warps only)
         uint64_t exact = 0;
-        for (uint64_t i = s; i < e; ++i) exact += a.tbl[a.bb[i] & bmask] >> 14;
+        for (uint64_t i = s; i < umin64(e, a.E); ++i) exact += a.tbl[a.bb[i] & bmask] >> 14;
         I = exact;
       }
       if (I >= kInstsLimit) latch(a.err, PHOTON_ERANGE, (int64_t)w);
@@ -677,7 +678,6 @@ cudaError_t launch_table_prep(const TraceDev& t, uint32_t* tbl, uint32_t* max_le
 cudaError_t launch_validate_offsets(const TraceDev& t, DevErr* err, cudaStream_t s) {
   uint64_t n = t.K > 0 ? t.K : 1;
   note_launch(), k_validate_offsets<<<(unsigned)ceil_div(n, 256), 256, 0, s>>>(t.kwo, t.K, t.weo, t.W, t.E, err);
-  if (t.W) note_launch(), k_validate_weo<<<(unsigned)ceil_div(t.W, 256), 256, 0, s>>>(t.weo, t.W, err);
   return cudaGetLastError();
 }
 

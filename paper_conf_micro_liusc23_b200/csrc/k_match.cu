@@ -239,31 +239,68 @@ __global__ void k_cand_scatter(const uint64_t* pairs, uint64_t n_host, const uin
 
 // Fixed point of the launch-order rule: state 1 = representative, 2 = matched.  k decides once all its candidate
 // predecessors have decided (or one of them is a representative).  One CTA; monotone state (races benign).
+// Each kernel keeps a cursor into its candidate list: entries before it are decided non-representatives, so every
+// candidate is examined O(1) times plus once per round it blocks.  State lives in shared memory when K fits.
+template <bool SMEM>
 __global__ void __launch_bounds__(1024) k_resolve_states(uint32_t K, const uint64_t* off, const uint32_t* cand,
-                                                         uint8_t* state, uint32_t pool_all) {
-  for (uint32_t k = threadIdx.x; k < K; k += blockDim.x) state[k] = 0;
+                                                         uint8_t* state, uint32_t* cursor, uint32_t* ulist,
+                                                         uint32_t* flag, uint32_t pool_all) {
+  extern __shared__ uint8_t sstate[];
+  uint8_t* st = SMEM ? sstate : state;
+  for (uint32_t k = threadIdx.x; k < K; k += blockDim.x) {
+    st[k] = 0;
+    cursor[k] = 0;
+  }
   __syncthreads();
   if (pool_all) {
     for (uint32_t k = threadIdx.x; k < K; k += blockDim.x) state[k] = off[k + 1] > off[k] ? 2 : 1;
+    if (threadIdx.x == 0) flag[0] = 1;
     return;
   }
-  volatile uint8_t* vs = state;
+  volatile uint8_t* vs = st;
+  __shared__ uint32_t n_next;
+  uint32_t rounds = 0;
+  uint32_t n = K;           // round 1 visits every kernel; later rounds only the undecided list
+  uint32_t* cur = nullptr;  // current list (nullptr = identity)
+  uint32_t* nxt = ulist;
   for (;;) {
-    int undecided = 0;
-    for (uint32_t k = threadIdx.x; k < K; k += blockDim.x) {
-      if (vs[k] != 0) continue;
-      bool any_rep = false, all_dec = true;
-      for (uint64_t i = off[k]; i < off[k + 1]; ++i) {
-        uint8_t s = vs[cand[i]];
-        if (s == 1) { any_rep = true; break; }
-        if (s == 0) all_dec = false;
+    ++rounds;
+    if (threadIdx.x == 0) n_next = 0;
+    __syncthreads();
+    for (uint32_t q = threadIdx.x; q < n; q += blockDim.x) {
+      const uint32_t k = cur ? cur[q] : q;
+      const uint64_t o0 = off[k], o1 = off[k + 1];
+      uint64_t first_undec = o1;
+      uint8_t res = 1;  // representative unless a candidate is one
+      // batches of 8 independent candidate loads (memory-level parallelism), then their states
+      for (uint64_t i0 = o0 + cursor[k]; i0 < o1 && res == 1; i0 += 8) {
+        uint32_t c8[8];
+#pragma unroll
+        for (int u = 0; u < 8; ++u) c8[u] = (i0 + u < o1) ? cand[i0 + u] : UINT32_MAX;
+#pragma unroll
+        for (int u = 0; u < 8; ++u) {
+          if (c8[u] == UINT32_MAX) break;
+          uint8_t s = vs[c8[u]];
+          if (s == 1) { res = 2; break; }
+          if (s == 0 && first_undec == o1) first_undec = i0 + u;
+        }
       }
-      if (any_rep) vs[k] = 2;
-      else if (all_dec) vs[k] = 1;
-      else undecided = 1;
+      if (res == 1 && first_undec < o1) {  // blocked by an undecided predecessor: resume there next round
+        cursor[k] = (uint32_t)(first_undec - o0);
+        nxt[atomicAdd(&n_next, 1u)] = k;
+      } else {
+        vs[k] = res;
+      }
     }
-    if (!__syncthreads_or(undecided)) break;
+    __syncthreads();
+    n = n_next;
+    if (n == 0) break;
+    cur = nxt;  // ping-pong between the two halves of ulist
+    nxt = (cur == ulist) ? ulist + K : ulist;
   }
+  if (SMEM)
+    for (uint32_t k = threadIdx.x; k < K; k += blockDim.x) state[k] = st[k];
+  if (threadIdx.x == 0) flag[0] = rounds;
 }
 
 // match[k] = argmin over eligible candidates of (|W_k - W_r|, r); match_dist exact -> fp64 (one warp per kernel)
@@ -355,7 +392,14 @@ cudaError_t launch_match_resolve(uint32_t K, const uint64_t* kto, const uint64_t
     note_launch(), k_cand_scatter<<<(unsigned)ceil_div(n_pairs, 256), 256, 0, s>>>(pairs, n_pairs, n_pairs_dev, K, mw.cand_off,
                                                                     mw.cand_cur, mw.cand);
   }
-  note_launch(), k_resolve_states<<<1, 1024, 0, s>>>(K, mw.cand_off, mw.cand, mw.state, p.pool_all_prior);
+  if (K <= 40960) {
+    cudaFuncSetAttribute(k_resolve_states<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, 40960);
+    note_launch(), k_resolve_states<true><<<1, 1024, K, s>>>(K, mw.cand_off, mw.cand, mw.state, mw.cand_cur, mw.ulist,
+                                                              mw.flag, p.pool_all_prior);
+  } else {
+    note_launch(), k_resolve_states<false><<<1, 1024, 0, s>>>(K, mw.cand_off, mw.cand, mw.state, mw.cand_cur,
+                                                               mw.ulist, mw.flag, p.pool_all_prior);
+  }
   note_launch(), k_resolve_match<<<(unsigned)ceil_div((uint64_t)K * 32, 256), 256, 0, s>>>(K, mw.cand_off, mw.cand, mw.state,
                                                                            p.pool_all_prior, wt, kto, sig, mass,
                                                                            match, match_dist);

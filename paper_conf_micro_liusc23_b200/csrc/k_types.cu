@@ -15,6 +15,7 @@ namespace photon {
 namespace {
 
 constexpr int SORT_SMEM_MAX = 4096;
+constexpr uint32_t WARP_SORT_MAX = 128;
 
 __global__ void k_ht_clear(HashTable ht) {
   uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
@@ -122,10 +123,66 @@ __global__ void __launch_bounds__(256) k_sort_warp(HashTable ht, uint32_t K, con
                                                    const uint32_t* list, const uint64_t* kwo,
                                                    const uint64_t* kernel_warps, photon_types out, uint32_t* canon,
                                                    uint32_t* big, uint32_t* nbig) {
-  const uint32_t lane = threadIdx.x & 31;
+  const uint32_t lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
   const uint32_t k = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   if (k >= K) return;
   const uint64_t off = kto[k], n = kto[k + 1] - off;
+  const uint64_t Wk = kernel_warps ? kernel_warps[k] : (kwo[k + 1] - kwo[k]);
+  if (n > 32 && n <= WARP_SORT_MAX) {
+    // 32 < T_k <= 128: warp-private shared-memory bitonic sort; count and key words 0-3 staged in shared memory
+    __shared__ uint32_t s_slot[8][WARP_SORT_MAX], s_cnt[8][WARP_SORT_MAX];
+    __shared__ uint4 s_k0[8][WARP_SORT_MAX];
+    __shared__ uint16_t s_idx[8][WARP_SORT_MAX];
+    uint32_t P = 64;
+    while (P < n) P <<= 1;
+    for (uint32_t i = lane; i < P; i += 32) {
+      s_idx[wib][i] = (uint16_t)i;
+      if (i < n) {
+        uint32_t sl = list[off + i];
+        s_slot[wib][i] = sl;
+        s_cnt[wib][i] = ht.count[sl];
+        s_k0[wib][i] = *(const uint4*)(ht.key + (uint64_t)sl * 16);
+      }
+    }
+    __syncwarp();
+    auto before = [&](uint32_t a, uint32_t b) -> bool {  // element a before element b (padding last)
+      if (b >= n) return a < n;
+      if (a >= n) return false;
+      uint32_t ca = s_cnt[wib][a], cb = s_cnt[wib][b];
+      if (ca != cb) return ca > cb;
+      uint4 ka = s_k0[wib][a], kb = s_k0[wib][b];
+      if (ka.x != kb.x) return ka.x < kb.x;
+      if (ka.y != kb.y) return ka.y < kb.y;
+      if (ka.z != kb.z) return ka.z < kb.z;
+      if (ka.w != kb.w) return ka.w < kb.w;
+      return type_before(ht, s_slot[wib][a], s_slot[wib][b]);  // words 4.. (rare)
+    };
+    for (uint32_t size = 2; size <= P; size <<= 1) {
+      for (uint32_t stride = size >> 1; stride > 0; stride >>= 1) {
+        for (uint32_t t = lane; t < P / 2; t += 32) {
+          uint32_t i = 2 * stride * (t / stride) + (t % stride), j = i + stride;
+          bool up = ((i & size) == 0);
+          uint32_t a = s_idx[wib][i], b = s_idx[wib][j];
+          if (up ? before(b, a) : before(a, b)) { s_idx[wib][i] = (uint16_t)b; s_idx[wib][j] = (uint16_t)a; }
+        }
+        __syncwarp();
+      }
+    }
+    for (uint32_t r = lane; r < n && off + r < out.capacity; r += 32) {
+      uint32_t sl = s_slot[wib][s_idx[wib][r]];
+      const uint4* src = (const uint4*)(ht.key + (uint64_t)sl * 16);
+      uint4* dst = (uint4*)(out.type_key + (off + r) * 16);
+      dst[0] = src[0]; dst[1] = src[1]; dst[2] = src[2]; dst[3] = src[3];
+      out.type_count[off + r] = ht.count[sl];
+      out.type_first_warp[off + r] = ht.first[sl];
+      canon[sl] = r;
+    }
+    if (lane == 0) {
+      uint64_t c0 = s_cnt[wib][s_idx[wib][0]];
+      out.warp_sampling_ok[k] = (Wk > 0 && 100ull * c0 > 95ull * Wk) ? 1 : 0;  // L249 [P-15]
+    }
+    return;
+  }
   if (n > 32) {
     if (lane == 0) {
       if (n <= SORT_SMEM_MAX) big[atomicAdd(&nbig[0], 1u)] = k;
@@ -133,7 +190,6 @@ __global__ void __launch_bounds__(256) k_sort_warp(HashTable ht, uint32_t K, con
     }
     return;
   }
-  const uint64_t Wk = kernel_warps ? kernel_warps[k] : (kwo[k + 1] - kwo[k]);
   uint32_t mine = lane < n ? list[off + lane] : UINT32_MAX;
   for (uint32_t size = 2; size <= 32; size <<= 1) {
     for (uint32_t stride = size >> 1; stride > 0; stride >>= 1) {
@@ -235,11 +291,21 @@ __global__ void k_entries_insert(TileEntries te, uint64_t n_tiles, HashTable ht,
     x = te.ent + i;
     out = te.tile_slot + i;
   } else {
-    uint64_t j = i - nfix;
-    uint64_t n = *te.ovf_count;
-    if (j >= n || j >= te.ovf_cap) return;
-    x = te.ovf + j;
-    out = te.ovf_slot + j;
+    // overflow entries (tiles with more than per_tile distinct keys): grid-stride over the device count
+    const uint64_t n = umin64(*te.ovf_count, te.ovf_cap);
+    const uint64_t stride = (uint64_t)gridDim.x * blockDim.x - nfix;
+    for (uint64_t j = i - nfix; j < n; j += stride) {
+      x = te.ovf + j;
+      uint32_t key[16];
+      const uint4* kp = (const uint4*)x->key;
+#pragma unroll
+      for (int q = 0; q < 4; ++q) {
+        uint4 v = kp[q];
+        key[4 * q] = v.x; key[4 * q + 1] = v.y; key[4 * q + 2] = v.z; key[4 * q + 3] = v.w;
+      }
+      te.ovf_slot[j] = ht_insert(ht, err, x->kernel, key, x->hash, x->count, x->first);
+    }
+    return;
   }
   uint32_t key[16];
   const uint4* kp = (const uint4*)x->key;
@@ -361,7 +427,8 @@ cudaError_t launch_canonicalise(const HashTable& ht, uint32_t K, const uint64_t*
 
 cudaError_t launch_entries_insert(const TileEntries& te, uint64_t n_tiles, const HashTable& ht, DevErr* err,
                                   cudaStream_t s) {
-  uint64_t n = n_tiles * te.per_tile + te.ovf_cap;
+  // fixed entry slots one thread each (rounded up to whole CTAs), then 64K threads striding over the overflow
+  uint64_t n = ceil_div(n_tiles * te.per_tile, 256) * 256 + 65536;
   if (n == 0) return cudaSuccess;
   note_launch(), k_entries_insert<<<(unsigned)ceil_div(n, 256), 256, 0, s>>>(te, n_tiles, ht, err);
   return cudaGetLastError();
