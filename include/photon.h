@@ -95,7 +95,7 @@ typedef struct {
   const uint64_t *kernel_warp_off; /* [K+1] non-decreasing, [0]=0, [K]=W: kernel k owns warps [off[k],off[k+1])    */
   const uint64_t *warp_event_off;  /* [W+1] non-decreasing, [0]=0, [W]=E: warp w owns events [off[w],off[w+1])     */
   const uint16_t *bb;              /* [E] BB id per event, execution order within a warp; 16-byte aligned          */
-  const uint32_t *bb_len;          /* [B] instructions per BB, 1 <= len < 2^18                                     */
+  const uint32_t *bb_len;          /* [B] instructions per BB, 1 <= len < 2^17                                    */
   const uint8_t *bb_bin;           /* [B] projection bin (< 16) of each BB [P-2]; NULL => bin(b) = b & 15          */
 } photon_trace;
 

@@ -26,7 +26,7 @@ typedef __int128 i128;
 constexpr uint64_t kTimeLimit = 1ull << 40;  // [P-16] ticks < 2^40
 constexpr uint64_t kMassLimit = 1ull << 50;  // N_k < 2^50 (u128 cross products stay exact)
 constexpr uint64_t kInstsLimit = 1ull << 32; // per-warp instructions < 2^32 (u32 bins)
-constexpr uint32_t kMaxLen = (1u << 18) - 1; // bb_len < 2^18 (packed table entry)
+constexpr uint32_t kMaxLen = (1u << 17) - 1; // bb_len < 2^17 (packed table entry)
 
 // ---- device error latch: first error wins (code, index) -----------------------------------------------------
 struct DevErr {
@@ -73,14 +73,15 @@ __device__ __forceinline__ uint64_t mix64(uint64_t x) {
   x ^= x >> 33;
   return x;
 }
+// Bucketing hash only (equality is always verified on the full key): a sum of 32x32->64-bit products with distinct
+// odd multipliers (one IMAD.WIDE each) followed by a 64-bit finaliser.
 __device__ __forceinline__ uint64_t hash_key(uint32_t k, const uint32_t* p) {
-  uint64_t h = 0x9E3779B97F4A7C15ull ^ ((uint64_t)k * 0xC2B2AE3D27D4EB4Full);
+  constexpr uint32_t M[17] = {0x9E3779B1u, 0x85EBCA77u, 0xC2B2AE3Du, 0x27D4EB2Fu, 0x165667B1u, 0xD3A2646Du,
+                              0xFD7046C5u, 0xB55A4F09u, 0x7FEB352Du, 0x846CA68Bu, 0xE6546B65u, 0x4CF5AD43u,
+                              0x2545F491u, 0x9E485565u, 0xEF1D6B47u, 0x5851F42Du, 0x14057B7Fu};
+  uint64_t h = (uint64_t)k * M[16] + 0x632BE59BD9B4E019ull;
 #pragma unroll
-  for (int j = 0; j < 16; j += 2) {
-    uint64_t v = (uint64_t)p[j] | ((uint64_t)p[j + 1] << 32);
-    h = (h ^ v) * 0x100000001B3ull;
-    h ^= h >> 29;
-  }
+  for (int j = 0; j < 16; ++j) h += (uint64_t)p[j] * M[j] + ((uint64_t)p[j] << (2 * j + 13));
   h = mix64(h);
   return h ? h : 1;
 }

@@ -29,13 +29,16 @@ namespace photon {
 namespace {
 
 constexpr int TPB = 256;            // threads per CTA = warps per tile
-constexpr int COLS = 264;           // column stride (u32) of the 16 x COLS result / HEAD arrays
-constexpr int COLB = COLS * 4;      // bin stride in bytes; table entry = len << 14 | bin * COLB
+constexpr int COLS = 288;           // column stride (u32) of the 16 x COLS arrays: a multiple of 32 banks, so a
+                                    // cell's bank is its column's (lanes on distinct columns never conflict)
+constexpr int COLB = COLS * 4;      // bin stride in bytes; table entry = len << LSH | bin * COLB
+constexpr int LSH = 15;             // length field shift (lengths < 2^17)
+constexpr uint32_t AMASK = 0x7FFCu; // cell byte offset bits of a table entry
 constexpr int DUMMY = 256;          // scratch column (events of neighbouring tiles)
 constexpr int CAPE = 24576;         // staging chunk (events, multiple of 8), 48 KB
 constexpr int SMEM_TBL_MAX = 4096;  // BB table entries kept in shared memory
 constexpr int LSLOTS = 256;         // CTA-local de-dup slots
-static_assert(15 * COLB < (1 << 14), "bin offset must fit below the length field");
+static_assert(15 * COLB < (1 << LSH) && (COLS % 32) == 0, "bin offset must fit below the length field");
 
 struct BbvArgs {
   const uint64_t* kwo;
@@ -58,7 +61,7 @@ constexpr size_t kStageBytes = (size_t)CAPE * 2;
 constexpr size_t kOffsBytes = (TPB + 4) * 8;
 constexpr size_t kLocalBytes = LSLOTS * (8 + 4 + 4 + 4 + 4);
 constexpr size_t kMiscBytes = 256;
-constexpr size_t kKidBytes = TPB * 4;
+constexpr size_t kKidBytes = TPB * 4 + (TPB + 8) * 2;
 
 __host__ __device__ constexpr size_t bbv_smem_bytes(uint32_t tbl_entries) {
   return 2 * kColBytes + kStageBytes + kOffsBytes + 16 + kLocalBytes + kMiscBytes + kKidBytes +
@@ -78,6 +81,7 @@ struct Smem {
   uint32_t* lent;    // [LSLOTS] dense local entry id
   uint32_t* misc;    // [64]: 0 n_entries; [2..3] u64 overflow base
   uint32_t* kid;     // [TPB] kernel of each thread's warp
+  uint16_t* nxt;     // [TPB+8] next non-empty warp after each (virtual) warp of the tile
   uint32_t* tbl;     // [P2]
 };
 
@@ -95,12 +99,13 @@ __device__ __forceinline__ Smem carve(uint8_t* s) {
   m.lent = m.lminw + LSLOTS;
   m.misc = m.lent + LSLOTS;
   m.kid = m.misc + kMiscBytes / 4;
-  m.tbl = m.kid + TPB;
+  m.nxt = (uint16_t*)(m.kid + TPB);
+  m.tbl = (uint32_t*)(m.nxt + TPB + 8);
   return m;
 }
 
 // ---- per-event accumulation --------------------------------------------------------------------------------
-// Table entry t: len << 14 | bin * COLB (bit 0 = id in [B, P2)); cell address = column + (t & 0x3FFC).
+// Table entry t: len << LSH | bin * COLB (bit 0 = id in [B, P2)); cell address = column + (t & AMASK).
 struct Acc {
   const uint32_t* tbl;
   uint32_t bmask;
@@ -108,26 +113,32 @@ struct Acc {
   __device__ __forceinline__ void one(uint32_t* col, uint32_t b) {
     uint32_t t = tbl[b & bmask];
     orr |= t;
-    *(uint32_t*)((uint8_t*)col + (t & 0x3FFCu)) += t >> 14;
+    *(uint32_t*)((uint8_t*)col + (t & AMASK)) += t >> LSH;
   }
-  // two events into columns c0 / c1: both cells read before either is written (equal cells merged)
-  __device__ __forceinline__ void two(uint32_t w, uint32_t* c0, uint32_t* c1) {
-    uint32_t t0 = tbl[w & bmask], t1 = tbl[(w >> 16) & bmask];
-    orr |= t0 | t1;
-    uint32_t* p0 = (uint32_t*)((uint8_t*)c0 + (t0 & 0x3FFCu));
-    uint32_t* p1 = (uint32_t*)((uint8_t*)c1 + (t1 & 0x3FFCu));
-    uint32_t l0 = t0 >> 14, l1 = t1 >> 14;
+  // two events whose table entries are already loaded; `same` = both go to the same column
+  __device__ __forceinline__ void pair(uint32_t t0, uint32_t t1, uint32_t* c0, uint32_t* c1, bool same) {
+    const uint32_t a0 = t0 & AMASK, a1 = t1 & AMASK;
+    uint32_t* p0 = (uint32_t*)((uint8_t*)c0 + a0);
+    uint32_t* p1 = (uint32_t*)((uint8_t*)c1 + a1);
+    const uint32_t l1 = t1 >> LSH;
     uint32_t h0 = *p0, h1 = *p1;
     *p1 = h1 + l1;
-    *p0 = h0 + l0 + (p0 == p1 ? l1 : 0u);
+    *p0 = h0 + (t0 >> LSH) + ((same && a0 == a1) ? l1 : 0u);
   }
-  // one 16-byte word: events j < bo into ca, j >= bo into cb
+  // one 16-byte word: events j < bo into ca, j >= bo into cb.  All 8 table entries are loaded before any
+  // histogram cell is written (the compiler cannot hoist them past the stores itself), so the word costs four
+  // short load->add->store chains instead of four chains that each also wait for their table reads.
   __device__ __forceinline__ void word(uint4 v, uint32_t bo, uint32_t* ca, uint32_t* cb) {
     raw |= v.x | v.y | v.z | v.w;
-    two(v.x, bo > 0 ? ca : cb, bo > 1 ? ca : cb);
-    two(v.y, bo > 2 ? ca : cb, bo > 3 ? ca : cb);
-    two(v.z, bo > 4 ? ca : cb, bo > 5 ? ca : cb);
-    two(v.w, bo > 6 ? ca : cb, bo > 7 ? ca : cb);
+    const uint32_t t0 = tbl[v.x & bmask], t1 = tbl[(v.x >> 16) & bmask];
+    const uint32_t t2 = tbl[v.y & bmask], t3 = tbl[(v.y >> 16) & bmask];
+    const uint32_t t4 = tbl[v.z & bmask], t5 = tbl[(v.z >> 16) & bmask];
+    const uint32_t t6 = tbl[v.w & bmask], t7 = tbl[(v.w >> 16) & bmask];
+    orr |= (t0 | t1 | t2 | t3) | (t4 | t5 | t6 | t7);
+    pair(t0, t1, bo > 0 ? ca : cb, bo > 1 ? ca : cb, bo != 1);
+    pair(t2, t3, bo > 2 ? ca : cb, bo > 3 ? ca : cb, bo != 3);
+    pair(t4, t5, bo > 4 ? ca : cb, bo > 5 ? ca : cb, bo != 5);
+    pair(t6, t7, bo > 6 ? ca : cb, bo > 7 ? ca : cb, bo != 7);
   }
 };
 
@@ -282,11 +293,6 @@ __device__ __forceinline__ void cursor_tile(const BbvArgs& a, Cursor& u, uint64_
   u.nch = ceil_div(u.Z - u.A, CAPE);
 }
 
-__device__ __forceinline__ uint32_t next_nonempty(const uint64_t* o, uint32_t s, uint32_t last) {
-  do { ++s; } while (s < last && o[s + 1] == o[s]);
-  return s;
-}
-
 template <bool SMEM_TBL, bool CHECK_MARK>
 __global__ void __launch_bounds__(TPB, 2) k_bbv(BbvArgs a) {
   extern __shared__ __align__(128) uint8_t smem_raw[];
@@ -357,6 +363,15 @@ __global__ void __launch_bounds__(TPB, 2) k_bbv(BbvArgs a) {
     const uint64_t s = valid ? m.offs[1 + tid] : te, e = valid ? m.offs[2 + tid] : te;
     const uint64_t nch = te > ts ? ceil_div(Zt - At, CAPE) : 0;
     const uint32_t last = nw + 1;  // index of the virtual tail warp
+    {
+      // nxt[s'] = next non-empty (virtual) warp after s' (last = sentinel); o[0] / o[nw+2] taken from registers
+      auto O = [&](uint32_t i) -> uint64_t { return i == 0 ? At : (i == nw + 2 ? Zt : m.offs[i]); };
+      for (uint32_t sp = tid; sp <= last; sp += TPB) {
+        uint32_t x = sp + 1;
+        while (x < last && O(x + 1) == O(x)) ++x;
+        m.nxt[sp] = (uint16_t)(x < last ? x : last);
+      }
+    }
     __syncthreads();
     uint32_t* const headcol = m.head + tid;
     uint32_t* const dummy = m.hist + DUMMY;
@@ -371,21 +386,36 @@ __global__ void __launch_bounds__(TPB, 2) k_bbv(BbvArgs a) {
       // my run of words [r0, r1) of the chunk
       const uint64_t r0 = cs + 8 * (((uint64_t)tid * nwc) / TPB), r1 = cs + 8 * (((uint64_t)(tid + 1) * nwc) / TPB);
       if (r0 < r1) {
-        // warp (with virtual ones) containing r0: last s' with o[s'] <= r0
+        // warp (with virtual ones) containing r0: last s' with o[s'] <= r0.  Start from the proportional guess
+        // and narrow a +-8 window around it when it brackets r0 (it usually does), else search everything.
         uint32_t lo = 0, hi = last;
+        {
+          const float fr = (float)(r0 - At) / (float)(Zt - At);
+          int g = (int)(fr * (float)(nw + 2));
+          int glo = g - 8 < 0 ? 0 : g - 8, ghi = g + 8 > (int)last ? (int)last : g + 8;
+          if (m.offs[glo] <= r0 && m.offs[ghi + 1] > r0) { lo = (uint32_t)glo; hi = (uint32_t)ghi; }
+        }
         while (lo < hi) {
           uint32_t mid = (lo + hi + 1) >> 1;
           if (m.offs[mid] <= r0) lo = mid; else hi = mid - 1;
         }
+        // all positions below are u32 offsets from the chunk start, clamped to [0, LIM]
+        const uint32_t LIM = (uint32_t)(ce - cs) + 8u;
+        auto rel = [&](uint64_t x) -> uint32_t {
+          return x <= cs ? 0u : (x - cs >= LIM ? LIM : (uint32_t)(x - cs));
+        };
         uint32_t sg = lo;
         uint32_t* col = (m.offs[sg] < r0) ? headcol : colof(sg);  // warp open at my run start -> HEAD
-        uint64_t nb = m.offs[sg + 1];
-        uint32_t sgn = sg < last ? next_nonempty(m.offs, sg, last) : sg;
+        uint32_t nb = rel(m.offs[sg + 1]);
+        uint32_t sgn = m.nxt[sg];
         uint32_t* coln = colof(sgn);
-        uint64_t nb2 = sgn != sg ? m.offs[sgn + 1] : ~0ull;
+        uint32_t nb2 = sgn != sg ? rel(m.offs[sgn + 1]) : LIM + 8u;
         const uint4* sb4 = (const uint4*)m.stage;
-        for (uint64_t q = r0; q < r1; q += 8) {
-          const uint4 v = sb4[(q - cs) >> 3];
+        const uint32_t q0 = (uint32_t)(r0 - cs), qe = (uint32_t)(r1 - cs);
+        uint4 vnext = sb4[q0 >> 3];
+        for (uint32_t q = q0; q < qe; q += 8) {
+          const uint4 v = vnext;
+          if (q + 8 < qe) vnext = sb4[(q + 8) >> 3];  // next word read before this word's stores
           if (nb2 < q + 8) {
             // several warp boundaries inside this word (warps shorter than 8 events): event by event
             acc.raw |= v.x | v.y | v.z | v.w;
@@ -393,32 +423,33 @@ __global__ void __launch_bounds__(TPB, 2) k_bbv(BbvArgs a) {
 #pragma unroll
             for (int j = 0; j < 8; ++j) {
               while (q + j >= nb) {
-                sg = next_nonempty(m.offs, sg, last);
+                sg = m.nxt[sg];
                 col = colof(sg);
-                nb = m.offs[sg + 1];
+                nb = rel(m.offs[sg + 1]);
               }
               acc.one(col, (j & 1) ? (wv[j >> 1] >> 16) : (wv[j >> 1] & 0xFFFFu));
             }
             while (q + 8 >= nb && sg < last) {  // move to the warp open after this word
-              sg = next_nonempty(m.offs, sg, last);
+              sg = m.nxt[sg];
               col = colof(sg);
-              nb = m.offs[sg + 1];
+              nb = rel(m.offs[sg + 1]);
             }
-            sgn = sg < last ? next_nonempty(m.offs, sg, last) : sg;
+            sgn = m.nxt[sg];
             coln = colof(sgn);
-            nb2 = sgn != sg ? m.offs[sgn + 1] : ~0ull;
+            nb2 = sgn != sg ? rel(m.offs[sgn + 1]) : LIM + 8u;
             continue;
           }
-          const uint32_t bo = nb < q + 8 ? (uint32_t)(nb - q) : 8u;  // first event of the next warp
+          const uint32_t bo = nb < q + 8 ? nb - q : 8u;  // first event of the next warp
           acc.word(v, bo, col, coln);
-          if (bo < 8u) {  // crossed one boundary: the next warp is now current
-            sg = sgn;
-            col = coln;
-            nb = nb2;
-            sgn = sg < last ? next_nonempty(m.offs, sg, last) : sg;
-            coln = colof(sgn);
-            nb2 = sgn != sg ? m.offs[sgn + 1] : ~0ull;
-          }
+          // advance past a crossed boundary without branching (lanes cross at different words; a divergent
+          // update would serialise): when bo == 8 the same values are recomputed
+          const bool cross = bo < 8u;
+          sg = cross ? sgn : sg;
+          col = cross ? coln : col;
+          nb = cross ? nb2 : nb;
+          sgn = m.nxt[sg];
+          coln = colof(sgn);
+          nb2 = sgn != sg ? rel(m.offs[sgn + 1]) : LIM + 8u;
         }
       }
       __syncthreads();  // accumulation done; the stage is free
@@ -472,7 +503,7 @@ __global__ void __launch_bounds__(TPB, 2) k_bbv(BbvArgs a) {
       if (e > s && (uint64_t)(e - s) * max_len >= kInstsLimit) {
         // bins may have wrapped: recompute the exact total (rare, long warps only)
         uint64_t exact = 0;
-        for (uint64_t i = s; i < umin64(e, a.E); ++i) exact += a.tbl[a.bb[i] & bmask] >> 14;
+        for (uint64_t i = s; i < umin64(e, a.E); ++i) exact += a.tbl[a.bb[i] & bmask] >> LSH;
         I = exact;
       }
       if (I >= kInstsLimit) latch(a.err, PHOTON_ERANGE, (int64_t)w);
@@ -548,7 +579,7 @@ __global__ void k_table_prep(const uint32_t* __restrict__ bb_len, const uint8_t*
     len = 0;
     bin = 0;
   }
-  tbl[b] = (len << 14) | (bin * (uint32_t)COLB);
+  tbl[b] = (len << LSH) | (bin * (uint32_t)COLB);
   atomicMax(max_len, len);
 }
 
@@ -572,12 +603,6 @@ __global__ void k_validate_offsets(const uint64_t* __restrict__ kwo, uint32_t K,
     if (weo[0] != 0 || weo[W] != E) latch(err, PHOTON_ERANGE, 0);
   }
   if (i < K && kwo[i + 1] < kwo[i]) latch(err, PHOTON_ERANGE, (int64_t)i);
-}
-
-// warp_event_off must be non-decreasing (the streaming kernel relies on it); one thread per warp
-__global__ void k_validate_weo(const uint64_t* __restrict__ weo, uint64_t W, DevErr* err) {
-  uint64_t w = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
-  if (w < W && weo[w + 1] < weo[w]) latch(err, PHOTON_ERANGE, (int64_t)w);
 }
 
 // ---- optional BB distribution kernel_bb_insts[k][b] (L208-210) ------------------------------------------------
@@ -609,12 +634,12 @@ __global__ void __launch_bounds__(256) k_kbb(const uint64_t* __restrict__ kwo, c
       __syncthreads();
       for (uint32_t b = threadIdx.x; b < B; b += blockDim.x)
         if (cnt[b])
-          atomicAdd((unsigned long long*)&kbb[(uint64_t)k * B + b], (unsigned long long)cnt[b] * (tbl[b] >> 14));
+          atomicAdd((unsigned long long*)&kbb[(uint64_t)k * B + b], (unsigned long long)cnt[b] * (tbl[b] >> LSH));
       __syncthreads();
     } else {
       for (uint64_t i = cs + threadIdx.x; i < ce; i += blockDim.x) {
         uint32_t b = bb[i];
-        if (b < B) atomicAdd((unsigned long long*)&kbb[(uint64_t)k * B + b], (unsigned long long)(tbl[b] >> 14));
+        if (b < B) atomicAdd((unsigned long long*)&kbb[(uint64_t)k * B + b], (unsigned long long)(tbl[b] >> LSH));
       }
     }
   }

@@ -323,7 +323,13 @@ __global__ void k_remap_entries(TileEntries te, uint64_t W, const uint32_t* cano
   if (w >= W) return;
   const uint64_t t = w >> 8;  // 256 warps per tile (k_bbv.cu TPB)
   const uint32_t e = te.lid[w];
-  uint32_t slot = e < te.per_tile ? te.tile_slot[t * te.per_tile + e] : te.ovf_slot[te.tile_ovf[t] + (e - te.per_tile)];
+  uint32_t slot;
+  if (e < te.per_tile) {
+    slot = te.tile_slot[t * te.per_tile + e];
+  } else {
+    const uint64_t j = te.tile_ovf[t] + (e - te.per_tile);  // beyond ovf_cap only after ECAPACITY was latched
+    slot = j < te.ovf_cap ? te.ovf_slot[j] : UINT32_MAX;
+  }
   warp_type[w] = slot == UINT32_MAX ? UINT32_MAX : canon[slot];
 }
 

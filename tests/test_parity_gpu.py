@@ -137,9 +137,9 @@ def test_errors(ph):
     with pytest.raises(PhotonError) as ei:
         ph.photon_warp_group(_dev(ph, tr))
     assert ei.value.code == -3
-    tr = tg.trace_from_warps([[[0] * 3]], bb_len=[(1 << 17) + 5])
-    tr.bb = np.array([0] * 40000, np.uint16)  # 40000 * (2^17+5) >= 2^32: per-warp instructions overflow
-    tr.warp_event_off = np.array([0, 40000], np.uint64)
+    tr = tg.trace_from_warps([[[0] * 3]], bb_len=[(1 << 16) + 5])
+    tr.bb = np.array([0] * 70000, np.uint16)  # 70000 * (2^16+5) >= 2^32: per-warp instructions overflow
+    tr.warp_event_off = np.array([0, 70000], np.uint64)
     with pytest.raises(PhotonError) as ei:
         ph.photon_bbv_build(_dev(ph, tr))
     assert ei.value.code == -3 and ei.value.index == 0
