@@ -199,7 +199,7 @@ PHOTON_API int photon_match_resolve(photon_ctx *ctx, uint32_t n_kernels, const u
  * Device errors: ERANGE (bb >= n_bb, retire < issue, retire decreasing within a kernel, time >= 2^40,
  * non-monotone kernel_rec_off; index = record or kernel). */
 typedef struct {
-  uint32_t n_kernels, n_bb;        /* K, B as in the trace                                                      */
+  uint32_t n_kernels, n_bb;        /* K, B as in the trace; K*B < 2^31 (batch kernels otherwise) -> else EINVAL */
   uint64_t n_records;              /* R (< 2^32)                                                                */
   const uint64_t *kernel_rec_off;  /* [K+1]                                                                     */
   const uint16_t *bb;              /* [R]                                                                       */

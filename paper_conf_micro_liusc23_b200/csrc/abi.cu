@@ -575,7 +575,8 @@ int photon_bb_stable(photon_ctx* ctx, const photon_timing* t, const uint64_t* kb
   if (!t || !t->kernel_rec_off || (t->n_records && (!t->bb || !t->issue || !t->retire)) || !kbb || !first_stable ||
       !switch_at || !ws)
     return fail(ctx, PHOTON_EINVAL, "NULL argument");
-  if (t->n_kernels == 0 || t->n_bb == 0 || t->n_bb > 65536 || t->n_records >= (1ull << 32))
+  if (t->n_kernels == 0 || t->n_bb == 0 || t->n_bb > 65536 || t->n_records >= (1ull << 32) ||
+      (uint64_t)t->n_kernels * t->n_bb >= (1ull << 31))
     return fail(ctx, PHOTON_EINVAL, "bad timing sizes");
   if (p.window_n == 0) { p.window_n = 2048; }
   if (p.delta_den == 0) { p.delta_num = 3; p.delta_den = 100; }

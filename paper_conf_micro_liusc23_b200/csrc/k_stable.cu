@@ -6,14 +6,18 @@
 // rate of stable basic blocks is larger than 95%).  Readings [P-11]..[P-18].
 //
 // Design:
-//   1. validate records and build composite keys (kernel << bbits | bb), one CTA per (kernel, 4096-record chunk);
-//   2. stable LSD radix sort of (key, record index), 8-bit digits: per-tile digit histograms -> device scan ->
-//      scatter with a stable in-tile rank (warp __match_any_sync + per-warp digit prefix);
-//   3. gather (issue, retire) into group order; find group heads; split every group with >= 2n executions into
-//      work items of 2048 positions;
-//   4. per work item (one CTA, 8 consecutive positions per thread): the window sums ending just before the item
-//      by a block reduction, per-thread deltas by a block scan, then each thread slides over its 8 positions and
-//      evaluates cond1/cond2 exactly in i128; the first passing position per group is an atomicMin;
+//   1-3. bring every group g = (b, k) (dense id b*K + k) together in retirement order, with (issue, retire):
+//      B <= 256: one pass -- one warp per (kernel, 2048-record) job histograms its bb ids, a bin-major scan of
+//      the histograms gives every (bb, job) its output offset, and the warp scatters its records stably
+//      (__match_any_sync rank + warp-private running counts), validating them on the way;
+//      B > 256: composite keys b*K + k, stable LSD radix sort (8-bit digits, per-tile histograms -> device scan
+//      -> scatter with a stable in-tile rank), gather (issue, retire), group starts by gap filling;
+//      every group with >= 2n executions is split into runs of 4 x 2048 positions;
+//   4. persistent CTAs take runs from a global ticket counter in run-major order (run 0 of every group first),
+//      skipping runs that start past an already-latched position.  Per run: the window sums ending just before
+//      it by a block reduction; per 2048-position item, per-thread deltas by a block scan, then each thread slides
+//      over its 8 positions and evaluates cond1/cond2 exactly in i128; the first passing position per group is an
+//      atomicMin; sums carry to the next item;
 //   5. S_n at the latched position, first_stable/stable_dur_sum, and the per-kernel switch point.
 #include "internal.h"
 
@@ -27,9 +31,12 @@ constexpr int RTILE = RT * RIPT;
 constexpr int RBITS = 8;
 constexpr int RNB = 1 << RBITS;
 constexpr int REC_CHUNK = 4096;
+constexpr int JOB = 2048;       // records per warp job (one-pass multisplit)
 constexpr int WT = 256;        // window threads
 constexpr int WPT = 8;         // positions per thread
 constexpr int WITEM = WT * WPT;
+constexpr int NI = 4;          // items per run
+constexpr int RUN = WITEM * NI;
 
 // ---- generic device-wide exclusive scan of u32 (values and total < 2^32) --------------------------------------
 constexpr int SB = 4096;
@@ -117,8 +124,8 @@ void scan_u32(const uint32_t* in, uint32_t* out, uint64_t n, uint32_t* bsum, uin
 }
 
 // ---- 1. per-kernel record chunks + validation + keys -------------------------------------------------------
-__global__ void __launch_bounds__(1024) k_rec_chunks(const uint64_t* kro, uint32_t K, uint64_t R, uint64_t* coff,
-                                                     DevErr* err) {
+__global__ void __launch_bounds__(1024) k_rec_chunks(const uint64_t* kro, uint32_t K, uint64_t R, uint64_t chunk,
+                                                     uint64_t* coff, DevErr* err) {
   __shared__ uint64_t ws[32];
   __shared__ uint64_t carry;
   if (threadIdx.x == 0) {
@@ -131,9 +138,9 @@ __global__ void __launch_bounds__(1024) k_rec_chunks(const uint64_t* kro, uint32
     uint32_t k = base + threadIdx.x;
     uint64_t v = 0;
     if (k < K) {
-      uint64_t a = kro[k], b = kro[k + 1];
-      if (b < a) latch(err, PHOTON_ERANGE, (int64_t)k);
-      v = b > a ? ceil_div(b - a, REC_CHUNK) : 0;
+      uint64_t a = umin64(kro[k], R), b = umin64(kro[k + 1], R);
+      if (kro[k + 1] < kro[k] || kro[k + 1] > R) latch(err, PHOTON_ERANGE, (int64_t)k);
+      v = b > a ? ceil_div(b - a, chunk) : 0;
     }
     uint64_t x = v;
     for (int o = 1; o < 32; o <<= 1) {
@@ -170,13 +177,13 @@ __device__ __forceinline__ uint32_t upper_idx(const uint64_t* a, uint32_t n, uin
   return lo;
 }
 
-__global__ void __launch_bounds__(256) k_rec_prep(photon_timing t, const uint64_t* coff, uint32_t bbits,
-                                                  uint64_t* key, DevErr* err) {
+__global__ void __launch_bounds__(256) k_rec_prep(photon_timing t, const uint64_t* coff, uint64_t* key,
+                                                  DevErr* err) {
   const uint64_t total = coff[t.n_kernels];
   for (uint64_t job = blockIdx.x; job < total; job += gridDim.x) {
     uint32_t k = upper_idx(coff, t.n_kernels, job);
     uint64_t c = job - coff[k];
-    uint64_t a = t.kernel_rec_off[k], b = t.kernel_rec_off[k + 1];
+    uint64_t a = umin64(t.kernel_rec_off[k], t.n_records), b = umin64(t.kernel_rec_off[k + 1], t.n_records);  // clamped: bad offsets are latched by k_rec_chunks
     uint64_t cs = a + c * REC_CHUNK, ce = umin64(cs + REC_CHUNK, b);
     for (uint64_t i = cs + threadIdx.x; i < ce; i += blockDim.x) {
       uint32_t bb = t.bb[i];
@@ -185,7 +192,7 @@ __global__ void __launch_bounds__(256) k_rec_prep(photon_timing t, const uint64_
         latch(err, PHOTON_ERANGE, (int64_t)i);
         bb = 0;
       }
-      key[i] = ((uint64_t)k << bbits) | bb;
+      key[i] = (uint64_t)bb * t.n_kernels + k;  // group id g = b*K + k
     }
   }
 }
@@ -260,29 +267,131 @@ __global__ void k_gather(const uint32_t* idx, uint64_t n, const uint64_t* issue,
   Y[p] = retire[i];
 }
 
-__global__ void k_heads(const uint64_t* key, uint64_t n, uint32_t* flag) {
+__global__ void k_set_u32(uint32_t* p, uint32_t v) { *p = v; }
+
+// gstart[g] = first sorted position with key >= g, for every g in [0, K*B] (empty groups have size 0)
+__global__ void k_fill_gstart(const uint64_t* key, uint64_t n, uint64_t G, uint64_t* gstart) {
   uint64_t p = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
-  if (p >= n) return;
-  flag[p] = (p == 0 || key[p] != key[p - 1]) ? 1u : 0u;
+  if (p > n) return;
+  uint64_t lo = p == 0 ? 0 : key[p - 1] + 1, hi = p == n ? G : key[p];
+  for (uint64_t g = lo; g <= hi && g <= G; ++g) gstart[g] = p;
 }
 
-__global__ void k_group_start(const uint64_t* key, uint64_t n, const uint32_t* gidx, uint64_t* gstart) {
-  uint64_t p = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
-  if (p >= n) return;
-  if (p == 0 || key[p] != key[p - 1]) gstart[gidx[p]] = p;
+constexpr uint32_t kNone = 0xFFFFFFFFu;  // padding lane (not a u16 id)
+
+// ---- 2'. one-pass stable multisplit for B <= 256 (the common case): one warp per job = (kernel, JOB records) --
+// Records of a job belong to one kernel, so a stable split by bb inside each job, with job offsets from a
+// bin-major scan of the per-job histograms, leaves group (b, k) contiguous, in retirement order, at
+// hist[b][first job of k] -- the group id g = b*K + k needs no key array.
+__global__ void __launch_bounds__(256) k_job_hist(photon_timing t, const uint64_t* coff, uint64_t n_jobs,
+                                                  uint32_t* hist) {
+  __shared__ uint32_t h[8][256];
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+  const uint32_t B = t.n_bb;
+  for (int d = lane; d < (int)B; d += 32) h[wid][d] = 0;
+  __syncwarp();
+  for (uint64_t job = (uint64_t)blockIdx.x * 8 + wid; job < n_jobs; job += (uint64_t)gridDim.x * 8) {
+    uint32_t k = upper_idx(coff, t.n_kernels, job);
+    uint64_t a = umin64(t.kernel_rec_off[k], t.n_records), b = umin64(t.kernel_rec_off[k + 1], t.n_records);  // clamped: bad offsets are latched by k_rec_chunks
+    uint64_t cs = a + (job - coff[k]) * JOB, ce = umin64(cs + JOB, b);
+    for (uint64_t i0 = cs; i0 < ce; i0 += 128) {
+      uint32_t d[4];
+#pragma unroll
+      for (int u = 0; u < 4; ++u) {
+        uint64_t i = i0 + u * 32 + lane;
+        d[u] = i < ce ? (uint32_t)t.bb[i] : kNone;
+      }
+#pragma unroll
+      for (int u = 0; u < 4; ++u) {
+        uint32_t x = d[u] < B || d[u] == kNone ? d[u] : 0u;  // bad ids count as bb 0 (latched by the scatter)
+        unsigned peers = __match_any_sync(0xffffffffu, x);
+        if (x != kNone && lane == __ffs(peers) - 1) h[wid][x] += __popc(peers);
+        __syncwarp();
+      }
+    }
+    for (int dd = lane; dd < (int)B; dd += 32) {
+      hist[(uint64_t)dd * n_jobs + job] = h[wid][dd];
+      h[wid][dd] = 0;
+    }
+    __syncwarp();
+  }
 }
 
-__global__ void k_group_end(uint64_t* gstart, const uint32_t* G, uint64_t n) { gstart[*G] = n; }
+__global__ void __launch_bounds__(256) k_job_scatter(photon_timing t, const uint64_t* coff, uint64_t n_jobs,
+                                                     const uint32_t* off, uint64_t* X, uint64_t* Y, uint32_t* idx,
+                                                     DevErr* err) {
+  __shared__ uint32_t run[8][256];
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+  const uint32_t B = t.n_bb;
+  const unsigned lt = (1u << lane) - 1u;
+  for (uint64_t job = (uint64_t)blockIdx.x * 8 + wid; job < n_jobs; job += (uint64_t)gridDim.x * 8) {
+    uint32_t k = upper_idx(coff, t.n_kernels, job);
+    uint64_t a = umin64(t.kernel_rec_off[k], t.n_records), b = umin64(t.kernel_rec_off[k + 1], t.n_records);  // clamped: bad offsets are latched by k_rec_chunks
+    uint64_t cs = a + (job - coff[k]) * JOB, ce = umin64(cs + JOB, b);
+    for (int dd = lane; dd < (int)B; dd += 32) run[wid][dd] = off[(uint64_t)dd * n_jobs + job];
+    __syncwarp();
+    for (uint64_t i0 = cs; i0 < ce; i0 += 128) {
+      uint32_t d[4];
+      uint64_t x[4], y[4], yp[4];
+#pragma unroll
+      for (int u = 0; u < 4; ++u) {
+        uint64_t i = i0 + u * 32 + lane;
+        bool v = i < ce;
+        d[u] = v ? (uint32_t)t.bb[i] : kNone;
+        x[u] = v ? t.issue[i] : 0;
+        y[u] = v ? t.retire[i] : 0;
+        yp[u] = v && i > a ? t.retire[i - 1] : 0;
+      }
+#pragma unroll
+      for (int u = 0; u < 4; ++u) {
+        uint64_t i = i0 + u * 32 + lane;
+        uint32_t dd = d[u];
+        if (dd != kNone) {
+          if (dd >= B || x[u] >= kTimeLimit || y[u] >= kTimeLimit || y[u] < x[u] || yp[u] > y[u]) {
+            latch(err, PHOTON_ERANGE, (int64_t)i);
+            if (dd >= B) dd = 0;
+          }
+        }
+        unsigned peers = __match_any_sync(0xffffffffu, dd);
+        uint32_t base = dd != kNone ? run[wid][dd] : 0;
+        __syncwarp();
+        if (dd != kNone) {
+          if (lane == __ffs(peers) - 1) run[wid][dd] = base + __popc(peers);
+          uint32_t dest = base + __popc(peers & lt);
+          X[dest] = x[u];
+          Y[dest] = y[u];
+          idx[dest] = (uint32_t)i;
+        }
+        __syncwarp();
+      }
+    }
+  }
+}
 
-__global__ void k_work_count(const uint64_t* gstart, const uint32_t* G, uint32_t n2, uint32_t* nwork,
-                             uint64_t* gfirst, uint64_t gcap) {
-  uint64_t g = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
-  if (g >= gcap) return;
-  uint32_t ng = *G;
-  if (g >= ng) { nwork[g] = 0; return; }
-  uint64_t sz = gstart[g + 1] - gstart[g];
-  nwork[g] = sz >= n2 ? (uint32_t)ceil_div(sz - n2 + 1, WITEM) : 0u;
-  gfirst[g] = ~0ull;
+// gstart[b*K + k] = start of group (b, k) = scanned hist[b][first job of k]; gstart[K*B] = R
+__global__ void k_job_gstart(const uint32_t* off, const uint64_t* coff, uint32_t K, uint32_t B, uint64_t n_jobs,
+                             uint64_t R, uint64_t* gstart, uint32_t* G) {
+  const uint64_t n = (uint64_t)K * B;
+  for (uint64_t g = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; g <= n; g += (uint64_t)gridDim.x * blockDim.x) {
+    if (g == n) { gstart[g] = R; *G = (uint32_t)n; continue; }
+    uint64_t b = g / K, k = g % K;
+    uint64_t j = b * n_jobs + umin64(coff[k], n_jobs);  // clamp keeps gstart monotone on malformed offsets
+    gstart[g] = j < (uint64_t)B * n_jobs ? off[j] : R;
+  }
+}
+
+// runs per group: a group of size sz tests positions [2n-1, sz) (L229: only once 2n executions exist), split
+// into runs of RUN positions; maxr = the largest run count (the number of ticket rounds)
+__global__ void k_work_count(const uint64_t* gstart, const uint32_t* G, uint32_t n2, uint32_t* nruns,
+                             uint64_t* gfirst, uint32_t* maxr) {
+  const uint32_t ng = *G;
+  for (uint32_t g = blockIdx.x * blockDim.x + threadIdx.x; g < ng; g += gridDim.x * blockDim.x) {
+    uint64_t sz = gstart[g + 1] - gstart[g];
+    uint32_t r = sz >= n2 ? (uint32_t)ceil_div(sz - n2 + 1, RUN) : 0u;
+    nruns[g] = r;
+    gfirst[g] = ~0ull;
+    if (r) atomicMax(maxr, r);
+  }
 }
 
 // ---- 4. windowed exact test ----------------------------------------------------------------------------------
@@ -335,231 +444,268 @@ struct WinArgs {
   const uint64_t* Y;
   const uint64_t* gstart;
   const uint32_t* G;
-  const uint32_t* work_off;  // exclusive scan of nwork, [gcap]
-  const uint32_t* n_work;    // total
-  uint64_t gcap;
+  const uint32_t* nruns;  // [G] runs per group
+  const uint32_t* maxr;   // max over groups
+  uint32_t* ticket;       // global ticket counter (zeroed)
   uint32_t n;
   uint32_t dnum, dden;
   uint64_t* gfirst;
 };
 
-__global__ void __launch_bounds__(WT) k_window(WinArgs a) {
+__device__ __forceinline__ void sums_sub(Sums& a, const Sums& b) {
+  a.sx -= b.sx; a.sy -= b.sy; a.sn -= b.sn; a.s2n -= b.s2n; a.sxy -= b.sxy; a.sxx -= b.sxx;
+}
+
+// Ticket t = r * G + g names run r of group g: every group's run 0 is handed out before any group's run 1, so a
+// group whose first stable position was latched early skips its later runs (the test wants only the FIRST j).
+// A run slides over up to NI items of WITEM positions, carrying the window sums from item to item, so the
+// 2n-position base reduction is paid once per run.  Exactness: every run whose first position is <= the final
+// answer is processed (a run is skipped only when gfirst[g] already holds a smaller position).
+__global__ void __launch_bounds__(WT, 2) k_window(WinArgs a) {
   __shared__ Sums part[WT / 32];
   __shared__ Sums wtot[WT / 32];
-  __shared__ uint64_t best;
+  __shared__ uint64_t best, s_gf;
+  __shared__ uint32_t s_mask, s_base;
+  __shared__ int s_stop;
   const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
-  const uint32_t total = *a.n_work;
-  const uint32_t G = *a.G;
+  const uint32_t G = *a.G, maxr = *a.maxr;
   const int64_t n = a.n;
-  for (uint32_t item = blockIdx.x; item < total; item += gridDim.x) {
-    // group of this work item: last g with work_off[g] <= item (and a non-empty item count)
-    uint32_t lo = 0, hi = G - 1;
-    while (lo < hi) {
-      uint32_t mid = (lo + hi + 1) >> 1;
-      if (a.work_off[mid] <= item) lo = mid; else hi = mid - 1;
-    }
-    uint32_t g = lo;
-    const int64_t gs = (int64_t)a.gstart[g], ge = (int64_t)a.gstart[g + 1];
-    const int64_t c = item - a.work_off[g];
-    const int64_t Q0 = gs + 2 * n - 1 + c * WITEM;
-    const int64_t Q1 = Q0 + WITEM < ge ? Q0 + WITEM : ge;
-    auto X = [&](int64_t q) -> int64_t { return q >= gs ? (int64_t)a.X[q] : 0; };
-    auto D = [&](int64_t q) -> int64_t { return q >= gs ? (int64_t)(a.Y[q] - a.X[q]) : 0; };
-    auto Y = [&](int64_t q) -> int64_t { return q >= gs ? (int64_t)a.Y[q] : 0; };
-    // base: windows ending at Q0-1 ([Q0-n, Q0-1] and [Q0-2n, Q0-1]); positions < gs contribute 0
-    Sums s;
-    sums_zero(s);
-    for (int64_t q = Q0 - 2 * n + tid; q < Q0; q += WT) {
-      int64_t d = D(q);
-      s.s2n += d;
-      if (q >= Q0 - n) {
-        int64_t x = X(q), y = Y(q);
-        s.sx += x; s.sy += y; s.sn += d;
-        s.sxy += (i128)x * y; s.sxx += (i128)x * x;
+  if (G == 0 || maxr == 0) return;
+  const uint64_t n_tickets = (uint64_t)G * maxr;
+  for (;;) {
+    // warp 0 claims 32 tickets and filters out the empty / already-decided ones
+    if (wid == 0) {
+      uint32_t base = 0;
+      if (lane == 0) base = atomicAdd(a.ticket, 32u);
+      base = __shfl_sync(0xffffffffu, base, 0);
+      uint64_t t = (uint64_t)base + lane;
+      bool ok = false;
+      if (t < n_tickets) {
+        uint32_t r = (uint32_t)(t / G), g = (uint32_t)(t % G);
+        if (r < a.nruns[g]) {
+          uint64_t P0 = a.gstart[g] + 2 * n - 1 + (uint64_t)r * RUN;
+          ok = *(volatile const uint64_t*)&a.gfirst[g] > P0;
+        }
       }
+      uint32_t m = __ballot_sync(0xffffffffu, ok);
+      if (lane == 0) { s_mask = m; s_base = base; s_stop = (uint64_t)base >= n_tickets; }
     }
-    for (int o = 16; o > 0; o >>= 1) sums_add(s, shfl_xor_sums(s, o));
-    if (lane == 0) part[wid] = s;
-    // per-thread deltas over its 8 positions
-    Sums dl;
-    sums_zero(dl);
-    const int64_t q0 = Q0 + (int64_t)tid * WPT;
-    int64_t xs[WPT], ys[WPT], xo[WPT], yo[WPT], do2[WPT];
+    __syncthreads();
+    const uint32_t mask = s_mask, tbase = s_base;
+    const int stop = s_stop;
+    __syncthreads();
+    if (stop) break;
+    for (uint32_t mm = mask; mm; mm &= mm - 1) {
+      const uint64_t t = (uint64_t)tbase + (__ffs(mm) - 1);
+      const uint32_t r = (uint32_t)(t / G), g = (uint32_t)(t % G);
+      const int64_t gs = (int64_t)a.gstart[g], ge = (int64_t)a.gstart[g + 1];
+      const int64_t P0 = gs + 2 * n - 1 + (int64_t)r * RUN;
+      const int64_t P1 = P0 + RUN < ge ? P0 + RUN : ge;
+      auto X = [&](int64_t q) -> int64_t { return q >= gs ? (int64_t)__ldg(a.X + q) : 0; };
+      auto Yv = [&](int64_t q) -> int64_t { return q >= gs ? (int64_t)__ldg(a.Y + q) : 0; };
+      // base: windows ending at P0-1 ([P0-n, P0-1] and [P0-2n, P0-1]); positions < gs contribute 0
+      Sums s;
+      sums_zero(s);
+#pragma unroll 4
+      for (int64_t q = P0 - 2 * n + tid; q < P0; q += WT) {
+        int64_t x = X(q), y = Yv(q), d = y - x;
+        s.s2n += d;
+        if (q >= P0 - n) {
+          s.sx += x; s.sy += y; s.sn += d;
+          s.sxy += (i128)x * y; s.sxx += (i128)x * x;
+        }
+      }
+      for (int o = 16; o > 0; o >>= 1) sums_add(s, shfl_xor_sums(s, o));
+      if (lane == 0) part[wid] = s;
+      if (tid == 0) best = ~0ull;
+      __syncthreads();
+      Sums base;
+      sums_zero(base);
+      for (int k = 0; k < WT / 32; ++k) sums_add(base, part[k]);
+      for (int64_t Q0 = P0; Q0 < P1; Q0 += WITEM) {
+        const int64_t Q1 = Q0 + WITEM < P1 ? Q0 + WITEM : P1;
+        const int64_t q0 = Q0 + (int64_t)tid * WPT;
+        // pass 1: this thread's deltas over its WPT positions
+        Sums dl;
+        sums_zero(dl);
 #pragma unroll
-    for (int u = 0; u < WPT; ++u) {
-      int64_t q = q0 + u;
-      if (q < Q1) {
-        xs[u] = X(q); ys[u] = Y(q); xo[u] = X(q - n); yo[u] = Y(q - n); do2[u] = D(q - 2 * n);
-      } else {
-        xs[u] = ys[u] = xo[u] = yo[u] = do2[u] = 0;
+        for (int u = 0; u < WPT; ++u) {
+          int64_t q = q0 + u;
+          if (q < Q1) {
+            int64_t xs = X(q), ys = Yv(q), xo = X(q - n), yo = Yv(q - n);
+            int64_t do2 = Yv(q - 2 * n) - X(q - 2 * n);
+            dl.sx += xs - xo; dl.sy += ys - yo;
+            dl.sn += (ys - xs) - (yo - xo);
+            dl.s2n += (ys - xs) - do2;
+            dl.sxy += (i128)xs * ys - (i128)xo * yo;
+            dl.sxx += (i128)xs * xs - (i128)xo * xo;
+          }
+        }
+        Sums incl = dl;
+        for (int o = 1; o < 32; o <<= 1) {
+          Sums tt = shfl_up_sums(incl, o);
+          if (lane >= o) sums_add(incl, tt);
+        }
+        if (lane == 31) wtot[wid] = incl;
+        __syncthreads();
+        Sums w = base, tot;
+        sums_zero(tot);
+        for (int k = 0; k < WT / 32; ++k) {
+          if (k < wid) sums_add(w, wtot[k]);
+          sums_add(tot, wtot[k]);
+        }
+        sums_add(w, incl);
+        sums_sub(w, dl);  // exclusive prefix: window sums ending at q0 - 1
+        // pass 2: slide and test (values re-read through L1)
+        uint64_t mine = ~0ull;
+        for (int u = 0; u < WPT; ++u) {
+          int64_t q = q0 + u;
+          if (q >= Q1) break;
+          int64_t xs = X(q), ys = Yv(q), xo = X(q - n), yo = Yv(q - n);
+          int64_t do2 = Yv(q - 2 * n) - X(q - 2 * n);
+          w.sx += xs - xo; w.sy += ys - yo;
+          w.sn += (ys - xs) - (yo - xo);
+          w.s2n += (ys - xs) - do2;
+          w.sxy += (i128)xs * ys - (i128)xo * yo;
+          w.sxx += (i128)xs * xs - (i128)xo * xo;
+          // cond1: den > 0 and dden*|den - num| < dnum*den  (Eq. 1: a = num/den)
+          i128 num = (i128)n * w.sxy - (i128)w.sx * w.sy;
+          i128 den = (i128)n * w.sxx - (i128)w.sx * w.sx;
+          bool c1 = false;
+          if (den > 0) {
+            i128 diff = den - num;
+            if (diff < 0) diff = -diff;
+            c1 = (i128)a.dden * diff < (i128)a.dnum * den;
+          }
+          bool c2 = false;
+          if (c1 && w.s2n > 0) {
+            i128 d2 = 2 * (i128)w.sn - w.s2n;
+            if (d2 < 0) d2 = -d2;
+            c2 = (i128)a.dden * d2 < (i128)a.dnum * w.s2n;
+          }
+          if (c1 && c2) { mine = (uint64_t)q; break; }
+        }
+        if (mine != ~0ull) atomicMin((unsigned long long*)&best, (unsigned long long)mine);
+        if (tid == 0) s_gf = *(volatile const uint64_t*)&a.gfirst[g];
+        sums_add(base, tot);
+        __syncthreads();
+        const uint64_t b = best;
+        if (b != ~0ull) {
+          if (tid == 0) atomicMin((unsigned long long*)&a.gfirst[g], (unsigned long long)b);
+          break;
+        }
+        // another run of this group latched an earlier position: the rest of this run cannot matter
+        if (s_gf < (uint64_t)Q1) break;
       }
-      dl.sx += xs[u] - xo[u];
-      dl.sy += ys[u] - yo[u];
-      dl.sn += (ys[u] - xs[u]) - (yo[u] - xo[u]);
-      dl.s2n += (ys[u] - xs[u]) - do2[u];
-      dl.sxy += (i128)xs[u] * ys[u] - (i128)xo[u] * yo[u];
-      dl.sxx += (i128)xs[u] * xs[u] - (i128)xo[u] * xo[u];
+      __syncthreads();
     }
-    // block exclusive scan of dl
-    Sums incl = dl;
-    for (int o = 1; o < 32; o <<= 1) {
-      Sums t = shfl_up_sums(incl, o);
-      if (lane >= o) sums_add(incl, t);
-    }
-    if (lane == 31) wtot[wid] = incl;
-    if (tid == 0) best = ~0ull;
-    __syncthreads();
-    Sums w;
-    sums_zero(w);
-    for (int k = 0; k < WT / 32; ++k) sums_add(w, part[k]);  // base
-    for (int k = 0; k < wid; ++k) sums_add(w, wtot[k]);
-    // exclusive = w + incl - dl
-    sums_add(w, incl);
-    w.sx -= dl.sx; w.sy -= dl.sy; w.sn -= dl.sn; w.s2n -= dl.s2n; w.sxy -= dl.sxy; w.sxx -= dl.sxx;
-    uint64_t mine = ~0ull;
-#pragma unroll
-    for (int u = 0; u < WPT; ++u) {
-      int64_t q = q0 + u;
-      if (q >= Q1) break;
-      w.sx += xs[u] - xo[u];
-      w.sy += ys[u] - yo[u];
-      w.sn += (ys[u] - xs[u]) - (yo[u] - xo[u]);
-      w.s2n += (ys[u] - xs[u]) - do2[u];
-      w.sxy += (i128)xs[u] * ys[u] - (i128)xo[u] * yo[u];
-      w.sxx += (i128)xs[u] * xs[u] - (i128)xo[u] * xo[u];
-      if (mine != ~0ull) continue;
-      // cond1: den > 0 and dden*|den - num| < dnum*den  (Eq. 1: a = num/den)
-      i128 num = (i128)n * w.sxy - (i128)w.sx * w.sy;
-      i128 den = (i128)n * w.sxx - (i128)w.sx * w.sx;
-      bool c1 = false;
-      if (den > 0) {
-        i128 diff = den - num;
-        if (diff < 0) diff = -diff;
-        c1 = (i128)a.dden * diff < (i128)a.dnum * den;
-      }
-      bool c2 = false;
-      if (c1 && w.s2n > 0) {
-        i128 d2 = 2 * (i128)w.sn - w.s2n;
-        if (d2 < 0) d2 = -d2;
-        c2 = (i128)a.dden * d2 < (i128)a.dnum * w.s2n;
-      }
-      if (c1 && c2) mine = (uint64_t)q;
-    }
-    if (mine != ~0ull) atomicMin((unsigned long long*)&best, (unsigned long long)mine);
-    __syncthreads();
-    if (tid == 0 && best != ~0ull) atomicMin((unsigned long long*)&a.gfirst[g], (unsigned long long)best);
-    __syncthreads();
   }
 }
 
 // ---- 5. outputs ----------------------------------------------------------------------------------------------
-__global__ void k_finish(const uint64_t* key, const uint32_t* idx, const uint64_t* X, const uint64_t* Y,
-                         const uint64_t* gstart, const uint32_t* G, const uint64_t* gfirst, const uint64_t* kro,
-                         uint32_t bbits, uint32_t B, uint32_t n, int64_t* first_stable, uint64_t* dur) {
-  uint32_t warp = (blockIdx.x * blockDim.x + threadIdx.x) >> 5, lane = threadIdx.x & 31;
-  if (warp >= *G) return;
-  uint64_t q = gfirst[warp];
-  if (q == ~0ull) return;
-  uint64_t k = key[q] >> bbits, b = key[q] & ((1ull << bbits) - 1);
-  uint64_t s = 0;
-  for (uint64_t i = q + 1 - n + lane; i <= q; i += 32) s += Y[i] - X[i];
-  for (int o = 16; o > 0; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
-  if (lane == 0) {
-    first_stable[k * B + b] = (int64_t)(idx[q] - kro[k]);
-    if (dur) dur[k * B + b] = s;
+__global__ void k_finish(const uint32_t* idx, const uint64_t* X, const uint64_t* Y, const uint32_t* G,
+                         const uint64_t* gfirst, const uint64_t* kro, uint32_t K, uint32_t B, uint32_t n,
+                         int64_t* first_stable, uint64_t* dur) {
+  const uint32_t lane = threadIdx.x & 31, ng = *G;
+  const uint32_t nw = (gridDim.x * blockDim.x) >> 5;
+  for (uint32_t g = (blockIdx.x * blockDim.x + threadIdx.x) >> 5; g < ng; g += nw) {
+    uint64_t q = gfirst[g];
+    if (q == ~0ull) continue;
+    uint64_t k = g % K, b = g / K;
+    uint64_t s = 0;
+    for (uint64_t i = q + 1 - n + lane; i <= q; i += 32) s += Y[i] - X[i];
+    for (int o = 16; o > 0; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
+    if (lane == 0) {
+      first_stable[k * B + b] = (int64_t)(idx[q] - kro[k]);
+      if (dur) dur[k * B + b] = s;
+    }
   }
 }
 
-// switch_at[k]: order stable BBs by position; first position where rate_den * acc > rate_num * total (L208)
-__global__ void __launch_bounds__(256) k_switch(const uint64_t* key, const uint64_t* gstart, const uint32_t* G,
-                                                const uint64_t* gfirst, const int64_t* first_stable,
-                                                const uint64_t* kbb, uint32_t K, uint32_t B, uint32_t bbits,
-                                                uint32_t rnum, uint32_t rden, int64_t* switch_at) {
-  __shared__ uint64_t tot_lo[8], tot_hi[8];
-  __shared__ int64_t best;
-  const uint32_t ng = *G;
+// switch_at[k]: order stable BBs by t_b; the first t_b at which rate_den * acc > rate_num * total, where acc sums
+// the weights of stable BBs with t <= t_b (L208, Fig 7) [P-14].  acc(t) is monotone and changes only at stable
+// t_b values, so the answer is the least t with rate_den * acc(t) > rate_num * total: a binary search over t in
+// [0, 2^32) with one block reduction per step (O(32 B) per kernel instead of sorting).
+__device__ __forceinline__ u128 block_sum_u128(u128 v, uint64_t* slo, uint64_t* shi) {
+  uint64_t lo = (uint64_t)v, hi = (uint64_t)(v >> 64);
+  for (int o = 16; o > 0; o >>= 1) {
+    uint64_t lo2 = __shfl_xor_sync(0xffffffffu, lo, o), hi2 = __shfl_xor_sync(0xffffffffu, hi, o);
+    uint64_t s = lo + lo2;
+    hi = hi + hi2 + (s < lo);
+    lo = s;
+  }
+  __syncthreads();
+  if ((threadIdx.x & 31) == 0) { slo[threadIdx.x >> 5] = lo; shi[threadIdx.x >> 5] = hi; }
+  __syncthreads();
+  u128 t = 0;
+  for (int w = 0; w < 8; ++w) t += ((u128)shi[w] << 64) | slo[w];
+  return t;
+}
+
+__global__ void __launch_bounds__(256) k_switch(const int64_t* first_stable, const uint64_t* kbb, uint32_t K,
+                                                uint32_t B, uint32_t rnum, uint32_t rden, int64_t* switch_at) {
+  __shared__ uint64_t slo[8], shi[8];
   for (uint32_t k = blockIdx.x; k < K; k += gridDim.x) {
-    // total weight of the kernel's BB distribution (u128)
-    u128 t = 0;
-    for (uint32_t b = threadIdx.x; b < B; b += blockDim.x) t += kbb[(uint64_t)k * B + b];
-    uint64_t lo = (uint64_t)t, hi = (uint64_t)(t >> 64);
-    for (int o = 16; o > 0; o >>= 1) {
-      uint64_t lo2 = __shfl_xor_sync(0xffffffffu, lo, o), hi2 = __shfl_xor_sync(0xffffffffu, hi, o);
-      uint64_t s = lo + lo2;
-      hi = hi + hi2 + (s < lo);
-      lo = s;
+    const int64_t* fs = first_stable + (uint64_t)k * B;
+    const uint64_t* w = kbb + (uint64_t)k * B;
+    u128 t = 0, a = 0;
+    for (uint32_t b = threadIdx.x; b < B; b += blockDim.x) {
+      t += w[b];
+      if (fs[b] >= 0) a += w[b];
     }
-    if ((threadIdx.x & 31) == 0) { tot_lo[threadIdx.x >> 5] = lo; tot_hi[threadIdx.x >> 5] = hi; }
-    if (threadIdx.x == 0) best = -1;
-    __syncthreads();
-    u128 total = 0;
-    for (int w = 0; w < 8; ++w) total += ((u128)tot_hi[w] << 64) | tot_lo[w];
-    // groups of kernel k: keys in [k << bbits, (k+1) << bbits)
-    uint32_t g_lo = 0, g_hi = 0;
-    if (ng > 0) {
-      uint64_t klo = (uint64_t)k << bbits, khi = (uint64_t)(k + 1) << bbits;
-      uint32_t a = 0, b = ng;  // first g with key >= klo
-      while (a < b) { uint32_t m = (a + b) >> 1; if (key[gstart[m]] < klo) a = m + 1; else b = m; }
-      g_lo = a;
-      b = ng;
-      while (a < b) { uint32_t m = (a + b) >> 1; if (key[gstart[m]] < khi) a = m + 1; else b = m; }
-      g_hi = a;
-    }
-    if (total > 0) {
-      for (uint32_t gi = g_lo + threadIdx.x; gi < g_hi; gi += blockDim.x) {
-        if (gfirst[gi] == ~0ull) continue;
-        uint32_t bi = (uint32_t)(key[gstart[gi]] & ((1ull << bbits) - 1));
-        int64_t ti = first_stable[(uint64_t)k * B + bi];
-        u128 acc = 0;
-        for (uint32_t gj = g_lo; gj < g_hi; ++gj) {
-          if (gfirst[gj] == ~0ull) continue;
-          uint32_t bj = (uint32_t)(key[gstart[gj]] & ((1ull << bbits) - 1));
-          if (first_stable[(uint64_t)k * B + bj] <= ti) acc += kbb[(uint64_t)k * B + bj];
-        }
-        if ((u128)rden * acc > (u128)rnum * total) {
-          // min over candidates
-          unsigned long long cur = (unsigned long long)ti;
-          atomicMin((unsigned long long*)&best, cur);  // best starts at -1 = 0xFF..: unsigned min works
-        }
+    const u128 total = block_sum_u128(t, slo, shi);
+    const u128 all = block_sum_u128(a, slo, shi);
+    int64_t ans = -1;
+    if (total > 0 && (u128)rden * all > (u128)rnum * total) {
+      uint64_t lo = 0, hi = 0xFFFFFFFFull;  // invariant: acc(hi) passes
+      while (lo < hi) {
+        uint64_t mid = (lo + hi) >> 1;
+        u128 m = 0;
+        for (uint32_t b = threadIdx.x; b < B; b += blockDim.x)
+          if (fs[b] >= 0 && (uint64_t)fs[b] <= mid) m += w[b];
+        m = block_sum_u128(m, slo, shi);
+        if ((u128)rden * m > (u128)rnum * total) hi = mid; else lo = mid + 1;
       }
+      ans = (int64_t)lo;
     }
-    __syncthreads();
-    if (threadIdx.x == 0) switch_at[k] = best;
+    if (threadIdx.x == 0) switch_at[k] = ans;
     __syncthreads();
   }
 }
 
 struct Layout {
-  uint64_t* key0; uint64_t* key1;
-  uint32_t* val0; uint32_t* val1;
+  bool onepass;      // B <= 256: job multisplit; else LSD radix sort of composite keys
+  uint64_t* key0; uint64_t* key1;  // radix path only
+  uint32_t* val0; uint32_t* val1;  // val0 = original record index of each sorted position (both paths)
   uint64_t* X; uint64_t* Y;
-  uint32_t* hist; uint32_t* bsum; uint32_t* misc;  // misc[0] = G, misc[1] = total work
-  uint32_t* flag;  // [R] heads -> group index (scan)
+  uint32_t* hist; uint32_t* bsum; uint32_t* misc;  // misc[0] = G, [1] = max runs, [2] = ticket, [4] = scan total
   uint64_t* gstart;  // [gcap+1]
-  uint32_t* nwork;   // [gcap]
+  uint32_t* nruns;   // [gcap]
   uint64_t* gfirst;  // [gcap]
-  uint64_t* coff;    // [K+1]
-  uint64_t gcap, n_tiles;
+  uint64_t* coff;    // [K+1] chunk (job) offsets per kernel
+  uint64_t gcap, n_tiles, n_jobs, hn;
   size_t bytes;
 };
 
 Layout make_layout(const photon_timing& t, void* base) {
   Carver c(base);
-  Layout L;
+  Layout L{};
   uint64_t R = t.n_records ? t.n_records : 1;
+  L.onepass = t.n_bb <= 256;
+  L.gcap = (uint64_t)t.n_kernels * t.n_bb;  // dense group ids g = b*K + k
+  if (L.gcap == 0) L.gcap = 1;
   L.n_tiles = ceil_div(R, RTILE);
-  L.gcap = R;
-  L.key0 = c.take<uint64_t>(R); L.key1 = c.take<uint64_t>(R);
-  L.val0 = c.take<uint32_t>(R); L.val1 = c.take<uint32_t>(R);
+  L.n_jobs = ceil_div(R, JOB) + t.n_kernels;
+  if (!L.onepass) { L.key0 = c.take<uint64_t>(R); L.key1 = c.take<uint64_t>(R); }
+  L.val0 = c.take<uint32_t>(R);
+  if (!L.onepass) L.val1 = c.take<uint32_t>(R);
   L.X = c.take<uint64_t>(R); L.Y = c.take<uint64_t>(R);
-  uint64_t hn = (uint64_t)RNB * L.n_tiles;
-  uint64_t scan_n = hn > R ? hn : R;
-  L.hist = c.take<uint32_t>(hn);
-  L.bsum = c.take<uint32_t>(ceil_div(scan_n, SB) + 1);
+  L.hn = L.onepass ? (uint64_t)t.n_bb * L.n_jobs : (uint64_t)RNB * L.n_tiles;
+  L.hist = c.take<uint32_t>(L.hn);
+  L.bsum = c.take<uint32_t>(ceil_div(L.hn, SB) + 1);
   L.misc = c.take<uint32_t>(16);
-  L.flag = c.take<uint32_t>(R);
   L.gstart = c.take<uint64_t>(L.gcap + 1);
-  L.nwork = c.take<uint32_t>(L.gcap);
+  L.nruns = c.take<uint32_t>(L.gcap);
   L.gfirst = c.take<uint64_t>(L.gcap);
   L.coff = c.take<uint64_t>((uint64_t)t.n_kernels + 1);
   L.bytes = c.off + 256;
@@ -577,50 +723,59 @@ cudaError_t launch_stable(const photon_timing& t, const uint64_t* kbb, photon_st
   Layout L = make_layout(t, ws);
   const uint64_t R = t.n_records;
   const uint32_t K = t.n_kernels, B = t.n_bb;
-  uint32_t bbits = 1;
-  while ((1u << bbits) < B) ++bbits;
-  uint32_t kbits = 1;
-  while ((1ull << kbits) < (uint64_t)K) ++kbits;
   cudaMemsetAsync(first_stable, 0xFF, sizeof(int64_t) * (size_t)K * B, s);
   if (dur) cudaMemsetAsync(dur, 0, sizeof(uint64_t) * (size_t)K * B, s);
   cudaMemsetAsync(L.misc, 0, 64, s);
-  note_launch(), k_rec_chunks<<<1, 1024, 0, s>>>(t.kernel_rec_off, K, R, L.coff, err);
+  const uint64_t chunk = L.onepass ? JOB : REC_CHUNK;
+  note_launch(), k_rec_chunks<<<1, 1024, 0, s>>>(t.kernel_rec_off, K, R, chunk, L.coff, err);
   if (R > 0) {
-    uint64_t jobs_ub = ceil_div(R, REC_CHUNK) + K;
-    unsigned grid = (unsigned)umin64(jobs_ub, (uint64_t)num_sms * 8);
-    note_launch(), k_rec_prep<<<grid, 256, 0, s>>>(t, L.coff, bbits, L.key0, err);
-    // radix passes over kbits + bbits bits
-    uint32_t bits = kbits + bbits;
-    uint64_t* kin = L.key0; uint64_t* kout = L.key1;
-    uint32_t* vin = L.val0; uint32_t* vout = L.val1;
-    int pass = 0;
-    for (uint32_t sh = 0; sh < bits; sh += RBITS, ++pass) {
-      note_launch(), k_radix_up<<<(unsigned)L.n_tiles, RT, 0, s>>>(kin, R, sh, L.hist, L.n_tiles);
-      scan_u32(L.hist, L.hist, (uint64_t)RNB * L.n_tiles, L.bsum, L.misc + 4, s);
-      note_launch(), k_radix_down<<<(unsigned)L.n_tiles, RT, 0, s>>>(kin, vin, R, sh, L.hist, L.n_tiles, kout, vout, pass == 0);
-      uint64_t* tk = kin; kin = kout; kout = tk;
-      uint32_t* tv = vin; vin = vout; vout = tv;
+    uint32_t* idx;
+    if (L.onepass) {
+      // 1-2. per-job histograms -> bin-major scan -> stable scatter of (issue, retire, index) into group order
+      unsigned gj = (unsigned)umin64(ceil_div(L.n_jobs, 8), (uint64_t)num_sms * 8);
+      cudaMemsetAsync(L.hist, 0, sizeof(uint32_t) * L.hn, s);
+      note_launch(), k_job_hist<<<gj, 256, 0, s>>>(t, L.coff, L.n_jobs, L.hist);
+      scan_u32(L.hist, L.hist, L.hn, L.bsum, L.misc + 4, s);
+      note_launch(), k_job_scatter<<<gj, 256, 0, s>>>(t, L.coff, L.n_jobs, L.hist, L.X, L.Y, L.val0, err);
+      note_launch(), k_job_gstart<<<(unsigned)umin64(ceil_div(L.gcap + 1, 256), (uint64_t)num_sms * 8), 256, 0, s>>>(
+          L.hist, L.coff, K, B, L.n_jobs, R, L.gstart, L.misc + 0);
+      idx = L.val0;
+    } else {
+      uint64_t jobs_ub = ceil_div(R, REC_CHUNK) + K;
+      unsigned grid = (unsigned)umin64(jobs_ub, (uint64_t)num_sms * 8);
+      cudaMemsetAsync(L.key0, 0, sizeof(uint64_t) * R, s);  // keys stay < K*B even if offsets are malformed
+      note_launch(), k_rec_prep<<<grid, 256, 0, s>>>(t, L.coff, L.key0, err);
+      // radix passes over the bits of the composite key b*K + k
+      uint32_t bits = 1;
+      while ((1ull << bits) < L.gcap) ++bits;
+      uint64_t* kin = L.key0; uint64_t* kout = L.key1;
+      uint32_t* vin = L.val0; uint32_t* vout = L.val1;
+      int pass = 0;
+      for (uint32_t sh = 0; sh < bits; sh += RBITS, ++pass) {
+        note_launch(), k_radix_up<<<(unsigned)L.n_tiles, RT, 0, s>>>(kin, R, sh, L.hist, L.n_tiles);
+        scan_u32(L.hist, L.hist, (uint64_t)RNB * L.n_tiles, L.bsum, L.misc + 4, s);
+        note_launch(), k_radix_down<<<(unsigned)L.n_tiles, RT, 0, s>>>(kin, vin, R, sh, L.hist, L.n_tiles, kout, vout, pass == 0);
+        uint64_t* tk = kin; kin = kout; kout = tk;
+        uint32_t* tv = vin; vin = vout; vout = tv;
+      }
+      unsigned gR = (unsigned)ceil_div(R + 1, 256);
+      note_launch(), k_gather<<<gR, 256, 0, s>>>(vin, R, t.issue, t.retire, L.X, L.Y);
+      note_launch(), k_fill_gstart<<<gR, 256, 0, s>>>(kin, R, L.gcap, L.gstart);
+      note_launch(), k_set_u32<<<1, 1, 0, s>>>(L.misc + 0, (uint32_t)L.gcap);
+      idx = vin;
     }
-    // sorted: kin / vin
-    unsigned gR = (unsigned)ceil_div(R, 256);
-    note_launch(), k_gather<<<gR, 256, 0, s>>>(vin, R, t.issue, t.retire, L.X, L.Y);
-    note_launch(), k_heads<<<gR, 256, 0, s>>>(kin, R, L.flag);
-    scan_u32(L.flag, L.flag, R, L.bsum, L.misc + 0, s);  // misc[0] = G
-    note_launch(), k_group_start<<<gR, 256, 0, s>>>(kin, R, L.flag, L.gstart);
-    note_launch(), k_group_end<<<1, 1, 0, s>>>(L.gstart, L.misc + 0, R);
-    note_launch(), k_work_count<<<(unsigned)ceil_div(L.gcap, 256), 256, 0, s>>>(L.gstart, L.misc + 0, 2 * p.window_n, L.nwork,
-                                                                 L.gfirst, L.gcap);
-    scan_u32(L.nwork, L.nwork, L.gcap, L.bsum, L.misc + 1, s);  // misc[1] = work items
+    // 3-4. runs per group, windowed exact test
+    note_launch(), k_work_count<<<(unsigned)umin64(ceil_div(L.gcap, 256), (uint64_t)num_sms * 4), 256, 0, s>>>(
+        L.gstart, L.misc + 0, 2 * p.window_n, L.nruns, L.gfirst, L.misc + 1);
     WinArgs wa{};
-    wa.X = L.X; wa.Y = L.Y; wa.gstart = L.gstart; wa.G = L.misc + 0; wa.work_off = L.nwork; wa.n_work = L.misc + 1;
-    wa.gcap = L.gcap; wa.n = p.window_n; wa.dnum = p.delta_num; wa.dden = p.delta_den; wa.gfirst = L.gfirst;
-    note_launch(), k_window<<<(unsigned)num_sms * 4, WT, 0, s>>>(wa);
-    note_launch(), k_finish<<<(unsigned)ceil_div(L.gcap * 32, 256), 256, 0, s>>>(kin, vin, L.X, L.Y, L.gstart, L.misc + 0, L.gfirst,
-                                                                 t.kernel_rec_off, bbits, B, p.window_n,
-                                                                 first_stable, dur);
+    wa.X = L.X; wa.Y = L.Y; wa.gstart = L.gstart; wa.G = L.misc + 0; wa.nruns = L.nruns; wa.maxr = L.misc + 1;
+    wa.ticket = L.misc + 2; wa.n = p.window_n; wa.dnum = p.delta_num; wa.dden = p.delta_den; wa.gfirst = L.gfirst;
+    note_launch(), k_window<<<(unsigned)num_sms * 2, WT, 0, s>>>(wa);
+    // 5. outputs
+    note_launch(), k_finish<<<(unsigned)umin64(ceil_div(L.gcap * 32, 256), (uint64_t)num_sms * 8), 256, 0, s>>>(
+        idx, L.X, L.Y, L.misc + 0, L.gfirst, t.kernel_rec_off, K, B, p.window_n, first_stable, dur);
     unsigned gk = (unsigned)umin64(K, (uint64_t)num_sms * 8);
-    note_launch(), k_switch<<<gk ? gk : 1, 256, 0, s>>>(kin, L.gstart, L.misc + 0, L.gfirst, first_stable, kbb, K, B, bbits,
-                                         p.rate_num, p.rate_den, switch_at);
+    note_launch(), k_switch<<<gk ? gk : 1, 256, 0, s>>>(first_stable, kbb, K, B, p.rate_num, p.rate_den, switch_at);
   } else {
     cudaMemsetAsync(switch_at, 0xFF, sizeof(int64_t) * K, s);
   }

@@ -229,3 +229,52 @@ def test_stable_errors(ph):
     with pytest.raises(PhotonError) as ei:
         check_stable(ph, tm, np.ones((1, 1), np.uint64), 2)
     assert ei.value.code == -3 and ei.value.index == 1
+
+
+def test_stable_late_multirun(ph):
+    # groups that stabilise only after many 8192-position runs, never stabilise, or stabilise at once, interleaved
+    # in one kernel (and repeated over 40 kernels so the ticket batches hold > 32 groups)
+    rng = np.random.default_rng(11)
+    offs, bbs, iss, ret = [0], [], [], []
+    for k in range(40):
+        L = 3000 + 700 * k
+        late = L // 2 + 5 * k
+        n_rec = 3 * L
+        x = np.cumsum(rng.integers(1, 50, n_rec)).astype(np.uint64) + np.uint64(10 ** 6 * k)
+        bb = np.tile(np.arange(3, dtype=np.uint16), L)
+        dur = np.empty(n_rec, np.uint64)
+        j = np.repeat(np.arange(L), 3)
+        dur[0::3] = np.where(j[0::3] < late, rng.integers(1, 5000, L), 100)          # late stabiliser
+        dur[1::3] = rng.integers(1, 5000, L)                                          # never
+        dur[2::3] = 200                                                                # immediate
+        y = x + dur
+        order = np.argsort(y, kind="stable")
+        bbs.append(bb[order]); iss.append(x[order]); ret.append(y[order])
+        offs.append(offs[-1] + n_rec)
+    tm = tg.Timing(kernel_rec_off=np.array(offs, np.uint64), bb=np.concatenate(bbs), issue=np.concatenate(iss),
+                   retire=np.concatenate(ret), n_bb=3)
+    kbb = np.ones((40, 3), np.uint64)
+    fs = check_stable(ph, tm, kbb, 256)
+    assert (fs[:, 0] > 0).all() and (fs[:, 2] >= 0).all()
+
+
+@pytest.mark.parametrize("B", [256, 257, 1000])
+def test_stable_many_bb(ph, B):
+    # B <= 256 takes the one-pass job multisplit, B > 256 the composite-key radix sort: both must agree with the oracle
+    rng = np.random.default_rng(B)
+    offs, bbs, iss, ret = [0], [], [], []
+    for k in range(6):
+        n_rec = 30000 + 9000 * k
+        x = np.cumsum(rng.integers(1, 20, n_rec)).astype(np.uint64)
+        bb = (rng.zipf(1.3, n_rec) % B).astype(np.uint16)
+        dur = np.where(rng.random(n_rec) < 0.9, 40 + (bb.astype(np.uint64) % 7), rng.integers(1, 400, n_rec))
+        y = x + dur.astype(np.uint64)
+        o = np.argsort(y, kind="stable")
+        bbs.append(bb[o]); iss.append(x[o]); ret.append(y[o])
+        offs.append(offs[-1] + n_rec)
+    offs.insert(3, offs[2])  # an empty kernel in the middle
+    tm = tg.Timing(kernel_rec_off=np.array(offs, np.uint64), bb=np.concatenate(bbs), issue=np.concatenate(iss),
+                   retire=np.concatenate(ret), n_bb=B)
+    kbb = rng.integers(0, 1000, (7, B)).astype(np.uint64)
+    fs = check_stable(ph, tm, kbb, 16)
+    assert (fs >= 0).sum() > 10
