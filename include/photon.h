@@ -74,7 +74,8 @@ enum {
   PHOTON_PROF_SCAN = 6,         /* A4 pair filter + exact check                                          */
   PHOTON_PROF_RESOLVE = 7,      /* A4 launch-order resolution                                            */
   PHOTON_PROF_STABLE = 8,       /* A5 (all kernels)                                                      */
-  PHOTON_PROF_N = 9
+  PHOTON_PROF_PREP = 9,         /* photon_warp_group set-up: table clear, BB table, work items            */
+  PHOTON_PROF_N = 10
 };
 PHOTON_API int photon_profile(photon_ctx *ctx, int enable);
 PHOTON_API int photon_profile_read(photon_ctx *ctx, void *stream, double *ms /*[PHOTON_PROF_N] HOST*/,

@@ -55,7 +55,7 @@ class StableParams(ctypes.Structure):
 
 
 TYPE_ROW_BYTES = 88  # photon_type_row
-PROF_SECTIONS = ["bbv_fused", "bbv", "kbb", "group_unfused", "canon", "sig", "scan", "resolve", "stable"]
+PROF_SECTIONS = ["bbv_fused", "bbv", "kbb", "group_unfused", "canon", "sig", "scan", "resolve", "stable", "prep"]
 
 # (name, restype, argtypes) — mirrors include/photon.h
 _SIGS = [

@@ -95,7 +95,7 @@ struct BbvWs {
   DevErr* err;
   uint32_t* tbl;        // [P2] packed (len, bin) table
   uint32_t* max_len;
-  uint32_t* tile_k0;    // [n_tiles]
+  ItemTable it;         // work items of the streaming pass
   uint64_t* kchunk;     // [K+1] kernel_bb_insts job prefix
   size_t bytes;
 };
@@ -106,7 +106,15 @@ BbvWs bbv_layout(const photon_trace* t, void* base) {
   uint32_t P2 = next_pow2_u32(t->n_bb < 16 ? 16 : t->n_bb);
   w.tbl = c.take<uint32_t>(P2);
   w.max_len = c.take<uint32_t>(4);
-  w.tile_k0 = c.take<uint32_t>(bbv_n_tiles(t->n_warps) + 1);
+  w.it.xs = kItemShift;
+  w.it.cap = bbv_item_cap(t->n_warps, t->n_events, kItemShift);
+  w.it.w0 = c.take<uint64_t>(w.it.cap + 1);
+  w.it.k0 = c.take<uint32_t>(w.it.cap);
+  w.it.boff = c.take<uint32_t>(bbv_n_blocks(t->n_warps) + 1);
+  w.it.split = c.take<uint32_t>(bbv_n_blocks(t->n_warps) + 1);
+  w.it.nsub = c.take<uint32_t>(bbv_n_blocks(t->n_warps) + 1);
+  w.it.part = c.take<uint32_t>(bbv_n_blocks(t->n_warps) / 256 + 2);
+  w.it.n = c.take<uint32_t>(4);
   w.kchunk = c.take<uint64_t>((size_t)t->n_kernels + 1);
   w.bytes = c.off + 256;
   return w;
@@ -124,7 +132,7 @@ void carve_entries(Carver& c, uint64_t n_tiles, uint64_t W, uint64_t ovf_cap, Ti
   te.ovf = c.take<TileEntry>(ovf_cap);
   te.ovf_slot = c.take<uint32_t>(ovf_cap);
   te.ovf_count = c.take<uint64_t>(1);
-  te.lid = c.take<uint16_t>(W + 1);
+  te.gid = c.take<uint32_t>(W + 1);
 }
 
 uint64_t ht_capacity(uint64_t hint, uint64_t W) {
@@ -164,7 +172,7 @@ struct GroupWs {
 GroupWs group_layout(const photon_trace* t, uint64_t hint, void* base, size_t ws_bytes) {
   GroupWs g;
   g.b = bbv_layout(t, base);
-  const uint64_t nt = bbv_n_tiles(t->n_warps);
+  const uint64_t nt = g.b.it.cap;
   uint64_t cap = ht_capacity(hint, t->n_warps);
   if (base && ws_bytes) {
     // the capacity actually used is the largest power of two that fits (callers may pass a larger workspace)
@@ -183,6 +191,7 @@ GroupWs group_layout(const photon_trace* t, uint64_t hint, void* base, size_t ws
   c.off = g.b.bytes;
   carve_ht(c, cap, t->n_kernels, g.h);
   carve_entries(c, nt, t->n_warps, cap, g.te);
+  g.te.n_items = g.b.it.n;
   g.bytes = c.off + 256;
   return g;
 }
@@ -377,10 +386,10 @@ int photon_bbv_build(photon_ctx* ctx, const photon_trace* t, void* ws, size_t ws
   TraceDev d = to_dev(t);
   CK(cudaMemsetAsync(w.err, 0, sizeof(DevErr), s), "memset");
   CK(launch_validate_offsets(d, w.err, s), "validate");
-  CK(launch_table_prep(d, w.tbl, w.max_len, nullptr, w.err, s), "table");
+  CK(launch_table_prep(d, w.tbl, w.max_len, w.it, nullptr, w.err, s), "table");
   if (warp_bbv16 || warp_insts) {
     ProfScope ps(ctx, PHOTON_PROF_BBV, s);
-    CK(launch_bbv(d, w.tbl, w.max_len, nullptr, warp_bbv16, warp_insts, nullptr, w.err, ctx->num_sms, s), "bbv");
+    CK(launch_bbv(d, w.tbl, w.max_len, w.it, warp_bbv16, warp_insts, nullptr, w.err, ctx->num_sms, s), "bbv");
   }
   if (kernel_bb_insts) {
     ProfScope ps(ctx, PHOTON_PROF_KBB, s);
@@ -415,20 +424,23 @@ int photon_warp_group(photon_ctx* ctx, const photon_trace* t, const uint32_t* wa
   TraceDev d = to_dev(t);
   DevErr* err = g.b.err;
   CK(cudaMemsetAsync(err, 0, sizeof(DevErr), s), "memset");
-  CK(launch_ht_clear(g.h.ht, s), "ht_clear");
-  CK(cudaMemsetAsync(g.te.ovf_count, 0, 8, s), "memset");
-  CK(launch_validate_offsets(d, err, s), "validate");
-  CK(launch_table_prep(d, g.b.tbl, g.b.max_len, g.b.tile_k0, err, s), "table");
+  {
+    ProfScope ps(ctx, PHOTON_PROF_PREP, s);
+    CK(launch_ht_clear(g.h.ht, s), "ht_clear");
+    CK(cudaMemsetAsync(g.te.ovf_count, 0, 8, s), "memset");
+    CK(launch_validate_offsets(d, err, s), "validate");
+    CK(launch_table_prep(d, g.b.tbl, g.b.max_len, g.b.it, &g.te, err, s), "table");
+  }
   if (warp_bbv16) {
     ProfScope ps(ctx, PHOTON_PROF_GROUP_UNFUSED, s);
-    CK(launch_group_from_bbv(d, warp_bbv16, g.b.tile_k0, g.te, err, s), "group_from_bbv");
+    CK(launch_group_from_bbv(d, warp_bbv16, g.b.it, g.te, err, s), "group_from_bbv");
   } else {
     ProfScope ps(ctx, PHOTON_PROF_BBV_FUSED, s);
-    CK(launch_bbv(d, g.b.tbl, g.b.max_len, g.b.tile_k0, nullptr, nullptr, &g.te, err, ctx->num_sms, s), "bbv_fused");
+    CK(launch_bbv(d, g.b.tbl, g.b.max_len, g.b.it, nullptr, nullptr, &g.te, err, ctx->num_sms, s), "bbv_fused");
   }
   {
     ProfScope ps(ctx, PHOTON_PROF_CANON, s);
-    CK(launch_entries_insert(g.te, bbv_n_tiles(t->n_warps), g.h.ht, err, s), "insert");
+    CK(launch_entries_insert(g.te, g.b.it.cap, g.h.ht, err, s), "insert");
     CK(launch_canonicalise(g.h.ht, t->n_kernels, t->kernel_warp_off, nullptr, *out, g.h.cw, err, ctx->num_sms, s),
        "canon");
     CK(launch_remap_entries(g.te, t->n_warps, g.h.cw.canon, out->warp_type, s), "remap");

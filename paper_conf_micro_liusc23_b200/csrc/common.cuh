@@ -73,15 +73,18 @@ __device__ __forceinline__ uint64_t mix64(uint64_t x) {
   x ^= x >> 33;
   return x;
 }
-// Bucketing hash only (equality is always verified on the full key): a sum of 32x32->64-bit products with distinct
-// odd multipliers (one IMAD.WIDE each) followed by a 64-bit finaliser.
+// Bucketing hash only (equality is always verified on the full key): a sum of products with distinct odd 64-bit
+// multipliers (two IMADs each, mod 2^64) followed by a 64-bit finaliser.
 __device__ __forceinline__ uint64_t hash_key(uint32_t k, const uint32_t* p) {
-  constexpr uint32_t M[17] = {0x9E3779B1u, 0x85EBCA77u, 0xC2B2AE3Du, 0x27D4EB2Fu, 0x165667B1u, 0xD3A2646Du,
-                              0xFD7046C5u, 0xB55A4F09u, 0x7FEB352Du, 0x846CA68Bu, 0xE6546B65u, 0x4CF5AD43u,
-                              0x2545F491u, 0x9E485565u, 0xEF1D6B47u, 0x5851F42Du, 0x14057B7Fu};
+  constexpr uint64_t M[17] = {0x9E3779B97F4A7C15ull, 0xC2B2AE3D27D4EB4Full, 0x165667B19E3779F9ull,
+                              0xD6E8FEB86659FD93ull, 0xFF51AFD7ED558CCDull, 0xC4CEB9FE1A85EC53ull,
+                              0x94D049BB133111EBull, 0xBF58476D1CE4E5B9ull, 0x2545F4914F6CDD1Dull,
+                              0x5851F42D4C957F2Dull, 0x14057B7EF767814Full, 0x7FB5D329728EA185ull,
+                              0x81DADEF4BC2DD44Dull, 0xA0761D6478BD642Full, 0xE7037ED1A0B428DBull,
+                              0x8EBC6AF09C88C6E3ull, 0x589965CC75374CC3ull};
   uint64_t h = (uint64_t)k * M[16] + 0x632BE59BD9B4E019ull;
 #pragma unroll
-  for (int j = 0; j < 16; ++j) h += (uint64_t)p[j] * M[j] + ((uint64_t)p[j] << (2 * j + 13));
+  for (int j = 0; j < 16; ++j) h += (uint64_t)p[j] * M[j];
   h = mix64(h);
   return h ? h : 1;
 }

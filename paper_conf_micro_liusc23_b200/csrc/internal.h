@@ -35,24 +35,43 @@ struct TileEntries {
   TileEntry* ovf;        // [ovf_cap]
   uint64_t* ovf_count;   // [1]
   uint64_t ovf_cap;
-  uint16_t* lid;         // [W] entry id of each warp within its tile
+  uint32_t* gid;         // [W] per warp: its entry's index in ent/tile_slot (item * per_tile + e), or
+                         // 0x80000000 | overflow index
   uint32_t* tile_slot;   // [n_tiles * per_tile] hash-table slot of each entry
   uint32_t* ovf_slot;    // [ovf_cap]
   uint32_t per_tile;
+  const uint32_t* n_items;  // device item count (tile_n is written for items below it)
 };
 
-uint64_t bbv_n_tiles(uint64_t W);
+// Work items of the streaming pass: the warps of each 256-warp block are split at 2^xs-event windows of the block
+// (an item = the warps whose first event falls in one window), so an item holds <= 256 warps and about 2^xs events
+// plus its last warp's length; the persistent CTAs take items from a counter (dynamic balance).
+struct ItemTable {
+  uint64_t* w0;     // [cap + 1] first warp of each item (w0[n] = W)
+  uint32_t* k0;     // [cap] kernel of each item's first warp
+  uint32_t* boff;   // [n_blocks + 1] first item of each block
+  uint32_t* split;  // [n_blocks] blocks with more than one item
+  uint32_t* nsub;   // [n_blocks] items per block
+  uint32_t* part;   // [n_blocks / 256 + 1] per-CTA item totals (scanned)
+  uint32_t* n;      // [4]: [0] item count, [1] work counter, [2] split blocks
+  uint64_t cap;
+  uint32_t xs;
+};
+uint64_t bbv_n_blocks(uint64_t W);
+uint64_t bbv_item_cap(uint64_t W, uint64_t E, uint32_t xs);
+constexpr uint32_t kItemShift = 15;  // 32K-event windows
 // packed per-BB table (len << 14 | bin << 10; bit 0 marks ids in [B, P2)), P2 = next pow2 >= B; tile -> kernel
 size_t bbv_table_bytes(uint32_t B);
-cudaError_t launch_table_prep(const TraceDev& t, uint32_t* tbl, uint32_t* max_len, uint32_t* tile_k0, DevErr* err,
-                              cudaStream_t s);
+// BB table + work items (+ zeroed per-item entry counts when te is given)
+cudaError_t launch_table_prep(const TraceDev& t, uint32_t* tbl, uint32_t* max_len, const ItemTable& it,
+                              const TileEntries* te, DevErr* err, cudaStream_t s);
 cudaError_t launch_validate_offsets(const TraceDev& t, DevErr* err, cudaStream_t s);
 // streaming K1 (+ fused K2a de-dup when te != nullptr)
-cudaError_t launch_bbv(const TraceDev& t, const uint32_t* tbl, const uint32_t* max_len, const uint32_t* tile_k0,
+cudaError_t launch_bbv(const TraceDev& t, const uint32_t* tbl, const uint32_t* max_len, const ItemTable& it,
                        uint32_t* warp_bbv16, uint64_t* warp_insts, const TileEntries* te, DevErr* err, int num_sms,
                        cudaStream_t s);
 // K2a de-dup from materialised BBVs (unfused path)
-cudaError_t launch_group_from_bbv(const TraceDev& t, const uint32_t* warp_bbv16, const uint32_t* tile_k0,
+cudaError_t launch_group_from_bbv(const TraceDev& t, const uint32_t* warp_bbv16, const ItemTable& it,
                                   const TileEntries& te, DevErr* err, cudaStream_t s);
 cudaError_t launch_kernel_bb_insts(const TraceDev& t, const uint32_t* tbl, uint64_t* kbb, uint64_t* kchunk_off,
                                    DevErr* err, int num_sms, cudaStream_t s);

@@ -46,22 +46,32 @@ struct BbvArgs {
   const uint16_t* bb;
   const uint32_t* tbl;
   const uint32_t* max_len;
-  const uint32_t* tile_k0;  // [n_tiles] kernel of each tile's first warp
+  const uint32_t* tile_k0;  // [cap] kernel of each item's first warp
+  const uint64_t* item_w0;  // [cap + 1] first warp of each item
+  const uint32_t* n_items;  // device item count
+  uint32_t* counter;        // dynamic item counter (zeroed before the launch)
   uint32_t K, B, P2;
   uint64_t W, E;
   uint32_t* warp_bbv16;
   uint64_t* warp_insts;
   TileEntries te;           // fused grouping outputs (te.tile_n == nullptr => not fused)
   DevErr* err;
-  uint64_t n_tiles;
+  uint64_t n_tiles;         // item capacity
 };
+
+// warps [w0, w1) of item it (clamped: malformed offsets stay memory-safe; they are latched by k_items_fill)
+__device__ __forceinline__ void item_range(const BbvArgs& a, uint64_t it, uint64_t& w0, uint64_t& w1) {
+  w0 = umin64(a.item_w0[it], a.W);
+  const uint64_t x = umax64(a.item_w0[it + 1], w0);
+  w1 = umin64(umin64(x, w0 + TPB), a.W);
+}
 
 constexpr size_t kColBytes = (size_t)16 * COLB;
 constexpr size_t kStageBytes = (size_t)CAPE * 2;
 constexpr size_t kOffsBytes = (TPB + 4) * 8;
 constexpr size_t kLocalBytes = LSLOTS * (8 + 4 + 4 + 4 + 4);
 constexpr size_t kMiscBytes = 256;
-constexpr size_t kKidBytes = TPB * 4 + (TPB + 8) * 2;
+constexpr size_t kKidBytes = TPB * 4 + (TPB + 4) * 8;
 
 __host__ __device__ constexpr size_t bbv_smem_bytes(uint32_t tbl_entries) {
   return 2 * kColBytes + kStageBytes + kOffsBytes + 16 + kLocalBytes + kMiscBytes + kKidBytes +
@@ -81,7 +91,9 @@ struct Smem {
   uint32_t* lent;    // [LSLOTS] dense local entry id
   uint32_t* misc;    // [64]: 0 n_entries; [2..3] u64 overflow base
   uint32_t* kid;     // [TPB] kernel of each thread's warp
-  uint16_t* nxt;     // [TPB+8] next non-empty warp after each (virtual) warp of the tile
+  uint2* info;       // [TPB+4] per (virtual) warp sp of the tile, for the current chunk: x = column (smem byte
+                     // offset) of nxt(sp) | end of nxt(sp) << 16, y = nxt(sp) | start of sp << 16 (chunk-relative
+                     // event offsets clamped to [0, LIM]; nxt = next non-empty warp, the tail sentinel maps to itself)
   uint32_t* tbl;     // [P2]
 };
 
@@ -99,8 +111,8 @@ __device__ __forceinline__ Smem carve(uint8_t* s) {
   m.lent = m.lminw + LSLOTS;
   m.misc = m.lent + LSLOTS;
   m.kid = m.misc + kMiscBytes / 4;
-  m.nxt = (uint16_t*)(m.kid + TPB);
-  m.tbl = (uint32_t*)(m.nxt + TPB + 8);
+  m.info = (uint2*)(m.kid + TPB);
+  m.tbl = (uint32_t*)(m.info + TPB + 4);
   return m;
 }
 
@@ -125,20 +137,31 @@ struct Acc {
     *p1 = h1 + l1;
     *p0 = h0 + (t0 >> LSH) + ((same && a0 == a1) ? l1 : 0u);
   }
-  // one 16-byte word: events j < bo into ca, j >= bo into cb.  All 8 table entries are loaded before any
-  // histogram cell is written (the compiler cannot hoist them past the stores itself), so the word costs four
-  // short load->add->store chains instead of four chains that each also wait for their table reads.
-  __device__ __forceinline__ void word(uint4 v, uint32_t bo, uint32_t* ca, uint32_t* cb) {
+  // a word whose events go to eight given columns (byte offsets from sbase)
+  __device__ __forceinline__ void word8(uint4 v, const uint32_t (&t)[8], const uint32_t (&c)[8], uint8_t* sbase) {
     raw |= v.x | v.y | v.z | v.w;
-    const uint32_t t0 = tbl[v.x & bmask], t1 = tbl[(v.x >> 16) & bmask];
-    const uint32_t t2 = tbl[v.y & bmask], t3 = tbl[(v.y >> 16) & bmask];
-    const uint32_t t4 = tbl[v.z & bmask], t5 = tbl[(v.z >> 16) & bmask];
-    const uint32_t t6 = tbl[v.w & bmask], t7 = tbl[(v.w >> 16) & bmask];
-    orr |= (t0 | t1 | t2 | t3) | (t4 | t5 | t6 | t7);
-    pair(t0, t1, bo > 0 ? ca : cb, bo > 1 ? ca : cb, bo != 1);
-    pair(t2, t3, bo > 2 ? ca : cb, bo > 3 ? ca : cb, bo != 3);
-    pair(t4, t5, bo > 4 ? ca : cb, bo > 5 ? ca : cb, bo != 5);
-    pair(t6, t7, bo > 6 ? ca : cb, bo > 7 ? ca : cb, bo != 7);
+    orr |= (t[0] | t[1] | t[2] | t[3]) | (t[4] | t[5] | t[6] | t[7]);
+#pragma unroll
+    for (int j = 0; j < 8; j += 2)
+      pair(t[j], t[j + 1], (uint32_t*)(sbase + c[j]), (uint32_t*)(sbase + c[j + 1]), c[j] == c[j + 1]);
+  }
+  // the 8 table entries of a 16-byte word (loaded one word ahead of its accumulation: the table is read-only, so
+  // issuing these before the previous word's cell stores is safe, and hides their latency)
+  __device__ __forceinline__ void lookup(uint4 v, uint32_t (&t)[8]) const {
+    t[0] = tbl[v.x & bmask]; t[1] = tbl[(v.x >> 16) & bmask];
+    t[2] = tbl[v.y & bmask]; t[3] = tbl[(v.y >> 16) & bmask];
+    t[4] = tbl[v.z & bmask]; t[5] = tbl[(v.z >> 16) & bmask];
+    t[6] = tbl[v.w & bmask]; t[7] = tbl[(v.w >> 16) & bmask];
+  }
+  // one 16-byte word with its table entries: events j < bo into ca, j >= bo into cb (four load->add->store
+  // steps of two events each)
+  __device__ __forceinline__ void word(uint4 v, const uint32_t (&t)[8], uint32_t bo, uint32_t* ca, uint32_t* cb) {
+    raw |= v.x | v.y | v.z | v.w;
+    orr |= (t[0] | t[1] | t[2] | t[3]) | (t[4] | t[5] | t[6] | t[7]);
+    pair(t[0], t[1], bo > 0 ? ca : cb, bo > 1 ? ca : cb, bo != 1);
+    pair(t[2], t[3], bo > 2 ? ca : cb, bo > 3 ? ca : cb, bo != 3);
+    pair(t[4], t[5], bo > 4 ? ca : cb, bo > 5 ? ca : cb, bo != 5);
+    pair(t[6], t[7], bo > 6 ? ca : cb, bo > 7 ? ca : cb, bo != 7);
   }
 };
 
@@ -247,8 +270,8 @@ __device__ void tile_group(const BbvArgs& a, const Smem& m, uint64_t t, uint64_t
   // members of a warp group take the leader's entry
   const uint32_t from_leader = __shfl_sync(0xffffffffu, my_ent, leader);
   if (valid) {
-    uint32_t e = (lane == leader || !eq) ? my_ent : from_leader;
-    a.te.lid[w0 + tid] = (uint16_t)(e & 0xFFFFu);
+    const uint32_t e = ((lane == leader || !eq) ? my_ent : from_leader) & 0x7FFFFFFFu;
+    a.te.gid[w0 + tid] = e < M ? (uint32_t)(t * M + e) : (0x80000000u | (uint32_t)(*ovf_base + (e - M)));
   }
   __syncthreads();
   for (int i = tid; i < LSLOTS; i += TPB) {
@@ -272,20 +295,19 @@ __device__ __forceinline__ void stage_chunk(const BbvArgs& a, const Smem& m, uin
   }
 }
 
-// Chunk sequence of the CTA: tiles blockIdx.x, +gridDim.x, ...; tile events widened to words [A, Z), split into
-// CAPE chunks; tiles without events have no chunk.
+// An item's events widened to words [A, Z), split into CAPE chunks; items without events have no chunk.
 struct Cursor {
   uint64_t t, A, Z, c, nch;
   bool valid;
 };
 __device__ __forceinline__ void cursor_tile(const BbvArgs& a, Cursor& u, uint64_t t) {
   u.t = t;
-  u.valid = t < a.n_tiles;
+  u.valid = true;
   u.c = 0;
   u.nch = 0;
   u.A = u.Z = 0;
-  if (!u.valid) return;
-  uint64_t w0 = t * TPB, w1 = umin64(a.W, w0 + TPB);
+  uint64_t w0, w1;
+  item_range(a, t, w0, w1);
   uint64_t te = umin64(a.weo[w1], a.E), ts = umin64(a.weo[w0], te);  // clamped: bad offsets stay memory-safe
   if (te <= ts) return;
   u.A = ts & ~7ull;
@@ -313,44 +335,75 @@ __global__ void __launch_bounds__(TPB, 2) k_bbv(BbvArgs a) {
   const uint32_t max_len = *a.max_len;
   const uint64_t E8 = a.E & ~7ull;
 
-  // producer cursor (thread 0): one chunk ahead of the consumers
-  Cursor pc;
+  // dynamic schedule: thread 0 takes items from the counter (skipping warp-less ones) one item ahead of the
+  // consumers; sched[0] / sched[1] publish the first / next item
+  const uint64_t NI = umin64(*a.n_items, a.n_tiles);
+  uint32_t* const sched = m.misc + 8;
+  __syncthreads();  // misc zeroed before thread 0 publishes the schedule
+  auto grab = [&]() -> uint64_t { return umin64(atomicAdd(a.counter, 1u), NI); };  // items may be warp-less
+  // producer (thread 0): the chunk in flight on the mbarrier, if any
+  uint64_t fl_t = ~0ull, fl_c = 0;
   if (tid == 0) {
-    cursor_tile(a, pc, blockIdx.x);
-    while (pc.valid && pc.nch == 0) cursor_tile(a, pc, pc.t + gridDim.x);
-    if (pc.valid) stage_chunk(a, m, pc.A, umin64(pc.A + CAPE, pc.Z), E8);
+    const uint64_t x = grab();
+    sched[0] = (uint32_t)x;
+    sched[1] = (uint32_t)(x < NI ? grab() : NI);
+    if (x < NI) {
+      Cursor pc;
+      cursor_tile(a, pc, x);
+      if (pc.nch) {
+        stage_chunk(a, m, pc.A, umin64(pc.A + CAPE, pc.Z), E8);
+        fl_t = x;
+        fl_c = 0;
+      }
+    }
   }
   uint32_t phase = 0;
 
   Acc acc;
   acc.tbl = SMEM_TBL ? m.tbl : a.tbl;
   acc.bmask = bmask;
+  __syncthreads();
 
-  uint64_t t = blockIdx.x;
-  uint64_t my_off = 0, last_off = 0;  // weo[w0 + tid] (clamped) and weo[w1] of the current tile
-  if (t < a.n_tiles) {
-    uint64_t w0 = t * TPB, nw = umin64(a.W, w0 + TPB) - w0;
+  uint64_t t = sched[0], tn = sched[1];
+  uint64_t my_off = 0, last_off = 0;  // weo[w0 + tid] (clamped) and weo[w1] of the current item
+  uint32_t my_k = 0;                  // kernel of the item's first warp (fused path), prefetched an item ahead
+  uint64_t my_kb = ~0ull;             // start of the kernel after it
+  if (t < NI) {
+    uint64_t w0, w1;
+    item_range(a, t, w0, w1);
+    const uint64_t nw = w1 - w0;
     my_off = a.weo[w0 + umin64((uint64_t)tid, nw)];
     if (tid == 0) last_off = a.weo[w0 + nw];
+    if (fused) {
+      my_k = a.tile_k0[t];
+      my_kb = my_k + 1 < a.K ? a.kwo[my_k + 1] : ~0ull;
+    }
   }
   __syncthreads();
 
-  while (t < a.n_tiles) {
-    const uint64_t w0 = t * TPB, w1 = umin64(a.W, w0 + TPB);
+  while (t < NI) {
+    uint64_t w0, w1;
+    item_range(a, t, w0, w1);
     const uint32_t nw = (uint32_t)(w1 - w0);
     const uint64_t w = w0 + tid;
     const bool valid = w < w1;
-    // o[1 + v] = start of warp v, o[nw + 1] = tile end; o[0] / o[nw + 2] = word-aligned bounds (virtual warps)
+    // o[1 + v] = start of warp v, o[nw + 1] = item end; o[0] / o[nw + 2] = word-aligned bounds (virtual warps)
     if ((uint32_t)tid <= nw) m.offs[1 + tid] = my_off;
     if (tid == 0) {
       m.offs[1 + nw] = last_off;
     }
-    const uint64_t tn = t + gridDim.x;
     uint64_t nx_off = 0, nx_last = 0;
-    if (tn < a.n_tiles) {
-      uint64_t n0 = tn * TPB, nn = umin64(a.W, n0 + TPB) - n0;
+    uint32_t nx_k = 0;
+    // the item after next: issued now, its value is only read at this item's end (latency hidden)
+    uint32_t x_after = 0;
+    if (tid == 0 && tn < NI) x_after = atomicAdd(a.counter, 1u);
+    if (tn < NI) {
+      uint64_t n0, n1;
+      item_range(a, tn, n0, n1);
+      const uint64_t nn = n1 - n0;
       nx_off = a.weo[n0 + umin64((uint64_t)tid, nn)];
       if (tid == 0) nx_last = a.weo[n0 + nn];
+      if (fused) nx_k = a.tile_k0[tn];
     }
     __syncthreads();
     // same clamping as cursor_tile (monotone offsets are validated per warp below: e < s latches ERANGE)
@@ -363,111 +416,156 @@ __global__ void __launch_bounds__(TPB, 2) k_bbv(BbvArgs a) {
     const uint64_t s = valid ? m.offs[1 + tid] : te, e = valid ? m.offs[2 + tid] : te;
     const uint64_t nch = te > ts ? ceil_div(Zt - At, CAPE) : 0;
     const uint32_t last = nw + 1;  // index of the virtual tail warp
-    {
-      // nxt[s'] = next non-empty (virtual) warp after s' (last = sentinel); o[0] / o[nw+2] taken from registers
-      auto O = [&](uint32_t i) -> uint64_t { return i == 0 ? At : (i == nw + 2 ? Zt : m.offs[i]); };
-      for (uint32_t sp = tid; sp <= last; sp += TPB) {
-        uint32_t x = sp + 1;
-        while (x < last && O(x + 1) == O(x)) ++x;
-        m.nxt[sp] = (uint16_t)(x < last ? x : last);
-      }
-    }
-    __syncthreads();
+    uint8_t* const sbase = smem_raw;
+    const uint32_t dummy_off = (uint32_t)((uint8_t*)(m.hist + DUMMY) - sbase);
     uint32_t* const headcol = m.head + tid;
-    uint32_t* const dummy = m.hist + DUMMY;
-    auto colof = [&](uint32_t sp) -> uint32_t* { return (sp == 0 || sp == last) ? dummy : m.hist + (sp - 1); };
+    const uint32_t head_off = (uint32_t)((uint8_t*)headcol - sbase);
     acc.raw = 0;
     acc.orr = 0;
+    auto colof = [&](uint32_t sp) -> uint32_t {
+      return (sp == 0 || sp == last) ? dummy_off : (uint32_t)((uint8_t*)(m.hist + (sp - 1)) - sbase);
+    };
+    // nxt(sp) = next non-empty (virtual) warp after sp (last = sentinel); o[0] / o[nw+2] taken from registers
+    auto O = [&](uint32_t i) -> uint64_t { return i == 0 ? At : (i == nw + 2 ? Zt : m.offs[i]); };
+    uint32_t nx[2] = {0u, 0u};
+#pragma unroll
+    for (int r = 0; r < 2; ++r) {
+      const uint32_t sp = tid + r * TPB;
+      if (sp <= last) {
+        uint32_t x = sp + 1;
+        while (x < last && O(x + 1) == O(x)) ++x;
+        nx[r] = x < last ? x : last;
+      }
+    }
     for (uint64_t c = 0; c < nch; ++c) {
       const uint64_t cs = At + c * CAPE, ce = umin64(cs + CAPE, Zt);
-      const uint64_t nwc = (ce - cs) >> 3;
+      const uint32_t nwc = (uint32_t)((ce - cs) >> 3);
+      // all positions in the loop are u32 offsets from the chunk start, clamped to [0, LIM]
+      const uint32_t LIM = (uint32_t)(ce - cs) + 8u;
+      auto rel = [&](uint64_t x) -> uint32_t {
+        return x <= cs ? 0u : (x - cs >= LIM ? LIM : (uint32_t)(x - cs));
+      };
+      // this chunk's warp table (the previous chunk's readers finished at its trailing barrier)
+#pragma unroll
+      for (int r = 0; r < 2; ++r) {
+        const uint32_t sp = tid + r * TPB;
+        if (sp <= last) {
+          const uint32_t n = nx[r];
+          const uint32_t endn = n != sp ? rel(O(n + 1)) : LIM + 8u;
+          m.info[sp] = make_uint2(colof(n) | (endn << 16), n | (rel(O(sp)) << 16));
+        }
+      }
+      __syncthreads();
+      if (tid == 0 && !(fl_t == t && fl_c == c)) {  // not prefetched (the previous item had no events)
+        stage_chunk(a, m, cs, ce, E8);
+        fl_t = t;
+        fl_c = c;
+      }
       mbar_wait(m.mbar, phase);
       phase ^= 1u;
       // my run of words [r0, r1) of the chunk
-      const uint64_t r0 = cs + 8 * (((uint64_t)tid * nwc) / TPB), r1 = cs + 8 * (((uint64_t)(tid + 1) * nwc) / TPB);
-      if (r0 < r1) {
-        // warp (with virtual ones) containing r0: last s' with o[s'] <= r0.  Start from the proportional guess
-        // and narrow a +-8 window around it when it brackets r0 (it usually does), else search everything.
+      const uint32_t q0 = 8u * ((tid * nwc) / TPB), qe = 8u * (((tid + 1) * nwc) / TPB);
+      if (q0 < qe) {
+        // warp (with virtual ones) containing q0: last sp with start(sp) <= q0.  Start from the proportional guess
+        // and narrow a +-8 window around it when it brackets q0 (it usually does), else search everything.
+        auto start = [&](uint32_t sp) -> uint32_t { return m.info[sp].y >> 16; };
         uint32_t lo = 0, hi = last;
         {
+          const uint64_t r0 = cs + q0;
           const float fr = (float)(r0 - At) / (float)(Zt - At);
           int g = (int)(fr * (float)(nw + 2));
           int glo = g - 8 < 0 ? 0 : g - 8, ghi = g + 8 > (int)last ? (int)last : g + 8;
-          if (m.offs[glo] <= r0 && m.offs[ghi + 1] > r0) { lo = (uint32_t)glo; hi = (uint32_t)ghi; }
+          if (start(glo) <= q0 && (ghi == (int)last || start(ghi + 1) > q0)) { lo = (uint32_t)glo; hi = (uint32_t)ghi; }
         }
         while (lo < hi) {
           uint32_t mid = (lo + hi + 1) >> 1;
-          if (m.offs[mid] <= r0) lo = mid; else hi = mid - 1;
+          if (start(mid) <= q0) lo = mid; else hi = mid - 1;
         }
-        // all positions below are u32 offsets from the chunk start, clamped to [0, LIM]
-        const uint32_t LIM = (uint32_t)(ce - cs) + 8u;
-        auto rel = [&](uint64_t x) -> uint32_t {
-          return x <= cs ? 0u : (x - cs >= LIM ? LIM : (uint32_t)(x - cs));
-        };
         uint32_t sg = lo;
-        uint32_t* col = (m.offs[sg] < r0) ? headcol : colof(sg);  // warp open at my run start -> HEAD
-        uint32_t nb = rel(m.offs[sg + 1]);
-        uint32_t sgn = m.nxt[sg];
-        uint32_t* coln = colof(sgn);
-        uint32_t nb2 = sgn != sg ? rel(m.offs[sgn + 1]) : LIM + 8u;
+        uint32_t col = (O(sg) < cs + q0) ? head_off : colof(sg);  // warp open at my run start -> HEAD
+        uint32_t nb = rel(O(sg + 1));
+        uint2 f = m.info[sg];
+        uint32_t sgn = f.y & 0xFFFFu, coln = f.x & 0xFFFFu, nb2 = f.x >> 16;
         const uint4* sb4 = (const uint4*)m.stage;
-        const uint32_t q0 = (uint32_t)(r0 - cs), qe = (uint32_t)(r1 - cs);
-        uint4 vnext = sb4[q0 >> 3];
-        for (uint32_t q = q0; q < qe; q += 8) {
-          const uint4 v = vnext;
-          if (q + 8 < qe) vnext = sb4[(q + 8) >> 3];  // next word read before this word's stores
+        // one word: v / t = this word and its table entries; vn / tn receive the next word's (software pipeline,
+        // unrolled by two below so the buffers swap roles without register moves)
+        auto step = [&](uint32_t q, const uint4& v, const uint32_t (&t)[8], uint4& vn, uint32_t (&tn)[8]) {
+          vn = sb4[(q + 8 < qe ? q + 8 : q) >> 3];
+          acc.lookup(vn, tn);
           if (nb2 < q + 8) {
-            // several warp boundaries inside this word (warps shorter than 8 events): event by event
-            acc.raw |= v.x | v.y | v.z | v.w;
-            const uint32_t wv[4] = {v.x, v.y, v.z, v.w};
+            // several warp boundaries inside this word (warps shorter than 8 events): each event's column by
+            // stepping (empty warps are skipped by nxt, so an event crosses at most one boundary), then the same
+            // paired accumulation as a one-boundary word
+            uint32_t c[8];
 #pragma unroll
             for (int j = 0; j < 8; ++j) {
-              while (q + j >= nb) {
-                sg = m.nxt[sg];
-                col = colof(sg);
-                nb = rel(m.offs[sg + 1]);
+              if (q + j >= nb) {
+                sg = sgn;
+                col = coln;
+                nb = nb2;
+                f = m.info[sg];
+                sgn = f.y & 0xFFFFu;
+                coln = f.x & 0xFFFFu;
+                nb2 = f.x >> 16;
               }
-              acc.one(col, (j & 1) ? (wv[j >> 1] >> 16) : (wv[j >> 1] & 0xFFFFu));
+              c[j] = col;
             }
-            while (q + 8 >= nb && sg < last) {  // move to the warp open after this word
-              sg = m.nxt[sg];
-              col = colof(sg);
-              nb = rel(m.offs[sg + 1]);
+            acc.word8(v, t, c, sbase);
+            if (q + 8 >= nb) {  // the next word starts in the next warp
+              sg = sgn;
+              col = coln;
+              nb = nb2;
             }
-            sgn = m.nxt[sg];
-            coln = colof(sgn);
-            nb2 = sgn != sg ? rel(m.offs[sgn + 1]) : LIM + 8u;
-            continue;
+          } else {
+            const uint32_t bo = nb < q + 8 ? nb - q : 8u;  // first event of the next warp
+            acc.word(v, t, bo, (uint32_t*)(sbase + col), (uint32_t*)(sbase + coln));
+            // advance past a crossed boundary without branching (lanes cross at different words; a divergent
+            // update would serialise): when bo == 8 the same values are reloaded
+            const bool cross = bo < 8u;
+            sg = cross ? sgn : sg;
+            col = cross ? coln : col;
+            nb = cross ? nb2 : nb;
           }
-          const uint32_t bo = nb < q + 8 ? nb - q : 8u;  // first event of the next warp
-          acc.word(v, bo, col, coln);
-          // advance past a crossed boundary without branching (lanes cross at different words; a divergent
-          // update would serialise): when bo == 8 the same values are recomputed
-          const bool cross = bo < 8u;
-          sg = cross ? sgn : sg;
-          col = cross ? coln : col;
-          nb = cross ? nb2 : nb;
-          sgn = m.nxt[sg];
-          coln = colof(sgn);
-          nb2 = sgn != sg ? rel(m.offs[sgn + 1]) : LIM + 8u;
+          f = m.info[sg];
+          sgn = f.y & 0xFFFFu;
+          coln = f.x & 0xFFFFu;
+          nb2 = f.x >> 16;
+        };
+        uint4 va = sb4[q0 >> 3], vb;
+        uint32_t ta[8], tb[8];
+        acc.lookup(va, ta);
+        for (uint32_t q = q0;;) {
+          step(q, va, ta, vb, tb);
+          q += 8;
+          if (q >= qe) break;
+          step(q, vb, tb, va, ta);
+          q += 8;
+          if (q >= qe) break;
         }
       }
       __syncthreads();  // accumulation done; the stage is free
-      if (tid == 0) {   // stage the next chunk (this tile's next, or the next tile's first) during the combine
-        ++pc.c;
-        if (pc.c >= pc.nch) {
-          do { cursor_tile(a, pc, pc.t + gridDim.x); } while (pc.valid && pc.nch == 0);
-        }
-        if (pc.valid) {
-          uint64_t ncs = pc.A + pc.c * CAPE;
-          stage_chunk(a, m, ncs, umin64(ncs + CAPE, pc.Z), E8);
+      if (tid == 0) {   // stage the next chunk (this item's next, or the next item's first) during the combine
+        fl_t = ~0ull;
+        if (c + 1 < nch) {
+          const uint64_t ncs = At + (c + 1) * CAPE;
+          stage_chunk(a, m, ncs, umin64(ncs + CAPE, Zt), E8);
+          fl_t = t;
+          fl_c = c + 1;
+        } else if (tn < NI) {  // thread 0 holds the next item's bounds (nx_off / nx_last), same clamping as cursor_tile
+          const uint64_t nte = umin64(nx_last, a.E), nts = umin64(nx_off, nte);
+          if (nte > nts) {
+            const uint64_t nA = nts & ~7ull, nZ = (nte + 7) & ~7ull;
+            stage_chunk(a, m, nA, umin64(nA + CAPE, nZ), E8);
+            fl_t = tn;
+            fl_c = 0;
+          }
         }
       }
       // combine: warp tid (if it has events in this chunk) adds the HEAD partials of the threads it spilled into
       if (valid && e > s && e > cs && s < ce) {
-        const uint64_t lo_e = umax64(s, cs), hi_e = umin64(e, ce) - 1;
-        const uint32_t ta = (uint32_t)((((lo_e - cs) >> 3) * TPB + TPB - 1) / nwc);
-        const uint32_t tb = (uint32_t)((((hi_e - cs) >> 3) * TPB + TPB - 1) / nwc);
+        const uint32_t lo_w = (uint32_t)((umax64(s, cs) - cs) >> 3), hi_w = (uint32_t)((umin64(e, ce) - 1 - cs) >> 3);
+        const uint32_t ta = (lo_w * TPB + TPB - 1) / nwc;  // thread whose run holds word lo_w
+        const uint32_t tb = (hi_w * TPB + TPB - 1) / nwc;
         const uint32_t from = ta + (s >= cs ? 1u : 0u);  // a warp starting in ta's run went straight into R
         if (from <= tb) {
           uint32_t sum[16];
@@ -497,7 +595,7 @@ __global__ void __launch_bounds__(TPB, 2) k_bbv(BbvArgs a) {
     const uint32_t raw = acc.raw, orr = acc.orr;
     const int bad_here = ((((raw | (raw >> 16)) & 0xFFFFu) & ~bmask) != 0u || (CHECK_MARK && (orr & 1u))) ? 1 : 0;
     if (__syncthreads_or(bad_here) && valid) report_bad_event(a, umin64(s, a.E), umin64(e, a.E));
-    uint32_t k = a.tile_k0 ? a.tile_k0[t] : 0u;
+    uint32_t k = my_k;
     if (valid) {
       if (e < s) latch(a.err, PHOTON_ERANGE, (int64_t)w);
       if (e > s && (uint64_t)(e - s) * max_len >= kInstsLimit) {
@@ -515,8 +613,10 @@ __global__ void __launch_bounds__(TPB, 2) k_bbv(BbvArgs a) {
         dst[3] = make_uint4(p[12], p[13], p[14], p[15]);
       }
       if (a.warp_insts) a.warp_insts[w] = I;
-      if (fused)
+      if (fused && w >= my_kb) {  // the tile crosses into later kernels
+        ++k;
         while (k + 1 < a.K && a.kwo[k + 1] <= w) ++k;
+      }
     }
     if (fused) {
       m.kid[tid] = k;
@@ -529,18 +629,31 @@ __global__ void __launch_bounds__(TPB, 2) k_bbv(BbvArgs a) {
     for (int j = 0; j < 16; ++j) m.hist[j * COLS + tid] = 0u;
     my_off = nx_off;
     last_off = nx_last;
+    if (fused && tn < NI) {
+      my_k = nx_k;
+      my_kb = my_k + 1 < a.K ? a.kwo[my_k + 1] : ~0ull;
+    }
+    if (tid == 0) sched[1] = (uint32_t)(tn < NI ? umin64(x_after, NI) : NI);
+    __syncthreads();  // result columns cleared and offs free before the next item
     t = tn;
-    __syncthreads();  // result columns cleared and offs free before the next tile
+    tn = sched[1];
   }
 }
 
-// K2a over materialised BBVs (the unfused API path): one CTA per tile, keys loaded from warp_bbv16.
+// K2a over materialised BBVs (the unfused API path): one CTA per item, keys loaded from warp_bbv16.
 __global__ void __launch_bounds__(TPB) k_group_from_bbv(BbvArgs a, const uint32_t* __restrict__ bbv) {
   extern __shared__ __align__(128) uint8_t smem_raw[];
   Smem m = carve(smem_raw);
   const int tid = threadIdx.x;
   const uint64_t t = blockIdx.x;
-  const uint64_t w0 = t * TPB, w1 = umin64(a.W, w0 + TPB), w = w0 + tid;
+  if (t >= umin64(*a.n_items, a.n_tiles)) return;
+  uint64_t w0, w1;
+  item_range(a, t, w0, w1);
+  if (w1 <= w0) {
+    if (tid == 0) a.te.tile_n[t] = 0u;
+    return;
+  }
+  const uint64_t w = w0 + tid;
   const bool valid = w < w1;
   for (int i = tid; i < LSLOTS; i += TPB) { m.lhash[i] = 0ull; m.lcount[i] = 0u; m.lminw[i] = UINT32_MAX; }
   if (tid < 64) m.misc[tid] = 0u;
@@ -583,16 +696,145 @@ __global__ void k_table_prep(const uint32_t* __restrict__ bb_len, const uint8_t*
   atomicMax(max_len, len);
 }
 
-__global__ void k_tile_k0(const uint64_t* __restrict__ kwo, uint32_t K, uint64_t n_tiles, uint32_t* tile_k0) {
-  uint64_t t = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
-  if (t >= n_tiles) return;
-  uint64_t w = t * TPB;
+// ---- work items -----------------------------------------------------------------------------------------------
+// Items of block b: nsub(b) = windows spanned by the starts of its warps (sub(w) = (start(w) - start(b0)) >> xs).
+// Two-level exclusive scan: k_items_count writes nsub, the CTA-local exclusive prefix (into boff) and each CTA's
+// total; k_items_scan scans the CTA totals; k_items_fill adds them.  n[0] = item count (clamped to cap), n[1] = work
+// counter, n[2] = split-block count.
+__global__ void __launch_bounds__(256) k_items_count(const uint64_t* __restrict__ weo, uint64_t W, uint64_t E,
+                                                     uint32_t xs, uint64_t n_blocks, uint32_t* nsub, uint32_t* boff,
+                                                     uint32_t* part) {
+  __shared__ uint32_t wsum[8];
+  const uint64_t b = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+  uint32_t v = 0;
+  if (b < n_blocks) {
+    const uint64_t b0 = b * TPB, bl = umin64(W, b0 + TPB) - 1;
+    const uint64_t s0 = umin64(weo[b0], E), sl = umin64(weo[bl], E);
+    v = (uint32_t)umin64(((sl > s0 ? sl - s0 : 0) >> xs) + 1, (uint64_t)TPB);
+    nsub[b] = v;
+  }
+  uint32_t x = v;
+  for (int o = 1; o < 32; o <<= 1) {
+    uint32_t y = __shfl_up_sync(0xffffffffu, x, o);
+    if (lane >= o) x += y;
+  }
+  if (lane == 31) wsum[wid] = x;
+  __syncthreads();
+  uint32_t pre = 0, tot = 0;
+  for (int k = 0; k < 8; ++k) {
+    pre += k < wid ? wsum[k] : 0u;
+    tot += wsum[k];
+  }
+  if (b < n_blocks) boff[b] = pre + x - v;
+  if (threadIdx.x == 0) part[blockIdx.x] = tot;
+}
+
+// exclusive scan of the CTA totals (one CTA, 16 per thread per pass)
+constexpr int ISCAN_PT = 16;
+__global__ void __launch_bounds__(1024) k_items_scan(uint32_t* part, uint64_t n_parts, uint64_t n_blocks, uint64_t cap,
+                                                     uint32_t* boff, uint32_t* n, DevErr* err) {
+  __shared__ uint64_t ws[32];
+  __shared__ uint64_t carry;
+  if (threadIdx.x == 0) carry = 0;
+  __syncthreads();
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+  for (uint64_t base = 0; base < n_parts; base += 1024 * ISCAN_PT) {
+    const uint64_t b0 = base + (uint64_t)threadIdx.x * ISCAN_PT;
+    uint32_t v[ISCAN_PT];
+    uint64_t tot = 0;
+#pragma unroll
+    for (int i = 0; i < ISCAN_PT; ++i) {
+      v[i] = b0 + i < n_parts ? part[b0 + i] : 0u;
+      tot += v[i];
+    }
+    uint64_t x = tot;
+    for (int o = 1; o < 32; o <<= 1) {
+      uint64_t y = __shfl_up_sync(0xffffffffu, x, o);
+      if (lane >= o) x += y;
+    }
+    if (lane == 31) ws[wid] = x;
+    __syncthreads();
+    if (wid == 0) {
+      uint64_t sacc = ws[lane];
+      for (int o = 1; o < 32; o <<= 1) {
+        uint64_t y = __shfl_up_sync(0xffffffffu, sacc, o);
+        if (lane >= o) sacc += y;
+      }
+      ws[lane] = sacc;
+    }
+    __syncthreads();
+    uint64_t ex = carry + (wid ? ws[wid - 1] : 0) + x - tot;
+#pragma unroll
+    for (int i = 0; i < ISCAN_PT; ++i) {
+      if (b0 + i < n_parts) part[b0 + i] = (uint32_t)umin64(ex, 0xFFFFFFFFull);
+      ex += v[i];
+    }
+    __syncthreads();
+    if (threadIdx.x == 1023) carry = ex;
+    __syncthreads();
+  }
+  if (threadIdx.x == 0) {
+    boff[n_blocks] = (uint32_t)umin64(carry, cap);
+    if (carry > cap) latch(err, PHOTON_ERANGE, 0);  // only with non-monotone warp_event_off
+    n[0] = (uint32_t)umin64(carry, cap);
+    n[1] = 0;
+    n[2] = 0;
+  }
+}
+
+// one thread per block: final first item; a one-item block starts at its first warp; split blocks are queued
+__global__ void k_items_fill(uint64_t W, uint32_t* boff, const uint32_t* __restrict__ nsub,
+                             const uint32_t* __restrict__ part, uint64_t n_blocks, uint64_t cap, uint32_t* n,
+                             uint64_t* item_w0, uint32_t* split) {
+  const uint64_t b = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (b == 0) item_w0[n[0]] = W;
+  if (b >= n_blocks) return;
+  const uint64_t it0 = umin64((uint64_t)boff[b] + part[blockIdx.x], cap);
+  const uint32_t nb = (uint32_t)umin64(nsub[b], cap - it0);
+  boff[b] = (uint32_t)it0;
+  if (nb == 1) item_w0[it0] = b * TPB;
+  else if (nb > 1) split[atomicAdd(&n[2], 1u)] = (uint32_t)b;
+}
+
+// one warp per split block: each warp opens the windows between the previous warp's and its own (windows holding no
+// start become empty items); non-monotone warp_event_off is latched
+__global__ void k_items_split(const uint64_t* __restrict__ weo, uint64_t W, uint64_t E, uint32_t xs,
+                              const uint32_t* __restrict__ boff, const uint32_t* __restrict__ nsub, uint64_t cap,
+                              const uint32_t* __restrict__ n, const uint32_t* __restrict__ split, uint64_t* item_w0,
+                              DevErr* err) {
+  const int lane = threadIdx.x & 31;
+  const uint64_t nwarps = ((uint64_t)gridDim.x * blockDim.x) >> 5;
+  for (uint64_t q = ((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; q < n[2]; q += nwarps) {
+    const uint64_t b = split[q], b0 = b * TPB, b1 = umin64(W, b0 + TPB);
+    const uint32_t it0 = boff[b], nb = nsub[b];
+    const uint64_t base = umin64(weo[b0], E);
+    for (uint64_t w = b0 + lane; w < b1; w += 32) {
+      const uint64_t sw = umin64(weo[w], E);
+      const uint64_t s = (sw > base ? sw - base : 0) >> xs;
+      int64_t sp = -1;
+      if (w > b0) {
+        if (weo[w - 1] > weo[w]) latch(err, PHOTON_ERANGE, (int64_t)(w - 1));
+        const uint64_t sv = umin64(weo[w - 1], E);
+        sp = (int64_t)((sv > base ? sv - base : 0) >> xs);
+      }
+      for (int64_t i = sp + 1; i <= (int64_t)s && (uint64_t)i < nb && it0 + (uint64_t)i < cap; ++i) item_w0[it0 + i] = w;
+    }
+  }
+}
+
+// kernel of each item's first warp (one thread per item)
+__global__ void k_items_k0(const uint64_t* __restrict__ kwo, uint32_t K, const uint32_t* __restrict__ n,
+                           const uint64_t* __restrict__ item_w0, uint64_t cap, uint32_t* item_k0) {
+  const uint64_t it = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (it >= cap || it >= n[0]) return;
+  const uint64_t w = item_w0[it];
   uint32_t lo = 0, hi = K - 1;  // last k with kwo[k] <= w
   while (lo < hi) {
     uint32_t mid = (lo + hi + 1) >> 1;
     if (kwo[mid] <= w) lo = mid; else hi = mid - 1;
   }
-  tile_k0[t] = lo;
+  item_k0[it] = lo;
 }
 
 __global__ void k_validate_offsets(const uint64_t* __restrict__ kwo, uint32_t K, const uint64_t* __restrict__ weo,
@@ -688,15 +930,27 @@ __global__ void __launch_bounds__(1024) k_kchunks(const uint64_t* __restrict__ k
 }  // namespace
 
 size_t bbv_table_bytes(uint32_t B) { return (size_t)next_pow2_u32(B < 16 ? 16 : B) * 4 + 64; }
-uint64_t bbv_n_tiles(uint64_t W) { return ceil_div(W, TPB); }
+uint64_t bbv_n_blocks(uint64_t W) { return ceil_div(W, TPB); }
+uint64_t bbv_item_cap(uint64_t W, uint64_t E, uint32_t xs) {
+  return bbv_n_blocks(W) + (xs < 63 ? (E >> xs) : 0) + 1;
+}
 
-cudaError_t launch_table_prep(const TraceDev& t, uint32_t* tbl, uint32_t* max_len, uint32_t* tile_k0, DevErr* err,
-                              cudaStream_t s) {
+cudaError_t launch_table_prep(const TraceDev& t, uint32_t* tbl, uint32_t* max_len, const ItemTable& it,
+                              const TileEntries* te, DevErr* err, cudaStream_t s) {
   uint32_t P2 = next_pow2_u32(t.B < 16 ? 16 : t.B);
   cudaMemsetAsync(max_len, 0, 4, s);
   note_launch(), k_table_prep<<<(P2 + 255) / 256, 256, 0, s>>>(t.bb_len, t.bb_bin, t.B, P2, tbl, max_len, err);
-  uint64_t nt = bbv_n_tiles(t.W);
-  if (tile_k0 && nt) note_launch(), k_tile_k0<<<(unsigned)ceil_div(nt, 256), 256, 0, s>>>(t.kwo, t.K, nt, tile_k0);
+  const uint64_t nb = bbv_n_blocks(t.W);
+  if (nb == 0) return cudaGetLastError();
+  (void)te;
+  const uint64_t gb = ceil_div(nb, 256);
+  note_launch(), k_items_count<<<(unsigned)gb, 256, 0, s>>>(t.weo, t.W, t.E, it.xs, nb, it.nsub, it.boff, it.part);
+  note_launch(), k_items_scan<<<1, 1024, 0, s>>>(it.part, gb, nb, it.cap, it.boff, it.n, err);
+  note_launch(), k_items_fill<<<(unsigned)gb, 256, 0, s>>>(t.W, it.boff, it.nsub, it.part, nb, it.cap, it.n, it.w0,
+                                                           it.split);
+  note_launch(), k_items_split<<<(unsigned)umin64(ceil_div(nb * 32, 256), 1184), 256, 0, s>>>(
+      t.weo, t.W, t.E, it.xs, it.boff, it.nsub, it.cap, it.n, it.split, it.w0, err);
+  note_launch(), k_items_k0<<<(unsigned)ceil_div(it.cap, 256), 256, 0, s>>>(t.kwo, t.K, it.n, it.w0, it.cap, it.k0);
   return cudaGetLastError();
 }
 
@@ -722,18 +976,20 @@ static cudaError_t launch_bbv_t(const BbvArgs& a, size_t smem, int num_sms, cuda
   return cudaGetLastError();
 }
 
-cudaError_t launch_bbv(const TraceDev& t, const uint32_t* tbl, const uint32_t* max_len, const uint32_t* tile_k0,
+cudaError_t launch_bbv(const TraceDev& t, const uint32_t* tbl, const uint32_t* max_len, const ItemTable& it,
                        uint32_t* warp_bbv16, uint64_t* warp_insts, const TileEntries* te, DevErr* err, int num_sms,
                        cudaStream_t s) {
   BbvArgs a{};
-  a.kwo = t.kwo; a.weo = t.weo; a.bb = t.bb; a.tbl = tbl; a.max_len = max_len; a.tile_k0 = tile_k0;
+  a.kwo = t.kwo; a.weo = t.weo; a.bb = t.bb; a.tbl = tbl; a.max_len = max_len; a.tile_k0 = it.k0;
+  a.item_w0 = it.w0; a.n_items = it.n; a.counter = it.n + 1;
   a.K = t.K; a.B = t.B; a.P2 = next_pow2_u32(t.B < 16 ? 16 : t.B);
   a.W = t.W; a.E = t.E;
   a.warp_bbv16 = warp_bbv16; a.warp_insts = warp_insts;
   if (te) a.te = *te;
   a.err = err;
-  a.n_tiles = bbv_n_tiles(t.W);
-  if (a.n_tiles == 0) return cudaSuccess;
+  a.n_tiles = it.cap;
+  if (t.W == 0) return cudaSuccess;
+  cudaMemsetAsync(a.counter, 0, 4, s);
   bool smem_tbl = a.P2 <= SMEM_TBL_MAX;
   bool mark = a.P2 != t.B;
   size_t smem = bbv_smem_bytes(smem_tbl ? a.P2 : 0);
@@ -741,13 +997,14 @@ cudaError_t launch_bbv(const TraceDev& t, const uint32_t* tbl, const uint32_t* m
   return mark ? launch_bbv_t<false, true>(a, smem, num_sms, s) : launch_bbv_t<false, false>(a, smem, num_sms, s);
 }
 
-cudaError_t launch_group_from_bbv(const TraceDev& t, const uint32_t* warp_bbv16, const uint32_t* tile_k0,
+cudaError_t launch_group_from_bbv(const TraceDev& t, const uint32_t* warp_bbv16, const ItemTable& it,
                                   const TileEntries& te, DevErr* err, cudaStream_t s) {
   BbvArgs a{};
-  a.kwo = t.kwo; a.K = t.K; a.W = t.W; a.te = te; a.err = err; a.tile_k0 = tile_k0;
-  uint64_t tiles = bbv_n_tiles(t.W);
+  a.kwo = t.kwo; a.K = t.K; a.W = t.W; a.te = te; a.err = err; a.tile_k0 = it.k0;
+  a.item_w0 = it.w0; a.n_items = it.n;
+  const uint64_t tiles = it.cap;
   a.n_tiles = tiles;
-  if (tiles == 0) return cudaSuccess;
+  if (t.W == 0) return cudaSuccess;
   size_t smem = bbv_smem_bytes(0);
   cudaError_t e = cudaFuncSetAttribute(k_group_from_bbv, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return e;

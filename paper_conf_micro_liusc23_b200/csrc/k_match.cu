@@ -83,6 +83,10 @@ struct ScanArgs {
   DevErr* err;
 };
 
+// Each thread scores a 4 x 4 block of (k, r) pairs of the tile: per bin, one 16-byte shared load of 4 k-profiles
+// and one of 4 r-profiles feed 16 |difference| accumulations (the profiles are stored bin-major).  Surviving pairs
+// are appended with one atomic per warp.
+constexpr int FTP = FT + 4;  // row stride (floats) of the bin-major profile tiles
 __global__ void __launch_bounds__(256) k_pair_filter(ScanArgs a, uint64_t t0) {
   // blockIdx.x enumerates lower-triangle tiles (kb, rb) with rb <= kb, kb over [k_lo, k_hi) in FT blocks
   uint64_t t = t0 + blockIdx.x;
@@ -92,87 +96,138 @@ __global__ void __launch_bounds__(256) k_pair_filter(ScanArgs a, uint64_t t0) {
   while ((uint64_t)kb * (kb + 1) / 2 > t) --kb;
   uint32_t rb = t - kb * (kb + 1) / 2;
 
-  uint32_t k0 = kb * FT, r0 = rb * FT;  // absolute kernel indices (k blocks start at 0; k < k_lo are skipped)
-  __shared__ float pk[FT][17], pr[FT][17];
-  __shared__ uint64_t wk[FT], wr[FT], nk[FT], nr[FT];
-  for (int i = threadIdx.x; i < FT * 16; i += 256) {
-    int row = i >> 4, j = i & 15;
-    uint32_t k = k0 + row, r = r0 + row;
-    pk[row][j] = k < a.K ? a.prof[(uint64_t)k * 16 + j] : 0.f;
-    pr[row][j] = r < a.K ? a.prof[(uint64_t)r * 16 + j] : 0.f;
+  const uint32_t k0 = kb * FT, r0 = rb * FT;  // absolute kernel indices
+  __shared__ __align__(16) float pk[16][FTP], pr[16][FTP];
+  __shared__ uint64_t wk[FT], wr[FT];
+  __shared__ uint32_t okk[FT], okr[FT];  // mass > 0 [P-19]
+  const int tid = threadIdx.x;
+  for (int i = tid; i < FT * 16; i += 256) {
+    const int row = i >> 4, j = i & 15;
+    const uint32_t k = k0 + row, r = r0 + row;
+    pk[j][row] = k < a.K ? a.prof[(uint64_t)k * 16 + j] : 0.f;
+    pr[j][row] = r < a.K ? a.prof[(uint64_t)r * 16 + j] : 0.f;
   }
-  for (int i = threadIdx.x; i < FT; i += 256) {
-    uint32_t k = k0 + i, r = r0 + i;
-    wk[i] = k < a.K ? a.wt[k] : 0; nk[i] = k < a.K ? a.mass[k] : 0;
-    wr[i] = r < a.K ? a.wt[r] : 0; nr[i] = r < a.K ? a.mass[r] : 0;
+  for (int i = tid; i < FT; i += 256) {
+    const uint32_t k = k0 + i, r = r0 + i;
+    wk[i] = k < a.K ? a.wt[k] : 0;
+    okk[i] = k < a.K && a.mass[k] != 0;
+    wr[i] = r < a.K ? a.wt[r] : 0;
+    okr[i] = r < a.K && a.mass[r] != 0;
   }
   __syncthreads();
-  for (int idx = threadIdx.x; idx < FT * FT; idx += 256) {
-    int i = idx / FT, j = idx % FT;
-    uint32_t k = k0 + i, r = r0 + j;
-    if (k >= a.k_hi || k < a.k_lo || r >= k) continue;
-    if (nk[i] == 0 || nr[j] == 0) continue;  // [P-19]
-    uint64_t Wk = wk[i], Wr = wr[j];
-    if (!(Wk == Wr || (Wk < Wr ? Wk : Wr) >= a.p.n_cores)) continue;  // [P-10]
-    float d = 0.f;
+  const int i0 = (tid >> 4) * 4, j0 = (tid & 15) * 4;
+  float d[4][4];
 #pragma unroll
-    for (int b = 0; b < 16; ++b) d += fabsf(pk[i][b] - pr[j][b]);
-    if (d >= a.bound) continue;
-    unsigned long long pos = atomicAdd((unsigned long long*)a.n_maybe, 1ull);
+  for (int u = 0; u < 4; ++u)
+#pragma unroll
+    for (int v = 0; v < 4; ++v) d[u][v] = 0.f;
+#pragma unroll
+  for (int b = 0; b < 16; ++b) {
+    const float4 x = *(const float4*)&pk[b][i0];
+    const float4 y = *(const float4*)&pr[b][j0];
+    const float xs[4] = {x.x, x.y, x.z, x.w}, ys[4] = {y.x, y.y, y.z, y.w};
+#pragma unroll
+    for (int u = 0; u < 4; ++u)
+#pragma unroll
+      for (int v = 0; v < 4; ++v) d[u][v] += fabsf(xs[u] - ys[v]);
+  }
+  uint32_t keep = 0;  // bit 4u+v
+#pragma unroll
+  for (int u = 0; u < 4; ++u) {
+    const int i = i0 + u;
+    const uint32_t k = k0 + i;
+    const bool kin = k >= a.k_lo && k < a.k_hi && okk[i];
+#pragma unroll
+    for (int v = 0; v < 4; ++v) {
+      const int j = j0 + v;
+      const uint32_t r = r0 + j;
+      const uint64_t Wk = wk[i], Wr = wr[j];
+      const bool ok = kin && r < k && okr[j] && (Wk == Wr || (Wk < Wr ? Wk : Wr) >= a.p.n_cores) &&  // [P-10]
+                      d[u][v] < a.bound;
+      keep |= (ok ? 1u : 0u) << (4 * u + v);
+    }
+  }
+  // warp-aggregated append
+  const int lane = tid & 31;
+  const uint32_t cnt = __popc(keep);
+  uint32_t incl = cnt;
+  for (int o = 1; o < 32; o <<= 1) {
+    uint32_t y = __shfl_up_sync(0xffffffffu, incl, o);
+    if (lane >= o) incl += y;
+  }
+  const uint32_t total = __shfl_sync(0xffffffffu, incl, 31);
+  if (total == 0) return;
+  unsigned long long base = 0;
+  if (lane == 31) base = atomicAdd((unsigned long long*)a.n_maybe, (unsigned long long)total);
+  base = __shfl_sync(0xffffffffu, base, 31);
+  unsigned long long pos = base + (incl - cnt);
+  for (uint32_t m = keep; m; m &= m - 1, ++pos) {
+    const int bit = __ffs(m) - 1;
+    const uint32_t k = k0 + i0 + (bit >> 2), r = r0 + j0 + (bit & 3);
     if (pos < a.cap) a.maybe[pos] = ((uint64_t)k << 32) | r;
     else latch(a.err, PHOTON_ECAPACITY, (int64_t)pos);
   }
 }
 
-// exact Dnum = sum_i |g_k[i] N_r - g_r[i] N_k| (zero padded), warp-cooperative; all lanes return the total
-__device__ u128 warp_dnum(const uint64_t* sig, const uint64_t* kto, const uint64_t* mass, uint32_t k, uint32_t r,
-                          u128 stop_at) {
-  const uint32_t lane = threadIdx.x & 31;
-  uint64_t ok = kto[k] * 16, orr = kto[r] * 16;
-  uint64_t Lk = (kto[k + 1] - kto[k]) * 16, Lr = (kto[r + 1] - kto[r]) * 16;
-  uint64_t L = Lk > Lr ? Lk : Lr;
-  uint64_t Nk = mass[k], Nr = mass[r];
-  u128 total = 0;
-  for (uint64_t base = 0; base < L; base += 32 * 8) {
-    u128 acc = 0;
-#pragma unroll 4
-    for (int u = 0; u < 8; ++u) {
-      uint64_t i = base + (uint64_t)u * 32 + lane;
-      if (i < L) {
-        uint64_t gk = i < Lk ? sig[ok + i] : 0, gr = i < Lr ? sig[orr + i] : 0;
-        u128 x = (u128)gk * Nr, y = (u128)gr * Nk;
-        acc += x > y ? x - y : y - x;
-      }
-    }
-    uint64_t lo = (uint64_t)acc, hi = (uint64_t)(acc >> 64);
-    for (int o = 16; o > 0; o >>= 1) {
-      uint64_t lo2 = __shfl_xor_sync(0xffffffffu, lo, o), hi2 = __shfl_xor_sync(0xffffffffu, hi, o);
-      uint64_t s = lo + lo2;
-      hi = hi + hi2 + (s < lo ? 1 : 0);
-      lo = s;
-    }
-    total += ((u128)hi << 64) | lo;
-    if (total >= stop_at) break;  // early exit: already not close
+// exact Dnum = sum_i |g_k[i] N_r - g_r[i] N_k| (zero padded), by a group of G lanes (G | 32, aligned); all lanes
+// of the group return the total
+template <int G>
+__device__ u128 group_dnum(const uint64_t* sig, const uint64_t* kto, const uint64_t* mass, uint32_t k, uint32_t r,
+                          bool act = true) {
+  const uint32_t l = threadIdx.x & (G - 1);
+  uint64_t ok = 0, orr = 0, Lk = 0, Lr = 0, Nk = 0, Nr = 0;
+  if (act) {  // inactive groups only join the shuffles
+    ok = kto[k] * 16;
+    orr = kto[r] * 16;
+    Lk = (kto[k + 1] - kto[k]) * 16;
+    Lr = (kto[r + 1] - kto[r]) * 16;
+    Nk = mass[k];
+    Nr = mass[r];
   }
-  return total;
+  const uint64_t L = Lk > Lr ? Lk : Lr;
+  u128 acc = 0;
+#pragma unroll 4
+  for (uint64_t i = l; i < L; i += G) {
+    const uint64_t gk = i < Lk ? sig[ok + i] : 0, gr = i < Lr ? sig[orr + i] : 0;
+    const u128 x = (u128)gk * Nr, y = (u128)gr * Nk;
+    acc += x > y ? x - y : y - x;
+  }
+  uint64_t lo = (uint64_t)acc, hi = (uint64_t)(acc >> 64);
+  for (int o = G / 2; o > 0; o >>= 1) {
+    const uint64_t lo2 = __shfl_xor_sync(0xffffffffu, lo, o), hi2 = __shfl_xor_sync(0xffffffffu, hi, o);
+    const uint64_t sm = lo + lo2;
+    hi = hi + hi2 + (sm < lo ? 1 : 0);
+    lo = sm;
+  }
+  return ((u128)hi << 64) | lo;
+}
+__device__ __forceinline__ u128 warp_dnum(const uint64_t* sig, const uint64_t* kto, const uint64_t* mass, uint32_t k,
+                                          uint32_t r) {
+  return group_dnum<32>(sig, kto, mass, k, r);
 }
 
-__global__ void k_pair_exact(ScanArgs a, uint64_t* pairs, uint64_t pair_cap, uint64_t* n_pairs) {
+// one group of XG lanes per filtered pair: close <=> theta_den * Dnum < theta_num * N_k * N_r (Fig 12, [P-15])
+constexpr int XG = 8;
+__global__ void __launch_bounds__(256) k_pair_exact(ScanArgs a, uint64_t* pairs, uint64_t pair_cap,
+                                                    uint64_t* n_pairs) {
   uint64_t n = *a.n_maybe;
   if (n > a.cap) n = a.cap;
-  uint64_t warp = ((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-  uint64_t nw = ((uint64_t)gridDim.x * blockDim.x) >> 5;
-  for (uint64_t q = warp; q < n; q += nw) {
-    uint64_t pr = a.maybe[q];
-    uint32_t k = (uint32_t)(pr >> 32), r = (uint32_t)pr;
-    u128 rhs = (u128)a.p.theta_num * ((u128)a.mass[k] * a.mass[r]);
-    // close <=> theta_den * Dnum < rhs ; stop once theta_den * Dnum >= rhs  <=>  Dnum >= ceil(rhs / theta_den)
-    u128 stop = (rhs + a.p.theta_den - 1) / a.p.theta_den;
-    u128 d = warp_dnum(a.sig, a.kto, a.mass, k, r, stop);
-    if ((threadIdx.x & 31) == 0 && (u128)a.p.theta_den * d < rhs) {
-      unsigned long long pos = atomicAdd((unsigned long long*)n_pairs, 1ull);
-      if (pos < pair_cap) pairs[pos] = pr;
-      else latch(a.err, PHOTON_ECAPACITY, (int64_t)pos);
+  const uint64_t g = ((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) / XG;
+  const uint64_t ng = ((uint64_t)gridDim.x * blockDim.x) / XG;
+  const uint64_t rounds = (n + ng - 1) / ng;  // every lane runs the same number of rounds (shuffles stay converged)
+  for (uint64_t it = 0; it < rounds; ++it) {
+    const uint64_t q = g + it * ng;
+    const bool act = q < n;
+    const uint64_t pr = act ? a.maybe[q] : 0;
+    const uint32_t k = (uint32_t)(pr >> 32), r = (uint32_t)pr;
+    const u128 d = group_dnum<XG>(a.sig, a.kto, a.mass, k, r, act);
+    if (act && (threadIdx.x & (XG - 1)) == 0) {
+      const u128 rhs = (u128)a.p.theta_num * ((u128)a.mass[k] * a.mass[r]);
+      if ((u128)a.p.theta_den * d < rhs) {
+        const unsigned long long pos = atomicAdd((unsigned long long*)n_pairs, 1ull);
+        if (pos < pair_cap) pairs[pos] = pr;
+        else latch(a.err, PHOTON_ECAPACITY, (int64_t)pos);
+      }
     }
   }
 }
@@ -331,7 +386,7 @@ __global__ void k_resolve_match(uint32_t K, const uint64_t* off, const uint32_t*
   }
   if (lane == 0) match[k] = (int64_t)best_r;
   if (dist) {
-    u128 d = warp_dnum(sig, kto, mass, k, best_r, ~(u128)0);
+    u128 d = warp_dnum(sig, kto, mass, k, best_r);
     if (lane == 0) {
       u128 den = (u128)mass[k] * mass[best_r];
       double dn = (double)(uint64_t)(d >> 64) * 18446744073709551616.0 + (double)(uint64_t)d;

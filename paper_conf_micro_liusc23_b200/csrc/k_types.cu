@@ -287,7 +287,7 @@ __global__ void k_entries_insert(TileEntries te, uint64_t n_tiles, HashTable ht,
   uint32_t* out;
   if (i < nfix) {
     uint64_t t = i / te.per_tile, e = i % te.per_tile;
-    if (e >= te.tile_n[t]) return;
+    if (t >= *te.n_items || e >= te.tile_n[t]) return;
     x = te.ent + i;
     out = te.tile_slot + i;
   } else {
@@ -321,13 +321,12 @@ __global__ void k_entries_insert(TileEntries te, uint64_t n_tiles, HashTable ht,
 __global__ void k_remap_entries(TileEntries te, uint64_t W, const uint32_t* canon, uint32_t* warp_type) {
   const uint64_t w = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
   if (w >= W) return;
-  const uint64_t t = w >> 8;  // 256 warps per tile (k_bbv.cu TPB)
-  const uint32_t e = te.lid[w];
+  const uint32_t g = te.gid[w];
   uint32_t slot;
-  if (e < te.per_tile) {
-    slot = te.tile_slot[t * te.per_tile + e];
+  if (!(g >> 31)) {
+    slot = te.tile_slot[g];
   } else {
-    const uint64_t j = te.tile_ovf[t] + (e - te.per_tile);  // beyond ovf_cap only after ECAPACITY was latched
+    const uint64_t j = g & 0x7FFFFFFFu;  // beyond ovf_cap only after ECAPACITY was latched
     slot = j < te.ovf_cap ? te.ovf_slot[j] : UINT32_MAX;
   }
   warp_type[w] = slot == UINT32_MAX ? UINT32_MAX : canon[slot];

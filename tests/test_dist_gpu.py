@@ -19,6 +19,8 @@ class FakeComm:
         self.world, self.rank, self.s = world, rank, shared
 
     def _exchange(self, x):
+        import torch
+        torch.cuda.synchronize()  # the other threads read x on their own streams: it must be complete
         s = self.s
         s["slots"][self.rank] = x
         s["bar"].wait()
@@ -26,10 +28,17 @@ class FakeComm:
         s["bar"].wait()
         return vals
 
+    def _done(self):
+        import torch
+        torch.cuda.synchronize()
+
     def allgather_varlen(self, x):
         import torch
         vals = self._exchange(x)
-        return torch.cat(vals), [v.shape[0] for v in vals]
+        out = torch.cat(vals)
+        self._done()
+        self.s["bar"].wait()
+        return out, [v.shape[0] for v in vals]
 
     def allreduce_sum(self, x):
         vals = self._exchange(x.clone())
@@ -37,6 +46,8 @@ class FakeComm:
         for v in vals[1:]:
             tot += v
         x.copy_(tot)
+        self._done()  # keep the slot tensors alive and read until every thread has summed them
+        self.s["bar"].wait()
         return x
 
 
