@@ -9,7 +9,7 @@ import os
 from ctypes import POINTER, c_double, c_int, c_int64, c_size_t, c_uint8, c_uint32, c_uint64, c_void_p, c_char_p
 
 HERE = os.path.dirname(os.path.abspath(__file__))
-SO_PATH = os.path.join(HERE, "libphoton.so")
+SO_PATH = os.environ.get("PHOTON_LIB_OVERRIDE") or os.path.join(HERE, "libphoton.so")  # override: profiling builds
 
 OK, EINVAL, ECUDA, ERANGE, ECAPACITY, EWORKSPACE = 0, -1, -2, -3, -4, -5
 STATUS = {0: "OK", -1: "EINVAL", -2: "ECUDA", -3: "ERANGE", -4: "ECAPACITY", -5: "EWORKSPACE"}

@@ -213,6 +213,8 @@ MatchLayout match_layout(uint32_t K, uint64_t T, uint64_t pair_cap, void* base) 
   m.sig = c.take<uint64_t>(16 * (T ? T : 1));
   m.mass = c.take<uint64_t>(K + 1);
   m.mw.prof = c.take<float>(16ull * K + 16);
+  m.mw.invn = c.take<double>(K + 1);
+  m.mw.prof8 = c.take<uint32_t>(4ull * K + 4);
   m.mw.maybe = c.take<uint64_t>(pair_cap);
   m.mw.n_maybe = c.take<uint64_t>(1);
   m.mw.cand_cnt = c.take<uint32_t>(K + 1);
@@ -222,6 +224,7 @@ MatchLayout match_layout(uint32_t K, uint64_t T, uint64_t pair_cap, void* base) 
   m.mw.state = c.take<uint8_t>(K + 1);
   m.mw.ulist = c.take<uint32_t>(2ull * K + 2);
   m.mw.flag = c.take<uint32_t>(4);
+  m.mw.rcnt = c.take<uint32_t>(K + 2);
   m.mw.pair_cap = pair_cap;
   m.pairs = c.take<uint64_t>(pair_cap);
   m.n_pairs = c.take<uint64_t>(1);
@@ -493,7 +496,7 @@ int photon_kernel_match(photon_ctx* ctx, uint32_t K, const photon_types* types, 
   {
     ProfScope ps(ctx, PHOTON_PROF_RESOLVE, s);
     CK(launch_match_resolve(K, types->kernel_type_off, m.sig, m.mass, warps_total, params, m.pairs, m.mw.pair_cap,
-                            m.n_pairs, m.mw, match, match_dist, m.err, s),
+                            m.n_pairs, m.mw, match, match_dist, m.err, ctx->num_sms, s),
        "resolve");
   }
   return PHOTON_OK;
@@ -573,7 +576,7 @@ int photon_match_resolve(photon_ctx* ctx, uint32_t K, const uint64_t* kto, const
   ctx->last_ws = ws;
   CK(cudaMemsetAsync(m.err, 0, sizeof(DevErr), s), "memset");
   CK(launch_match_resolve(K, kto, sig, mass, warps_total, params, pairs, n_pairs, nullptr, m.mw, match, match_dist,
-                          m.err, s),
+                          m.err, ctx->num_sms, s),
      "resolve");
   return PHOTON_OK;
 }

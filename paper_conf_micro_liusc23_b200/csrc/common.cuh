@@ -36,6 +36,7 @@ struct DevErr {
 };
 
 __device__ __forceinline__ void latch(DevErr* e, int code, int64_t index) {
+  if (*(volatile int32_t*)&e->code != 0) return;  // already latched: skip the contended CAS
   if (atomicCAS(&e->code, 0, code) == 0) {
     e->index = index;
   }
@@ -131,6 +132,14 @@ __device__ __forceinline__ uint32_t ld_acquire_u32(const uint32_t* p) {
 __device__ __forceinline__ void st_release_u32(uint32_t* p, uint32_t v) {
   asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
 }
+__device__ __forceinline__ uint4 ld_relaxed_v4(const uint32_t* p) {
+  uint4 v;
+  asm volatile("ld.relaxed.gpu.global.v4.u32 {%0, %1, %2, %3}, [%4];"
+               : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w)
+               : "l"(p)
+               : "memory");
+  return v;
+}
 __device__ __forceinline__ uint32_t ld_relaxed_u32(const uint32_t* p) {
   uint32_t v;
   asm volatile("ld.relaxed.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
@@ -177,7 +186,10 @@ __device__ __forceinline__ uint32_t ht_insert(const HashTable& ht, DevErr* err, 
       }
       mine = ld_relaxed_u32(&ht.kern[i]) == k;
 #pragma unroll
-      for (int j = 0; j < 16; ++j) mine = mine && (ld_relaxed_u32(&ht.key[i * 16 + j]) == p[j]);
+      for (int q = 0; q < 4; ++q) {  // 16-byte loads (the key row is 64-byte aligned)
+        const uint4 v = ld_relaxed_v4(&ht.key[i * 16 + 4 * q]);
+        mine = mine && v.x == p[4 * q] && v.y == p[4 * q + 1] && v.z == p[4 * q + 2] && v.w == p[4 * q + 3];
+      }
     }
     if (mine) {
       atomicAdd(&ht.count[i], cnt);

@@ -108,6 +108,8 @@ cudaError_t launch_remap_direct(const uint64_t* kwo_local, uint32_t K_local, uin
 // ---- A3/A4 (k_match.cu) -----------------------------------------------------------------------------------
 struct MatchWs {
   float* prof;         // [K][16] normalised per-bin profile (filter)
+  double* invn;        // [K] 1 / N_k (fp64 screen of the exact check)
+  uint32_t* prof8;     // [K][4] the profile quantised to u8 (round(255 P)), packed 4 bins per word (coarse filter)
   uint64_t* maybe;     // [pair_cap] profile-filter survivors
   uint64_t* n_maybe;   // [1]
   uint32_t* cand_cnt;  // [K]
@@ -117,6 +119,7 @@ struct MatchWs {
   uint8_t* state;      // [K] 0 undecided, 1 representative, 2 matched
   uint32_t* ulist;     // [2K] undecided-kernel lists (resolution rounds)
   uint32_t* flag;      // [4]
+  uint32_t* rcnt;      // [K+2] undecided count of each resolution round
   uint64_t pair_cap;
 };
 cudaError_t launch_sig_build(uint32_t K, const uint64_t* kto, const uint32_t* type_key, const uint64_t* type_count,
@@ -128,7 +131,7 @@ cudaError_t launch_match_scan(uint32_t K, const uint64_t* kto, const uint64_t* s
 cudaError_t launch_match_resolve(uint32_t K, const uint64_t* kto, const uint64_t* sig, const uint64_t* mass,
                                  const uint64_t* wt, photon_match_params p, const uint64_t* pairs, uint64_t n_pairs,
                                  const uint64_t* n_pairs_dev, const MatchWs& mw, int64_t* match, double* match_dist,
-                                 DevErr* err, cudaStream_t s);
+                                 DevErr* err, int num_sms, cudaStream_t s);
 
 // ---- A5 (k_stable.cu) -------------------------------------------------------------------------------------
 size_t stable_ws_bytes(const photon_timing& t);

@@ -24,6 +24,10 @@
 // inserts the entries into the global type table.
 #include "internal.h"
 
+#ifndef PHOTON_EXP
+#define PHOTON_EXP 0  // profiling experiments only (1: no accumulation, 2: no tile de-dup); never set in builds
+#endif
+
 namespace photon {
 
 namespace {
@@ -122,11 +126,6 @@ struct Acc {
   const uint32_t* tbl;
   uint32_t bmask;
   uint32_t raw, orr;
-  __device__ __forceinline__ void one(uint32_t* col, uint32_t b) {
-    uint32_t t = tbl[b & bmask];
-    orr |= t;
-    *(uint32_t*)((uint8_t*)col + (t & AMASK)) += t >> LSH;
-  }
   // two events whose table entries are already loaded; `same` = both go to the same column
   __device__ __forceinline__ void pair(uint32_t t0, uint32_t t1, uint32_t* c0, uint32_t* c1, bool same) {
     const uint32_t a0 = t0 & AMASK, a1 = t1 & AMASK;
@@ -282,6 +281,12 @@ __device__ void tile_group(const BbvArgs& a, const Smem& m, uint64_t t, uint64_t
   if (tid == 0) m.misc[0] = 0u;
 }
 
+// Runs: thread t takes words [run_start(t), run_start(t+1)) of an nwc-word chunk (an equal split; moving starts
+// to put each quarter-warp's LDS.128 in distinct bank groups was measured slower overall)
+__device__ __forceinline__ uint32_t run_start(uint32_t t, uint32_t nwc) { return (t * nwc) / TPB; }
+// the thread whose run holds word x (x < nwc): the largest t with run_start(t) <= x
+__device__ __forceinline__ uint32_t run_holder(uint32_t x, uint32_t nwc) { return (x * TPB + TPB - 1) / nwc; }
+
 // thread 0: stage the word-aligned events [cs, ce) into shared memory (bulk part on the TMA copy engine; events
 // at or past E8 with plain loads, positions past E zero-filled), completing on the mbarrier
 __device__ __forceinline__ void stage_chunk(const BbvArgs& a, const Smem& m, uint64_t cs, uint64_t ce, uint64_t E8) {
@@ -291,7 +296,8 @@ __device__ __forceinline__ void stage_chunk(const BbvArgs& a, const Smem& m, uin
   mbar_arrive_expect_tx(m.mbar, bytes);
   for (uint32_t off = 0; off < bytes; off += 16384) {
     uint32_t n = bytes - off < 16384 ? bytes - off : 16384;
-    bulk_g2s((uint8_t*)m.stage + off, (const uint8_t*)(a.bb + cs) + off, n, m.mbar);
+    const uint64_t src = PHOTON_EXP == 3 ? (cs & 0x7FFF8ull) : cs;  // experiment 3: L2-resident source
+    bulk_g2s((uint8_t*)m.stage + off, (const uint8_t*)(a.bb + src) + off, n, m.mbar);
   }
 }
 
@@ -464,7 +470,7 @@ __global__ void __launch_bounds__(TPB, 2) k_bbv(BbvArgs a) {
       mbar_wait(m.mbar, phase);
       phase ^= 1u;
       // my run of words [r0, r1) of the chunk
-      const uint32_t q0 = 8u * ((tid * nwc) / TPB), qe = 8u * (((tid + 1) * nwc) / TPB);
+      const uint32_t q0 = 8u * run_start(tid, nwc), qe = 8u * run_start(tid + 1, nwc);
       if (q0 < qe) {
         // warp (with virtual ones) containing q0: last sp with start(sp) <= q0.  Start from the proportional guess
         // and narrow a +-8 window around it when it brackets q0 (it usually does), else search everything.
@@ -534,6 +540,10 @@ __global__ void __launch_bounds__(TPB, 2) k_bbv(BbvArgs a) {
         uint4 va = sb4[q0 >> 3], vb;
         uint32_t ta[8], tb[8];
         acc.lookup(va, ta);
+        if (PHOTON_EXP == 1) {  // profiling experiment: no accumulation
+          acc.raw |= va.x;
+          goto chunk_done;
+        }
         for (uint32_t q = q0;;) {
           step(q, va, ta, vb, tb);
           q += 8;
@@ -543,6 +553,7 @@ __global__ void __launch_bounds__(TPB, 2) k_bbv(BbvArgs a) {
           if (q >= qe) break;
         }
       }
+    chunk_done:
       __syncthreads();  // accumulation done; the stage is free
       if (tid == 0) {   // stage the next chunk (this item's next, or the next item's first) during the combine
         fl_t = ~0ull;
@@ -564,8 +575,8 @@ __global__ void __launch_bounds__(TPB, 2) k_bbv(BbvArgs a) {
       // combine: warp tid (if it has events in this chunk) adds the HEAD partials of the threads it spilled into
       if (valid && e > s && e > cs && s < ce) {
         const uint32_t lo_w = (uint32_t)((umax64(s, cs) - cs) >> 3), hi_w = (uint32_t)((umin64(e, ce) - 1 - cs) >> 3);
-        const uint32_t ta = (lo_w * TPB + TPB - 1) / nwc;  // thread whose run holds word lo_w
-        const uint32_t tb = (hi_w * TPB + TPB - 1) / nwc;
+        const uint32_t ta = run_holder(lo_w, nwc);  // thread whose run holds word lo_w
+        const uint32_t tb = run_holder(hi_w, nwc);
         const uint32_t from = ta + (s >= cs ? 1u : 0u);  // a warp starting in ta's run went straight into R
         if (from <= tb) {
           uint32_t sum[16];
@@ -618,7 +629,7 @@ __global__ void __launch_bounds__(TPB, 2) k_bbv(BbvArgs a) {
         while (k + 1 < a.K && a.kwo[k + 1] <= w) ++k;
       }
     }
-    if (fused) {
+    if (fused && PHOTON_EXP != 2) {
       m.kid[tid] = k;
       __syncthreads();
       tile_group(a, m, t, w0, valid, k, p);

@@ -12,6 +12,7 @@
 // triangle inequality; a pair is dropped only if that bound exceeds theta by more than its worst rounding error.
 // Survivors get the exact u128 check (one warp per pair).  Launch-order resolution (leader clustering) is then a
 // parallel fixed point: k is a representative iff none of its close predecessors is one.
+#include <cooperative_groups.h>
 #include <math.h>
 
 #include "internal.h"
@@ -52,7 +53,8 @@ __global__ void k_sig(uint32_t k_lo, uint32_t k_hi, const uint64_t* __restrict__
 
 // per-bin profile P_k[j] = sum_t g[16t+j] / N_k (filter only), one warp per kernel
 __global__ void k_prof(uint32_t K, const uint64_t* __restrict__ kto, const uint64_t* __restrict__ sig,
-                       const uint64_t* __restrict__ mass, float* __restrict__ prof) {
+                       const uint64_t* __restrict__ mass, float* __restrict__ prof, double* __restrict__ invn,
+                       uint32_t* __restrict__ prof8) {
   uint32_t warp = (blockIdx.x * blockDim.x + threadIdx.x) >> 5, lane = threadIdx.x & 31;
   if (warp >= K) return;
   uint32_t k = warp;
@@ -60,9 +62,18 @@ __global__ void k_prof(uint32_t K, const uint64_t* __restrict__ kto, const uint6
   uint64_t acc = 0;
   for (uint64_t r = r0 + (lane >> 4); r < r1; r += 2) acc += sig[r * 16 + (lane & 15)];
   acc += __shfl_xor_sync(0xffffffffu, acc, 16);
+  const uint64_t N = mass[k];
+  const double P = N ? (double)acc / (double)N : 0.0;
+  // u8 quantisation for the coarse filter: q = round(255 P) in [0, 255], four bins per word (bin j in byte j & 3)
+  uint32_t q = (uint32_t)rint(P * 255.0);
+  q = q > 255u ? 255u : q;
+  uint32_t w = q << (8 * (lane & 3));
+  w |= __shfl_xor_sync(0xffffffffu, w, 1);
+  w |= __shfl_xor_sync(0xffffffffu, w, 2);
   if (lane < 16) {
-    uint64_t N = mass[k];
-    prof[(uint64_t)k * 16 + lane] = N ? (float)((double)acc / (double)N) : 0.f;
+    prof[(uint64_t)k * 16 + lane] = (float)P;
+    if ((lane & 3) == 0) prof8[(uint64_t)k * 4 + (lane >> 2)] = w;
+    if (lane == 0) invn[k] = N ? 1.0 / (double)N : 0.0;
   }
 }
 
@@ -75,6 +86,9 @@ struct ScanArgs {
   const uint64_t* mass;
   const uint64_t* wt;
   const float* prof;
+  const uint32_t* prof8;
+  uint32_t thr8;  // coarse reject: sum_j |q_k[j] - q_r[j]| >= thr8 implies D >= theta
+  const double* invn;
   photon_match_params p;
   float bound;  // reject if profile distance >= bound
   uint64_t* maybe;
@@ -83,89 +97,146 @@ struct ScanArgs {
   DevErr* err;
 };
 
-// Each thread scores a 4 x 4 block of (k, r) pairs of the tile: per bin, one 16-byte shared load of 4 k-profiles
-// and one of 4 r-profiles feed 16 |difference| accumulations (the profiles are stored bin-major).  Surviving pairs
-// are appended with one atomic per warp.
-constexpr int FTP = FT + 4;  // row stride (floats) of the bin-major profile tiles
-__global__ void __launch_bounds__(256) k_pair_filter(ScanArgs a, uint64_t t0) {
-  // blockIdx.x enumerates lower-triangle tiles (kb, rb) with rb <= kb, kb over [k_lo, k_hi) in FT blocks
-  uint64_t t = t0 + blockIdx.x;
-  // invert t = kb*(kb+1)/2 + rb relative to the first k block
-  uint32_t kb = (uint32_t)((sqrt(8.0 * (double)t + 1.0) - 1.0) * 0.5);
-  while ((uint64_t)(kb + 1) * (kb + 2) / 2 <= t) ++kb;
-  while ((uint64_t)kb * (kb + 1) / 2 > t) --kb;
-  uint32_t rb = t - kb * (kb + 1) / 2;
+// Jobs: one k-block (FT kernels) against a run of up to FR r-blocks (rb <= kb).  S(kb) = jobs before k-block kb
+//   = sum_{y=1..kb} ceil(y / FR) = FR q(q+1)/2 + rem (q+1), q = kb / FR, rem = kb % FR.
+constexpr int FR = 8;
+__host__ __device__ __forceinline__ uint64_t filter_jobs_before(uint64_t kb) {
+  const uint64_t q = kb / FR, rem = kb % FR;
+  return FR * q * (q + 1) / 2 + rem * (q + 1);
+}
 
-  const uint32_t k0 = kb * FT, r0 = rb * FT;  // absolute kernel indices
-  __shared__ __align__(16) float pk[16][FTP], pr[16][FTP];
-  __shared__ uint64_t wk[FT], wr[FT];
-  __shared__ uint32_t okk[FT], okr[FT];  // mass > 0 [P-19]
-  const int tid = threadIdx.x;
+// Each thread scores a 4 x 4 block of (k, r) pairs per tile.  Coarse level: the u8-quantised profiles, 4 bins per
+// word, give sum_j |q_k[j] - q_r[j]| with four VABSDIFF4.ACC per pair (the k-side words stay in registers for the
+// whole job); a sum >= thr8 proves D >= theta.  Fine level, only for pairs the coarse level keeps: the fp32
+// profile distance (bin-major shared tiles).  The k-block stays in shared memory for the job; the next r-block is
+// fetched into registers while the current one is scored.  Surviving pairs are appended with one atomic per warp.
+constexpr int FTP = FT + 4;  // row stride (floats) of the bin-major profile tiles
+__device__ __forceinline__ uint32_t sad4(uint32_t a, uint32_t b, uint32_t acc) { return __vsadu4(a, b) + acc; }
+__global__ void __launch_bounds__(256) k_pair_filter(ScanArgs a, uint64_t job0, uint32_t kb_lo, uint32_t kb_hi) {
+  const uint64_t job = job0 + blockIdx.x;
+  uint32_t lo = kb_lo, hi = kb_hi - 1;  // last kb with filter_jobs_before(kb) <= job
+  while (lo < hi) {
+    const uint32_t mid = (lo + hi + 1) >> 1;
+    if (filter_jobs_before(mid) <= job) lo = mid; else hi = mid - 1;
+  }
+  const uint32_t kb = lo;
+  const uint32_t rb0 = (uint32_t)(job - filter_jobs_before(kb)) * FR;
+  const uint32_t rb1 = rb0 + FR - 1 < kb ? rb0 + FR - 1 : kb;  // inclusive
+
+  const uint32_t k0 = kb * FT;
+  __shared__ __align__(16) float pk[16][FTP], prb[2][16][FTP];
+  __shared__ __align__(16) uint4 q8rb[2][FT];
+  __shared__ uint64_t wk[FT], wrb[2][FT];
+  __shared__ uint32_t okk[FT], okrb[2][FT];  // mass > 0 [P-19]
+  const int tid = threadIdx.x, lane = tid & 31;
   for (int i = tid; i < FT * 16; i += 256) {
     const int row = i >> 4, j = i & 15;
-    const uint32_t k = k0 + row, r = r0 + row;
+    const uint32_t k = k0 + row;
     pk[j][row] = k < a.K ? a.prof[(uint64_t)k * 16 + j] : 0.f;
-    pr[j][row] = r < a.K ? a.prof[(uint64_t)r * 16 + j] : 0.f;
   }
-  for (int i = tid; i < FT; i += 256) {
-    const uint32_t k = k0 + i, r = r0 + i;
-    wk[i] = k < a.K ? a.wt[k] : 0;
-    okk[i] = k < a.K && a.mass[k] != 0;
-    wr[i] = r < a.K ? a.wt[r] : 0;
-    okr[i] = r < a.K && a.mass[r] != 0;
+  if (tid < FT) {
+    const uint32_t k = k0 + tid;
+    wk[tid] = k < a.K ? a.wt[k] : 0;
+    okk[tid] = k < a.K && a.mass[k] != 0;
   }
-  __syncthreads();
   const int i0 = (tid >> 4) * 4, j0 = (tid & 15) * 4;
-  float d[4][4];
-#pragma unroll
-  for (int u = 0; u < 4; ++u)
-#pragma unroll
-    for (int v = 0; v < 4; ++v) d[u][v] = 0.f;
-#pragma unroll
-  for (int b = 0; b < 16; ++b) {
-    const float4 x = *(const float4*)&pk[b][i0];
-    const float4 y = *(const float4*)&pr[b][j0];
-    const float xs[4] = {x.x, x.y, x.z, x.w}, ys[4] = {y.x, y.y, y.z, y.w};
-#pragma unroll
-    for (int u = 0; u < 4; ++u)
-#pragma unroll
-      for (int v = 0; v < 4; ++v) d[u][v] += fabsf(xs[u] - ys[v]);
-  }
-  uint32_t keep = 0;  // bit 4u+v
+  uint4 qk[4];  // u8 profiles of this thread's 4 k rows
 #pragma unroll
   for (int u = 0; u < 4; ++u) {
-    const int i = i0 + u;
-    const uint32_t k = k0 + i;
-    const bool kin = k >= a.k_lo && k < a.k_hi && okk[i];
+    const uint32_t k = k0 + i0 + u;
+    qk[u] = k < a.K ? *(const uint4*)(a.prof8 + (uint64_t)k * 4) : make_uint4(0, 0, 0, 0);
+  }
+  // register stage of one r-block: 4 fp32 profile values + one u8 word per thread, (wt, mass != 0) for tid < FT
+  float sv[4];
+  uint32_t sq = 0;
+  uint64_t swr = 0;
+  uint32_t sok = 0;
+  auto fetch = [&](uint32_t rb) {
+#pragma unroll
+    for (int u = 0; u < 4; ++u) {
+      const int i = tid + u * 256, row = i >> 4, j = i & 15;
+      const uint32_t r = rb * FT + row;
+      sv[u] = r < a.K ? a.prof[(uint64_t)r * 16 + j] : 0.f;
+    }
+    {
+      const uint32_t r = rb * FT + (tid >> 2);
+      sq = r < a.K ? a.prof8[(uint64_t)r * 4 + (tid & 3)] : 0u;
+    }
+    if (tid < FT) {
+      const uint32_t r = rb * FT + tid;
+      swr = r < a.K ? a.wt[r] : 0;
+      sok = r < a.K && a.mass[r] != 0;
+    }
+  };
+  auto store = [&](int buf) {
+#pragma unroll
+    for (int u = 0; u < 4; ++u) {
+      const int i = tid + u * 256;
+      prb[buf][i & 15][i >> 4] = sv[u];
+    }
+    ((uint32_t*)q8rb[buf])[tid] = sq;
+    if (tid < FT) { wrb[buf][tid] = swr; okrb[buf][tid] = sok; }
+  };
+  fetch(rb0);
+  store(0);
+  __syncthreads();
+  int cur = 0;
+  for (uint32_t rb = rb0; rb <= rb1; ++rb, cur ^= 1) {
+    if (rb < rb1) fetch(rb + 1);  // in flight while this block is scored
+    const float (*pr)[FTP] = prb[cur];
+    const uint4* q8r = q8rb[cur];
+    const uint64_t* wr = wrb[cur];
+    const uint32_t* okr = okrb[cur];
+    const uint32_t r0 = rb * FT;
+    // coarse level for all 16 pairs (four VABSDIFF4.ACC each); the per-pair eligibility rules only for survivors
+    uint32_t keep = 0;  // bit 4u+v
 #pragma unroll
     for (int v = 0; v < 4; ++v) {
-      const int j = j0 + v;
-      const uint32_t r = r0 + j;
-      const uint64_t Wk = wk[i], Wr = wr[j];
-      const bool ok = kin && r < k && okr[j] && (Wk == Wr || (Wk < Wr ? Wk : Wr) >= a.p.n_cores) &&  // [P-10]
-                      d[u][v] < a.bound;
-      keep |= (ok ? 1u : 0u) << (4 * u + v);
+      const uint4 qr = q8r[j0 + v];
+#pragma unroll
+      for (int u = 0; u < 4; ++u) {
+        const uint32_t sad = sad4(qk[u].w, qr.w, sad4(qk[u].z, qr.z, sad4(qk[u].y, qr.y, __vsadu4(qk[u].x, qr.x))));
+        keep |= (sad < a.thr8 ? 1u : 0u) << (4 * u + v);
+      }
     }
-  }
-  // warp-aggregated append
-  const int lane = tid & 31;
-  const uint32_t cnt = __popc(keep);
-  uint32_t incl = cnt;
-  for (int o = 1; o < 32; o <<= 1) {
-    uint32_t y = __shfl_up_sync(0xffffffffu, incl, o);
-    if (lane >= o) incl += y;
-  }
-  const uint32_t total = __shfl_sync(0xffffffffu, incl, 31);
-  if (total == 0) return;
-  unsigned long long base = 0;
-  if (lane == 31) base = atomicAdd((unsigned long long*)a.n_maybe, (unsigned long long)total);
-  base = __shfl_sync(0xffffffffu, base, 31);
-  unsigned long long pos = base + (incl - cnt);
-  for (uint32_t m = keep; m; m &= m - 1, ++pos) {
-    const int bit = __ffs(m) - 1;
-    const uint32_t k = k0 + i0 + (bit >> 2), r = r0 + j0 + (bit & 3);
-    if (pos < a.cap) a.maybe[pos] = ((uint64_t)k << 32) | r;
-    else latch(a.err, PHOTON_ECAPACITY, (int64_t)pos);
+    for (uint32_t m = keep; m; m &= m - 1) {
+      const int bit = __ffs(m) - 1, i = i0 + (bit >> 2), j = j0 + (bit & 3);
+      const uint32_t k = k0 + i, r = r0 + j;
+      const uint64_t Wk = wk[i], Wr = wr[j];
+      const bool ok = okr[j] && r < k && k >= a.k_lo && k < a.k_hi && okk[i] &&
+                      (Wk == Wr || (Wk < Wr ? Wk : Wr) >= a.p.n_cores);  // [P-10]
+      if (!ok) keep &= ~(1u << bit);
+    }
+    // fine level for the coarse survivors: fp32 profile distance
+    for (uint32_t m = keep; m; m &= m - 1) {
+      const int bit = __ffs(m) - 1, i = i0 + (bit >> 2), j = j0 + (bit & 3);
+      float d = 0.f;
+#pragma unroll
+      for (int b = 0; b < 16; ++b) d += fabsf(pk[b][i] - pr[b][j]);
+      if (!(d < a.bound)) keep &= ~(1u << bit);
+    }
+    // warp-aggregated append
+    const uint32_t cnt = __popc(keep);
+    uint32_t incl = cnt;
+    for (int o = 1; o < 32; o <<= 1) {
+      uint32_t y = __shfl_up_sync(0xffffffffu, incl, o);
+      if (lane >= o) incl += y;
+    }
+    const uint32_t total = __shfl_sync(0xffffffffu, incl, 31);
+    if (total) {
+      unsigned long long base = 0;
+      if (lane == 31) base = atomicAdd((unsigned long long*)a.n_maybe, (unsigned long long)total);
+      base = __shfl_sync(0xffffffffu, base, 31);
+      unsigned long long pos = base + (incl - cnt);
+      for (uint32_t m = keep; m; m &= m - 1, ++pos) {
+        const int bit = __ffs(m) - 1;
+        const uint32_t k = k0 + i0 + (bit >> 2), r = r0 + j0 + (bit & 3);
+        if (pos < a.cap) a.maybe[pos] = ((uint64_t)k << 32) | r;
+        else latch(a.err, PHOTON_ECAPACITY, (int64_t)pos);
+      }
+    }
+    if (rb < rb1) store(cur ^ 1);  // that buffer was last read before the previous barrier
+    __syncthreads();
   }
 }
 
@@ -206,7 +277,42 @@ __device__ __forceinline__ u128 warp_dnum(const uint64_t* sig, const uint64_t* k
   return group_dnum<32>(sig, kto, mass, k, r);
 }
 
-// one group of XG lanes per filtered pair: close <=> theta_den * Dnum < theta_num * N_k * N_r (Fig 12, [P-15])
+// fp64 screen of D = sum_i |g_k[i]/N_k - g_r[i]/N_r| by a group of G lanes (all lanes return the sum).  Every term
+// is computed as RN(RN(g) * RN(1/N)) with g < 2^50 exact in fp64, so each normalised value carries a relative error
+// below 2^-52 and the sum of |a - b| over L terms is within (L + 8) * 2^-50 of D (both profiles have unit mass).
+template <int G>
+__device__ double group_dfp(const uint64_t* __restrict__ sig, const uint64_t* __restrict__ kto,
+                            const double* __restrict__ invn, uint32_t k, uint32_t r, bool act, uint64_t& Lout) {
+  const uint32_t l = threadIdx.x & (G - 1);
+  uint64_t Lk = 0, Lr = 0;
+  const uint64_t* pk = sig;
+  const uint64_t* pr = sig;
+  double ik = 0.0, ir = 0.0;
+  if (act) {
+    const uint64_t ok = kto[k], orr = kto[r];
+    Lk = (kto[k + 1] - ok) * 16;
+    Lr = (kto[r + 1] - orr) * 16;
+    pk = sig + ok * 16;
+    pr = sig + orr * 16;
+    ik = invn[k];
+    ir = invn[r];
+  }
+  const uint64_t L = Lk > Lr ? Lk : Lr;
+  double acc = 0.0;
+#pragma unroll 4
+  for (uint64_t i = l; i < L; i += G) {
+    const double a = i < Lk ? (double)pk[i] * ik : 0.0;
+    const double b = i < Lr ? (double)pr[i] * ir : 0.0;
+    acc += fabs(a - b);
+  }
+  for (int o = G / 2; o > 0; o >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, o);
+  Lout = L;
+  return acc;
+}
+
+// one group of XG lanes per filtered pair: close <=> theta_den * Dnum < theta_num * N_k * N_r (Fig 12, [P-15]).
+// The fp64 screen decides every pair whose distance is farther than its error bound from theta; the rest (ties
+// within ~1e-9) take the exact u128 sum.
 constexpr int XG = 8;
 __global__ void __launch_bounds__(256) k_pair_exact(ScanArgs a, uint64_t* pairs, uint64_t pair_cap,
                                                     uint64_t* n_pairs) {
@@ -215,19 +321,25 @@ __global__ void __launch_bounds__(256) k_pair_exact(ScanArgs a, uint64_t* pairs,
   const uint64_t g = ((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) / XG;
   const uint64_t ng = ((uint64_t)gridDim.x * blockDim.x) / XG;
   const uint64_t rounds = (n + ng - 1) / ng;  // every lane runs the same number of rounds (shuffles stay converged)
+  const double theta = (double)a.p.theta_num / (double)a.p.theta_den;
   for (uint64_t it = 0; it < rounds; ++it) {
     const uint64_t q = g + it * ng;
     const bool act = q < n;
     const uint64_t pr = act ? a.maybe[q] : 0;
     const uint32_t k = (uint32_t)(pr >> 32), r = (uint32_t)pr;
-    const u128 d = group_dnum<XG>(a.sig, a.kto, a.mass, k, r, act);
-    if (act && (threadIdx.x & (XG - 1)) == 0) {
-      const u128 rhs = (u128)a.p.theta_num * ((u128)a.mass[k] * a.mass[r]);
-      if ((u128)a.p.theta_den * d < rhs) {
-        const unsigned long long pos = atomicAdd((unsigned long long*)n_pairs, 1ull);
-        if (pos < pair_cap) pairs[pos] = pr;
-        else latch(a.err, PHOTON_ECAPACITY, (int64_t)pos);
-      }
+    uint64_t L = 0;
+    const double d = group_dfp<XG>(a.sig, a.kto, a.invn, k, r, act, L);
+    const double eps = (double)(L + 8) * 0x1p-50 + theta * 0x1p-50;
+    bool close = d < theta - eps;
+    const bool unsure = act && !close && !(d > theta + eps);
+    if (__any_sync(0xffffffffu, unsure)) {  // rare: exact u128 decision for this round's unsure pairs
+      const u128 dn = group_dnum<XG>(a.sig, a.kto, a.mass, k, r, unsure);
+      if (unsure) close = (u128)a.p.theta_den * dn < (u128)a.p.theta_num * ((u128)a.mass[k] * a.mass[r]);
+    }
+    if (act && close && (threadIdx.x & (XG - 1)) == 0) {
+      const unsigned long long pos = atomicAdd((unsigned long long*)n_pairs, 1ull);
+      if (pos < pair_cap) pairs[pos] = pr;
+      else latch(a.err, PHOTON_ECAPACITY, (int64_t)pos);
     }
   }
 }
@@ -358,6 +470,75 @@ __global__ void __launch_bounds__(1024) k_resolve_states(uint32_t K, const uint6
   if (threadIdx.x == 0) flag[0] = rounds;
 }
 
+// The same fixed point over the whole GPU: a cooperative grid, one grid-wide barrier per round (rounds are few: the
+// longest chain of kernels blocked on undecided predecessors).  Each round visits the undecided list of the previous
+// round; a blocked kernel keeps its cursor.  Stale state reads only postpone a decision (states are monotone).
+__global__ void __launch_bounds__(256) k_resolve_coop(uint32_t K, const uint64_t* __restrict__ off,
+                                                      const uint32_t* __restrict__ cand, uint8_t* state,
+                                                      uint32_t* cursor, uint32_t* ulist, uint32_t* rcnt,
+                                                      uint32_t* flag) {
+  namespace cg = cooperative_groups;
+  cg::grid_group grid = cg::this_grid();
+  const uint64_t gt = grid.thread_rank(), gs = grid.size();
+  for (uint64_t k = gt; k < K; k += gs) {
+    state[k] = 0;
+    cursor[k] = 0;
+  }
+  for (uint64_t i = gt; i < (uint64_t)K + 2; i += gs) rcnt[i] = 0;
+  grid.sync();
+  volatile uint8_t* vs = state;
+  const uint32_t lane = threadIdx.x & 31;
+  const uint64_t gw = gt >> 5, nw = gs >> 5;
+  uint32_t n = K;
+  const uint32_t* cur = nullptr;  // nullptr = identity (round 1 visits every kernel)
+  uint32_t* nxt = ulist;
+  uint32_t round = 0;
+  for (;;) {
+    // one warp per undecided kernel: 128 candidates (4 x 32 independent loads) per step, ballots decide
+    for (uint64_t q = gw; q < n; q += nw) {
+      const uint32_t k = cur ? cur[q] : (uint32_t)q;
+      const uint64_t o0 = off[k], o1 = off[k + 1];
+      uint64_t first_undec = o1;
+      bool rep_found = false;
+      for (uint64_t i0 = o0 + cursor[k]; i0 < o1; i0 += 128) {
+        uint32_t c4[4];
+#pragma unroll
+        for (int u = 0; u < 4; ++u) {
+          const uint64_t i = i0 + u * 32 + lane;
+          c4[u] = i < o1 ? cand[i] : UINT32_MAX;
+        }
+        uint8_t st[4];
+#pragma unroll
+        for (int u = 0; u < 4; ++u) st[u] = c4[u] != UINT32_MAX ? vs[c4[u]] : (uint8_t)2;
+        bool stop = false;
+#pragma unroll
+        for (int u = 0; u < 4; ++u) {
+          const unsigned rep = __ballot_sync(0xffffffffu, st[u] == 1);
+          const unsigned und = __ballot_sync(0xffffffffu, st[u] == 0);
+          if (rep) { rep_found = true; stop = true; break; }
+          if (und && first_undec == o1) first_undec = i0 + u * 32 + (__ffs(und) - 1);
+        }
+        if (stop) break;
+      }
+      if (lane == 0) {
+        if (!rep_found && first_undec < o1) {  // blocked by an undecided predecessor: resume there next round
+          cursor[k] = (uint32_t)(first_undec - o0);
+          nxt[atomicAdd(&rcnt[round], 1u)] = k;
+        } else {
+          vs[k] = rep_found ? 2 : 1;
+        }
+      }
+    }
+    grid.sync();
+    n = *(volatile uint32_t*)&rcnt[round];
+    ++round;
+    if (n == 0 || round > K) break;
+    cur = nxt;  // ping-pong between the two halves of ulist (the other half was fully read before the barrier)
+    nxt = (cur == ulist) ? ulist + K : ulist;
+  }
+  if (gt == 0) flag[0] = round;
+}
+
 // match[k] = argmin over eligible candidates of (|W_k - W_r|, r); match_dist exact -> fp64 (one warp per kernel)
 __global__ void k_resolve_match(uint32_t K, const uint64_t* off, const uint32_t* cand, const uint8_t* state,
                                 uint32_t pool_all, const uint64_t* wt, const uint64_t* kto, const uint64_t* sig,
@@ -414,20 +595,20 @@ cudaError_t launch_match_scan(uint32_t K, const uint64_t* kto, const uint64_t* s
   cudaMemsetAsync(n_pairs, 0, 8, s);
   cudaMemsetAsync(mw.n_maybe, 0, 8, s);
   if (K == 0 || k_hi <= k_lo) return cudaGetLastError();
-  note_launch(), k_prof<<<(unsigned)ceil_div((uint64_t)K * 32, 256), 256, 0, s>>>(K, kto, sig, mass, mw.prof);
+  note_launch(), k_prof<<<(unsigned)ceil_div((uint64_t)K * 32, 256), 256, 0, s>>>(K, kto, sig, mass, mw.prof, mw.invn,
+                                                                                mw.prof8);
   ScanArgs a{};
-  a.K = K; a.k_lo = k_lo; a.k_hi = k_hi; a.kto = kto; a.sig = sig; a.mass = mass; a.wt = wt; a.prof = mw.prof;
+  a.K = K; a.k_lo = k_lo; a.k_hi = k_hi; a.kto = kto; a.sig = sig; a.mass = mass; a.wt = wt; a.prof = mw.prof; a.invn = mw.invn; a.prof8 = mw.prof8;
   a.p = p;
   // rigorous margin: each |P_k - P_r| term carries <= 3 fp32 roundings of values in [0, 1] plus 16 additions
   a.bound = (float)((double)p.theta_num / (double)p.theta_den) + 1e-5f;
+  // |q - 255 P| <= 1/2 + 2^-40 per value, so sum_j |q_k - q_r| <= 255 sum_j |P_k - P_r| + 16 + 2^-30 <= 255 D + 17:
+  // a pair with sum >= 255 theta + 17 has D >= theta
+  a.thr8 = (uint32_t)ceil(255.0 * (double)p.theta_num / (double)p.theta_den + 17.0);
   a.maybe = mw.maybe; a.n_maybe = mw.n_maybe; a.cap = mw.pair_cap; a.err = err;
-  uint32_t kb_hi = (uint32_t)ceil_div(k_hi, FT);
-  uint32_t kb_lo = k_lo / FT;
-  // tiles (kb, rb) with kb in [kb_lo, kb_hi), rb <= kb: enumerate t in [kb_lo(kb_lo+1)/2, kb_hi(kb_hi+1)/2)
-  uint64_t t0 = (uint64_t)kb_lo * (kb_lo + 1) / 2, t1 = (uint64_t)kb_hi * (kb_hi + 1) / 2;
-  // launch with blockIdx offset by t0 via a shifted grid: simplest is to launch t1 tiles and skip kb < kb_lo
-
-  if (t1 > t0) note_launch(), k_pair_filter<<<(unsigned)(t1 - t0), 256, 0, s>>>(a, t0);
+  const uint32_t kb_hi = (uint32_t)ceil_div(k_hi, FT), kb_lo = k_lo / FT;
+  const uint64_t j0 = filter_jobs_before(kb_lo), j1 = filter_jobs_before(kb_hi);
+  if (j1 > j0) note_launch(), k_pair_filter<<<(unsigned)(j1 - j0), 256, 0, s>>>(a, j0, kb_lo, kb_hi);
   unsigned grid = (unsigned)num_sms * 8;
   note_launch(), k_pair_exact<<<grid, 256, 0, s>>>(a, pairs, pair_cap, n_pairs);
   return cudaGetLastError();
@@ -436,7 +617,7 @@ cudaError_t launch_match_scan(uint32_t K, const uint64_t* kto, const uint64_t* s
 cudaError_t launch_match_resolve(uint32_t K, const uint64_t* kto, const uint64_t* sig, const uint64_t* mass,
                                  const uint64_t* wt, photon_match_params p, const uint64_t* pairs, uint64_t n_pairs,
                                  const uint64_t* n_pairs_dev, const MatchWs& mw, int64_t* match, double* match_dist,
-                                 DevErr* err, cudaStream_t s) {
+                                 DevErr* err, int num_sms, cudaStream_t s) {
   if (K == 0) return cudaSuccess;
   cudaMemsetAsync(mw.cand_cnt, 0, sizeof(uint32_t) * K, s);
   if (n_pairs) {
@@ -447,7 +628,21 @@ cudaError_t launch_match_resolve(uint32_t K, const uint64_t* kto, const uint64_t
     note_launch(), k_cand_scatter<<<(unsigned)ceil_div(n_pairs, 256), 256, 0, s>>>(pairs, n_pairs, n_pairs_dev, K, mw.cand_off,
                                                                     mw.cand_cur, mw.cand);
   }
-  if (K <= 40960) {
+  if (!p.pool_all_prior && K > 2048) {  // large K: the whole GPU, one grid barrier per round
+    static int per_sm = 0;
+    if (!per_sm) {
+      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_resolve_coop, 256, 0);
+      if (per_sm < 1) per_sm = 1;
+    }
+    unsigned grid = (unsigned)umin64((uint64_t)per_sm * num_sms, ceil_div((uint64_t)K * 32, 256));
+    const uint64_t* off = mw.cand_off;
+    const uint32_t* cand = mw.cand;
+    void* args[] = {(void*)&K, (void*)&off, (void*)&cand, (void*)&mw.state, (void*)&mw.cand_cur, (void*)&mw.ulist,
+                    (void*)&mw.rcnt, (void*)&mw.flag};
+    note_launch();
+    cudaError_t e = cudaLaunchCooperativeKernel((void*)k_resolve_coop, grid, 256, args, 0, s);
+    if (e != cudaSuccess) return e;
+  } else if (K <= 40960) {
     cudaFuncSetAttribute(k_resolve_states<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, 40960);
     note_launch(), k_resolve_states<true><<<1, 1024, K, s>>>(K, mw.cand_off, mw.cand, mw.state, mw.cand_cur, mw.ulist,
                                                               mw.flag, p.pool_all_prior);

@@ -190,16 +190,37 @@ __global__ void __launch_bounds__(256) k_sort_warp(HashTable ht, uint32_t K, con
     }
     return;
   }
+  // register bitonic over (count, key words 0-3, slot): values travel with the slot; full-key compare only on ties
   uint32_t mine = lane < n ? list[off + lane] : UINT32_MAX;
+  uint32_t mc = 0;
+  uint4 mk = make_uint4(0, 0, 0, 0);
+  if (mine != UINT32_MAX) {
+    mc = ht.count[mine];
+    mk = *(const uint4*)(ht.key + (uint64_t)mine * 16);
+  }
   for (uint32_t size = 2; size <= 32; size <<= 1) {
     for (uint32_t stride = size >> 1; stride > 0; stride >>= 1) {
-      uint32_t other = __shfl_xor_sync(0xffffffffu, mine, stride);
-      bool up = (lane & size) == 0;
-      bool lower = (lane & stride) == 0;
-      bool mb = type_before(ht, mine, other);
+      const uint32_t other = __shfl_xor_sync(0xffffffffu, mine, stride);
+      const uint32_t oc = __shfl_xor_sync(0xffffffffu, mc, stride);
+      uint4 ok;
+      ok.x = __shfl_xor_sync(0xffffffffu, mk.x, stride);
+      ok.y = __shfl_xor_sync(0xffffffffu, mk.y, stride);
+      ok.z = __shfl_xor_sync(0xffffffffu, mk.z, stride);
+      ok.w = __shfl_xor_sync(0xffffffffu, mk.w, stride);
+      const bool up = (lane & size) == 0;
+      const bool lower = (lane & stride) == 0;
+      bool mb;  // mine before other (padding last)
+      if (other == UINT32_MAX) mb = mine != UINT32_MAX;
+      else if (mine == UINT32_MAX) mb = false;
+      else if (mc != oc) mb = mc > oc;
+      else if (mk.x != ok.x) mb = mk.x < ok.x;
+      else if (mk.y != ok.y) mb = mk.y < ok.y;
+      else if (mk.z != ok.z) mb = mk.z < ok.z;
+      else if (mk.w != ok.w) mb = mk.w < ok.w;
+      else mb = type_before(ht, mine, other);  // words 4.. (rare)
       bool keep = (lower == up) ? mb : !mb;
       if (mine == other) keep = true;
-      mine = keep ? mine : other;
+      if (!keep) { mine = other; mc = oc; mk = ok; }
     }
   }
   if (lane < n && off + lane < out.capacity) {
@@ -210,7 +231,7 @@ __global__ void __launch_bounds__(256) k_sort_warp(HashTable ht, uint32_t K, con
     out.type_first_warp[off + lane] = ht.first[mine];
     canon[mine] = lane;
   }
-  uint32_t c0 = __shfl_sync(0xffffffffu, mine != UINT32_MAX ? ht.count[mine] : 0u, 0);
+  uint32_t c0 = __shfl_sync(0xffffffffu, mine != UINT32_MAX ? mc : 0u, 0);
   if (lane == 0) out.warp_sampling_ok[k] = (Wk > 0 && 100ull * c0 > 95ull * Wk) ? 1 : 0;  // L249 [P-15]
 }
 
@@ -317,19 +338,31 @@ __global__ void k_entries_insert(TileEntries te, uint64_t n_tiles, HashTable ht,
   *out = ht_insert(ht, err, x->kernel, key, x->hash, x->count, x->first);
 }
 
-// K2c: warp_type[w] = canonical id of the warp's tile entry
-__global__ void k_remap_entries(TileEntries te, uint64_t W, const uint32_t* canon, uint32_t* warp_type) {
-  const uint64_t w = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
-  if (w >= W) return;
-  const uint32_t g = te.gid[w];
-  uint32_t slot;
-  if (!(g >> 31)) {
-    slot = te.tile_slot[g];
-  } else {
-    const uint64_t j = g & 0x7FFFFFFFu;  // beyond ovf_cap only after ECAPACITY was latched
-    slot = j < te.ovf_cap ? te.ovf_slot[j] : UINT32_MAX;
+// K2c: warp_type[w] = canonical id of the warp's tile entry.  Four warps per thread (strided by the grid) so each
+// thread keeps four independent gid -> slot -> canon chains in flight.
+constexpr int REMAP_ILP = 4;
+__device__ __forceinline__ uint32_t entry_slot(const TileEntries& te, uint32_t g) {
+  if (!(g >> 31)) return te.tile_slot[g];
+  const uint64_t j = g & 0x7FFFFFFFu;  // beyond ovf_cap only after ECAPACITY was latched
+  return j < te.ovf_cap ? te.ovf_slot[j] : UINT32_MAX;
+}
+__global__ void __launch_bounds__(256) k_remap_entries(TileEntries te, uint64_t W, const uint32_t* canon,
+                                                       uint32_t* warp_type) {
+  const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+  const uint64_t w0 = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  uint32_t g[REMAP_ILP], sl[REMAP_ILP];
+#pragma unroll
+  for (int u = 0; u < REMAP_ILP; ++u) {
+    const uint64_t w = w0 + u * stride;
+    g[u] = w < W ? te.gid[w] : 0u;
   }
-  warp_type[w] = slot == UINT32_MAX ? UINT32_MAX : canon[slot];
+#pragma unroll
+  for (int u = 0; u < REMAP_ILP; ++u) sl[u] = w0 + u * stride < W ? entry_slot(te, g[u]) : UINT32_MAX;
+#pragma unroll
+  for (int u = 0; u < REMAP_ILP; ++u) {
+    const uint64_t w = w0 + u * stride;
+    if (w < W) warp_type[w] = sl[u] == UINT32_MAX ? UINT32_MAX : canon[sl[u]];
+  }
 }
 
 __device__ __forceinline__ uint32_t row_kernel(const uint64_t* kto, uint32_t K, uint64_t row) {
@@ -433,7 +466,8 @@ cudaError_t launch_canonicalise(const HashTable& ht, uint32_t K, const uint64_t*
 cudaError_t launch_entries_insert(const TileEntries& te, uint64_t n_tiles, const HashTable& ht, DevErr* err,
                                   cudaStream_t s) {
   // fixed entry slots one thread each (rounded up to whole CTAs), then 64K threads striding over the overflow
-  uint64_t n = ceil_div(n_tiles * te.per_tile, 256) * 256 + 65536;
+  // one thread per fixed slot, then one per possible overflow entry (the device count is unknown here)
+  uint64_t n = ceil_div(n_tiles * te.per_tile, 256) * 256 + ceil_div(te.ovf_cap, 256) * 256;
   if (n == 0) return cudaSuccess;
   note_launch(), k_entries_insert<<<(unsigned)ceil_div(n, 256), 256, 0, s>>>(te, n_tiles, ht, err);
   return cudaGetLastError();
@@ -442,7 +476,8 @@ cudaError_t launch_entries_insert(const TileEntries& te, uint64_t n_tiles, const
 cudaError_t launch_remap_entries(const TileEntries& te, uint64_t W, const uint32_t* canon, uint32_t* warp_type,
                                  cudaStream_t s) {
   if (W == 0) return cudaSuccess;
-  note_launch(), k_remap_entries<<<(unsigned)ceil_div(W, 256), 256, 0, s>>>(te, W, canon, warp_type);
+  note_launch(), k_remap_entries<<<(unsigned)ceil_div(ceil_div(W, REMAP_ILP), 256), 256, 0, s>>>(te, W, canon,
+                                                                                                 warp_type);
   return cudaGetLastError();
 }
 

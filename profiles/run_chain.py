@@ -15,6 +15,7 @@ reps = int(sys.argv[2]) if len(sys.argv) > 2 else 3
 ph = Photon(0)
 g = tg.Generator(cfg)
 d = DeviceTrace.from_host(g.trace(), ph.device)
+ph.analyse(d)  # checked once: learns the table / pair capacities (an unchecked call never retries)
 for _ in range(reps):
     ph.analyse(d, check=False)
 torch.cuda.synchronize()

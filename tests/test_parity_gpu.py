@@ -278,3 +278,40 @@ def test_stable_many_bb(ph, B):
     kbb = rng.integers(0, 1000, (7, B)).astype(np.uint64)
     fs = check_stable(ph, tm, kbb, 16)
     assert (fs >= 0).sum() > 10
+
+
+@pytest.mark.parametrize("K", [3000, 6000])
+def test_match_many_kernels_synthetic(ph, K):
+    # K > 2048 takes the cooperative (grid-barrier) resolution; type tables are synthetic clusters of near-copies
+    # (many close pairs, long launch-order chains), checked against the oracle's signature + match
+    from paper_conf_micro_liusc23_b200 import to_device
+    rng = np.random.default_rng(K)
+    n_tmpl = 40
+    tmpl = rng.integers(1, 400, (n_tmpl, 4, 16)).astype(np.uint32)
+    T = rng.integers(1, 5, K)
+    kto = np.zeros(K + 1, np.uint64)
+    kto[1:] = np.cumsum(T)
+    keys, counts = [], []
+    for k in range(K):
+        t = rng.integers(0, n_tmpl)
+        for r in range(T[k]):
+            key = tmpl[t, r].astype(np.int64) + rng.integers(-2, 3, 16) * (rng.random(16) < 0.3)
+            keys.append(np.clip(key, 0, None).astype(np.uint32))
+            counts.append(int(rng.integers(50, 60) if r == 0 else rng.integers(1, 8)))
+    keys = np.array(keys, np.uint32)
+    counts = np.array(counts, np.uint64)
+    wt = np.where(rng.random(K) < 0.5, 64 + rng.integers(0, 200, K), rng.integers(1, 4, K) * 16).astype(np.uint64)
+    ty = ph.alloc_types(K, 1, len(counts))
+    ty["kernel_type_off"].copy_(to_device(kto, ph.device))
+    ty["type_key"].copy_(to_device(keys.reshape(-1), ph.device))
+    ty["type_count"].copy_(to_device(counts, ph.device))
+    m = ph.photon_kernel_match(K, ty, to_device(wt, ph.device), (1, 20), 64, 0, want_dist=True)
+    sig, mass = oracle.signature(kto, keys, counts)
+    om, od = oracle.match(kto, sig, mass, wt, (1, 20), 64, 0)
+    gm = _np(m["match"], np.int64)
+    assert (om >= 0).sum() > K // 4  # the clusters really produce matches
+    assert np.array_equal(gm, om)
+    gd = _np(m["match_dist"], np.float64)
+    fin = np.isfinite(od)
+    assert np.array_equal(np.isfinite(gd), fin)
+    np.testing.assert_allclose(gd[fin], od[fin], rtol=1e-6, atol=0)
