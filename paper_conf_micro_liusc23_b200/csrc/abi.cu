@@ -214,6 +214,7 @@ MatchLayout match_layout(uint32_t K, uint64_t T, uint64_t pair_cap, void* base) 
   m.mass = c.take<uint64_t>(K + 1);
   m.mw.prof = c.take<float>(16ull * K + 16);
   m.mw.invn = c.take<double>(K + 1);
+  m.mw.sigf = c.take<float>(16 * (T ? T : 1));
   m.mw.prof8 = c.take<uint32_t>(4ull * K + 4);
   m.mw.maybe = c.take<uint64_t>(pair_cap);
   m.mw.n_maybe = c.take<uint64_t>(1);
@@ -551,6 +552,7 @@ int photon_match_scan(photon_ctx* ctx, uint32_t K, const uint64_t* kto, const ui
   CK(cudaSetDevice(ctx->device), "cudaSetDevice");
   ctx->last_ws = ws;
   CK(cudaMemsetAsync(m.err, 0, sizeof(DevErr), s), "memset");
+  m.mw.sigf = nullptr;  // T is not known here: the exact screen converts the u64 signature on the fly
   CK(launch_match_scan(K, kto, sig, mass, warps_total, params, k_lo, k_hi, m.mw, pairs, pair_capacity, n_pairs, m.err,
                        ctx->num_sms, s),
      "scan");

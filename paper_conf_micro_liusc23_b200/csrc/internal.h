@@ -109,6 +109,7 @@ cudaError_t launch_remap_direct(const uint64_t* kwo_local, uint32_t K_local, uin
 struct MatchWs {
   float* prof;         // [K][16] normalised per-bin profile (filter)
   double* invn;        // [K] 1 / N_k (fp64 screen of the exact check)
+  float* sigf;         // [16 T] g / N in fp32 (screen of the exact check; nullptr: converted on the fly)
   uint32_t* prof8;     // [K][4] the profile quantised to u8 (round(255 P)), packed 4 bins per word (coarse filter)
   uint64_t* maybe;     // [pair_cap] profile-filter survivors
   uint64_t* n_maybe;   // [1]

@@ -17,6 +17,13 @@
 
 #include "internal.h"
 
+#ifndef PHOTON_UNR
+#define PHOTON_UNR 8  // exact-check unroll (profiling builds may override)
+#endif
+namespace photon {
+constexpr int kExactUnroll = PHOTON_UNR;
+}
+
 namespace photon {
 
 namespace {
@@ -54,13 +61,18 @@ __global__ void k_sig(uint32_t k_lo, uint32_t k_hi, const uint64_t* __restrict__
 // per-bin profile P_k[j] = sum_t g[16t+j] / N_k (filter only), one warp per kernel
 __global__ void k_prof(uint32_t K, const uint64_t* __restrict__ kto, const uint64_t* __restrict__ sig,
                        const uint64_t* __restrict__ mass, float* __restrict__ prof, double* __restrict__ invn,
-                       uint32_t* __restrict__ prof8) {
+                       uint32_t* __restrict__ prof8, float* __restrict__ sigf) {
   uint32_t warp = (blockIdx.x * blockDim.x + threadIdx.x) >> 5, lane = threadIdx.x & 31;
   if (warp >= K) return;
   uint32_t k = warp;
   uint64_t r0 = kto[k], r1 = kto[k + 1];
   uint64_t acc = 0;
-  for (uint64_t r = r0 + (lane >> 4); r < r1; r += 2) acc += sig[r * 16 + (lane & 15)];
+  const double inv = mass[k] ? 1.0 / (double)mass[k] : 0.0;
+  for (uint64_t r = r0 + (lane >> 4); r < r1; r += 2) {
+    const uint64_t g = sig[r * 16 + (lane & 15)];
+    acc += g;
+    if (sigf) sigf[r * 16 + (lane & 15)] = (float)((double)g * inv);
+  }
   acc += __shfl_xor_sync(0xffffffffu, acc, 16);
   const uint64_t N = mass[k];
   const double P = N ? (double)acc / (double)N : 0.0;
@@ -89,6 +101,7 @@ struct ScanArgs {
   const uint32_t* prof8;
   uint32_t thr8;  // coarse reject: sum_j |q_k[j] - q_r[j]| >= thr8 implies D >= theta
   const double* invn;
+  const float* sigf;
   photon_match_params p;
   float bound;  // reject if profile distance >= bound
   uint64_t* maybe;
@@ -277,43 +290,61 @@ __device__ __forceinline__ u128 warp_dnum(const uint64_t* sig, const uint64_t* k
   return group_dnum<32>(sig, kto, mass, k, r);
 }
 
-// fp64 screen of D = sum_i |g_k[i]/N_k - g_r[i]/N_r| by a group of G lanes (all lanes return the sum).  Every term
-// is computed as RN(RN(g) * RN(1/N)) with g < 2^50 exact in fp64, so each normalised value carries a relative error
-// below 2^-52 and the sum of |a - b| over L terms is within (L + 8) * 2^-50 of D (both profiles have unit mass).
+// Screen of D = sum_i |g_k[i]/N_k - g_r[i]/N_r| by a group of G lanes (all lanes return the sum and its error
+// bound).  With the fp32 copy sigf (each value RN32(g / N), relative error <= 2^-24, unit mass per kernel) the fp32
+// |a - b| terms and their fp32 sum are within (L + 8) * 2^-21 of D.  Without it every term is RN(RN(g) * RN(1/N))
+// in fp64 (g < 2^50 is exact), within (L + 8) * 2^-50.
 template <int G>
-__device__ double group_dfp(const uint64_t* __restrict__ sig, const uint64_t* __restrict__ kto,
-                            const double* __restrict__ invn, uint32_t k, uint32_t r, bool act, uint64_t& Lout) {
+__device__ double group_dfp(const uint64_t* __restrict__ sig, const float* __restrict__ sigf,
+                            const uint64_t* __restrict__ kto, const double* __restrict__ invn, uint32_t k, uint32_t r,
+                            bool act, double& eps) {
   const uint32_t l = threadIdx.x & (G - 1);
-  uint64_t Lk = 0, Lr = 0;
-  const uint64_t* pk = sig;
-  const uint64_t* pr = sig;
+  uint64_t Lk = 0, Lr = 0, ok = 0, orr = 0;
   double ik = 0.0, ir = 0.0;
   if (act) {
-    const uint64_t ok = kto[k], orr = kto[r];
+    ok = kto[k];
+    orr = kto[r];
     Lk = (kto[k + 1] - ok) * 16;
     Lr = (kto[r + 1] - orr) * 16;
-    pk = sig + ok * 16;
-    pr = sig + orr * 16;
     ik = invn[k];
     ir = invn[r];
   }
   const uint64_t L = Lk > Lr ? Lk : Lr;
   double acc = 0.0;
-#pragma unroll 4
-  for (uint64_t i = l; i < L; i += G) {
-    const double a = i < Lk ? (double)pk[i] * ik : 0.0;
-    const double b = i < Lr ? (double)pr[i] * ir : 0.0;
-    acc += fabs(a - b);
+  if (sigf) {
+    const float* pk = sigf + ok * 16;
+    const float* pr = sigf + orr * 16;
+    float af = 0.f;
+#pragma unroll kExactUnroll
+    for (uint64_t i = l; i < L; i += G) {
+      const float a = i < Lk ? pk[i] : 0.f;
+      const float b = i < Lr ? pr[i] : 0.f;
+      af += fabsf(a - b);
+    }
+    acc = af;
+    eps = (double)(L + 8) * 0x1p-21;
+  } else {
+    const uint64_t* pk = sig + ok * 16;
+    const uint64_t* pr = sig + orr * 16;
+#pragma unroll kExactUnroll
+    for (uint64_t i = l; i < L; i += G) {
+      const double a = i < Lk ? (double)pk[i] * ik : 0.0;
+      const double b = i < Lr ? (double)pr[i] * ir : 0.0;
+      acc += fabs(a - b);
+    }
+    eps = (double)(L + 8) * 0x1p-50;
   }
   for (int o = G / 2; o > 0; o >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, o);
-  Lout = L;
   return acc;
 }
 
 // one group of XG lanes per filtered pair: close <=> theta_den * Dnum < theta_num * N_k * N_r (Fig 12, [P-15]).
 // The fp64 screen decides every pair whose distance is farther than its error bound from theta; the rest (ties
 // within ~1e-9) take the exact u128 sum.
-constexpr int XG = 8;
+#ifndef PHOTON_XG
+#define PHOTON_XG 16  // lanes per pair (profiling builds may override)
+#endif
+constexpr int XG = PHOTON_XG;
 __global__ void __launch_bounds__(256) k_pair_exact(ScanArgs a, uint64_t* pairs, uint64_t pair_cap,
                                                     uint64_t* n_pairs) {
   uint64_t n = *a.n_maybe;
@@ -327,9 +358,9 @@ __global__ void __launch_bounds__(256) k_pair_exact(ScanArgs a, uint64_t* pairs,
     const bool act = q < n;
     const uint64_t pr = act ? a.maybe[q] : 0;
     const uint32_t k = (uint32_t)(pr >> 32), r = (uint32_t)pr;
-    uint64_t L = 0;
-    const double d = group_dfp<XG>(a.sig, a.kto, a.invn, k, r, act, L);
-    const double eps = (double)(L + 8) * 0x1p-50 + theta * 0x1p-50;
+    double eps = 0.0;
+    const double d = group_dfp<XG>(a.sig, a.sigf, a.kto, a.invn, k, r, act, eps);
+    eps += theta * 0x1p-50;
     bool close = d < theta - eps;
     const bool unsure = act && !close && !(d > theta + eps);
     if (__any_sync(0xffffffffu, unsure)) {  // rare: exact u128 decision for this round's unsure pairs
@@ -596,9 +627,9 @@ cudaError_t launch_match_scan(uint32_t K, const uint64_t* kto, const uint64_t* s
   cudaMemsetAsync(mw.n_maybe, 0, 8, s);
   if (K == 0 || k_hi <= k_lo) return cudaGetLastError();
   note_launch(), k_prof<<<(unsigned)ceil_div((uint64_t)K * 32, 256), 256, 0, s>>>(K, kto, sig, mass, mw.prof, mw.invn,
-                                                                                mw.prof8);
+                                                                                mw.prof8, mw.sigf);
   ScanArgs a{};
-  a.K = K; a.k_lo = k_lo; a.k_hi = k_hi; a.kto = kto; a.sig = sig; a.mass = mass; a.wt = wt; a.prof = mw.prof; a.invn = mw.invn; a.prof8 = mw.prof8;
+  a.K = K; a.k_lo = k_lo; a.k_hi = k_hi; a.kto = kto; a.sig = sig; a.mass = mass; a.wt = wt; a.prof = mw.prof; a.invn = mw.invn; a.prof8 = mw.prof8; a.sigf = mw.sigf;
   a.p = p;
   // rigorous margin: each |P_k - P_r| term carries <= 3 fp32 roundings of values in [0, 1] plus 16 additions
   a.bound = (float)((double)p.theta_num / (double)p.theta_den) + 1e-5f;
