@@ -237,7 +237,7 @@ MatchLayout match_layout(uint32_t K, uint64_t T, uint64_t pair_cap, void* base) 
 MatchLayout match_layout_fit(uint32_t K, uint64_t T, void* base, size_t ws_bytes) {
   uint64_t cap = 16ull * K + 65536;
   MatchLayout m = match_layout(K, T, cap, nullptr);
-  while (m.bytes > ws_bytes && cap > 1024) { cap /= 2; m = match_layout(K, T, cap, nullptr); }
+  while (m.bytes > ws_bytes && cap > 1) { cap /= 2; m = match_layout(K, T, cap, nullptr); }
   for (;;) {
     MatchLayout bigger = match_layout(K, T, cap * 2, nullptr);
     if (bigger.bytes > ws_bytes) break;
@@ -570,9 +570,11 @@ int photon_match_resolve(photon_ctx* ctx, uint32_t K, const uint64_t* kto, const
   int rc = check_match_params(ctx, params);
   if (rc) return rc;
   // resolve needs cand arrays for n_pairs entries
+  // (exactly the layout photon_match_workspace_bytes(K, 1, n_pairs) sized: a fitted layout could pick a larger
+  // pair capacity than the buffer holds and carve the state arrays past its end)
   MatchLayout m = match_layout(K, 1, n_pairs ? n_pairs : 1, nullptr);
   if (ws_bytes < m.bytes) return fail(ctx, PHOTON_EWORKSPACE, "workspace %zu < %zu bytes", ws_bytes, m.bytes);
-  m = match_layout_fit(K, 1, ws, ws_bytes);
+  m = match_layout(K, 1, n_pairs ? n_pairs : 1, ws);
   cudaStream_t s = (cudaStream_t)stream;
   CK(cudaSetDevice(ctx->device), "cudaSetDevice");
   ctx->last_ws = ws;
