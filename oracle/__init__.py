@@ -55,6 +55,8 @@ def _L():
         L.or_match.argtypes = [u32, vp, vp, vp, vp, u32, u32, u64, u32, vp, vp]
         L.or_stable.restype = i32
         L.or_stable.argtypes = [u32, u32, u64, vp, vp, vp, vp, vp, u32, u32, u32, u32, u32, i32, vp, vp, vp, vp]
+        L.or_warp_stable.restype = i32
+        L.or_warp_stable.argtypes = [u32, u64, vp, vp, vp, vp, u32, u32, u32, i32, vp, vp, vp]
         _lib = L
     return _lib
 
@@ -148,6 +150,22 @@ def stable(timing, kernel_bb_insts, n=2048, delta=(3, 100), rate=(95, 100), brut
     if rc != OK:
         raise OracleError(rc, bad.value)
     return fs, ds, sw[:K]
+
+
+def warp_stable(timing, ok=None, n=1024, delta=(3, 100), brute=False):
+    """N1: (switch_at [K] i64, dur_sum [K] u64) of the warp-level stability test over the kernels' warp streams
+    (records = warps in retirement order; timing.bb is ignored); ok [K] u8 gates kernels without a dominant type."""
+    K, R = timing.n_kernels, timing.n_records
+    sw = np.zeros(max(K, 1), np.int64)
+    ds = np.zeros(max(K, 1), np.uint64)
+    bad = ctypes.c_int64(-1)
+    okc = None if ok is None else _c(ok, np.uint8)
+    rc = _L().or_warp_stable(K, R, _p(_c(timing.kernel_rec_off, np.uint64)), _p(_c(timing.issue, np.uint64)),
+                             _p(_c(timing.retire, np.uint64)), None if okc is None else _p(okc), int(n),
+                             int(delta[0]), int(delta[1]), 1 if brute else 0, _p(sw), _p(ds), ctypes.byref(bad))
+    if rc != OK:
+        raise OracleError(rc, bad.value)
+    return sw[:K], ds[:K]
 
 
 def analyse(trace, theta=(1, 20), n_cores=64, pool_all_prior=0):

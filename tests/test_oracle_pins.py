@@ -503,3 +503,91 @@ def test_oracle_modes_agree_on_generated_timing():
     for x, y in zip(a, b):
         assert np.array_equal(x, y)
     assert (a[0] >= 0).any()  # something stabilises
+
+
+# ---- N1: warp-level stability (L249, L262, Fig 10) ---------------------------------------------------------------
+def _warp_stream(kernels):
+    """kernels: list of (xs, ys) warp records, each kernel retire-sorted; returns a photon_timing-like Timing."""
+    off = np.zeros(len(kernels) + 1, np.uint64)
+    off[1:] = np.cumsum([len(x) for x, _ in kernels])
+    xs = np.array([v for x, _ in kernels for v in x], np.uint64)
+    ys = np.array([v for _, y in kernels for v in y], np.uint64)
+    return tg.Timing(kernel_rec_off=off, bb=np.zeros(len(xs), np.uint16), issue=xs, retire=ys, n_bb=1)
+
+
+def test_warp_stable_constructed_and_gating():
+    n = 1024  # L262 "we set n=1024"
+    xs = [100 * i for i in range(3 * n)]
+    ys = [x + 423 for x in xs]  # the L227 MM line, as warps
+    # a kernel whose warp durations drift (a = 1.2): never within 3% of 1
+    dx = [100 * i for i in range(3 * n)]
+    dy = [int(Fraction(6, 5) * x) + 500 for x in dx]
+    tm = _warp_stream([(xs, ys), (dx, dy), (xs, ys)])
+    sw, ds = oracle.warp_stable(tm, np.array([1, 1, 0], np.uint8), n=n)
+    # first evaluable retirement (the 2n-th warp) is stable; S_n = 423 n; the prediction is S_n / n = 423 ticks
+    assert sw.tolist() == [2 * n - 1, -1, -1] and int(ds[0]) == 423 * n
+    sw, _ = oracle.warp_stable(tm, None, n=n)  # no gate: the third kernel switches too
+    assert sw.tolist() == [2 * n - 1, -1, 2 * n - 1]
+    # fewer than 2n warps: never evaluable [P-11]
+    sw, _ = oracle.warp_stable(_warp_stream([(xs[:2 * n - 1], ys[:2 * n - 1])]), None, n=n)
+    assert sw[0] == -1
+
+
+@pytest.mark.parametrize("entry", _gold("paper_lines.json")["lines"] + _gold("paper_lines.json")["boundary"])
+def test_warp_stable_paper_lines(entry):
+    # L262: "the a of the least square method on the last n warps ... is close to 1 (|a-1| < delta)"; the same Eq. 1
+    # lines (L145, L227) and the strict 0.97 / 1.03 boundaries decide the warp-sampling switch
+    a = Fraction(entry["a"])
+    b = Fraction(entry.get("b", "0")) * 100
+    n = 8
+    xs, ys = _line_stream(a, b, n, 2 * n)
+    sw, ds = oracle.warp_stable(_warp_stream([(xs, ys)]), None, n=n)
+    assert (sw[0] == 2 * n - 1) == entry["stable"], entry
+
+
+@pytest.mark.parametrize("seed", range(6))
+def test_warp_stable_bruteforce_fraction(seed):
+    """Random warp streams: the switch position equals a from-scratch Fraction recomputation of cond1 (Eq. 1 over
+    the last n warps) and cond2 (mean of the last n vs the last 2n) at every retirement, in both oracle modes."""
+    rs = np.random.default_rng(100 + seed)
+    n = int(rs.choice([2, 3, 4, 8]))
+    kernels, expect, ok = [], [], []
+    for k in range(3):
+        R = int(rs.integers(0, 80))
+        t, xs, ys = 0, [], []
+        for i in range(R):
+            t += int(rs.integers(0, 5))
+            d = 20 + int(rs.integers(0, 3)) if rs.random() < 0.85 else int(rs.integers(5, 40))
+            xs.append(t)
+            ys.append(t + d)
+        order = sorted(range(R), key=lambda i: (ys[i], i))
+        xs, ys = [xs[i] for i in order], [ys[i] for i in order]
+        kernels.append((xs, ys))
+        g = int(rs.integers(0, 4) > 0)
+        ok.append(g)
+        want = -1
+        for j in range(2 * n, R + 1):
+            wx, wy = xs[j - n:j], ys[j - n:j]
+            c1 = len(set(wx)) >= 2 and abs(1 - _exact_slope(wx, wy)) < Fraction(3, 100)
+            sn = sum(y - x for x, y in zip(wx, wy))
+            s2n = sum(y - x for x, y in zip(xs[j - 2 * n:j], ys[j - 2 * n:j]))
+            c2 = s2n > 0 and abs(Fraction(sn, n) - Fraction(s2n, 2 * n)) < Fraction(3, 100) * Fraction(s2n, 2 * n)
+            if c1 and c2:
+                want = j - 1
+                break
+        expect.append(want if g else -1)
+    tm = _warp_stream(kernels)
+    for brute in (True, False):
+        sw, _ = oracle.warp_stable(tm, np.array(ok, np.uint8), n=n, brute=brute)
+        assert sw.tolist() == expect
+
+
+def test_warp_stable_generated_modes_agree_and_range_errors():
+    tm = tg.Generator(4).warp_timing(0, 30)  # ResNet-152 stem and first blocks, slot-model warp streams
+    a = oracle.warp_stable(tm, None, n=64, brute=True)
+    b = oracle.warp_stable(tm, None, n=64, brute=False)
+    assert np.array_equal(a[0], b[0]) and np.array_equal(a[1], b[1])
+    assert 0 < (a[0] >= 0).sum() < len(a[0])  # some kernels switch, some do not
+    with pytest.raises(oracle.OracleError) as ei:
+        oracle.warp_stable(_warp_stream([([1, 2], [9, 8])]), None, n=2)  # not retire-sorted
+    assert ei.value.index == 1

@@ -58,6 +58,7 @@ def _L():
         L.tg_sel_counts.argtypes = [vp, u64, u64, u64, vp, i32]
         L.tg_sel_events.argtypes = [vp, u64, u64, u64, vp, vp, i32]
         L.tg_timing.argtypes = [vp, u32, u32, vp, vp, vp, vp, i32]
+        L.tg_warp_timing.argtypes = [vp, u32, u32, vp, vp, vp, i32]
         _lib = L
     return _lib
 
@@ -216,6 +217,21 @@ class Generator:
         ret = np.empty(R, np.uint64)
         L.tg_timing(self._h, k0, k1, _ptr(off), _ptr(bb), _ptr(iss), _ptr(ret), T)
         return Timing(kernel_rec_off=off, bb=bb, issue=iss, retire=ret, n_bb=self.n_bb)
+
+
+    def warp_timing(self, k0: int = 0, k1: Optional[int] = None, threads=None) -> Timing:
+        """N1 warp streams of kernels [k0, k1): one (issue, retire) record per warp, slot model, sorted by retire
+        within each kernel (bb is all zero, n_bb = 1)."""
+        L = _L()
+        k1 = self.n_kernels if k1 is None else int(k1)
+        per_k = np.asarray(self.kernel_warps[k0:k1], np.uint64)
+        off = np.zeros(k1 - k0 + 1, np.uint64)
+        np.cumsum(per_k, out=off[1:])
+        R = int(off[-1])
+        iss = np.empty(R, np.uint64)
+        ret = np.empty(R, np.uint64)
+        L.tg_warp_timing(self._h, k0, k1, _ptr(off), _ptr(iss), _ptr(ret), _threads(threads))
+        return Timing(kernel_rec_off=off, bb=np.zeros(R, np.uint16), issue=iss, retire=ret, n_bb=1)
 
 
 def make_trace(cfg: int, seed: Optional[int] = None, scale: float = 1.0, **kw) -> Trace:

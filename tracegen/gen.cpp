@@ -584,4 +584,67 @@ void tg_timing(void* h, uint32_t k0, uint32_t k1, const uint64_t* rec_off, uint1
   for (auto& t : ts) t.join();
 }
 
+// Warp records of kernel k (N1): one record per warp, (issue, retire) of the whole warp.  Slot model: 2560 warp
+// slots (64 CUs x 40, Table 1); warp v takes the slot freed by warp v - 2560 (its issue = that warp's retire), and
+// runs its BBs back to back with the same per-BB durations as kernel_timing.  Records sorted by (retire, warp).
+static void kernel_warp_timing(const Gen* g, uint32_t k, uint64_t* issue, uint64_t* retire) {
+  const Kern& K = g->kerns[k];
+  uint64_t P = 0;
+  warp_seq(*g, k, 0, [&](uint32_t id) { P += 4ull * g->bb_len[id]; });
+  if (P == 0) P = 1;
+  uint64_t waves = (K.n_warps + 2559) / 2560;
+  double Tw = 0.25 * (double)(waves * P) + 1.0;
+  struct Rec { uint64_t retire, issue, warp; };
+  std::vector<Rec> recs(K.n_warps);
+  std::vector<uint64_t> slot(2560, 0);
+  for (uint64_t v = 0; v < K.n_warps; ++v) {
+    const uint64_t t0 = slot[v % 2560];
+    uint64_t t = t0;
+    uint32_t seq = 0;
+    warp_seq(*g, k, v, [&](uint32_t id) {
+      uint64_t len = g->bb_len[id];
+      uint64_t d;
+      int cls = g->drift_class[id];
+      if (cls == 0) {
+        double ramp = 4.0 * (double)len * std::max(0.0, 1.0 - (double)t / Tw);
+        d = 4 * len + (uint64_t)ramp + (rng(g->seed, P_JIT, k, v, seq) & 7);
+      } else {
+        d = 4 * len + (cls == 1 ? v / 8 : v / 2);
+      }
+      t += d;
+      ++seq;
+    });
+    if (t == t0) t = t0 + 1;  // an empty warp still occupies its slot for a tick
+    slot[v % 2560] = t;
+    recs[v] = Rec{t, t0, v};
+  }
+  std::sort(recs.begin(), recs.end(), [](const Rec& a, const Rec& b) {
+    if (a.retire != b.retire) return a.retire < b.retire;
+    return a.warp < b.warp;
+  });
+  for (size_t i = 0; i < recs.size(); ++i) {
+    issue[i] = recs[i].issue;
+    retire[i] = recs[i].retire;
+  }
+}
+
+// Warp records of kernels [k0, k1) into arrays at rec_off[k - k0] (= warps before kernel k0+i).
+void tg_warp_timing(void* h, uint32_t k0, uint32_t k1, const uint64_t* rec_off, uint64_t* issue, uint64_t* retire,
+                    int threads) {
+  const Gen* g = (const Gen*)h;
+  std::vector<std::thread> ts;
+  std::atomic<uint32_t> next{k0};
+  int nt = threads < 1 ? 1 : threads;
+  for (int t = 0; t < nt; ++t)
+    ts.emplace_back([&] {
+      for (;;) {
+        uint32_t k = next.fetch_add(1);
+        if (k >= k1) break;
+        uint64_t o = rec_off[k - k0];
+        kernel_warp_timing(g, k, issue + o, retire + o);
+      }
+    });
+  for (auto& t : ts) t.join();
+}
+
 }  // extern "C"
