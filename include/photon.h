@@ -217,6 +217,31 @@ PHOTON_API int photon_bb_stable(photon_ctx *ctx, const photon_timing *timing, co
                      photon_stable_params params, void *ws, size_t ws_bytes, int64_t *first_stable /*[K][B]*/,
                      uint64_t *stable_dur_sum /*[K][B] or NULL*/, int64_t *switch_at /*[K]*/, void *stream);
 
+/* ---- N1: warp-level stability + warp-sampling switch (L249, L262, Fig 10 Step 3) -------------------------------
+ * Warp stream: one record per warp of the detailed simulation (x = the warp's issue, y = its retire time), CSR by
+ * kernel (timing->kernel_rec_off), each kernel's records sorted by retire (ties keep input order) [P-18]; times are
+ * integer ticks < 2^40 [P-16]; timing->bb and timing->n_bb are ignored (every record belongs to the kernel's one
+ * warp stream: "the issue and retired time for all warps", L262) [N1-c].
+ * Kernel k is tested only when warp_sampling_ok[k] != 0 (one warp type holds more than 95% of the warps, L249; the
+ * A2 output; NULL = every kernel) [N1-d].  At its j-th warp retirement (1-based) with j >= 2n (n = window_n,
+ * default 1024, L262), over the last n warps: cond1 (Eq. 1 slope, |1-a| < delta) and cond2 (mean duration of the
+ * last n vs the last 2n: "n and n0" read as n and 2n) [N1-b], both exactly as in photon_bb_stable.  The first such
+ * retirement is the switch to warp sampling: switch_at[k] = its 0-based position in kernel k's stream and
+ * dur_sum[k] = S_n there, so the predicted time of every later warp is S_n / n ("the average time of the last n1
+ * warps", n1 read as n) [N1-e]; else -1 / 0.
+ * Workspace: photon_warp_stable_workspace_bytes(K) bytes, caller-owned.  Device errors (photon_check): ERANGE
+ * (retire < issue, retire decreasing within a kernel, time >= 2^40, bad kernel_rec_off; index = record or kernel).
+ * Host errors: EINVAL (NULL arrays, K = 0, n outside [2, 8192], bad delta), EWORKSPACE. */
+typedef struct {
+  uint32_t window_n;             /* n, default 1024 (L262); 2 <= n <= 8192                                     */
+  uint32_t delta_num, delta_den; /* delta, default 3/100 (L229, L262); 1 <= den <= 2^16, num <= den           */
+} photon_warp_stable_params;
+
+PHOTON_API size_t photon_warp_stable_workspace_bytes(uint32_t n_kernels);
+PHOTON_API int photon_warp_stable(photon_ctx *ctx, const photon_timing *warps, const uint8_t *warp_sampling_ok /*[K]|NULL*/,
+                                  photon_warp_stable_params params, void *ws, size_t ws_bytes,
+                                  int64_t *switch_at /*[K]*/, uint64_t *dur_sum /*[K] or NULL*/, void *stream);
+
 /* ---- Multi-GPU merge helpers ------------------------------------------------------------------
  * A shard is a contiguous warp range of the global trace; its local kernel l is global kernel kernel_base + l and
  * its local warp v is global warp warp_base + v.  Rows exchanged between ranks (88 bytes each):       */

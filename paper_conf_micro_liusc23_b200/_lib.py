@@ -54,6 +54,10 @@ class StableParams(ctypes.Structure):
                 ("rate_den", c_uint32)]
 
 
+class WarpStableParams(ctypes.Structure):
+    _fields_ = [("window_n", c_uint32), ("delta_num", c_uint32), ("delta_den", c_uint32)]
+
+
 TYPE_ROW_BYTES = 88  # photon_type_row
 PROF_SECTIONS = ["bbv_fused", "bbv", "kbb", "group_unfused", "canon", "sig", "scan", "resolve", "stable", "prep"]
 
@@ -86,6 +90,9 @@ _SIGS = [
     ("photon_stable_workspace_bytes", c_size_t, [POINTER(Timing)]),
     ("photon_bb_stable", c_int, [c_void_p, POINTER(Timing), c_void_p, StableParams, c_void_p, c_size_t, c_void_p,
                                  c_void_p, c_void_p, c_void_p]),
+    ("photon_warp_stable_workspace_bytes", c_size_t, [c_uint32]),
+    ("photon_warp_stable", c_int, [c_void_p, POINTER(Timing), c_void_p, WarpStableParams, c_void_p, c_size_t,
+                                   c_void_p, c_void_p, c_void_p]),
     ("photon_types_export", c_int, [c_void_p, c_uint32, POINTER(Types), c_uint32, c_uint64, c_void_p, c_void_p]),
     ("photon_merge_workspace_bytes", c_size_t, [c_uint64, c_uint32]),
     ("photon_types_merge", c_int, [c_void_p, c_void_p, c_uint64, c_uint32, c_void_p, c_void_p, c_size_t,

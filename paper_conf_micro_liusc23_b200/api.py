@@ -319,6 +319,26 @@ class Photon:
             self.check(ws, stream)
         return o
 
+    # -- N1: warp-level stability (L249, L262, Fig 10) --------------------------------------------------------
+    def photon_warp_stable(self, tm: DeviceTiming, warp_sampling_ok=None, n: int = 1024, delta=(3, 100),
+                           want_dur: bool = True, stream=None, check: bool = True, out: Optional[dict] = None) -> dict:
+        """switch_at [K] (first stable warp retirement per kernel, -1 = none) and dur_sum [K] (S_n there)."""
+        ct = tm.c()
+        ws = self.workspace("warp_stable", self.L.photon_warp_stable_workspace_bytes(tm.n_kernels))
+        o = out if out is not None else {}
+        o.setdefault("switch_at", self.empty(tm.n_kernels, "int64"))
+        if want_dur:
+            o.setdefault("dur_sum", self.empty(tm.n_kernels, "int64"))
+        prm = _lib.WarpStableParams(int(n), int(delta[0]), int(delta[1]))
+        ok = None if warp_sampling_ok is None else warp_sampling_ok.data_ptr()
+        self._rc(self.L.photon_warp_stable(self.ctx, ctypes.byref(ct), ok, prm, ws.data_ptr(), ws.numel(),
+                                           o["switch_at"].data_ptr(), o["dur_sum"].data_ptr() if want_dur else None,
+                                           self.stream_ptr(stream)))
+        o["_ws"] = ws
+        if check:
+            self.check(ws, stream)
+        return o
+
     # -- multi-GPU helpers -------------------------------------------------------------------------------------
     def photon_types_export(self, K_local, ty, kernel_base, warp_base, rows, stream=None):
         tc = self.types_c(ty)

@@ -614,6 +614,33 @@ int photon_bb_stable(photon_ctx* ctx, const photon_timing* t, const uint64_t* kb
   return PHOTON_OK;
 }
 
+// ---- N1 -----------------------------------------------------------------------------------------------------
+size_t photon_warp_stable_workspace_bytes(uint32_t K) { return 512 + warp_stable_ws_bytes(K); }
+
+int photon_warp_stable(photon_ctx* ctx, const photon_timing* t, const uint8_t* ok, photon_warp_stable_params p,
+                       void* ws, size_t ws_bytes, int64_t* switch_at, uint64_t* dur, void* stream) {
+  if (!ctx) return PHOTON_EINVAL;
+  if (!t || !t->kernel_rec_off || (t->n_records && (!t->issue || !t->retire)) || !switch_at || !ws)
+    return fail(ctx, PHOTON_EINVAL, "NULL argument");
+  if (t->n_kernels == 0 || t->n_records >= (1ull << 32)) return fail(ctx, PHOTON_EINVAL, "bad warp stream sizes");
+  if (p.window_n == 0) p.window_n = 1024;
+  if (p.delta_den == 0) { p.delta_num = 3; p.delta_den = 100; }
+  if (p.window_n < 2 || p.window_n > 8192 || p.delta_den > (1u << 16) || p.delta_num > p.delta_den)
+    return fail(ctx, PHOTON_EINVAL, "bad warp stable params");
+  const size_t need = photon_warp_stable_workspace_bytes(t->n_kernels);
+  if (ws_bytes < need) return fail(ctx, PHOTON_EWORKSPACE, "workspace %zu < %zu bytes", ws_bytes, need);
+  cudaStream_t s = (cudaStream_t)stream;
+  CK(cudaSetDevice(ctx->device), "cudaSetDevice");
+  ctx->last_ws = ws;
+  DevErr* err = (DevErr*)ws;
+  CK(cudaMemsetAsync(err, 0, sizeof(DevErr), s), "memset");
+  ProfScope ps(ctx, PHOTON_PROF_STABLE, s);
+  CK(launch_warp_stable(*t, ok, p.window_n, p.delta_num, p.delta_den, (uint8_t*)ws + 512, switch_at, dur, err,
+                        ctx->num_sms, s),
+     "warp_stable");
+  return PHOTON_OK;
+}
+
 // ---- multi-GPU helpers ------------------------------------------------------------------------------------
 int photon_types_export(photon_ctx* ctx, uint32_t K_local, const photon_types* local, uint32_t kernel_base,
                         uint64_t warp_base, photon_type_row* rows, void* stream) {

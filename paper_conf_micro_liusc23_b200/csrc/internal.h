@@ -136,6 +136,11 @@ cudaError_t launch_match_resolve(uint32_t K, const uint64_t* kto, const uint64_t
 
 // ---- A5 (k_stable.cu) -------------------------------------------------------------------------------------
 size_t stable_ws_bytes(const photon_timing& t);
+// N1: warp-level stability over per-kernel warp streams (groups = kernels)
+size_t warp_stable_ws_bytes(uint32_t K);
+cudaError_t launch_warp_stable(const photon_timing& t, const uint8_t* ok, uint32_t n, uint32_t dnum, uint32_t dden,
+                               void* ws, int64_t* switch_at, uint64_t* dur, DevErr* err, int num_sms,
+                               cudaStream_t s);
 cudaError_t launch_stable(const photon_timing& t, const uint64_t* kbb, photon_stable_params p, void* ws,
                           size_t ws_bytes, int64_t* first_stable, uint64_t* dur, int64_t* switch_at, DevErr* err,
                           int num_sms, cudaStream_t s);

@@ -673,6 +673,58 @@ __global__ void __launch_bounds__(256) k_switch(const int64_t* first_stable, con
   }
 }
 
+// ---- N1: warp-level stability (L249, L262, Fig 10) ------------------------------------------------------------
+// The warp streams need no partition: a kernel's warp records are already one group in retirement order, so the
+// groups are the kernels (gstart = kernel_rec_off) and k_window runs on issue / retire directly.
+// One warp per kernel: retire >= issue, times < 2^40, retire non-decreasing within the kernel [P-16][P-18].
+__global__ void k_warp_validate(const uint64_t* kro, uint32_t K, uint64_t R, const uint64_t* issue,
+                                const uint64_t* retire, DevErr* err) {
+  const uint32_t lane = threadIdx.x & 31, nw = (gridDim.x * blockDim.x) >> 5;
+  for (uint32_t k = (blockIdx.x * blockDim.x + threadIdx.x) >> 5; k < K; k += nw) {
+    const uint64_t a = kro[k], b = kro[k + 1];
+    if (lane == 0 && ((k == 0 && a != 0) || b < a || b > R || (k + 1 == K && b != R))) {
+      latch(err, PHOTON_ERANGE, (int64_t)k);
+      continue;
+    }
+    if (b < a || b > R) continue;
+    for (uint64_t i = a + lane; i < b; i += 32) {
+      const uint64_t x = issue[i], y = retire[i];
+      if (y < x || y >= kTimeLimit || x >= kTimeLimit || (i > a && retire[i - 1] > y)) latch(err, PHOTON_ERANGE, (int64_t)i);
+    }
+  }
+}
+
+// runs per kernel; kernels without a dominant warp type (ok[k] == 0) get none (warp sampling stays off, L249)
+__global__ void k_warp_runs(const uint64_t* kro, uint32_t K, uint64_t R, const uint8_t* ok, uint32_t n2,
+                            uint32_t* nruns, uint64_t* gfirst, uint32_t* misc) {
+  for (uint32_t k = blockIdx.x * blockDim.x + threadIdx.x; k < K; k += gridDim.x * blockDim.x) {
+    const uint64_t a = kro[k], b = kro[k + 1];
+    const uint64_t sz = (b >= a && b <= R) ? b - a : 0;
+    const uint32_t r = (sz >= n2 && (!ok || ok[k])) ? (uint32_t)ceil_div(sz - n2 + 1, RUN) : 0u;
+    nruns[k] = r;
+    gfirst[k] = ~0ull;
+    if (r) atomicMax(misc + 1, r);
+    if (k == 0) misc[0] = K;
+  }
+}
+
+// switch position (0-based within the kernel's stream) and S_n = sum of the last n durations there
+__global__ void k_warp_finish(const uint64_t* kro, uint32_t K, const uint64_t* issue, const uint64_t* retire,
+                              const uint64_t* gfirst, uint32_t n, int64_t* switch_at, uint64_t* dur) {
+  const uint32_t lane = threadIdx.x & 31, nw = (gridDim.x * blockDim.x) >> 5;
+  for (uint32_t k = (blockIdx.x * blockDim.x + threadIdx.x) >> 5; k < K; k += nw) {
+    const uint64_t q = gfirst[k];
+    if (q == ~0ull) continue;
+    uint64_t sum = 0;
+    for (uint64_t i = q + 1 - n + lane; i <= q; i += 32) sum += retire[i] - issue[i];
+    for (int o = 16; o > 0; o >>= 1) sum += __shfl_xor_sync(0xffffffffu, sum, o);
+    if (lane == 0) {
+      switch_at[k] = (int64_t)(q - kro[k]);
+      if (dur) dur[k] = sum;
+    }
+  }
+}
+
 struct Layout {
   bool onepass;      // B <= 256: job multisplit; else LSD radix sort of composite keys
   uint64_t* key0; uint64_t* key1;  // radix path only
@@ -779,6 +831,38 @@ cudaError_t launch_stable(const photon_timing& t, const uint64_t* kbb, photon_st
   } else {
     cudaMemsetAsync(switch_at, 0xFF, sizeof(int64_t) * K, s);
   }
+  return cudaGetLastError();
+}
+
+size_t warp_stable_ws_bytes(uint32_t K) {
+  Carver c(nullptr);
+  c.take<uint32_t>(16);
+  c.take<uint32_t>((uint64_t)K + 1);
+  c.take<uint64_t>((uint64_t)K + 1);
+  return c.off + 256;
+}
+
+cudaError_t launch_warp_stable(const photon_timing& t, const uint8_t* ok, uint32_t n, uint32_t dnum, uint32_t dden,
+                               void* ws, int64_t* switch_at, uint64_t* dur, DevErr* err, int num_sms,
+                               cudaStream_t s) {
+  Carver c(ws);
+  uint32_t* misc = c.take<uint32_t>(16);
+  uint32_t* nruns = c.take<uint32_t>((uint64_t)t.n_kernels + 1);
+  uint64_t* gfirst = c.take<uint64_t>((uint64_t)t.n_kernels + 1);
+  const uint32_t K = t.n_kernels;
+  cudaMemsetAsync(switch_at, 0xFF, sizeof(int64_t) * K, s);
+  if (dur) cudaMemsetAsync(dur, 0, sizeof(uint64_t) * K, s);
+  cudaMemsetAsync(misc, 0, 64, s);
+  const unsigned gk = (unsigned)umin64(ceil_div((uint64_t)K * 32, 256), (uint64_t)num_sms * 8);
+  note_launch(), k_warp_validate<<<gk, 256, 0, s>>>(t.kernel_rec_off, K, t.n_records, t.issue, t.retire, err);
+  if (t.n_records == 0) return cudaGetLastError();
+  note_launch(), k_warp_runs<<<(unsigned)ceil_div(K, 256), 256, 0, s>>>(t.kernel_rec_off, K, t.n_records, ok, 2 * n,
+                                                                       nruns, gfirst, misc);
+  WinArgs wa{};
+  wa.X = t.issue; wa.Y = t.retire; wa.gstart = t.kernel_rec_off; wa.G = misc + 0; wa.nruns = nruns;
+  wa.maxr = misc + 1; wa.ticket = misc + 2; wa.n = n; wa.dnum = dnum; wa.dden = dden; wa.gfirst = gfirst;
+  note_launch(), k_window<<<(unsigned)num_sms * 2, WT, 0, s>>>(wa);
+  note_launch(), k_warp_finish<<<gk, 256, 0, s>>>(t.kernel_rec_off, K, t.issue, t.retire, gfirst, n, switch_at, dur);
   return cudaGetLastError();
 }
 

@@ -315,3 +315,64 @@ def test_match_many_kernels_synthetic(ph, K):
     fin = np.isfinite(od)
     assert np.array_equal(np.isfinite(gd), fin)
     np.testing.assert_allclose(gd[fin], od[fin], rtol=1e-6, atol=0)
+
+
+# ---- N1: warp-level stability (L249, L262, Fig 10) ---------------------------------------------------------------
+def check_warp_stable(ph, tm, ok, n, delta=(3, 100)):
+    from paper_conf_micro_liusc23_b200 import DeviceTiming, to_device
+    dt = DeviceTiming.from_host(tm, ph.device)
+    okd = None if ok is None else to_device(np.ascontiguousarray(ok, np.uint8), ph.device)
+    o = ph.photon_warp_stable(dt, okd, n, delta)
+    sw, ds = oracle.warp_stable(tm, ok, n, delta)
+    assert np.array_equal(_np(o["switch_at"], np.int64), sw)
+    assert np.array_equal(_np(o["dur_sum"], np.uint64), ds)
+    return sw
+
+
+@pytest.mark.parametrize("cfg", [3, 4, 2])
+def test_warp_stable_configs_gated_by_dominance(ph, cfg):
+    # the slot-model warp streams of every kernel, gated by A2's warp_sampling_ok of the same trace (the fused GPU
+    # path computes it; the oracle's dominance decision must agree first)
+    g = tg.Generator(cfg)
+    tr = g.trace()
+    ty = ph.photon_warp_group(_dev(ph, tr))
+    p16, _, _ = oracle.bbv(tr, want_kbb=False)
+    ok = oracle.group(tr, p16)["warp_sampling_ok"]
+    assert np.array_equal(_np(ty["warp_sampling_ok"], np.uint8), ok)
+    tm = g.warp_timing()
+    sw = check_warp_stable(ph, tm, ok, 1024)
+    sw_all = check_warp_stable(ph, tm, None, 1024)
+    assert (sw_all >= 0).any()
+    assert np.all(sw[ok == 0] == -1)
+
+
+@pytest.mark.parametrize("n", [2, 64, 1024])
+def test_warp_stable_c4_prefix_windows(ph, n):
+    check_warp_stable(ph, tg.Generator(4).warp_timing(0, 60), None, n)
+    check_warp_stable(ph, tg.Generator(4).warp_timing(0, 60), None, n, delta=(1, 100))
+
+
+def test_warp_stable_paper_lines_and_errors(ph):
+    from fractions import Fraction
+    from paper_conf_micro_liusc23_b200 import PhotonError
+    n = 64
+    recs = []
+    for a in ["1.00", "0.99", "32.87", "0.97", "0.9701", "1.03", "1.0299"]:
+        xs = [10_000 * (i + 1) for i in range(3 * n)]
+        ys = [int(Fraction(a) * x + 10 ** 9) for x in xs]
+        recs.append((xs, ys))
+    recs.append(([5] * 10, [6] * 10))  # too short to evaluate
+    off = np.cumsum([0] + [len(x) for x, _ in recs]).astype(np.uint64)
+    tm = tg.Timing(kernel_rec_off=off, bb=np.zeros(int(off[-1]), np.uint16),
+                   issue=np.concatenate([np.array(x, np.uint64) for x, _ in recs]),
+                   retire=np.concatenate([np.array(y, np.uint64) for _, y in recs]), n_bb=1)
+    sw = check_warp_stable(ph, tm, None, n)
+    assert sw.tolist() == [2 * n - 1, 2 * n - 1, -1, -1, 2 * n - 1, -1, 2 * n - 1, -1]
+    ok = np.array([1, 0, 1, 1, 1, 1, 0, 1], np.uint8)
+    sw = check_warp_stable(ph, tm, ok, n)
+    assert sw.tolist() == [2 * n - 1, -1, -1, -1, 2 * n - 1, -1, -1, -1]
+    bad = tg.Timing(kernel_rec_off=np.array([0, 3], np.uint64), bb=np.zeros(3, np.uint16),
+                    issue=np.array([1, 2, 3], np.uint64), retire=np.array([5, 4, 9], np.uint64), n_bb=1)
+    with pytest.raises(PhotonError) as ei:
+        check_warp_stable(ph, bad, None, 2)
+    assert ei.value.code == -3 and ei.value.index == 1
