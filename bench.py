@@ -340,6 +340,38 @@ def run_photon(args):
                                    "algorithmic_bytes": abytes, "traffic": None},
                       "stable_bb_types": int((to_numpy_i64(o["first_stable"]) >= 0).sum())}
 
+    # ---- N1 (warp-level stability, L262) on the same config's warp streams, gated by A2's dominance ----
+    if not args.skip_a5 and ws == 1:
+        gw = tg.Generator(args.a5_config)
+        tw = gw.warp_timing()
+        ty = ph.photon_warp_group(DeviceTrace.from_host(gw.trace(), dev))
+        okd = ty["warp_sampling_ok"]
+        dw = DeviceTiming.from_host(tw, dev)
+        o = ph.photon_warp_stable(dw, okd, 1024)
+        for _ in range(max(args.warmup - 1, 0)):
+            o = ph.photon_warp_stable(dw, okd, 1024, check=False, out=o)
+        torch.cuda.synchronize()
+        c0, c1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        c0.record(s)
+        n6 = max(args.steps // 4, 3)
+        for _ in range(n6):
+            o = ph.photon_warp_stable(dw, okd, 1024, check=False, out=o)
+        c1.record(s)
+        torch.cuda.synchronize()
+        ph.check(o["_ws"])
+        wms = c0.elapsed_time(c1) / n6
+        RW = tw.n_records
+        wbytes = 16 * RW
+        line["n1"] = {"metric": "warp records tested/sec (warp-level stability + warp-sampling switch)",
+                      "value": RW / (wms / 1000), "unit": "records/s", "ms_per_step": wms, "records": RW,
+                      "workload": f"{CONFIG_DESC.get(args.a5_config)} warp streams (2560-slot model), n=1024, "
+                                  "delta=3/100, gated by warp_sampling_ok",
+                      "roofline": {"bound": "hbm", "achieved": wbytes / (wms / 1000) / 1e9, "peak": hbm_peak,
+                                   "unit": "GB/s", "frac": wbytes / (wms / 1000) / 1e9 / hbm_peak,
+                                   "algorithmic_bytes": wbytes, "traffic": None},
+                      "switched_kernels": int((to_numpy_i64(o["switch_at"]) >= 0).sum()),
+                      "dominant_kernels": int(okd.to(torch.int64).sum().item())}
+
     if rank == 0 and ws == 1 and not args.skip_cpu:
         line["cpu_baseline"] = cpu_baseline(args)
     if rank == 0:

@@ -229,7 +229,7 @@ PHOTON_API int photon_bb_stable(photon_ctx *ctx, const photon_timing *timing, co
  * retirement is the switch to warp sampling: switch_at[k] = its 0-based position in kernel k's stream and
  * dur_sum[k] = S_n there, so the predicted time of every later warp is S_n / n ("the average time of the last n1
  * warps", n1 read as n) [N1-e]; else -1 / 0.
- * Workspace: photon_warp_stable_workspace_bytes(K) bytes, caller-owned.  Device errors (photon_check): ERANGE
+ * Workspace: photon_warp_stable_workspace_bytes(warps) bytes, caller-owned.  Device errors (photon_check): ERANGE
  * (retire < issue, retire decreasing within a kernel, time >= 2^40, bad kernel_rec_off; index = record or kernel).
  * Host errors: EINVAL (NULL arrays, K = 0, n outside [2, 8192], bad delta), EWORKSPACE. */
 typedef struct {
@@ -237,7 +237,7 @@ typedef struct {
   uint32_t delta_num, delta_den; /* delta, default 3/100 (L229, L262); 1 <= den <= 2^16, num <= den           */
 } photon_warp_stable_params;
 
-PHOTON_API size_t photon_warp_stable_workspace_bytes(uint32_t n_kernels);
+PHOTON_API size_t photon_warp_stable_workspace_bytes(const photon_timing *warps);
 PHOTON_API int photon_warp_stable(photon_ctx *ctx, const photon_timing *warps, const uint8_t *warp_sampling_ok /*[K]|NULL*/,
                                   photon_warp_stable_params params, void *ws, size_t ws_bytes,
                                   int64_t *switch_at /*[K]*/, uint64_t *dur_sum /*[K] or NULL*/, void *stream);

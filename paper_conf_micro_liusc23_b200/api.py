@@ -324,7 +324,7 @@ class Photon:
                            want_dur: bool = True, stream=None, check: bool = True, out: Optional[dict] = None) -> dict:
         """switch_at [K] (first stable warp retirement per kernel, -1 = none) and dur_sum [K] (S_n there)."""
         ct = tm.c()
-        ws = self.workspace("warp_stable", self.L.photon_warp_stable_workspace_bytes(tm.n_kernels))
+        ws = self.workspace("warp_stable", self.L.photon_warp_stable_workspace_bytes(ctypes.byref(ct)))
         o = out if out is not None else {}
         o.setdefault("switch_at", self.empty(tm.n_kernels, "int64"))
         if want_dur:

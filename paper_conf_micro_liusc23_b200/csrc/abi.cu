@@ -615,7 +615,9 @@ int photon_bb_stable(photon_ctx* ctx, const photon_timing* t, const uint64_t* kb
 }
 
 // ---- N1 -----------------------------------------------------------------------------------------------------
-size_t photon_warp_stable_workspace_bytes(uint32_t K) { return 512 + warp_stable_ws_bytes(K); }
+size_t photon_warp_stable_workspace_bytes(const photon_timing* t) {
+  return t ? 512 + warp_stable_ws_bytes(t->n_kernels, t->n_records) : 0;
+}
 
 int photon_warp_stable(photon_ctx* ctx, const photon_timing* t, const uint8_t* ok, photon_warp_stable_params p,
                        void* ws, size_t ws_bytes, int64_t* switch_at, uint64_t* dur, void* stream) {
@@ -627,7 +629,7 @@ int photon_warp_stable(photon_ctx* ctx, const photon_timing* t, const uint8_t* o
   if (p.delta_den == 0) { p.delta_num = 3; p.delta_den = 100; }
   if (p.window_n < 2 || p.window_n > 8192 || p.delta_den > (1u << 16) || p.delta_num > p.delta_den)
     return fail(ctx, PHOTON_EINVAL, "bad warp stable params");
-  const size_t need = photon_warp_stable_workspace_bytes(t->n_kernels);
+  const size_t need = photon_warp_stable_workspace_bytes(t);
   if (ws_bytes < need) return fail(ctx, PHOTON_EWORKSPACE, "workspace %zu < %zu bytes", ws_bytes, need);
   cudaStream_t s = (cudaStream_t)stream;
   CK(cudaSetDevice(ctx->device), "cudaSetDevice");

@@ -137,7 +137,7 @@ cudaError_t launch_match_resolve(uint32_t K, const uint64_t* kto, const uint64_t
 // ---- A5 (k_stable.cu) -------------------------------------------------------------------------------------
 size_t stable_ws_bytes(const photon_timing& t);
 // N1: warp-level stability over per-kernel warp streams (groups = kernels)
-size_t warp_stable_ws_bytes(uint32_t K);
+size_t warp_stable_ws_bytes(uint32_t K, uint64_t R);
 cudaError_t launch_warp_stable(const photon_timing& t, const uint8_t* ok, uint32_t n, uint32_t dnum, uint32_t dden,
                                void* ws, int64_t* switch_at, uint64_t* dur, DevErr* err, int num_sms,
                                cudaStream_t s);

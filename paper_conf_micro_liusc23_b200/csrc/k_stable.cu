@@ -394,6 +394,45 @@ __global__ void k_work_count(const uint64_t* gstart, const uint32_t* G, uint32_t
   }
 }
 
+// The compact run list, run-major (every group's run 0 before any group's run 1): count the groups per run index,
+// scan, fill (the order of groups inside one run index is immaterial).  list[i] = g | (uint64)r << 32.
+__global__ void k_runs_count(const uint32_t* G, const uint32_t* nruns, uint32_t* cnt) {
+  const uint32_t ng = *G;
+  for (uint32_t g = blockIdx.x * blockDim.x + threadIdx.x; g < ng; g += gridDim.x * blockDim.x)
+    for (uint32_t r = 0; r < nruns[g]; ++r) atomicAdd(&cnt[r], 1u);
+}
+__global__ void __launch_bounds__(1024) k_runs_scan(const uint32_t* maxr, uint32_t* cnt, uint32_t* total) {
+  __shared__ uint32_t ws[32];
+  __shared__ uint32_t carry;
+  if (threadIdx.x == 0) carry = 0;
+  __syncthreads();
+  const uint32_t m = *maxr, lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+  for (uint32_t base = 0; base < m; base += 1024) {
+    const uint32_t i = base + threadIdx.x;
+    const uint32_t v = i < m ? cnt[i] : 0u;
+    uint32_t x = v;
+    for (int o = 1; o < 32; o <<= 1) {
+      const uint32_t y = __shfl_up_sync(0xffffffffu, x, o);
+      if (lane >= (uint32_t)o) x += y;
+    }
+    if (lane == 31) ws[wid] = x;
+    __syncthreads();
+    uint32_t pre = carry;
+    for (uint32_t k = 0; k < wid; ++k) pre += ws[k];
+    if (i < m) cnt[i] = pre + x - v;  // exclusive
+    __syncthreads();
+    if (threadIdx.x == 1023) carry = pre + x;
+    __syncthreads();
+  }
+  if (threadIdx.x == 0) *total = carry;
+}
+__global__ void k_runs_fill(const uint32_t* G, const uint32_t* nruns, const uint32_t* off, uint32_t* fill,
+                            uint64_t* list) {
+  const uint32_t ng = *G;
+  for (uint32_t g = blockIdx.x * blockDim.x + threadIdx.x; g < ng; g += gridDim.x * blockDim.x)
+    for (uint32_t r = 0; r < nruns[g]; ++r) list[off[r] + atomicAdd(&fill[r], 1u)] = (uint64_t)g | ((uint64_t)r << 32);
+}
+
 // ---- 4. windowed exact test ----------------------------------------------------------------------------------
 struct Sums {
   int64_t sx, sy, sn, s2n;
@@ -444,8 +483,8 @@ struct WinArgs {
   const uint64_t* Y;
   const uint64_t* gstart;
   const uint32_t* G;
-  const uint32_t* nruns;  // [G] runs per group
-  const uint32_t* maxr;   // max over groups
+  const uint64_t* list;   // compact run-major run list (k_runs_*)
+  const uint32_t* total;  // its length
   uint32_t* ticket;       // global ticket counter (zeroed)
   uint32_t n;
   uint32_t dnum, dden;
@@ -465,39 +504,30 @@ __global__ void __launch_bounds__(WT, 2) k_window(WinArgs a) {
   __shared__ Sums part[WT / 32];
   __shared__ Sums wtot[WT / 32];
   __shared__ uint64_t best, s_gf;
-  __shared__ uint32_t s_mask, s_base;
-  __shared__ int s_stop;
   const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
-  const uint32_t G = *a.G, maxr = *a.maxr;
+  __shared__ uint64_t s_item;
+  const uint32_t total = *a.total;
   const int64_t n = a.n;
-  if (G == 0 || maxr == 0) return;
-  const uint64_t n_tickets = (uint64_t)G * maxr;
   for (;;) {
-    // warp 0 claims 32 tickets and filters out the empty / already-decided ones
-    if (wid == 0) {
-      uint32_t base = 0;
-      if (lane == 0) base = atomicAdd(a.ticket, 32u);
-      base = __shfl_sync(0xffffffffu, base, 0);
-      uint64_t t = (uint64_t)base + lane;
-      bool ok = false;
-      if (t < n_tickets) {
-        uint32_t r = (uint32_t)(t / G), g = (uint32_t)(t % G);
-        if (r < a.nruns[g]) {
-          uint64_t P0 = a.gstart[g] + 2 * n - 1 + (uint64_t)r * RUN;
-          ok = *(volatile const uint64_t*)&a.gfirst[g] > P0;
-        }
+    // one run per claim: the next entry of the run-major list that no earlier latch has made pointless
+    if (tid == 0) {
+      uint64_t it = ~0ull;
+      for (;;) {
+        const uint32_t t = atomicAdd(a.ticket, 1u);
+        if (t >= total) break;
+        const uint64_t e = a.list[t];
+        const uint32_t g = (uint32_t)e, r = (uint32_t)(e >> 32);
+        const uint64_t P0 = a.gstart[g] + 2 * (uint64_t)n - 1 + (uint64_t)r * RUN;
+        if (*(volatile const uint64_t*)&a.gfirst[g] > P0) { it = e; break; }
       }
-      uint32_t m = __ballot_sync(0xffffffffu, ok);
-      if (lane == 0) { s_mask = m; s_base = base; s_stop = (uint64_t)base >= n_tickets; }
+      s_item = it;
     }
     __syncthreads();
-    const uint32_t mask = s_mask, tbase = s_base;
-    const int stop = s_stop;
+    const uint64_t item = s_item;
     __syncthreads();
-    if (stop) break;
-    for (uint32_t mm = mask; mm; mm &= mm - 1) {
-      const uint64_t t = (uint64_t)tbase + (__ffs(mm) - 1);
-      const uint32_t r = (uint32_t)(t / G), g = (uint32_t)(t % G);
+    if (item == ~0ull) break;
+    {
+      const uint32_t g = (uint32_t)item, r = (uint32_t)(item >> 32);
       const int64_t gs = (int64_t)a.gstart[g], ge = (int64_t)a.gstart[g + 1];
       const int64_t P0 = gs + 2 * n - 1 + (int64_t)r * RUN;
       const int64_t P1 = P0 + RUN < ge ? P0 + RUN : ge;
@@ -568,22 +598,25 @@ __global__ void __launch_bounds__(WT, 2) k_window(WinArgs a) {
           w.s2n += (ys - xs) - do2;
           w.sxy += (i128)xs * ys - (i128)xo * yo;
           w.sxx += (i128)xs * xs - (i128)xo * xo;
-          // cond1: den > 0 and dden*|den - num| < dnum*den  (Eq. 1: a = num/den)
-          i128 num = (i128)n * w.sxy - (i128)w.sx * w.sy;
-          i128 den = (i128)n * w.sxx - (i128)w.sx * w.sx;
-          bool c1 = false;
-          if (den > 0) {
-            i128 diff = den - num;
-            if (diff < 0) diff = -diff;
-            c1 = (i128)a.dden * diff < (i128)a.dnum * den;
-          }
+          // cond2 first (64-bit: |2 S_n - S_2n| < 2^41, times delta_den <= 2^16), then cond1 only where it holds
           bool c2 = false;
-          if (c1 && w.s2n > 0) {
-            i128 d2 = 2 * (i128)w.sn - w.s2n;
+          if (w.s2n > 0) {
+            int64_t d2 = 2 * w.sn - w.s2n;
             if (d2 < 0) d2 = -d2;
             c2 = (i128)a.dden * d2 < (i128)a.dnum * w.s2n;
           }
-          if (c1 && c2) { mine = (uint64_t)q; break; }
+          if (c2) {
+            // cond1: den > 0 and dden*|den - num| < dnum*den  (Eq. 1: a = num/den)
+            i128 num = (i128)n * w.sxy - (i128)w.sx * w.sy;
+            i128 den = (i128)n * w.sxx - (i128)w.sx * w.sx;
+            bool c1 = false;
+            if (den > 0) {
+              i128 diff = den - num;
+              if (diff < 0) diff = -diff;
+              c1 = (i128)a.dden * diff < (i128)a.dnum * den;
+            }
+            if (c1) { mine = (uint64_t)q; break; }
+          }
         }
         if (mine != ~0ull) atomicMin((unsigned long long*)&best, (unsigned long long)mine);
         if (tid == 0) s_gf = *(volatile const uint64_t*)&a.gfirst[g];
@@ -676,21 +709,28 @@ __global__ void __launch_bounds__(256) k_switch(const int64_t* first_stable, con
 // ---- N1: warp-level stability (L249, L262, Fig 10) ------------------------------------------------------------
 // The warp streams need no partition: a kernel's warp records are already one group in retirement order, so the
 // groups are the kernels (gstart = kernel_rec_off) and k_window runs on issue / retire directly.
-// One warp per kernel: retire >= issue, times < 2^40, retire non-decreasing within the kernel [P-16][P-18].
+// Grid-stride over records: retire >= issue, times < 2^40, retire non-decreasing within a kernel [P-16][P-18] (a
+// decrease is an error unless the record starts a kernel: binary search of kernel_rec_off, rare path); one thread
+// per kernel checks the offsets.
 __global__ void k_warp_validate(const uint64_t* kro, uint32_t K, uint64_t R, const uint64_t* issue,
                                 const uint64_t* retire, DevErr* err) {
-  const uint32_t lane = threadIdx.x & 31, nw = (gridDim.x * blockDim.x) >> 5;
-  for (uint32_t k = (blockIdx.x * blockDim.x + threadIdx.x) >> 5; k < K; k += nw) {
+  const uint64_t tid = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x, nt = (uint64_t)gridDim.x * blockDim.x;
+  for (uint64_t k = tid; k < K; k += nt) {
     const uint64_t a = kro[k], b = kro[k + 1];
-    if (lane == 0 && ((k == 0 && a != 0) || b < a || b > R || (k + 1 == K && b != R))) {
-      latch(err, PHOTON_ERANGE, (int64_t)k);
-      continue;
+    if ((k == 0 && a != 0) || b < a || b > R || (k + 1 == K && b != R)) latch(err, PHOTON_ERANGE, (int64_t)k);
+  }
+  for (uint64_t i = tid; i < R; i += nt) {
+    const uint64_t x = issue[i], y = retire[i];
+    bool bad = y < x || y >= kTimeLimit || x >= kTimeLimit;
+    if (!bad && i > 0 && retire[i - 1] > y) {
+      uint32_t lo = 0, hi = K;  // is i a kernel start? (largest k with kro[k] <= i)
+      while (lo < hi) {
+        const uint32_t mid = (lo + hi + 1) >> 1;
+        if (kro[mid] <= i) lo = mid; else hi = mid - 1;
+      }
+      bad = kro[lo] != i;
     }
-    if (b < a || b > R) continue;
-    for (uint64_t i = a + lane; i < b; i += 32) {
-      const uint64_t x = issue[i], y = retire[i];
-      if (y < x || y >= kTimeLimit || x >= kTimeLimit || (i > a && retire[i - 1] > y)) latch(err, PHOTON_ERANGE, (int64_t)i);
-    }
+    if (bad) latch(err, PHOTON_ERANGE, (int64_t)i);
   }
 }
 
@@ -725,6 +765,34 @@ __global__ void k_warp_finish(const uint64_t* kro, uint32_t K, const uint64_t* i
   }
 }
 
+// run list workspace: runs per group <= R / RUN + 1; total runs <= R / RUN + R / (2n) + 1 (groups with >= 2n records)
+struct RunList {
+  uint32_t* cnt;   // [cap_r] groups per run index, then their exclusive prefix
+  uint32_t* fill;  // [cap_r]
+  uint64_t* list;  // [cap_l]
+  uint64_t cap_r, cap_l;
+};
+inline void carve_runlist(Carver& c, uint64_t R, RunList& rl) {
+  rl.cap_r = R / RUN + 2;
+  rl.cap_l = R / RUN + R / 4 + 2;  // n >= 2
+  rl.cnt = c.take<uint32_t>(rl.cap_r);
+  rl.fill = c.take<uint32_t>(rl.cap_r);
+  rl.list = c.take<uint64_t>(rl.cap_l);
+}
+// k_work_count / k_warp_runs have written nruns and misc[1] = max runs: build the list, set the window args
+inline void build_runlist(const RunList& rl, const uint32_t* G, const uint32_t* nruns, uint32_t* misc, uint64_t gcap,
+                          int num_sms, WinArgs& wa, cudaStream_t s) {
+  cudaMemsetAsync(rl.cnt, 0, sizeof(uint32_t) * rl.cap_r, s);
+  cudaMemsetAsync(rl.fill, 0, sizeof(uint32_t) * rl.cap_r, s);
+  const unsigned gg = (unsigned)umin64(ceil_div(gcap, 256), (uint64_t)num_sms * 4);
+  note_launch(), k_runs_count<<<gg ? gg : 1, 256, 0, s>>>(G, nruns, rl.cnt);
+  note_launch(), k_runs_scan<<<1, 1024, 0, s>>>(misc + 1, rl.cnt, misc + 3);
+  note_launch(), k_runs_fill<<<gg ? gg : 1, 256, 0, s>>>(G, nruns, rl.cnt, rl.fill, rl.list);
+  wa.list = rl.list;
+  wa.total = misc + 3;
+  wa.ticket = misc + 2;
+}
+
 struct Layout {
   bool onepass;      // B <= 256: job multisplit; else LSD radix sort of composite keys
   uint64_t* key0; uint64_t* key1;  // radix path only
@@ -735,6 +803,7 @@ struct Layout {
   uint32_t* nruns;   // [gcap]
   uint64_t* gfirst;  // [gcap]
   uint64_t* coff;    // [K+1] chunk (job) offsets per kernel
+  RunList rl;
   uint64_t gcap, n_tiles, n_jobs, hn;
   size_t bytes;
 };
@@ -760,6 +829,7 @@ Layout make_layout(const photon_timing& t, void* base) {
   L.nruns = c.take<uint32_t>(L.gcap);
   L.gfirst = c.take<uint64_t>(L.gcap);
   L.coff = c.take<uint64_t>((uint64_t)t.n_kernels + 1);
+  carve_runlist(c, R, L.rl);
   L.bytes = c.off + 256;
   return L;
 }
@@ -820,8 +890,9 @@ cudaError_t launch_stable(const photon_timing& t, const uint64_t* kbb, photon_st
     note_launch(), k_work_count<<<(unsigned)umin64(ceil_div(L.gcap, 256), (uint64_t)num_sms * 4), 256, 0, s>>>(
         L.gstart, L.misc + 0, 2 * p.window_n, L.nruns, L.gfirst, L.misc + 1);
     WinArgs wa{};
-    wa.X = L.X; wa.Y = L.Y; wa.gstart = L.gstart; wa.G = L.misc + 0; wa.nruns = L.nruns; wa.maxr = L.misc + 1;
-    wa.ticket = L.misc + 2; wa.n = p.window_n; wa.dnum = p.delta_num; wa.dden = p.delta_den; wa.gfirst = L.gfirst;
+    wa.X = L.X; wa.Y = L.Y; wa.gstart = L.gstart; wa.G = L.misc + 0;
+    wa.n = p.window_n; wa.dnum = p.delta_num; wa.dden = p.delta_den; wa.gfirst = L.gfirst;
+    build_runlist(L.rl, L.misc + 0, L.nruns, L.misc, L.gcap, num_sms, wa, s);
     note_launch(), k_window<<<(unsigned)num_sms * 2, WT, 0, s>>>(wa);
     // 5. outputs
     note_launch(), k_finish<<<(unsigned)umin64(ceil_div(L.gcap * 32, 256), (uint64_t)num_sms * 8), 256, 0, s>>>(
@@ -834,11 +905,13 @@ cudaError_t launch_stable(const photon_timing& t, const uint64_t* kbb, photon_st
   return cudaGetLastError();
 }
 
-size_t warp_stable_ws_bytes(uint32_t K) {
+size_t warp_stable_ws_bytes(uint32_t K, uint64_t R) {
   Carver c(nullptr);
   c.take<uint32_t>(16);
   c.take<uint32_t>((uint64_t)K + 1);
   c.take<uint64_t>((uint64_t)K + 1);
+  RunList rl;
+  carve_runlist(c, R, rl);
   return c.off + 256;
 }
 
@@ -849,18 +922,23 @@ cudaError_t launch_warp_stable(const photon_timing& t, const uint8_t* ok, uint32
   uint32_t* misc = c.take<uint32_t>(16);
   uint32_t* nruns = c.take<uint32_t>((uint64_t)t.n_kernels + 1);
   uint64_t* gfirst = c.take<uint64_t>((uint64_t)t.n_kernels + 1);
+  RunList rl;
+  carve_runlist(c, t.n_records, rl);
   const uint32_t K = t.n_kernels;
   cudaMemsetAsync(switch_at, 0xFF, sizeof(int64_t) * K, s);
   if (dur) cudaMemsetAsync(dur, 0, sizeof(uint64_t) * K, s);
   cudaMemsetAsync(misc, 0, 64, s);
   const unsigned gk = (unsigned)umin64(ceil_div((uint64_t)K * 32, 256), (uint64_t)num_sms * 8);
-  note_launch(), k_warp_validate<<<gk, 256, 0, s>>>(t.kernel_rec_off, K, t.n_records, t.issue, t.retire, err);
+  const unsigned gv = (unsigned)umin64(ceil_div(umax64(t.n_records, K), 256), (uint64_t)num_sms * 8);
+  note_launch(), k_warp_validate<<<gv ? gv : 1, 256, 0, s>>>(t.kernel_rec_off, K, t.n_records, t.issue, t.retire,
+                                                             err);
   if (t.n_records == 0) return cudaGetLastError();
   note_launch(), k_warp_runs<<<(unsigned)ceil_div(K, 256), 256, 0, s>>>(t.kernel_rec_off, K, t.n_records, ok, 2 * n,
                                                                        nruns, gfirst, misc);
   WinArgs wa{};
-  wa.X = t.issue; wa.Y = t.retire; wa.gstart = t.kernel_rec_off; wa.G = misc + 0; wa.nruns = nruns;
-  wa.maxr = misc + 1; wa.ticket = misc + 2; wa.n = n; wa.dnum = dnum; wa.dden = dden; wa.gfirst = gfirst;
+  wa.X = t.issue; wa.Y = t.retire; wa.gstart = t.kernel_rec_off; wa.G = misc + 0;
+  wa.n = n; wa.dnum = dnum; wa.dden = dden; wa.gfirst = gfirst;
+  build_runlist(rl, misc + 0, nruns, misc, K, num_sms, wa, s);
   note_launch(), k_window<<<(unsigned)num_sms * 2, WT, 0, s>>>(wa);
   note_launch(), k_warp_finish<<<gk, 256, 0, s>>>(t.kernel_rec_off, K, t.issue, t.retire, gfirst, n, switch_at, dur);
   return cudaGetLastError();
