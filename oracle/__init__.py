@@ -57,6 +57,10 @@ def _L():
         L.or_stable.argtypes = [u32, u32, u64, vp, vp, vp, vp, vp, u32, u32, u32, u32, u32, i32, vp, vp, vp, vp]
         L.or_warp_stable.restype = i32
         L.or_warp_stable.argtypes = [u32, u64, vp, vp, vp, vp, u32, u32, u32, i32, vp, vp, vp]
+        L.or_kernel_predict.restype = i32
+        L.or_kernel_predict.argtypes = [u32, vp, vp, vp, vp, vp, vp, vp]
+        L.or_bb_predict.restype = i32
+        L.or_bb_predict.argtypes = [u32, u32, u64, u64, vp, vp, vp, vp, vp, vp, vp, vp]
         _lib = L
     return _lib
 
@@ -114,8 +118,8 @@ def signature(kernel_type_off, type_key, type_count):
     sig = np.zeros(max(16 * T, 1), np.uint64)
     mass = np.zeros(max(K, 1), np.uint64)
     bad = ctypes.c_int64(-1)
-    rc = _L().or_signature(K, _p(kto), _p(_c(type_key, np.uint32)), _p(_c(type_count, np.uint64)), _p(sig),
-                           _p(mass), ctypes.byref(bad))
+    tk, tc = _c(type_key, np.uint32), _c(type_count, np.uint64)  # converted copies must outlive the call
+    rc = _L().or_signature(K, _p(kto), _p(tk), _p(tc), _p(sig), _p(mass), ctypes.byref(bad))
     if rc != OK:
         raise OracleError(rc, bad.value)
     return sig[:16 * T], mass[:K]
@@ -128,8 +132,9 @@ def match(kernel_type_off, sig, mass, warps_total, theta=(1, 20), n_cores=64, po
     m = np.zeros(max(K, 1), np.int64)
     d = np.zeros(max(K, 1), np.float64)
     sg = _c(sig, np.uint64) if len(sig) else np.zeros(1, np.uint64)
-    rc = _L().or_match(K, _p(kto), _p(sg), _p(_c(mass, np.uint64)), _p(_c(warps_total, np.uint64)),
-                       int(theta[0]), int(theta[1]), int(n_cores), int(pool_all_prior), _p(m), _p(d))
+    ms, wt = _c(mass, np.uint64), _c(warps_total, np.uint64)  # converted copies must outlive the call
+    rc = _L().or_match(K, _p(kto), _p(sg), _p(ms), _p(wt), int(theta[0]), int(theta[1]), int(n_cores),
+                       int(pool_all_prior), _p(m), _p(d))
     if rc != OK:
         raise OracleError(rc, -1)
     return m[:K], d[:K]
@@ -143,8 +148,9 @@ def stable(timing, kernel_bb_insts, n=2048, delta=(3, 100), rate=(95, 100), brut
     sw = np.zeros(max(K, 1), np.int64)
     bad = ctypes.c_int64(-1)
     kbb = _c(kernel_bb_insts, np.uint64)
-    rc = _L().or_stable(K, B, R, _p(_c(timing.kernel_rec_off, np.uint64)), _p(_c(timing.bb, np.uint16)),
-                        _p(_c(timing.issue, np.uint64)), _p(_c(timing.retire, np.uint64)), _p(kbb), int(n),
+    kro, bbs = _c(timing.kernel_rec_off, np.uint64), _c(timing.bb, np.uint16)  # copies must outlive the call
+    iss, ret = _c(timing.issue, np.uint64), _c(timing.retire, np.uint64)
+    rc = _L().or_stable(K, B, R, _p(kro), _p(bbs), _p(iss), _p(ret), _p(kbb), int(n),
                         int(delta[0]), int(delta[1]), int(rate[0]), int(rate[1]), 1 if brute else 0, _p(fs),
                         _p(ds), _p(sw), ctypes.byref(bad))
     if rc != OK:
@@ -160,12 +166,42 @@ def warp_stable(timing, ok=None, n=1024, delta=(3, 100), brute=False):
     ds = np.zeros(max(K, 1), np.uint64)
     bad = ctypes.c_int64(-1)
     okc = None if ok is None else _c(ok, np.uint8)
-    rc = _L().or_warp_stable(K, R, _p(_c(timing.kernel_rec_off, np.uint64)), _p(_c(timing.issue, np.uint64)),
-                             _p(_c(timing.retire, np.uint64)), None if okc is None else _p(okc), int(n),
+    kro, iss = _c(timing.kernel_rec_off, np.uint64), _c(timing.issue, np.uint64)  # copies must outlive the call
+    ret = _c(timing.retire, np.uint64)
+    rc = _L().or_warp_stable(K, R, _p(kro), _p(iss), _p(ret), None if okc is None else _p(okc), int(n),
                              int(delta[0]), int(delta[1]), 1 if brute else 0, _p(sw), _p(ds), ctypes.byref(bad))
     if rc != OK:
         raise OracleError(rc, bad.value)
     return sw[:K], ds[:K]
+
+
+def kernel_predict(match, mass, full_insts, full_cycles):
+    """N3 kernel level: (pred_insts [K] u64, pred_cycles [K] u64) from each kernel's representative."""
+    K = len(match)
+    pi = np.zeros(max(K, 1), np.uint64)
+    pc = np.zeros(max(K, 1), np.uint64)
+    bad = ctypes.c_int64(-1)
+    m, ms, fi, fc = (_c(match, np.int64), _c(mass, np.uint64), _c(full_insts, np.uint64),
+                     _c(full_cycles, np.uint64))  # converted copies must outlive the call
+    rc = _L().or_kernel_predict(K, _p(m), _p(ms), _p(fi), _p(fc), _p(pi), _p(pc), ctypes.byref(bad))
+    if rc != OK:
+        raise OracleError(rc, bad.value)
+    return pi[:K], pc[:K]
+
+
+def bb_predict(trace, first_stable, stable_dur_sum):
+    """N3 BB level: (pred_dur_sum [W] u64, unpredicted [W] u32) of every warp of the trace."""
+    W = trace.n_warps
+    pd = np.zeros(max(W, 1), np.uint64)
+    un = np.zeros(max(W, 1), np.uint32)
+    bad = ctypes.c_int64(-1)
+    a = [_c(trace.kernel_warp_off, np.uint64), _c(trace.warp_event_off, np.uint64), _c(trace.bb, np.uint16),
+         _c(first_stable, np.int64), _c(stable_dur_sum, np.uint64)]  # converted copies must outlive the call
+    rc = _L().or_bb_predict(trace.n_kernels, trace.n_bb, W, trace.n_events, *[_p(x) for x in a], _p(pd), _p(un),
+                            ctypes.byref(bad))
+    if rc != OK:
+        raise OracleError(rc, bad.value)
+    return pd[:W], un[:W]
 
 
 def analyse(trace, theta=(1, 20), n_cores=64, pool_all_prior=0):

@@ -591,3 +591,76 @@ def test_warp_stable_generated_modes_agree_and_range_errors():
     with pytest.raises(oracle.OracleError) as ei:
         oracle.warp_stable(_warp_stream([([1, 2], [9, 8])]), None, n=2)  # not retire-sorted
     assert ei.value.index == 1
+
+
+# ---- N3: kernel- and BB-level prediction (Fig 12 Step 4 / L279-281, Fig 7 Step 3) ------------------------------
+def _half_up(num: Fraction) -> int:
+    return int((num + Fraction(1, 2)) // 1)
+
+
+def test_kernel_predict_formula_and_rounding():
+    # #insts = #insts^K' * #insts_sample / #insts^K'_sample (L279-281); IPC(K) = IPC(K') => the same ratio scales
+    # the cycles; a representative keeps its simulated counts
+    match = np.array([-1, 0, 0, -1, 3], np.int64)
+    mass = np.array([3, 2, 1, 4, 2], np.uint64)          # N_k: instructions of the analysed sample (A3 masses)
+    full_i = np.array([1000, 0, 0, 7, 0], np.uint64)
+    full_c = np.array([3, 0, 0, 5, 0], np.uint64)
+    pi, pc = oracle.kernel_predict(match, mass, full_i, full_c)
+    assert pi.tolist() == [1000, 667, 333, 7, 4]          # 2000/3 -> 667, 1000/3 -> 333, 7*2/4 = 3.5 -> 4 (half up)
+    assert pc.tolist() == [3, 2, 1, 5, 3]                 # 5*2/4 = 2.5 -> 3
+    rs = np.random.default_rng(5)
+    for _ in range(200):
+        K = int(rs.integers(1, 6))
+        match = np.array([-1] + [int(rs.integers(-1, k)) for k in range(1, K)], np.int64)
+        mass = rs.integers(1, 1 << 40, K).astype(np.uint64)
+        fi = rs.integers(0, 1 << 62, K).astype(np.uint64)
+        fc = rs.integers(0, 1 << 62, K).astype(np.uint64)
+        exact = [max(_half_up(Fraction(int(fi[r]) * int(mass[k]), int(mass[r]))),
+                     _half_up(Fraction(int(fc[r]) * int(mass[k]), int(mass[r])))) if r >= 0 else 0
+                 for k, r in enumerate(int(x) for x in match)]
+        if max(exact) >= 1 << 64:  # a prediction that does not fit u64 is a range error, not a wrapped value
+            with pytest.raises(oracle.OracleError):
+                oracle.kernel_predict(match, mass, fi, fc)
+            continue
+        pi, pc = oracle.kernel_predict(match, mass, fi, fc)
+        for k in range(K):
+            r = int(match[k])
+            if r < 0:
+                assert (int(pi[k]), int(pc[k])) == (int(fi[k]), int(fc[k]))
+            else:
+                assert int(pi[k]) == _half_up(Fraction(int(fi[r]) * int(mass[k]), int(mass[r])))
+                assert int(pc[k]) == _half_up(Fraction(int(fc[r]) * int(mass[k]), int(mass[r])))
+
+
+def test_bb_predict_worked_example_and_invariants():
+    # the worked example's kernel A (L178 pipeline): warps [0,1,1,2] x3 and [0,1,2]; types 0 and 1 stable with
+    # S_n = 40 and 90 (n = 10: mean durations 4 and 9 ticks), type 2 never stable (a rare BB: interval model, out)
+    g = _gold("worked_example.json")
+    tr = tg.trace_from_warps(g["kernels"], g["bb_len"])
+    K, B = tr.n_kernels, tr.n_bb
+    fs = np.full((K, B), -1, np.int64)
+    ds = np.zeros((K, B), np.uint64)
+    fs[0, 0], ds[0, 0] = 5, 40
+    fs[0, 1], ds[0, 1] = 9, 90
+    pd, un = oracle.bb_predict(tr, fs, ds)
+    W0 = int(tr.kernel_warp_off[1])
+    assert pd[:W0].tolist() == [40 + 2 * 90, 40 + 2 * 90, 40 + 90, 40 + 2 * 90]
+    assert un[:W0].tolist() == [1, 1, 1, 1]
+    assert pd[W0:].tolist() == [0] * (tr.n_warps - W0) and un[W0:].tolist() == [4] * (tr.n_warps - W0)
+    # invariant on a generated trace: per kernel, sum_w pred = sum_b (executions of b) * S_n(b) over stable b, with
+    # the executions taken independently from the A1 BB distribution (kernel_bb_insts / len)
+    g6 = tg.Generator(6)
+    tr6 = g6.kernels_trace(0, 10)
+    _, _, kbb = oracle.bbv(tr6)
+    rs = np.random.default_rng(9)
+    fs = np.where(rs.random((tr6.n_kernels, tr6.n_bb)) < 0.7, 1, -1).astype(np.int64)
+    ds = rs.integers(1, 1 << 30, (tr6.n_kernels, tr6.n_bb)).astype(np.uint64)
+    pd, un = oracle.bb_predict(tr6, fs, ds)
+    kwo = np.asarray(tr6.kernel_warp_off, np.int64)
+    blen = np.asarray(tr6.bb_len, np.uint64)
+    for k in range(tr6.n_kernels):
+        execs = kbb[k] // blen
+        want = sum(int(execs[b]) * int(ds[k, b]) for b in range(tr6.n_bb) if fs[k, b] >= 0)
+        miss = sum(int(execs[b]) for b in range(tr6.n_bb) if fs[k, b] < 0)
+        assert sum(int(x) for x in pd[kwo[k]:kwo[k + 1]]) == want
+        assert int(un[kwo[k]:kwo[k + 1]].sum()) == miss
