@@ -93,6 +93,10 @@ _SIGS = [
     ("photon_warp_stable_workspace_bytes", c_size_t, [POINTER(Timing)]),
     ("photon_warp_stable", c_int, [c_void_p, POINTER(Timing), c_void_p, WarpStableParams, c_void_p, c_size_t,
                                    c_void_p, c_void_p, c_void_p]),
+    ("photon_kernel_predict", c_int, [c_void_p, c_uint32, c_void_p, c_void_p, c_void_p, c_void_p, c_void_p,
+                                      c_size_t, c_void_p, c_void_p, c_void_p]),
+    ("photon_bb_predict", c_int, [c_void_p, POINTER(Trace), c_void_p, c_void_p, c_void_p, c_size_t, c_void_p,
+                                  c_void_p, c_void_p]),
     ("photon_types_export", c_int, [c_void_p, c_uint32, POINTER(Types), c_uint32, c_uint64, c_void_p, c_void_p]),
     ("photon_merge_workspace_bytes", c_size_t, [c_uint64, c_uint32]),
     ("photon_types_merge", c_int, [c_void_p, c_void_p, c_uint64, c_uint32, c_void_p, c_void_p, c_size_t,

@@ -339,6 +339,35 @@ class Photon:
             self.check(ws, stream)
         return o
 
+    # -- N3: kernel- and BB-level prediction (Fig 12 Step 4 / L279-281; Fig 7 Step 3) -------------------------
+    def photon_kernel_predict(self, match, mass, full_insts, full_cycles, stream=None, check: bool = True) -> dict:
+        """pred_insts / pred_cycles [K] of every kernel from its representative (round half up)."""
+        K = int(match.numel())
+        ws = self.workspace("kpredict", 256)
+        o = {"pred_insts": self.empty(K, "int64"), "pred_cycles": self.empty(K, "int64")}
+        self._rc(self.L.photon_kernel_predict(self.ctx, K, match.data_ptr(), mass.data_ptr(), full_insts.data_ptr(),
+                                              full_cycles.data_ptr(), ws.data_ptr(), ws.numel(),
+                                              o["pred_insts"].data_ptr(), o["pred_cycles"].data_ptr(),
+                                              self.stream_ptr(stream)))
+        o["_ws"] = ws
+        if check:
+            self.check(ws, stream)
+        return o
+
+    def photon_bb_predict(self, t: DeviceTrace, first_stable, stable_dur_sum, stream=None, check: bool = True) -> dict:
+        """pred_dur_sum [W] (sum of the stable types' S_n over each warp's events) and unpredicted [W]."""
+        ct = t.c()
+        ws = self.workspace("bpredict", 256)
+        o = {"pred_dur_sum": self.empty(t.n_warps, "int64"), "unpredicted": self.empty(t.n_warps, "int32")}
+        self._rc(self.L.photon_bb_predict(self.ctx, ctypes.byref(ct), first_stable.data_ptr(),
+                                          stable_dur_sum.data_ptr(), ws.data_ptr(), ws.numel(),
+                                          o["pred_dur_sum"].data_ptr(), o["unpredicted"].data_ptr(),
+                                          self.stream_ptr(stream)))
+        o["_ws"] = ws
+        if check:
+            self.check(ws, stream)
+        return o
+
     # -- multi-GPU helpers -------------------------------------------------------------------------------------
     def photon_types_export(self, K_local, ty, kernel_base, warp_base, rows, stream=None):
         tc = self.types_c(ty)

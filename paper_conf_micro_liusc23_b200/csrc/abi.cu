@@ -643,6 +643,41 @@ int photon_warp_stable(photon_ctx* ctx, const photon_timing* t, const uint8_t* o
   return PHOTON_OK;
 }
 
+// ---- N3 -----------------------------------------------------------------------------------------------------
+int photon_kernel_predict(photon_ctx* ctx, uint32_t K, const int64_t* match, const uint64_t* mass,
+                          const uint64_t* full_insts, const uint64_t* full_cycles, void* ws, size_t ws_bytes,
+                          uint64_t* pred_insts, uint64_t* pred_cycles, void* stream) {
+  if (!ctx) return PHOTON_EINVAL;
+  if (!match || !mass || !full_insts || !full_cycles || !pred_insts || !pred_cycles || !ws || K == 0)
+    return fail(ctx, PHOTON_EINVAL, "bad kernel_predict arguments");
+  if (ws_bytes < 256) return fail(ctx, PHOTON_EWORKSPACE, "kernel_predict workspace must be >= 256 bytes");
+  cudaStream_t s = (cudaStream_t)stream;
+  CK(cudaSetDevice(ctx->device), "cudaSetDevice");
+  ctx->last_ws = ws;
+  DevErr* err = (DevErr*)ws;
+  CK(cudaMemsetAsync(err, 0, sizeof(DevErr), s), "memset");
+  CK(launch_kernel_predict(K, match, mass, full_insts, full_cycles, pred_insts, pred_cycles, err, s), "predict");
+  return PHOTON_OK;
+}
+
+int photon_bb_predict(photon_ctx* ctx, const photon_trace* t, const int64_t* first_stable, const uint64_t* dur,
+                      void* ws, size_t ws_bytes, uint64_t* pred, uint32_t* unpred, void* stream) {
+  if (!ctx) return PHOTON_EINVAL;
+  int rc = check_trace(ctx, t);
+  if (rc) return rc;
+  if (!first_stable || !dur || !pred || !unpred || !ws) return fail(ctx, PHOTON_EINVAL, "NULL argument");
+  if (ws_bytes < 256) return fail(ctx, PHOTON_EWORKSPACE, "bb_predict workspace must be >= 256 bytes");
+  cudaStream_t s = (cudaStream_t)stream;
+  CK(cudaSetDevice(ctx->device), "cudaSetDevice");
+  ctx->last_ws = ws;
+  DevErr* err = (DevErr*)ws;
+  CK(cudaMemsetAsync(err, 0, sizeof(DevErr), s), "memset");
+  TraceDev d = to_dev(t);
+  CK(launch_validate_offsets(d, err, s), "validate");
+  CK(launch_bb_predict(d, first_stable, dur, pred, unpred, err, ctx->num_sms, s), "bb_predict");
+  return PHOTON_OK;
+}
+
 // ---- multi-GPU helpers ------------------------------------------------------------------------------------
 int photon_types_export(photon_ctx* ctx, uint32_t K_local, const photon_types* local, uint32_t kernel_base,
                         uint64_t warp_base, photon_type_row* rows, void* stream) {

@@ -141,6 +141,12 @@ size_t warp_stable_ws_bytes(uint32_t K, uint64_t R);
 cudaError_t launch_warp_stable(const photon_timing& t, const uint8_t* ok, uint32_t n, uint32_t dnum, uint32_t dden,
                                void* ws, int64_t* switch_at, uint64_t* dur, DevErr* err, int num_sms,
                                cudaStream_t s);
+// ---- N3 (k_predict.cu) --------------------------------------------------------------------------------------
+cudaError_t launch_kernel_predict(uint32_t K, const int64_t* match, const uint64_t* mass, const uint64_t* full_insts,
+                                  const uint64_t* full_cycles, uint64_t* pred_insts, uint64_t* pred_cycles,
+                                  DevErr* err, cudaStream_t s);
+cudaError_t launch_bb_predict(const TraceDev& t, const int64_t* first_stable, const uint64_t* dur, uint64_t* pred,
+                              uint32_t* unpred, DevErr* err, int num_sms, cudaStream_t s);
 cudaError_t launch_stable(const photon_timing& t, const uint64_t* kbb, photon_stable_params p, void* ws,
                           size_t ws_bytes, int64_t* first_stable, uint64_t* dur, int64_t* switch_at, DevErr* err,
                           int num_sms, cudaStream_t s);

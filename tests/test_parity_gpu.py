@@ -376,3 +376,67 @@ def test_warp_stable_paper_lines_and_errors(ph):
     with pytest.raises(PhotonError) as ei:
         check_warp_stable(ph, bad, None, 2)
     assert ei.value.code == -3 and ei.value.index == 1
+
+
+# ---- N3: kernel- and BB-level prediction (Fig 12 Step 4 / L279-281; Fig 7 Step 3) -------------------------------
+def test_kernel_predict_chain_c4(ph):
+    # ResNet-152: the GPU chain's matches and masses feed the prediction; synthetic "detailed simulation" counts for
+    # the representatives; compared element by element with the oracle on the same inputs
+    from paper_conf_micro_liusc23_b200 import to_device
+    tr = tg.Generator(4).trace()
+    d = _dev(ph, tr)
+    r = ph.analyse(d)
+    match = _np(r["match"], np.int64)
+    ref = oracle.analyse(tr)
+    assert np.array_equal(match, ref["match"])
+    mass = ref["mass"]
+    rs = np.random.default_rng(4)
+    fi = rs.integers(1, 1 << 40, len(match)).astype(np.uint64)
+    fc = rs.integers(1, 1 << 40, len(match)).astype(np.uint64)
+    dv = lambda a, dt: to_device(np.ascontiguousarray(a, dt), ph.device)
+    o = ph.photon_kernel_predict(dv(match, np.int64), dv(mass, np.uint64), dv(fi, np.uint64), dv(fc, np.uint64))
+    pi, pc = oracle.kernel_predict(match, mass, fi, fc)
+    assert np.array_equal(_np(o["pred_insts"], np.uint64), pi)
+    assert np.array_equal(_np(o["pred_cycles"], np.uint64), pc)
+    assert (match >= 0).sum() > 100  # the repeated conv4_x blocks are predicted, not simulated
+
+
+def test_kernel_predict_errors(ph):
+    from paper_conf_micro_liusc23_b200 import PhotonError, to_device
+    dv = lambda a, dt: to_device(np.ascontiguousarray(a, dt), ph.device)
+    with pytest.raises(PhotonError) as ei:  # representative index must precede the kernel
+        ph.photon_kernel_predict(dv([-1, 1], np.int64), dv([3, 2], np.uint64), dv([5, 5], np.uint64),
+                                 dv([5, 5], np.uint64))
+    assert ei.value.code == -3 and ei.value.index == 1
+
+
+@pytest.mark.parametrize("cfg", [3, 6])
+def test_bb_predict_from_gpu_stability(ph, cfg):
+    # A5 on the GPU gives first_stable / S_n; the per-warp BB-level prediction over the same config's trace
+    from paper_conf_micro_liusc23_b200 import DeviceTiming, to_device
+    g = tg.Generator(cfg)
+    tr = g.trace()
+    d = _dev(ph, tr)
+    kbb = ph.photon_bbv_build(d, bbv16=False, insts=False, kbb=True)["kernel_bb_insts"]
+    n = 2048 if cfg == 3 else 32
+    st = ph.photon_bb_stable(DeviceTiming.from_host(g.timing(), ph.device), kbb, n)
+    o = ph.photon_bb_predict(d, st["first_stable"], st["stable_dur_sum"])
+    fs = _np(st["first_stable"], np.int64).reshape(tr.n_kernels, tr.n_bb)
+    ds = _np(st["stable_dur_sum"], np.uint64).reshape(tr.n_kernels, tr.n_bb)
+    pd, un = oracle.bb_predict(tr, fs, ds)
+    assert np.array_equal(_np(o["pred_dur_sum"], np.uint64), pd)
+    assert np.array_equal(_np(o["unpredicted"], np.uint32), un)
+    assert (pd > 0).any() and (un > 0).any()
+
+
+def test_bb_predict_random_tables(ph):
+    from paper_conf_micro_liusc23_b200 import to_device
+    for seed in range(4):
+        tr = tg.random_trace(seed, n_kernels=1 + seed, max_warps=700, max_events=300, n_bb=[7, 300, 5000, 16][seed])
+        rs = np.random.default_rng(seed)
+        fs = np.where(rs.random((tr.n_kernels, tr.n_bb)) < 0.6, 1, -1).astype(np.int64)
+        ds = rs.integers(1, 1 << 50, (tr.n_kernels, tr.n_bb)).astype(np.uint64)
+        o = ph.photon_bb_predict(_dev(ph, tr), to_device(fs, ph.device), to_device(ds, ph.device))
+        pd, un = oracle.bb_predict(tr, fs, ds)
+        assert np.array_equal(_np(o["pred_dur_sum"], np.uint64), pd)
+        assert np.array_equal(_np(o["unpredicted"], np.uint32), un)
