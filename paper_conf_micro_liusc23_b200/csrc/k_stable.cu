@@ -396,10 +396,11 @@ __global__ void k_work_count(const uint64_t* gstart, const uint32_t* G, uint32_t
 
 // The compact run list, run-major (every group's run 0 before any group's run 1): count the groups per run index,
 // scan, fill (the order of groups inside one run index is immaterial).  list[i] = g | (uint64)r << 32.
+// one warp per group, lanes over its runs (a long group's runs are not a serial chain of atomics)
 __global__ void k_runs_count(const uint32_t* G, const uint32_t* nruns, uint32_t* cnt) {
-  const uint32_t ng = *G;
-  for (uint32_t g = blockIdx.x * blockDim.x + threadIdx.x; g < ng; g += gridDim.x * blockDim.x)
-    for (uint32_t r = 0; r < nruns[g]; ++r) atomicAdd(&cnt[r], 1u);
+  const uint32_t ng = *G, lane = threadIdx.x & 31, nw = (gridDim.x * blockDim.x) >> 5;
+  for (uint32_t g = (blockIdx.x * blockDim.x + threadIdx.x) >> 5; g < ng; g += nw)
+    for (uint32_t r = lane; r < nruns[g]; r += 32) atomicAdd(&cnt[r], 1u);
 }
 __global__ void __launch_bounds__(1024) k_runs_scan(const uint32_t* maxr, uint32_t* cnt, uint32_t* total) {
   __shared__ uint32_t ws[32];
@@ -428,9 +429,10 @@ __global__ void __launch_bounds__(1024) k_runs_scan(const uint32_t* maxr, uint32
 }
 __global__ void k_runs_fill(const uint32_t* G, const uint32_t* nruns, const uint32_t* off, uint32_t* fill,
                             uint64_t* list) {
-  const uint32_t ng = *G;
-  for (uint32_t g = blockIdx.x * blockDim.x + threadIdx.x; g < ng; g += gridDim.x * blockDim.x)
-    for (uint32_t r = 0; r < nruns[g]; ++r) list[off[r] + atomicAdd(&fill[r], 1u)] = (uint64_t)g | ((uint64_t)r << 32);
+  const uint32_t ng = *G, lane = threadIdx.x & 31, nw = (gridDim.x * blockDim.x) >> 5;
+  for (uint32_t g = (blockIdx.x * blockDim.x + threadIdx.x) >> 5; g < ng; g += nw)
+    for (uint32_t r = lane; r < nruns[g]; r += 32)
+      list[off[r] + atomicAdd(&fill[r], 1u)] = (uint64_t)g | ((uint64_t)r << 32);
 }
 
 // ---- 4. windowed exact test ----------------------------------------------------------------------------------
@@ -784,7 +786,7 @@ inline void build_runlist(const RunList& rl, const uint32_t* G, const uint32_t* 
                           int num_sms, WinArgs& wa, cudaStream_t s) {
   cudaMemsetAsync(rl.cnt, 0, sizeof(uint32_t) * rl.cap_r, s);
   cudaMemsetAsync(rl.fill, 0, sizeof(uint32_t) * rl.cap_r, s);
-  const unsigned gg = (unsigned)umin64(ceil_div(gcap, 256), (uint64_t)num_sms * 4);
+  const unsigned gg = (unsigned)umin64(ceil_div(gcap * 32, 256), (uint64_t)num_sms * 8);
   note_launch(), k_runs_count<<<gg ? gg : 1, 256, 0, s>>>(G, nruns, rl.cnt);
   note_launch(), k_runs_scan<<<1, 1024, 0, s>>>(misc + 1, rl.cnt, misc + 3);
   note_launch(), k_runs_fill<<<gg ? gg : 1, 256, 0, s>>>(G, nruns, rl.cnt, rl.fill, rl.list);
