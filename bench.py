@@ -332,6 +332,27 @@ def run_photon(args):
         ams = b0.elapsed_time(b1) / n5
         R = tm.n_records
         abytes = 18 * R
+        # ---- N3 BB-level prediction over the same config's trace with these stability tables ----
+        o3 = ph.photon_bb_predict(da, o["first_stable"], o["stable_dur_sum"])
+        for _ in range(max(args.warmup - 1, 0)):
+            o3 = ph.photon_bb_predict(da, o["first_stable"], o["stable_dur_sum"], check=False)
+        torch.cuda.synchronize()
+        p0, p1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        p0.record(s)
+        for _ in range(n5):
+            o3 = ph.photon_bb_predict(da, o["first_stable"], o["stable_dur_sum"], check=False)
+        p1.record(s)
+        torch.cuda.synchronize()
+        ph.check(o3["_ws"])
+        pms = p0.elapsed_time(p1) / n5
+        EA, WA = ta.n_events, ta.n_warps
+        pbytes = 2 * EA + 8 * (WA + 1) + 12 * WA  # events + offsets + the two per-warp outputs
+        line["n3"] = {"metric": "trace events predicted/sec (BB-level per-warp time prediction)",
+                      "value": EA / (pms / 1000), "unit": "events/s", "ms_per_step": pms, "events": EA,
+                      "workload": f"{CONFIG_DESC.get(args.a5_config)} trace with its A5 tables (n=2048)",
+                      "roofline": {"bound": "hbm", "achieved": pbytes / (pms / 1000) / 1e9, "peak": hbm_peak,
+                                   "unit": "GB/s", "frac": pbytes / (pms / 1000) / 1e9 / hbm_peak,
+                                   "algorithmic_bytes": pbytes, "traffic": None}}
         line["a5"] = {"metric": "BB timing records tested/sec (stability test + switch)", "value": R / (ams / 1000),
                       "unit": "records/s", "ms_per_step": ams, "records": R,
                       "workload": f"{CONFIG_DESC.get(args.a5_config)} timing stream (wave model), n=2048, delta=3/100",

@@ -7,8 +7,8 @@
 // BB level, Fig 7 Step 3 / L204: the remaining warps' time is "accumulating the predicted time of their basic
 // blocks"; a stable type's time is its mean at the latch, S_n / n (A5).  pred_dur_sum[w] = sum of S_n(k, b) over
 // the warp's events of stable types, unpredicted[w] = its events of types never stable [N3-b].  A segmented sum
-// over the trace: one hardware warp per analysed warp (coalesced u16 event loads, the kernel's row of the A5
-// tables stays in L1/L2), grid-stride; u64 overflow of a warp's sum is latched as ERANGE.
+// over the trace: one thread per analysed warp (the kernel's row of the A5 tables stays in L1/L2; a warp's events
+// are read in order, so each 32-byte sector is fetched once), grid-stride; u64 overflow of a warp's sum is ERANGE.
 #include "internal.h"
 
 namespace photon {
@@ -38,59 +38,79 @@ __global__ void k_kernel_predict(uint32_t K, const int64_t* __restrict__ match, 
   }
 }
 
+// One thread per analysed warp, 256 consecutive warps per CTA step (the block's first kernel by one binary search,
+// each thread then steps forward); a thread walks its warp's events in aligned 16-byte words (eight events per
+// load, independent table loads); the trace base is 16-byte aligned (photon_trace contract).
 __global__ void __launch_bounds__(256) k_bb_predict(const uint64_t* __restrict__ kwo, uint32_t K, uint32_t B,
                                                     const uint64_t* __restrict__ weo, uint64_t W, uint64_t E,
                                                     const uint16_t* __restrict__ bb,
                                                     const int64_t* __restrict__ first_stable,
                                                     const uint64_t* __restrict__ dur, uint64_t* pred,
                                                     uint32_t* unpred, DevErr* err) {
-  const uint32_t lane = threadIdx.x & 31;
-  const uint64_t hw = ((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-  const uint64_t nhw = ((uint64_t)gridDim.x * blockDim.x) >> 5;
-  // a contiguous range of analysed warps per hardware warp: the kernel index only moves forward
-  const uint64_t per = ceil_div(W, nhw), w0 = hw * per, w1 = umin64(w0 + per, W);
-  uint32_t k = 0;
-  if (w0 < w1) {  // last kernel with kwo[k] <= w0
-    uint32_t lo = 0, hi2 = K - 1;
-    while (lo < hi2) {
-      const uint32_t mid = (lo + hi2 + 1) >> 1;
-      if (kwo[mid] <= w0) lo = mid; else hi2 = mid - 1;
+  __shared__ uint32_t s_k0;
+  for (uint64_t w0 = (uint64_t)blockIdx.x * 256; w0 < W; w0 += (uint64_t)gridDim.x * 256) {
+    if (threadIdx.x == 0) {  // last kernel with kwo[k] <= w0
+      uint32_t lo = 0, hi = K - 1;
+      while (lo < hi) {
+        const uint32_t mid = (lo + hi + 1) >> 1;
+        if (kwo[mid] <= w0) lo = mid; else hi = mid - 1;
+      }
+      s_k0 = lo;
     }
-    k = lo;
-  }
-  for (uint64_t w = w0; w < w1; ++w) {
+    __syncthreads();
+    const uint64_t w = w0 + threadIdx.x;
+    uint32_t k = s_k0;
+    __syncthreads();
+    if (w >= W) continue;
     while (k + 1 < K && kwo[k + 1] <= w) ++k;
     const uint64_t s = umin64(weo[w], E), e = umin64(umax64(weo[w + 1], s), E);
     const int64_t* fs = first_stable + (uint64_t)k * B;
     const uint64_t* ds = dur + (uint64_t)k * B;
-    uint64_t lo = 0, hi = 0;  // this lane's u128 sum
+    uint64_t lo = 0, hi = 0;  // u128 sum
     uint32_t miss = 0;
-    for (uint64_t i = s + lane; i < e; i += 32) {
-      const uint32_t b = bb[i];
-      if (b >= B) {
+    bool bad = weo[w + 1] < weo[w];
+    auto add1 = [&](uint32_t bv, uint64_t i) {
+      if (bv >= B) {
         latch(err, PHOTON_ERANGE, (int64_t)i);
-        continue;
+        return;
       }
-      if (fs[b] >= 0) {
-        const uint64_t v = ds[b];
-        lo += v;
-        hi += lo < v;
-      } else {
-        ++miss;
+      const int64_t f = fs[bv];
+      const uint64_t x = f >= 0 ? ds[bv] : 0ull;
+      miss += f < 0 ? 1u : 0u;
+      lo += x;
+      hi += lo < x;
+    };
+    // unaligned head, then whole 16-byte words (8 events per load, table loads independent), then the tail
+    const uint64_t a8 = umin64((s + 7) & ~7ull, e), z8 = umax64(e & ~7ull, a8);
+    for (uint64_t i = s; i < a8; ++i) add1(bb[i], i);
+    for (uint64_t i0 = a8; i0 < z8; i0 += 8) {
+      const uint4 q = *(const uint4*)(bb + i0);
+      const uint32_t b8[8] = {q.x & 0xFFFFu, q.x >> 16, q.y & 0xFFFFu, q.y >> 16,
+                              q.z & 0xFFFFu, q.z >> 16, q.w & 0xFFFFu, q.w >> 16};
+      int64_t f[8];
+      uint64_t v[8];
+#pragma unroll
+      for (int u = 0; u < 8; ++u) {
+        const uint32_t bu = b8[u] < B ? b8[u] : 0u;
+        f[u] = fs[bu];
+        v[u] = ds[bu];
+      }
+#pragma unroll
+      for (int u = 0; u < 8; ++u) {
+        if (b8[u] >= B) {
+          latch(err, PHOTON_ERANGE, (int64_t)(i0 + u));
+          continue;
+        }
+        const uint64_t x = f[u] >= 0 ? v[u] : 0ull;
+        miss += f[u] < 0 ? 1u : 0u;
+        lo += x;
+        hi += lo < x;
       }
     }
-    for (int o = 16; o > 0; o >>= 1) {
-      const uint64_t lo2 = __shfl_xor_sync(0xffffffffu, lo, o), hi2 = __shfl_xor_sync(0xffffffffu, hi, o);
-      const uint64_t t = lo + lo2;
-      hi = hi + hi2 + (t < lo);
-      lo = t;
-      miss += __shfl_xor_sync(0xffffffffu, miss, o);
-    }
-    if (lane == 0) {
-      if (hi != 0 || weo[w + 1] < weo[w]) latch(err, PHOTON_ERANGE, (int64_t)w);
-      pred[w] = lo;
-      unpred[w] = miss;
-    }
+    for (uint64_t i = z8; i < e; ++i) add1(bb[i], i);
+    if (hi != 0 || bad) latch(err, PHOTON_ERANGE, (int64_t)w);
+    pred[w] = lo;
+    unpred[w] = miss;
   }
 }
 
@@ -108,7 +128,7 @@ cudaError_t launch_kernel_predict(uint32_t K, const int64_t* match, const uint64
 cudaError_t launch_bb_predict(const TraceDev& t, const int64_t* first_stable, const uint64_t* dur, uint64_t* pred,
                               uint32_t* unpred, DevErr* err, int num_sms, cudaStream_t s) {
   if (t.W == 0) return cudaSuccess;
-  const unsigned grid = (unsigned)umin64(ceil_div(t.W * 32, 256), (uint64_t)num_sms * 16);
+  const unsigned grid = (unsigned)umin64(ceil_div(t.W, 256), (uint64_t)num_sms * 8);
   note_launch(), k_bb_predict<<<grid, 256, 0, s>>>(t.kwo, t.K, t.B, t.weo, t.W, t.E, t.bb, first_stable, dur, pred,
                                                    unpred, err);
   return cudaGetLastError();
