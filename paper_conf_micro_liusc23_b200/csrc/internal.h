@@ -70,6 +70,11 @@ cudaError_t launch_validate_offsets(const TraceDev& t, DevErr* err, cudaStream_t
 cudaError_t launch_bbv(const TraceDev& t, const uint32_t* tbl, const uint32_t* max_len, const ItemTable& it,
                        uint32_t* warp_bbv16, uint64_t* warp_insts, const TileEntries* te, DevErr* err, int num_sms,
                        cudaStream_t s);
+// K1 v2 (k_bbv2.cu): lane-range accumulation with red.shared into lane-private columns; needs the BB table in
+// shared memory (next_pow2(B) <= 4096); launch_bbv dispatches to it when supported
+bool bbv2_supported(uint32_t B);
+cudaError_t launch_bbv2(const TraceDev& t, const uint32_t* tbl, const ItemTable& it, uint32_t* warp_bbv16,
+                        uint64_t* warp_insts, const TileEntries* te, DevErr* err, int num_sms, cudaStream_t s);
 // K2a de-dup from materialised BBVs (unfused path)
 cudaError_t launch_group_from_bbv(const TraceDev& t, const uint32_t* warp_bbv16, const ItemTable& it,
                                   const TileEntries& te, DevErr* err, cudaStream_t s);

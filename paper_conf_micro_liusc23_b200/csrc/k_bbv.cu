@@ -22,6 +22,8 @@
 // memory table; the tile's distinct (kernel, key, count, first warp) entries go to a per-tile slot area and each
 // warp gets its local entry id (u16).  No global atomics on the streaming path: k_entries_insert (k_types.cu)
 // inserts the entries into the global type table.
+#include <stdlib.h>
+
 #include "internal.h"
 
 #ifndef PHOTON_EXP
@@ -990,6 +992,8 @@ static cudaError_t launch_bbv_t(const BbvArgs& a, size_t smem, int num_sms, cuda
 cudaError_t launch_bbv(const TraceDev& t, const uint32_t* tbl, const uint32_t* max_len, const ItemTable& it,
                        uint32_t* warp_bbv16, uint64_t* warp_insts, const TileEntries* te, DevErr* err, int num_sms,
                        cudaStream_t s) {
+  if (bbv2_supported(t.B) && !getenv("PHOTON_K1_V1"))
+    return launch_bbv2(t, tbl, it, warp_bbv16, warp_insts, te, err, num_sms, s);
   BbvArgs a{};
   a.kwo = t.kwo; a.weo = t.weo; a.bb = t.bb; a.tbl = tbl; a.max_len = max_len; a.tile_k0 = it.k0;
   a.item_w0 = it.w0; a.n_items = it.n; a.counter = it.n + 1;
