@@ -15,12 +15,12 @@
 //    chunk's lane tables are built).  Each chunk is split into 256 equal lane ranges of Q <= 9 words (Q odd, so the 32 lanes' 16-byte LDS hit distinct
 //    bank groups).  Lane t walks its range in order; the piece of each analysed warp it meets is accumulated in a
 //    column private to the lane with red.shared.add (no read-modify-write latency chain): the first piece in the
-//    lane's slot-0 column (bank = lane, conflict-free), further pieces in pool columns handed out by an exclusive
-//    scan over the lanes (a chunk starts at most 256 warps, so the pool never overflows).  Per event: one LDS of
+//    lane's slot-0 column (bank = lane, conflict-free); a warp starting inside the lane's range goes to the pool
+//    column of its own index (an item holds <= 256 warps, so pool columns are unique).  Per event: one LDS of
 //    the packed (len, bin) entry, one RED.
 //  * Thread u then sums its warp's pieces (the owner column in the lane holding the warp's first event of the
-//    chunk, then slot 0 of every later lane the warp spans) into its key registers.  Every column that received
-//    events is zeroed by its single reader, so there are no bulk clears.
+//    chunk, then slot 0 of every later lane the warp spans) into its key registers.  The cells are cleared with
+//    16-byte stores (conflict-free) while the next chunk's lane tables are built.
 //  * Bin cells are u32: a chunk holds <= 18432 events of length < 2^17, so a chunk piece cannot wrap; the per-warp
 //    totals are carried in u64 and checked against 2^32 (PHOTON_ERANGE).
 #include "internal.h"
@@ -38,6 +38,7 @@ constexpr int ROWB = ROW * 4;        // bin stride in bytes; local table entry =
 constexpr uint32_t TOFF = 0x7800u;   // bin * ROWB bits of an entry
 constexpr int TSH = 15;              // length shift
 constexpr int LSLOTS = 256;          // CTA-local de-dup slots
+constexpr int LPROBE = 16;           // probes before a leader takes an entry of its own (the global insert merges)
 constexpr int SMEM_TBL_MAX = 4096;   // BB table entries kept in shared memory
 static_assert(ROWB == 2048 && 15 * ROWB <= (int)TOFF, "bin offset layout");
 
@@ -64,14 +65,13 @@ constexpr size_t kCellBytes = (size_t)16 * ROWB;     // 32 KB
 constexpr size_t kStageBytes = (size_t)CHE * 2;      // 36 KB
 constexpr size_t kOffBytes = (size_t)(NT + 4) * 8;   // item warp offsets (u64)
 constexpr size_t kRelBytes = (size_t)(NT + 4) * 4;   // chunk-relative warp starts (u32)
-constexpr size_t kLaneBytes = (size_t)3 * NT * 2;    // fw, fl, pb (u16)
 constexpr size_t kLocalBytes = (size_t)LSLOTS * (8 + 4 + 4 + 4 + 4);
 constexpr size_t kMiscBytes = 256;
 constexpr size_t kKidBytes = (size_t)NT * 4;
 
 // everything but the cells and the stage
 __host__ __device__ constexpr size_t small_bytes(uint32_t tbl_entries) {
-  return kOffBytes + kRelBytes + kLaneBytes + 32 + 16 + kLocalBytes + kMiscBytes + kKidBytes +
+  return kOffBytes + kRelBytes + 16 + kLocalBytes + kMiscBytes + kKidBytes +
          (size_t)tbl_entries * 4;
 }
 // Layout: the cells must start on a 32 KB boundary of the shared window (cell address = column | bin offset).  The
@@ -86,10 +86,6 @@ struct Smem {
   uint16_t* stage;   // [CHE]
   uint64_t* off;     // [NT+4] weo of the item's warps (monotone), off[nw] = item end, padded
   uint32_t* rel;     // [NT+4] chunk-relative starts (clamped to [0, LIM])
-  uint16_t* fw;      // [NT] first warp of each lane's range
-  uint16_t* fl;      // [NT] last warp of each lane's range
-  uint16_t* pb;      // [NT] first pool column of each lane
-  uint32_t* wsum;    // [8]
   uint64_t* mbar;    // [1]
   uint64_t* lhash;   // [LSLOTS]
   uint32_t* lowner;  // [LSLOTS]
@@ -108,11 +104,6 @@ __device__ __forceinline__ Smem carve(uint8_t* s, uint32_t pre, uint32_t P2) {
   size_t o = small_bytes(P2) <= pre ? 0 : pre + kCellBytes + kStageBytes;
   m.off = (uint64_t*)(s + o); o += kOffBytes;
   m.rel = (uint32_t*)(s + o); o += kRelBytes;
-  m.fw = (uint16_t*)(s + o);
-  m.fl = m.fw + NT;
-  m.pb = m.fl + NT;
-  o += kLaneBytes;
-  m.wsum = (uint32_t*)(s + o); o += 32;
   m.mbar = (uint64_t*)(s + o); o += 16;
   m.lhash = (uint64_t*)(s + o);
   m.lowner = (uint32_t*)(m.lhash + LSLOTS);
@@ -171,7 +162,7 @@ __device__ void report_bad_event(const Args& a, uint64_t s, uint64_t e) {
 
 // ---- item finalisation: CTA de-duplication and per-item entries ------------------------------------------------
 // Each thread holds its warp's key p (registers).  A slot owner publishes its key in its slot-0 column of `cells`
-// (zero at this point) so pending claimers can verify it; owners clear their columns before returning.
+// (overwritten; the next chunk's bulk clear resets the cells) so pending claimers can verify it.
 __device__ void item_group(const Args& a, const Smem& m, uint64_t t, uint64_t w0, bool valid, uint32_t k,
                            const uint32_t* p) {
   const int tid = threadIdx.x, lane = tid & 31;
@@ -186,16 +177,15 @@ __device__ void item_group(const Args& a, const Smem& m, uint64_t t, uint64_t w0
   const bool is_leader = valid && (lane == leader || !eq);
   const uint32_t cnt = (lane == leader) ? (uint32_t)__popc(peers & eqm & active) : 1u;
   int slot = -1;
-  bool pending = false, owner = false;
+  bool pending = false;
   if (is_leader) {
     uint32_t i = (uint32_t)(h & (LSLOTS - 1));
-    for (int probe = 0; probe < LSLOTS; ++probe) {
+    for (int probe = 0; probe < LPROBE; ++probe) {
       unsigned long long cur = atomicCAS((unsigned long long*)&m.lhash[i], 0ull, (unsigned long long)h);
       if (cur == 0ull) {
         m.lowner[i] = (uint32_t)tid;
         m.lent[i] = atomicAdd(&m.misc[0], 1u);
         slot = (int)i;
-        owner = true;
 #pragma unroll
         for (int j = 0; j < 16; ++j) m.cells[j * ROW + tid] = p[j];
         m.kid[tid] = k;
@@ -223,6 +213,8 @@ __device__ void item_group(const Args& a, const Smem& m, uint64_t t, uint64_t w0
     } else {
       my_ent = atomicAdd(&m.misc[0], 1u) | 0x80000000u;  // equal hash, different key: an entry of its own
     }
+  } else if (is_leader) {
+    my_ent = atomicAdd(&m.misc[0], 1u) | 0x80000000u;  // no free slot within LPROBE probes: an entry of its own
   }
   __syncthreads();
   const uint32_t n_ent = m.misc[0];
@@ -279,23 +271,20 @@ __device__ void item_group(const Args& a, const Smem& m, uint64_t t, uint64_t w0
     m.lcount[i] = 0u;
     m.lminw[i] = UINT32_MAX;
   }
-  if (owner) {
-#pragma unroll
-    for (int j = 0; j < 16; ++j) m.cells[j * ROW + tid] = 0u;
-  }
   if (tid == 0) m.misc[0] = 0u;
 }
 
-// column (byte offset in cells) of piece s of lane t: slot 0 = the lane's own column, s >= 1 = pool
-__device__ __forceinline__ uint32_t colof(uint32_t t, uint32_t pbt, uint32_t s) {
-  return s == 0 ? t * 4u : (uint32_t)(NT + pbt + s - 1) * 4u;
+// column (byte offset in cells) of warp u's piece in lane t: the lane's first warp fw goes to the lane's own
+// slot-0 column, a warp starting inside the lane's range to the pool column of its index (<= 256 warps per item)
+__device__ __forceinline__ uint32_t colof(uint32_t t, uint32_t fw, uint32_t u) {
+  return u == fw ? t * 4u : (uint32_t)(NT + u) * 4u;
 }
 
 template <bool CHECK_MARK>
 __global__ void __launch_bounds__(NT, 2) k_bbv2(Args a) {
   extern __shared__ __align__(128) uint8_t smem_raw[];
   Smem m = carve(smem_raw, a.pre, a.P2);
-  const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
+  const int tid = threadIdx.x;
   const uint32_t bmask = a.P2 - 1, mask4 = bmask << 2;
   const bool fused = a.te.tile_n != nullptr;
   const uint32_t cbase = smem_u32(m.cells);
@@ -406,40 +395,41 @@ __global__ void __launch_bounds__(NT, 2) k_bbv2(Args a) {
       const uint32_t nwd = (c.hi + 7) >> 3;
       const uint32_t Q = (((nwd + NT - 1) / NT) | 1u);
       const uint32_t L = Q * 8u;
+      // x / L == umulhi(x >> 3, ceil(2^32 / Q)) for x < 2^20
+      const uint32_t qinv = Q == 3u ? 0x55555556u : Q == 5u ? 0x33333334u : Q == 7u ? 0x24924925u : 0x1C71C71Du;
+      auto divL = [&](uint32_t x) -> uint32_t { return Q == 1u ? (x >> 3) : __umulhi(x >> 3, qinv); };
       const uint32_t LIM = CHE + 16u;
       auto relx = [&](uint64_t x) -> uint32_t { return x <= c.a8 ? 0u : (x - c.a8 >= LIM ? LIM : (uint32_t)(x - c.a8)); };
-      // [A] chunk-relative warp starts; lanes' first / last warps (scatter from the warps)
+      // [A] chunk-relative warp starts; the previous chunk's (or item's) cells cleared with 16-byte stores
       for (uint32_t u = tid; u < nw + 4; u += NT) m.rel[u] = relx(m.off[u]);
+#pragma unroll
+      for (int i = 0; i < (int)(kCellBytes / 16 / NT); ++i) ((uint4*)m.cells)[i * NT + tid] = make_uint4(0u, 0u, 0u, 0u);
       __syncthreads();
-      const uint32_t nact = (c.hi + L - 1) / L;  // lanes with events
-      const uint32_t tl = nact - 1;
-      if ((uint32_t)tid < nw) {
-        const uint32_t x0 = umax(m.rel[tid], c.lo), x1 = umin(m.rel[tid + 1], c.hi);
-        if (x0 < x1) {
-          if (x0 == c.lo) m.fw[0] = (uint16_t)tid;
-          for (uint32_t u = umax((x0 + L - 1) / L, 1u); u < (x1 + L - 1) / L && u < nact; ++u) m.fw[u] = (uint16_t)tid;
-          for (uint32_t u = (x0 + L) / L - 1; u < (x1 + L) / L - 1 && u < tl; ++u) m.fl[u] = (uint16_t)tid;
-          if (x1 == c.hi) m.fl[tl] = (uint16_t)tid;
-        }
-      }
-      __syncthreads();
-      // [B] pool bases: exclusive scan of (pieces - 1) over the lanes
+      const uint32_t nact = divL(c.hi + L - 1);  // lanes with events
+      // [B] my lane's first warp: the last warp starting at or before my first event (empty warps start where the
+      // next one does, so the search lands on the non-empty one); a proportional guess, then a search
       const bool act = (uint32_t)tid < nact;
-      const uint32_t myfw = act ? m.fw[tid] : 0u;
-      const uint32_t extra = act ? (uint32_t)m.fl[tid] - myfw : 0u;
-      uint32_t xs = extra;
+      uint32_t myfw = 0;
+      if (act) {
+        const uint32_t r = umax((uint32_t)tid * L, c.lo);
+        uint32_t lo = 0, hi = nw - 1;
+        uint32_t g = umin((uint32_t)((float)r * ((float)nw / (float)c.hi)), nw - 1);
 #pragma unroll
-      for (int o = 1; o < 32; o <<= 1) {
-        const uint32_t y = __shfl_up_sync(0xffffffffu, xs, o);
-        if (lane >= o) xs += y;
+        for (int step = 0; step < 3; ++step) {
+          if (m.rel[g] > r && g > 0) --g;
+          else if (g + 1 < nw && m.rel[g + 1] <= r) ++g;
+        }
+        if (m.rel[g] <= r && (g + 1 == nw || m.rel[g + 1] > r)) {
+          lo = g;
+        } else {
+          while (lo < hi) {
+            const uint32_t mid = (lo + hi + 1) >> 1;
+            if (m.rel[mid] <= r) lo = mid; else hi = mid - 1;
+          }
+        }
+        myfw = lo;
       }
-      if (lane == 31) m.wsum[wid] = xs;
       if (tid == 0 && !staged) stage_chunk(a, m, c, E8);  // not prefetched (the previous item had no events)
-      __syncthreads();
-      uint32_t pbt = xs - extra;
-#pragma unroll
-      for (int q = 0; q < NT / 32 - 1; ++q) pbt += q < wid ? m.wsum[q] : 0u;
-      if (act) m.pb[tid] = (uint16_t)pbt;
       // [C] accumulate my lane range
       mbar_wait(m.mbar, phase);
       phase ^= 1u;
@@ -447,9 +437,9 @@ __global__ void __launch_bounds__(NT, 2) k_bbv2(Args a) {
         const uint32_t t0 = (uint32_t)tid;
         const uint32_t r = umax(t0 * L, c.lo), e = umin((t0 + 1) * L, c.hi);
         const uint4* sb4 = (const uint4*)m.stage + t0 * Q;
-        uint32_t u = myfw, s = 0;
+        uint32_t u = myfw;
         uint32_t nb = m.rel[u + 1], nb2 = m.rel[u + 2];
-        uint32_t col = cbase + colof(t0, pbt, 0), coln = cbase + colof(t0, pbt, 1);
+        uint32_t col = cbase + t0 * 4u, coln = cbase + (NT + u + 1) * 4u;
         for (uint32_t k = 0; k < Q; ++k) {
           const uint32_t p0 = (t0 * Q + k) * 8u;
           if (p0 >= e) break;
@@ -465,16 +455,15 @@ __global__ void __launch_bounds__(NT, 2) k_bbv2(Args a) {
           tv[6] = *(const uint32_t*)(tb8 + ((v.w << 2) & mask4));
           tv[7] = *(const uint32_t*)(tb8 + ((v.w >> 14) & mask4));
           if (CHECK_MARK) orr |= (tv[0] | tv[1] | tv[2] | tv[3]) | (tv[4] | tv[5] | tv[6] | tv[7]);
-          const bool fast = p0 >= r && p0 + 8u <= e && (nb >= p0 + 8u || nb2 >= p0 + 8u);
+          const bool fast = p0 >= r && p0 + 8u <= e && nb2 >= p0 + 8u;  // nb2 >= nb: at most one boundary
           if (fast) {
             const uint32_t mcut = nb - p0;  // events j >= mcut belong to the next warp
 #pragma unroll
             for (int j = 0; j < 8; ++j) red_add(((uint32_t)j < mcut ? col : coln) | (tv[j] & TOFF), tv[j] >> TSH);
             if (nb <= p0 + 8u) {  // crossed into the next warp
               ++u;
-              ++s;
               col = coln;
-              coln = cbase + colof(t0, pbt, s + 1);
+              coln += 4u;
               nb = nb2;
               nb2 = m.rel[u + 2];
             }
@@ -486,18 +475,16 @@ __global__ void __launch_bounds__(NT, 2) k_bbv2(Args a) {
               if (pos < r || pos >= e) continue;
               while (pos >= nb && u < nw) {
                 ++u;
-                ++s;
                 nb = m.rel[u + 1];
               }
-              red_add((cbase + colof(t0, pbt, s)) | (tv[j] & TOFF), tv[j] >> TSH);
+              red_add((cbase + colof(t0, myfw, u)) | (tv[j] & TOFF), tv[j] >> TSH);
             }
             while (p0 + 8u < e && nb <= p0 + 8u && u < nw) {  // the next word starts in a later warp
               ++u;
-              ++s;
               nb = m.rel[u + 1];
             }
-            col = cbase + colof(t0, pbt, s);
-            coln = cbase + colof(t0, pbt, s + 1);
+            col = cbase + colof(t0, myfw, u);
+            coln = cbase + (NT + u + 1) * 4u;
             nb2 = m.rel[u + 2];
           }
         }
@@ -516,29 +503,28 @@ __global__ void __launch_bounds__(NT, 2) k_bbv2(Args a) {
         }
       }
       // [D] each warp with events in this chunk sums its pieces (its owner column in the lane holding its first
-      // event here, then slot 0 of each later lane it spans) into its key registers, clearing them
+      // event here, then slot 0 of each later lane it spans) into its key registers
       if (valid) {
         const uint32_t x0 = umax(m.rel[tid], c.lo), x1 = umin(m.rel[tid + 1], c.hi);
         if (x0 < x1) {
-          const uint32_t ta = x0 / L, tb = (x1 - 1) / L;
-          uint32_t oc = colof(ta, m.pb[ta], (uint32_t)tid - m.fw[ta]) >> 2;
-          uint32_t csum = 0;  // < 2^31: a chunk holds <= CHE events of length < 2^17
+          const uint32_t ta = divL(x0), tb = divL(x1 - 1);
+          // owner column: slot 0 of lane ta when the warp is that lane's first piece, else the warp's pool column
+          uint32_t oc = x0 == umax(ta * L, c.lo) ? ta : NT + (uint32_t)tid;
           for (uint32_t tt = ta;;) {
 #pragma unroll
-            for (int j = 0; j < 16; ++j) {
-              const uint32_t x = m.cells[j * ROW + oc];
-              m.cells[j * ROW + oc] = 0u;
-              p[j] += x;
-              csum += x;
-            }
+            for (int j = 0; j < 16; ++j) p[j] += m.cells[j * ROW + oc];
             if (++tt > tb) break;
             oc = tt;
           }
-          I += csum;
+          // the chunk added < 2^31 (<= CHE events of length < 2^17): the exact u64 total follows from the u32 sum
+          uint32_t sum = 0;
+#pragma unroll
+          for (int j = 0; j < 16; ++j) sum += p[j];
+          I += (uint32_t)(sum - (uint32_t)I);
         }
       }
       cs = ce;
-      __syncthreads();  // columns clear; rel / fw / fl / pb free for the next chunk
+      __syncthreads();  // pieces read; rel / fw / pb free for the next chunk
     }
 
     // ---- finalise the item ----
