@@ -92,7 +92,8 @@ struct Smem {
   uint32_t* lcount;  // [LSLOTS]
   uint32_t* lminw;   // [LSLOTS]
   uint32_t* lent;    // [LSLOTS]
-  uint32_t* misc;    // [64]: 0 n_entries, [2..3] u64 overflow base, [8..9] schedule
+  uint32_t* misc;    // [64]: 0 n_entries, [2..3] next free overflow entry of the CTA's block, [4..5] its end,
+                     // [6..7] the current item's overflow base, [8..9] schedule
   uint32_t* kid;     // [NT]
   uint32_t* tbl;     // [P2]
 };
@@ -172,7 +173,7 @@ __device__ void item_group(const Args& a, const Smem& m, uint64_t t, uint64_t w0
   const int leader = __ffs(peers) - 1;
   bool eq = (__shfl_sync(0xffffffffu, k, leader) == k);
 #pragma unroll
-  for (int j = 0; j < 16; ++j) eq = eq && (__shfl_sync(0xffffffffu, p[j], leader) == p[j]);
+  for (int j = 0; j < 16; ++j) eq &= (__shfl_sync(0xffffffffu, p[j], leader) == p[j]);  // no short circuit
   const unsigned eqm = __ballot_sync(0xffffffffu, eq);
   const bool is_leader = valid && (lane == leader || !eq);
   const uint32_t cnt = (lane == leader) ? (uint32_t)__popc(peers & eqm & active) : 1u;
@@ -203,7 +204,7 @@ __device__ void item_group(const Args& a, const Smem& m, uint64_t t, uint64_t w0
       const uint32_t o = m.lowner[slot];
       bool same = (m.kid[o] == k);
 #pragma unroll
-      for (int j = 0; j < 16; ++j) same = same && (m.cells[j * ROW + o] == p[j]);
+      for (int j = 0; j < 16; ++j) same &= (m.cells[j * ROW + o] == p[j]);  // independent loads
       own = same;
     }
     if (own) {
@@ -220,22 +221,34 @@ __device__ void item_group(const Args& a, const Smem& m, uint64_t t, uint64_t w0
   const uint32_t n_ent = m.misc[0];
   const uint32_t M = a.te.per_tile;
   uint64_t* ovf_base = (uint64_t*)(m.misc + 2);
-  if (n_ent > M) {  // more distinct keys than the item's fixed entry slots
+  if (n_ent > M) {  // more distinct keys than the item's fixed entry slots: overflow entries from the CTA's block
     if (tid == 0) {
-      unsigned long long pos = atomicAdd((unsigned long long*)a.te.ovf_count, (unsigned long long)(n_ent - M));
-      if (pos + (n_ent - M) > a.te.ovf_cap) latch(a.err, PHOTON_ECAPACITY, (int64_t)pos);
+      uint64_t* ovf_end = (uint64_t*)(m.misc + 4);
+      const uint64_t need = n_ent - M;
+      uint64_t pos = *ovf_base;
+      if (pos + need > *ovf_end) {  // refill (rare): a block of at least 256 entries; the old block's unused tail
+                                     // is marked empty (count 0, skipped by the insertion)
+        for (uint64_t j = pos; j < umin64(*ovf_end, a.te.ovf_cap); ++j) a.te.ovf[j].count = 0u;
+        const uint64_t blk = need > 256 ? need : 256;
+        pos = atomicAdd((unsigned long long*)a.te.ovf_count, (unsigned long long)blk);
+        if (pos + need > a.te.ovf_cap) latch(a.err, PHOTON_ECAPACITY, (int64_t)pos);
+        *ovf_end = pos + blk;
+      }
       a.te.tile_ovf[t] = pos;
-      *ovf_base = pos;
+      m.misc[6] = (uint32_t)pos;  // this item's base (low word; the high word below)
+      m.misc[7] = (uint32_t)(pos >> 32);
+      *ovf_base = pos + need;
     }
     __syncthreads();
   }
+  const uint64_t obase = ((uint64_t)m.misc[7] << 32) | m.misc[6];
   if (tid == 0) a.te.tile_n[t] = n_ent;
   auto put = [&](uint32_t e, uint32_t kern, const uint32_t* key, uint32_t count, uint32_t minw, uint64_t hh) {
     TileEntry* dst;
     if (e < M) {
       dst = a.te.ent + t * M + e;
     } else {
-      uint64_t pos = *ovf_base + (e - M);
+      uint64_t pos = obase + (e - M);
       if (pos >= a.te.ovf_cap) return;
       dst = a.te.ovf + pos;
     }
@@ -263,7 +276,7 @@ __device__ void item_group(const Args& a, const Smem& m, uint64_t t, uint64_t w0
   const uint32_t from_leader = __shfl_sync(0xffffffffu, my_ent, leader);
   if (valid) {
     const uint32_t e = ((lane == leader || !eq) ? my_ent : from_leader) & 0x7FFFFFFFu;
-    a.te.gid[w0 + tid] = e < M ? (uint32_t)(t * M + e) : (0x80000000u | (uint32_t)(*ovf_base + (e - M)));
+    a.te.gid[w0 + tid] = e < M ? (uint32_t)(t * M + e) : (0x80000000u | (uint32_t)(obase + (e - M)));
   }
   __syncthreads();
   for (int i = tid; i < LSLOTS; i += NT) {
@@ -360,13 +373,22 @@ __global__ void __launch_bounds__(NT, 2) k_bbv2(Args a) {
     uint32_t nx_k = 0;
     uint32_t x_after = 0;
     if (tid == 0 && tn < NI) x_after = atomicAdd(a.counter, 1u);
+    // the next item's warp range is loaded now; the dependent offset loads are issued once it has surely arrived
+    // (before the first chunk's event loop), so no warp waits on the two-step chain
+    uint64_t nr0 = 0, nr1 = 0;
+    bool nx_issued = !(tn < NI);
     if (tn < NI) {
-      uint64_t n0, n1;
-      item_range(a, tn, n0, n1);
-      nx_off = a.weo[n0 + umin64((uint64_t)tid, n1 - n0)];
-      if (tid == 0) nx_last = a.weo[n1];
+      nr0 = a.item_w0[tn];
+      nr1 = a.item_w0[tn + 1];
       if (fused) nx_k = a.tile_k0[tn];
     }
+    auto issue_next = [&]() {
+      if (nx_issued) return;
+      nx_issued = true;
+      const uint64_t n0 = umin64(nr0, a.W), n1 = umin64(umin64(umax64(nr1, n0), n0 + NT), a.W);
+      nx_off = a.weo[n0 + umin64((uint64_t)tid, n1 - n0)];
+      if (tid == 0) nx_last = a.weo[n1];
+    };
     __syncthreads();
     // item bounds; non-monotone offsets are latched and made monotone (memory safety of the lane walks)
     const uint64_t te = umin64(m.off[nw], a.E), ts = umin64(m.off[0], te);
@@ -430,6 +452,7 @@ __global__ void __launch_bounds__(NT, 2) k_bbv2(Args a) {
         myfw = lo;
       }
       if (tid == 0 && !staged) stage_chunk(a, m, c, E8);  // not prefetched (the previous item had no events)
+      issue_next();
       // [C] accumulate my lane range
       mbar_wait(m.mbar, phase);
       phase ^= 1u;
@@ -528,6 +551,7 @@ __global__ void __launch_bounds__(NT, 2) k_bbv2(Args a) {
     }
 
     // ---- finalise the item ----
+    issue_next();  // items without events
     const uint64_t s = m.off[tid <= (int)nw ? tid : nw], e = m.off[tid < (int)nw ? tid + 1 : nw];
     const int bad_here = ((((raw | (raw >> 16)) & 0xFFFFu) & ~bmask) != 0u || (CHECK_MARK && (orr & 1u))) ? 1 : 0;
     if (__syncthreads_or(bad_here)) {
@@ -562,6 +586,11 @@ __global__ void __launch_bounds__(NT, 2) k_bbv2(Args a) {
     __syncthreads();
     t = tn;
     tn = sched[1];
+  }
+  // the unused rest of the CTA's overflow block: count 0 marks an entry the insertion skips
+  if (fused) {
+    const uint64_t nxt = *(const uint64_t*)(m.misc + 2), end = umin64(*(const uint64_t*)(m.misc + 4), a.te.ovf_cap);
+    for (uint64_t j = nxt + tid; j < end; j += NT) a.te.ovf[j].count = 0u;
   }
 }
 

@@ -317,6 +317,10 @@ __global__ void k_entries_insert(TileEntries te, uint64_t n_tiles, HashTable ht,
     const uint64_t stride = (uint64_t)gridDim.x * blockDim.x - nfix;
     for (uint64_t j = i - nfix; j < n; j += stride) {
       x = te.ovf + j;
+      if (x->count == 0u) {  // reserved by K1 but unused (no warp refers to it)
+        te.ovf_slot[j] = UINT32_MAX;
+        continue;
+      }
       uint32_t key[16];
       const uint4* kp = (const uint4*)x->key;
 #pragma unroll
