@@ -249,7 +249,7 @@ def run_photon(args):
     k1_ms = pms[0] / max(int(pcnt[0]), 1)
     k1_bytes = 2 * tr.n_events + 8 * (tr.n_warps + 1) + 4 * tr.n_warps  # algorithmic: bb + offsets + warp type
     achieved = k1_bytes / (k1_ms / 1000) / 1e9
-    roofline = {"bound": "hbm", "kernel": "k_bbv (fused A1+A2 streaming pass)", "achieved": achieved,
+    roofline = {"bound": "hbm", "kernel": "k_bbv2 (fused A1+A2 streaming pass)", "achieved": achieved,
                 "peak": hbm_peak, "peak_source": peak_src, "unit": "GB/s", "frac": achieved / hbm_peak,
                 "traffic": _traffic(args.config), "algorithmic_bytes_per_launch": k1_bytes,
                 "k1_ms": k1_ms, "k1_share_of_step": (pms[0] / args.steps) / ms if ms else None,
