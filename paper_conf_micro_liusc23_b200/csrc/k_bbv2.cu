@@ -118,8 +118,10 @@ __device__ __forceinline__ Smem carve(uint8_t* s, uint32_t pre, uint32_t P2) {
   return m;
 }
 
+// No "memory" clobber: the cells are only written by these adds and only read after a __syncthreads(), so the
+// compiler may move the (read-only) stage and table loads across them, which the event loop relies on.
 __device__ __forceinline__ void red_add(uint32_t saddr, uint32_t v) {
-  asm volatile("red.shared.add.u32 [%0], %1;" ::"r"(saddr), "r"(v) : "memory");
+  asm volatile("red.shared.add.u32 [%0], %1;" ::"r"(saddr), "r"(v));
 }
 
 // warps [w0, w1) of item it (clamped: malformed offsets stay memory-safe; they are latched by k_items_fill)
@@ -463,12 +465,8 @@ __global__ void __launch_bounds__(NT, 2) k_bbv2(Args a) {
         uint32_t u = myfw;
         uint32_t nb = m.rel[u + 1], nb2 = m.rel[u + 2];
         uint32_t col = cbase + t0 * 4u, coln = cbase + (NT + u + 1) * 4u;
-        for (uint32_t k = 0; k < Q; ++k) {
-          const uint32_t p0 = (t0 * Q + k) * 8u;
-          if (p0 >= e) break;
-          const uint4 v = sb4[k];
-          raw |= v.x | v.y | v.z | v.w;
-          uint32_t tv[8];
+        const uint32_t kn = umin(Q, (e - t0 * L + 7u) >> 3);  // words holding my events
+        auto lookup = [&](const uint4& v, uint32_t (&tv)[8]) {
           tv[0] = *(const uint32_t*)(tb8 + ((v.x << 2) & mask4));
           tv[1] = *(const uint32_t*)(tb8 + ((v.x >> 14) & mask4));
           tv[2] = *(const uint32_t*)(tb8 + ((v.y << 2) & mask4));
@@ -477,6 +475,15 @@ __global__ void __launch_bounds__(NT, 2) k_bbv2(Args a) {
           tv[5] = *(const uint32_t*)(tb8 + ((v.z >> 14) & mask4));
           tv[6] = *(const uint32_t*)(tb8 + ((v.w << 2) & mask4));
           tv[7] = *(const uint32_t*)(tb8 + ((v.w >> 14) & mask4));
+        };
+        // software pipeline: word k+1 is loaded (stage, then table) while word k's adds are issued
+        uint4 vnx = sb4[0];
+        uint32_t tv[8];
+        lookup(vnx, tv);
+        for (uint32_t k = 0; k < kn; ++k) {
+          const uint32_t p0 = (t0 * Q + k) * 8u;
+          raw |= (vnx.x | vnx.y) | (vnx.z | vnx.w);
+          vnx = sb4[k + 1 < kn ? k + 1 : k];
           if (CHECK_MARK) orr |= (tv[0] | tv[1] | tv[2] | tv[3]) | (tv[4] | tv[5] | tv[6] | tv[7]);
           const bool fast = p0 >= r && p0 + 8u <= e && nb2 >= p0 + 8u;  // nb2 >= nb: at most one boundary
           if (fast) {
@@ -510,6 +517,7 @@ __global__ void __launch_bounds__(NT, 2) k_bbv2(Args a) {
             coln = cbase + (NT + u + 1) * 4u;
             nb2 = m.rel[u + 2];
           }
+          lookup(vnx, tv);
         }
       }
       __syncthreads();  // pieces complete; the stage is free
