@@ -264,6 +264,37 @@ PHOTON_API int photon_bb_predict(photon_ctx *ctx, const photon_trace *trace, con
                                  const uint64_t *stable_dur_sum /*[K][B]*/, void *ws, size_t ws_bytes,
                                  uint64_t *pred_dur_sum /*[W]*/, uint32_t *unpredicted /*[W]*/, void *stream);
 
+/* ---- N4: persisted signature pool, offline reuse of the analysis (L402, §6.3 "Online/Offline Tradeoff") -------
+ * "All data that is generated by the online analysis ... is micro-architecture agnostic.  Hardware researchers can
+ * reuse these data" (L402).  Reading [N4-a]: a pool holds the REPRESENTATIVE kernels (match[k] < 0) of one or more
+ * earlier runs -- their canonical type rows and launched warp counts -- in launch order; a later run is matched as
+ * if the pool's kernels had been launched before its own kernels (the A4 rule above, unchanged), so one of its
+ * kernels that is close to a pooled representative reuses that representative's simulation.
+ * photon_pool_export: pool <- the representatives of a run (K kernels, types as from photon_warp_group, match as
+ *   from photon_kernel_match).  pool->kernel_type_off needs K+1 entries, type_key/type_count pool->capacity rows
+ *   (>= the run's total types suffices); warp_type, type_first_warp and warp_sampling_ok of `pool` are unused (may
+ *   be NULL).  pool_warps_total [K], pool_kernel_id [K] (the run's index of each pooled kernel) and *n_pool (DEVICE
+ *   u32: pooled kernels) are written; ws >= photon_pool_export_workspace_bytes(K).  No device errors.
+ * photon_kernel_match_pooled: match[] / match_dist[] over the combined index space [0, Kp + K): indices < Kp are
+ *   the pool's kernels (in pool order), Kp + k is this run's kernel k; params and semantics as photon_kernel_match
+ *   (a pooled kernel is never matched to a later one; reading [P-8] applies to pool and run alike).  `pool` holds
+ *   Kp kernels and Tp_bound >= its total types, `types` the run's K kernels and T_bound >= their total; ws >=
+ *   photon_pool_match_workspace_bytes(Kp, Tp_bound, K, T_bound, 0).  Device errors as photon_kernel_match. */
+PHOTON_API size_t photon_pool_export_workspace_bytes(uint32_t n_kernels);
+PHOTON_API int photon_pool_export(photon_ctx *ctx, uint32_t n_kernels, const photon_types *types,
+                                  const uint64_t *warps_total /*[K]*/, const int64_t *match /*[K]*/, void *ws,
+                                  size_t ws_bytes, photon_types *pool, uint64_t *pool_warps_total /*[K]*/,
+                                  uint32_t *pool_kernel_id /*[K]*/, uint32_t *n_pool /*DEVICE [1]*/, void *stream);
+PHOTON_API size_t photon_pool_match_workspace_bytes(uint32_t n_pool, uint64_t pool_types_bound, uint32_t n_kernels,
+                                                    uint64_t types_bound, uint64_t pair_capacity);
+PHOTON_API int photon_kernel_match_pooled(photon_ctx *ctx, uint32_t n_pool, const photon_types *pool,
+                                          const uint64_t *pool_warps_total /*[Kp]*/, uint64_t pool_types_bound,
+                                          uint32_t n_kernels, const photon_types *types,
+                                          const uint64_t *warps_total /*[K]*/, uint64_t types_bound,
+                                          photon_match_params params, void *ws, size_t ws_bytes,
+                                          int64_t *match /*[Kp+K]*/, double *match_dist /*[Kp+K] or NULL*/,
+                                          void *stream);
+
 /* ---- Multi-GPU merge helpers ------------------------------------------------------------------
  * A shard is a contiguous warp range of the global trace; its local kernel l is global kernel kernel_base + l and
  * its local warp v is global warp warp_base + v.  Rows exchanged between ranks (88 bytes each):       */

@@ -204,6 +204,40 @@ def bb_predict(trace, first_stable, stable_dur_sum):
     return pd[:W], un[:W]
 
 
+def pool_export(types, warps_total, match_):
+    """N4 (L402, reading [N4-a]): the run's representative kernels (match < 0), in launch order: dict(n_pool,
+    kernel_type_off, type_key, type_count, warps_total, kernel_id)."""
+    kto = np.asarray(types["kernel_type_off"], np.uint64)
+    reps = [k for k in range(len(kto) - 1) if int(match_[k]) < 0]
+    off, keys, cnts = [0], [], []
+    for k in reps:
+        a, b = int(kto[k]), int(kto[k + 1])
+        keys.append(np.asarray(types["type_key"], np.uint32).reshape(-1, 16)[a:b])
+        cnts.append(np.asarray(types["type_count"], np.uint64)[a:b])
+        off.append(off[-1] + (b - a))
+    return dict(n_pool=len(reps), kernel_type_off=np.array(off, np.uint64),
+                type_key=np.concatenate(keys) if keys else np.zeros((0, 16), np.uint32),
+                type_count=np.concatenate(cnts) if cnts else np.zeros(0, np.uint64),
+                warps_total=np.array([int(warps_total[k]) for k in reps], np.uint64),
+                kernel_id=np.array(reps, np.uint32))
+
+
+def match_pooled(pool, types, warps_total, theta=(1, 20), n_cores=64, pool_all_prior=0):
+    """N4: A4 with the pool's kernels launched before the run's (reading [N4-a]); indices < n_pool are pooled."""
+    kto = np.asarray(types["kernel_type_off"], np.uint64)
+    K, T = len(kto) - 1, int(kto[-1])
+    pk = np.asarray(pool["kernel_type_off"], np.uint64)
+    Tp = int(pk[-1])
+    comb_kto = np.concatenate([pk, Tp + kto[1:]])
+    keys = np.concatenate([np.asarray(pool["type_key"], np.uint32).reshape(-1, 16)[:Tp],
+                           np.asarray(types["type_key"], np.uint32).reshape(-1, 16)[:T]])
+    cnts = np.concatenate([np.asarray(pool["type_count"], np.uint64)[:Tp],
+                           np.asarray(types["type_count"], np.uint64)[:T]])
+    sig, mass = signature(comb_kto, keys, cnts)
+    wt = np.concatenate([np.asarray(pool["warps_total"], np.uint64), np.asarray(warps_total, np.uint64)[:K]])
+    return match(comb_kto, sig, mass, wt, theta, n_cores, pool_all_prior)
+
+
 def analyse(trace, theta=(1, 20), n_cores=64, pool_all_prior=0):
     """The benchmarked chain A1 -> A2 -> A3 -> A4 on one trace; returns a dict of every output."""
     p16, ins, kbb = bbv(trace, want_kbb=False)

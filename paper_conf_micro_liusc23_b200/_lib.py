@@ -97,6 +97,13 @@ _SIGS = [
                                       c_size_t, c_void_p, c_void_p, c_void_p]),
     ("photon_bb_predict", c_int, [c_void_p, POINTER(Trace), c_void_p, c_void_p, c_void_p, c_size_t, c_void_p,
                                   c_void_p, c_void_p]),
+    ("photon_pool_export_workspace_bytes", c_size_t, [c_uint32]),
+    ("photon_pool_export", c_int, [c_void_p, c_uint32, POINTER(Types), c_void_p, c_void_p, c_void_p, c_size_t,
+                                   POINTER(Types), c_void_p, c_void_p, c_void_p, c_void_p]),
+    ("photon_pool_match_workspace_bytes", c_size_t, [c_uint32, c_uint64, c_uint32, c_uint64, c_uint64]),
+    ("photon_kernel_match_pooled", c_int, [c_void_p, c_uint32, POINTER(Types), c_void_p, c_uint64, c_uint32,
+                                           POINTER(Types), c_void_p, c_uint64, MatchParams, c_void_p, c_size_t,
+                                           c_void_p, c_void_p, c_void_p]),
     ("photon_types_export", c_int, [c_void_p, c_uint32, POINTER(Types), c_uint32, c_uint64, c_void_p, c_void_p]),
     ("photon_merge_workspace_bytes", c_size_t, [c_uint64, c_uint32]),
     ("photon_types_merge", c_int, [c_void_p, c_void_p, c_uint64, c_uint32, c_void_p, c_void_p, c_size_t,

@@ -269,6 +269,70 @@ class Photon:
                                            self.stream_ptr(stream)))
         return dict(filter_pairs=int(st[0]), close_pairs=int(st[1]), rounds=int(st[2]), pair_capacity=int(st[3]))
 
+    # -- N4: persisted signature pool (L402) -------------------------------------------------------------------
+    def photon_pool_export(self, n_kernels: int, ty: dict, warps_total, match, stream=None) -> dict:
+        """The representatives of a run (match < 0) as a pool: dict(n_pool, capacity, kernel_type_off, type_key,
+        type_count, warps_total, kernel_id) of device tensors.  Syncs once to read the pool's size."""
+        K = n_kernels
+        ws = self.workspace("pool", self.L.photon_pool_export_workspace_bytes(K))
+        pool = dict(capacity=ty["capacity"], kernel_type_off=self.empty(K + 1, "int64"),
+                    type_key=self.empty(16 * ty["capacity"], "int32"), type_count=self.empty(ty["capacity"], "int64"))
+        pwt, pkid, npool = self.empty(K, "int64"), self.empty(K, "int32"), self.empty(1, "int32")
+        pc = self.types_c(pool)
+        self._rc(self.L.photon_pool_export(self.ctx, K, ctypes.byref(self.types_c(ty)), warps_total.data_ptr(),
+                                           match.data_ptr(), ws.data_ptr(), ws.numel(), ctypes.byref(pc),
+                                           pwt.data_ptr(), pkid.data_ptr(), npool.data_ptr(),
+                                           self.stream_ptr(stream)))
+        self.torch.cuda.synchronize(self.device)
+        Kp = int(npool.item())
+        T = int(pool["kernel_type_off"][Kp].item())
+        return dict(n_pool=Kp, capacity=max(T, 1), kernel_type_off=pool["kernel_type_off"][:Kp + 1],
+                    type_key=pool["type_key"][:16 * max(T, 1)], type_count=pool["type_count"][:max(T, 1)],
+                    warps_total=pwt[:Kp], kernel_id=pkid[:Kp])
+
+    def photon_kernel_match_pooled(self, pool: dict, n_kernels: int, ty: dict, warps_total, theta=(1, 20),
+                                   n_cores=64, pool_all_prior=0, want_dist: bool = True, stream=None) -> dict:
+        """A4 against a pool (N4): match / match_dist over [0, Kp + K); index < Kp = a pooled kernel."""
+        Kp, K = pool["n_pool"], n_kernels
+        Tp, T = pool["capacity"], ty["capacity"]
+        cap = 1024
+        for _ in range(8):
+            nb = self.L.photon_pool_match_workspace_bytes(Kp, Tp, K, T, max(cap, 16 * (Kp + K) + 65536))
+            ws = self.workspace("pool_match", nb)
+            off = (self.L.photon_pool_match_workspace_bytes(Kp, Tp, K, T, 1024)
+                   - self.L.photon_match_workspace_bytes(Kp + K, Tp + T, 1024))
+            o = dict(match=self.empty(Kp + K, "int64"))
+            if want_dist:
+                o["match_dist"] = self.empty(Kp + K, "float64")
+            self._rc(self.L.photon_kernel_match_pooled(
+                self.ctx, Kp, ctypes.byref(self.types_c(pool)), pool["warps_total"].data_ptr() if Kp else None, Tp,
+                K, ctypes.byref(self.types_c(ty)), warps_total.data_ptr(), T,
+                self.match_params(theta, n_cores, pool_all_prior), ws.data_ptr(), ws.numel(), o["match"].data_ptr(),
+                o["match_dist"].data_ptr() if want_dist else None, self.stream_ptr(stream)))
+            rc, bad = self.ws_status(ws[off:], stream)
+            if rc == _lib.ECAPACITY:
+                cap *= 4
+                continue
+            if rc != 0:
+                raise PhotonError(rc, self.L.photon_last_error(self.ctx).decode(), bad)
+            return o
+        raise PhotonError(_lib.ECAPACITY, "pair table kept overflowing")
+
+    @staticmethod
+    def save_pool(pool: dict, path: str):
+        """Persist a pool (host .npz; the analysis data is micro-architecture agnostic, L402)."""
+        import numpy as np
+        np.savez(path, **{k: (v.cpu().numpy() if hasattr(v, "cpu") else np.asarray(v)) for k, v in pool.items()})
+
+    def load_pool(self, path: str) -> dict:
+        import numpy as np
+        z = np.load(path)
+        out = {}
+        for k in z.files:
+            v = z[k]
+            out[k] = int(v) if v.ndim == 0 else self.torch.from_numpy(v).to(self.device)
+        return out
+
     # split form (multi-GPU driver)
     def photon_sig_build(self, K, kto, type_key, type_count, k_lo, k_hi, sig, mass, stream=None):
         ws = self.workspace("sig", 256)

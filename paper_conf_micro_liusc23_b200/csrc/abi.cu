@@ -503,6 +503,86 @@ int photon_kernel_match(photon_ctx* ctx, uint32_t K, const photon_types* types, 
   return PHOTON_OK;
 }
 
+// ---- N4: persisted signature pool (k_pool.cu) ----------------------------------------------------------------
+size_t photon_pool_export_workspace_bytes(uint32_t K) {
+  Carver c(nullptr);
+  c.take<uint64_t>((size_t)K + 1);
+  c.take<uint64_t>((size_t)K + 1);
+  return c.off + 256;
+}
+
+int photon_pool_export(photon_ctx* ctx, uint32_t K, const photon_types* types, const uint64_t* warps_total,
+                       const int64_t* match, void* ws, size_t ws_bytes, photon_types* pool, uint64_t* pool_wt,
+                       uint32_t* pool_kid, uint32_t* n_pool, void* stream) {
+  if (!ctx) return PHOTON_EINVAL;
+  if (!types || !types->kernel_type_off || !types->type_key || !types->type_count || !warps_total || !match ||
+      !pool || !pool->kernel_type_off || !pool->type_key || !pool->type_count || !pool_wt || !pool_kid || !n_pool ||
+      !ws)
+    return fail(ctx, PHOTON_EINVAL, "NULL argument");
+  if (K == 0) return fail(ctx, PHOTON_EINVAL, "K must be >= 1");
+  if (ws_bytes < photon_pool_export_workspace_bytes(K))
+    return fail(ctx, PHOTON_EWORKSPACE, "workspace %zu < %zu bytes", ws_bytes, photon_pool_export_workspace_bytes(K));
+  Carver c(ws);
+  uint64_t* keep = c.take<uint64_t>((size_t)K + 1);
+  uint64_t* ntypes = c.take<uint64_t>((size_t)K + 1);
+  CK(cudaSetDevice(ctx->device), "cudaSetDevice");
+  CK(launch_pool_export(K, *types, warps_total, match, keep, ntypes, *pool, pool_wt, pool_kid, n_pool,
+                        (cudaStream_t)stream),
+     "pool_export");
+  return PHOTON_OK;
+}
+
+namespace {
+struct PoolLayout {
+  uint64_t* kto;
+  uint32_t* key;
+  uint64_t* cnt;
+  uint64_t* wt;
+  size_t off;  // start of the match workspace
+};
+PoolLayout pool_layout(uint32_t Kp, uint64_t Tp, uint32_t K, uint64_t T, void* base) {
+  Carver c(base);
+  PoolLayout p;
+  p.kto = c.take<uint64_t>((size_t)Kp + K + 1);
+  p.key = c.take<uint32_t>(16 * (Tp + T + 1));
+  p.cnt = c.take<uint64_t>(Tp + T + 1);
+  p.wt = c.take<uint64_t>((size_t)Kp + K + 1);
+  p.off = (c.off + 255) & ~(size_t)255;
+  return p;
+}
+}  // namespace
+
+size_t photon_pool_match_workspace_bytes(uint32_t Kp, uint64_t Tp, uint32_t K, uint64_t T, uint64_t pair_cap) {
+  return pool_layout(Kp, Tp, K, T, nullptr).off + match_layout(Kp + K, Tp + T, pair_cap, nullptr).bytes;
+}
+
+int photon_kernel_match_pooled(photon_ctx* ctx, uint32_t Kp, const photon_types* pool, const uint64_t* pool_wt,
+                               uint64_t Tp, uint32_t K, const photon_types* types, const uint64_t* warps_total,
+                               uint64_t T, photon_match_params params, void* ws, size_t ws_bytes, int64_t* match,
+                               double* match_dist, void* stream) {
+  if (!ctx) return PHOTON_EINVAL;
+  if (!pool || !pool->kernel_type_off || (Kp && (!pool->type_key || !pool->type_count || !pool_wt)) || !types ||
+      !types->kernel_type_off || !types->type_key || !types->type_count || !warps_total || !match || !ws)
+    return fail(ctx, PHOTON_EINVAL, "NULL argument");
+  if (K == 0) return fail(ctx, PHOTON_EINVAL, "K must be >= 1");
+  if ((uint64_t)Kp + K >= (1ull << 32)) return fail(ctx, PHOTON_EINVAL, "Kp + K too large");
+  const PoolLayout p = pool_layout(Kp, Tp, K, T, ws);
+  if (ws_bytes < photon_pool_match_workspace_bytes(Kp, Tp, K, T, 1024))
+    return fail(ctx, PHOTON_EWORKSPACE, "workspace %zu < %zu bytes", ws_bytes,
+                photon_pool_match_workspace_bytes(Kp, Tp, K, T, 1024));
+  CK(cudaSetDevice(ctx->device), "cudaSetDevice");
+  CK(launch_pool_concat(Kp, *pool, pool_wt, K, *types, warps_total, p.kto, p.key, p.cnt, p.wt, Tp + T,
+                        ctx->num_sms, (cudaStream_t)stream),
+     "pool_concat");
+  photon_types comb{};
+  comb.capacity = Tp + T;
+  comb.kernel_type_off = p.kto;
+  comb.type_key = p.key;
+  comb.type_count = p.cnt;
+  return photon_kernel_match(ctx, Kp + K, &comb, p.wt, params, (uint8_t*)ws + p.off, ws_bytes - p.off, match,
+                             match_dist, stream);
+}
+
 int photon_match_stats(photon_ctx* ctx, uint32_t K, uint64_t T, const void* ws, size_t ws_bytes, uint64_t* stats,
                        void* stream) {
   if (!ctx || !ws || !stats) return PHOTON_EINVAL;

@@ -146,6 +146,13 @@ size_t warp_stable_ws_bytes(uint32_t K, uint64_t R);
 cudaError_t launch_warp_stable(const photon_timing& t, const uint8_t* ok, uint32_t n, uint32_t dnum, uint32_t dden,
                                void* ws, int64_t* switch_at, uint64_t* dur, DevErr* err, int num_sms,
                                cudaStream_t s);
+// ---- N4 (k_pool.cu): persisted signature pool --------------------------------------------------------------
+cudaError_t launch_pool_export(uint32_t K, const photon_types& ty, const uint64_t* wt, const int64_t* match,
+                               uint64_t* keep, uint64_t* ntypes, const photon_types& pool, uint64_t* pwt,
+                               uint32_t* pkid, uint32_t* n_pool, cudaStream_t s);
+cudaError_t launch_pool_concat(uint32_t Kp, const photon_types& pool, const uint64_t* pwt, uint32_t K,
+                               const photon_types& ty, const uint64_t* wt, uint64_t* okto, uint32_t* okey,
+                               uint64_t* ocnt, uint64_t* owt, uint64_t T_bound, int num_sms, cudaStream_t s);
 // ---- N3 (k_predict.cu) --------------------------------------------------------------------------------------
 cudaError_t launch_kernel_predict(uint32_t K, const int64_t* match, const uint64_t* mass, const uint64_t* full_insts,
                                   const uint64_t* full_cycles, uint64_t* pred_insts, uint64_t* pred_cycles,

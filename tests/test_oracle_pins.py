@@ -664,3 +664,52 @@ def test_bb_predict_worked_example_and_invariants():
         miss = sum(int(execs[b]) for b in range(tr6.n_bb) if fs[k, b] < 0)
         assert sum(int(x) for x in pd[kwo[k]:kwo[k + 1]]) == want
         assert int(un[kwo[k]:kwo[k + 1]].sum()) == miss
+
+
+# N4: persisted signature pool (L402, reading [N4-a]).  Pins: a run matched against its own pool has no
+# representative left and each of its representatives reuses its own pooled copy at distance 0; the pooled
+# decisions for run B equal an independent Fraction brute force over A's representatives followed by B.
+def _split_runs(seed):
+    tr = tg.random_trace(seed, n_kernels=10, max_warps=10, max_events=12, n_bb=10, dup_p=0.8)
+    h = tr.n_kernels // 2
+    return tr, tg.trace_from_warps([_warps_of(tr, k) for k in range(h)], tr.bb_len,
+                                   warps_total=tr.warps_total[:h]), \
+        tg.trace_from_warps([_warps_of(tr, k) for k in range(h, tr.n_kernels)], tr.bb_len,
+                            warps_total=tr.warps_total[h:])
+
+
+@pytest.mark.parametrize("seed", range(4))
+def test_pool_self_reuse(seed):
+    _, a, _ = _split_runs(40 + seed)
+    t, sig, mass = _pipeline(a)
+    m, _ = oracle.match(t["kernel_type_off"], sig, mass, a.warps_total)
+    pool = oracle.pool_export(t, a.warps_total, m)
+    assert pool["n_pool"] == int((m < 0).sum()) and list(pool["kernel_id"]) == [k for k in range(a.n_kernels) if m[k] < 0]
+    mp, dp = oracle.match_pooled(pool, t, a.warps_total)
+    Kp = pool["n_pool"]
+    cur = mp[Kp:]
+    assert (mp[:Kp] < 0).all()  # pooled representatives stay representatives
+    for k in range(a.n_kernels):
+        if mass[k] == 0:
+            assert cur[k] < 0  # N = 0 never matches [P-19]
+            continue
+        assert 0 <= cur[k] < Kp  # every kernel reuses a pooled representative
+        if m[k] < 0:  # a representative finds its own copy (distance 0, equal warps, earliest such)
+            assert cur[k] == list(pool["kernel_id"]).index(k) and dp[Kp + k] == 0.0
+
+
+@pytest.mark.parametrize("seed", range(4))
+@pytest.mark.parametrize("theta", [(1, 20), (1, 5)])
+def test_pool_matches_bruteforce(seed, theta):
+    _, a, b = _split_runs(60 + seed)
+    ta, sa, ma_ = _pipeline(a)
+    m_a, _ = oracle.match(ta["kernel_type_off"], sa, ma_, a.warps_total, theta=theta)
+    pool = oracle.pool_export(ta, a.warps_total, m_a)
+    tb, _, mb_ = _pipeline(b)
+    mp, _ = oracle.match_pooled(pool, tb, b.warps_total, theta=theta)
+    reps = [k for k in range(a.n_kernels) if m_a[k] < 0]
+    vecs = [_frac_gpu_bbv(ta, k) for k in reps] + [_frac_gpu_bbv(tb, k) for k in range(b.n_kernels)]
+    masses = [int(ma_[k]) for k in reps] + [int(x) for x in mb_]
+    wt = [int(a.warps_total[k]) for k in reps] + [int(x) for x in b.warps_total]
+    ref = _brute_resolve(vecs, masses, wt, Fraction(*theta), 64, 0)
+    assert list(mp) == ref

@@ -90,6 +90,20 @@ def test_random_small(ph, seed):
     full_chain(ph, tr, thetas=((1, 20), (1, 5), (1, 2)), pools=(0, 1))
 
 
+@pytest.mark.parametrize("cfg", [1, 6])
+def test_k1_round1_kernel_matches(ph, cfg, monkeypatch):
+    # PHOTON_K1_V1 routes K1 to the round-1 kernel (k_bbv.cu, the path for B > 4096); both kernels must give the
+    # oracle's BBVs and types on the same inputs (C1: items of two chunks; C6: every template, tiny warps)
+    tr = tg.make_trace(cfg)
+    ref = None
+    for v1 in (False, True):
+        if v1:
+            monkeypatch.setenv("PHOTON_K1_V1", "1")
+        d, o, p16 = check_bbv(ph, tr)
+        ref = ref if ref is not None else oracle.group(tr, p16)
+        check_types(ph, tr, ph.photon_warp_group(d), ref)
+
+
 def test_empty_warps_kernels_and_ragged(ph):
     kernels = [[[], [], [0, 1]], [], [[2] * 1000 + [1] * 3], [[]], [[0, 1, 2, 3, 4, 5, 6]] * 300 + [[1]]]
     tr = tg.trace_from_warps(kernels, bb_len=[3, 1, 7, 2, 9, 4, 5], warps_total=[3, 64, 1, 1, 301])
@@ -440,3 +454,45 @@ def test_bb_predict_random_tables(ph):
         pd, un = oracle.bb_predict(tr, fs, ds)
         assert np.array_equal(_np(o["pred_dur_sum"], np.uint64), pd)
         assert np.array_equal(_np(o["unpredicted"], np.uint32), un)
+
+
+# ---- N4: persisted signature pool (L402) -------------------------------------------------------------------
+@pytest.mark.parametrize("cfg", [6, 4])
+def test_pool_reuse(ph, cfg, tmp_path):
+    # run A -> pool of its representatives (device export, persisted to disk and reloaded); run B matched against
+    # it: pool, match and distances equal the oracle's on the same split
+    g = tg.Generator(cfg)
+    h = g.n_kernels // 2
+    a, b = g.kernels_trace(0, h), g.kernels_trace(h, g.n_kernels)
+    da, db = _dev(ph, a), _dev(ph, b)
+    ty_a = ph.photon_warp_group(da)
+    m_a = ph.photon_kernel_match(a.n_kernels, ty_a, da.warps_total)
+    pool = ph.photon_pool_export(a.n_kernels, ty_a, da.warps_total, m_a["match"])
+    ra = oracle.group(a, oracle.bbv(a, want_kbb=False)[0])
+    sa, ma_ = oracle.signature(ra["kernel_type_off"], ra["type_key"], ra["type_count"])
+    ref_m_a, _ = oracle.match(ra["kernel_type_off"], sa, ma_, a.warps_total)
+    assert np.array_equal(_np(m_a["match"], np.int64), ref_m_a)
+    rp = oracle.pool_export(ra, a.warps_total, ref_m_a)
+    Kp = rp["n_pool"]
+    assert pool["n_pool"] == Kp
+    assert np.array_equal(_np(pool["kernel_type_off"], np.uint64), rp["kernel_type_off"])
+    Tp = int(rp["kernel_type_off"][-1])
+    assert np.array_equal(_np(pool["type_key"], np.uint32).reshape(-1, 16)[:Tp], rp["type_key"])
+    assert np.array_equal(_np(pool["type_count"], np.uint64)[:Tp], rp["type_count"])
+    assert np.array_equal(_np(pool["warps_total"], np.uint64), rp["warps_total"])
+    assert np.array_equal(_np(pool["kernel_id"], np.uint32), rp["kernel_id"])
+    path = str(tmp_path / "pool.npz")
+    ph.save_pool(pool, path)
+    pool2 = ph.load_pool(path)
+    ty_b = ph.photon_warp_group(db)
+    rb = oracle.group(b, oracle.bbv(b, want_kbb=False)[0])
+    for th in ((1, 20), (1, 5)):
+        o = ph.photon_kernel_match_pooled(pool2, b.n_kernels, ty_b, db.warps_total, theta=th)
+        rm, rd = oracle.match_pooled(rp, rb, b.warps_total, theta=th)
+        assert np.array_equal(_np(o["match"], np.int64), rm)
+        got = _np(o["match_dist"], np.float64)
+        fin = np.isfinite(rd)
+        assert np.array_equal(np.isfinite(got), fin)
+        assert np.allclose(got[fin], rd[fin], rtol=1e-6, atol=0)
+        if th == (1, 20):
+            assert (rm[Kp:] >= 0).sum() > 0  # some of run B reuses run A
