@@ -264,6 +264,28 @@ PHOTON_API int photon_bb_predict(photon_ctx *ctx, const photon_trace *trace, con
                                  const uint64_t *stable_dur_sum /*[K][B]*/, void *ws, size_t ws_bytes,
                                  uint64_t *pred_dur_sum /*[W]*/, uint32_t *unpredicted /*[W]*/, void *stream);
 
+/* ---- N2: full-BBV exact grouping and tagged-stream ingest (L154, L161) -----------------------------------------
+ * photon_warp_group_full: warp types keyed on the FULL BBV -- the execution count of every BB id, "warps that
+ *   execute the same instruction sequence ... have the same BBV" (L154, L161) -- instead of the 16-bin projection
+ *   of L178 [P-3]: warps w, v of one kernel share a type iff their event multisets are equal.  Outputs as
+ *   photon_warp_group (out->capacity >= the number of types, else ECAPACITY); type_key = the 16-bin projection of
+ *   the type (warp_bbv16 from photon_bbv_build, identical for all members); rows ordered by (count desc, key asc,
+ *   lowest warp asc) [N2-a]; warp_sampling_ok as A2 (L249).  Decided by a 128-bit order-independent hash and then
+ *   VERIFIED exactly on every member's sorted event list: a hash collision (probability ~2^-128 per pair) latches
+ *   PHOTON_ERANGE with the warp index instead of a result.  ERANGE also for bb >= n_bb and bad offsets.
+ *   ws >= photon_group_full_workspace_bytes(trace) (grows with W and E; the error latch is at its start).
+ * photon_ingest_tagged: n tagged events (warp[i] u32 < n_warps: the analysed-warp index, bb[i] u16), interleaved
+ *   in any order (as a functional simulator retires them), to the CSR of photon_trace: bb_out[n] = the events
+ *   stably sorted by warp (each warp keeps its events' stream order, L125) and warp_event_off[n_warps + 1].
+ *   ERANGE (index = event): warp[i] >= n_warps.  ws >= photon_ingest_workspace_bytes(n, n_warps). */
+PHOTON_API size_t photon_group_full_workspace_bytes(const photon_trace *trace);
+PHOTON_API int photon_warp_group_full(photon_ctx *ctx, const photon_trace *trace, const uint32_t *warp_bbv16 /*[W][16]*/,
+                                      void *ws, size_t ws_bytes, photon_types *out, void *stream);
+PHOTON_API size_t photon_ingest_workspace_bytes(uint64_t n_events, uint64_t n_warps);
+PHOTON_API int photon_ingest_tagged(photon_ctx *ctx, uint64_t n_events, uint64_t n_warps, const uint32_t *warp /*[n]*/,
+                                    const uint16_t *bb /*[n]*/, void *ws, size_t ws_bytes, uint16_t *bb_out /*[n]*/,
+                                    uint64_t *warp_event_off /*[n_warps+1]*/, void *stream);
+
 /* ---- N4: persisted signature pool, offline reuse of the analysis (L402, §6.3 "Online/Offline Tradeoff") -------
  * "All data that is generated by the online analysis ... is micro-architecture agnostic.  Hardware researchers can
  * reuse these data" (L402).  Reading [N4-a]: a pool holds the REPRESENTATIVE kernels (match[k] < 0) of one or more

@@ -204,6 +204,51 @@ def bb_predict(trace, first_stable, stable_dur_sum):
     return pd[:W], un[:W]
 
 
+def group_full(trace, warp_bbv16):
+    """N2 (L154, L161, reading [N2-a]): warp types keyed on the full BBV (the count of every BB id); rows ordered
+    by (count desc, projected key asc, lowest warp asc); type_key = the members' 16-bin projection.  Plain Python
+    over each warp's events (small traces)."""
+    K, W = trace.n_kernels, trace.n_warps
+    kwo = np.asarray(trace.kernel_warp_off, np.int64)
+    weo = np.asarray(trace.warp_event_off, np.int64)
+    bb = np.asarray(trace.bb)
+    p16 = np.asarray(warp_bbv16, np.uint32).reshape(-1, 16)
+    warp_type = np.zeros(W, np.uint32)
+    kto = np.zeros(K + 1, np.uint64)
+    keys, cnts, firsts = [], [], []
+    ok = np.zeros(K, np.uint8)
+    for k in range(K):
+        groups = {}  # full BBV -> [first warp, count, members]
+        for w in range(int(kwo[k]), int(kwo[k + 1])):
+            ids, c = np.unique(bb[weo[w]:weo[w + 1]], return_counts=True)
+            fk = (tuple(int(x) for x in ids), tuple(int(x) for x in c))
+            g = groups.setdefault(fk, [w, 0, []])
+            g[1] += 1
+            g[2].append(w)
+        rows = sorted(groups.values(), key=lambda g: (-g[1], tuple(int(x) for x in p16[g[0]]), g[0]))
+        for r, g in enumerate(rows):
+            for w in g[2]:
+                warp_type[w] = r
+            keys.append(p16[g[0]])
+            cnts.append(g[1])
+            firsts.append(g[0])
+        kto[k + 1] = kto[k] + len(rows)
+        Wk = int(kwo[k + 1] - kwo[k])
+        ok[k] = 1 if Wk > 0 and rows and 100 * rows[0][1] > 95 * Wk else 0
+    return dict(warp_type=warp_type, kernel_type_off=kto,
+                type_key=np.array(keys, np.uint32).reshape(-1, 16), type_count=np.array(cnts, np.uint64),
+                type_first_warp=np.array(firsts, np.uint64), warp_sampling_ok=ok)
+
+
+def ingest(warp, bb, n_warps):
+    """N2 ingest: tagged (warp, bb) events in stream order -> (bb by warp, stream order kept; warp_event_off)."""
+    warp = np.asarray(warp, np.int64)
+    order = np.argsort(warp, kind="stable")
+    off = np.zeros(n_warps + 1, np.uint64)
+    off[1:] = np.cumsum(np.bincount(warp, minlength=n_warps)[:n_warps])
+    return np.asarray(bb)[order], off
+
+
 def pool_export(types, warps_total, match_):
     """N4 (L402, reading [N4-a]): the run's representative kernels (match < 0), in launch order: dict(n_pool,
     kernel_type_off, type_key, type_count, warps_total, kernel_id)."""

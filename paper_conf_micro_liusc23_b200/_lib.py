@@ -97,6 +97,12 @@ _SIGS = [
                                       c_size_t, c_void_p, c_void_p, c_void_p]),
     ("photon_bb_predict", c_int, [c_void_p, POINTER(Trace), c_void_p, c_void_p, c_void_p, c_size_t, c_void_p,
                                   c_void_p, c_void_p]),
+    ("photon_group_full_workspace_bytes", c_size_t, [POINTER(Trace)]),
+    ("photon_warp_group_full", c_int, [c_void_p, POINTER(Trace), c_void_p, c_void_p, c_size_t, POINTER(Types),
+                                       c_void_p]),
+    ("photon_ingest_workspace_bytes", c_size_t, [c_uint64, c_uint64]),
+    ("photon_ingest_tagged", c_int, [c_void_p, c_uint64, c_uint64, c_void_p, c_void_p, c_void_p, c_size_t,
+                                     c_void_p, c_void_p, c_void_p]),
     ("photon_pool_export_workspace_bytes", c_size_t, [c_uint32]),
     ("photon_pool_export", c_int, [c_void_p, c_uint32, POINTER(Types), c_void_p, c_void_p, c_void_p, c_size_t,
                                    POINTER(Types), c_void_p, c_void_p, c_void_p, c_void_p]),

@@ -269,6 +269,34 @@ class Photon:
                                            self.stream_ptr(stream)))
         return dict(filter_pairs=int(st[0]), close_pairs=int(st[1]), rounds=int(st[2]), pair_capacity=int(st[3]))
 
+    # -- N2: full-BBV exact grouping and tagged-stream ingest (L154, L161) -------------------------------------
+    def photon_warp_group_full(self, t: DeviceTrace, warp_bbv16=None, stream=None, check: bool = True) -> dict:
+        """Warp types keyed on the full BBV (N2); warp_bbv16 from photon_bbv_build (computed when None)."""
+        if warp_bbv16 is None:
+            warp_bbv16 = self.photon_bbv_build(t, bbv16=True, insts=False, stream=stream, check=check)["warp_bbv16"]
+        ct = t.c()
+        ws = self.workspace("group_full", self.L.photon_group_full_workspace_bytes(ctypes.byref(ct)))
+        ty = self.alloc_types(t.n_kernels, t.n_warps, max(t.n_warps, 1))
+        self._rc(self.L.photon_warp_group_full(self.ctx, ctypes.byref(ct), warp_bbv16.data_ptr(), ws.data_ptr(),
+                                               ws.numel(), ctypes.byref(self.types_c(ty)), self.stream_ptr(stream)))
+        if check:
+            self.check(ws, stream)
+        ty["_ws"] = ws
+        return ty
+
+    def photon_ingest_tagged(self, warp, bb, n_warps: int, stream=None, check: bool = True) -> dict:
+        """Interleaved (warp, bb) tagged events -> CSR by warp (stable): dict(bb, warp_event_off)."""
+        n = int(warp.numel())
+        ws = self.workspace("ingest", self.L.photon_ingest_workspace_bytes(n, n_warps))
+        out = dict(bb=self.empty(n, "int16"), warp_event_off=self.empty(n_warps + 1, "int64"))
+        self._rc(self.L.photon_ingest_tagged(self.ctx, n, n_warps, warp.data_ptr() if n else None,
+                                             bb.data_ptr() if n else None, ws.data_ptr(), ws.numel(),
+                                             out["bb"].data_ptr() if n else None, out["warp_event_off"].data_ptr(),
+                                             self.stream_ptr(stream)))
+        if check:
+            self.check(ws, stream)
+        return out
+
     # -- N4: persisted signature pool (L402) -------------------------------------------------------------------
     def photon_pool_export(self, n_kernels: int, ty: dict, warps_total, match, stream=None) -> dict:
         """The representatives of a run (match < 0) as a pool: dict(n_pool, capacity, kernel_type_off, type_key,

@@ -503,6 +503,100 @@ int photon_kernel_match(photon_ctx* ctx, uint32_t K, const photon_types* types, 
   return PHOTON_OK;
 }
 
+// ---- N2: full-BBV exact grouping and tagged-stream ingest (k_full.cu) ------------------------------------------
+namespace {
+struct FullLayout {
+  DevErr* err;
+  FullWs f;
+  HtWs h;
+  size_t bytes;
+};
+FullLayout full_layout(const photon_trace* t, void* base) {
+  Carver c(base);
+  FullLayout L;
+  const uint64_t W = t->n_warps + 1, E = t->n_events + 8;
+  L.err = c.take<DevErr>(1);
+  L.f.h_lo = c.take<uint64_t>(W);
+  L.f.h_hi = c.take<uint64_t>(W);
+  L.f.k64 = c.take<uint64_t>(W);
+  L.f.g64 = c.take<uint64_t>(W);
+  L.f.gstart = c.take<uint64_t>(W);
+  L.f.kid = c.take<uint32_t>(W);
+  L.f.perm_a = c.take<uint32_t>(W);
+  L.f.perm_b = c.take<uint32_t>(W);
+  L.f.k32 = c.take<uint32_t>(W);
+  L.f.g32 = c.take<uint32_t>(W);
+  L.f.flag = c.take<uint32_t>(W);
+  L.f.gid = c.take<uint32_t>(W);
+  L.f.wgroup = c.take<uint32_t>(W);
+  L.f.sorted = c.take<uint16_t>(E);
+  uint64_t cap = 1024;
+  while (cap < t->n_warps) cap <<= 1;
+  carve_ht(c, cap, t->n_kernels, L.h);
+  L.h.ht.mask = cap - 1;
+  L.f.cub_bytes = full_cub_bytes(t->n_warps, t->n_events);
+  L.f.cub = c.take<uint8_t>(L.f.cub_bytes + 16);
+  L.bytes = c.off + 256;
+  return L;
+}
+}  // namespace
+
+size_t photon_group_full_workspace_bytes(const photon_trace* t) {
+  if (!t) return 0;
+  return full_layout(t, nullptr).bytes;
+}
+
+int photon_warp_group_full(photon_ctx* ctx, const photon_trace* t, const uint32_t* warp_bbv16, void* ws,
+                           size_t ws_bytes, photon_types* out, void* stream) {
+  if (!ctx) return PHOTON_EINVAL;
+  int rc = check_trace(ctx, t);
+  if (rc) return rc;
+  if (!warp_bbv16 || !ws || !out || !out->kernel_type_off || !out->type_key || !out->type_count ||
+      !out->type_first_warp || !out->warp_sampling_ok || !out->warp_type)
+    return fail(ctx, PHOTON_EINVAL, "NULL argument");
+  if (t->n_warps >= (1ull << 32)) return fail(ctx, PHOTON_EINVAL, "n_warps must be < 2^32");
+  const size_t need = photon_group_full_workspace_bytes(t);
+  if (ws_bytes < need) return fail(ctx, PHOTON_EWORKSPACE, "workspace %zu < %zu bytes", ws_bytes, need);
+  FullLayout L = full_layout(t, ws);
+  cudaStream_t s = (cudaStream_t)stream;
+  CK(cudaSetDevice(ctx->device), "cudaSetDevice");
+  ctx->last_ws = ws;
+  CK(cudaMemsetAsync(L.err, 0, sizeof(DevErr), s), "memset");
+  TraceDev d = to_dev(t);
+  CK(launch_validate_offsets(d, L.err, s), "validate");
+  CK(launch_group_full(d, warp_bbv16, L.f, L.h.ht, L.h.cw, *out, L.err, ctx->num_sms, s), "group_full");
+  return PHOTON_OK;
+}
+
+size_t photon_ingest_workspace_bytes(uint64_t n, uint64_t W) {
+  (void)W;
+  Carver c(nullptr);
+  c.take<DevErr>(1);
+  c.take<uint32_t>(n + 1);
+  c.take<uint8_t>(ingest_cub_bytes(n) + 16);
+  return c.off + 256;
+}
+
+int photon_ingest_tagged(photon_ctx* ctx, uint64_t n, uint64_t W, const uint32_t* warp, const uint16_t* bb, void* ws,
+                         size_t ws_bytes, uint16_t* bb_out, uint64_t* warp_event_off, void* stream) {
+  if (!ctx) return PHOTON_EINVAL;
+  if ((n && (!warp || !bb || !bb_out)) || !warp_event_off || !ws) return fail(ctx, PHOTON_EINVAL, "NULL argument");
+  if (W >= (1ull << 32) || n >= (1ull << 40)) return fail(ctx, PHOTON_EINVAL, "n_warps must be < 2^32");
+  const size_t need = photon_ingest_workspace_bytes(n, W);
+  if (ws_bytes < need) return fail(ctx, PHOTON_EWORKSPACE, "workspace %zu < %zu bytes", ws_bytes, need);
+  Carver c(ws);
+  DevErr* err = c.take<DevErr>(1);
+  uint32_t* key_out = c.take<uint32_t>(n + 1);
+  const size_t cb = ingest_cub_bytes(n);
+  void* cub = c.take<uint8_t>(cb + 16);
+  cudaStream_t s = (cudaStream_t)stream;
+  CK(cudaSetDevice(ctx->device), "cudaSetDevice");
+  ctx->last_ws = ws;
+  CK(cudaMemsetAsync(err, 0, sizeof(DevErr), s), "memset");
+  CK(launch_ingest(n, W, warp, bb, cub, cb, key_out, bb_out, warp_event_off, err, s), "ingest");
+  return PHOTON_OK;
+}
+
 // ---- N4: persisted signature pool (k_pool.cu) ----------------------------------------------------------------
 size_t photon_pool_export_workspace_bytes(uint32_t K) {
   Carver c(nullptr);

@@ -146,6 +146,20 @@ size_t warp_stable_ws_bytes(uint32_t K, uint64_t R);
 cudaError_t launch_warp_stable(const photon_timing& t, const uint8_t* ok, uint32_t n, uint32_t dnum, uint32_t dden,
                                void* ws, int64_t* switch_at, uint64_t* dur, DevErr* err, int num_sms,
                                cudaStream_t s);
+// ---- N2 (k_full.cu): full-BBV exact grouping and tagged-stream ingest ----------------------------------------
+struct FullWs {
+  uint64_t *h_lo, *h_hi, *k64, *g64, *gstart;  // [W]
+  uint32_t *kid, *perm_a, *perm_b, *k32, *g32, *flag, *gid, *wgroup;  // [W]
+  uint16_t* sorted;  // [E] per-warp sorted events
+  void* cub;
+  size_t cub_bytes;
+};
+size_t full_cub_bytes(uint64_t W, uint64_t E);
+size_t ingest_cub_bytes(uint64_t n);
+cudaError_t launch_group_full(const TraceDev& t, const uint32_t* bbv16, const FullWs& f, const HashTable& ht,
+                              const CanonWs& cw, const photon_types& out, DevErr* err, int num_sms, cudaStream_t s);
+cudaError_t launch_ingest(uint64_t n, uint64_t W, const uint32_t* warp, const uint16_t* bb, void* cub, size_t cub_bytes,
+                          uint32_t* key_out, uint16_t* bb_out, uint64_t* off, DevErr* err, cudaStream_t s);
 // ---- N4 (k_pool.cu): persisted signature pool --------------------------------------------------------------
 cudaError_t launch_pool_export(uint32_t K, const photon_types& ty, const uint64_t* wt, const int64_t* match,
                                uint64_t* keep, uint64_t* ntypes, const photon_types& pool, uint64_t* pwt,

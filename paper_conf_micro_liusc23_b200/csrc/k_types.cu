@@ -86,7 +86,8 @@ __global__ void k_scatter_types(HashTable ht, uint32_t K, const uint64_t* kto, u
   if (pos < capacity) list[pos] = (uint32_t)i;
 }
 
-// canonical order: count descending, then key lexicographically ascending [P-4]; UINT32_MAX = padding (last)
+// canonical order: count descending, then key lexicographically ascending [P-4], then the lowest warp [N2-a] (the
+// projected grouping has unique keys per kernel, so only full-BBV types reach it); UINT32_MAX = padding (last)
 __device__ __forceinline__ bool type_before(const HashTable& ht, uint32_t a, uint32_t b) {
   if (b == UINT32_MAX) return a != UINT32_MAX;
   if (a == UINT32_MAX) return false;
@@ -97,7 +98,7 @@ __device__ __forceinline__ bool type_before(const HashTable& ht, uint32_t a, uin
 #pragma unroll 1
   for (int j = 0; j < 16; ++j)
     if (ka[j] != kb[j]) return ka[j] < kb[j];
-  return false;
+  return ht.first[a] < ht.first[b];
 }
 
 __device__ void emit_rows(const HashTable& ht, uint32_t k, const uint32_t* sorted, uint64_t n, uint64_t off,

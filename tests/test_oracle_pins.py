@@ -713,3 +713,61 @@ def test_pool_matches_bruteforce(seed, theta):
     wt = [int(a.warps_total[k]) for k in reps] + [int(x) for x in b.warps_total]
     ref = _brute_resolve(vecs, masses, wt, Fraction(*theta), 64, 0)
     assert list(mp) == ref
+
+
+# N2: full-BBV grouping (reading [N2-a]) and tagged ingest.  Pins: with B <= 16 and the identity fold the full BBV
+# IS the projected one, so the types equal A2's; brute force on tiny traces (same type <=> equal event multisets,
+# counts = class sizes, the row order rule recomputed); refinement of the projected grouping; ingest of a random
+# order-preserving interleaving gives back the CSR.
+def test_group_full_equals_projected_when_fold_is_identity():
+    for tr in (tg.make_trace(1), tg.random_trace(5, n_kernels=4, max_warps=60, max_events=30, n_bb=16, dup_p=0.7)):
+        p16, _, _ = oracle.bbv(tr, want_kbb=False)
+        a, b = oracle.group(tr, p16), oracle.group_full(tr, p16)
+        T = int(a["kernel_type_off"][-1])
+        for f in ("warp_type", "kernel_type_off", "warp_sampling_ok"):
+            assert np.array_equal(a[f], b[f]), f
+        assert np.array_equal(a["type_key"][:T], b["type_key"])
+        assert np.array_equal(a["type_count"][:T], b["type_count"])
+        assert np.array_equal(a["type_first_warp"][:T], b["type_first_warp"])
+
+
+@pytest.mark.parametrize("seed", range(4))
+def test_group_full_bruteforce_and_refinement(seed):
+    import collections
+    tr = tg.random_trace(70 + seed, n_kernels=3, max_warps=40, max_events=10, n_bb=40, dup_p=0.7)
+    p16, _, _ = oracle.bbv(tr, want_kbb=False)
+    t = oracle.group_full(tr, p16)
+    proj = oracle.group(tr, p16)
+    kwo, weo = tr.kernel_warp_off, tr.warp_event_off
+    for k in range(tr.n_kernels):
+        ws = list(range(int(kwo[k]), int(kwo[k + 1])))
+        ms = {w: collections.Counter(tr.bb[int(weo[w]):int(weo[w + 1])].tolist()) for w in ws}
+        for a in ws:
+            for b in ws:
+                assert (t["warp_type"][a] == t["warp_type"][b]) == (ms[a] == ms[b])
+                if ms[a] == ms[b]:
+                    assert proj["warp_type"][a] == proj["warp_type"][b]  # refinement
+        o = int(t["kernel_type_off"][k])
+        n = int(t["kernel_type_off"][k + 1]) - o
+        rows = []
+        for r in range(n):
+            mem = [w for w in ws if t["warp_type"][w] == r]
+            assert int(t["type_count"][o + r]) == len(mem) and int(t["type_first_warp"][o + r]) == min(mem)
+            assert np.array_equal(t["type_key"][o + r], p16[min(mem)])
+            rows.append((-len(mem), tuple(int(x) for x in p16[min(mem)]), min(mem)))
+        assert rows == sorted(rows)
+
+
+def test_ingest_interleaved_stream():
+    tr = tg.random_trace(9, n_kernels=3, max_warps=50, max_events=20, n_bb=30)
+    rs = np.random.default_rng(9)
+    W, weo = tr.n_warps, tr.warp_event_off.astype(np.int64)
+    owner = np.repeat(np.arange(W), np.diff(weo))
+    order = np.argsort(rs.random(len(owner)), kind="stable")  # a random interleaving ...
+    order = np.concatenate([np.sort(order[owner[order] == w]) for w in range(W)])[np.argsort(
+        np.concatenate([np.flatnonzero(owner[order] == w) for w in range(W)]), kind="stable")]  # ... keeping each warp's order
+    warp, bb = owner[order], tr.bb[order]
+    for w in range(W):  # the stream keeps each warp's event order
+        assert np.array_equal(bb[warp == w], tr.bb[weo[w]:weo[w + 1]])
+    out_bb, off = oracle.ingest(warp, bb, W)
+    assert np.array_equal(off, tr.warp_event_off.astype(np.uint64)) and np.array_equal(out_bb, tr.bb)

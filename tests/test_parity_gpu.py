@@ -496,3 +496,53 @@ def test_pool_reuse(ph, cfg, tmp_path):
         assert np.allclose(got[fin], rd[fin], rtol=1e-6, atol=0)
         if th == (1, 20):
             assert (rm[Kp:] >= 0).sum() > 0  # some of run B reuses run A
+
+
+# ---- N2: full-BBV exact grouping and tagged-stream ingest (L154, L161) ------------------------------------------
+@pytest.mark.parametrize("which", ["c6", "c1", "rand5000", "ragged"])
+def test_group_full(ph, which):
+    if which == "c6":
+        tr = tg.make_trace(6)
+    elif which == "c1":
+        tr = tg.make_trace(1)
+    elif which == "rand5000":
+        tr = tg.random_trace(11, n_kernels=5, max_warps=400, max_events=60, n_bb=5000, dup_p=0.7)
+    else:
+        kernels = [[[], [], [0, 1]], [], [[2] * 1000 + [1] * 3], [[]], [[0, 1, 2, 3, 4, 5, 6]] * 300 + [[1]],
+                   [[1, 0], [0, 1], [1, 1, 0], [0, 1, 1], [2]]]
+        tr = tg.trace_from_warps(kernels, bb_len=[3, 1, 7, 2, 9, 4, 5])
+    d = _dev(ph, tr)
+    p16, _, _ = oracle.bbv(tr, want_kbb=False)
+    ref = oracle.group_full(tr, p16)
+    ty = ph.photon_warp_group_full(d)
+    T = int(ref["kernel_type_off"][-1])
+    assert np.array_equal(_np(ty["kernel_type_off"], np.uint64), ref["kernel_type_off"])
+    assert np.array_equal(_np(ty["warp_type"], np.uint32), ref["warp_type"])
+    assert np.array_equal(_np(ty["type_key"], np.uint32).reshape(-1, 16)[:T], ref["type_key"].reshape(-1, 16))
+    assert np.array_equal(_np(ty["type_count"], np.uint64)[:T], ref["type_count"])
+    assert np.array_equal(_np(ty["type_first_warp"], np.uint64)[:T], ref["type_first_warp"])
+    assert np.array_equal(_np(ty["warp_sampling_ok"], np.uint8), ref["warp_sampling_ok"])
+
+
+def test_ingest_tagged(ph):
+    import torch
+    tr = tg.make_trace(6)
+    W, weo = tr.n_warps, tr.warp_event_off.astype(np.int64)
+    owner = np.repeat(np.arange(W), np.diff(weo)).astype(np.uint32)
+    # interleave warps in slices of the generator's 2560-slot wave order: event i of warp w at key (w % 2560, i, w)
+    pos = np.arange(len(owner)) - weo[owner]
+    order = np.lexsort((owner, pos, owner % 2560))
+    warp, bb = owner[order], tr.bb[order]
+    out = ph.photon_ingest_tagged(torch.from_numpy(warp.astype(np.int32)).to(ph.device),
+                                  torch.from_numpy(bb.astype(np.int16)).to(ph.device), W)
+    rb, roff = oracle.ingest(warp, bb, W)
+    assert np.array_equal(_np(out["warp_event_off"], np.uint64), roff)
+    assert np.array_equal(_np(out["bb"], np.uint16), rb)
+    assert np.array_equal(rb, tr.bb)  # and it is the CSR trace back
+    from paper_conf_micro_liusc23_b200 import PhotonError
+    bad = warp.copy()
+    bad[7] = W
+    with pytest.raises(PhotonError) as ei:
+        ph.photon_ingest_tagged(torch.from_numpy(bad.astype(np.int32)).to(ph.device),
+                                torch.from_numpy(bb.astype(np.int16)).to(ph.device), W)
+    assert ei.value.code == -3 and ei.value.index == 7
