@@ -393,6 +393,59 @@ def run_photon(args):
                       "switched_kernels": int((to_numpy_i64(o["switch_at"]) >= 0).sum()),
                       "dominant_kernels": int(okd.to(torch.int64).sum().item())}
 
+    # ---- N2 (full-BBV exact grouping, L154/L161) on the same config's trace ----
+    if not args.skip_a5 and ws == 1:
+        g2 = tg.Generator(args.a5_config)
+        t2 = g2.trace()
+        d2 = DeviceTrace.from_host(t2, dev)
+        b16 = ph.photon_bbv_build(d2, bbv16=True, insts=False)["warp_bbv16"]
+        o = ph.photon_warp_group_full(d2, b16)
+        torch.cuda.synchronize()
+        f0, f1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        n7 = max(args.steps // 4, 3)
+        f0.record(s)
+        for _ in range(n7):
+            o = ph.photon_warp_group_full(d2, b16, check=False)
+        f1.record(s)
+        torch.cuda.synchronize()
+        ph.check(o["_ws"])
+        fms = f0.elapsed_time(f1) / n7
+        E2, W2 = t2.n_events, t2.n_warps
+        fbytes = 2 * E2 + 12 * W2
+        line["n2"] = {"metric": "trace events grouped/sec (full-BBV exact warp types, verified)",
+                      "value": E2 / (fms / 1000), "unit": "events/s", "ms_per_step": fms, "events": E2,
+                      "workload": f"{CONFIG_DESC.get(args.a5_config)} trace",
+                      "roofline": {"bound": "hbm", "achieved": fbytes / (fms / 1000) / 1e9, "peak": hbm_peak,
+                                   "unit": "GB/s", "frac": fbytes / (fms / 1000) / 1e9 / hbm_peak,
+                                   "algorithmic_bytes": fbytes, "traffic": None},
+                      "full_types": int(o["kernel_type_off"][-1].item())}
+        # ---- N4 (persisted signature pool, L402): ResNet-152's second half matched against its first half ----
+        g4 = tg.Generator(4)
+        h = g4.n_kernels // 2
+        ta4, tb4 = g4.kernels_trace(0, h), g4.kernels_trace(h, g4.n_kernels)
+        da4, db4 = DeviceTrace.from_host(ta4, dev), DeviceTrace.from_host(tb4, dev)
+        ty_a = ph.photon_warp_group(da4)
+        pool = ph.photon_pool_export(ta4.n_kernels, ty_a, da4.warps_total,
+                                     ph.photon_kernel_match(ta4.n_kernels, ty_a, da4.warps_total)["match"])
+        ty_b = ph.photon_warp_group(db4)
+        m4 = ph.photon_kernel_match_pooled(pool, tb4.n_kernels, ty_b, db4.warps_total)
+        torch.cuda.synchronize()
+        q0, q1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        q0.record(s)
+        for _ in range(n7):
+            m4 = ph.photon_kernel_match_pooled(pool, tb4.n_kernels, ty_b, db4.warps_total, want_dist=False)
+        q1.record(s)
+        torch.cuda.synchronize()
+        qms = q0.elapsed_time(q1) / n7
+        mm = to_numpy_i64(m4["match"])
+        Kp = pool["n_pool"]
+        line["n4"] = {"metric": "kernels matched/sec against a persisted signature pool",
+                      "value": tb4.n_kernels / (qms / 1000), "unit": "kernels/s", "ms_per_step": qms,
+                      "workload": f"C4 ResNet-152: kernels [{h}, {g4.n_kernels}) against the pool of kernels [0, {h})",
+                      "pool_kernels": Kp, "kernels": tb4.n_kernels,
+                      "reused_from_pool": int(((mm[Kp:] >= 0) & (mm[Kp:] < Kp)).sum()),
+                      "roofline": None, "note": "A3/A4 over pool + run: compare ops (ALU), not a streaming pass"}
+
     if rank == 0 and ws == 1 and not args.skip_cpu:
         line["cpu_baseline"] = cpu_baseline(args)
     if rank == 0:

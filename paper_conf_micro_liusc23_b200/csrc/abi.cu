@@ -529,7 +529,8 @@ FullLayout full_layout(const photon_trace* t, void* base) {
   L.f.flag = c.take<uint32_t>(W);
   L.f.gid = c.take<uint32_t>(W);
   L.f.wgroup = c.take<uint32_t>(W);
-  L.f.sorted = c.take<uint16_t>(E);
+  L.f.ekey = c.take<uint64_t>(E);
+  L.f.sorted = c.take<uint64_t>(E);
   uint64_t cap = 1024;
   while (cap < t->n_warps) cap <<= 1;
   carve_ht(c, cap, t->n_kernels, L.h);

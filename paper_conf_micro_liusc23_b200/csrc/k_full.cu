@@ -13,14 +13,14 @@
 //     contiguous, members in ascending warp order.
 //  3. k_full_groups: group ids (CUB scan of the boundary flags), one slot per group in a type table (kernel,
 //     projected key of the first member, count, first warp) and each warp's group.
-//  4. k_full_verify: every member is compared with its group's first warp on the per-warp SORTED event lists (CUB
-//     segmented sort): a hash collision is detected exactly and latched (PHOTON_ERANGE, index = the warp).
+//  4. k_full_verify: every member is compared with its group's first warp on the per-warp SORTED event lists (one
+//     CUB radix sort of the (warp << 16 | bb) keys written in step 1): a hash collision is detected exactly and
+//     latched (PHOTON_ERANGE, index = the warp).
 //  5. the A2 canonicalisation (k_types.cu) over the group table; k_full_remap writes warp_type.
 // Ingest: a stream of (warp, bb) tagged events in arbitrary interleaving -> CSR by warp with a stable radix sort
 // (each warp keeps its events' stream order) and boundary-filled offsets.
 #include <cub/device/device_radix_sort.cuh>
 #include <cub/device/device_scan.cuh>
-#include <cub/device/device_segmented_sort.cuh>
 
 #include "internal.h"
 
@@ -37,10 +37,12 @@ __device__ __forceinline__ uint64_t hmix(uint64_t x) {
   return x;
 }
 
-// one hardware warp per analysed warp (grid-stride): 128-bit hash of its event multiset, its kernel, perm = w
+// One hardware warp per analysed warp (grid-stride): lanes read its events coalesced and sum two 64-bit mixes of
+// each BB id (the 128-bit hash of the event multiset), write each event's sort key (warp << 16 | bb), and lane 0
+// finds the warp's kernel; perm = w.
 __global__ void k_full_hash(const uint64_t* __restrict__ kwo, uint32_t K, const uint64_t* __restrict__ weo,
                             uint64_t W, uint64_t E, const uint16_t* __restrict__ bb, uint32_t B, uint64_t* h_lo,
-                            uint64_t* h_hi, uint32_t* kid, uint32_t* perm, DevErr* err) {
+                            uint64_t* h_hi, uint32_t* kid, uint32_t* perm, uint64_t* ekey, DevErr* err) {
   const int lane = threadIdx.x & 31;
   const uint64_t nw = ((uint64_t)gridDim.x * blockDim.x) >> 5;
   for (uint64_t w = ((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; w < W; w += nw) {
@@ -52,6 +54,7 @@ __global__ void k_full_hash(const uint64_t* __restrict__ kwo, uint32_t K, const 
       if (x >= B) latch(err, PHOTON_ERANGE, (int64_t)i);
       a += hmix(0x9E3779B97F4A7C15ull * (x + 1));
       b += hmix(0xC2B2AE3D27D4EB4Full * (x + 1) + 0x165667B19E3779F9ull);
+      ekey[i] = (w << 16) | x;
     }
 #pragma unroll
     for (int o = 16; o > 0; o >>= 1) {
@@ -105,7 +108,6 @@ __global__ void k_full_groups(uint64_t W, const uint32_t* __restrict__ perm, con
   if (i >= W) return;
   const uint32_t w = perm[i], g = gid[i] - 1;
   wgroup[w] = g;
-  atomicAdd(&ht.count[g], 1u);
   if (flag[i]) {
     gstart[g] = i;
     ht.hkey[g] = 1ull;  // occupied
@@ -117,10 +119,19 @@ __global__ void k_full_groups(uint64_t W, const uint32_t* __restrict__ perm, con
   }
 }
 
+// count of group g = next group's start - its start (G = gid[W-1] groups)
+__global__ void k_full_counts(uint64_t W, const uint32_t* __restrict__ gid, const uint64_t* __restrict__ gstart,
+                              HashTable ht) {
+  const uint64_t g = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  const uint64_t G = W ? gid[W - 1] : 0;
+  if (g >= G) return;
+  ht.count[g] = (uint32_t)((g + 1 < G ? gstart[g + 1] : W) - gstart[g]);
+}
+
 // one hardware warp per sorted position that is not a group start: its sorted event list equals the group's first
 __global__ void k_full_verify(uint64_t W, const uint32_t* __restrict__ perm, const uint32_t* __restrict__ flag,
                               const uint32_t* __restrict__ gid, const uint64_t* __restrict__ gstart,
-                              const uint64_t* __restrict__ weo, uint64_t E, const uint16_t* __restrict__ sorted,
+                              const uint64_t* __restrict__ weo, uint64_t E, const uint64_t* __restrict__ sorted,
                               DevErr* err) {
   const int lane = threadIdx.x & 31;
   const uint64_t nw = ((uint64_t)gridDim.x * blockDim.x) >> 5;
@@ -130,7 +141,8 @@ __global__ void k_full_verify(uint64_t W, const uint32_t* __restrict__ perm, con
     const uint64_t ws = umin64(weo[w], E), we = umin64(umax64(weo[w + 1], ws), E);
     const uint64_t rs = umin64(weo[r], E), re = umin64(umax64(weo[r + 1], rs), E);
     bool same = (we - ws) == (re - rs);
-    for (uint64_t j = lane; same && j < we - ws; j += 32) same = sorted[ws + j] == sorted[rs + j];
+    for (uint64_t j = lane; same && j < we - ws; j += 32)
+      same = (sorted[ws + j] & 0xFFFFu) == (sorted[rs + j] & 0xFFFFu);
     same = __all_sync(0xffffffffu, same);
     if (!same && lane == 0) latch(err, PHOTON_ERANGE, (int64_t)w);  // a 128-bit hash collision, detected exactly
   }
@@ -168,8 +180,7 @@ size_t full_cub_bytes(uint64_t W, uint64_t E) {
   cub::DeviceRadixSort::SortPairs(nullptr, b, (const uint32_t*)nullptr, (uint32_t*)nullptr,
                                   (const uint32_t*)nullptr, (uint32_t*)nullptr, (int64_t)W);
   cub::DeviceScan::InclusiveSum(nullptr, c, (const uint32_t*)nullptr, (uint32_t*)nullptr, (int64_t)W);
-  cub::DeviceSegmentedSort::SortKeys(nullptr, d, (const uint16_t*)nullptr, (uint16_t*)nullptr, (int64_t)E,
-                                     (int64_t)W, (const uint64_t*)nullptr, (const uint64_t*)nullptr);
+  cub::DeviceRadixSort::SortKeys(nullptr, d, (const uint64_t*)nullptr, (uint64_t*)nullptr, (int64_t)E);
   size_t m = a > b ? a : b;
   m = m > c ? m : c;
   return m > d ? m : d;
@@ -188,7 +199,7 @@ cudaError_t launch_group_full(const TraceDev& t, const uint32_t* bbv16, const Fu
   cudaError_t e;
   const unsigned hg = (unsigned)umin64(ceil_div(W * 32, 256), (uint64_t)num_sms * 16);
   note_launch(), k_full_hash<<<hg, 256, 0, s>>>(t.kwo, t.K, t.weo, W, t.E, t.bb, t.B, f.h_lo, f.h_hi, f.kid, f.perm_a,
-                                                err);
+                                                f.ekey, err);
   size_t tb = f.cub_bytes;
   // stable passes: h_lo, then h_hi, then kernel (each carries the warp permutation)
   if ((e = cub::DeviceRadixSort::SortPairs(f.cub, tb, f.h_lo, f.k64, f.perm_a, f.perm_b, (int64_t)W, 0, 64, s)))
@@ -206,12 +217,14 @@ cudaError_t launch_group_full(const TraceDev& t, const uint32_t* bbv16, const Fu
   tb = f.cub_bytes;
   if ((e = cub::DeviceScan::InclusiveSum(f.cub, tb, f.flag, f.gid, (int64_t)W, s))) return e;
   cudaMemsetAsync(ht.hkey, 0, sizeof(uint64_t) * (ht.mask + 1), s);
-  cudaMemsetAsync(ht.count, 0, sizeof(uint32_t) * (ht.mask + 1), s);
   note_launch(), k_full_groups<<<grid_for(W, 256), 256, 0, s>>>(W, perm, f.flag, f.gid, f.kid, bbv16, ht, f.gstart,
                                                                f.wgroup);
+  note_launch(), k_full_counts<<<grid_for(W, 256), 256, 0, s>>>(W, f.gid, f.gstart, ht);
+  // every warp's events sorted (by warp, then BB id): one radix sort of (warp << 16 | bb) over the bits in use
+  int wbits = 1;
+  while (wbits < 48 && (1ull << wbits) < W) ++wbits;
   tb = f.cub_bytes;
-  if ((e = cub::DeviceSegmentedSort::SortKeys(f.cub, tb, t.bb, f.sorted, (int64_t)t.E, (int64_t)W, t.weo, t.weo + 1,
-                                              s)))
+  if (t.E && (e = cub::DeviceRadixSort::SortKeys(f.cub, tb, f.ekey, f.sorted, (int64_t)t.E, 0, 16 + wbits, s)))
     return e;
   note_launch(), k_full_verify<<<hg, 256, 0, s>>>(W, perm, f.flag, f.gid, f.gstart, t.weo, t.E, f.sorted, err);
   if ((e = launch_canonicalise(ht, t.K, t.kwo, nullptr, out, cw, err, num_sms, s))) return e;
