@@ -31,7 +31,7 @@ CONFIG_DESC = {1: "C1 tiny", 2: "C2 micro mix (10 VADD + 10 GEMM, 64K warps each
 def parse():
     p = argparse.ArgumentParser()
     p.add_argument("--gpus", type=int, default=1)
-    p.add_argument("--steps", type=int, default=20)
+    p.add_argument("--steps", type=int, default=200)  # ~0.5 s timed: several nvidia-smi clock samples
     p.add_argument("--warmup", type=int, default=5)
     p.add_argument("--impl", default="photon", choices=["photon", "reference"])
     p.add_argument("--config", type=int, default=5)
