@@ -256,10 +256,12 @@ PHOTON_API int photon_warp_stable(photon_ctx *ctx, const photon_timing *warps, c
  * first_stable[k][bb_e] >= 0 (photon_bb_stable's outputs; the predicted time is pred_dur_sum[w] / n ticks), and
  * unpredicted[w] = the number of w's events whose type never became stable (rare BBs: the interval model of
  * L231-245, out of scope) [N3-b].  ERANGE: bb >= n_bb (index = event), a warp sum >= 2^64 or decreasing
- * warp_event_off (index = warp).  ws >= 256 bytes (error latch). */
+ * warp_event_off (index = warp).  ws >= photon_bb_predict_workspace_bytes(trace) (error latch + a work list of
+ * the long warps). */
 PHOTON_API int photon_kernel_predict(photon_ctx *ctx, uint32_t n_kernels, const int64_t *match, const uint64_t *mass,
                                      const uint64_t *full_insts, const uint64_t *full_cycles, void *ws, size_t ws_bytes,
                                      uint64_t *pred_insts, uint64_t *pred_cycles, void *stream);
+PHOTON_API size_t photon_bb_predict_workspace_bytes(const photon_trace *trace);
 PHOTON_API int photon_bb_predict(photon_ctx *ctx, const photon_trace *trace, const int64_t *first_stable /*[K][B]*/,
                                  const uint64_t *stable_dur_sum /*[K][B]*/, void *ws, size_t ws_bytes,
                                  uint64_t *pred_dur_sum /*[W]*/, uint32_t *unpredicted /*[W]*/, void *stream);

@@ -95,6 +95,7 @@ _SIGS = [
                                    c_void_p, c_void_p, c_void_p]),
     ("photon_kernel_predict", c_int, [c_void_p, c_uint32, c_void_p, c_void_p, c_void_p, c_void_p, c_void_p,
                                       c_size_t, c_void_p, c_void_p, c_void_p]),
+    ("photon_bb_predict_workspace_bytes", c_size_t, [POINTER(Trace)]),
     ("photon_bb_predict", c_int, [c_void_p, POINTER(Trace), c_void_p, c_void_p, c_void_p, c_size_t, c_void_p,
                                   c_void_p, c_void_p]),
     ("photon_group_full_workspace_bytes", c_size_t, [POINTER(Trace)]),

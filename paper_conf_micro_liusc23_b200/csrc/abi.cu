@@ -835,21 +835,34 @@ int photon_kernel_predict(photon_ctx* ctx, uint32_t K, const int64_t* match, con
   return PHOTON_OK;
 }
 
+size_t photon_bb_predict_workspace_bytes(const photon_trace* t) {
+  if (!t) return 0;
+  Carver c(nullptr);
+  c.take<DevErr>(1);
+  c.take<uint32_t>(4);
+  c.take<uint64_t>(t->n_warps + 1);
+  return c.off + 256;
+}
+
 int photon_bb_predict(photon_ctx* ctx, const photon_trace* t, const int64_t* first_stable, const uint64_t* dur,
                       void* ws, size_t ws_bytes, uint64_t* pred, uint32_t* unpred, void* stream) {
   if (!ctx) return PHOTON_EINVAL;
   int rc = check_trace(ctx, t);
   if (rc) return rc;
   if (!first_stable || !dur || !pred || !unpred || !ws) return fail(ctx, PHOTON_EINVAL, "NULL argument");
-  if (ws_bytes < 256) return fail(ctx, PHOTON_EWORKSPACE, "bb_predict workspace must be >= 256 bytes");
+  const size_t need = photon_bb_predict_workspace_bytes(t);
+  if (ws_bytes < need) return fail(ctx, PHOTON_EWORKSPACE, "workspace %zu < %zu bytes", ws_bytes, need);
+  Carver c(ws);
+  DevErr* err = c.take<DevErr>(1);
+  uint32_t* n_long = c.take<uint32_t>(4);
+  uint64_t* long_list = c.take<uint64_t>(t->n_warps + 1);
   cudaStream_t s = (cudaStream_t)stream;
   CK(cudaSetDevice(ctx->device), "cudaSetDevice");
   ctx->last_ws = ws;
-  DevErr* err = (DevErr*)ws;
   CK(cudaMemsetAsync(err, 0, sizeof(DevErr), s), "memset");
   TraceDev d = to_dev(t);
   CK(launch_validate_offsets(d, err, s), "validate");
-  CK(launch_bb_predict(d, first_stable, dur, pred, unpred, err, ctx->num_sms, s), "bb_predict");
+  CK(launch_bb_predict(d, first_stable, dur, pred, unpred, long_list, n_long, err, ctx->num_sms, s), "bb_predict");
   return PHOTON_OK;
 }
 

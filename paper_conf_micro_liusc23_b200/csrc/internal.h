@@ -173,7 +173,8 @@ cudaError_t launch_kernel_predict(uint32_t K, const int64_t* match, const uint64
                                   const uint64_t* full_cycles, uint64_t* pred_insts, uint64_t* pred_cycles,
                                   DevErr* err, cudaStream_t s);
 cudaError_t launch_bb_predict(const TraceDev& t, const int64_t* first_stable, const uint64_t* dur, uint64_t* pred,
-                              uint32_t* unpred, DevErr* err, int num_sms, cudaStream_t s);
+                              uint32_t* unpred, uint64_t* long_list, uint32_t* n_long, DevErr* err, int num_sms,
+                              cudaStream_t s);
 cudaError_t launch_stable(const photon_timing& t, const uint64_t* kbb, photon_stable_params p, void* ws,
                           size_t ws_bytes, int64_t* first_stable, uint64_t* dur, int64_t* switch_at, DevErr* err,
                           int num_sms, cudaStream_t s);

@@ -8,7 +8,8 @@
 // blocks"; a stable type's time is its mean at the latch, S_n / n (A5).  pred_dur_sum[w] = sum of S_n(k, b) over
 // the warp's events of stable types, unpredicted[w] = its events of types never stable [N3-b].  A segmented sum
 // over the trace: one thread per analysed warp (the kernel's row of the A5 tables stays in L1/L2; a warp's events
-// are read in order, so each 32-byte sector is fetched once), grid-stride; u64 overflow of a warp's sum is ERANGE.
+// are read in order, so each 32-byte sector is fetched once), grid-stride; warps longer than LONG_W events go to
+// a work list that a second pass sums with one hardware warp each.  u64 overflow of a warp's sum is ERANGE.
 #include "internal.h"
 
 namespace photon {
@@ -41,12 +42,15 @@ __global__ void k_kernel_predict(uint32_t K, const int64_t* __restrict__ match, 
 // One thread per analysed warp, 256 consecutive warps per CTA step (the block's first kernel by one binary search,
 // each thread then steps forward); a thread walks its warp's events in aligned 16-byte words (eight events per
 // load, independent table loads); the trace base is 16-byte aligned (photon_trace contract).
+constexpr uint64_t LONG_W = 128;  // events above which a warp goes to the work list (pass 2; 128 measured best on C3)
+
 __global__ void __launch_bounds__(256) k_bb_predict(const uint64_t* __restrict__ kwo, uint32_t K, uint32_t B,
                                                     const uint64_t* __restrict__ weo, uint64_t W, uint64_t E,
                                                     const uint16_t* __restrict__ bb,
                                                     const int64_t* __restrict__ first_stable,
                                                     const uint64_t* __restrict__ dur, uint64_t* pred,
-                                                    uint32_t* unpred, DevErr* err) {
+                                                    uint32_t* unpred, uint64_t* long_list, uint32_t* n_long,
+                                                    DevErr* err) {
   __shared__ uint32_t s_k0;
   for (uint64_t w0 = (uint64_t)blockIdx.x * 256; w0 < W; w0 += (uint64_t)gridDim.x * 256) {
     if (threadIdx.x == 0) {  // last kernel with kwo[k] <= w0
@@ -64,6 +68,11 @@ __global__ void __launch_bounds__(256) k_bb_predict(const uint64_t* __restrict__
     if (w >= W) continue;
     while (k + 1 < K && kwo[k + 1] <= w) ++k;
     const uint64_t s = umin64(weo[w], E), e = umin64(umax64(weo[w + 1], s), E);
+    if (e - s > LONG_W) {  // a long warp: summed by a whole hardware warp in pass 2 (long warps are often
+                           // contiguous, e.g. fully connected layers, so they are spread over the grid)
+      long_list[atomicAdd(n_long, 1u)] = w | ((uint64_t)k << 40);
+      continue;
+    }
     const int64_t* fs = first_stable + (uint64_t)k * B;
     const uint64_t* ds = dur + (uint64_t)k * B;
     uint64_t lo = 0, hi = 0;  // u128 sum
@@ -114,6 +123,52 @@ __global__ void __launch_bounds__(256) k_bb_predict(const uint64_t* __restrict__
   }
 }
 
+// pass 2: one hardware warp per listed long warp (grid-stride over the list), lanes stride its events coalesced,
+// u128 shuffle reduction
+__global__ void __launch_bounds__(256) k_bb_predict_long(uint32_t B, const uint64_t* __restrict__ weo, uint64_t E,
+                                                         const uint16_t* __restrict__ bb,
+                                                         const int64_t* __restrict__ first_stable,
+                                                         const uint64_t* __restrict__ dur, uint64_t* pred,
+                                                         uint32_t* unpred, const uint64_t* __restrict__ long_list,
+                                                         const uint32_t* n_long, DevErr* err) {
+  const int lane = threadIdx.x & 31;
+  const uint32_t nl = *n_long;
+  const uint64_t nw = ((uint64_t)gridDim.x * blockDim.x) >> 5;
+  for (uint64_t j = ((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; j < nl; j += nw) {
+    const uint64_t ent = long_list[j], w = ent & ((1ull << 40) - 1), k = ent >> 40;
+    const uint64_t s = umin64(weo[w], E), e = umin64(umax64(weo[w + 1], s), E);
+    const int64_t* fs = first_stable + k * B;
+    const uint64_t* ds = dur + k * B;
+    uint64_t lo = 0, hi = 0;
+    uint32_t miss = 0;
+#pragma unroll 4
+    for (uint64_t i = s + lane; i < e; i += 32) {
+      const uint32_t bv = bb[i];
+      if (bv >= B) {
+        latch(err, PHOTON_ERANGE, (int64_t)i);
+        continue;
+      }
+      const int64_t f = fs[bv];
+      const uint64_t x = f >= 0 ? ds[bv] : 0ull;
+      miss += f < 0 ? 1u : 0u;
+      lo += x;
+      hi += lo < x;
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) {
+      const uint64_t ol = __shfl_xor_sync(0xffffffffu, lo, o), oh = __shfl_xor_sync(0xffffffffu, hi, o);
+      lo += ol;
+      hi += oh + (lo < ol);
+      miss += __shfl_xor_sync(0xffffffffu, miss, o);
+    }
+    if (lane == 0) {
+      if (hi != 0) latch(err, PHOTON_ERANGE, (int64_t)w);
+      pred[w] = lo;
+      unpred[w] = miss;
+    }
+  }
+}
+
 }  // namespace
 
 cudaError_t launch_kernel_predict(uint32_t K, const int64_t* match, const uint64_t* mass, const uint64_t* full_insts,
@@ -126,11 +181,17 @@ cudaError_t launch_kernel_predict(uint32_t K, const int64_t* match, const uint64
 }
 
 cudaError_t launch_bb_predict(const TraceDev& t, const int64_t* first_stable, const uint64_t* dur, uint64_t* pred,
-                              uint32_t* unpred, DevErr* err, int num_sms, cudaStream_t s) {
+                              uint32_t* unpred, uint64_t* long_list, uint32_t* n_long, DevErr* err, int num_sms,
+                              cudaStream_t s) {
   if (t.W == 0) return cudaSuccess;
+  cudaMemsetAsync(n_long, 0, 4, s);
   const unsigned grid = (unsigned)umin64(ceil_div(t.W, 256), (uint64_t)num_sms * 8);
   note_launch(), k_bb_predict<<<grid, 256, 0, s>>>(t.kwo, t.K, t.B, t.weo, t.W, t.E, t.bb, first_stable, dur, pred,
-                                                   unpred, err);
+                                                   unpred, long_list, n_long, err);
+  const unsigned g2 = (unsigned)umin64(ceil_div(umin64(t.W, t.E / (LONG_W + 1) + 1) * 32, 256),
+                                       (uint64_t)num_sms * 16);
+  note_launch(), k_bb_predict_long<<<g2 ? g2 : 1, 256, 0, s>>>(t.B, t.weo, t.E, t.bb, first_stable, dur, pred, unpred,
+                                                                long_list, n_long, err);
   return cudaGetLastError();
 }
 
