@@ -343,9 +343,9 @@ __global__ void k_entries_insert(TileEntries te, uint64_t n_tiles, HashTable ht,
   *out = ht_insert(ht, err, x->kernel, key, x->hash, x->count, x->first);
 }
 
-// K2c: warp_type[w] = canonical id of the warp's tile entry.  Four warps per thread (strided by the grid) so each
+// K2c: warp_type[w] = canonical id of the warp's tile entry.  Eight warps per thread (strided by the grid) so each
 // thread keeps four independent gid -> slot -> canon chains in flight.
-constexpr int REMAP_ILP = 4;
+constexpr int REMAP_ILP = 8;
 __device__ __forceinline__ uint32_t entry_slot(const TileEntries& te, uint32_t g) {
   if (!(g >> 31)) return te.tile_slot[g];
   const uint64_t j = g & 0x7FFFFFFFu;  // beyond ovf_cap only after ECAPACITY was latched
