@@ -344,7 +344,7 @@ __global__ void k_entries_insert(TileEntries te, uint64_t n_tiles, HashTable ht,
 }
 
 // K2c: warp_type[w] = canonical id of the warp's tile entry.  Eight warps per thread (strided by the grid) so each
-// thread keeps four independent gid -> slot -> canon chains in flight.
+// thread keeps eight independent gid -> slot -> canon chains in flight.
 constexpr int REMAP_ILP = 8;
 __device__ __forceinline__ uint32_t entry_slot(const TileEntries& te, uint32_t g) {
   if (!(g >> 31)) return te.tile_slot[g];
