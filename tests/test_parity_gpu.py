@@ -456,6 +456,29 @@ def test_bb_predict_random_tables(ph):
         assert np.array_equal(_np(o["unpredicted"], np.uint32), un)
 
 
+def test_bb_predict_long_warp_list(ph):
+    # warps above 128 events go to the device work list (pass 2): contiguous runs of long warps (as C3's fully
+    # connected layers) next to tiny ones, a long warp of 9000 events, a bad id inside a long warp
+    from paper_conf_micro_liusc23_b200 import PhotonError, to_device
+    rs = np.random.default_rng(7)
+    kernels = [[list(rs.integers(0, 9, 4)) for _ in range(300)],
+               [list(rs.integers(0, 9, int(rs.integers(129, 700)))) for _ in range(200)],
+               [list(rs.integers(0, 9, int(n))) for n in rs.integers(0, 200, 500)] + [list(rs.integers(0, 9, 9000))]]
+    tr = tg.trace_from_warps(kernels, bb_len=list(range(1, 10)))
+    fs = np.where(rs.random((tr.n_kernels, tr.n_bb)) < 0.7, 1, -1).astype(np.int64)
+    ds = rs.integers(1, 1 << 50, (tr.n_kernels, tr.n_bb)).astype(np.uint64)
+    o = ph.photon_bb_predict(_dev(ph, tr), to_device(fs, ph.device), to_device(ds, ph.device))
+    pd, un = oracle.bb_predict(tr, fs, ds)
+    assert np.array_equal(_np(o["pred_dur_sum"], np.uint64), pd)
+    assert np.array_equal(_np(o["unpredicted"], np.uint32), un)
+    bad = int(tr.warp_event_off[300]) + 77  # inside the first long warp
+    tr.bb = tr.bb.copy()
+    tr.bb[bad] = 9
+    with pytest.raises(PhotonError) as ei:
+        ph.photon_bb_predict(_dev(ph, tr), to_device(fs, ph.device), to_device(ds, ph.device))
+    assert ei.value.code == -3 and ei.value.index == bad
+
+
 # ---- N4: persisted signature pool (L402) -------------------------------------------------------------------
 @pytest.mark.parametrize("cfg", [6, 4])
 def test_pool_reuse(ph, cfg, tmp_path):
