@@ -330,11 +330,11 @@ __global__ void __launch_bounds__(256) k_job_scatter(photon_timing t, const uint
     uint64_t cs = a + (job - coff[k]) * JOB, ce = umin64(cs + JOB, b);
     for (int dd = lane; dd < (int)B; dd += 32) run[wid][dd] = off[(uint64_t)dd * n_jobs + job];
     __syncwarp();
-    for (uint64_t i0 = cs; i0 < ce; i0 += 128) {
-      uint32_t d[4];
-      uint64_t x[4], y[4], yp[4];
+    for (uint64_t i0 = cs; i0 < ce; i0 += 256) {
+      uint32_t d[8];
+      uint64_t x[8], y[8], yp[8];
 #pragma unroll
-      for (int u = 0; u < 4; ++u) {
+      for (int u = 0; u < 8; ++u) {
         uint64_t i = i0 + u * 32 + lane;
         bool v = i < ce;
         d[u] = v ? (uint32_t)t.bb[i] : kNone;
@@ -343,7 +343,7 @@ __global__ void __launch_bounds__(256) k_job_scatter(photon_timing t, const uint
         yp[u] = v && i > a ? t.retire[i - 1] : 0;
       }
 #pragma unroll
-      for (int u = 0; u < 4; ++u) {
+      for (int u = 0; u < 8; ++u) {
         uint64_t i = i0 + u * 32 + lane;
         uint32_t dd = d[u];
         if (dd != kNone) {
