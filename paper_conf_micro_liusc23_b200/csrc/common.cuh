@@ -178,8 +178,7 @@ __device__ __forceinline__ uint32_t ht_insert(const HashTable& ht, DevErr* err, 
       dst[1] = make_uint4(p[4], p[5], p[6], p[7]);
       dst[2] = make_uint4(p[8], p[9], p[10], p[11]);
       dst[3] = make_uint4(p[12], p[13], p[14], p[15]);
-      __threadfence();
-      st_release_u32(&ht.ready[i], 1u);
+      st_release_u32(&ht.ready[i], 1u);  // release: the key and kernel writes above are visible first
       mine = true;
     } else if (cur == h) {
       while (ld_acquire_u32(&ht.ready[i]) == 0u) {
