@@ -529,6 +529,8 @@ FullLayout full_layout(const photon_trace* t, void* base) {
   L.f.flag = c.take<uint32_t>(W);
   L.f.gid = c.take<uint32_t>(W);
   L.f.wgroup = c.take<uint32_t>(W);
+  L.f.list = c.take<uint64_t>(W);
+  L.f.nlist = c.take<uint32_t>(4);
   L.f.ekey = c.take<uint64_t>(E);
   L.f.sorted = c.take<uint64_t>(E);
   uint64_t cap = 1024;

@@ -150,6 +150,8 @@ cudaError_t launch_warp_stable(const photon_timing& t, const uint8_t* ok, uint32
 struct FullWs {
   uint64_t *h_lo, *h_hi, *k64, *g64, *gstart;  // [W]
   uint32_t *kid, *perm_a, *perm_b, *k32, *g32, *flag, *gid, *wgroup;  // [W]
+  uint64_t* list;    // [W] work list of long warps (hash pass), then of long members (verification)
+  uint32_t* nlist;   // [2] its lengths
   uint64_t* ekey;    // [E] (warp << 16 | bb) of every event
   uint64_t* sorted;  // [E] the keys sorted: each warp's events by BB id
   void* cub;

@@ -7,13 +7,15 @@
 // BBVs project equally); rows are ordered by (count desc, key asc, lowest warp asc).
 //
 // Steps (one stream, every step on the device):
-//  1. k_full_hash: one hardware warp per analysed warp; lanes sum two 64-bit mixes of each event's BB id (an
-//     order-independent 128-bit hash, = sum over b of count(b) * H(b) mod 2^64 per half) and find its kernel.
+//  1. k_full_hash_short / _long: one thread per analysed warp of <= 16 events, longer warps from a work list with
+//     one hardware warp each; two 64-bit mixes of each event's BB id are summed (an order-independent 128-bit
+//     hash, = sum over b of count(b) * H(b) mod 2^64 per half), each event's (warp << 16 | bb) key is written.
 //  2. three stable radix sorts (CUB) of the warp indices by h_lo, h_hi, kernel: groups of equal (kernel, hash) are
 //     contiguous, members in ascending warp order.
 //  3. k_full_groups: group ids (CUB scan of the boundary flags), one slot per group in a type table (kernel,
 //     projected key of the first member, count, first warp) and each warp's group.
-//  4. k_full_verify: every member is compared with its group's first warp on the per-warp SORTED event lists (one
+//  4. k_full_verify_short / k_full_verify (long members from the work list): every member is compared with its
+//     group's first warp on the per-warp SORTED event lists (one
 //     CUB radix sort of the (warp << 16 | bb) keys written in step 1): a hash collision is detected exactly and
 //     latched (PHOTON_ERANGE, index = the warp).
 //  5. the A2 canonicalisation (k_types.cu) over the group table; k_full_remap writes warp_type.
@@ -37,23 +39,71 @@ __device__ __forceinline__ uint64_t hmix(uint64_t x) {
   return x;
 }
 
-// One hardware warp per analysed warp (grid-stride): lanes read its events coalesced and sum two 64-bit mixes of
-// each BB id (the 128-bit hash of the event multiset), write each event's sort key (warp << 16 | bb), and lane 0
-// finds the warp's kernel; perm = w.
-__global__ void k_full_hash(const uint64_t* __restrict__ kwo, uint32_t K, const uint64_t* __restrict__ weo,
-                            uint64_t W, uint64_t E, const uint16_t* __restrict__ bb, uint32_t B, uint64_t* h_lo,
-                            uint64_t* h_hi, uint32_t* kid, uint32_t* perm, uint64_t* ekey, DevErr* err) {
-  const int lane = threadIdx.x & 31;
-  const uint64_t nw = ((uint64_t)gridDim.x * blockDim.x) >> 5;
-  for (uint64_t w = ((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; w < W; w += nw) {
+constexpr uint64_t FULL_LONG = 16;  // events above which a warp is handled by a whole hardware warp (work list; 16 measured best on C3)
+
+__device__ __forceinline__ void full_mix(uint32_t x, uint64_t& a, uint64_t& b) {
+  a += hmix(0x9E3779B97F4A7C15ull * (x + 1));
+  b += hmix(0xC2B2AE3D27D4EB4Full * (x + 1) + 0x165667B19E3779F9ull);
+}
+
+// one thread per analysed warp, 256 consecutive warps per CTA step (the step's first kernel by one binary search,
+// then each thread steps forward): short warps are hashed here, longer ones go to the work list
+__global__ void __launch_bounds__(256) k_full_hash_short(const uint64_t* __restrict__ kwo, uint32_t K,
+                                                         const uint64_t* __restrict__ weo, uint64_t W, uint64_t E,
+                                                         const uint16_t* __restrict__ bb, uint32_t B, uint64_t* h_lo,
+                                                         uint64_t* h_hi, uint32_t* kid, uint32_t* perm, uint64_t* ekey,
+                                                         uint64_t* list, uint32_t* nlist, DevErr* err) {
+  __shared__ uint32_t s_k0;
+  for (uint64_t w0 = (uint64_t)blockIdx.x * 256; w0 < W; w0 += (uint64_t)gridDim.x * 256) {
+    if (threadIdx.x == 0) {
+      uint32_t lo = 0, hi = K - 1;
+      while (lo < hi) {
+        const uint32_t mid = (lo + hi + 1) >> 1;
+        if (kwo[mid] <= w0) lo = mid; else hi = mid - 1;
+      }
+      s_k0 = lo;
+    }
+    __syncthreads();
+    const uint64_t w = w0 + threadIdx.x;
+    uint32_t k = s_k0;
+    __syncthreads();
+    if (w >= W) continue;
+    while (k + 1 < K && kwo[k + 1] <= w) ++k;
+    kid[w] = k;
+    perm[w] = (uint32_t)w;
+    if (weo[w + 1] < weo[w]) latch(err, PHOTON_ERANGE, (int64_t)w);
     const uint64_t s = umin64(weo[w], E), e = umin64(umax64(weo[w + 1], s), E);
-    if (lane == 0 && weo[w + 1] < weo[w]) latch(err, PHOTON_ERANGE, (int64_t)w);
+    if (e - s > FULL_LONG) {
+      list[atomicAdd(nlist, 1u)] = w;
+      continue;
+    }
+    uint64_t a = 0, b = 0;
+    for (uint64_t i = s; i < e; ++i) {
+      const uint32_t x = bb[i];
+      if (x >= B) latch(err, PHOTON_ERANGE, (int64_t)i);
+      full_mix(x, a, b);
+      ekey[i] = (w << 16) | x;
+    }
+    h_lo[w] = a;
+    h_hi[w] = b;
+  }
+}
+
+// one hardware warp per listed long warp: lanes read its events coalesced
+__global__ void k_full_hash_long(const uint64_t* __restrict__ weo, uint64_t E, const uint16_t* __restrict__ bb,
+                                 uint32_t B, uint64_t* h_lo, uint64_t* h_hi, uint64_t* ekey,
+                                 const uint64_t* __restrict__ list, const uint32_t* nlist, DevErr* err) {
+  const int lane = threadIdx.x & 31;
+  const uint32_t nl = *nlist;
+  const uint64_t nw = ((uint64_t)gridDim.x * blockDim.x) >> 5;
+  for (uint64_t j = ((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; j < nl; j += nw) {
+    const uint64_t w = list[j];
+    const uint64_t s = umin64(weo[w], E), e = umin64(umax64(weo[w + 1], s), E);
     uint64_t a = 0, b = 0;
     for (uint64_t i = s + lane; i < e; i += 32) {
       const uint32_t x = bb[i];
       if (x >= B) latch(err, PHOTON_ERANGE, (int64_t)i);
-      a += hmix(0x9E3779B97F4A7C15ull * (x + 1));
-      b += hmix(0xC2B2AE3D27D4EB4Full * (x + 1) + 0x165667B19E3779F9ull);
+      full_mix(x, a, b);
       ekey[i] = (w << 16) | x;
     }
 #pragma unroll
@@ -62,16 +112,34 @@ __global__ void k_full_hash(const uint64_t* __restrict__ kwo, uint32_t K, const 
       b += __shfl_xor_sync(0xffffffffu, b, o);
     }
     if (lane == 0) {
-      uint32_t lo = 0, hi = K - 1;  // last k with kwo[k] <= w
-      while (lo < hi) {
-        const uint32_t mid = (lo + hi + 1) >> 1;
-        if (kwo[mid] <= w) lo = mid; else hi = mid - 1;
-      }
       h_lo[w] = a;
       h_hi[w] = b;
-      kid[w] = lo;
-      perm[w] = (uint32_t)w;
     }
+  }
+}
+
+// exact verification, one thread per sorted position that is not a group start (short warps), longer ones listed
+__global__ void k_full_verify_short(uint64_t W, const uint32_t* __restrict__ perm, const uint32_t* __restrict__ flag,
+                                    const uint32_t* __restrict__ gid, const uint64_t* __restrict__ gstart,
+                                    const uint64_t* __restrict__ weo, uint64_t E, const uint64_t* __restrict__ sorted,
+                                    uint64_t* list, uint32_t* nlist, DevErr* err) {
+  const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+  for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < W; i += stride) {
+    if (flag[i]) continue;
+    const uint32_t w = perm[i], r = perm[gstart[gid[i] - 1]];
+    const uint64_t ws = umin64(weo[w], E), we = umin64(umax64(weo[w + 1], ws), E);
+    const uint64_t rs = umin64(weo[r], E), re = umin64(umax64(weo[r + 1], rs), E);
+    if (we - ws != re - rs) {
+      latch(err, PHOTON_ERANGE, (int64_t)w);  // a 128-bit hash collision, detected exactly
+      continue;
+    }
+    if (we - ws > FULL_LONG) {
+      list[atomicAdd(nlist, 1u)] = i;
+      continue;
+    }
+    bool same = true;
+    for (uint64_t j = 0; same && j < we - ws; ++j) same = (sorted[ws + j] & 0xFFFFu) == (sorted[rs + j] & 0xFFFFu);
+    if (!same) latch(err, PHOTON_ERANGE, (int64_t)w);
   }
 }
 
@@ -128,15 +196,16 @@ __global__ void k_full_counts(uint64_t W, const uint32_t* __restrict__ gid, cons
   ht.count[g] = (uint32_t)((g + 1 < G ? gstart[g + 1] : W) - gstart[g]);
 }
 
-// one hardware warp per sorted position that is not a group start: its sorted event list equals the group's first
+// one hardware warp per listed long member: its sorted event list equals the group's first
 __global__ void k_full_verify(uint64_t W, const uint32_t* __restrict__ perm, const uint32_t* __restrict__ flag,
                               const uint32_t* __restrict__ gid, const uint64_t* __restrict__ gstart,
                               const uint64_t* __restrict__ weo, uint64_t E, const uint64_t* __restrict__ sorted,
-                              DevErr* err) {
+                              const uint64_t* __restrict__ list, const uint32_t* nlist, DevErr* err) {
   const int lane = threadIdx.x & 31;
+  const uint32_t nl = *nlist;
   const uint64_t nw = ((uint64_t)gridDim.x * blockDim.x) >> 5;
-  for (uint64_t i = ((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; i < W; i += nw) {
-    if (flag[i]) continue;
+  for (uint64_t j0 = ((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; j0 < nl; j0 += nw) {
+    const uint64_t i = list[j0];
     const uint32_t w = perm[i], r = perm[gstart[gid[i] - 1]];
     const uint64_t ws = umin64(weo[w], E), we = umin64(umax64(weo[w + 1], ws), E);
     const uint64_t rs = umin64(weo[r], E), re = umin64(umax64(weo[r + 1], rs), E);
@@ -198,8 +267,12 @@ cudaError_t launch_group_full(const TraceDev& t, const uint32_t* bbv16, const Fu
   if (W == 0) return cudaSuccess;
   cudaError_t e;
   const unsigned hg = (unsigned)umin64(ceil_div(W * 32, 256), (uint64_t)num_sms * 16);
-  note_launch(), k_full_hash<<<hg, 256, 0, s>>>(t.kwo, t.K, t.weo, W, t.E, t.bb, t.B, f.h_lo, f.h_hi, f.kid, f.perm_a,
-                                                f.ekey, err);
+  const unsigned tg = (unsigned)umin64(ceil_div(W, 256), (uint64_t)num_sms * 8);
+  cudaMemsetAsync(f.nlist, 0, 8, s);
+  note_launch(), k_full_hash_short<<<tg, 256, 0, s>>>(t.kwo, t.K, t.weo, W, t.E, t.bb, t.B, f.h_lo, f.h_hi, f.kid,
+                                                     f.perm_a, f.ekey, f.list, f.nlist, err);
+  note_launch(), k_full_hash_long<<<hg, 256, 0, s>>>(t.weo, t.E, t.bb, t.B, f.h_lo, f.h_hi, f.ekey, f.list, f.nlist,
+                                                     err);
   size_t tb = f.cub_bytes;
   // stable passes: h_lo, then h_hi, then kernel (each carries the warp permutation)
   if ((e = cub::DeviceRadixSort::SortPairs(f.cub, tb, f.h_lo, f.k64, f.perm_a, f.perm_b, (int64_t)W, 0, 64, s)))
@@ -226,7 +299,10 @@ cudaError_t launch_group_full(const TraceDev& t, const uint32_t* bbv16, const Fu
   tb = f.cub_bytes;
   if (t.E && (e = cub::DeviceRadixSort::SortKeys(f.cub, tb, f.ekey, f.sorted, (int64_t)t.E, 0, 16 + wbits, s)))
     return e;
-  note_launch(), k_full_verify<<<hg, 256, 0, s>>>(W, perm, f.flag, f.gid, f.gstart, t.weo, t.E, f.sorted, err);
+  note_launch(), k_full_verify_short<<<tg, 256, 0, s>>>(W, perm, f.flag, f.gid, f.gstart, t.weo, t.E, f.sorted,
+                                                       f.list, f.nlist + 1, err);
+  note_launch(), k_full_verify<<<hg, 256, 0, s>>>(W, perm, f.flag, f.gid, f.gstart, t.weo, t.E, f.sorted, f.list,
+                                                  f.nlist + 1, err);
   if ((e = launch_canonicalise(ht, t.K, t.kwo, nullptr, out, cw, err, num_sms, s))) return e;
   if (out.warp_type)
     note_launch(), k_full_remap<<<grid_for(W, 256), 256, 0, s>>>(W, f.wgroup, cw.canon, out.warp_type);
