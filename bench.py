@@ -405,7 +405,7 @@ def run_photon(args):
         n7 = max(args.steps // 4, 3)
         f0.record(s)
         for _ in range(n7):
-            o = ph.photon_warp_group_full(d2, b16, check=False)
+            o = ph.photon_warp_group_full(d2, b16, check=False, out=o)
         f1.record(s)
         torch.cuda.synchronize()
         ph.check(o["_ws"])

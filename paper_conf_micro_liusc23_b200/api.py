@@ -270,13 +270,16 @@ class Photon:
         return dict(filter_pairs=int(st[0]), close_pairs=int(st[1]), rounds=int(st[2]), pair_capacity=int(st[3]))
 
     # -- N2: full-BBV exact grouping and tagged-stream ingest (L154, L161) -------------------------------------
-    def photon_warp_group_full(self, t: DeviceTrace, warp_bbv16=None, stream=None, check: bool = True) -> dict:
-        """Warp types keyed on the full BBV (N2); warp_bbv16 from photon_bbv_build (computed when None)."""
+    def photon_warp_group_full(self, t: DeviceTrace, warp_bbv16=None, stream=None, check: bool = True,
+                               out: Optional[dict] = None) -> dict:
+        """Warp types keyed on the full BBV (N2); warp_bbv16 from photon_bbv_build (computed when None).  `out` (a
+        previous result for the same trace) is reused instead of allocating new tables."""
         if warp_bbv16 is None:
             warp_bbv16 = self.photon_bbv_build(t, bbv16=True, insts=False, stream=stream, check=check)["warp_bbv16"]
         ct = t.c()
         ws = self.workspace("group_full", self.L.photon_group_full_workspace_bytes(ctypes.byref(ct)))
-        ty = self.alloc_types(t.n_kernels, t.n_warps, max(t.n_warps, 1))
+        cap = max(t.n_warps, 1)
+        ty = out if (out is not None and out["capacity"] >= cap) else self.alloc_types(t.n_kernels, t.n_warps, cap)
         self._rc(self.L.photon_warp_group_full(self.ctx, ctypes.byref(ct), warp_bbv16.data_ptr(), ws.data_ptr(),
                                                ws.numel(), ctypes.byref(self.types_c(ty)), self.stream_ptr(stream)))
         if check:
