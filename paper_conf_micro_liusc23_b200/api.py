@@ -488,11 +488,15 @@ class Photon:
 
     # -- the benchmarked chain ---------------------------------------------------------------------------------
     def analyse(self, t: DeviceTrace, theta=(1, 20), n_cores=64, pool_all_prior=0, want_dist=False, stream=None,
-                check: bool = True, capacity_hint: int = 0, pair_capacity: int = 0) -> dict:
+                check: bool = True, capacity_hint: int = 0, pair_capacity: int = 0, out: Optional[dict] = None) -> dict:
         """A1 -> A2 -> A3 -> A4 on one device (fused BBV + grouping pass, then canonical tables, signatures,
-        match).  With check=False nothing synchronises (errors stay latched in the returned workspaces)."""
-        ty = self.photon_warp_group(t, None, capacity_hint, stream=stream, check=check)
+        match).  With check=False nothing synchronises (errors stay latched in the returned workspaces).  `out` (a
+        previous result for the same trace) is reused instead of allocating new output tables."""
+        ty = self.photon_warp_group(t, None, capacity_hint, stream=stream, check=check, out=out)
+        mo = {"match": out["match"]} if (out is not None and out.get("match") is not None) else None
+        if mo is not None and want_dist and out.get("match_dist") is not None:
+            mo["match_dist"] = out["match_dist"]
         m = self.photon_kernel_match(t.n_kernels, ty, t.warps_total, theta, n_cores, pool_all_prior, want_dist,
-                                     pair_capacity, stream=stream, check=check)
+                                     pair_capacity, stream=stream, check=check, out=mo)
         ty.update(match=m["match"], match_dist=m.get("match_dist"), _mws=m["_ws"])
         return ty
