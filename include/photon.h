@@ -242,7 +242,7 @@ PHOTON_API int photon_warp_stable(photon_ctx *ctx, const photon_timing *warps, c
                                   photon_warp_stable_params params, void *ws, size_t ws_bytes,
                                   int64_t *switch_at /*[K]*/, uint64_t *dur_sum /*[K] or NULL*/, void *stream);
 
-/* ---- N3: kernel- and BB-level prediction (Fig 12 Step 4 / L279-281; Fig 7 Step 3 / L204) ---------------------
+/* ---- N3: kernel- and BB-level prediction (Fig 12 Step 4 / L279-281; Fig 7 Step 3, caption L201 / L208) ---------------------
  * photon_kernel_predict: for a kernel k matched to r = match[k] >= 0 (photon_kernel_match), "#insts = #insts^K' *
  * #insts_sample / #insts^K'_sample" and "the IPC of K is predicted to be the same as K'" (L279-281):
  *   pred_insts[k]  = round_half_up(full_insts[r]  * mass[k] / mass[r]),
@@ -252,11 +252,12 @@ PHOTON_API int photon_warp_stable(photon_ctx *ctx, const photon_timing *warps, c
  * (match[k] < 0) copies its own full_*.  Exact u128; ERANGE (index k) when r >= k, mass[r] = 0, mass >= 2^50 or a
  * result >= 2^64.  All arrays [K] device, caller-owned; ws >= 256 bytes (error latch).
  * photon_bb_predict: per analysed warp w of kernel k, "accumulating the predicted time of their basic blocks"
- * (L204): pred_dur_sum[w] = sum over w's events e of stable_dur_sum[k][bb_e] for the types with
+ * (L208, Fig 7 caption L201): pred_dur_sum[w] = sum over w's events e of stable_dur_sum[k][bb_e] for the types with
  * first_stable[k][bb_e] >= 0 (photon_bb_stable's outputs; the predicted time is pred_dur_sum[w] / n ticks), and
  * unpredicted[w] = the number of w's events whose type never became stable (rare BBs: the interval model of
  * L231-245, out of scope) [N3-b].  ERANGE: bb >= n_bb (index = event), a warp sum >= 2^64 or decreasing
- * warp_event_off (index = warp).  ws >= photon_bb_predict_workspace_bytes(trace) (error latch + a work list of
+ * warp_event_off (index = warp).  EINVAL when n_kernels >= 2^24 or n_warps >= 2^40 (the long-warp work list
+ * packs both ids in one u64).  ws >= photon_bb_predict_workspace_bytes(trace) (error latch + a work list of
  * the long warps). */
 PHOTON_API int photon_kernel_predict(photon_ctx *ctx, uint32_t n_kernels, const int64_t *match, const uint64_t *mass,
                                      const uint64_t *full_insts, const uint64_t *full_cycles, void *ws, size_t ws_bytes,

@@ -186,6 +186,16 @@ class Photon:
                     warp_sampling_ok=self.empty(n_kernels, "uint8"))
 
     @staticmethod
+    def _types_fit(ty: Optional[dict], n_kernels: int, n_warps: int, capacity: int) -> bool:
+        """A previous result's tables may be reused only when every array has exactly this trace's sizes (the
+        kernels write W / K / K+1 entries and up to `capacity` rows)."""
+        if ty is None or ty.get("capacity", 0) < capacity:
+            return False
+        need = dict(warp_type=n_warps, kernel_type_off=n_kernels + 1, warp_sampling_ok=n_kernels,
+                    type_key=16 * ty["capacity"], type_count=ty["capacity"], type_first_warp=ty["capacity"])
+        return all(ty.get(k) is not None and ty[k].numel() == n for k, n in need.items())
+
+    @staticmethod
     def types_c(ty: dict) -> _lib.Types:
         p = lambda k: ty[k].data_ptr() if (ty.get(k) is not None and ty[k].numel()) else None
         return _lib.Types(ty["capacity"], p("warp_type"), p("kernel_type_off"), p("type_key"), p("type_count"),
@@ -200,7 +210,7 @@ class Photon:
             nb = self.L.photon_group_workspace_bytes(ctypes.byref(ct), hint)
             ws = self.workspace("group", nb)
             cap = min(max(t.n_warps, 1), ht_capacity(hint, t.n_warps))
-            ty = out if (out is not None and out["capacity"] >= cap) else self.alloc_types(t.n_kernels, t.n_warps, cap)
+            ty = out if self._types_fit(out, t.n_kernels, t.n_warps, cap) else self.alloc_types(t.n_kernels, t.n_warps, cap)
             tc = self.types_c(ty)
             self._rc(self.L.photon_warp_group(self.ctx, ctypes.byref(ct),
                                               None if warp_bbv16 is None else warp_bbv16.data_ptr(), ws.data_ptr(),
@@ -279,7 +289,7 @@ class Photon:
         ct = t.c()
         ws = self.workspace("group_full", self.L.photon_group_full_workspace_bytes(ctypes.byref(ct)))
         cap = max(t.n_warps, 1)
-        ty = out if (out is not None and out["capacity"] >= cap) else self.alloc_types(t.n_kernels, t.n_warps, cap)
+        ty = out if self._types_fit(out, t.n_kernels, t.n_warps, cap) else self.alloc_types(t.n_kernels, t.n_warps, cap)
         self._rc(self.L.photon_warp_group_full(self.ctx, ctypes.byref(ct), warp_bbv16.data_ptr(), ws.data_ptr(),
                                                ws.numel(), ctypes.byref(self.types_c(ty)), self.stream_ptr(stream)))
         if check:
@@ -363,6 +373,18 @@ class Photon:
             v = z[k]
             out[k] = int(v) if v.ndim == 0 else self.torch.from_numpy(v).to(self.device)
         return out
+
+    def photon_gpu_bbv(self, n_kernels: int, ty: dict, stream=None, check: bool = True) -> dict:
+        """A3 (L178, Fig 5): every kernel's GPU-BBV signature g_k (sig [16T] u64 in the rows' order, so
+        sig_off = 16 * kernel_type_off) and its mass N_k = sum(g_k) (mass [K] u64), via photon_sig_build."""
+        K = n_kernels
+        o = dict(sig=self.empty(16 * ty["capacity"], "int64"), mass=self.empty(max(K, 1), "int64"))
+        ws = self.photon_sig_build(K, ty["kernel_type_off"], ty["type_key"], ty["type_count"], 0, K, o["sig"],
+                                   o["mass"], stream=stream)
+        if check:
+            self.check(ws, stream)
+        o["mass"] = o["mass"][:K]
+        return o
 
     # split form (multi-GPU driver)
     def photon_sig_build(self, K, kto, type_key, type_count, k_lo, k_hi, sig, mass, stream=None):
@@ -493,8 +515,10 @@ class Photon:
         match).  With check=False nothing synchronises (errors stay latched in the returned workspaces).  `out` (a
         previous result for the same trace) is reused instead of allocating new output tables."""
         ty = self.photon_warp_group(t, None, capacity_hint, stream=stream, check=check, out=out)
-        mo = {"match": out["match"]} if (out is not None and out.get("match") is not None) else None
-        if mo is not None and want_dist and out.get("match_dist") is not None:
+        K = t.n_kernels
+        ok = lambda k: out is not None and out.get(k) is not None and out[k].numel() == K
+        mo = {"match": out["match"]} if ok("match") else None
+        if mo is not None and want_dist and ok("match_dist"):
             mo["match_dist"] = out["match_dist"]
         m = self.photon_kernel_match(t.n_kernels, ty, t.warps_total, theta, n_cores, pool_all_prior, want_dist,
                                      pair_capacity, stream=stream, check=check, out=mo)

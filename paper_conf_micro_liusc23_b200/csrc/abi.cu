@@ -558,6 +558,8 @@ int photon_warp_group_full(photon_ctx* ctx, const photon_trace* t, const uint32_
       !out->type_first_warp || !out->warp_sampling_ok || !out->warp_type)
     return fail(ctx, PHOTON_EINVAL, "NULL argument");
   if (t->n_warps >= (1ull << 32)) return fail(ctx, PHOTON_EINVAL, "n_warps must be < 2^32");
+  if (!aligned(warp_bbv16, 16)) return fail(ctx, PHOTON_EINVAL, "warp_bbv16 must be 16-byte aligned");
+  if (!aligned(out->type_key, 16)) return fail(ctx, PHOTON_EINVAL, "type_key must be 16-byte aligned");
   const size_t need = photon_group_full_workspace_bytes(t);
   if (ws_bytes < need) return fail(ctx, PHOTON_EWORKSPACE, "workspace %zu < %zu bytes", ws_bytes, need);
   FullLayout L = full_layout(t, ws);
@@ -852,6 +854,9 @@ int photon_bb_predict(photon_ctx* ctx, const photon_trace* t, const int64_t* fir
   int rc = check_trace(ctx, t);
   if (rc) return rc;
   if (!first_stable || !dur || !pred || !unpred || !ws) return fail(ctx, PHOTON_EINVAL, "NULL argument");
+  // the long-warp work list packs (warp | kernel << 40): kernel ids must fit in 24 bits, warp ids in 40
+  if (t->n_kernels >= (1u << 24) || t->n_warps >= (1ull << 40))
+    return fail(ctx, PHOTON_EINVAL, "photon_bb_predict needs n_kernels < 2^24 and n_warps < 2^40");
   const size_t need = photon_bb_predict_workspace_bytes(t);
   if (ws_bytes < need) return fail(ctx, PHOTON_EWORKSPACE, "workspace %zu < %zu bytes", ws_bytes, need);
   Carver c(ws);

@@ -4,7 +4,7 @@
 // The IPC of K is predicted to be the same as K'", so cycles(K) = cycles(K') * N_K / N_K' with N the analysed
 // sample's instruction count (the A3 mass).  Exact u128 quotients rounded half up [N3-a]; one thread per kernel.
 //
-// BB level, Fig 7 Step 3 / L204: the remaining warps' time is "accumulating the predicted time of their basic
+// BB level, Fig 7 Step 3, caption L201 / L208: the remaining warps' time is "accumulating the predicted time of their basic
 // blocks"; a stable type's time is its mean at the latch, S_n / n (A5).  pred_dur_sum[w] = sum of S_n(k, b) over
 // the warp's events of stable types, unpredicted[w] = its events of types never stable [N3-b].  A segmented sum
 // over the trace: one thread per analysed warp (the kernel's row of the A5 tables stays in L1/L2; a warp's events
