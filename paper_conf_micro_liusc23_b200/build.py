@@ -11,7 +11,7 @@ CSRC = os.path.join(HERE, "csrc")
 ROOT = os.path.dirname(HERE)
 SO = os.path.join(HERE, "libphoton.so")
 OBJ = os.path.join(HERE, "_obj")
-SOURCES = ["abi.cu", "k_bbv.cu", "k_bbv2.cu", "k_types.cu", "k_match.cu", "k_stable.cu", "k_predict.cu", "k_pool.cu", "k_full.cu"]
+SOURCES = ["abi.cu", "k_bbv3.cu", "k_types.cu", "k_match.cu", "k_stable.cu", "k_predict.cu", "k_pool.cu", "k_full.cu"]
 HEADERS = ["common.cuh", "internal.h"]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 FLAGS = ["-gencode", "arch=compute_100a,code=sm_100a", "-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC",

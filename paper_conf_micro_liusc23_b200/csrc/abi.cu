@@ -93,9 +93,7 @@ TraceDev to_dev(const photon_trace* t) {
 // ---- workspace layouts ----------------------------------------------------------------------------------
 struct BbvWs {
   DevErr* err;
-  uint32_t* tbl;        // [P2] packed (len, bin) table
-  uint32_t* max_len;
-  ItemTable it;         // work items of the streaming pass
+  BbvTables tb;         // per-BB tables (neutral / narrow / wide) and max_len
   uint64_t* kchunk;     // [K+1] kernel_bb_insts job prefix
   size_t bytes;
 };
@@ -104,35 +102,25 @@ BbvWs bbv_layout(const photon_trace* t, void* base) {
   BbvWs w;
   w.err = c.take<DevErr>(1);
   uint32_t P2 = next_pow2_u32(t->n_bb < 16 ? 16 : t->n_bb);
-  w.tbl = c.take<uint32_t>(P2);
-  w.max_len = c.take<uint32_t>(4);
-  w.it.xs = kItemShift;
-  w.it.cap = bbv_item_cap(t->n_warps, t->n_events, kItemShift);
-  w.it.w0 = c.take<uint64_t>(w.it.cap + 1);
-  w.it.k0 = c.take<uint32_t>(w.it.cap);
-  w.it.boff = c.take<uint32_t>(bbv_n_blocks(t->n_warps) + 1);
-  w.it.split = c.take<uint32_t>(bbv_n_blocks(t->n_warps) + 1);
-  w.it.nsub = c.take<uint32_t>(bbv_n_blocks(t->n_warps) + 1);
-  w.it.part = c.take<uint32_t>(bbv_n_blocks(t->n_warps) / 256 + 2);
-  w.it.n = c.take<uint32_t>(4);
+  w.tb.neutral = c.take<uint32_t>(P2);
+  w.tb.narrow = c.take<uint32_t>(P2);
+  w.tb.wide = c.take<uint32_t>(P2);
+  w.tb.max_len = c.take<uint32_t>(4);
   w.kchunk = c.take<uint64_t>((size_t)t->n_kernels + 1);
   w.bytes = c.off + 256;
   return w;
 }
 
-constexpr uint32_t kEntriesPerTile = 8;
-
-void carve_entries(Carver& c, uint64_t n_tiles, uint64_t W, uint64_t ovf_cap, TileEntries& te) {
-  te.per_tile = kEntriesPerTile;
-  te.tile_n = c.take<uint32_t>(n_tiles + 1);
-  te.tile_ovf = c.take<uint64_t>(n_tiles + 1);
-  te.ent = c.take<TileEntry>(n_tiles * kEntriesPerTile + 1);
-  te.tile_slot = c.take<uint32_t>(n_tiles * kEntriesPerTile + 1);
-  te.ovf_cap = ovf_cap;
-  te.ovf = c.take<TileEntry>(ovf_cap);
-  te.ovf_slot = c.take<uint32_t>(ovf_cap);
-  te.ovf_count = c.take<uint64_t>(1);
-  te.gid = c.take<uint32_t>(W + 1);
+// Entry pool: one entry per distinct (kernel, key) of each 32-warp block -- at most W -- bounded by 8x the
+// type-table capacity (ECAPACITY beyond: the caller retries with a larger hint), plus room for every K1 worker's
+// partly used last block of 64 entries (<= 160 SMs x 16 workers).
+constexpr uint64_t kPoolSlack = 160ull * 16 * 64;
+void carve_entries(Carver& c, uint64_t W, uint64_t cap, EntryPool& ep) {
+  ep.cap = (W < 8 * cap ? W : 8 * cap) + kPoolSlack;
+  ep.ent = c.take<TileEntry>(ep.cap);
+  ep.slot = c.take<uint32_t>(ep.cap);
+  ep.count = c.take<uint64_t>(1);
+  ep.gid = c.take<uint32_t>(W + 1);
 }
 
 uint64_t ht_capacity(uint64_t hint, uint64_t W) {
@@ -166,13 +154,12 @@ void carve_ht(Carver& c, uint64_t cap, uint32_t K, HtWs& w) {
 struct GroupWs {
   BbvWs b;
   HtWs h;
-  TileEntries te;
+  EntryPool ep;
   size_t bytes;
 };
 GroupWs group_layout(const photon_trace* t, uint64_t hint, void* base, size_t ws_bytes) {
   GroupWs g;
   g.b = bbv_layout(t, base);
-  const uint64_t nt = g.b.it.cap;
   uint64_t cap = ht_capacity(hint, t->n_warps);
   if (base && ws_bytes) {
     // the capacity actually used is the largest power of two that fits (callers may pass a larger workspace)
@@ -180,9 +167,9 @@ GroupWs group_layout(const photon_trace* t, uint64_t hint, void* base, size_t ws
       Carver probe(nullptr);
       probe.off = g.b.bytes;
       HtWs tmp;
-      TileEntries tt;
+      EntryPool tp;
       carve_ht(probe, cap * 2, t->n_kernels, tmp);
-      carve_entries(probe, nt, t->n_warps, cap * 2, tt);
+      carve_entries(probe, t->n_warps, cap * 2, tp);
       if (probe.off + 256 > ws_bytes) break;
       cap *= 2;
     }
@@ -190,8 +177,7 @@ GroupWs group_layout(const photon_trace* t, uint64_t hint, void* base, size_t ws
   Carver c(base);
   c.off = g.b.bytes;
   carve_ht(c, cap, t->n_kernels, g.h);
-  carve_entries(c, nt, t->n_warps, cap, g.te);
-  g.te.n_items = g.b.it.n;
+  carve_entries(c, t->n_warps, cap, g.ep);
   g.bytes = c.off + 256;
   return g;
 }
@@ -390,14 +376,14 @@ int photon_bbv_build(photon_ctx* ctx, const photon_trace* t, void* ws, size_t ws
   TraceDev d = to_dev(t);
   CK(cudaMemsetAsync(w.err, 0, sizeof(DevErr), s), "memset");
   CK(launch_validate_offsets(d, w.err, s), "validate");
-  CK(launch_table_prep(d, w.tbl, w.max_len, w.it, nullptr, w.err, s), "table");
+  CK(launch_table_prep(d, w.tb, w.err, s), "table");
   if (warp_bbv16 || warp_insts) {
     ProfScope ps(ctx, PHOTON_PROF_BBV, s);
-    CK(launch_bbv(d, w.tbl, w.max_len, w.it, warp_bbv16, warp_insts, nullptr, w.err, ctx->num_sms, s), "bbv");
+    CK(launch_bbv3(d, w.tb, warp_bbv16, warp_insts, nullptr, w.err, ctx->num_sms, s), "bbv");
   }
   if (kernel_bb_insts) {
     ProfScope ps(ctx, PHOTON_PROF_KBB, s);
-    CK(launch_kernel_bb_insts(d, w.tbl, kernel_bb_insts, w.kchunk, w.err, ctx->num_sms, s), "kbb");
+    CK(launch_kernel_bb_insts(d, w.tb, kernel_bb_insts, w.kchunk, w.err, ctx->num_sms, s), "kbb");
   }
   return PHOTON_OK;
 }
@@ -431,23 +417,23 @@ int photon_warp_group(photon_ctx* ctx, const photon_trace* t, const uint32_t* wa
   {
     ProfScope ps(ctx, PHOTON_PROF_PREP, s);
     CK(launch_ht_clear(g.h.ht, s), "ht_clear");
-    CK(cudaMemsetAsync(g.te.ovf_count, 0, 8, s), "memset");
+    CK(cudaMemsetAsync(g.ep.count, 0, 8, s), "memset");
     CK(launch_validate_offsets(d, err, s), "validate");
-    CK(launch_table_prep(d, g.b.tbl, g.b.max_len, g.b.it, &g.te, err, s), "table");
+    if (!warp_bbv16) CK(launch_table_prep(d, g.b.tb, err, s), "table");
   }
   if (warp_bbv16) {
     ProfScope ps(ctx, PHOTON_PROF_GROUP_UNFUSED, s);
-    CK(launch_group_from_bbv(d, warp_bbv16, g.b.it, g.te, err, s), "group_from_bbv");
+    CK(launch_group_from_bbv(d, warp_bbv16, g.ep, err, ctx->num_sms, s), "group_from_bbv");
   } else {
     ProfScope ps(ctx, PHOTON_PROF_BBV_FUSED, s);
-    CK(launch_bbv(d, g.b.tbl, g.b.max_len, g.b.it, nullptr, nullptr, &g.te, err, ctx->num_sms, s), "bbv_fused");
+    CK(launch_bbv3(d, g.b.tb, nullptr, nullptr, &g.ep, err, ctx->num_sms, s), "bbv_fused");
   }
   {
     ProfScope ps(ctx, PHOTON_PROF_CANON, s);
-    CK(launch_entries_insert(g.te, g.b.it.cap, g.h.ht, err, s), "insert");
+    CK(launch_entries_insert(g.ep, g.h.ht, err, ctx->num_sms, s), "insert");
     CK(launch_canonicalise(g.h.ht, t->n_kernels, t->kernel_warp_off, nullptr, *out, g.h.cw, err, ctx->num_sms, s),
        "canon");
-    CK(launch_remap_entries(g.te, t->n_warps, g.h.cw.canon, out->warp_type, s), "remap");
+    CK(launch_remap_entries(g.ep, t->n_warps, g.h.cw.canon, out->warp_type, s), "remap");
   }
   return PHOTON_OK;
 }

@@ -7,7 +7,7 @@
 
 namespace photon {
 
-// ---- A1 / A2 (k_bbv.cu) -------------------------------------------------------------------------------------
+// ---- A1 / A2 (k_bbv3.cu) -------------------------------------------------------------------------------------
 struct TraceDev {
   const uint64_t* kwo;
   const uint64_t* weo;
@@ -18,74 +18,49 @@ struct TraceDev {
   uint64_t W, E;
 };
 
-// One distinct (kernel, key) of a tile, with its warp count and lowest warp (written by K1, inserted by K2a).
+// One distinct (kernel, key) of a 32-warp block, with its warp count and lowest warp (written by K1 / the unfused
+// de-duplication, merged into the global type table by k_entries_insert).  count == 0 marks an unused entry.
 struct alignas(16) TileEntry {
   uint32_t key[16];  // 16-byte aligned (vector stores)
-  uint64_t hash;
   uint64_t first;
   uint32_t kernel;
   uint32_t count;
-  uint32_t pad[2];
 };
-static_assert(sizeof(TileEntry) == 96, "TileEntry layout");
-struct TileEntries {
-  uint32_t* tile_n;      // [n_tiles] distinct keys of the tile
-  uint64_t* tile_ovf;    // [n_tiles] first overflow entry of the tile (when tile_n > per_tile)
-  TileEntry* ent;        // [n_tiles * per_tile]
-  TileEntry* ovf;        // [ovf_cap]
-  uint64_t* ovf_count;   // [1]
-  uint64_t ovf_cap;
-  uint32_t* gid;         // [W] per warp: its entry's index in ent/tile_slot (item * per_tile + e), or
-                         // 0x80000000 | overflow index
-  uint32_t* tile_slot;   // [n_tiles * per_tile] hash-table slot of each entry
-  uint32_t* ovf_slot;    // [ovf_cap]
-  uint32_t per_tile;
-  const uint32_t* n_items;  // device item count (tile_n is written for items below it)
+static_assert(sizeof(TileEntry) == 80, "TileEntry layout");
+// The pool of entries: workers take blocks of entries with one atomic on `count`; every warp records its entry.
+struct EntryPool {
+  TileEntry* ent;     // [cap]
+  uint64_t* count;    // [1] entries handed out (may exceed cap: ECAPACITY is latched)
+  uint64_t cap;
+  uint32_t* slot;     // [cap] hash-table slot of each entry (k_entries_insert)
+  uint32_t* gid;      // [W] entry index of each warp
 };
 
-// Work items of the streaming pass: the warps of each 256-warp block are split at 2^xs-event windows of the block
-// (an item = the warps whose first event falls in one window), so an item holds <= 256 warps and about 2^xs events
-// plus its last warp's length; the persistent CTAs take items from a counter (dynamic balance).
-struct ItemTable {
-  uint64_t* w0;     // [cap + 1] first warp of each item (w0[n] = W)
-  uint32_t* k0;     // [cap] kernel of each item's first warp
-  uint32_t* boff;   // [n_blocks + 1] first item of each block
-  uint32_t* split;  // [n_blocks] blocks with more than one item
-  uint32_t* nsub;   // [n_blocks] items per block
-  uint32_t* part;   // [n_blocks / 256 + 1] per-CTA item totals (scanned)
-  uint32_t* n;      // [4]: [0] item count, [1] work counter, [2] split blocks
-  uint64_t cap;
-  uint32_t xs;
+// Per-BB tables (k_table_prep): neutral (len << 4 | bin) for the BB distribution, and K1's packed entries in its
+// narrow (u16 cells) and wide (u32 cells) formats; ids in [B, P2) are marked.  P2 = next pow2 >= max(B, 16).
+struct BbvTables {
+  uint32_t* neutral;  // [P2]
+  uint32_t* narrow;   // [P2]
+  uint32_t* wide;     // [P2]
+  uint32_t* max_len;  // [1] max bb_len (device)
 };
-uint64_t bbv_n_blocks(uint64_t W);
-uint64_t bbv_item_cap(uint64_t W, uint64_t E, uint32_t xs);
-constexpr uint32_t kItemShift = 15;  // 32K-event windows
-// packed per-BB table (len << 14 | bin << 10; bit 0 marks ids in [B, P2)), P2 = next pow2 >= B; tile -> kernel
 size_t bbv_table_bytes(uint32_t B);
-// BB table + work items (+ zeroed per-item entry counts when te is given)
-cudaError_t launch_table_prep(const TraceDev& t, uint32_t* tbl, uint32_t* max_len, const ItemTable& it,
-                              const TileEntries* te, DevErr* err, cudaStream_t s);
+cudaError_t launch_table_prep(const TraceDev& t, const BbvTables& tb, DevErr* err, cudaStream_t s);
 cudaError_t launch_validate_offsets(const TraceDev& t, DevErr* err, cudaStream_t s);
-// streaming K1 (+ fused K2a de-dup when te != nullptr)
-cudaError_t launch_bbv(const TraceDev& t, const uint32_t* tbl, const uint32_t* max_len, const ItemTable& it,
-                       uint32_t* warp_bbv16, uint64_t* warp_insts, const TileEntries* te, DevErr* err, int num_sms,
-                       cudaStream_t s);
-// K1 v2 (k_bbv2.cu): lane-range accumulation with red.shared into lane-private columns; needs the BB table in
-// shared memory (next_pow2(B) <= 4096); launch_bbv dispatches to it when supported
-bool bbv2_supported(uint32_t B);
-cudaError_t launch_bbv2(const TraceDev& t, const uint32_t* tbl, const ItemTable& it, uint32_t* warp_bbv16,
-                        uint64_t* warp_insts, const TileEntries* te, DevErr* err, int num_sms, cudaStream_t s);
-// K2a de-dup from materialised BBVs (unfused path)
-cudaError_t launch_group_from_bbv(const TraceDev& t, const uint32_t* warp_bbv16, const ItemTable& it,
-                                  const TileEntries& te, DevErr* err, cudaStream_t s);
-cudaError_t launch_kernel_bb_insts(const TraceDev& t, const uint32_t* tbl, uint64_t* kbb, uint64_t* kchunk_off,
+// K1 (k_bbv3.cu): streaming BBV pass; fused with A2's per-worker de-duplication when ep != nullptr
+cudaError_t launch_bbv3(const TraceDev& t, const BbvTables& tb, uint32_t* warp_bbv16, uint64_t* warp_insts,
+                        const EntryPool* ep, DevErr* err, int num_sms, cudaStream_t s);
+// A2 de-duplication from materialised BBVs (unfused path)
+cudaError_t launch_group_from_bbv(const TraceDev& t, const uint32_t* warp_bbv16, const EntryPool& ep, DevErr* err,
+                                  int num_sms, cudaStream_t s);
+cudaError_t launch_kernel_bb_insts(const TraceDev& t, const BbvTables& tb, uint64_t* kbb, uint64_t* kchunk_off,
                                    DevErr* err, int num_sms, cudaStream_t s);
 
 // ---- A2 insertion + canonicalisation (k_types.cu) ------------------------------------------------------------
 cudaError_t launch_ht_clear(const HashTable& ht, cudaStream_t s);
-cudaError_t launch_entries_insert(const TileEntries& te, uint64_t n_tiles, const HashTable& ht, DevErr* err,
+cudaError_t launch_entries_insert(const EntryPool& ep, const HashTable& ht, DevErr* err, int num_sms,
                                   cudaStream_t s);
-cudaError_t launch_remap_entries(const TileEntries& te, uint64_t W, const uint32_t* canon, uint32_t* warp_type,
+cudaError_t launch_remap_entries(const EntryPool& ep, uint64_t W, const uint32_t* canon, uint32_t* warp_type,
                                  cudaStream_t s);
 struct CanonWs {
   uint32_t* tcount;   // [K] types per kernel

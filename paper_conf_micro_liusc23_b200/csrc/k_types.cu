@@ -301,57 +301,35 @@ __global__ void __launch_bounds__(1024) k_sort_large(HashTable ht, uint32_t K, c
   }
 }
 
-// K2a: insert every tile entry (and overflow entry) into the global table; one thread per entry slot.
-__global__ void k_entries_insert(TileEntries te, uint64_t n_tiles, HashTable ht, DevErr* err) {
-  const uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
-  const uint64_t nfix = n_tiles * te.per_tile;
-  const TileEntry* x;
-  uint32_t* out;
-  if (i < nfix) {
-    uint64_t t = i / te.per_tile, e = i % te.per_tile;
-    if (t >= *te.n_items || e >= te.tile_n[t]) return;
-    x = te.ent + i;
-    out = te.tile_slot + i;
-  } else {
-    // overflow entries (tiles with more than per_tile distinct keys): grid-stride over the device count
-    const uint64_t n = umin64(*te.ovf_count, te.ovf_cap);
-    const uint64_t stride = (uint64_t)gridDim.x * blockDim.x - nfix;
-    for (uint64_t j = i - nfix; j < n; j += stride) {
-      x = te.ovf + j;
-      if (x->count == 0u) {  // reserved by K1 but unused (no warp refers to it)
-        te.ovf_slot[j] = UINT32_MAX;
-        continue;
-      }
-      uint32_t key[16];
-      const uint4* kp = (const uint4*)x->key;
-#pragma unroll
-      for (int q = 0; q < 4; ++q) {
-        uint4 v = kp[q];
-        key[4 * q] = v.x; key[4 * q + 1] = v.y; key[4 * q + 2] = v.z; key[4 * q + 3] = v.w;
-      }
-      te.ovf_slot[j] = ht_insert(ht, err, x->kernel, key, x->hash, x->count, x->first);
+// K2a: insert every used pool entry into the global table (grid-stride over the device count; unused entries carry
+// count 0 and get no slot).
+__global__ void k_entries_insert(EntryPool ep, HashTable ht, DevErr* err) {
+  const uint64_t n = umin64(*ep.count, ep.cap);
+  const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+  for (uint64_t j = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; j < n; j += stride) {
+    const TileEntry* x = ep.ent + j;
+    if (x->count == 0u) {
+      ep.slot[j] = UINT32_MAX;
+      continue;
     }
-    return;
-  }
-  uint32_t key[16];
-  const uint4* kp = (const uint4*)x->key;
+    uint32_t key[16];
+    const uint4* kp = (const uint4*)x->key;
 #pragma unroll
-  for (int q = 0; q < 4; ++q) {
-    uint4 v = kp[q];
-    key[4 * q] = v.x; key[4 * q + 1] = v.y; key[4 * q + 2] = v.z; key[4 * q + 3] = v.w;
+    for (int q = 0; q < 4; ++q) {
+      uint4 v = kp[q];
+      key[4 * q] = v.x; key[4 * q + 1] = v.y; key[4 * q + 2] = v.z; key[4 * q + 3] = v.w;
+    }
+    ep.slot[j] = ht_insert(ht, err, x->kernel, key, hash_key(x->kernel, key), x->count, x->first);
   }
-  *out = ht_insert(ht, err, x->kernel, key, x->hash, x->count, x->first);
 }
 
-// K2c: warp_type[w] = canonical id of the warp's tile entry.  Eight warps per thread (strided by the grid) so each
+// K2c: warp_type[w] = canonical id of the warp's entry.  Eight warps per thread (strided by the grid) so each
 // thread keeps eight independent gid -> slot -> canon chains in flight.
 constexpr int REMAP_ILP = 8;
-__device__ __forceinline__ uint32_t entry_slot(const TileEntries& te, uint32_t g) {
-  if (!(g >> 31)) return te.tile_slot[g];
-  const uint64_t j = g & 0x7FFFFFFFu;  // beyond ovf_cap only after ECAPACITY was latched
-  return j < te.ovf_cap ? te.ovf_slot[j] : UINT32_MAX;
+__device__ __forceinline__ uint32_t entry_slot(const EntryPool& ep, uint32_t g) {
+  return g < ep.cap ? ep.slot[g] : UINT32_MAX;  // beyond cap only after ECAPACITY was latched
 }
-__global__ void __launch_bounds__(256) k_remap_entries(TileEntries te, uint64_t W, const uint32_t* canon,
+__global__ void __launch_bounds__(256) k_remap_entries(EntryPool ep, uint64_t W, const uint32_t* canon,
                                                        uint32_t* warp_type) {
   const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
   const uint64_t w0 = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
@@ -359,10 +337,10 @@ __global__ void __launch_bounds__(256) k_remap_entries(TileEntries te, uint64_t 
 #pragma unroll
   for (int u = 0; u < REMAP_ILP; ++u) {
     const uint64_t w = w0 + u * stride;
-    g[u] = w < W ? te.gid[w] : 0u;
+    g[u] = w < W ? ep.gid[w] : 0u;
   }
 #pragma unroll
-  for (int u = 0; u < REMAP_ILP; ++u) sl[u] = w0 + u * stride < W ? entry_slot(te, g[u]) : UINT32_MAX;
+  for (int u = 0; u < REMAP_ILP; ++u) sl[u] = w0 + u * stride < W ? entry_slot(ep, g[u]) : UINT32_MAX;
 #pragma unroll
   for (int u = 0; u < REMAP_ILP; ++u) {
     const uint64_t w = w0 + u * stride;
@@ -468,20 +446,21 @@ cudaError_t launch_canonicalise(const HashTable& ht, uint32_t K, const uint64_t*
   return cudaGetLastError();
 }
 
-cudaError_t launch_entries_insert(const TileEntries& te, uint64_t n_tiles, const HashTable& ht, DevErr* err,
+cudaError_t launch_entries_insert(const EntryPool& ep, const HashTable& ht, DevErr* err, int num_sms,
                                   cudaStream_t s) {
-  // fixed entry slots one thread each (rounded up to whole CTAs), then 64K threads striding over the overflow
-  // one thread per fixed slot, then one per possible overflow entry (the device count is unknown here)
-  uint64_t n = ceil_div(n_tiles * te.per_tile, 256) * 256 + ceil_div(te.ovf_cap, 256) * 256;
-  if (n == 0) return cudaSuccess;
-  note_launch(), k_entries_insert<<<(unsigned)ceil_div(n, 256), 256, 0, s>>>(te, n_tiles, ht, err);
+  // grid-stride over the device entry count (unknown here): enough threads for the pool, at most 16 CTAs per SM
+  uint64_t g = ceil_div(ep.cap, 256);
+  const uint64_t gmax = (uint64_t)num_sms * 16;
+  if (g > gmax) g = gmax;
+  if (g == 0) return cudaSuccess;
+  note_launch(), k_entries_insert<<<(unsigned)g, 256, 0, s>>>(ep, ht, err);
   return cudaGetLastError();
 }
 
-cudaError_t launch_remap_entries(const TileEntries& te, uint64_t W, const uint32_t* canon, uint32_t* warp_type,
+cudaError_t launch_remap_entries(const EntryPool& ep, uint64_t W, const uint32_t* canon, uint32_t* warp_type,
                                  cudaStream_t s) {
   if (W == 0) return cudaSuccess;
-  note_launch(), k_remap_entries<<<(unsigned)ceil_div(ceil_div(W, REMAP_ILP), 256), 256, 0, s>>>(te, W, canon,
+  note_launch(), k_remap_entries<<<(unsigned)ceil_div(ceil_div(W, REMAP_ILP), 256), 256, 0, s>>>(ep, W, canon,
                                                                                                  warp_type);
   return cudaGetLastError();
 }
