@@ -169,7 +169,9 @@ __device__ __forceinline__ uint32_t ht_insert(const HashTable& ht, DevErr* err, 
                                               uint64_t h, uint32_t cnt, uint64_t wmin) {
   uint64_t i = h & ht.mask;
   for (uint64_t probe = 0; probe <= ht.mask; ++probe) {
-    unsigned long long cur = atomicCAS((unsigned long long*)&ht.hkey[i], 0ull, (unsigned long long)h);
+    // a plain read first: most insertions find their key already published (no CAS round trip)
+    unsigned long long cur = *(volatile unsigned long long*)&ht.hkey[i];
+    if (cur == 0ull) cur = atomicCAS((unsigned long long*)&ht.hkey[i], 0ull, (unsigned long long)h);
     bool mine = false;
     if (cur == 0ull) {
       ht.kern[i] = k;

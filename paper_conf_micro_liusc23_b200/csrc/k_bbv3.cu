@@ -34,7 +34,15 @@ namespace photon {
 
 namespace {
 
-constexpr int WPC = 16;             // workers (hardware warps) per CTA, one CTA per SM
+#ifndef K1_WPC
+#define K1_WPC 20
+#endif
+#ifndef K1_NBUF
+#define K1_NBUF 1
+#endif
+constexpr int WPC = K1_WPC;         // workers (hardware warps) per CTA, one CTA per SM
+constexpr int NBUF = K1_NBUF;       // staging buffers per worker (2: chunk i+1 in flight during chunk i; 1: issued
+                                    // after chunk i's event loop, landing during its collect / finalisation)
 constexpr int NCOL = 64;            // columns per worker: [0, 32) lane slot-0 columns, [32, 64) block-warp pool columns
 constexpr int GRP = 4;              // workers sharing a row array (row stride GRP * NCOL * 4 = 1 KB)
 constexpr uint32_t ROWB = GRP * NCOL * 4;
@@ -269,7 +277,7 @@ __global__ void __launch_bounds__(WPC * 32, 1) k_bbv3(Args3 a) {
   }
   const uint32_t bmask = a.P2 - 1, mask4 = bmask << 2;
   WMisc* wm = (WMisc*)(smem + a.off_misc + wid * kWMiscBytes);
-  uint4* stage0 = (uint4*)(smem + a.off_stage + wid * 2 * CW * 16);
+  uint4* stage0 = (uint4*)(smem + a.off_stage + wid * NBUF * CW * 16);
   const uint32_t cw = smem_u32(smem + a.off_cells + (wid / GRP) * ROWS * ROWB) + (wid % GRP) * NCOL * 4;
   // the OR addressing needs the row array aligned to its size
   if (((cw - (wid % GRP) * NCOL * 4) & (ROWS * ROWB - 1)) != 0u) {
@@ -323,7 +331,7 @@ __global__ void __launch_bounds__(WPC * 32, 1) k_bbv3(Args3 a) {
   auto issue = [&]() {  // lane 0 only
     if (!wm->i_live) return;
     const uint32_t n = wm->i_n;
-    const uint32_t buf = n & 1u;
+    const uint32_t buf = NBUF == 2 ? (n & 1u) : 0u;
     uint4* dst = stage0 + buf * CW;
     const uint64_t cs = wm->i_cs, te = wm->i_te;
     const uint64_t a8 = cs & ~7ull;
@@ -426,9 +434,9 @@ __global__ void __launch_bounds__(WPC * 32, 1) k_bbv3(Args3 a) {
       // rel[u] = start of warp u (u < nw), rel[nw] = block end, beyond: "never" (the virtual warp after the block)
       wm->rel[lane] = lane <= nw ? my_rel : LIM;
       if (lane < 8) wm->rel[32 + lane] = lane + 32 == nw ? rel_te : LIM;
-      const uint32_t buf = n_done & 1u, par = (n_done >> 1) & 1u;
+      const uint32_t buf = NBUF == 2 ? (n_done & 1u) : 0u, par = NBUF == 2 ? ((n_done >> 1) & 1u) : (n_done & 1u);
       ++n_done;
-      if (lane == 0) issue();  // the next chunk (this block's or the next block's) into the other buffer
+      if (NBUF == 2 && lane == 0) issue();  // the next chunk (this block's or the next block's) into the other buffer
       const uint32_t nwd = (hi + 7) >> 3;
       const uint32_t Qe = ((nwd + 31) >> 5) | 1u;
       const uint32_t L = Qe * 8u, qinv = qinv_of(Qe);
@@ -532,6 +540,7 @@ __global__ void __launch_bounds__(WPC * 32, 1) k_bbv3(Args3 a) {
         }
       }
       __syncwarp();
+      if (NBUF == 1 && lane == 0) issue();  // the stage is free: the next chunk lands during collect / finalise
       // collect: lane u sums its warp's pieces (owner column, then slot 0 of each later lane it spans)
       {
         const uint32_t x0 = umax(my_rel, lo), x1 = umin(my_rel_end, hi);
@@ -796,7 +805,7 @@ Layout3 layout3(uint32_t P2, bool gtbl, int reserved) {
   const uint32_t A = M::ROWS * ROWB;  // row arrays aligned to their size (OR addressing)
   L.off_cells = up(L.off_tbl + tbl, A);
   L.off_stage = L.off_cells + (WPC / GRP) * A;
-  L.bytes = L.off_stage + WPC * 2 * 32 * M::Q * 16;
+  L.bytes = L.off_stage + WPC * NBUF * 32 * M::Q * 16;
   return L;
 }
 
