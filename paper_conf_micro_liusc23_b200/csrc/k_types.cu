@@ -301,25 +301,56 @@ __global__ void __launch_bounds__(1024) k_sort_large(HashTable ht, uint32_t K, c
   }
 }
 
-// K2a: insert every used pool entry into the global table (grid-stride over the device count; unused entries carry
-// count 0 and get no slot).
-__global__ void k_entries_insert(EntryPool ep, HashTable ht, DevErr* err) {
+// K2a: insert every used pool entry into the global table.  One hardware warp takes 32 consecutive entries (a K1
+// worker's entries are consecutive, so neighbours often share a key): equal (kernel, key) entries are grouped with
+// __match_any_sync on the hash plus an exact key check, their counts / first warps combined in shared memory, and
+// only each group's leader probes the table.  Unused entries (count 0) get no slot.
+__global__ void __launch_bounds__(256) k_entries_insert(EntryPool ep, HashTable ht, DevErr* err) {
+  __shared__ uint32_t s_cnt[256];
+  __shared__ unsigned long long s_first[256];
   const uint64_t n = umin64(*ep.count, ep.cap);
-  const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
-  for (uint64_t j = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; j < n; j += stride) {
-    const TileEntry* x = ep.ent + j;
-    if (x->count == 0u) {
-      ep.slot[j] = UINT32_MAX;
-      continue;
-    }
-    uint32_t key[16];
-    const uint4* kp = (const uint4*)x->key;
+  const uint32_t lane = threadIdx.x & 31, wb = threadIdx.x & ~31u;
+  const uint64_t nwarps = ((uint64_t)gridDim.x * blockDim.x) >> 5;
+  for (uint64_t base = (((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5) << 5; base < n; base += nwarps << 5) {
+    const uint64_t j = base + lane;
+    uint32_t key[16], k = 0, cnt = 0;
+    uint64_t first = ~0ull;
+    if (j < n) {
+      const TileEntry* x = ep.ent + j;
+      const uint4* kp = (const uint4*)x->key;
 #pragma unroll
-    for (int q = 0; q < 4; ++q) {
-      uint4 v = kp[q];
-      key[4 * q] = v.x; key[4 * q + 1] = v.y; key[4 * q + 2] = v.z; key[4 * q + 3] = v.w;
+      for (int q = 0; q < 4; ++q) {
+        const uint4 v = kp[q];
+        key[4 * q] = v.x; key[4 * q + 1] = v.y; key[4 * q + 2] = v.z; key[4 * q + 3] = v.w;
+      }
+      const uint4 m = kp[4];  // first (u64), kernel, count
+      first = ((uint64_t)m.y << 32) | m.x;
+      k = m.z;
+      cnt = m.w;
+    } else {
+#pragma unroll
+      for (int q = 0; q < 16; ++q) key[q] = 0u;
     }
-    ep.slot[j] = ht_insert(ht, err, x->kernel, key, hash_key(x->kernel, key), x->count, x->first);
+    const bool valid = cnt != 0u;
+    const uint64_t h = valid ? hash_key(k, key) : 0ull;
+    const unsigned peers = __match_any_sync(0xffffffffu, (unsigned long long)h);
+    const int leader = __ffs(peers) - 1;
+    bool eq = __shfl_sync(0xffffffffu, k, leader) == k;
+#pragma unroll
+    for (int q = 0; q < 16; ++q) eq &= (__shfl_sync(0xffffffffu, key[q], leader) == key[q]);
+    const int g = (valid && eq) ? leader : (int)lane;  // my group's representative lane
+    s_cnt[threadIdx.x] = 0u;
+    s_first[threadIdx.x] = ~0ull;
+    __syncwarp();
+    if (valid) {
+      atomicAdd(&s_cnt[wb + g], cnt);
+      atomicMin(&s_first[wb + g], (unsigned long long)first);
+    }
+    __syncwarp();
+    uint32_t slot = UINT32_MAX;
+    if (valid && g == (int)lane) slot = ht_insert(ht, err, k, key, h, s_cnt[threadIdx.x], s_first[threadIdx.x]);
+    const uint32_t gs = __shfl_sync(0xffffffffu, slot, g);
+    if (j < n) ep.slot[j] = valid ? gs : UINT32_MAX;
   }
 }
 
