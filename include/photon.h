@@ -148,7 +148,12 @@ PHOTON_API int photon_types_total(photon_ctx *ctx, const photon_types *types, ui
  * For k in launch order: cand = { r < k : r in pool, close, warp rule } where pool = representatives (kernels
  * that were not themselves matched) [P-8] or all prior kernels when pool_all_prior = 1.  cand empty => k is a
  * representative, match[k] = -1; else match[k] = argmin over cand of (|W_k - W_r|, r) [P-9] ("closest warp
- * count", L271 Step 3).  match_dist[k] = D(k, match[k]) in fp64 (rel. err < 1e-6), +inf for representatives.
+ * count", L271 Step 3).  match_dist[k] = D(k, match[k]) in fp64 (rel. err < 1e-6); for a representative the
+ * minimum D to any earlier member of the pool (warp rule ignored), +inf when there is none or N_k = 0 [P-19]
+ * (SURVEY.md §8(a) A4 output).  match_dist is a report: it never changes a decision, and NULL skips it (the
+ * representatives' minimum is an extra pass over the pool).
+ * The A3 outputs themselves (sig, N = mass; sig_off = 16 * kernel_type_off) are produced by photon_sig_build
+ * below with k_lo = 0, k_hi = K: photon_kernel_match recomputes them into its workspace.
  * Device errors: ERANGE (N_k >= 2^50, index = kernel); ECAPACITY (candidate-pair table full). */
 typedef struct {
   uint32_t theta_num, theta_den; /* theta = num/den; default 1/20; 1 <= den <= 2^20, num <= 2*den               */
@@ -162,8 +167,10 @@ PHOTON_API int photon_kernel_match(photon_ctx *ctx, uint32_t n_kernels, const ph
                         const uint64_t *warps_total /*[K]*/, photon_match_params params, void *ws, size_t ws_bytes,
                         int64_t *match /*[K]*/, double *match_dist /*[K] or NULL*/, void *stream);
 
-/* Split form of photon_kernel_match, used by the multi-GPU driver (signatures all-reduced, pair lists
- * all-gathered between the steps).  sig_build writes g and N only for kernels [k_lo, k_hi) (others untouched).
+/* A3 (L178, Fig 5) and the split form of photon_kernel_match used by the multi-GPU driver (signatures
+ * all-reduced, pair lists all-gathered between the steps).  photon_sig_build is the A3 entry point: it writes g_k
+ * (sig, u64, the rows' order: sig_off = 16 * kernel_type_off) and N_k (mass, u64) for kernels [k_lo, k_hi)
+ * (others untouched); ERANGE when N_k >= 2^50.
  * match_scan appends the close pairs (k, r) with k in [k_lo, k_hi) to pairs[] (u64: k << 32 | r), count in
  * *n_pairs (DEVICE u64, zeroed by the call); `pair_capacity` entries fit.  match_resolve takes the union of all
  * pair lists (any order) and runs the launch-order resolution; its result does not depend on pair order. */

@@ -608,6 +608,56 @@ __global__ void k_resolve_match(uint32_t K, const uint64_t* off, const uint32_t*
   }
 }
 
+// match_dist of a representative (match[k] < 0): the minimum D to any earlier member of the pool [P-8] (warp rule
+// ignored; SURVEY.md §8(a) A4 output), +inf when there is none or N_k = 0 [P-19].  One warp per kernel: an fp64
+// pass over the pool (each D within (L + 8) * 2^-50 of exact) finds the minimum, then the exact u128 numerator of
+// every candidate within twice that bound of it picks the exact minimum.  Only when match_dist is requested.
+__device__ __forceinline__ double warp_d64(const uint64_t* sig, const uint64_t* kto, const uint64_t* mass, uint32_t k,
+                                           uint32_t r, double& eps) {
+  const uint32_t lane = threadIdx.x & 31;
+  const uint64_t ok = kto[k], orr = kto[r];
+  const uint64_t Lk = (kto[k + 1] - ok) * 16, Lr = (kto[r + 1] - orr) * 16, L = Lk > Lr ? Lk : Lr;
+  const double ik = 1.0 / (double)mass[k], ir = 1.0 / (double)mass[r];
+  double acc = 0.0;
+  for (uint64_t i = lane; i < L; i += 32) {
+    const double a = i < Lk ? (double)sig[ok * 16 + i] * ik : 0.0;
+    const double b = i < Lr ? (double)sig[orr * 16 + i] * ir : 0.0;
+    acc += fabs(a - b);
+  }
+  for (int o = 16; o > 0; o >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, o);
+  eps = (double)(L + 8) * 0x1p-50;
+  return acc;
+}
+__device__ __forceinline__ double u128_to_double(u128 x) {
+  return (double)(uint64_t)(x >> 64) * 18446744073709551616.0 + (double)(uint64_t)x;
+}
+__global__ void k_rep_mindist(uint32_t K, const int64_t* match, uint32_t pool_all, const uint64_t* kto,
+                              const uint64_t* sig, const uint64_t* mass, double* dist) {
+  const uint32_t k = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  if (k >= K || match[k] >= 0) return;
+  const uint32_t lane = threadIdx.x & 31;
+  if (mass[k] == 0) return;  // +inf already written
+  double best = INFINITY, best_eps = 0.0;
+  for (uint32_t r = 0; r < k; ++r) {
+    if ((!pool_all && match[r] >= 0) || mass[r] == 0) continue;
+    double eps;
+    const double d = warp_d64(sig, kto, mass, k, r, eps);
+    if (d < best) { best = d; best_eps = eps; }
+  }
+  if (best == INFINITY) return;
+  double exact = INFINITY;
+  for (uint32_t r = 0; r < k; ++r) {
+    if ((!pool_all && match[r] >= 0) || mass[r] == 0) continue;
+    double eps;
+    const double d = warp_d64(sig, kto, mass, k, r, eps);
+    if (d > best + best_eps + eps) continue;
+    const u128 dn = warp_dnum(sig, kto, mass, k, r);
+    const double v = u128_to_double(dn) / u128_to_double((u128)mass[k] * mass[r]);
+    if (v < exact) exact = v;
+  }
+  if (lane == 0) dist[k] = exact;
+}
+
 }  // namespace
 
 cudaError_t launch_sig_build(uint32_t K, const uint64_t* kto, const uint32_t* type_key, const uint64_t* type_count,
@@ -684,6 +734,9 @@ cudaError_t launch_match_resolve(uint32_t K, const uint64_t* kto, const uint64_t
   note_launch(), k_resolve_match<<<(unsigned)ceil_div((uint64_t)K * 32, 256), 256, 0, s>>>(K, mw.cand_off, mw.cand, mw.state,
                                                                            p.pool_all_prior, wt, kto, sig, mass,
                                                                            match, match_dist);
+  if (match_dist)
+    note_launch(), k_rep_mindist<<<(unsigned)ceil_div((uint64_t)K * 32, 256), 256, 0, s>>>(K, match, p.pool_all_prior,
+                                                                                          kto, sig, mass, match_dist);
   return cudaGetLastError();
 }
 

@@ -127,6 +127,9 @@ class NumpyBackend:
                     best = c if best is None or c < best else best
             if best is None:
                 rep[k] = True
+                pool = [r for r in range(k) if (params.pool_all_prior or rep[r]) and int(m[r]) > 0]
+                if int(m[k]) > 0 and pool:  # a representative: its minimum distance to the earlier pool
+                    dist[k] = float(min(Fraction(self._dnum(g, s, m, k, r), int(m[k]) * int(m[r])) for r in pool))
             else:
                 match[k] = best[1]
                 dist[k] = float(Fraction(self._dnum(g, s, m, k, best[1]), int(m[k]) * int(m[best[1]])))

@@ -51,8 +51,8 @@ def test_worked_example_full_chain():
                               ("match_theta_2_5_cores_2", (2, 5), 2)]:
         m, d = oracle.match(t["kernel_type_off"], sig, mass, tr.warps_total, theta, cores)
         assert m.tolist() == e[key], key
-        if m[1] == 0:
-            assert d[1] == pytest.approx(e["D_AB_num"] / e["D_AB_den"], rel=1e-12)
+        # matched or not, kernel B reports D(A, B) = 216/594: its representative, else the nearest representative
+        assert d[1] == pytest.approx(e["D_AB_num"] / e["D_AB_den"], rel=1e-12)
         assert np.isinf(d[0])
 
 
@@ -277,6 +277,13 @@ def test_match_bruteforce_random(seed, theta):
         for k in range(len(kernels)):
             if m[k] >= 0:
                 assert d[k] == pytest.approx(float(_frac_dist(vecs[k], vecs[int(m[k])])), rel=1e-12)
+            else:  # a representative: the minimum D to any earlier member of the pool [P-8] (warp rule ignored)
+                pool = [r for r in range(k) if (pool_all or m[r] < 0) and int(mass[r]) > 0]
+                if int(mass[k]) == 0 or not pool:
+                    assert np.isinf(d[k])
+                else:
+                    want = min(_frac_dist(vecs[k], vecs[r]) for r in pool)
+                    assert d[k] == pytest.approx(float(want), rel=1e-12)
 
 
 def test_match_scenarios():
@@ -286,6 +293,9 @@ def test_match_scenarios():
     t, sig, mass = _pipeline(tr)
     m, d = oracle.match(t["kernel_type_off"], sig, mass, tr.warps_total)
     assert m.tolist() == [-1, 0, 0, -1] and d[1] == 0.0 and np.isinf(d[0])
+    # the representative k3 reports its distance to the only earlier representative, k0
+    v = [_frac_gpu_bbv(t, k) for k in range(4)]
+    assert d[3] == pytest.approx(float(_frac_dist(v[3], v[0])), rel=1e-12) and 0 < d[3] < 2
     # fewer warps than GPU cores (64): unequal counts never match; equal counts do (L271 Fig 12 note, L277)
     m, _ = oracle.match(t["kernel_type_off"], sig, mass, np.array([32, 33, 32, 32], np.uint64))
     assert m.tolist() == [-1, -1, 0, -1]
