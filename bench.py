@@ -39,10 +39,12 @@ def parse():
     p.add_argument("--theta", default="1/20")
     p.add_argument("--e2e-steps", type=int, default=3)
     p.add_argument("--a5-config", type=int, default=3)
+    p.add_argument("--a5-c5-kernels", type=int, default=1000, help="C5 kernel batch timed for A5 (a5_c5)")
     p.add_argument("--skip-e2e", action="store_true")
     p.add_argument("--skip-a5", action="store_true")
     p.add_argument("--skip-cpu", action="store_true")
-    p.add_argument("--cpu-kernels", type=int, default=6000, help="C5 kernel prefix timed for cpu_baseline")
+    p.add_argument("--cpu-kernels", type=int, default=3000, help="C5 kernel prefix timed for cpu_baseline")
+    p.add_argument("--skip-configs", action="store_true", help="skip the C1-C4 chain lines")
     return p.parse_args()
 
 
@@ -149,19 +151,41 @@ def run_reference(args):
     print(json.dumps(line), flush=True)
 
 
+def _cpu_model():
+    try:
+        with open("/proc/cpuinfo") as f:
+            for line in f:
+                if line.startswith("model name"):
+                    return line.split(":", 1)[1].strip()
+    except OSError:
+        pass
+    return None
+
+
 def cpu_baseline(args):
+    """The oracle as it stands on the box's host cores: the plain single-threaded chain, and the
+    same oracle functions with the per-kernel steps (A1-A3) of kernel ranges on every host core (A4's launch-order
+    match stays sequential).  A bounded sample of the workload (a C5 kernel prefix)."""
     import oracle
     import tracegen as tg
     g = tg.Generator(args.config, args.seed)
     k1 = min(g.n_kernels, args.cpu_kernels) if args.config == 5 else g.n_kernels
     tr = g.kernels_trace(0, k1)
     num, den = (int(x) for x in args.theta.split("/"))
+    cores = len(os.sched_getaffinity(0))
     t0 = time.perf_counter()
     oracle.analyse(tr, theta=(num, den))
-    dt = time.perf_counter() - t0
-    return {"value": tr.n_events / dt, "unit": "events/s", "cores": 1, "kind": "oracle",
-            "sample": f"kernels [0,{k1}) of {CONFIG_DESC.get(args.config)}: {tr.n_events} events in {dt:.1f} s "
-                      f"(single-threaded C++ oracle, full chain A1-A4)"}
+    dt1 = time.perf_counter() - t0
+    t0 = time.perf_counter()
+    oracle.analyse_threads(tr, cores, theta=(num, den))
+    dtn = time.perf_counter() - t0
+    sample = f"kernels [0,{k1}) of {CONFIG_DESC.get(args.config)}: {tr.n_events} events"
+    return {"value": tr.n_events / dt1, "unit": "events/s", "cores": 1, "kind": "oracle",
+            "sample": f"{sample} in {dt1:.1f} s (single-threaded C++ oracle, full chain A1-A4)",
+            "cpu_model": _cpu_model(), "host_cores": cores,
+            "all_cores": {"value": tr.n_events / dtn, "unit": "events/s", "cores": cores,
+                          "sample": f"{sample} in {dtn:.1f} s (A1-A3 over kernel ranges on {cores} threads, "
+                                    "A4 match sequential)"}}
 
 
 def run_photon(args):
@@ -253,11 +277,14 @@ def run_photon(args):
     k1_ms = pms[0] / max(int(pcnt[0]), 1)
     k1_bytes = 2 * tr.n_events + 8 * (tr.n_warps + 1) + 4 * tr.n_warps  # algorithmic: bb + offsets + warp type
     achieved = k1_bytes / (k1_ms / 1000) / 1e9
-    roofline = {"bound": "hbm", "kernel": "k_bbv2 (fused A1+A2 streaming pass)", "achieved": achieved,
+    chain_gbps = (2 * E_total + 12 * W_total) / (ms / 1000) / 1e9
+    roofline = {"bound": "hbm", "kernel": "k_bbv3 (fused A1+A2 streaming pass)", "achieved": achieved,
                 "peak": hbm_peak, "peak_source": peak_src, "unit": "GB/s", "frac": achieved / hbm_peak,
+                "frac_nominal_8TBps": achieved / 8000.0,
                 "traffic": _traffic(args.config), "algorithmic_bytes_per_launch": k1_bytes,
                 "k1_ms": k1_ms, "k1_share_of_step": (pms[0] / args.steps) / ms if ms else None,
-                "chain_algorithmic_GBps": (2 * E_total + 12 * W_total) / (ms / 1000) / 1e9}
+                "chain_algorithmic_GBps": chain_gbps, "chain_frac": chain_gbps / hbm_peak,
+                "chain_frac_nominal_8TBps": chain_gbps / 8000.0}
     value = E_total / (ms / 1000)
 
     line = {"metric": METRIC, "value": value, "unit": "events/s", "n_gpus": ws, "steps": args.steps,
@@ -267,7 +294,9 @@ def run_photon(args):
             "config": {"workload": CONFIG_DESC.get(args.config), "events": E_total, "warps": W_total,
                        "kernels": g.n_kernels, "bb_ids": g.n_bb, "theta": args.theta,
                        "parallelism": f"dp{ws} (warp shards)" if ws > 1 else "1 GPU",
-                       "l2": f"inputs ({(2 * E_total + 8 * W_total) / 1e9:.2f} GB) exceed the 126 MB L2; no flush"},
+                       "l2": f"inputs ({(2 * E_total + 8 * W_total) / 1e9:.2f} GB) exceed the 126 MB L2; no flush",
+                       "match_dist": "not requested in the timed chain (the metric counts decisions; the reported "
+                                     "distances are a separate pass)"},
             "roofline": roofline, "sections": sections, "clocks": clk, "gpu_launches": int(launches)}
 
     # ---- e2e: the same chain through the API with host (pinned) inputs; H2D + D2H inside the timed region ----
@@ -310,6 +339,49 @@ def run_photon(args):
             e2e_ms = float(t.item())
         line["e2e"] = {"value": E_total / (e2e_ms / 1000), "unit": "events/s", "h2d_bytes_per_step": int(h2d),
                        "d2h_bytes_per_step": int(d2h), "ms_per_step": e2e_ms, "steps": args.e2e_steps}
+
+    # ---- the metric's chain on C1-C4 (C2 also with a 2x-L2 scrub between steps: its HBM fraction) ----
+    if not args.skip_configs and ws == 1:
+        import ctypes as _ct
+        line["configs"] = {}
+        for cfg, scrub in ((1, 0), (2, 0), (2, 256 << 20), (3, 0), (4, 0)):
+            gc = tg.Generator(cfg)
+            tc = gc.trace()
+            dc = DeviceTrace.from_host(tc, dev)
+            rc = ph.analyse(dc, theta=(num, den))
+            for _ in range(max(args.warmup - 1, 0)):
+                rc = ph.analyse(dc, theta=(num, den), check=False, out=rc)
+            buf = torch.empty(scrub // 4, dtype=torch.int32, device=dev) if scrub else None
+            nst = max(args.steps // 4, 5)
+            torch.cuda.synchronize()
+            L.photon_profile(ph.ctx, 1)
+            tot = 0.0
+            for i in range(nst):
+                if buf is not None:
+                    buf.fill_(i)  # evicts the trace from the 126 MB L2 (outside the timed events)
+                c0, c1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                c0.record(s)
+                rc = ph.analyse(dc, theta=(num, den), check=False, out=rc)
+                c1.record(s)
+                c1.synchronize()
+                tot += c0.elapsed_time(c1)
+            cms = (_ct.c_double * 16)()
+            ccnt = (_ct.c_uint64 * 16)()
+            L.photon_profile_read(ph.ctx, ph.stream_ptr(), cms, ccnt)
+            L.photon_profile(ph.ctx, 0)
+            ph.check(rc["_ws"])
+            cm = tot / nst
+            k1c = cms[0] / max(int(ccnt[0]), 1)
+            kb = 2 * tc.n_events + 12 * tc.n_warps + 8
+            name = f"C{cfg}" + ("_l2scrub" if scrub else "")
+            line["configs"][name] = {
+                "workload": CONFIG_DESC.get(cfg), "events": tc.n_events, "warps": tc.n_warps,
+                "kernels": tc.n_kernels, "ms_per_step": cm, "value": tc.n_events / (cm / 1000), "unit": "events/s",
+                "k1_ms": k1c, "k1_frac": kb / (k1c / 1000) / 1e9 / hbm_peak,
+                "chain_frac": kb / (cm / 1000) / 1e9 / hbm_peak,
+                "l2": ("2x-L2 scrub (256 MB written) before every step, outside the timed region" if scrub else
+                       "no flush (inputs " + ("< 126 MB L2" if kb < 126e6 else "> 126 MB L2") + ")")}
+            del dc, rc, buf
 
     # ---- A5 on its own timing stream (reported beside the metric) ----
     if not args.skip_a5 and ws == 1:
@@ -364,6 +436,36 @@ def run_photon(args):
                                    "unit": "GB/s", "frac": abytes / (ams / 1000) / 1e9 / hbm_peak,
                                    "algorithmic_bytes": abytes, "traffic": None},
                       "stable_bb_types": int((to_numpy_i64(o["first_stable"]) >= 0).sum())}
+
+    # ---- A5 on C5 stress kernels (B = 4096 > 256: the composite-key radix path), a kernel batch ----
+    if not args.skip_a5 and ws == 1:
+        g5 = tg.Generator(5)
+        k5 = min(args.a5_c5_kernels, g5.n_kernels)
+        tm5 = g5.timing(0, k5)
+        d5 = DeviceTrace.from_host(g5.kernels_trace(0, k5), dev)
+        kbb5 = ph.photon_bbv_build(d5, bbv16=False, insts=False, kbb=True)["kernel_bb_insts"]
+        dt5 = DeviceTiming.from_host(tm5, dev)
+        o5 = ph.photon_bb_stable(dt5, kbb5, 2048)
+        for _ in range(max(args.warmup - 1, 0)):
+            o5 = ph.photon_bb_stable(dt5, kbb5, 2048, check=False, out=o5)
+        torch.cuda.synchronize()
+        h0, h1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        n8 = max(args.steps // 8, 3)
+        h0.record(s)
+        for _ in range(n8):
+            o5 = ph.photon_bb_stable(dt5, kbb5, 2048, check=False, out=o5)
+        h1.record(s)
+        torch.cuda.synchronize()
+        ph.check(o5["_ws"])
+        a5ms = h0.elapsed_time(h1) / n8
+        R5 = tm5.n_records
+        line["a5_c5"] = {"metric": "BB timing records tested/sec (stability test + switch)",
+                         "value": R5 / (a5ms / 1000), "unit": "records/s", "ms_per_step": a5ms, "records": R5,
+                         "workload": f"C5 stress kernels [0, {k5}) timing stream, n=2048, delta=3/100 (B = 4096)",
+                         "roofline": {"bound": "hbm", "achieved": 18 * R5 / (a5ms / 1000) / 1e9, "peak": hbm_peak,
+                                      "unit": "GB/s", "frac": 18 * R5 / (a5ms / 1000) / 1e9 / hbm_peak,
+                                      "algorithmic_bytes": 18 * R5, "traffic": None}}
+        del dt5, o5, d5, kbb5
 
     # ---- N1 (warp-level stability, L262) on the same config's warp streams, gated by A2's dominance ----
     if not args.skip_a5 and ws == 1:

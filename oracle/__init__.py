@@ -283,6 +283,55 @@ def match_pooled(pool, types, warps_total, theta=(1, 20), n_cores=64, pool_all_p
     return match(comb_kto, sig, mass, wt, theta, n_cores, pool_all_prior)
 
 
+def _kernel_slice(trace, k0, k1):
+    """Kernels [k0, k1) of a trace as a trace of their own (offsets rebased; arrays are views)."""
+    from types import SimpleNamespace
+    kwo = np.asarray(trace.kernel_warp_off, np.uint64)
+    weo = np.asarray(trace.warp_event_off, np.uint64)
+    w0, w1 = int(kwo[k0]), int(kwo[k1])
+    e0, e1 = int(weo[w0]), int(weo[w1])
+    t = SimpleNamespace(kernel_warp_off=kwo[k0:k1 + 1] - kwo[k0], warp_event_off=weo[w0:w1 + 1] - weo[w0],
+                        bb=np.asarray(trace.bb)[e0:e1], bb_len=trace.bb_len, bb_bin=trace.bb_bin,
+                        warps_total=np.asarray(trace.warps_total)[k0:k1])
+    t.n_kernels, t.n_warps, t.n_events, t.n_bb = k1 - k0, w1 - w0, e1 - e0, len(trace.bb_len)
+    return t, w0
+
+
+def analyse_threads(trace, threads, theta=(1, 20), n_cores=64, pool_all_prior=0):
+    """analyse() with the per-kernel steps (A1 BBVs, A2 grouping, A3 signatures) of contiguous kernel ranges run on
+    `threads` host threads (the C calls release the GIL), then the launch-order match (A4) on one thread.  The
+    all-cores CPU baseline of bench.py; results are identical to analyse()."""
+    from concurrent.futures import ThreadPoolExecutor
+    K = trace.n_kernels
+    weo = np.asarray(trace.warp_event_off, np.uint64)
+    kwo = np.asarray(trace.kernel_warp_off, np.uint64)
+    kev = weo[kwo.astype(np.int64)].astype(np.float64)  # first event of each kernel (and the end)
+    cuts = sorted(set([0, K] + [int(np.searchsorted(kev, trace.n_events * i / threads)) for i in range(1, threads)]))
+    cuts = [min(max(c, 0), K) for c in cuts]
+
+    def part(i):
+        sub, w0 = _kernel_slice(trace, cuts[i], cuts[i + 1])
+        p16, _, _ = bbv(sub, want_kbb=False)
+        t = group(sub, p16)
+        sig, mass = signature(t["kernel_type_off"], t["type_key"], t["type_count"])
+        return t, sig, mass, w0
+
+    with ThreadPoolExecutor(max_workers=threads) as ex:
+        parts = list(ex.map(part, range(len(cuts) - 1)))
+    kto, keys, cnts, firsts, wtype, ok, sigs, masses = [np.zeros(1, np.uint64)], [], [], [], [], [], [], []
+    for t, sig, mass, w0 in parts:
+        kto.append(kto[-1][-1] + t["kernel_type_off"][1:])
+        keys.append(t["type_key"]); cnts.append(t["type_count"]); firsts.append(t["type_first_warp"] + np.uint64(w0))
+        wtype.append(t["warp_type"]); ok.append(t["warp_sampling_ok"]); sigs.append(sig); masses.append(mass)
+    out = dict(kernel_type_off=np.concatenate(kto), type_key=np.concatenate(keys), type_count=np.concatenate(cnts),
+               type_first_warp=np.concatenate(firsts), warp_type=np.concatenate(wtype),
+               warp_sampling_ok=np.concatenate(ok))
+    sig, mass = np.concatenate(sigs), np.concatenate(masses)
+    m, d = match(out["kernel_type_off"], sig, mass, trace.warps_total, theta, n_cores, pool_all_prior)
+    out.update(sig=sig, mass=mass, match=m, match_dist=d)
+    return out
+
+
 def analyse(trace, theta=(1, 20), n_cores=64, pool_all_prior=0):
     """The benchmarked chain A1 -> A2 -> A3 -> A4 on one trace; returns a dict of every output."""
     p16, ins, kbb = bbv(trace, want_kbb=False)

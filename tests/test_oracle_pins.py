@@ -781,3 +781,23 @@ def test_ingest_interleaved_stream():
         assert np.array_equal(bb[warp == w], tr.bb[weo[w]:weo[w + 1]])
     out_bb, off = oracle.ingest(warp, bb, W)
     assert np.array_equal(off, tr.warp_event_off.astype(np.uint64)) and np.array_equal(out_bb, tr.bb)
+
+
+# ---------------------------------------------------------------------------------------------------------------
+# The all-cores CPU baseline (bench.py cpu_baseline): the same oracle functions over kernel ranges on host threads
+# must give exactly analyse()'s tables and decisions.
+@pytest.mark.parametrize("which", ["c6", "c4", "random"])
+def test_analyse_threads_equals_analyse(which):
+    if which == "random":
+        tr = tg.random_trace(3, n_kernels=7, max_warps=300, max_events=60, n_bb=40)
+    else:
+        tr = tg.make_trace(6 if which == "c6" else 4)
+    a = oracle.analyse(tr)
+    for threads in (1, 3, 8):
+        b = oracle.analyse_threads(tr, threads)
+        for k in ("kernel_type_off", "type_key", "type_count", "type_first_warp", "warp_type", "warp_sampling_ok",
+                  "sig", "mass", "match"):
+            assert np.array_equal(np.asarray(a[k]), np.asarray(b[k])), (k, threads)
+        assert np.array_equal(np.isinf(a["match_dist"]), np.isinf(b["match_dist"]))
+        fin = np.isfinite(a["match_dist"])
+        assert np.array_equal(a["match_dist"][fin], b["match_dist"][fin])
