@@ -279,21 +279,148 @@ __global__ void k_fill_gstart(const uint64_t* key, uint64_t n, uint64_t G, uint6
 
 constexpr uint32_t kNone = 0xFFFFFFFFu;  // padding lane (not a u16 id)
 
-// ---- 2'. one-pass stable multisplit for B <= 256 (the common case): one warp per job = (kernel, JOB records) --
-// Records of a job belong to one kernel, so a stable split by bb inside each job, with job offsets from a
-// bin-major scan of the per-job histograms, leaves group (b, k) contiguous, in retirement order, at
-// hist[b][first job of k] -- the group id g = b*K + k needs no key array.
-__global__ void __launch_bounds__(256) k_job_hist(photon_timing t, const uint64_t* coff, uint64_t n_jobs,
-                                                  uint32_t* hist) {
-  __shared__ uint32_t h[8][256];
+// ---- 2'. one-pass stable multisplit: one warp per job = (kernel, JOB records) --------------------------------
+// Records of a job belong to one kernel, so a stable split by BB inside each job, with job offsets from a scan of
+// the per-job histograms laid out kernel-major ((k, l, job) with l the kernel-local BB id), leaves every group
+// (k, l) contiguous, in retirement order.  Local ids: B <= 256 -- the BB id itself (B_k = B, group g = k*B + b);
+// 256 < B <= kCompactMaxB -- the rank of b among the BB ids present in kernel k's stream (a presence bitmap per
+// kernel; C5 kernels use 16 of 4096 ids), groups g = goff[k] + l.  Kernels with more than 256 local ids keep their
+// histogram / running offsets in global memory (atomics, still stable) instead of shared memory.
+constexpr uint32_t kCompactMaxB = 8192;
+constexpr uint32_t kSmemBins = 256;
+struct JobMap {
+  const uint64_t* coff;  // [K+1] jobs per kernel (scanned)
+  const uint32_t* bits;  // compact: [K][nw] presence bitmap
+  const uint32_t* lbase; // compact: [K][nw] local ids before each word
+  const uint32_t* bk;    // compact: [K] local ids of kernel k
+  const uint64_t* hb;    // compact: [K+1] first histogram entry of kernel k (scanned B_k * jobs_k)
+  uint32_t nw;           // words per kernel bitmap
+  bool compact;
+  uint64_t hcap;         // histogram entries available (compact: the device total must fit, else ECAPACITY)
+  __device__ __forceinline__ bool fits() const { return !compact || hb[nkern] <= hcap; }
+  uint32_t nkern;
+  __device__ __forceinline__ uint32_t nbins(uint32_t k, uint32_t B) const { return compact ? bk[k] : B; }
+  __device__ __forceinline__ uint64_t hbase(uint32_t k, uint32_t B) const { return compact ? hb[k] : (uint64_t)B * coff[k]; }
+  __device__ __forceinline__ uint32_t lid(uint32_t k, uint32_t b) const {
+    if (!compact) return b;
+    const uint64_t w = (uint64_t)k * nw + (b >> 5);
+    return lbase[w] + __popc(bits[w] & ((1u << (b & 31)) - 1u));
+  }
+};
+
+// presence bitmap per kernel (compact ids): one warp per job ORs its BB ids into a shared bitmap, then into global
+__global__ void __launch_bounds__(256) k_presence(photon_timing t, const uint64_t* coff, uint64_t n_jobs, uint32_t nw,
+                                                  uint32_t* bits) {
+  extern __shared__ uint32_t pm[];  // [8][nw]
   const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
-  const uint32_t B = t.n_bb;
-  for (int d = lane; d < (int)B; d += 32) h[wid][d] = 0;
+  uint32_t* m = pm + wid * nw;
+  for (uint32_t w = lane; w < nw; w += 32) m[w] = 0u;
   __syncwarp();
   for (uint64_t job = (uint64_t)blockIdx.x * 8 + wid; job < n_jobs; job += (uint64_t)gridDim.x * 8) {
-    uint32_t k = upper_idx(coff, t.n_kernels, job);
-    uint64_t a = umin64(t.kernel_rec_off[k], t.n_records), b = umin64(t.kernel_rec_off[k + 1], t.n_records);  // clamped: bad offsets are latched by k_rec_chunks
-    uint64_t cs = a + (job - coff[k]) * JOB, ce = umin64(cs + JOB, b);
+    const uint32_t k = upper_idx(coff, t.n_kernels, job);
+    const uint64_t a = umin64(t.kernel_rec_off[k], t.n_records), e = umin64(t.kernel_rec_off[k + 1], t.n_records);
+    const uint64_t cs = a + (job - coff[k]) * JOB, ce = umin64(cs + JOB, e);
+    for (uint64_t i = cs + lane; i < ce; i += 32) {
+      uint32_t bb = t.bb[i];
+      if (bb >= t.n_bb) bb = 0;  // bad ids are latched by the scatter
+      atomicOr(&m[bb >> 5], 1u << (bb & 31));
+    }
+    __syncwarp();
+    for (uint32_t w = lane; w < nw; w += 32) {
+      const uint32_t v = m[w];
+      if (v) {
+        atomicOr(&bits[(uint64_t)k * nw + w], v);
+        m[w] = 0u;
+      }
+    }
+    __syncwarp();
+  }
+}
+// per kernel (one warp): local ids before each bitmap word, and B_k
+__global__ void k_lid_prep(uint32_t K, uint32_t nw, const uint32_t* bits, uint32_t* lbase, uint32_t* bk) {
+  const uint32_t lane = threadIdx.x & 31, nwarps = (gridDim.x * blockDim.x) >> 5;
+  for (uint32_t k = (blockIdx.x * blockDim.x + threadIdx.x) >> 5; k < K; k += nwarps) {
+    uint32_t carry = 0;
+    for (uint32_t w0 = 0; w0 < nw; w0 += 32) {
+      const uint32_t w = w0 + lane;
+      const uint32_t c = w < nw ? __popc(bits[(uint64_t)k * nw + w]) : 0u;
+      uint32_t x = c;
+      for (int o = 1; o < 32; o <<= 1) {
+        const uint32_t y = __shfl_up_sync(0xffffffffu, x, o);
+        if (lane >= (uint32_t)o) x += y;
+      }
+      if (w < nw) lbase[(uint64_t)k * nw + w] = carry + x - c;
+      carry += __shfl_sync(0xffffffffu, x, 31);
+    }
+    if (lane == 0) bk[k] = carry;
+  }
+}
+// exclusive scans over kernels (one CTA): goff = groups before k, hb = histogram entries before k (B_k * jobs_k);
+// misc[0] = total groups
+__global__ void __launch_bounds__(1024) k_lid_scan(uint32_t K, const uint64_t* coff, const uint32_t* bk, uint64_t* goff,
+                                                   uint64_t* hb, uint32_t* misc, uint64_t hcap, DevErr* err) {
+  __shared__ uint64_t wa[32], wb[32];
+  __shared__ uint64_t ca, cb;
+  if (threadIdx.x == 0) ca = cb = 0;
+  __syncthreads();
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+  for (uint32_t base = 0; base < K; base += 1024) {
+    const uint32_t k = base + threadIdx.x;
+    const uint64_t va = k < K ? bk[k] : 0, vb = k < K ? (uint64_t)bk[k] * (coff[k + 1] - coff[k]) : 0;
+    uint64_t xa = va, xb = vb;
+    for (int o = 1; o < 32; o <<= 1) {
+      const uint64_t ya = __shfl_up_sync(0xffffffffu, xa, o), yb = __shfl_up_sync(0xffffffffu, xb, o);
+      if (lane >= o) { xa += ya; xb += yb; }
+    }
+    if (lane == 31) { wa[wid] = xa; wb[wid] = xb; }
+    __syncthreads();
+    uint64_t pa = ca, pb = cb;
+    for (int w = 0; w < wid; ++w) { pa += wa[w]; pb += wb[w]; }
+    if (k < K) { goff[k] = pa + xa - va; hb[k] = pb + xb - vb; }
+    __syncthreads();
+    if (threadIdx.x == 1023) { ca = pa + xa; cb = pb + xb; }
+    __syncthreads();
+  }
+  if (threadIdx.x == 0) {
+    goff[K] = ca;
+    hb[K] = cb;
+    misc[0] = cb <= hcap ? (uint32_t)ca : 0u;  // no groups when the histogram does not fit
+    if (cb > hcap) latch(err, PHOTON_ECAPACITY, (int64_t)cb);
+  }
+}
+// per kernel (one warp): gkb[goff[k] + l] = k << 16 | b for its present BB ids
+__global__ void k_lid_groups(uint32_t K, uint32_t nw, const uint32_t* bits, const uint32_t* lbase, const uint64_t* goff,
+                             uint64_t* gkb) {
+  const uint32_t lane = threadIdx.x & 31, nwarps = (gridDim.x * blockDim.x) >> 5;
+  for (uint32_t k = (blockIdx.x * blockDim.x + threadIdx.x) >> 5; k < K; k += nwarps)
+    for (uint32_t w = lane; w < nw; w += 32) {
+      uint32_t v = bits[(uint64_t)k * nw + w];
+      uint64_t g = goff[k] + lbase[(uint64_t)k * nw + w];
+      while (v) {
+        const uint32_t bit = __ffs(v) - 1;
+        v &= v - 1;
+        gkb[g++] = ((uint64_t)k << 16) | (w * 32 + bit);
+      }
+    }
+}
+
+__global__ void __launch_bounds__(256) k_job_hist(photon_timing t, JobMap jm, uint64_t n_jobs, uint32_t* hist) {
+  __shared__ uint32_t h[8][kSmemBins];
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+  const uint32_t B = t.n_bb;
+  for (int d = lane; d < (int)kSmemBins; d += 32) h[wid][d] = 0;
+  __syncwarp();
+  if (!jm.fits()) return;  // ECAPACITY latched by k_lid_scan
+  n_jobs = umin64(n_jobs, jm.coff[t.n_kernels]);  // real jobs only: a job past the last would address the next
+                                                  // group's cells in the kernel-major layout
+  for (uint64_t job = (uint64_t)blockIdx.x * 8 + wid; job < n_jobs; job += (uint64_t)gridDim.x * 8) {
+    const uint32_t k = upper_idx(jm.coff, t.n_kernels, job);
+    const uint64_t jl = job - jm.coff[k], nj = jm.coff[k + 1] - jm.coff[k];
+    const uint32_t nb = jm.nbins(k, B);
+    const bool sm = nb <= kSmemBins;
+    const uint64_t hb = jm.hbase(k, B);
+    uint64_t a = umin64(t.kernel_rec_off[k], t.n_records), e = umin64(t.kernel_rec_off[k + 1], t.n_records);  // clamped: bad offsets are latched by k_rec_chunks
+    uint64_t cs = a + jl * JOB, ce = umin64(cs + JOB, e);
     for (uint64_t i0 = cs; i0 < ce; i0 += 128) {
       uint32_t d[4];
 #pragma unroll
@@ -303,32 +430,44 @@ __global__ void __launch_bounds__(256) k_job_hist(photon_timing t, const uint64_
       }
 #pragma unroll
       for (int u = 0; u < 4; ++u) {
-        uint32_t x = d[u] < B || d[u] == kNone ? d[u] : 0u;  // bad ids count as bb 0 (latched by the scatter)
+        uint32_t x = d[u] == kNone ? kNone : jm.lid(k, d[u] < B ? d[u] : 0u);  // bad ids count as bb 0 (latched by the scatter)
         unsigned peers = __match_any_sync(0xffffffffu, x);
-        if (x != kNone && lane == __ffs(peers) - 1) h[wid][x] += __popc(peers);
+        if (x != kNone && lane == __ffs(peers) - 1) {
+          if (sm) h[wid][x] += __popc(peers);
+          else atomicAdd(&hist[hb + (uint64_t)x * nj + jl], (uint32_t)__popc(peers));
+        }
         __syncwarp();
       }
     }
-    for (int dd = lane; dd < (int)B; dd += 32) {
-      hist[(uint64_t)dd * n_jobs + job] = h[wid][dd];
-      h[wid][dd] = 0;
+    if (sm) {
+      for (int dd = lane; dd < (int)nb; dd += 32) {
+        hist[hb + (uint64_t)dd * nj + jl] = h[wid][dd];
+        h[wid][dd] = 0;
+      }
     }
     __syncwarp();
   }
 }
 
-__global__ void __launch_bounds__(256) k_job_scatter(photon_timing t, const uint64_t* coff, uint64_t n_jobs,
-                                                     const uint32_t* off, uint64_t* X, uint64_t* Y, uint32_t* idx,
-                                                     DevErr* err) {
-  __shared__ uint32_t run[8][256];
+__global__ void __launch_bounds__(256) k_job_scatter(photon_timing t, JobMap jm, uint64_t n_jobs, uint32_t* off,
+                                                     uint64_t* X, uint64_t* Y, uint32_t* idx, DevErr* err) {
+  __shared__ uint32_t run[8][kSmemBins];
   const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
   const uint32_t B = t.n_bb;
   const unsigned lt = (1u << lane) - 1u;
+  if (!jm.fits()) return;  // ECAPACITY latched by k_lid_scan
+  n_jobs = umin64(n_jobs, jm.coff[t.n_kernels]);  // real jobs only: a job past the last would address the next
+                                                  // group's cells in the kernel-major layout
   for (uint64_t job = (uint64_t)blockIdx.x * 8 + wid; job < n_jobs; job += (uint64_t)gridDim.x * 8) {
-    uint32_t k = upper_idx(coff, t.n_kernels, job);
-    uint64_t a = umin64(t.kernel_rec_off[k], t.n_records), b = umin64(t.kernel_rec_off[k + 1], t.n_records);  // clamped: bad offsets are latched by k_rec_chunks
-    uint64_t cs = a + (job - coff[k]) * JOB, ce = umin64(cs + JOB, b);
-    for (int dd = lane; dd < (int)B; dd += 32) run[wid][dd] = off[(uint64_t)dd * n_jobs + job];
+    const uint32_t k = upper_idx(jm.coff, t.n_kernels, job);
+    const uint64_t jl = job - jm.coff[k], nj = jm.coff[k + 1] - jm.coff[k];
+    const uint32_t nb = jm.nbins(k, B);
+    const bool sm = nb <= kSmemBins;
+    const uint64_t hb = jm.hbase(k, B);
+    uint64_t a = umin64(t.kernel_rec_off[k], t.n_records), e = umin64(t.kernel_rec_off[k + 1], t.n_records);  // clamped: bad offsets are latched by k_rec_chunks
+    uint64_t cs = a + jl * JOB, ce = umin64(cs + JOB, e);
+    if (sm)
+      for (int dd = lane; dd < (int)nb; dd += 32) run[wid][dd] = off[hb + (uint64_t)dd * nj + jl];
     __syncwarp();
     for (uint64_t i0 = cs; i0 < ce; i0 += 256) {
       uint32_t d[8];
@@ -351,12 +490,20 @@ __global__ void __launch_bounds__(256) k_job_scatter(photon_timing t, const uint
             latch(err, PHOTON_ERANGE, (int64_t)i);
             if (dd >= B) dd = 0;
           }
+          dd = jm.lid(k, dd);
         }
         unsigned peers = __match_any_sync(0xffffffffu, dd);
-        uint32_t base = dd != kNone ? run[wid][dd] : 0;
-        __syncwarp();
+        const int lead = __ffs(peers) - 1;
+        uint32_t base = 0;
+        if (sm) {
+          base = dd != kNone ? run[wid][dd] : 0;
+          __syncwarp();
+          if (dd != kNone && lane == lead) run[wid][dd] = base + __popc(peers);
+        } else {
+          if (dd != kNone && lane == lead) base = atomicAdd(&off[hb + (uint64_t)dd * nj + jl], (uint32_t)__popc(peers));
+          base = __shfl_sync(0xffffffffu, base, lead);
+        }
         if (dd != kNone) {
-          if (lane == __ffs(peers) - 1) run[wid][dd] = base + __popc(peers);
           uint32_t dest = base + __popc(peers & lt);
           X[dest] = x[u];
           Y[dest] = y[u];
@@ -368,15 +515,21 @@ __global__ void __launch_bounds__(256) k_job_scatter(photon_timing t, const uint
   }
 }
 
-// gstart[b*K + k] = start of group (b, k) = scanned hist[b][first job of k]; gstart[K*B] = R
-__global__ void k_job_gstart(const uint32_t* off, const uint64_t* coff, uint32_t K, uint32_t B, uint64_t n_jobs,
-                             uint64_t R, uint64_t* gstart, uint32_t* G) {
-  const uint64_t n = (uint64_t)K * B;
+// gstart[g] = start of group g = (k, l) (g = k*B + b, or goff[k] + l): the scanned histogram entry (k, l, first
+// job); groups of a kernel without records start where the next kernel's do; gstart[G] = R
+__global__ void k_job_gstart(const uint32_t* off, JobMap jm, const uint64_t* goff, const uint64_t* gkb, uint32_t K,
+                             uint32_t B, uint64_t R, uint64_t Htot_host, uint64_t* gstart, uint32_t* G) {
+  if (!jm.fits()) return;
+  const uint64_t n = jm.compact ? goff[K] : (uint64_t)K * B;
+  const uint64_t Htot = jm.compact ? jm.hb[K] : Htot_host;
   for (uint64_t g = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; g <= n; g += (uint64_t)gridDim.x * blockDim.x) {
-    if (g == n) { gstart[g] = R; *G = (uint32_t)n; continue; }
-    uint64_t b = g / K, k = g % K;
-    uint64_t j = b * n_jobs + umin64(coff[k], n_jobs);  // clamp keeps gstart monotone on malformed offsets
-    gstart[g] = j < (uint64_t)B * n_jobs ? off[j] : R;
+    if (g == n) { gstart[g] = R; if (!jm.compact) *G = (uint32_t)n; continue; }
+    uint32_t k, l;
+    if (jm.compact) { k = (uint32_t)(gkb[g] >> 16); l = (uint32_t)(g - goff[k]); }
+    else { k = (uint32_t)(g / B); l = (uint32_t)(g % B); }
+    const uint64_t nj = jm.coff[k + 1] - jm.coff[k];
+    const uint64_t j = jm.hbase(k, B) + (uint64_t)l * nj;
+    gstart[g] = j < Htot ? off[j] : R;
   }
 }
 
@@ -638,15 +791,19 @@ __global__ void __launch_bounds__(WT, 2) k_window(WinArgs a) {
 }
 
 // ---- 5. outputs ----------------------------------------------------------------------------------------------
+// group g -> (k, b): mode 0 (radix path) g = b*K + k; 1 (job path, B <= 256) g = k*B + b; 2 (compact) gkb[g]
 __global__ void k_finish(const uint32_t* idx, const uint64_t* X, const uint64_t* Y, const uint32_t* G,
                          const uint64_t* gfirst, const uint64_t* kro, uint32_t K, uint32_t B, uint32_t n,
-                         int64_t* first_stable, uint64_t* dur) {
+                         int mode, const uint64_t* gkb, int64_t* first_stable, uint64_t* dur) {
   const uint32_t lane = threadIdx.x & 31, ng = *G;
   const uint32_t nw = (gridDim.x * blockDim.x) >> 5;
   for (uint32_t g = (blockIdx.x * blockDim.x + threadIdx.x) >> 5; g < ng; g += nw) {
     uint64_t q = gfirst[g];
     if (q == ~0ull) continue;
-    uint64_t k = g % K, b = g / K;
+    uint64_t k, b;
+    if (mode == 0) { k = g % K; b = g / K; }
+    else if (mode == 1) { k = g / B; b = g % B; }
+    else { k = gkb[g] >> 16; b = gkb[g] & 0xFFFFu; }
     uint64_t s = 0;
     for (uint64_t i = q + 1 - n + lane; i <= q; i += 32) s += Y[i] - X[i];
     for (int o = 16; o > 0; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
@@ -796,15 +953,20 @@ inline void build_runlist(const RunList& rl, const uint32_t* G, const uint32_t* 
 }
 
 struct Layout {
-  bool onepass;      // B <= 256: job multisplit; else LSD radix sort of composite keys
+  int mode;          // 1: job multisplit on BB ids (B <= 256); 2: on per-kernel compacted ids (B <= 8192);
+                     // 0: LSD radix sort of composite keys (larger B)
   uint64_t* key0; uint64_t* key1;  // radix path only
-  uint32_t* val0; uint32_t* val1;  // val0 = original record index of each sorted position (both paths)
+  uint32_t* val0; uint32_t* val1;  // val0 = original record index of each sorted position (all paths)
   uint64_t* X; uint64_t* Y;
   uint32_t* hist; uint32_t* bsum; uint32_t* misc;  // misc[0] = G, [1] = max runs, [2] = ticket, [4] = scan total
   uint64_t* gstart;  // [gcap+1]
   uint32_t* nruns;   // [gcap]
   uint64_t* gfirst;  // [gcap]
   uint64_t* coff;    // [K+1] chunk (job) offsets per kernel
+  // compact ids
+  uint32_t nw;       // bitmap words per kernel
+  uint32_t* bits; uint32_t* lbase; uint32_t* bk;  // [K*nw], [K*nw], [K]
+  uint64_t* goff; uint64_t* hb; uint64_t* gkb;    // [K+1], [K+1], [gcap]
   RunList rl;
   uint64_t gcap, n_tiles, n_jobs, hn;
   size_t bytes;
@@ -814,16 +976,19 @@ Layout make_layout(const photon_timing& t, void* base) {
   Carver c(base);
   Layout L{};
   uint64_t R = t.n_records ? t.n_records : 1;
-  L.onepass = t.n_bb <= 256;
-  L.gcap = (uint64_t)t.n_kernels * t.n_bb;  // dense group ids g = b*K + k
+  const uint64_t KB = (uint64_t)t.n_kernels * t.n_bb;
+  L.mode = t.n_bb <= kSmemBins ? 1 : (t.n_bb <= kCompactMaxB ? 2 : 0);
+  L.gcap = L.mode == 2 ? (KB < R ? KB : R) : KB;  // dense group ids, or one per (kernel, BB present)
   if (L.gcap == 0) L.gcap = 1;
   L.n_tiles = ceil_div(R, RTILE);
   L.n_jobs = ceil_div(R, JOB) + t.n_kernels;
-  if (!L.onepass) { L.key0 = c.take<uint64_t>(R); L.key1 = c.take<uint64_t>(R); }
+  if (L.mode == 0) { L.key0 = c.take<uint64_t>(R); L.key1 = c.take<uint64_t>(R); }
   L.val0 = c.take<uint32_t>(R);
-  if (!L.onepass) L.val1 = c.take<uint32_t>(R);
+  if (L.mode == 0) L.val1 = c.take<uint32_t>(R);
   L.X = c.take<uint64_t>(R); L.Y = c.take<uint64_t>(R);
-  L.hn = L.onepass ? (uint64_t)t.n_bb * L.n_jobs : (uint64_t)RNB * L.n_tiles;
+  // histogram cells: B * jobs; compact: sum_k B_k * jobs_k <= 2R + ... whenever no kernel has more than 2048
+  // distinct BB ids (ECAPACITY otherwise)
+  L.hn = L.mode == 1 ? (uint64_t)t.n_bb * L.n_jobs : (L.mode == 2 ? 2 * R + 65536 : (uint64_t)RNB * L.n_tiles);
   L.hist = c.take<uint32_t>(L.hn);
   L.bsum = c.take<uint32_t>(ceil_div(L.hn, SB) + 1);
   L.misc = c.take<uint32_t>(16);
@@ -831,6 +996,15 @@ Layout make_layout(const photon_timing& t, void* base) {
   L.nruns = c.take<uint32_t>(L.gcap);
   L.gfirst = c.take<uint64_t>(L.gcap);
   L.coff = c.take<uint64_t>((uint64_t)t.n_kernels + 1);
+  if (L.mode == 2) {
+    L.nw = (t.n_bb + 31) / 32;
+    L.bits = c.take<uint32_t>((uint64_t)t.n_kernels * L.nw + 1);
+    L.lbase = c.take<uint32_t>((uint64_t)t.n_kernels * L.nw + 1);
+    L.bk = c.take<uint32_t>((uint64_t)t.n_kernels + 1);
+    L.goff = c.take<uint64_t>((uint64_t)t.n_kernels + 1);
+    L.hb = c.take<uint64_t>((uint64_t)t.n_kernels + 1);
+    L.gkb = c.take<uint64_t>(L.gcap);
+  }
   carve_runlist(c, R, L.rl);
   L.bytes = c.off + 256;
   return L;
@@ -850,19 +1024,37 @@ cudaError_t launch_stable(const photon_timing& t, const uint64_t* kbb, photon_st
   cudaMemsetAsync(first_stable, 0xFF, sizeof(int64_t) * (size_t)K * B, s);
   if (dur) cudaMemsetAsync(dur, 0, sizeof(uint64_t) * (size_t)K * B, s);
   cudaMemsetAsync(L.misc, 0, 64, s);
-  const uint64_t chunk = L.onepass ? JOB : REC_CHUNK;
+  const uint64_t chunk = L.mode != 0 ? JOB : REC_CHUNK;
   note_launch(), k_rec_chunks<<<1, 1024, 0, s>>>(t.kernel_rec_off, K, R, chunk, L.coff, err);
   if (R > 0) {
     uint32_t* idx;
-    if (L.onepass) {
-      // 1-2. per-job histograms -> bin-major scan -> stable scatter of (issue, retire, index) into group order
+    if (L.mode != 0) {
+      // 1-2. per-job histograms of (kernel-local) BB ids -> kernel-major scan -> stable scatter of (issue, retire,
+      // index) into group order
       unsigned gj = (unsigned)umin64(ceil_div(L.n_jobs, 8), (uint64_t)num_sms * 8);
+      JobMap jm{};
+      jm.coff = L.coff;
+      jm.compact = L.mode == 2;
+      jm.nkern = K;
+      jm.hcap = L.hn;
+      if (jm.compact) {
+        jm.bits = L.bits; jm.lbase = L.lbase; jm.bk = L.bk; jm.hb = L.hb; jm.nw = L.nw;
+        cudaMemsetAsync(L.bits, 0, sizeof(uint32_t) * (size_t)K * L.nw, s);
+        const size_t psm = (size_t)8 * L.nw * 4;
+        cudaFuncSetAttribute(k_presence, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)psm);
+        note_launch(), k_presence<<<gj, 256, psm, s>>>(t, L.coff, L.n_jobs, L.nw, L.bits);
+        const unsigned gk = (unsigned)umin64(ceil_div((uint64_t)K * 32, 256), (uint64_t)num_sms * 8);
+        note_launch(), k_lid_prep<<<gk, 256, 0, s>>>(K, L.nw, L.bits, L.lbase, L.bk);
+        note_launch(), k_lid_scan<<<1, 1024, 0, s>>>(K, L.coff, L.bk, L.goff, L.hb, L.misc + 0, L.hn, err);
+        note_launch(), k_lid_groups<<<gk, 256, 0, s>>>(K, L.nw, L.bits, L.lbase, L.goff, L.gkb);
+      }
       cudaMemsetAsync(L.hist, 0, sizeof(uint32_t) * L.hn, s);
-      note_launch(), k_job_hist<<<gj, 256, 0, s>>>(t, L.coff, L.n_jobs, L.hist);
+      note_launch(), k_job_hist<<<gj, 256, 0, s>>>(t, jm, L.n_jobs, L.hist);
       scan_u32(L.hist, L.hist, L.hn, L.bsum, L.misc + 4, s);
-      note_launch(), k_job_scatter<<<gj, 256, 0, s>>>(t, L.coff, L.n_jobs, L.hist, L.X, L.Y, L.val0, err);
+      // group starts first: kernels with > 256 local ids use the scanned cells as running offsets in the scatter
       note_launch(), k_job_gstart<<<(unsigned)umin64(ceil_div(L.gcap + 1, 256), (uint64_t)num_sms * 8), 256, 0, s>>>(
-          L.hist, L.coff, K, B, L.n_jobs, R, L.gstart, L.misc + 0);
+          L.hist, jm, L.goff, L.gkb, K, B, R, (uint64_t)B * L.n_jobs, L.gstart, L.misc + 0);
+      note_launch(), k_job_scatter<<<gj, 256, 0, s>>>(t, jm, L.n_jobs, L.hist, L.X, L.Y, L.val0, err);
       idx = L.val0;
     } else {
       uint64_t jobs_ub = ceil_div(R, REC_CHUNK) + K;
@@ -898,7 +1090,7 @@ cudaError_t launch_stable(const photon_timing& t, const uint64_t* kbb, photon_st
     note_launch(), k_window<<<(unsigned)num_sms * 2, WT, 0, s>>>(wa);
     // 5. outputs
     note_launch(), k_finish<<<(unsigned)umin64(ceil_div(L.gcap * 32, 256), (uint64_t)num_sms * 8), 256, 0, s>>>(
-        idx, L.X, L.Y, L.misc + 0, L.gfirst, t.kernel_rec_off, K, B, p.window_n, first_stable, dur);
+        idx, L.X, L.Y, L.misc + 0, L.gfirst, t.kernel_rec_off, K, B, p.window_n, L.mode, L.gkb, first_stable, dur);
     unsigned gk = (unsigned)umin64(K, (uint64_t)num_sms * 8);
     note_launch(), k_switch<<<gk ? gk : 1, 256, 0, s>>>(first_stable, kbb, K, B, p.rate_num, p.rate_den, switch_at);
   } else {

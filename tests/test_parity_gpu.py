@@ -272,9 +272,10 @@ def test_stable_late_multirun(ph):
     assert (fs[:, 0] > 0).all() and (fs[:, 2] >= 0).all()
 
 
-@pytest.mark.parametrize("B", [256, 257, 1000])
+@pytest.mark.parametrize("B", [256, 257, 1000, 5000, 9000])
 def test_stable_many_bb(ph, B):
-    # B <= 256 takes the one-pass job multisplit, B > 256 the composite-key radix sort: both must agree with the oracle
+    # B <= 256: job multisplit on BB ids; 256 < B <= 8192: on per-kernel compacted ids (kernels with > 256 local ids
+    # keep their counters in global memory); B > 8192: composite-key radix sort -- all must agree with the oracle
     rng = np.random.default_rng(B)
     offs, bbs, iss, ret = [0], [], [], []
     for k in range(6):
