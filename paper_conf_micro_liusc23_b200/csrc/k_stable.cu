@@ -40,9 +40,17 @@ constexpr int RUN = WITEM * NI;
 
 // ---- generic device-wide exclusive scan of u32 (values and total < 2^32) --------------------------------------
 constexpr int SB = 4096;
-__global__ void __launch_bounds__(256) k_scan_reduce(const uint32_t* in, uint64_t n, uint32_t* bsum) {
+// ndev (optional): the live length on the device (n is then its capacity); cells past it are not touched
+__device__ __forceinline__ uint64_t live_n(uint64_t n, const uint64_t* ndev) { return ndev ? umin64(n, *ndev) : n; }
+__global__ void __launch_bounds__(256) k_scan_reduce(const uint32_t* in, uint64_t n, const uint64_t* ndev,
+                                                     uint32_t* bsum) {
   __shared__ uint32_t ws[8];
+  n = live_n(n, ndev);
   uint64_t base = (uint64_t)blockIdx.x * SB;
+  if (base >= n) {
+    if (threadIdx.x == 0) bsum[blockIdx.x] = 0;
+    return;
+  }
   uint32_t s = 0;
   for (int i = threadIdx.x; i < SB; i += 256) {
     uint64_t j = base + i;
@@ -57,8 +65,9 @@ __global__ void __launch_bounds__(256) k_scan_reduce(const uint32_t* in, uint64_
     bsum[blockIdx.x] = t;
   }
 }
-__global__ void __launch_bounds__(1024) k_scan_single(uint32_t* a, uint64_t n, uint32_t* total) {
+__global__ void __launch_bounds__(1024) k_scan_single(uint32_t* a, uint64_t n, const uint64_t* ndev, uint32_t* total) {
   __shared__ uint32_t ws[32];
+  if (ndev) n = umin64(n, ceil_div(*ndev, (uint64_t)SB));
   __shared__ uint32_t carry;
   if (threadIdx.x == 0) carry = 0;
   __syncthreads();
@@ -89,10 +98,12 @@ __global__ void __launch_bounds__(1024) k_scan_single(uint32_t* a, uint64_t n, u
   }
   if (threadIdx.x == 0 && total) *total = carry;
 }
-__global__ void __launch_bounds__(256) k_scan_apply(const uint32_t* in, uint64_t n, const uint32_t* bsum,
-                                                    uint32_t* out) {
+__global__ void __launch_bounds__(256) k_scan_apply(const uint32_t* in, uint64_t n, const uint64_t* ndev,
+                                                    const uint32_t* bsum, uint32_t* out) {
   __shared__ uint32_t ws[8];
   __shared__ uint32_t carry;
+  n = live_n(n, ndev);
+  if ((uint64_t)blockIdx.x * SB >= n) return;
   if (threadIdx.x == 0) carry = bsum[blockIdx.x];
   __syncthreads();
   const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
@@ -115,12 +126,19 @@ __global__ void __launch_bounds__(256) k_scan_apply(const uint32_t* in, uint64_t
     __syncthreads();
   }
 }
-// out may alias in; bsum needs ceil(n/SB) entries; total (device) receives the sum
-void scan_u32(const uint32_t* in, uint32_t* out, uint64_t n, uint32_t* bsum, uint32_t* total, cudaStream_t s) {
+// out may alias in; bsum needs ceil(n/SB) entries; total (device) receives the sum; ndev (optional, device): scan
+// only the first min(n, *ndev) cells
+void scan_u32(const uint32_t* in, uint32_t* out, uint64_t n, uint32_t* bsum, uint32_t* total, cudaStream_t s,
+              const uint64_t* ndev = nullptr) {
   uint64_t nb = ceil_div(n ? n : 1, SB);
-  note_launch(), k_scan_reduce<<<(unsigned)nb, 256, 0, s>>>(in, n, bsum);
-  note_launch(), k_scan_single<<<1, 1024, 0, s>>>(bsum, nb, total);
-  note_launch(), k_scan_apply<<<(unsigned)nb, 256, 0, s>>>(in, n, bsum, out);
+  note_launch(), k_scan_reduce<<<(unsigned)nb, 256, 0, s>>>(in, n, ndev, bsum);
+  note_launch(), k_scan_single<<<1, 1024, 0, s>>>(bsum, nb, ndev, total);
+  note_launch(), k_scan_apply<<<(unsigned)nb, 256, 0, s>>>(in, n, ndev, bsum, out);
+}
+__global__ void k_zero_live(uint32_t* a, uint64_t n, const uint64_t* ndev) {
+  n = live_n(n, ndev);
+  for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x)
+    a[i] = 0u;
 }
 
 // ---- 1. per-kernel record chunks + validation + keys -------------------------------------------------------
@@ -308,6 +326,46 @@ struct JobMap {
   }
 };
 
+// The BB ids of one job [cs, ce) (at most JOB records), loaded up front as 16-byte vectors (9 per lane: enough
+// memory parallelism for these order-free passes) and handed one per lane per step to f(id) -- kNone outside the
+// job -- in warp-uniform steps (f may use warp collectives).  Vectors are aligned 8-id blocks; a block reaching
+// past R (or an unaligned bb array) is read element by element.
+template <class F>
+__device__ __forceinline__ void job_ids(const uint16_t* bb, uint64_t R, uint64_t cs, uint64_t ce, int lane, F&& f) {
+  constexpr int NV = JOB / 256 + 1;
+  const uint64_t c0 = cs & ~7ull;
+  const bool vec = ((uintptr_t)bb & 15) == 0;
+  uint4 v[NV];
+#pragma unroll
+  for (int r = 0; r < NV; ++r) {
+    const uint64_t i = c0 + (uint64_t)r * 256 + lane * 8;
+    v[r] = make_uint4(~0u, ~0u, ~0u, ~0u);
+    if (i < ce) {
+      if (vec && i + 8 <= R) {
+        v[r] = __ldg(reinterpret_cast<const uint4*>(bb + i));
+      } else {
+        uint32_t e[4];
+#pragma unroll
+        for (int h = 0; h < 4; ++h) {
+          const uint32_t lo = i + 2 * h < R ? bb[i + 2 * h] : 0xFFFFu, hi = i + 2 * h + 1 < R ? bb[i + 2 * h + 1] : 0xFFFFu;
+          e[h] = lo | hi << 16;
+        }
+        v[r] = make_uint4(e[0], e[1], e[2], e[3]);
+      }
+    }
+  }
+#pragma unroll
+  for (int r = 0; r < NV; ++r) {
+    const uint64_t i = c0 + (uint64_t)r * 256 + lane * 8;
+    const uint32_t w[4] = {v[r].x, v[r].y, v[r].z, v[r].w};
+#pragma unroll
+    for (int j = 0; j < 8; ++j) {
+      const uint64_t q = i + j;
+      f(q >= cs && q < ce ? (w[j >> 1] >> ((j & 1) * 16)) & 0xFFFFu : kNone);
+    }
+  }
+}
+
 // presence bitmap per kernel (compact ids): one warp per job ORs its BB ids into a shared bitmap, then into global
 __global__ void __launch_bounds__(256) k_presence(photon_timing t, const uint64_t* coff, uint64_t n_jobs, uint32_t nw,
                                                   uint32_t* bits) {
@@ -320,10 +378,16 @@ __global__ void __launch_bounds__(256) k_presence(photon_timing t, const uint64_
     const uint32_t k = upper_idx(coff, t.n_kernels, job);
     const uint64_t a = umin64(t.kernel_rec_off[k], t.n_records), e = umin64(t.kernel_rec_off[k + 1], t.n_records);
     const uint64_t cs = a + (job - coff[k]) * JOB, ce = umin64(cs + JOB, e);
-    for (uint64_t i = cs + lane; i < ce; i += 32) {
-      uint32_t bb = t.bb[i];
+    // lanes hitting the same bitmap word OR their bits together first (one shared atomic per distinct word: a
+    // kernel's few BB ids share words, and 32 same-address atomics would serialise)
+    for (uint64_t i0 = cs; i0 < ce; i0 += 32) {
+      const uint64_t i = i0 + lane;
+      uint32_t bb = i < ce ? (uint32_t)t.bb[i] : 0u;
       if (bb >= t.n_bb) bb = 0;  // bad ids are latched by the scatter
-      atomicOr(&m[bb >> 5], 1u << (bb & 31));
+      const uint32_t w = i < ce ? bb >> 5 : kNone;
+      const unsigned peers = __match_any_sync(0xffffffffu, w);
+      const uint32_t v = __reduce_or_sync(peers, 1u << (bb & 31));
+      if (w != kNone && lane == __ffs(peers) - 1) atomicOr(&m[w], v);
     }
     __syncwarp();
     for (uint32_t w = lane; w < nw; w += 32) {
@@ -404,52 +468,75 @@ __global__ void k_lid_groups(uint32_t K, uint32_t nw, const uint32_t* bits, cons
     }
 }
 
-__global__ void __launch_bounds__(256) k_job_hist(photon_timing t, JobMap jm, uint64_t n_jobs, uint32_t* hist) {
-  __shared__ uint32_t h[8][kSmemBins];
+// Per-job histograms.  Kernels with <= 256 (local) ids: lane-private byte counters in shared memory ([bin][lane],
+// a lane counts at most JOB/32 = 64 ids of a job), no atomics and no warp collectives per id; the 32 columns of a
+// bin are summed with dp4a at the end of the job.  More ids: __match_any_sync-aggregated global atomics.
+constexpr int HW = 4;  // warps per k_job_hist block (4 x 8 KB of counters)
+static_assert(JOB / 32 < 256, "byte counters");
+__global__ void __launch_bounds__(HW * 32) k_job_hist(photon_timing t, JobMap jm, uint64_t n_jobs, uint32_t* hist) {
+  __shared__ uint32_t h[HW][kSmemBins * 8];  // per warp: bin-major rows of 32 byte counters
   const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
   const uint32_t B = t.n_bb;
-  for (int d = lane; d < (int)kSmemBins; d += 32) h[wid][d] = 0;
+  uint8_t* hb8 = reinterpret_cast<uint8_t*>(h[wid]);
+  for (int d = lane; d < (int)kSmemBins * 8; d += 32) h[wid][d] = 0;
   __syncwarp();
   if (!jm.fits()) return;  // ECAPACITY latched by k_lid_scan
   n_jobs = umin64(n_jobs, jm.coff[t.n_kernels]);  // real jobs only: a job past the last would address the next
                                                   // group's cells in the kernel-major layout
-  for (uint64_t job = (uint64_t)blockIdx.x * 8 + wid; job < n_jobs; job += (uint64_t)gridDim.x * 8) {
+  const bool vec = ((uintptr_t)t.bb & 15) == 0;
+  for (uint64_t job = (uint64_t)blockIdx.x * HW + wid; job < n_jobs; job += (uint64_t)gridDim.x * HW) {
     const uint32_t k = upper_idx(jm.coff, t.n_kernels, job);
     const uint64_t jl = job - jm.coff[k], nj = jm.coff[k + 1] - jm.coff[k];
     const uint32_t nb = jm.nbins(k, B);
-    const bool sm = nb <= kSmemBins;
     const uint64_t hb = jm.hbase(k, B);
     uint64_t a = umin64(t.kernel_rec_off[k], t.n_records), e = umin64(t.kernel_rec_off[k + 1], t.n_records);  // clamped: bad offsets are latched by k_rec_chunks
     uint64_t cs = a + jl * JOB, ce = umin64(cs + JOB, e);
-    for (uint64_t i0 = cs; i0 < ce; i0 += 128) {
-      uint32_t d[4];
+    if (nb > kSmemBins) {
+      job_ids(t.bb, t.n_records, cs, ce, lane, [&](uint32_t d) {
+        const uint32_t x = d == kNone ? kNone : jm.lid(k, d < B ? d : 0u);  // bad ids count as bb 0 (latched by the scatter)
+        const unsigned peers = __match_any_sync(0xffffffffu, x);
+        if (x != kNone && lane == __ffs(peers) - 1) atomicAdd(&hist[hb + (uint64_t)x * nj + jl], (uint32_t)__popc(peers));
+      });
+      continue;
+    }
+    // lane-contiguous 8-id blocks from the aligned start: a lane counts at most 8 ids per 256-id step
+    const uint64_t c0 = cs & ~7ull;
+    for (uint64_t i = c0 + lane * 8; i < ce; i += 256) {
+      uint32_t w[4];
+      if (vec && i + 8 <= t.n_records) {
+        const uint4 v = __ldg(reinterpret_cast<const uint4*>(t.bb + i));
+        w[0] = v.x; w[1] = v.y; w[2] = v.z; w[3] = v.w;
+      } else {
 #pragma unroll
-      for (int u = 0; u < 4; ++u) {
-        uint64_t i = i0 + u * 32 + lane;
-        d[u] = i < ce ? (uint32_t)t.bb[i] : kNone;
+        for (int hh = 0; hh < 4; ++hh)
+          w[hh] = (i + 2 * hh < t.n_records ? t.bb[i + 2 * hh] : 0u) |
+                  (i + 2 * hh + 1 < t.n_records ? (uint32_t)t.bb[i + 2 * hh + 1] : 0u) << 16;
       }
 #pragma unroll
-      for (int u = 0; u < 4; ++u) {
-        uint32_t x = d[u] == kNone ? kNone : jm.lid(k, d[u] < B ? d[u] : 0u);  // bad ids count as bb 0 (latched by the scatter)
-        unsigned peers = __match_any_sync(0xffffffffu, x);
-        if (x != kNone && lane == __ffs(peers) - 1) {
-          if (sm) h[wid][x] += __popc(peers);
-          else atomicAdd(&hist[hb + (uint64_t)x * nj + jl], (uint32_t)__popc(peers));
+      for (int j = 0; j < 8; ++j) {
+        const uint64_t q = i + j;
+        uint32_t d = (w[j >> 1] >> ((j & 1) * 16)) & 0xFFFFu;
+        if (q >= cs && q < ce) {
+          const uint32_t x = jm.lid(k, d < B ? d : 0u);  // bad ids count as bb 0 (latched by the scatter)
+          hb8[x * 32 + lane] += 1;
         }
-        __syncwarp();
       }
     }
-    if (sm) {
-      for (int dd = lane; dd < (int)nb; dd += 32) {
-        hist[hb + (uint64_t)dd * nj + jl] = h[wid][dd];
-        h[wid][dd] = 0;
+    __syncwarp();
+    for (int dd = lane; dd < (int)nb; dd += 32) {
+      uint32_t c = 0;
+#pragma unroll
+      for (int q = 0; q < 8; ++q) {
+        c = __dp4a(h[wid][dd * 8 + q], 0x01010101u, c);
+        h[wid][dd * 8 + q] = 0;
       }
+      hist[hb + (uint64_t)dd * nj + jl] = c;
     }
     __syncwarp();
   }
 }
 
-__global__ void __launch_bounds__(256) k_job_scatter(photon_timing t, JobMap jm, uint64_t n_jobs, uint32_t* off,
+__global__ void __launch_bounds__(256, 3) k_job_scatter(photon_timing t, JobMap jm, uint64_t n_jobs, uint32_t* off,
                                                      uint64_t* X, uint64_t* Y, uint32_t* idx, DevErr* err) {
   __shared__ uint32_t run[8][kSmemBins];
   const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
@@ -469,20 +556,37 @@ __global__ void __launch_bounds__(256) k_job_scatter(photon_timing t, JobMap jm,
     if (sm)
       for (int dd = lane; dd < (int)nb; dd += 32) run[wid][dd] = off[hb + (uint64_t)dd * nj + jl];
     __syncwarp();
-    for (uint64_t i0 = cs; i0 < ce; i0 += 256) {
-      uint32_t d[8];
-      uint64_t x[8], y[8], yp[8];
+    // tiles of TS x 32 records, the next tile's loads in flight while this one is ranked and written
+    constexpr int TS = 4;
+    uint32_t d[TS];
+    uint64_t x[TS], y[TS];
+    auto load = [&](uint64_t i0, uint32_t* dd, uint64_t* xx, uint64_t* yy) {
 #pragma unroll
-      for (int u = 0; u < 8; ++u) {
-        uint64_t i = i0 + u * 32 + lane;
-        bool v = i < ce;
-        d[u] = v ? (uint32_t)t.bb[i] : kNone;
-        x[u] = v ? t.issue[i] : 0;
-        y[u] = v ? t.retire[i] : 0;
-        yp[u] = v && i > a ? t.retire[i - 1] : 0;
+      for (int u = 0; u < TS; ++u) {
+        const uint64_t i = i0 + u * 32 + lane;
+        const bool v = i < ce;
+        dd[u] = v ? (uint32_t)t.bb[i] : kNone;
+        xx[u] = v ? t.issue[i] : 0;
+        yy[u] = v ? t.retire[i] : 0;
       }
+    };
+    load(cs, d, x, y);
+    // retire[i - 1] of lane 0 in slot 0: the previous tile's last record (the job's first tile: one load)
+    uint64_t carry = lane == 0 && cs > a && cs < ce ? t.retire[cs - 1] : 0;
+    for (uint64_t i0 = cs; i0 < ce; i0 += 32 * TS) {
+      uint32_t nd[TS];
+      uint64_t nx[TS], ny[TS];
+      load(i0 + 32 * TS, nd, nx, ny);
+      uint64_t yp[TS];
 #pragma unroll
-      for (int u = 0; u < 8; ++u) {
+      for (int u = 0; u < TS; ++u) {
+        const uint64_t up = __shfl_up_sync(0xffffffffu, y[u], 1);
+        const uint64_t wrap = u ? __shfl_sync(0xffffffffu, y[u ? u - 1 : 0], 31) : carry;
+        yp[u] = lane ? up : wrap;
+      }
+      carry = __shfl_sync(0xffffffffu, y[TS - 1], 31);
+#pragma unroll
+      for (int u = 0; u < TS; ++u) {
         uint64_t i = i0 + u * 32 + lane;
         uint32_t dd = d[u];
         if (dd != kNone) {
@@ -511,6 +615,8 @@ __global__ void __launch_bounds__(256) k_job_scatter(photon_timing t, JobMap jm,
         }
         __syncwarp();
       }
+#pragma unroll
+      for (int u = 0; u < TS; ++u) { d[u] = nd[u]; x[u] = nx[u]; y[u] = ny[u]; }
     }
   }
 }
@@ -644,10 +750,168 @@ struct WinArgs {
   uint32_t n;
   uint32_t dnum, dden;
   uint64_t* gfirst;
+  uint32_t ring;   // fast path: shared positions per run (2n + RUN), 0 = off (n too large for shared memory)
+  int64_t lim;     // fast path: shifted times must lie in (-lim, lim) (n * lim^2 < 2^61: int64 sums are exact)
 };
 
 __device__ __forceinline__ void sums_sub(Sums& a, const Sums& b) {
   a.sx -= b.sx; a.sy -= b.sy; a.sn -= b.sn; a.s2n -= b.s2n; a.sxy -= b.sxy; a.sxx -= b.sxx;
+}
+
+// ---- 4'. fast path of one run: shifted 32-bit times staged in shared memory, int64 sums ----------------------
+// Eq. 1's numerator n*Sxy - Sx*Sy and denominator n*Sxx - Sx^2 are invariant under x -> x - c, y -> y - c over a
+// full window of n positions, and S_n, S_2n are sums of durations (shift-free).  Every tested window lies inside
+// its group (q >= gs + 2n - 1), so with c = the run's first retire time and every shifted time in (-lim, lim),
+// all window sums fit int64 exactly; cond1 / cond2 are then evaluated exactly as on the
+// unshifted values (in i128); n * lim^2 < 2^61 also bounds every difference of two window sums (the
+// per-thread deltas and their block scan).  A run whose span has a time outside the range takes the general path below.
+constexpr int WPT_F = 33;                 // positions per thread (odd: conflict-free 8-byte shared reads)
+constexpr int WITEM_F = WT * WPT_F;       // one item covers a run
+static_assert(RUN <= WITEM_F, "a fast-path run is one item");
+struct FSums {
+  int64_t sx, sy, s2n, sxy, sxx;
+};
+__device__ __forceinline__ void fs_add(FSums& a, const FSums& b) {
+  a.sx += b.sx; a.sy += b.sy; a.s2n += b.s2n; a.sxy += b.sxy; a.sxx += b.sxx;
+}
+__device__ __forceinline__ void fs_zero(FSums& a) { a.sx = a.sy = a.s2n = a.sxy = a.sxx = 0; }
+__device__ __forceinline__ FSums fs_shfl_up(const FSums& v, int d) {
+  FSums r;
+  r.sx = __shfl_up_sync(0xffffffffu, v.sx, d);
+  r.sy = __shfl_up_sync(0xffffffffu, v.sy, d);
+  r.s2n = __shfl_up_sync(0xffffffffu, v.s2n, d);
+  r.sxy = __shfl_up_sync(0xffffffffu, v.sxy, d);
+  r.sxx = __shfl_up_sync(0xffffffffu, v.sxx, d);
+  return r;
+}
+__device__ __forceinline__ FSums fs_shfl_xor(const FSums& v, int m) {
+  FSums r;
+  r.sx = __shfl_xor_sync(0xffffffffu, v.sx, m);
+  r.sy = __shfl_xor_sync(0xffffffffu, v.sy, m);
+  r.s2n = __shfl_xor_sync(0xffffffffu, v.s2n, m);
+  r.sxy = __shfl_xor_sync(0xffffffffu, v.sxy, m);
+  r.sxx = __shfl_xor_sync(0xffffffffu, v.sxx, m);
+  return r;
+}
+// cond2 (mean check, L229) then cond1 (Eq. 1 slope within delta, L222-225) on the fast path's int64 window sums.  cond2 in int64: S_2n < 4 n lim <= 2^39, delta_den <= 2^16.  cond1 by
+// a filtered predicate: num, den and the two sides of the comparison in fp64 with a rigorous bound on their error
+// (every int64 -> double conversion, product and difference rounds by at most 2^-53 relative; 2^-50 covers their
+// sum); only a comparison within the bound (or den within its bound of 0) is re-done exactly in i128.
+__device__ __forceinline__ bool window_pass_fast(int64_t n, int64_t sx, int64_t sy, int64_t s2n, int64_t sxy,
+                                                 int64_t sxx, uint32_t dnum, uint32_t dden) {
+  if (s2n <= 0) return false;
+  int64_t d2 = 2 * (sy - sx) - s2n;
+  if (d2 < 0) d2 = -d2;
+  if (!((int64_t)dden * d2 < (int64_t)dnum * s2n)) return false;
+  const double fn = (double)n, fx = (double)sx, fy = (double)sy;
+  const double a1 = fn * (double)sxy, a2 = fx * fy, b1 = fn * (double)sxx, b2 = fx * fx;
+  const double num = a1 - a2, den = b1 - b2;
+  const double en = 0x1p-50 * (fabs(a1) + fabs(a2)), ed = 0x1p-50 * (b1 + b2);
+  if (den < -ed) return false;
+  if (den > ed) {
+    const double L = (double)dden * fabs(den - num), R = (double)dnum * den;
+    const double m = (double)dden * (en + ed) + (double)dnum * ed + 0x1p-50 * (L + R);
+    if (L + m < R) return true;
+    if (L - m > R) return false;
+  }
+  const i128 inum = (i128)n * sxy - (i128)sx * sy;
+  const i128 iden = (i128)n * sxx - (i128)sx * sx;
+  if (iden <= 0) return false;
+  i128 diff = iden - inum;
+  if (diff < 0) diff = -diff;
+  return (i128)dden * diff < (i128)dnum * iden;
+}
+// returns false (nothing written but the shared buffer) when a time falls outside the range: caller goes general
+__device__ bool window_run_fast(const WinArgs& a, uint32_t g, int64_t gs, int64_t P0, int64_t P1, int2* ring,
+                                FSums* wpart, unsigned long long* best) {
+  const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
+  const int64_t n = a.n, base0 = P0 - 2 * n, span = P1 - base0;
+  const int64_t c = (int64_t)__ldg(a.Y + (base0 > gs ? base0 : gs));
+  bool ok = true;
+  constexpr int FU = 8;  // loads in flight per thread (the fill is latency-bound otherwise)
+  for (int64_t i0 = 0; i0 < span; i0 += WT * FU) {
+    uint64_t xv[FU], yv[FU];
+#pragma unroll
+    for (int u = 0; u < FU; ++u) {
+      const int64_t i = i0 + u * WT + tid, q = base0 + i;
+      const bool in = i < span && q >= gs;
+      xv[u] = in ? __ldg(a.X + q) : (uint64_t)c;
+      yv[u] = in ? __ldg(a.Y + q) : (uint64_t)c;
+    }
+#pragma unroll
+    for (int u = 0; u < FU; ++u) {
+      const int64_t i = i0 + u * WT + tid;
+      const int64_t x = (int64_t)xv[u] - c, y = (int64_t)yv[u] - c;  // positions < gs: (0, 0)
+      ok &= x > -a.lim && x < a.lim && y > -a.lim && y < a.lim;
+      if (i < span) ring[i] = make_int2((int)x, (int)y);
+    }
+  }
+  if (!__syncthreads_and(ok)) return false;
+  // base: windows ending at P0 - 1 ([P0-n, P0-1] and [P0-2n, P0-1]); positions < gs are (0, 0)
+  FSums s;
+  fs_zero(s);
+  for (int64_t i = tid; i < 2 * n; i += WT) {
+    const int2 v = ring[i];
+    s.s2n += (int64_t)v.y - v.x;
+    if (i >= n) {
+      s.sx += v.x; s.sy += v.y;
+      s.sxy += (int64_t)v.x * v.y; s.sxx += (int64_t)v.x * v.x;
+    }
+  }
+  for (int o = 16; o > 0; o >>= 1) fs_add(s, fs_shfl_xor(s, o));
+  if (lane == 0) wpart[wid] = s;
+  if (tid == 0) *best = ~0ull;
+  __syncthreads();
+  FSums base;
+  fs_zero(base);
+  for (int k = 0; k < WT / 32; ++k) fs_add(base, wpart[k]);
+  __syncthreads();
+  // pass 1: this thread's deltas over its WPT_F positions
+  const int64_t r0 = 2 * n + (int64_t)tid * WPT_F, rend = P1 - base0;  // ring index of q = q - base0
+  FSums dl;
+  fs_zero(dl);
+#pragma unroll 3
+  for (int u = 0; u < WPT_F; ++u) {
+    const int64_t i = r0 + u;
+    if (i < rend) {
+      const int2 vs = ring[i], vo = ring[i - n], v2 = ring[i - 2 * n];
+      dl.sx += (int64_t)vs.x - vo.x; dl.sy += (int64_t)vs.y - vo.y;
+      dl.s2n += ((int64_t)vs.y - vs.x) - ((int64_t)v2.y - v2.x);
+      dl.sxy += (int64_t)vs.x * vs.y - (int64_t)vo.x * vo.y;
+      dl.sxx += (int64_t)vs.x * vs.x - (int64_t)vo.x * vo.x;
+    }
+  }
+  FSums incl = dl;
+  for (int o = 1; o < 32; o <<= 1) {
+    const FSums t = fs_shfl_up(incl, o);
+    if (lane >= o) fs_add(incl, t);
+  }
+  if (lane == 31) wpart[wid] = incl;
+  __syncthreads();
+  FSums w = base;
+  for (int k = 0; k < wid; ++k) fs_add(w, wpart[k]);
+  fs_add(w, incl);
+  w.sx -= dl.sx; w.sy -= dl.sy; w.s2n -= dl.s2n; w.sxy -= dl.sxy; w.sxx -= dl.sxx;  // exclusive
+  // pass 2: slide and test
+  uint64_t mine = ~0ull;
+  for (int u = 0; u < WPT_F; ++u) {
+    const int64_t i = r0 + u;
+    if (i >= rend) break;
+    const int2 vs = ring[i], vo = ring[i - n], v2 = ring[i - 2 * n];
+    w.sx += (int64_t)vs.x - vo.x; w.sy += (int64_t)vs.y - vo.y;
+    w.s2n += ((int64_t)vs.y - vs.x) - ((int64_t)v2.y - v2.x);
+    w.sxy += (int64_t)vs.x * vs.y - (int64_t)vo.x * vo.y;
+    w.sxx += (int64_t)vs.x * vs.x - (int64_t)vo.x * vo.x;
+    if (window_pass_fast(n, w.sx, w.sy, w.s2n, w.sxy, w.sxx, a.dnum, a.dden)) {
+      mine = (uint64_t)(base0 + i);
+      break;
+    }
+  }
+  if (mine != ~0ull) atomicMin(best, (unsigned long long)mine);
+  __syncthreads();
+  if (tid == 0 && *best != ~0ull) atomicMin((unsigned long long*)&a.gfirst[g], *best);
+  __syncthreads();
+  return true;
 }
 
 // Ticket t = r * G + g names run r of group g: every group's run 0 is handed out before any group's run 1, so a
@@ -661,6 +925,9 @@ __global__ void __launch_bounds__(WT, 2) k_window(WinArgs a) {
   __shared__ uint64_t best, s_gf;
   const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
   __shared__ uint64_t s_item;
+  __shared__ FSums fpart[WT / 32];
+  __shared__ unsigned long long fbest;
+  extern __shared__ int2 ring[];  // fast path: [2n + RUN] shifted (issue, retire) of the run's span
   const uint32_t total = *a.total;
   const int64_t n = a.n;
   for (;;) {
@@ -686,6 +953,7 @@ __global__ void __launch_bounds__(WT, 2) k_window(WinArgs a) {
       const int64_t gs = (int64_t)a.gstart[g], ge = (int64_t)a.gstart[g + 1];
       const int64_t P0 = gs + 2 * n - 1 + (int64_t)r * RUN;
       const int64_t P1 = P0 + RUN < ge ? P0 + RUN : ge;
+      if (a.ring && window_run_fast(a, g, gs, P0, P1, ring, fpart, &fbest)) continue;
       auto X = [&](int64_t q) -> int64_t { return q >= gs ? (int64_t)__ldg(a.X + q) : 0; };
       auto Yv = [&](int64_t q) -> int64_t { return q >= gs ? (int64_t)__ldg(a.Y + q) : 0; };
       // base: windows ending at P0-1 ([P0-n, P0-1] and [P0-2n, P0-1]); positions < gs contribute 0
@@ -952,6 +1220,21 @@ inline void build_runlist(const RunList& rl, const uint32_t* G, const uint32_t* 
   wa.ticket = misc + 2;
 }
 
+// k_window launch: the fast path's shared span when it fits (n <= ~10K), and the shifted-time range
+inline void window_launch(WinArgs& wa, int num_sms, cudaStream_t s) {
+  const uint64_t span = 2 * (uint64_t)wa.n + RUN;
+  const size_t smem = span * sizeof(int2);
+  wa.ring = smem <= 200 * 1024 ? (uint32_t)span : 0u;
+  int lg = 0;
+  while ((1ull << lg) < (uint64_t)(wa.n ? wa.n : 1)) ++lg;  // ceil(log2 n)
+  int L = (61 - lg) / 2;  // n * lim^2 < 2^61: window sums and their differences (deltas, scans) fit int64
+  if (L > 31) L = 31;
+  wa.lim = (int64_t)1 << L;
+  const size_t dyn = wa.ring ? smem : 0;
+  if (dyn) cudaFuncSetAttribute(k_window, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)dyn);
+  note_launch(), k_window<<<(unsigned)num_sms * 2, WT, dyn, s>>>(wa);
+}
+
 struct Layout {
   int mode;          // 1: job multisplit on BB ids (B <= 256); 2: on per-kernel compacted ids (B <= 8192);
                      // 0: LSD radix sort of composite keys (larger B)
@@ -1048,9 +1331,13 @@ cudaError_t launch_stable(const photon_timing& t, const uint64_t* kbb, photon_st
         note_launch(), k_lid_scan<<<1, 1024, 0, s>>>(K, L.coff, L.bk, L.goff, L.hb, L.misc + 0, L.hn, err);
         note_launch(), k_lid_groups<<<gk, 256, 0, s>>>(K, L.nw, L.bits, L.lbase, L.goff, L.gkb);
       }
-      cudaMemsetAsync(L.hist, 0, sizeof(uint32_t) * L.hn, s);
-      note_launch(), k_job_hist<<<gj, 256, 0, s>>>(t, jm, L.n_jobs, L.hist);
-      scan_u32(L.hist, L.hist, L.hn, L.bsum, L.misc + 4, s);
+      // compact: only hb[K] cells are live (C5: ~R/128 of the 2R + 65536 reserved)
+      const uint64_t* hlive = jm.compact ? L.hb + K : nullptr;
+      if (jm.compact) note_launch(), k_zero_live<<<(unsigned)num_sms * 4, 256, 0, s>>>(L.hist, L.hn, hlive);
+      else cudaMemsetAsync(L.hist, 0, sizeof(uint32_t) * L.hn, s);
+      const unsigned gh = (unsigned)umin64(ceil_div(L.n_jobs, HW), (uint64_t)num_sms * 12);
+      note_launch(), k_job_hist<<<gh, HW * 32, 0, s>>>(t, jm, L.n_jobs, L.hist);
+      scan_u32(L.hist, L.hist, L.hn, L.bsum, L.misc + 4, s, hlive);
       // group starts first: kernels with > 256 local ids use the scanned cells as running offsets in the scatter
       note_launch(), k_job_gstart<<<(unsigned)umin64(ceil_div(L.gcap + 1, 256), (uint64_t)num_sms * 8), 256, 0, s>>>(
           L.hist, jm, L.goff, L.gkb, K, B, R, (uint64_t)B * L.n_jobs, L.gstart, L.misc + 0);
@@ -1087,7 +1374,7 @@ cudaError_t launch_stable(const photon_timing& t, const uint64_t* kbb, photon_st
     wa.X = L.X; wa.Y = L.Y; wa.gstart = L.gstart; wa.G = L.misc + 0;
     wa.n = p.window_n; wa.dnum = p.delta_num; wa.dden = p.delta_den; wa.gfirst = L.gfirst;
     build_runlist(L.rl, L.misc + 0, L.nruns, L.misc, L.gcap, num_sms, wa, s);
-    note_launch(), k_window<<<(unsigned)num_sms * 2, WT, 0, s>>>(wa);
+    window_launch(wa, num_sms, s);
     // 5. outputs
     note_launch(), k_finish<<<(unsigned)umin64(ceil_div(L.gcap * 32, 256), (uint64_t)num_sms * 8), 256, 0, s>>>(
         idx, L.X, L.Y, L.misc + 0, L.gfirst, t.kernel_rec_off, K, B, p.window_n, L.mode, L.gkb, first_stable, dur);
@@ -1133,7 +1420,7 @@ cudaError_t launch_warp_stable(const photon_timing& t, const uint8_t* ok, uint32
   wa.X = t.issue; wa.Y = t.retire; wa.gstart = t.kernel_rec_off; wa.G = misc + 0;
   wa.n = n; wa.dnum = dnum; wa.dden = dden; wa.gfirst = gfirst;
   build_runlist(rl, misc + 0, nruns, misc, K, num_sms, wa, s);
-  note_launch(), k_window<<<(unsigned)num_sms * 2, WT, 0, s>>>(wa);
+  window_launch(wa, num_sms, s);
   note_launch(), k_warp_finish<<<gk, 256, 0, s>>>(t.kernel_rec_off, K, t.issue, t.retire, gfirst, n, switch_at, dur);
   return cudaGetLastError();
 }

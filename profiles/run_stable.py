@@ -12,11 +12,13 @@ from paper_conf_micro_liusc23_b200 import DeviceTiming, DeviceTrace, Photon  # n
 
 cfg = int(sys.argv[1]) if len(sys.argv) > 1 else 3
 reps = int(sys.argv[2]) if len(sys.argv) > 2 else 3
+k1 = int(sys.argv[3]) if len(sys.argv) > 3 else None  # a kernel prefix (C5: 1000 as in bench.py)
 ph = Photon(0)
 g = tg.Generator(cfg)
-d = DeviceTrace.from_host(g.trace(), ph.device)
+k1 = g.n_kernels if k1 is None else k1
+d = DeviceTrace.from_host(g.kernels_trace(0, k1), ph.device)
 kbb = ph.photon_bbv_build(d, bbv16=False, insts=False, kbb=True)["kernel_bb_insts"]
-dt = DeviceTiming.from_host(g.timing(), ph.device)
+dt = DeviceTiming.from_host(g.timing(0, k1), ph.device)
 o = ph.photon_bb_stable(dt, kbb, 2048)
 a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
 a.record()

@@ -109,6 +109,41 @@ def test_stable_degenerate_cases(ph):
     _check_stable(ph, tm, kbb, n, rate=(951, 1000))
 
 
+@pytest.mark.parametrize("n", [16, 2048])
+def test_stable_wide_time_ranges(ph, n):
+    # k_window's fast path stages run spans as 32-bit times shifted by the run's first retire time and needs every
+    # shifted time within 2^((61 - ceil(log2 n)) / 2); these streams force the general path (huge issue gaps, huge
+    # durations: issue far before the first retire) and switch between the two paths inside one group
+    rng = np.random.default_rng(n)
+    streams = []
+    for kind in range(4):
+        m = 3 * n + 9000 if kind != 3 else 6 * n + 20000
+        if kind == 0:    # gaps up to 2^25: every run spans more than the range
+            gaps = rng.integers(1, 1 << 25, m)
+            dur = np.full(m, 1000) + (rng.random(m) < 0.2) * rng.integers(0, 50, m)
+        elif kind == 1:  # durations ~2^33: shifted issue times far below the range
+            gaps = rng.integers(1, 64, m)
+            dur = (1 << 33) + rng.integers(0, 1000, m)
+        elif kind == 2:  # noisy, never stable, wide
+            gaps = rng.integers(1, 1 << 24, m)
+            dur = rng.integers(1, 1 << 30, m)
+        else:            # narrow for a while, then wide gaps, then narrow again (both paths in one group)
+            gaps = np.where((np.arange(m) > 2 * n + 3000) & (np.arange(m) < 3 * n + 9000),
+                            rng.integers(1, 1 << 26, m), rng.integers(1, 40, m))
+            i = np.arange(m)
+            dur = np.where(i < 3 * n + 9000, 50 + 3 * i, 500)  # drifting mean: stable only after the wide part
+        x = np.cumsum(gaps).astype(np.uint64) + np.uint64(5)
+        y = x + dur.astype(np.uint64)
+        assert int(y.max()) < (1 << 40)
+        bb = (rng.random(m) < 0.1).astype(np.uint16)  # two BBs per kernel
+        o = np.argsort(y, kind="stable")
+        streams.append(list(zip(bb[o].tolist(), x[o].tolist(), y[o].tolist())))
+    tm = _one_kernel_streams(streams, 2)
+    kbb = np.array([[9, 1], [5, 5], [1, 1], [3, 1]], np.uint64)
+    fs, _, _ = _check_stable(ph, tm, kbb, n)
+    assert (fs >= 0).sum() >= 2
+
+
 # ---- K1 on long warps ---------------------------------------------------------------------------------------------
 def _trace_from_lengths(seed, kernels, n_bb, max_len, dup_every=3):
     """kernels: per kernel a list of warp lengths.  Every `dup_every`-th warp repeats the previous warp of the same
