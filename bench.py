@@ -42,6 +42,8 @@ def parse():
     p.add_argument("--a5-c5-kernels", type=int, default=1000, help="C5 kernel batch timed for A5 (a5_c5)")
     p.add_argument("--skip-e2e", action="store_true")
     p.add_argument("--skip-a5", action="store_true")
+    p.add_argument("--sharded", action="store_true",
+                   help="run the multi-GPU code path (plan + per-rank CUDA graph with NCCL) even at one GPU")
     p.add_argument("--skip-cpu", action="store_true")
     p.add_argument("--cpu-kernels", type=int, default=3000, help="C5 kernel prefix timed for cpu_baseline")
     p.add_argument("--skip-configs", action="store_true", help="skip the C1-C4 chain lines")
@@ -199,12 +201,20 @@ def run_photon(args):
     ws, rank, local = dist_env()
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
-    if ws > 1:
+    sh = ws > 1 or args.sharded  # the sharded (multi-GPU) code path
+    if sh:
         import torch.distributed as dist
+        if "MASTER_ADDR" not in os.environ:  # --sharded on one GPU without a launcher
+            import socket
+            so = socket.socket()
+            so.bind(("127.0.0.1", 0))
+            os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(so.getsockname()[1]), RANK="0",
+                              WORLD_SIZE="1")
+            so.close()
         dist.init_process_group("nccl", device_id=dev)
     num, den = (int(x) for x in args.theta.split("/"))
     g = tg.Generator(args.config, args.seed)
-    if ws > 1:
+    if sh:
         cuts = tg.shard_bounds(g.warp_counts(), ws)
         tr = g.trace(int(cuts[rank]), int(cuts[rank + 1]))
     else:
@@ -212,13 +222,23 @@ def run_photon(args):
     ph = Photon(local)
     L = load()
     d = DeviceTrace.from_host(tr, dev)
-    E_total = int(g.warp_counts().sum()) if ws > 1 else tr.n_events
+    E_total = int(g.warp_counts().sum()) if sh else tr.n_events
     W_total = g.n_warps
 
-    if ws > 1:
+    if sh:
+        # sized once (plan: the only host reads), then one CUDA graph per rank: kernels + NCCL collectives, no
+        # host synchronisation and no allocation inside a step
         from paper_conf_micro_liusc23_b200 import dist as pdist
         runner = pdist.ShardedAnalysis(ph, g.n_kernels, g.kernel_warps, tr, d, theta=(num, den))
-        step = lambda check=False: runner.run(check=check)
+        runner.run(check=True)
+        graph = runner.capture()
+
+        def step(check=False):
+            graph.replay()
+            if check:
+                torch.cuda.synchronize()
+                runner.check()
+            return runner.result
     else:
         prev = {}
         def step(check=False):  # the previous step's output tables are reused (no allocation in the timed loop)
@@ -231,7 +251,7 @@ def run_photon(args):
     for _ in range(max(args.warmup - 1, 0)):
         res = step(check=False)
     torch.cuda.synchronize()
-    if ws > 1:
+    if sh:
         torch.distributed.barrier()
 
     clocks = Clocks(local)
@@ -241,7 +261,7 @@ def run_photon(args):
     launches0 = L.photon_launch_count()
     s = torch.cuda.current_stream(dev)
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    if ws > 1:
+    if sh:
         torch.distributed.barrier()
     torch.cuda.synchronize()
     e0.record(s)
@@ -249,7 +269,7 @@ def run_photon(args):
         res = step(check=False)
     e1.record(s)
     torch.cuda.synchronize()
-    if ws > 1:
+    if sh:
         torch.distributed.barrier()
     launches = L.photon_launch_count() - launches0
     ms = e0.elapsed_time(e1) / args.steps
@@ -259,18 +279,31 @@ def run_photon(args):
     L.photon_profile_read(ph.ctx, ph.stream_ptr(), pms, pcnt)
     L.photon_profile(ph.ctx, 0)
     clk = clocks.stop()
-    # errors latched during the timed steps?
+    if sh:
+        # graph replays launch nothing from the host and record no section events: the same step run eagerly
+        # (same kernels, same buffers) gives the per-section times and the launches per step
+        L.photon_profile(ph.ctx, 1)
+        l0 = L.photon_launch_count()
+        for _ in range(args.steps):
+            runner.step()
+        torch.cuda.synchronize()
+        launches = (L.photon_launch_count() - l0)  # = per-step launches x steps, as replayed by the graph
+        L.photon_profile_read(ph.ctx, ph.stream_ptr(), pms, pcnt)
+        L.photon_profile(ph.ctx, 0)
+    # errors latched during the timed steps? (N > 1: also every rank's fixed exchange capacities)
+    if sh:
+        runner.check()
     for k in ("_ws", "_mws"):
         if k in res and res[k] is not None:
             ph.check(res[k])
-    if ws > 1:
+    if sh:
         t = torch.tensor([ms], device=dev, dtype=torch.float64)
         torch.distributed.all_reduce(t, op=torch.distributed.ReduceOp.MAX)
         ms = float(t.item())
 
     sections = {PROF_SECTIONS[i]: {"ms_per_step": pms[i] / args.steps, "launches": int(pcnt[i])}
                 for i in range(len(PROF_SECTIONS)) if pcnt[i]}
-    if ws == 1:
+    if not sh:
         sections["match_stats"] = ph.match_stats(g.n_kernels, res, {"_ws": res["_mws"]})
         sections["types"] = ph.photon_types_total(res, g.n_kernels)
     hbm_peak, peak_src = _peaks()
@@ -293,7 +326,7 @@ def run_photon(args):
             "dtype": "u16/u32/u64 integer (u128 exact compares)", "data": "synthetic (tracegen, seeded; no datasets)",
             "config": {"workload": CONFIG_DESC.get(args.config), "events": E_total, "warps": W_total,
                        "kernels": g.n_kernels, "bb_ids": g.n_bb, "theta": args.theta,
-                       "parallelism": f"dp{ws} (warp shards)" if ws > 1 else "1 GPU",
+                       "parallelism": f"dp{ws} (warp shards)" if sh else "1 GPU",
                        "l2": f"inputs ({(2 * E_total + 8 * W_total) / 1e9:.2f} GB) exceed the 126 MB L2; no flush",
                        "match_dist": "not requested in the timed chain (the metric counts decisions; the reported "
                                      "distances are a separate pass)"},
@@ -311,6 +344,12 @@ def run_photon(args):
         times = []
         d2h = 0
         pinned_out = None  # page-locked result buffers, allocated once (outside the timed region)
+        if sh:  # the API's sharded runner on the copied inputs, planned once outside the timed region
+            runner_e2e = pdist.ShardedAnalysis(ph, g.n_kernels, g.kernel_warps, tr, dd, theta=(num, den))
+            for k, dst in zip(("kernel_warp_off", "warp_event_off", "bb", "bb_len", "warps_total"),
+                              (dd.kernel_warp_off, dd.warp_event_off, dd.bb, dd.bb_len, dd.warps_total)):
+                dst.copy_(host[k])
+            runner_e2e.run(check=True)
         for i in range(args.e2e_steps + 1):
             torch.cuda.synchronize()
             a0, a1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
@@ -318,8 +357,8 @@ def run_photon(args):
             for k, dst in zip(("kernel_warp_off", "warp_event_off", "bb", "bb_len", "warps_total"),
                               (dd.kernel_warp_off, dd.warp_event_off, dd.bb, dd.bb_len, dd.warps_total)):
                 dst.copy_(host[k], non_blocking=True)
-            if ws > 1:
-                r = pdist.ShardedAnalysis(ph, g.n_kernels, g.kernel_warps, tr, dd, theta=(num, den)).run(check=False)
+            if sh:
+                r = runner_e2e.step()
             else:
                 r = ph.analyse(dd, theta=(num, den), check=False)
             outs = [r["warp_type"], r["kernel_type_off"], r["warp_sampling_ok"], r["match"]]
@@ -333,7 +372,7 @@ def run_photon(args):
             if i > 0:
                 times.append(a0.elapsed_time(a1))
         e2e_ms = statistics.mean(times)
-        if ws > 1:
+        if sh:
             t = torch.tensor([e2e_ms], device=dev, dtype=torch.float64)
             torch.distributed.all_reduce(t, op=torch.distributed.ReduceOp.MAX)
             e2e_ms = float(t.item())
@@ -341,7 +380,7 @@ def run_photon(args):
                        "d2h_bytes_per_step": int(d2h), "ms_per_step": e2e_ms, "steps": args.e2e_steps}
 
     # ---- the metric's chain on C1-C4 (C2 also with a 2x-L2 scrub between steps: its HBM fraction) ----
-    if not args.skip_configs and ws == 1:
+    if not args.skip_configs and not sh:
         import ctypes as _ct
         line["configs"] = {}
         for cfg, scrub in ((1, 0), (2, 0), (2, 256 << 20), (3, 0), (4, 0)):
@@ -383,8 +422,45 @@ def run_photon(args):
                        "no flush (inputs " + ("< 126 MB L2" if kb < 126e6 else "> 126 MB L2") + ")")}
             del dc, rc, buf
 
+    # ---- N > 1: the kernel-sharded A5 (whole kernels per rank, ~equal records; outputs all-gathered), one CUDA
+    # graph per rank (kernels + NCCL all-gathers), time = max over ranks ----
+    if not args.skip_a5 and sh:
+        ga = tg.Generator(args.a5_config)
+        wc = np.concatenate([[0], np.cumsum(ga.warp_counts().astype(np.int64))])  # records = events per warp
+        rec = wc[ga.kwoff[1:].astype(np.int64)] - wc[ga.kwoff[:-1].astype(np.int64)]
+        kc = pdist.kernel_ranges(rec, ws)
+        k0, k1 = int(kc[rank]), int(kc[rank + 1])
+        tml = ga.timing(k0, k1)
+        dal = DeviceTrace.from_host(ga.kernels_trace(k0, k1), dev)
+        kbl = ph.photon_bbv_build(dal, bbv16=False, insts=False, kbb=True)["kernel_bb_insts"]
+        st = pdist.ShardedStable(ph, DeviceTiming.from_host(tml, dev, n_bb=ga.n_bb), kbl, kc, ga.n_bb).plan()
+        sgraph = st.capture()
+        for _ in range(max(args.warmup - 1, 0)):
+            sgraph.replay()
+        torch.cuda.synchronize()
+        torch.distributed.barrier()
+        b0, b1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        n5 = max(args.steps // 4, 3)
+        b0.record(s)
+        for _ in range(n5):
+            sgraph.replay()
+        b1.record(s)
+        torch.cuda.synchronize()
+        torch.distributed.barrier()
+        st.check()
+        t = torch.tensor([b0.elapsed_time(b1) / n5], device=dev, dtype=torch.float64)
+        torch.distributed.all_reduce(t, op=torch.distributed.ReduceOp.MAX)
+        ams = float(t.item())
+        R = int(rec.sum())
+        line["a5"] = {"metric": "BB timing records tested/sec (stability test + switch)", "value": R / (ams / 1000),
+                      "unit": "records/s", "ms_per_step": ams, "records": R, "scaling": "strong",
+                      "parallelism": f"dp{ws} (kernel shards by records; first_stable / stable_dur_sum / switch_at "
+                                     "all-gathered; one CUDA graph per rank)",
+                      "workload": f"{CONFIG_DESC.get(args.a5_config)} timing stream (wave model), n=2048, "
+                                  "delta=3/100"}
+
     # ---- A5 on its own timing stream (reported beside the metric) ----
-    if not args.skip_a5 and ws == 1:
+    if not args.skip_a5 and not sh:
         ga = tg.Generator(args.a5_config)
         tm = ga.timing()
         ta = ga.trace()
@@ -438,7 +514,7 @@ def run_photon(args):
                       "stable_bb_types": int((to_numpy_i64(o["first_stable"]) >= 0).sum())}
 
     # ---- A5 on C5 stress kernels (B = 4096 > 256: the composite-key radix path), a kernel batch ----
-    if not args.skip_a5 and ws == 1:
+    if not args.skip_a5 and not sh:
         g5 = tg.Generator(5)
         k5 = min(args.a5_c5_kernels, g5.n_kernels)
         tm5 = g5.timing(0, k5)
@@ -468,7 +544,7 @@ def run_photon(args):
         del dt5, o5, d5, kbb5
 
     # ---- N1 (warp-level stability, L262) on the same config's warp streams, gated by A2's dominance ----
-    if not args.skip_a5 and ws == 1:
+    if not args.skip_a5 and not sh:
         gw = tg.Generator(args.a5_config)
         tw = gw.warp_timing()
         ty = ph.photon_warp_group(DeviceTrace.from_host(gw.trace(), dev))
@@ -500,7 +576,7 @@ def run_photon(args):
                       "dominant_kernels": int(okd.to(torch.int64).sum().item())}
 
     # ---- N2 (full-BBV exact grouping, L154/L161) on the same config's trace ----
-    if not args.skip_a5 and ws == 1:
+    if not args.skip_a5 and not sh:
         g2 = tg.Generator(args.a5_config)
         t2 = g2.trace()
         d2 = DeviceTrace.from_host(t2, dev)
@@ -552,11 +628,11 @@ def run_photon(args):
                       "reused_from_pool": int(((mm[Kp:] >= 0) & (mm[Kp:] < Kp)).sum()),
                       "roofline": None, "note": "A3/A4 over pool + run: compare ops (ALU), not a streaming pass"}
 
-    if rank == 0 and ws == 1 and not args.skip_cpu:
+    if rank == 0 and not sh and not args.skip_cpu:
         line["cpu_baseline"] = cpu_baseline(args)
     if rank == 0:
         print(json.dumps(line), flush=True)
-    if ws > 1:
+    if sh:
         torch.distributed.destroy_process_group()
 
 

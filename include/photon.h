@@ -170,10 +170,14 @@ PHOTON_API int photon_kernel_match(photon_ctx *ctx, uint32_t n_kernels, const ph
 /* A3 (L178, Fig 5) and the split form of photon_kernel_match used by the multi-GPU driver (signatures
  * all-reduced, pair lists all-gathered between the steps).  photon_sig_build is the A3 entry point: it writes g_k
  * (sig, u64, the rows' order: sig_off = 16 * kernel_type_off) and N_k (mass, u64) for kernels [k_lo, k_hi)
- * (others untouched); ERANGE when N_k >= 2^50.
+ * and zeros for every other kernel (so the buffers of ranks owning disjoint kernel ranges sum, by an all-reduce,
+ * to the whole table); ERANGE when N_k >= 2^50.
  * match_scan appends the close pairs (k, r) with k in [k_lo, k_hi) to pairs[] (u64: k << 32 | r), count in
- * *n_pairs (DEVICE u64, zeroed by the call); `pair_capacity` entries fit.  match_resolve takes the union of all
- * pair lists (any order) and runs the launch-order resolution; its result does not depend on pair order. */
+ * *n_pairs (DEVICE u64, zeroed by the call; > pair_capacity means pairs were dropped); `pair_capacity` entries
+ * fit and every entry past the last pair holds PHOTON_PAIR_PAD, so fixed-capacity buffers of several ranks can be
+ * all-gathered as they are.  match_resolve takes the union of all pair lists (any order; PHOTON_PAIR_PAD entries
+ * are skipped) and runs the launch-order resolution; its result does not depend on pair order. */
+#define PHOTON_PAIR_PAD 0xFFFFFFFFFFFFFFFFull
 PHOTON_API int photon_sig_build(photon_ctx *ctx, uint32_t n_kernels, const uint64_t *kernel_type_off, const uint32_t *type_key,
                      const uint64_t *type_count, uint32_t k_lo, uint32_t k_hi, uint64_t *sig /*[16*T]*/,
                      uint64_t *mass /*[K]*/, void *ws /* >= 256 bytes: error latch */, size_t ws_bytes, void *stream);
@@ -337,9 +341,14 @@ typedef struct {
   uint64_t count;
   uint64_t first_warp; /* global warp index */
 } photon_type_row;
-/* Writes the local types as rows (global ids) to rows[0..T_local); T_local = local->kernel_type_off[K_local]. */
+/* Writes the local types as rows (global ids) to rows[0..min(T_local, row_capacity)) and padding rows (kernel =
+ * PHOTON_ROW_PAD, skipped by photon_types_merge) to rows[T_local..row_capacity); T_local =
+ * local->kernel_type_off[K_local] is stored to *n_rows (DEVICE u64, may be NULL) -- T_local > row_capacity means
+ * rows were dropped.  Fixed-capacity row buffers of all ranks can thus be all-gathered without a host sync. */
+#define PHOTON_ROW_PAD 0xFFFFFFFFu
 PHOTON_API int photon_types_export(photon_ctx *ctx, uint32_t n_kernels_local, const photon_types *local, uint32_t kernel_base,
-                        uint64_t warp_base, photon_type_row *rows, void *stream);
+                        uint64_t warp_base, photon_type_row *rows, uint64_t row_capacity, uint64_t *n_rows,
+                        void *stream);
 /* Merges rows of all shards (any order; rows with equal (kernel, key) add counts and take the min first_warp)
  * into canonical global tables for K kernels; `kernel_warps` [K] = analysed warps per kernel (for the dominance
  * decision).  global->warp_type is ignored. */

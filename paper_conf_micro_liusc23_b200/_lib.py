@@ -59,6 +59,8 @@ class WarpStableParams(ctypes.Structure):
 
 
 TYPE_ROW_BYTES = 88  # photon_type_row
+ROW_PAD = 0xFFFFFFFF  # PHOTON_ROW_PAD: kernel id of a padding row
+PAIR_PAD = 0xFFFFFFFFFFFFFFFF  # PHOTON_PAIR_PAD: an unused pair slot
 PROF_SECTIONS = ["bbv_fused", "bbv", "kbb", "group_unfused", "canon", "sig", "scan", "resolve", "stable", "prep"]
 
 # (name, restype, argtypes) — mirrors include/photon.h
@@ -111,7 +113,8 @@ _SIGS = [
     ("photon_kernel_match_pooled", c_int, [c_void_p, c_uint32, POINTER(Types), c_void_p, c_uint64, c_uint32,
                                            POINTER(Types), c_void_p, c_uint64, MatchParams, c_void_p, c_size_t,
                                            c_void_p, c_void_p, c_void_p]),
-    ("photon_types_export", c_int, [c_void_p, c_uint32, POINTER(Types), c_uint32, c_uint64, c_void_p, c_void_p]),
+    ("photon_types_export", c_int, [c_void_p, c_uint32, POINTER(Types), c_uint32, c_uint64, c_void_p, c_uint64,
+                                    c_void_p, c_void_p]),
     ("photon_merge_workspace_bytes", c_size_t, [c_uint64, c_uint32]),
     ("photon_types_merge", c_int, [c_void_p, c_void_p, c_uint64, c_uint32, c_void_p, c_void_p, c_size_t,
                                    POINTER(Types), c_void_p]),

@@ -394,8 +394,11 @@ class Photon:
                                          ws.data_ptr(), ws.numel(), self.stream_ptr(stream)))
         return ws
 
-    def photon_match_scan(self, K, kto, sig, mass, warps_total, params, k_lo, k_hi, pairs, n_pairs, stream=None):
-        nb = self.L.photon_match_workspace_bytes(K, 1, pairs.numel())
+    def photon_match_scan(self, K, kto, sig, mass, warps_total, params, k_lo, k_hi, pairs, n_pairs, stream=None,
+                          ws_pairs: int = 0):
+        """ws_pairs: room for the filter's candidate list in the workspace (default: the pair buffer's size; a
+        candidate list that does not fit latches ECAPACITY in the workspace)."""
+        nb = self.L.photon_match_workspace_bytes(K, 1, max(int(ws_pairs), pairs.numel()))
         ws = self.workspace("scan", nb)
         self._rc(self.L.photon_match_scan(self.ctx, K, kto.data_ptr(), sig.data_ptr() if sig.numel() else None,
                                           mass.data_ptr(), warps_total.data_ptr(), params, k_lo, k_hi, ws.data_ptr(),
@@ -486,10 +489,12 @@ class Photon:
         return o
 
     # -- multi-GPU helpers -------------------------------------------------------------------------------------
-    def photon_types_export(self, K_local, ty, kernel_base, warp_base, rows, stream=None):
+    def photon_types_export(self, K_local, ty, kernel_base, warp_base, rows, n_rows=None, stream=None):
+        """rows: [row_capacity, 88] uint8 (padded with PHOTON_ROW_PAD rows); n_rows: device int64 [1] or None."""
         tc = self.types_c(ty)
         self._rc(self.L.photon_types_export(self.ctx, K_local, ctypes.byref(tc), kernel_base, warp_base,
-                                            rows.data_ptr(), self.stream_ptr(stream)))
+                                            rows.data_ptr(), int(rows.shape[0]),
+                                            None if n_rows is None else n_rows.data_ptr(), self.stream_ptr(stream)))
 
     def photon_types_merge(self, rows, n_rows, K, kernel_warps, out: dict, stream=None):
         nb = self.L.photon_merge_workspace_bytes(n_rows, K)

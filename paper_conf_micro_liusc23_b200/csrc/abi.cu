@@ -718,6 +718,7 @@ int photon_match_scan(photon_ctx* ctx, uint32_t K, const uint64_t* kto, const ui
   ctx->last_ws = ws;
   CK(cudaMemsetAsync(m.err, 0, sizeof(DevErr), s), "memset");
   m.mw.sigf = nullptr;  // T is not known here: the exact screen converts the u64 signature on the fly
+  CK(cudaMemsetAsync(pairs, 0xFF, sizeof(uint64_t) * pair_capacity, s), "memset");  // unused slots: PHOTON_PAIR_PAD
   CK(launch_match_scan(K, kto, sig, mass, warps_total, params, k_lo, k_hi, m.mw, pairs, pair_capacity, n_pairs, m.err,
                        ctx->num_sms, s),
      "scan");
@@ -861,11 +862,13 @@ int photon_bb_predict(photon_ctx* ctx, const photon_trace* t, const int64_t* fir
 
 // ---- multi-GPU helpers ------------------------------------------------------------------------------------
 int photon_types_export(photon_ctx* ctx, uint32_t K_local, const photon_types* local, uint32_t kernel_base,
-                        uint64_t warp_base, photon_type_row* rows, void* stream) {
+                        uint64_t warp_base, photon_type_row* rows, uint64_t row_capacity, uint64_t* n_rows,
+                        void* stream) {
   if (!ctx) return PHOTON_EINVAL;
-  if (!local || !rows || K_local == 0) return fail(ctx, PHOTON_EINVAL, "bad export arguments");
+  if (!local || !rows || K_local == 0 || row_capacity == 0) return fail(ctx, PHOTON_EINVAL, "bad export arguments");
   CK(cudaSetDevice(ctx->device), "cudaSetDevice");
-  CK(launch_types_export(K_local, *local, kernel_base, warp_base, rows, (cudaStream_t)stream), "export");
+  CK(launch_types_export(K_local, *local, kernel_base, warp_base, rows, row_capacity, n_rows, (cudaStream_t)stream),
+     "export");
   return PHOTON_OK;
 }
 

@@ -77,7 +77,7 @@ cudaError_t launch_canonicalise(const HashTable& ht, uint32_t K, const uint64_t*
                                 DevErr* err, int num_sms, cudaStream_t s);
 // multi-GPU helpers
 cudaError_t launch_types_export(uint32_t K, const photon_types& local, uint32_t kernel_base, uint64_t warp_base,
-                                photon_type_row* rows, cudaStream_t s);
+                                photon_type_row* rows, uint64_t row_cap, uint64_t* n_rows, cudaStream_t s);
 cudaError_t launch_rows_insert(const photon_type_row* rows, uint64_t n, uint32_t K, const HashTable& ht,
                                DevErr* err, cudaStream_t s);
 // warp_type_global[v] = canonical id (in the merged table) of local warp v's type (direct hash lookup)

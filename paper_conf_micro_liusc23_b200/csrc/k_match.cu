@@ -29,13 +29,18 @@ namespace photon {
 namespace {
 
 // ---- A3: g = count * key, N = sum g (one warp per kernel) ------------------------------------------------
-__global__ void k_sig(uint32_t k_lo, uint32_t k_hi, const uint64_t* __restrict__ kto,
+__global__ void k_sig(uint32_t K, uint32_t k_lo, uint32_t k_hi, const uint64_t* __restrict__ kto,
                       const uint32_t* __restrict__ key, const uint64_t* __restrict__ count, uint64_t* __restrict__ sig,
                       uint64_t* __restrict__ mass, DevErr* err) {
   uint32_t warp = (blockIdx.x * blockDim.x + threadIdx.x) >> 5, lane = threadIdx.x & 31;
-  uint32_t k = k_lo + warp;
-  if (k >= k_hi) return;
+  uint32_t k = warp;
+  if (k >= K) return;
   uint64_t r0 = kto[k], r1 = kto[k + 1];
+  if (k < k_lo || k >= k_hi) {  // not this caller's kernel: zero (rank buffers then sum to the whole table)
+    for (uint64_t i = r0 * 16 + lane; i < r1 * 16; i += 32) sig[i] = 0;
+    if (lane == 0) mass[k] = 0;
+    return;
+  }
   uint64_t acc = 0;
   bool over = false;
   for (uint64_t i = r0 * 16 + lane; i < r1 * 16; i += 32) {
@@ -385,6 +390,7 @@ __global__ void k_cand_count(const uint64_t* pairs, uint64_t n_host, const uint6
   uint64_t n = pair_count(n_host, n_dev);
   uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
   if (i >= n) return;
+  if (pairs[i] == PHOTON_PAIR_PAD) return;  // padding of a fixed-capacity exchange
   uint32_t k = (uint32_t)(pairs[i] >> 32), r = (uint32_t)pairs[i];
   if (k >= K || r >= k) { latch(err, PHOTON_EINVAL, (int64_t)i); return; }
   atomicAdd(&cnt[k], 1u);
@@ -662,10 +668,9 @@ __global__ void k_rep_mindist(uint32_t K, const int64_t* match, uint32_t pool_al
 
 cudaError_t launch_sig_build(uint32_t K, const uint64_t* kto, const uint32_t* type_key, const uint64_t* type_count,
                              uint32_t k_lo, uint32_t k_hi, uint64_t* sig, uint64_t* mass, DevErr* err, cudaStream_t s) {
-  (void)K;
-  if (k_hi <= k_lo) return cudaSuccess;
-  uint32_t n = k_hi - k_lo;
-  note_launch(), k_sig<<<(unsigned)ceil_div((uint64_t)n * 32, 256), 256, 0, s>>>(k_lo, k_hi, kto, type_key, type_count, sig, mass, err);
+  if (K == 0) return cudaSuccess;
+  note_launch(), k_sig<<<(unsigned)ceil_div((uint64_t)K * 32, 256), 256, 0, s>>>(K, k_lo, k_hi, kto, type_key,
+                                                                                 type_count, sig, mass, err);
   return cudaGetLastError();
 }
 

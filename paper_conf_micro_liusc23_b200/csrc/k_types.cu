@@ -388,12 +388,24 @@ __device__ __forceinline__ uint32_t row_kernel(const uint64_t* kto, uint32_t K, 
   return lo;
 }
 
+// rows [0, min(T, cap)) = the local types; [T, cap) = padding rows (kernel PHOTON_ROW_PAD, skipped by the merge);
+// n_rows (device, optional) = T, so a caller with a fixed capacity can detect T > cap
 __global__ void k_export(uint32_t K, photon_types local, uint32_t kernel_base, uint64_t warp_base,
-                         photon_type_row* rows) {
+                         photon_type_row* rows, uint64_t cap, uint64_t* n_rows) {
   uint64_t T = local.kernel_type_off[K];
   uint64_t r = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
-  if (r >= T) return;
+  if (r == 0 && n_rows) *n_rows = T;
+  if (r >= cap) return;
   photon_type_row x;
+  if (r >= T) {
+    x.kernel = PHOTON_ROW_PAD;
+    x.pad = 0;
+    for (int j = 0; j < 16; ++j) x.key[j] = 0;
+    x.count = 0;
+    x.first_warp = 0;
+    rows[r] = x;
+    return;
+  }
   x.kernel = kernel_base + row_kernel(local.kernel_type_off, K, r);
   x.pad = 0;
   for (int j = 0; j < 16; ++j) x.key[j] = local.type_key[r * 16 + j];
@@ -406,6 +418,7 @@ __global__ void k_rows_insert(const photon_type_row* rows, uint64_t n, uint32_t 
   uint64_t r = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
   if (r >= n) return;
   const photon_type_row x = rows[r];
+  if (x.kernel == PHOTON_ROW_PAD) return;  // padding of a fixed-capacity exchange
   if (x.kernel >= K || x.count >= (1ull << 32)) { latch(err, PHOTON_ERANGE, (int64_t)r); return; }
   uint64_t h = hash_key(x.kernel, x.key);
   ht_insert(ht, err, x.kernel, x.key, h, (uint32_t)x.count, x.first_warp);
@@ -497,10 +510,11 @@ cudaError_t launch_remap_entries(const EntryPool& ep, uint64_t W, const uint32_t
 }
 
 cudaError_t launch_types_export(uint32_t K, const photon_types& local, uint32_t kernel_base, uint64_t warp_base,
-                                photon_type_row* rows, cudaStream_t s) {
-  // T is on the device; launch for the capacity bound and guard inside
-  uint64_t cap = local.capacity ? local.capacity : 1;
-  note_launch(), k_export<<<(unsigned)ceil_div(cap, 256), 256, 0, s>>>(K, local, kernel_base, warp_base, rows);
+                                photon_type_row* rows, uint64_t row_cap, uint64_t* n_rows, cudaStream_t s) {
+  // T is on the device: launch for the row capacity and guard inside
+  const uint64_t cap = row_cap ? row_cap : 1;
+  note_launch(), k_export<<<(unsigned)ceil_div(cap, 256), 256, 0, s>>>(K, local, kernel_base, warp_base, rows,
+                                                                         row_cap, n_rows);
   return cudaGetLastError();
 }
 
