@@ -513,6 +513,23 @@ class Photon:
                                            warp_type_global.data_ptr() if W_local else None,
                                            self.stream_ptr(stream)))
 
+    # -- CUDA graphs ------------------------------------------------------------------------------------------
+    def capture(self, fn):
+        """Capture fn() -- a sync-free sequence of libphoton calls on the current stream (check=False, buffers
+        reused through `out=`) -- in one CUDA graph.  fn runs once eagerly on the capture stream first (so every
+        cached workspace already has its final size and nothing is allocated inside the graph).  Returns
+        (graph, the captured call's result); graph.replay() re-runs the whole sequence with one launch."""
+        torch = self.torch
+        s = torch.cuda.Stream(device=self.device)
+        s.wait_stream(torch.cuda.current_stream(self.device))
+        with torch.cuda.stream(s):
+            fn()
+        torch.cuda.current_stream(self.device).wait_stream(s)
+        g = torch.cuda.CUDAGraph()
+        with torch.cuda.graph(g):
+            res = fn()
+        return g, res
+
     # -- the benchmarked chain ---------------------------------------------------------------------------------
     def analyse(self, t: DeviceTrace, theta=(1, 20), n_cores=64, pool_all_prior=0, want_dist=False, stream=None,
                 check: bool = True, capacity_hint: int = 0, pair_capacity: int = 0, out: Optional[dict] = None) -> dict:

@@ -289,3 +289,30 @@ def test_out_reuse_analyse_and_full(ph):
     assert h1["warp_type"] is not f6["warp_type"]
     p16, _, _ = oracle.bbv(tr1, want_kbb=False)
     assert np.array_equal(_np(h1["warp_type"], np.uint32), oracle.group_full(tr1, p16)["warp_type"])
+
+
+@pytest.mark.parametrize("cfg", [6, 1])
+def test_chain_cuda_graph_replay_matches_oracle(ph, cfg):
+    # bench.py times the chain as one CUDA graph replay per step: the replayed result must equal the oracle
+    import torch
+    from paper_conf_micro_liusc23_b200 import DeviceTrace
+    g = tg.Generator(cfg)
+    tr = g.trace()
+    d = DeviceTrace.from_host(tr, ph.device)
+    r0 = ph.analyse(d, check=True)
+    graph, r = ph.capture(lambda: ph.analyse(d, check=False, out=r0))
+    for k in ("warp_type", "match"):
+        r[k].fill_(-7)  # the replay must rewrite every output
+    graph.replay()
+    graph.replay()
+    torch.cuda.synchronize()
+    ph.check(r["_ws"])
+    ph.check(r["_mws"])
+    ref = oracle.analyse(tr)
+    T = int(ref["kernel_type_off"][-1])
+    assert np.array_equal(_np(r["kernel_type_off"], np.uint64), ref["kernel_type_off"])
+    assert np.array_equal(_np(r["type_key"], np.uint32).reshape(-1, 16)[:T], ref["type_key"])
+    assert np.array_equal(_np(r["type_count"], np.uint64)[:T], ref["type_count"])
+    assert np.array_equal(_np(r["warp_type"], np.uint32), ref["warp_type"])
+    assert np.array_equal(_np(r["warp_sampling_ok"], np.uint8), ref["warp_sampling_ok"])
+    assert np.array_equal(_np(r["match"], np.int64), ref["match"])
