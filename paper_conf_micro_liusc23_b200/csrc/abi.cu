@@ -500,31 +500,19 @@ struct FullLayout {
 FullLayout full_layout(const photon_trace* t, void* base) {
   Carver c(base);
   FullLayout L;
-  const uint64_t W = t->n_warps + 1, E = t->n_events + 8;
+  const uint64_t W = t->n_warps + 1;
   L.err = c.take<DevErr>(1);
   L.f.h_lo = c.take<uint64_t>(W);
   L.f.h_hi = c.take<uint64_t>(W);
-  L.f.k64 = c.take<uint64_t>(W);
-  L.f.g64 = c.take<uint64_t>(W);
-  L.f.gstart = c.take<uint64_t>(W);
-  L.f.kid = c.take<uint32_t>(W);
-  L.f.perm_a = c.take<uint32_t>(W);
-  L.f.perm_b = c.take<uint32_t>(W);
-  L.f.k32 = c.take<uint32_t>(W);
-  L.f.g32 = c.take<uint32_t>(W);
-  L.f.flag = c.take<uint32_t>(W);
-  L.f.gid = c.take<uint32_t>(W);
-  L.f.wgroup = c.take<uint32_t>(W);
   L.f.list = c.take<uint64_t>(W);
+  L.f.list2 = c.take<uint64_t>(W);
+  L.f.kid = c.take<uint32_t>(W);
+  L.f.wslot = c.take<uint32_t>(W);
   L.f.nlist = c.take<uint32_t>(4);
-  L.f.ekey = c.take<uint64_t>(E);
-  L.f.sorted = c.take<uint64_t>(E);
+  L.f.htab = c.take<ulonglong2>((uint64_t)t->n_bb + 1);
   uint64_t cap = 1024;
-  while (cap < t->n_warps) cap <<= 1;
+  while (cap < 2 * t->n_warps) cap <<= 1;  // groups <= W: load factor <= 1/2
   carve_ht(c, cap, t->n_kernels, L.h);
-  L.h.ht.mask = cap - 1;
-  L.f.cub_bytes = full_cub_bytes(t->n_warps, t->n_events);
-  L.f.cub = c.take<uint8_t>(L.f.cub_bytes + 16);
   L.bytes = c.off + 256;
   return L;
 }
@@ -563,8 +551,8 @@ size_t photon_ingest_workspace_bytes(uint64_t n, uint64_t W) {
   (void)W;
   Carver c(nullptr);
   c.take<DevErr>(1);
-  c.take<uint32_t>(n + 1);
-  c.take<uint8_t>(ingest_cub_bytes(n) + 16);
+  c.take<uint64_t>(n + 1);
+  c.take<uint8_t>(radix_pairs_ws_bytes(n));
   return c.off + 256;
 }
 
@@ -572,19 +560,18 @@ int photon_ingest_tagged(photon_ctx* ctx, uint64_t n, uint64_t W, const uint32_t
                          size_t ws_bytes, uint16_t* bb_out, uint64_t* warp_event_off, void* stream) {
   if (!ctx) return PHOTON_EINVAL;
   if ((n && (!warp || !bb || !bb_out)) || !warp_event_off || !ws) return fail(ctx, PHOTON_EINVAL, "NULL argument");
-  if (W >= (1ull << 32) || n >= (1ull << 40)) return fail(ctx, PHOTON_EINVAL, "n_warps must be < 2^32");
+  if (W >= (1ull << 32) || n >= (1ull << 32)) return fail(ctx, PHOTON_EINVAL, "n and n_warps must be < 2^32");
   const size_t need = photon_ingest_workspace_bytes(n, W);
   if (ws_bytes < need) return fail(ctx, PHOTON_EWORKSPACE, "workspace %zu < %zu bytes", ws_bytes, need);
   Carver c(ws);
   DevErr* err = c.take<DevErr>(1);
-  uint32_t* key_out = c.take<uint32_t>(n + 1);
-  const size_t cb = ingest_cub_bytes(n);
-  void* cub = c.take<uint8_t>(cb + 16);
+  uint64_t* key = c.take<uint64_t>(n + 1);
+  void* sort_ws = c.take<uint8_t>(radix_pairs_ws_bytes(n));
   cudaStream_t s = (cudaStream_t)stream;
   CK(cudaSetDevice(ctx->device), "cudaSetDevice");
   ctx->last_ws = ws;
   CK(cudaMemsetAsync(err, 0, sizeof(DevErr), s), "memset");
-  CK(launch_ingest(n, W, warp, bb, cub, cb, key_out, bb_out, warp_event_off, err, s), "ingest");
+  CK(launch_ingest(n, W, warp, bb, key, sort_ws, bb_out, warp_event_off, err, s), "ingest");
   return PHOTON_OK;
 }
 

@@ -123,21 +123,20 @@ cudaError_t launch_warp_stable(const photon_timing& t, const uint8_t* ok, uint32
                                cudaStream_t s);
 // ---- N2 (k_full.cu): full-BBV exact grouping and tagged-stream ingest ----------------------------------------
 struct FullWs {
-  uint64_t *h_lo, *h_hi, *k64, *g64, *gstart;  // [W]
-  uint32_t *kid, *perm_a, *perm_b, *k32, *g32, *flag, *gid, *wgroup;  // [W]
-  uint64_t* list;    // [W] work list of long warps (hash pass), then of long members (verification)
-  uint32_t* nlist;   // [2] its lengths
-  uint64_t* ekey;    // [E] (warp << 16 | bb) of every event
-  uint64_t* sorted;  // [E] the keys sorted: each warp's events by BB id
-  void* cub;
-  size_t cub_bytes;
+  uint64_t *h_lo, *h_hi;  // [W] order-independent 128-bit hash of each warp's event multiset
+  uint32_t *kid, *wslot;  // [W] kernel of each warp; its hash-table slot
+  uint64_t* list;         // [W] work list of long warps (> 16 events)
+  uint64_t* list2;        // [W] long warps whose sequence differs from their type's first (count verification)
+  uint32_t* nlist;        // [2] the two lengths
+  ulonglong2* htab;       // [B] the two 64-bit mixes of every BB id
 };
-size_t full_cub_bytes(uint64_t W, uint64_t E);
-size_t ingest_cub_bytes(uint64_t n);
+size_t radix_pairs_ws_bytes(uint64_t n);
+cudaError_t launch_radix_pairs(uint64_t* key, uint64_t n, uint32_t bits, void* ws, uint64_t** key_out,
+                               uint32_t** perm_out, cudaStream_t s);
 cudaError_t launch_group_full(const TraceDev& t, const uint32_t* bbv16, const FullWs& f, const HashTable& ht,
                               const CanonWs& cw, const photon_types& out, DevErr* err, int num_sms, cudaStream_t s);
-cudaError_t launch_ingest(uint64_t n, uint64_t W, const uint32_t* warp, const uint16_t* bb, void* cub, size_t cub_bytes,
-                          uint32_t* key_out, uint16_t* bb_out, uint64_t* off, DevErr* err, cudaStream_t s);
+cudaError_t launch_ingest(uint64_t n, uint64_t W, const uint32_t* warp, const uint16_t* bb, uint64_t* key,
+                          void* sort_ws, uint16_t* bb_out, uint64_t* off, DevErr* err, cudaStream_t s);
 // ---- N4 (k_pool.cu): persisted signature pool --------------------------------------------------------------
 cudaError_t launch_pool_export(uint32_t K, const photon_types& ty, const uint64_t* wt, const int64_t* match,
                                uint64_t* keep, uint64_t* ntypes, const photon_types& pool, uint64_t* pwt,

@@ -1297,6 +1297,46 @@ Layout make_layout(const photon_timing& t, void* base) {
 
 size_t stable_ws_bytes(const photon_timing& t) { return make_layout(t, nullptr).bytes; }
 
+// ---- the stable LSD radix sort of (u64 key, u32 index) pairs, also used by the N2 ingest (k_full.cu) -----------
+size_t radix_pairs_ws_bytes(uint64_t n) {
+  Carver c(nullptr);
+  const uint64_t N = n ? n : 1, nt = ceil_div(N, RTILE);
+  c.take<uint64_t>(N);
+  c.take<uint32_t>(N);
+  c.take<uint32_t>(N);
+  c.take<uint32_t>((uint64_t)RNB * nt);
+  c.take<uint32_t>(ceil_div((uint64_t)RNB * nt, SB) + 1);
+  c.take<uint32_t>(16);
+  return c.off + 256;
+}
+// key[] (n keys < 2^bits, overwritten) sorted stably; *perm_out = the sorted position -> original index array
+// (inside ws); keys end in *key_out (key or the workspace copy)
+cudaError_t launch_radix_pairs(uint64_t* key, uint64_t n, uint32_t bits, void* ws, uint64_t** key_out,
+                               uint32_t** perm_out, cudaStream_t s) {
+  Carver c(ws);
+  const uint64_t N = n ? n : 1, nt = ceil_div(N, RTILE);
+  uint64_t* key1 = c.take<uint64_t>(N);
+  uint32_t* val0 = c.take<uint32_t>(N);
+  uint32_t* val1 = c.take<uint32_t>(N);
+  uint32_t* hist = c.take<uint32_t>((uint64_t)RNB * nt);
+  uint32_t* bsum = c.take<uint32_t>(ceil_div((uint64_t)RNB * nt, SB) + 1);
+  uint32_t* misc = c.take<uint32_t>(16);
+  uint64_t* kin = key; uint64_t* kout = key1;
+  uint32_t* vin = val0; uint32_t* vout = val1;
+  int pass = 0;
+  for (uint32_t sh = 0; sh < (bits ? bits : 1); sh += RBITS, ++pass) {
+    if (n == 0) break;
+    note_launch(), k_radix_up<<<(unsigned)nt, RT, 0, s>>>(kin, n, sh, hist, nt);
+    scan_u32(hist, hist, (uint64_t)RNB * nt, bsum, misc, s);
+    note_launch(), k_radix_down<<<(unsigned)nt, RT, 0, s>>>(kin, vin, n, sh, hist, nt, kout, vout, pass == 0);
+    uint64_t* tk = kin; kin = kout; kout = tk;
+    uint32_t* tv = vin; vin = vout; vout = tv;
+  }
+  *key_out = kin;
+  *perm_out = vin;
+  return cudaGetLastError();
+}
+
 cudaError_t launch_stable(const photon_timing& t, const uint64_t* kbb, photon_stable_params p, void* ws,
                           size_t ws_bytes, int64_t* first_stable, uint64_t* dur, int64_t* switch_at, DevErr* err,
                           int num_sms, cudaStream_t s) {

@@ -8,7 +8,9 @@ import sys
 
 
 def main(rep, fname, n_units, top=40):
-    out = subprocess.run(["ncu", "-i", rep, "--page", "source", "--csv", "--print-source", "cuda,sass"],
+    import os
+    kf = ["-k", "regex:" + os.environ["KFILTER"]] if os.environ.get("KFILTER") else []  # one kernel of a report
+    out = subprocess.run(["ncu", "-i", rep] + kf + ["--page", "source", "--csv", "--print-source", "cuda,sass"],
                          capture_output=True, text=True).stdout
     rows = list(csv.reader(io.StringIO(out)))
     hdr, cur, agg = None, None, {}

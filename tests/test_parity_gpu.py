@@ -523,10 +523,27 @@ def test_pool_reuse(ph, cfg, tmp_path):
 
 
 # ---- N2: full-BBV exact grouping and tagged-stream ingest (L154, L161) ------------------------------------------
-@pytest.mark.parametrize("which", ["c6", "c1", "rand5000", "ragged"])
+@pytest.mark.parametrize("which", ["c6", "c1", "rand5000", "ragged", "perm", pytest.param("c3", marks=pytest.mark.slow)])
 def test_group_full(ph, which):
     if which == "c6":
         tr = tg.make_trace(6)
+    elif which == "c3":  # the bench's N2 workload at full size (1.75M warps, 9% long)
+        tr = tg.make_trace(3)
+    elif which == "perm":  # long warps that are permutations of each other (the histogram verification, ids in
+        rs = np.random.default_rng(5)  # three 4096-id chunks), near-misses differing in one event, short ones
+        kernels = []
+        for k in range(6):
+            base = rs.integers(0, 9000, 40 + 30 * k).tolist()
+            ws = [base]
+            for j in range(12):
+                p = list(rs.permutation(base))
+                if j % 5 == 4:
+                    p[0] = (p[0] + 4096) % 9000  # same length, another id in another chunk
+                ws.append([int(v) for v in p])
+            sh = rs.integers(0, 9000, 9).tolist()
+            ws += [sh, [int(v) for v in rs.permutation(sh)], sh[::-1]]
+            kernels.append(ws)
+        tr = tg.trace_from_warps(kernels, bb_len=rs.integers(1, 9, 9000).tolist())
     elif which == "c1":
         tr = tg.make_trace(1)
     elif which == "rand5000":
