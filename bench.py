@@ -221,6 +221,20 @@ def run_photon(args):
         tr = g.trace()
     ph = Photon(local)
     L = load()
+
+    def graph_ms(fn, n):
+        """fn (a sync-free libphoton call sequence) captured in one CUDA graph; mean ms of n timed replays."""
+        gr, res = ph.capture(fn)
+        for _ in range(max(args.warmup - 1, 1)):
+            gr.replay()
+        torch.cuda.synchronize()
+        t0, t1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        t0.record()
+        for _ in range(n):
+            gr.replay()
+        t1.record()
+        torch.cuda.synchronize()
+        return t0.elapsed_time(t1) / n, res
     d = DeviceTrace.from_host(tr, dev)
     E_total = int(g.warp_counts().sum()) if sh else tr.n_events
     W_total = g.n_warps
@@ -485,35 +499,16 @@ def run_photon(args):
         kbb = ph.photon_bbv_build(da, bbv16=False, insts=False, kbb=True)["kernel_bb_insts"]
         dt = DeviceTiming.from_host(tm, dev)
         o = ph.photon_bb_stable(dt, kbb, 2048)
-        for _ in range(max(args.warmup - 1, 0)):
-            o = ph.photon_bb_stable(dt, kbb, 2048, check=False, out=o)
-        torch.cuda.synchronize()
-        L.photon_profile(ph.ctx, 1)
-        b0, b1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-        b0.record(s)
         n5 = max(args.steps // 4, 3)
-        for _ in range(n5):
-            o = ph.photon_bb_stable(dt, kbb, 2048, check=False, out=o)
-        b1.record(s)
-        torch.cuda.synchronize()
+        ams, o = graph_ms(lambda: ph.photon_bb_stable(dt, kbb, 2048, check=False, out=o), n5)
         ph.check(o["_ws"])
-        L.photon_profile(ph.ctx, 0)
-        ams = b0.elapsed_time(b1) / n5
         R = tm.n_records
         abytes = 18 * R
         # ---- N3 BB-level prediction over the same config's trace with these stability tables ----
         o3 = ph.photon_bb_predict(da, o["first_stable"], o["stable_dur_sum"])
-        for _ in range(max(args.warmup - 1, 0)):
-            o3 = ph.photon_bb_predict(da, o["first_stable"], o["stable_dur_sum"], check=False)
-        torch.cuda.synchronize()
-        p0, p1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-        p0.record(s)
-        for _ in range(n5):
-            o3 = ph.photon_bb_predict(da, o["first_stable"], o["stable_dur_sum"], check=False)
-        p1.record(s)
-        torch.cuda.synchronize()
+        pms, o3 = graph_ms(lambda: ph.photon_bb_predict(da, o["first_stable"], o["stable_dur_sum"], check=False,
+                                                        out=o3), n5)
         ph.check(o3["_ws"])
-        pms = p0.elapsed_time(p1) / n5
         EA, WA = ta.n_events, ta.n_warps
         pbytes = 2 * EA + 8 * (WA + 1) + 12 * WA  # events + offsets + the two per-warp outputs
         line["n3"] = {"metric": "trace events predicted/sec (BB-level per-warp time prediction)",
@@ -539,18 +534,9 @@ def run_photon(args):
         kbb5 = ph.photon_bbv_build(d5, bbv16=False, insts=False, kbb=True)["kernel_bb_insts"]
         dt5 = DeviceTiming.from_host(tm5, dev)
         o5 = ph.photon_bb_stable(dt5, kbb5, 2048)
-        for _ in range(max(args.warmup - 1, 0)):
-            o5 = ph.photon_bb_stable(dt5, kbb5, 2048, check=False, out=o5)
-        torch.cuda.synchronize()
-        h0, h1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         n8 = max(args.steps // 8, 3)
-        h0.record(s)
-        for _ in range(n8):
-            o5 = ph.photon_bb_stable(dt5, kbb5, 2048, check=False, out=o5)
-        h1.record(s)
-        torch.cuda.synchronize()
+        a5ms, o5 = graph_ms(lambda: ph.photon_bb_stable(dt5, kbb5, 2048, check=False, out=o5), n8)
         ph.check(o5["_ws"])
-        a5ms = h0.elapsed_time(h1) / n8
         R5 = tm5.n_records
         line["a5_c5"] = {"metric": "BB timing records tested/sec (stability test + switch)",
                          "value": R5 / (a5ms / 1000), "unit": "records/s", "ms_per_step": a5ms, "records": R5,
@@ -568,18 +554,9 @@ def run_photon(args):
         okd = ty["warp_sampling_ok"]
         dw = DeviceTiming.from_host(tw, dev)
         o = ph.photon_warp_stable(dw, okd, 1024)
-        for _ in range(max(args.warmup - 1, 0)):
-            o = ph.photon_warp_stable(dw, okd, 1024, check=False, out=o)
-        torch.cuda.synchronize()
-        c0, c1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-        c0.record(s)
         n6 = max(args.steps // 4, 3)
-        for _ in range(n6):
-            o = ph.photon_warp_stable(dw, okd, 1024, check=False, out=o)
-        c1.record(s)
-        torch.cuda.synchronize()
+        wms, o = graph_ms(lambda: ph.photon_warp_stable(dw, okd, 1024, check=False, out=o), n6)
         ph.check(o["_ws"])
-        wms = c0.elapsed_time(c1) / n6
         RW = tw.n_records
         wbytes = 16 * RW
         line["n1"] = {"metric": "warp records tested/sec (warp-level stability + warp-sampling switch)",
@@ -599,16 +576,9 @@ def run_photon(args):
         d2 = DeviceTrace.from_host(t2, dev)
         b16 = ph.photon_bbv_build(d2, bbv16=True, insts=False)["warp_bbv16"]
         o = ph.photon_warp_group_full(d2, b16)
-        torch.cuda.synchronize()
-        f0, f1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         n7 = max(args.steps // 4, 3)
-        f0.record(s)
-        for _ in range(n7):
-            o = ph.photon_warp_group_full(d2, b16, check=False, out=o)
-        f1.record(s)
-        torch.cuda.synchronize()
+        fms, o = graph_ms(lambda: ph.photon_warp_group_full(d2, b16, check=False, out=o), n7)
         ph.check(o["_ws"])
-        fms = f0.elapsed_time(f1) / n7
         E2, W2 = t2.n_events, t2.n_warps
         fbytes = 2 * E2 + 12 * W2
         line["n2"] = {"metric": "trace events grouped/sec (full-BBV exact warp types, verified)",

@@ -474,11 +474,15 @@ class Photon:
             self.check(ws, stream)
         return o
 
-    def photon_bb_predict(self, t: DeviceTrace, first_stable, stable_dur_sum, stream=None, check: bool = True) -> dict:
-        """pred_dur_sum [W] (sum of the stable types' S_n over each warp's events) and unpredicted [W]."""
+    def photon_bb_predict(self, t: DeviceTrace, first_stable, stable_dur_sum, stream=None, check: bool = True,
+                          out: Optional[dict] = None) -> dict:
+        """pred_dur_sum [W] (sum of the stable types' S_n over each warp's events) and unpredicted [W]; `out` (a
+        previous result for the same trace) is reused."""
         ct = t.c()
         ws = self.workspace("bpredict", self.L.photon_bb_predict_workspace_bytes(ctypes.byref(ct)))
-        o = {"pred_dur_sum": self.empty(t.n_warps, "int64"), "unpredicted": self.empty(t.n_warps, "int32")}
+        o = out if out is not None else {}
+        o.setdefault("pred_dur_sum", self.empty(t.n_warps, "int64"))
+        o.setdefault("unpredicted", self.empty(t.n_warps, "int32"))
         self._rc(self.L.photon_bb_predict(self.ctx, ctypes.byref(ct), first_stable.data_ptr(),
                                           stable_dur_sum.data_ptr(), ws.data_ptr(), ws.numel(),
                                           o["pred_dur_sum"].data_ptr(), o["unpredicted"].data_ptr(),
