@@ -59,14 +59,44 @@ def _peaks():
         return 6650.0, "fallback (B200_PROFILING.md)"
 
 
+SECTION_TRAFFIC = os.path.join(ROOT, "profiles", "round2", "section_traffic.json")
+
+
+def _section(name):
+    """One section's entry of the committed per-section ncu capture (profiles/section_traffic.py), else None."""
+    try:
+        with open(SECTION_TRAFFIC) as f:
+            j = json.load(f)
+        e = j.get(name)
+        if e is not None:
+            e = dict(e, source=j.get("source"), commit=j.get("commit"))
+        return e
+    except Exception:
+        return None
+
+
 def _traffic(cfg):
-    """Per-launch DRAM bytes of the fused K1 from the committed ncu --set full capture (profiles/), else None."""
+    """Per-launch DRAM bytes of the fused K1 (C5: the per-section capture of this round), else None."""
+    if cfg == 5:
+        e = _section("chain")
+        if e is not None and "k_bbv3<0, 0, 0, 1>" in e["kernels"]:
+            return e["kernels"]["k_bbv3<0, 0, 0, 1>"]["dram_bytes"]
     try:
         with open(os.path.join(ROOT, "profiles", "k1_traffic.json")) as f:
             j = json.load(f)
         return j.get(str(cfg))
     except Exception:
         return None
+
+
+def _sec_traffic(name, algorithmic):
+    """`traffic` fields of a section's roofline: measured DRAM bytes per call (ncu, committed) and the ratio to the
+    algorithmic bytes."""
+    e = _section(name)
+    if e is None:
+        return {"traffic": None}
+    return {"traffic": e["dram_bytes"], "traffic_ratio": e["dram_bytes"] / algorithmic if algorithmic else None,
+            "traffic_source": f"{os.path.relpath(SECTION_TRAFFIC, ROOT)} (commit {e.get('commit')})"}
 
 
 class Clocks:
@@ -343,6 +373,10 @@ def run_photon(args):
                 "peak": hbm_peak, "peak_source": peak_src, "unit": "GB/s", "frac": achieved / hbm_peak,
                 "frac_nominal_8TBps": achieved / 8000.0,
                 "traffic": _traffic(args.config), "algorithmic_bytes_per_launch": k1_bytes,
+                "traffic_ratio": (_traffic(args.config) or 0) / k1_bytes or None,
+                "traffic_source": (f"{os.path.relpath(SECTION_TRAFFIC, ROOT)} (commit "
+                                   f"{(_section('chain') or {}).get('commit')})" if args.config == 5 and
+                                   _section("chain") else "profiles/k1_traffic.json"),
                 "k1_ms": k1_ms, "k1_share_of_step": (pms[0] / args.steps) / ms if ms else None,
                 "chain_algorithmic_GBps": chain_gbps, "chain_frac": chain_gbps / hbm_peak,
                 "chain_frac_nominal_8TBps": chain_gbps / 8000.0}
@@ -516,13 +550,13 @@ def run_photon(args):
                       "workload": f"{CONFIG_DESC.get(args.a5_config)} trace with its A5 tables (n=2048)",
                       "roofline": {"bound": "hbm", "achieved": pbytes / (pms / 1000) / 1e9, "peak": hbm_peak,
                                    "unit": "GB/s", "frac": pbytes / (pms / 1000) / 1e9 / hbm_peak,
-                                   "algorithmic_bytes": pbytes, "traffic": None}}
+                                   "algorithmic_bytes": pbytes, **_sec_traffic("n3", pbytes)}}
         line["a5"] = {"metric": "BB timing records tested/sec (stability test + switch)", "value": R / (ams / 1000),
                       "unit": "records/s", "ms_per_step": ams, "records": R,
                       "workload": f"{CONFIG_DESC.get(args.a5_config)} timing stream (wave model), n=2048, delta=3/100",
                       "roofline": {"bound": "hbm", "achieved": abytes / (ams / 1000) / 1e9, "peak": hbm_peak,
                                    "unit": "GB/s", "frac": abytes / (ams / 1000) / 1e9 / hbm_peak,
-                                   "algorithmic_bytes": abytes, "traffic": None},
+                                   "algorithmic_bytes": abytes, **_sec_traffic("a5", abytes)},
                       "stable_bb_types": int((to_numpy_i64(o["first_stable"]) >= 0).sum())}
 
     # ---- A5 on C5 stress kernels (B = 4096 > 256: the composite-key radix path), a kernel batch ----
@@ -543,7 +577,7 @@ def run_photon(args):
                          "workload": f"C5 stress kernels [0, {k5}) timing stream, n=2048, delta=3/100 (B = 4096)",
                          "roofline": {"bound": "hbm", "achieved": 18 * R5 / (a5ms / 1000) / 1e9, "peak": hbm_peak,
                                       "unit": "GB/s", "frac": 18 * R5 / (a5ms / 1000) / 1e9 / hbm_peak,
-                                      "algorithmic_bytes": 18 * R5, "traffic": None}}
+                                      "algorithmic_bytes": 18 * R5, **_sec_traffic("a5_c5", 18 * R5)}}
         del dt5, o5, d5, kbb5
 
     # ---- N1 (warp-level stability, L262) on the same config's warp streams, gated by A2's dominance ----
@@ -565,7 +599,7 @@ def run_photon(args):
                                   "delta=3/100, gated by warp_sampling_ok",
                       "roofline": {"bound": "hbm", "achieved": wbytes / (wms / 1000) / 1e9, "peak": hbm_peak,
                                    "unit": "GB/s", "frac": wbytes / (wms / 1000) / 1e9 / hbm_peak,
-                                   "algorithmic_bytes": wbytes, "traffic": None},
+                                   "algorithmic_bytes": wbytes, **_sec_traffic("n1", wbytes)},
                       "switched_kernels": int((to_numpy_i64(o["switch_at"]) >= 0).sum()),
                       "dominant_kernels": int(okd.to(torch.int64).sum().item())}
 
@@ -586,7 +620,7 @@ def run_photon(args):
                       "workload": f"{CONFIG_DESC.get(args.a5_config)} trace",
                       "roofline": {"bound": "hbm", "achieved": fbytes / (fms / 1000) / 1e9, "peak": hbm_peak,
                                    "unit": "GB/s", "frac": fbytes / (fms / 1000) / 1e9 / hbm_peak,
-                                   "algorithmic_bytes": fbytes, "traffic": None},
+                                   "algorithmic_bytes": fbytes, **_sec_traffic("n2", fbytes)},
                       "full_types": int(o["kernel_type_off"][-1].item())}
         # ---- N4 (persisted signature pool, L402): ResNet-152's second half matched against its first half ----
         g4 = tg.Generator(4)

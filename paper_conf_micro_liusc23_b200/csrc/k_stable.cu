@@ -32,6 +32,20 @@ constexpr int RBITS = 8;
 constexpr int RNB = 1 << RBITS;
 constexpr int REC_CHUNK = 4096;
 constexpr int JOB = 2048;       // records per warp job (one-pass multisplit)
+// the grouped copy holds retire (u64) and the duration retire - issue (u32); a duration >= kDurEsc is stored as
+// kDurEsc with the issue time in a side array (written only for those records)
+constexpr uint32_t kDurEsc = 0xFFFFFFFFu;
+__device__ __forceinline__ void put_rec(uint64_t* Y, uint32_t* D, uint64_t* Xw, uint64_t dest, uint64_t x,
+                                        uint64_t y) {
+  Y[dest] = y;
+  const uint64_t d = y - x;
+  if (d < kDurEsc) {
+    D[dest] = (uint32_t)d;
+  } else {
+    D[dest] = kDurEsc;
+    Xw[dest] = x;
+  }
+}
 constexpr int WT = 256;        // window threads
 constexpr int WPT = 8;         // positions per thread
 constexpr int WITEM = WT * WPT;
@@ -276,13 +290,12 @@ __global__ void __launch_bounds__(RT) k_radix_down(const uint64_t* key, const ui
 }
 
 // ---- 3. gather + groups + work items -------------------------------------------------------------------------
-__global__ void k_gather(const uint32_t* idx, uint64_t n, const uint64_t* issue, const uint64_t* retire, uint64_t* X,
-                         uint64_t* Y) {
+__global__ void k_gather(const uint32_t* idx, uint64_t n, const uint64_t* issue, const uint64_t* retire, uint64_t* Y,
+                         uint32_t* D, uint64_t* Xw) {
   uint64_t p = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
   if (p >= n) return;
   uint32_t i = idx[p];
-  X[p] = issue[i];
-  Y[p] = retire[i];
+  put_rec(Y, D, Xw, p, issue[i], retire[i]);
 }
 
 __global__ void k_set_u32(uint32_t* p, uint32_t v) { *p = v; }
@@ -537,7 +550,7 @@ __global__ void __launch_bounds__(HW * 32) k_job_hist(photon_timing t, JobMap jm
 }
 
 __global__ void __launch_bounds__(256, 3) k_job_scatter(photon_timing t, JobMap jm, uint64_t n_jobs, uint32_t* off,
-                                                     uint64_t* X, uint64_t* Y, uint32_t* idx, DevErr* err) {
+                                                     uint64_t* Y, uint32_t* D, uint64_t* Xw, DevErr* err) {
   __shared__ uint32_t run[8][kSmemBins];
   const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
   const uint32_t B = t.n_bb;
@@ -607,12 +620,7 @@ __global__ void __launch_bounds__(256, 3) k_job_scatter(photon_timing t, JobMap 
           if (dd != kNone && lane == lead) base = atomicAdd(&off[hb + (uint64_t)dd * nj + jl], (uint32_t)__popc(peers));
           base = __shfl_sync(0xffffffffu, base, lead);
         }
-        if (dd != kNone) {
-          uint32_t dest = base + __popc(peers & lt);
-          X[dest] = x[u];
-          Y[dest] = y[u];
-          idx[dest] = (uint32_t)i;
-        }
+        if (dd != kNone) put_rec(Y, D, Xw, base + __popc(peers & lt), x[u], y[u]);
         __syncwarp();
       }
 #pragma unroll
@@ -740,8 +748,9 @@ __device__ __forceinline__ Sums shfl_xor_sums(const Sums& s, int m) {
 }
 
 struct WinArgs {
-  const uint64_t* X;
-  const uint64_t* Y;
+  const uint64_t* X;  // issue times (D == nullptr), else the escape side array of the grouped copy
+  const uint64_t* Y;  // retire times
+  const uint32_t* D;  // grouped copy: durations (kDurEsc: issue in X), or nullptr
   const uint64_t* gstart;
   const uint32_t* G;
   const uint64_t* list;   // compact run-major run list (k_runs_*)
@@ -753,6 +762,13 @@ struct WinArgs {
   uint32_t ring;   // fast path: shared positions per run (2n + RUN), 0 = off (n too large for shared memory)
   int64_t lim;     // fast path: shifted times must lie in (-lim, lim) (n * lim^2 < 2^61: int64 sums are exact)
 };
+
+// issue time of position q whose retire time is y
+__device__ __forceinline__ uint64_t win_x(const WinArgs& a, int64_t q, uint64_t y) {
+  if (!a.D) return __ldg(a.X + q);
+  const uint32_t d = __ldg(a.D + q);
+  return d != kDurEsc ? y - d : __ldg(a.X + q);
+}
 
 __device__ __forceinline__ void sums_sub(Sums& a, const Sums& b) {
   a.sx -= b.sx; a.sy -= b.sy; a.sn -= b.sn; a.s2n -= b.s2n; a.sxy -= b.sxy; a.sxx -= b.sxx;
@@ -835,8 +851,15 @@ __device__ bool window_run_fast(const WinArgs& a, uint32_t g, int64_t gs, int64_
     for (int u = 0; u < FU; ++u) {
       const int64_t i = i0 + u * WT + tid, q = base0 + i;
       const bool in = i < span && q >= gs;
-      xv[u] = in ? __ldg(a.X + q) : (uint64_t)c;
       yv[u] = in ? __ldg(a.Y + q) : (uint64_t)c;
+      xv[u] = in ? (a.D ? (uint64_t)__ldg(a.D + q) : __ldg(a.X + q)) : (uint64_t)c;
+    }
+    if (a.D) {
+#pragma unroll
+      for (int u = 0; u < FU; ++u) {  // durations -> issue times (escaped ones from the side array)
+        const int64_t i = i0 + u * WT + tid, q = base0 + i;
+        if (i < span && q >= gs) xv[u] = xv[u] != kDurEsc ? yv[u] - xv[u] : __ldg(a.X + q);
+      }
     }
 #pragma unroll
     for (int u = 0; u < FU; ++u) {
@@ -954,7 +977,7 @@ __global__ void __launch_bounds__(WT, 2) k_window(WinArgs a) {
       const int64_t P0 = gs + 2 * n - 1 + (int64_t)r * RUN;
       const int64_t P1 = P0 + RUN < ge ? P0 + RUN : ge;
       if (a.ring && window_run_fast(a, g, gs, P0, P1, ring, fpart, &fbest)) continue;
-      auto X = [&](int64_t q) -> int64_t { return q >= gs ? (int64_t)__ldg(a.X + q) : 0; };
+      auto X = [&](int64_t q) -> int64_t { return q >= gs ? (int64_t)win_x(a, q, __ldg(a.Y + q)) : 0; };
       auto Yv = [&](int64_t q) -> int64_t { return q >= gs ? (int64_t)__ldg(a.Y + q) : 0; };
       // base: windows ending at P0-1 ([P0-n, P0-1] and [P0-2n, P0-1]); positions < gs contribute 0
       Sums s;
@@ -1059,11 +1082,72 @@ __global__ void __launch_bounds__(WT, 2) k_window(WinArgs a) {
 }
 
 // ---- 5. outputs ----------------------------------------------------------------------------------------------
+// Record index of the latched sorted position q of group (k, b) on the job paths (no index array is kept): the
+// group's job cells give the job holding q (kernels with <= 256 local ids: cells = the jobs' start positions,
+// unmodified; more ids: the scatter's atomics left the jobs' END positions), then one warp counts the job's
+// records of b up to q's rank.
+__device__ uint64_t locate_record(const photon_timing& t, const JobMap& jm, const uint32_t* cells, uint32_t k,
+                                  uint32_t b, uint64_t q, uint64_t gs) {
+  const uint32_t lane = threadIdx.x & 31, B = t.n_bb;
+  const bool sm = jm.nbins(k, B) <= kSmemBins;
+  const uint64_t nj = jm.coff[k + 1] - jm.coff[k];
+  const uint32_t* c = cells + jm.hbase(k, B) + (uint64_t)jm.lid(k, b) * nj;
+  // P = the number of cells <= q (monotone cells: a prefix), by a 32-ary search; sm: the job is P - 1 (its start
+  // is <= q), else P (the first job ending after q)
+  uint64_t lo = 0, hi = nj;  // c[j] <= q for j < lo, c[j] > q for j >= hi
+  while (hi > lo) {
+    const uint64_t step = (hi - lo + 31) / 32, j = lo + lane * step;
+    const unsigned m = __ballot_sync(0xffffffffu, j < hi && c[j] <= q);
+    const uint64_t n = __popc(m), lo0 = lo;
+    if (n == 0) { hi = lo; break; }
+    lo = lo0 + (n - 1) * step + 1;
+    hi = umin64(hi, lo0 + n * step);
+  }
+  const uint64_t jl = sm ? (lo ? lo - 1 : 0) : lo;
+  const uint64_t start = sm ? c[jl] : (jl ? c[jl - 1] : gs);
+  const uint64_t rank = q - start;
+  // the job's records: each lane counts b in its 64-record slice, a warp scan finds the slice, that lane the record
+  const uint64_t a = umin64(t.kernel_rec_off[k], t.n_records), e = umin64(t.kernel_rec_off[k + 1], t.n_records);
+  const uint64_t cs = a + jl * JOB, ce = umin64(cs + JOB, e);
+  constexpr int PER = JOB / 32;
+  const uint64_t l0 = cs + (uint64_t)lane * PER;
+  uint32_t cnt = 0;
+#pragma unroll 16
+  for (int u = 0; u < PER; ++u) {  // independent loads: the compiler keeps many in flight
+    const uint64_t i = l0 + u;
+    uint32_t x = i < ce ? (uint32_t)t.bb[i] : kNone;
+    if (x != kNone && x >= B) x = 0;  // as the scatter placed it (the error is latched)
+    cnt += x == b;
+  }
+  uint32_t incl = cnt;
+  for (int o = 1; o < 32; o <<= 1) {
+    const uint32_t y = __shfl_up_sync(0xffffffffu, incl, o);
+    if ((int)lane >= o) incl += y;
+  }
+  const unsigned hit = __ballot_sync(0xffffffffu, rank < incl && rank >= incl - cnt);
+  const int owner = __ffs(hit) - 1;
+  uint64_t pos = ~0ull;
+  if ((int)lane == owner) {
+    uint32_t r = (uint32_t)(rank - (incl - cnt));
+    for (int u = 0; u < PER; ++u) {
+      const uint64_t i = l0 + u;
+      uint32_t x = t.bb[i];
+      if (x >= B) x = 0;
+      if (x == b) {
+        if (r == 0) { pos = i - a; break; }
+        --r;
+      }
+    }
+  }
+  return __shfl_sync(0xffffffffu, pos, owner < 0 ? 0 : owner);
+}
+
 // group g -> (k, b): mode 0 (radix path) g = b*K + k; 1 (job path, B <= 256) g = k*B + b; 2 (compact) gkb[g]
-__global__ void k_finish(const uint32_t* idx, const uint64_t* X, const uint64_t* Y, const uint32_t* G,
-                         const uint64_t* gfirst, const uint64_t* kro, uint32_t K, uint32_t B, uint32_t n,
-                         int mode, const uint64_t* gkb, int64_t* first_stable, uint64_t* dur) {
-  const uint32_t lane = threadIdx.x & 31, ng = *G;
+__global__ void k_finish(photon_timing t, JobMap jm, const uint32_t* cells, const uint32_t* idx, const uint64_t* Y,
+                         const uint32_t* D, const uint64_t* Xw, const uint32_t* G, const uint64_t* gfirst,
+                         const uint64_t* gstart, uint32_t n, int mode, const uint64_t* gkb, int64_t* first_stable,
+                         uint64_t* dur) {
+  const uint32_t lane = threadIdx.x & 31, ng = *G, K = t.n_kernels, B = t.n_bb;
   const uint32_t nw = (gridDim.x * blockDim.x) >> 5;
   for (uint32_t g = (blockIdx.x * blockDim.x + threadIdx.x) >> 5; g < ng; g += nw) {
     uint64_t q = gfirst[g];
@@ -1073,10 +1157,12 @@ __global__ void k_finish(const uint32_t* idx, const uint64_t* X, const uint64_t*
     else if (mode == 1) { k = g / B; b = g % B; }
     else { k = gkb[g] >> 16; b = gkb[g] & 0xFFFFu; }
     uint64_t s = 0;
-    for (uint64_t i = q + 1 - n + lane; i <= q; i += 32) s += Y[i] - X[i];
+    for (uint64_t i = q + 1 - n + lane; i <= q; i += 32) s += D[i] != kDurEsc ? D[i] : Y[i] - Xw[i];
     for (int o = 16; o > 0; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
+    const uint64_t pos = mode == 0 ? idx[q] - t.kernel_rec_off[k]
+                                   : locate_record(t, jm, cells, (uint32_t)k, (uint32_t)b, q, gstart[g]);
     if (lane == 0) {
-      first_stable[k * B + b] = (int64_t)(idx[q] - kro[k]);
+      first_stable[k * B + b] = (int64_t)pos;
       if (dur) dur[k * B + b] = s;
     }
   }
@@ -1240,7 +1326,7 @@ struct Layout {
                      // 0: LSD radix sort of composite keys (larger B)
   uint64_t* key0; uint64_t* key1;  // radix path only
   uint32_t* val0; uint32_t* val1;  // val0 = original record index of each sorted position (all paths)
-  uint64_t* X; uint64_t* Y;
+  uint64_t* Y; uint32_t* D; uint64_t* Xw;  // the grouped copy: retire, duration (kDurEsc: issue in Xw)
   uint32_t* hist; uint32_t* bsum; uint32_t* misc;  // misc[0] = G, [1] = max runs, [2] = ticket, [4] = scan total
   uint64_t* gstart;  // [gcap+1]
   uint32_t* nruns;   // [gcap]
@@ -1265,10 +1351,11 @@ Layout make_layout(const photon_timing& t, void* base) {
   if (L.gcap == 0) L.gcap = 1;
   L.n_tiles = ceil_div(R, RTILE);
   L.n_jobs = ceil_div(R, JOB) + t.n_kernels;
-  if (L.mode == 0) { L.key0 = c.take<uint64_t>(R); L.key1 = c.take<uint64_t>(R); }
-  L.val0 = c.take<uint32_t>(R);
-  if (L.mode == 0) L.val1 = c.take<uint32_t>(R);
-  L.X = c.take<uint64_t>(R); L.Y = c.take<uint64_t>(R);
+  if (L.mode == 0) {
+    L.key0 = c.take<uint64_t>(R); L.key1 = c.take<uint64_t>(R);
+    L.val0 = c.take<uint32_t>(R); L.val1 = c.take<uint32_t>(R);
+  }
+  L.Y = c.take<uint64_t>(R); L.D = c.take<uint32_t>(R); L.Xw = c.take<uint64_t>(R);
   // histogram cells: B * jobs; compact: sum_k B_k * jobs_k <= 2R + ... whenever no kernel has more than 2048
   // distinct BB ids (ECAPACITY otherwise)
   L.hn = L.mode == 1 ? (uint64_t)t.n_bb * L.n_jobs : (L.mode == 2 ? 2 * R + 65536 : (uint64_t)RNB * L.n_tiles);
@@ -1351,6 +1438,7 @@ cudaError_t launch_stable(const photon_timing& t, const uint64_t* kbb, photon_st
   note_launch(), k_rec_chunks<<<1, 1024, 0, s>>>(t.kernel_rec_off, K, R, chunk, L.coff, err);
   if (R > 0) {
     uint32_t* idx;
+    JobMap jmf{};  // the job map (job paths), for k_finish
     if (L.mode != 0) {
       // 1-2. per-job histograms of (kernel-local) BB ids -> kernel-major scan -> stable scatter of (issue, retire,
       // index) into group order
@@ -1381,8 +1469,9 @@ cudaError_t launch_stable(const photon_timing& t, const uint64_t* kbb, photon_st
       // group starts first: kernels with > 256 local ids use the scanned cells as running offsets in the scatter
       note_launch(), k_job_gstart<<<(unsigned)umin64(ceil_div(L.gcap + 1, 256), (uint64_t)num_sms * 8), 256, 0, s>>>(
           L.hist, jm, L.goff, L.gkb, K, B, R, (uint64_t)B * L.n_jobs, L.gstart, L.misc + 0);
-      note_launch(), k_job_scatter<<<gj, 256, 0, s>>>(t, jm, L.n_jobs, L.hist, L.X, L.Y, L.val0, err);
-      idx = L.val0;
+      note_launch(), k_job_scatter<<<gj, 256, 0, s>>>(t, jm, L.n_jobs, L.hist, L.Y, L.D, L.Xw, err);
+      idx = nullptr;
+      jmf = jm;
     } else {
       uint64_t jobs_ub = ceil_div(R, REC_CHUNK) + K;
       unsigned grid = (unsigned)umin64(jobs_ub, (uint64_t)num_sms * 8);
@@ -1402,7 +1491,7 @@ cudaError_t launch_stable(const photon_timing& t, const uint64_t* kbb, photon_st
         uint32_t* tv = vin; vin = vout; vout = tv;
       }
       unsigned gR = (unsigned)ceil_div(R + 1, 256);
-      note_launch(), k_gather<<<gR, 256, 0, s>>>(vin, R, t.issue, t.retire, L.X, L.Y);
+      note_launch(), k_gather<<<gR, 256, 0, s>>>(vin, R, t.issue, t.retire, L.Y, L.D, L.Xw);
       note_launch(), k_fill_gstart<<<gR, 256, 0, s>>>(kin, R, L.gcap, L.gstart);
       note_launch(), k_set_u32<<<1, 1, 0, s>>>(L.misc + 0, (uint32_t)L.gcap);
       idx = vin;
@@ -1411,13 +1500,14 @@ cudaError_t launch_stable(const photon_timing& t, const uint64_t* kbb, photon_st
     note_launch(), k_work_count<<<(unsigned)umin64(ceil_div(L.gcap, 256), (uint64_t)num_sms * 4), 256, 0, s>>>(
         L.gstart, L.misc + 0, 2 * p.window_n, L.nruns, L.gfirst, L.misc + 1);
     WinArgs wa{};
-    wa.X = L.X; wa.Y = L.Y; wa.gstart = L.gstart; wa.G = L.misc + 0;
+    wa.X = L.Xw; wa.Y = L.Y; wa.D = L.D; wa.gstart = L.gstart; wa.G = L.misc + 0;
     wa.n = p.window_n; wa.dnum = p.delta_num; wa.dden = p.delta_den; wa.gfirst = L.gfirst;
     build_runlist(L.rl, L.misc + 0, L.nruns, L.misc, L.gcap, num_sms, wa, s);
     window_launch(wa, num_sms, s);
     // 5. outputs
     note_launch(), k_finish<<<(unsigned)umin64(ceil_div(L.gcap * 32, 256), (uint64_t)num_sms * 8), 256, 0, s>>>(
-        idx, L.X, L.Y, L.misc + 0, L.gfirst, t.kernel_rec_off, K, B, p.window_n, L.mode, L.gkb, first_stable, dur);
+        t, jmf, L.hist, idx, L.Y, L.D, L.Xw, L.misc + 0, L.gfirst, L.gstart, p.window_n, L.mode, L.gkb, first_stable,
+        dur);
     unsigned gk = (unsigned)umin64(K, (uint64_t)num_sms * 8);
     note_launch(), k_switch<<<gk ? gk : 1, 256, 0, s>>>(first_stable, kbb, K, B, p.rate_num, p.rate_den, switch_at);
   } else {
@@ -1457,7 +1547,7 @@ cudaError_t launch_warp_stable(const photon_timing& t, const uint8_t* ok, uint32
   note_launch(), k_warp_runs<<<(unsigned)ceil_div(K, 256), 256, 0, s>>>(t.kernel_rec_off, K, t.n_records, ok, 2 * n,
                                                                        nruns, gfirst, misc);
   WinArgs wa{};
-  wa.X = t.issue; wa.Y = t.retire; wa.gstart = t.kernel_rec_off; wa.G = misc + 0;
+  wa.X = t.issue; wa.Y = t.retire; wa.D = nullptr; wa.gstart = t.kernel_rec_off; wa.G = misc + 0;
   wa.n = n; wa.dnum = dnum; wa.dden = dden; wa.gfirst = gfirst;
   build_runlist(rl, misc + 0, nruns, misc, K, num_sms, wa, s);
   window_launch(wa, num_sms, s);
