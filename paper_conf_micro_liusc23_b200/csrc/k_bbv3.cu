@@ -12,8 +12,9 @@
 //    warps are cut into blocks of 32 consecutive warps; worker g takes the blocks whose first event lies in its
 //    1/G share of the trace (event-balanced contiguous ranges, found by a 32-ary search), so a worker sees few
 //    kernels and few warp types.  Lane u owns warp u of the current block.
-//  * A block's events are staged in chunks of <= 32*Q 16-byte words with cp.async.bulk (TMA copy engine) into one
-//    of two per-worker buffers; chunk i+1 is in flight while chunk i is processed.
+//  * A block's events are staged in chunks of <= 32*Q 16-byte words with cp.async.bulk (TMA copy engine) into a
+//    per-worker buffer (K1_NBUF = 1, the default: chunk i+1 is issued right after chunk i's event loop and lands
+//    during its collect / finalisation; K1_NBUF = 2 double-buffers at the cost of occupancy).
 //  * A chunk is cut into 32 equal lane ranges (Q' words, Q' odd so the quarter-warp 16-byte loads hit distinct
 //    bank groups).  Lane t walks its range; the piece of each analysed warp it meets is accumulated with
 //    red.shared.add into a column private to the lane: the first piece into the lane's slot-0 column, a warp
@@ -24,10 +25,9 @@
 //  * After the loop each lane sums its warp's pieces (owner column, then slot 0 of every later lane it spans) into
 //    16 key registers, carried across the chunks of a block; the worker's cells are cleared with 16-byte stores.
 //  * Fused: at the block's end the keys are hashed, grouped with __match_any_sync plus an exact 17-word check, and
-//    each distinct (kernel, key) is looked up in the worker's 8-slot cache of open type entries (full keys in
-//    shared memory): a hit adds the count, a miss evicts an entry (its count and first warp written) and opens a
-//    new one in the worker's block of the global entry pool.  Each warp records its entry index (u32).  The
-//    entries are inserted into the global type table afterwards (k_types.cu).
+//    each distinct (kernel, key) of the block becomes one 80-byte entry (key, first warp, kernel, count) taken
+//    from the worker's run of the global entry pool (one atomic per ENT_BLK entries).  Each warp records its
+//    entry index (u32).  The entries are inserted into the global type table afterwards (k_types.cu).
 #include "internal.h"
 
 namespace photon {
