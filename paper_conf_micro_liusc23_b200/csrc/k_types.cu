@@ -118,8 +118,9 @@ __device__ void emit_rows(const HashTable& ht, uint32_t k, const uint32_t* sorte
   }
 }
 
-// Kernels with T_k <= 32 (almost all): one warp each, bitonic network over lanes with shuffles.  Larger kernels
-// are queued: 32 < T_k <= SORT_SMEM_MAX at the front of cw.big (k_sort_mid), larger ones at the back (k_sort_large).
+// Kernels with T_k <= 32 (almost all): one warp each, bitonic network over the first P = next_pow2(T_k) lanes with
+// shuffles; 32 < T_k <= 128: the same warp, a warp-private shared-memory bitonic sort.  Larger kernels are queued:
+// T_k <= SORT_SMEM_MAX at the front of cw.big (k_sort_mid, one CTA each), larger ones at the back (k_sort_large).
 __global__ void __launch_bounds__(256) k_sort_warp(HashTable ht, uint32_t K, const uint64_t* kto,
                                                    const uint32_t* list, const uint64_t* kwo,
                                                    const uint64_t* kernel_warps, photon_types out, uint32_t* canon,
@@ -199,7 +200,9 @@ __global__ void __launch_bounds__(256) k_sort_warp(HashTable ht, uint32_t K, con
     mc = ht.count[mine];
     mk = *(const uint4*)(ht.key + (uint64_t)mine * 16);
   }
-  for (uint32_t size = 2; size <= 32; size <<= 1) {
+  uint32_t P = 1;  // the network over the first P >= n lanes only (xor partners stay inside aligned P-blocks)
+  while (P < n) P <<= 1;
+  for (uint32_t size = 2; size <= P; size <<= 1) {
     for (uint32_t stride = size >> 1; stride > 0; stride >>= 1) {
       const uint32_t other = __shfl_xor_sync(0xffffffffu, mine, stride);
       const uint32_t oc = __shfl_xor_sync(0xffffffffu, mc, stride);
