@@ -260,6 +260,7 @@ template <bool WIDE, bool GTBL, bool MARK, bool FUSED>
 __global__ void __launch_bounds__(WPC * 32, 1) k_bbv3(Args3 a) {
   using M = Mode<WIDE>;
   constexpr uint32_t Q = M::Q, CW = 32 * Q, CE = CW * 8;
+  static_assert((uint64_t)CE * kMaxLen < (1ull << 32), "a chunk adds < 2^32 to a warp's bins (u32 delta of I)");
   constexpr int ROWS = M::ROWS;
   extern __shared__ __align__(128) uint8_t smem[];
   const uint32_t lane = threadIdx.x & 31, wid = threadIdx.x >> 5;

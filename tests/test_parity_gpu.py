@@ -91,17 +91,14 @@ def test_random_small(ph, seed):
 
 
 @pytest.mark.parametrize("cfg", [1, 6])
-def test_k1_round1_kernel_matches(ph, cfg, monkeypatch):
-    # PHOTON_K1_V1 routes K1 to the round-1 kernel (k_bbv.cu, the path for B > 4096); both kernels must give the
-    # oracle's BBVs and types on the same inputs (C1: items of two chunks; C6: every template, tiny warps)
+def test_k1_fused_and_unfused_grouping_match(ph, cfg):
+    # the fused K1 (BBV + de-dup in one pass) and the unfused path (materialised BBVs -> k_group3_from_bbv) must
+    # both give the oracle's types (C1: blocks of several chunks; C6: every template, tiny warps)
     tr = tg.make_trace(cfg)
-    ref = None
-    for v1 in (False, True):
-        if v1:
-            monkeypatch.setenv("PHOTON_K1_V1", "1")
-        d, o, p16 = check_bbv(ph, tr)
-        ref = ref if ref is not None else oracle.group(tr, p16)
-        check_types(ph, tr, ph.photon_warp_group(d), ref)
+    d, o, p16 = check_bbv(ph, tr)
+    ref = oracle.group(tr, p16)
+    check_types(ph, tr, ph.photon_warp_group(d), ref)
+    check_types(ph, tr, ph.photon_warp_group(d, o["warp_bbv16"]), ref)
 
 
 def test_empty_warps_kernels_and_ragged(ph):

@@ -203,9 +203,9 @@ def test_k1_long_warps(ph, n_bb, max_len):
 
 
 @pytest.mark.parametrize("n_bb", [300, 5000])
-def test_k1_long_warps_round1_kernel(ph, n_bb, monkeypatch):
-    # the same traces through the round-1 kernel k_bbv (forced), the path for B > 4096 today
-    monkeypatch.setenv("PHOTON_K1_V1", "1")
+def test_k1_long_warps_unfused_grouping(ph, n_bb):
+    # the same kind of traces through the unfused grouping (materialised BBVs -> k_group3_from_bbv); B = 5000 >
+    # 4096 reads the BB table through L1 instead of shared memory
     rs = np.random.default_rng(n_bb)
     tr = _trace_from_lengths(n_bb + 1, _long_kernels(rs), n_bb, 64)
     d = _dev(ph, tr)
@@ -213,7 +213,7 @@ def test_k1_long_warps_round1_kernel(ph, n_bb, monkeypatch):
     o = ph.photon_bbv_build(d, bbv16=True, insts=True)
     assert np.array_equal(_np(o["warp_bbv16"], np.uint32).reshape(-1, 16), p16)
     assert np.array_equal(_np(o["warp_insts"], np.uint64), ins)
-    _check_types(ph.photon_warp_group(d), oracle.group(tr, p16))
+    _check_types(ph.photon_warp_group(d, o["warp_bbv16"]), oracle.group(tr, p16))
 
 
 # ---- A3 ------------------------------------------------------------------------------------------------------------
