@@ -470,14 +470,14 @@ int photon_kernel_match(photon_ctx* ctx, uint32_t K, const photon_types* types, 
   CK(cudaMemsetAsync(m.err, 0, sizeof(DevErr), s), "memset");
   {
     ProfScope ps(ctx, PHOTON_PROF_SIG, s);
-    CK(launch_sig_build(K, types->kernel_type_off, types->type_key, types->type_count, 0, K, m.sig, m.mass, m.err,
-                        s),
+    CK(launch_sig_prof(K, types->kernel_type_off, types->type_key, types->type_count, m.sig, m.mass, m.mw, m.err,
+                       s),
        "sig");
   }
   {
     ProfScope ps(ctx, PHOTON_PROF_SCAN, s);
     CK(launch_match_scan(K, types->kernel_type_off, m.sig, m.mass, warps_total, params, 0, K, m.mw, m.pairs,
-                         m.mw.pair_cap, m.n_pairs, m.err, ctx->num_sms, s),
+                         m.mw.pair_cap, m.n_pairs, m.err, ctx->num_sms, s, /*prof_ready=*/true),
        "scan");
   }
   {

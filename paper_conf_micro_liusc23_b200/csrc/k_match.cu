@@ -94,6 +94,55 @@ __global__ void k_prof(uint32_t K, const uint64_t* __restrict__ kto, const uint6
   }
 }
 
+// A3 fused with the filter profiles (the single-GPU photon_kernel_match: every kernel, one pass over the type
+// rows): g = count x key, N = sum g with the 2^50 bound (as k_sig), then P_k[j], its u8 quantisation, 1/N and the
+// normalised copy sigf = g / N (as k_prof).  Lane l covers bin l & 15 of every other row.
+__global__ void k_sig_prof(uint32_t K, const uint64_t* __restrict__ kto, const uint32_t* __restrict__ key,
+                           const uint64_t* __restrict__ count, uint64_t* __restrict__ sig, uint64_t* __restrict__ mass,
+                           float* __restrict__ prof, double* __restrict__ invn, uint32_t* __restrict__ prof8,
+                           float* __restrict__ sigf, DevErr* err) {
+  const uint32_t k = (blockIdx.x * blockDim.x + threadIdx.x) >> 5, lane = threadIdx.x & 31;
+  if (k >= K) return;
+  const uint64_t r0 = kto[k], r1 = kto[k + 1];
+  uint64_t acc = 0;
+  bool over = false;
+  for (uint64_t r = r0 + (lane >> 4); r < r1; r += 2) {
+    const uint64_t i = r * 16 + (lane & 15);
+    const uint64_t c = count[r];
+    over |= c >= (1ull << 32);
+    const uint64_t g = c * (uint64_t)key[i];
+    sig[i] = g;
+    over |= g >= kMassLimit;
+    acc += g;
+    over |= acc >= kMassLimit;
+  }
+  uint64_t bin = acc + __shfl_xor_sync(0xffffffffu, acc, 16);  // this lane's bin over all rows
+  uint64_t N = bin;
+  for (int o = 8; o > 0; o >>= 1) N += __shfl_xor_sync(0xffffffffu, N, o);  // 16 bins (lanes 0-15 == 16-31)
+  over = __any_sync(0xffffffffu, over) || N >= kMassLimit;
+  if (lane == 0) {
+    if (over) latch(err, PHOTON_ERANGE, (int64_t)k);
+    mass[k] = N;
+  }
+  const double inv = N ? 1.0 / (double)N : 0.0;
+  if (sigf)
+    for (uint64_t r = r0 + (lane >> 4); r < r1; r += 2) {
+      const uint64_t i = r * 16 + (lane & 15);
+      sigf[i] = (float)((double)sig[i] * inv);  // this lane's own store, read back
+    }
+  const double P = N ? (double)bin / (double)N : 0.0;
+  uint32_t q = (uint32_t)rint(P * 255.0);
+  q = q > 255u ? 255u : q;
+  uint32_t w = q << (8 * (lane & 3));
+  w |= __shfl_xor_sync(0xffffffffu, w, 1);
+  w |= __shfl_xor_sync(0xffffffffu, w, 2);
+  if (lane < 16) {
+    prof[(uint64_t)k * 16 + lane] = (float)P;
+    if ((lane & 3) == 0) prof8[(uint64_t)k * 4 + (lane >> 2)] = w;
+    if (lane == 0) invn[k] = inv;
+  }
+}
+
 // ---- pair filter: 64 x 64 tiles of (k, r < k) --------------------------------------------------------------
 constexpr int FT = 64;
 struct ScanArgs {
@@ -674,15 +723,24 @@ cudaError_t launch_sig_build(uint32_t K, const uint64_t* kto, const uint32_t* ty
   return cudaGetLastError();
 }
 
+cudaError_t launch_sig_prof(uint32_t K, const uint64_t* kto, const uint32_t* type_key, const uint64_t* type_count,
+                            uint64_t* sig, uint64_t* mass, const MatchWs& mw, DevErr* err, cudaStream_t s) {
+  if (K == 0) return cudaSuccess;
+  note_launch(), k_sig_prof<<<(unsigned)ceil_div((uint64_t)K * 32, 256), 256, 0, s>>>(
+      K, kto, type_key, type_count, sig, mass, mw.prof, mw.invn, mw.prof8, mw.sigf, err);
+  return cudaGetLastError();
+}
+
 cudaError_t launch_match_scan(uint32_t K, const uint64_t* kto, const uint64_t* sig, const uint64_t* mass,
                               const uint64_t* wt, photon_match_params p, uint32_t k_lo, uint32_t k_hi,
                               const MatchWs& mw, uint64_t* pairs, uint64_t pair_cap, uint64_t* n_pairs, DevErr* err,
-                              int num_sms, cudaStream_t s) {
+                              int num_sms, cudaStream_t s, bool prof_ready) {
   cudaMemsetAsync(n_pairs, 0, 8, s);
   cudaMemsetAsync(mw.n_maybe, 0, 8, s);
   if (K == 0 || k_hi <= k_lo) return cudaGetLastError();
-  note_launch(), k_prof<<<(unsigned)ceil_div((uint64_t)K * 32, 256), 256, 0, s>>>(K, kto, sig, mass, mw.prof, mw.invn,
-                                                                                mw.prof8, mw.sigf);
+  if (!prof_ready)
+    note_launch(), k_prof<<<(unsigned)ceil_div((uint64_t)K * 32, 256), 256, 0, s>>>(K, kto, sig, mass, mw.prof,
+                                                                                  mw.invn, mw.prof8, mw.sigf);
   ScanArgs a{};
   a.K = K; a.k_lo = k_lo; a.k_hi = k_hi; a.kto = kto; a.sig = sig; a.mass = mass; a.wt = wt; a.prof = mw.prof; a.invn = mw.invn; a.prof8 = mw.prof8; a.sigf = mw.sigf;
   a.p = p;
