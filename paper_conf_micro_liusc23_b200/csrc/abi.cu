@@ -208,6 +208,7 @@ MatchLayout match_layout(uint32_t K, uint64_t T, uint64_t pair_cap, void* base) 
   m.mw.cand_off = c.take<uint64_t>(K + 1);
   m.mw.cand_cur = c.take<uint32_t>(K + 1);
   m.mw.cand = c.take<uint32_t>(pair_cap);
+  m.mw.close_cnt = c.take<uint32_t>(K + 1);
   m.mw.state = c.take<uint8_t>(K + 1);
   m.mw.ulist = c.take<uint32_t>(2ull * K + 2);
   m.mw.flag = c.take<uint32_t>(4);
@@ -477,13 +478,13 @@ int photon_kernel_match(photon_ctx* ctx, uint32_t K, const photon_types* types, 
   {
     ProfScope ps(ctx, PHOTON_PROF_SCAN, s);
     CK(launch_match_scan(K, types->kernel_type_off, m.sig, m.mass, warps_total, params, 0, K, m.mw, m.pairs,
-                         m.mw.pair_cap, m.n_pairs, m.err, ctx->num_sms, s, /*prof_ready=*/true),
+                         m.mw.pair_cap, m.n_pairs, m.err, ctx->num_sms, s, /*prof_ready=*/true, /*fused=*/true),
        "scan");
   }
   {
     ProfScope ps(ctx, PHOTON_PROF_RESOLVE, s);
     CK(launch_match_resolve(K, types->kernel_type_off, m.sig, m.mass, warps_total, params, m.pairs, m.mw.pair_cap,
-                            m.n_pairs, m.mw, match, match_dist, m.err, ctx->num_sms, s),
+                            m.n_pairs, m.mw, match, match_dist, m.err, ctx->num_sms, s, /*fused=*/true),
        "resolve");
   }
   return PHOTON_OK;

@@ -97,6 +97,7 @@ struct MatchWs {
   uint64_t* cand_off;  // [K+1]
   uint32_t* cand_cur;  // [K]
   uint32_t* cand;      // [pair_cap] r per (k, r), grouped by k
+  uint32_t* close_cnt; // [K] fused path: close candidates in k's segment of cand (starting at cand_off[k])
   uint8_t* state;      // [K] 0 undecided, 1 representative, 2 matched
   uint32_t* ulist;     // [2K] undecided-kernel lists (resolution rounds)
   uint32_t* flag;      // [4]
@@ -108,14 +109,14 @@ cudaError_t launch_sig_build(uint32_t K, const uint64_t* kto, const uint32_t* ty
 cudaError_t launch_match_scan(uint32_t K, const uint64_t* kto, const uint64_t* sig, const uint64_t* mass,
                               const uint64_t* wt, photon_match_params p, uint32_t k_lo, uint32_t k_hi,
                               const MatchWs& mw, uint64_t* pairs, uint64_t pair_cap, uint64_t* n_pairs, DevErr* err,
-                              int num_sms, cudaStream_t s, bool prof_ready = false);
+                              int num_sms, cudaStream_t s, bool prof_ready = false, bool fused = false);
 // the single-GPU fused A3: signatures + the filter profiles in one pass (launch_match_scan(prof_ready = true))
 cudaError_t launch_sig_prof(uint32_t K, const uint64_t* kto, const uint32_t* type_key, const uint64_t* type_count,
                             uint64_t* sig, uint64_t* mass, const MatchWs& mw, DevErr* err, cudaStream_t s);
 cudaError_t launch_match_resolve(uint32_t K, const uint64_t* kto, const uint64_t* sig, const uint64_t* mass,
                                  const uint64_t* wt, photon_match_params p, const uint64_t* pairs, uint64_t n_pairs,
                                  const uint64_t* n_pairs_dev, const MatchWs& mw, int64_t* match, double* match_dist,
-                                 DevErr* err, int num_sms, cudaStream_t s);
+                                 DevErr* err, int num_sms, cudaStream_t s, bool fused = false);
 
 // ---- A5 (k_stable.cu) -------------------------------------------------------------------------------------
 size_t stable_ws_bytes(const photon_timing& t);

@@ -162,6 +162,10 @@ struct ScanArgs {
   uint64_t* n_maybe;
   uint64_t cap;
   DevErr* err;
+  // fused path: close pairs go straight into k's segment [cbeg[k], cbeg[k] + ccnt[k]) of cand (else: pairs list)
+  uint32_t* cand;
+  const uint64_t* cbeg;
+  uint32_t* ccnt;
 };
 
 // Jobs: one k-block (FT kernels) against a run of up to FR r-blocks (rb <= kb).  S(kb) = jobs before k-block kb
@@ -423,8 +427,13 @@ __global__ void __launch_bounds__(256) k_pair_exact(ScanArgs a, uint64_t* pairs,
     }
     if (act && close && (threadIdx.x & (XG - 1)) == 0) {
       const unsigned long long pos = atomicAdd((unsigned long long*)n_pairs, 1ull);
-      if (pos < pair_cap) pairs[pos] = pr;
-      else latch(a.err, PHOTON_ECAPACITY, (int64_t)pos);
+      if (a.cand) {  // fused path: the close r into k's segment of the k-bucketed survivors
+        a.cand[a.cbeg[k] + atomicAdd(&a.ccnt[k], 1u)] = r;
+      } else if (pos < pair_cap) {
+        pairs[pos] = pr;
+      } else {
+        latch(a.err, PHOTON_ECAPACITY, (int64_t)pos);
+      }
     }
   }
 }
@@ -437,12 +446,12 @@ __device__ __forceinline__ uint64_t pair_count(uint64_t n_host, const uint64_t* 
 __global__ void k_cand_count(const uint64_t* pairs, uint64_t n_host, const uint64_t* n_dev, uint32_t K, uint32_t* cnt,
                              DevErr* err) {
   uint64_t n = pair_count(n_host, n_dev);
-  uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
-  if (i >= n) return;
-  if (pairs[i] == PHOTON_PAIR_PAD) return;  // padding of a fixed-capacity exchange
-  uint32_t k = (uint32_t)(pairs[i] >> 32), r = (uint32_t)pairs[i];
-  if (k >= K || r >= k) { latch(err, PHOTON_EINVAL, (int64_t)i); return; }
-  atomicAdd(&cnt[k], 1u);
+  for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x) {
+    if (pairs[i] == PHOTON_PAIR_PAD) continue;  // padding of a fixed-capacity exchange
+    uint32_t k = (uint32_t)(pairs[i] >> 32), r = (uint32_t)pairs[i];
+    if (k >= K || r >= k) { latch(err, PHOTON_EINVAL, (int64_t)i); continue; }
+    atomicAdd(&cnt[k], 1u);
+  }
 }
 
 __global__ void __launch_bounds__(1024) k_cand_scan(const uint32_t* cnt, uint32_t K, uint64_t* off, uint32_t* cur) {
@@ -490,12 +499,25 @@ __global__ void k_cand_scatter(const uint64_t* pairs, uint64_t n_host, const uin
   cand[off[k] + atomicAdd(&cur[k], 1u)] = r;
 }
 
+// the filter survivors bucketed by k (stable order inside a bucket is immaterial): the exact check then visits
+// every candidate of one k back to back, so g_k stays in L1 for the run
+__global__ void k_pair_bucket(const uint64_t* pairs, uint64_t n_host, const uint64_t* n_dev, uint32_t K,
+                              const uint64_t* off, uint32_t* cur, uint64_t* out) {
+  uint64_t n = pair_count(n_host, n_dev);
+  for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x) {
+    const uint64_t pr = pairs[i];
+    const uint32_t k = (uint32_t)(pr >> 32);
+    if (k < K) out[off[k] + atomicAdd(&cur[k], 1u)] = pr;
+  }
+}
+
 // Fixed point of the launch-order rule: state 1 = representative, 2 = matched.  k decides once all its candidate
 // predecessors have decided (or one of them is a representative).  One CTA; monotone state (races benign).
 // Each kernel keeps a cursor into its candidate list: entries before it are decided non-representatives, so every
 // candidate is examined O(1) times plus once per round it blocks.  State lives in shared memory when K fits.
 template <bool SMEM>
-__global__ void __launch_bounds__(1024) k_resolve_states(uint32_t K, const uint64_t* off, const uint32_t* cand,
+__global__ void __launch_bounds__(1024) k_resolve_states(uint32_t K, const uint64_t* beg, const uint32_t* cnt,
+                                                         const uint32_t* cand,
                                                          uint8_t* state, uint32_t* cursor, uint32_t* ulist,
                                                          uint32_t* flag, uint32_t pool_all) {
   extern __shared__ uint8_t sstate[];
@@ -506,7 +528,7 @@ __global__ void __launch_bounds__(1024) k_resolve_states(uint32_t K, const uint6
   }
   __syncthreads();
   if (pool_all) {
-    for (uint32_t k = threadIdx.x; k < K; k += blockDim.x) state[k] = off[k + 1] > off[k] ? 2 : 1;
+    for (uint32_t k = threadIdx.x; k < K; k += blockDim.x) state[k] = cnt[k] > 0 ? 2 : 1;
     if (threadIdx.x == 0) flag[0] = 1;
     return;
   }
@@ -522,7 +544,7 @@ __global__ void __launch_bounds__(1024) k_resolve_states(uint32_t K, const uint6
     __syncthreads();
     for (uint32_t q = threadIdx.x; q < n; q += blockDim.x) {
       const uint32_t k = cur ? cur[q] : q;
-      const uint64_t o0 = off[k], o1 = off[k + 1];
+      const uint64_t o0 = beg[k], o1 = o0 + cnt[k];
       uint64_t first_undec = o1;
       uint8_t res = 1;  // representative unless a candidate is one
       // batches of 8 independent candidate loads (memory-level parallelism), then their states
@@ -559,7 +581,8 @@ __global__ void __launch_bounds__(1024) k_resolve_states(uint32_t K, const uint6
 // The same fixed point over the whole GPU: a cooperative grid, one grid-wide barrier per round (rounds are few: the
 // longest chain of kernels blocked on undecided predecessors).  Each round visits the undecided list of the previous
 // round; a blocked kernel keeps its cursor.  Stale state reads only postpone a decision (states are monotone).
-__global__ void __launch_bounds__(256) k_resolve_coop(uint32_t K, const uint64_t* __restrict__ off,
+__global__ void __launch_bounds__(256) k_resolve_coop(uint32_t K, const uint64_t* __restrict__ beg,
+                                                      const uint32_t* __restrict__ cnt,
                                                       const uint32_t* __restrict__ cand, uint8_t* state,
                                                       uint32_t* cursor, uint32_t* ulist, uint32_t* rcnt,
                                                       uint32_t* flag) {
@@ -583,7 +606,7 @@ __global__ void __launch_bounds__(256) k_resolve_coop(uint32_t K, const uint64_t
     // one warp per undecided kernel: 128 candidates (4 x 32 independent loads) per step, ballots decide
     for (uint64_t q = gw; q < n; q += nw) {
       const uint32_t k = cur ? cur[q] : (uint32_t)q;
-      const uint64_t o0 = off[k], o1 = off[k + 1];
+      const uint64_t o0 = beg[k], o1 = o0 + cnt[k];
       uint64_t first_undec = o1;
       bool rep_found = false;
       for (uint64_t i0 = o0 + cursor[k]; i0 < o1; i0 += 128) {
@@ -626,7 +649,8 @@ __global__ void __launch_bounds__(256) k_resolve_coop(uint32_t K, const uint64_t
 }
 
 // match[k] = argmin over eligible candidates of (|W_k - W_r|, r); match_dist exact -> fp64 (one warp per kernel)
-__global__ void k_resolve_match(uint32_t K, const uint64_t* off, const uint32_t* cand, const uint8_t* state,
+__global__ void k_resolve_match(uint32_t K, const uint64_t* beg, const uint32_t* cnt, const uint32_t* cand,
+                                const uint8_t* state,
                                 uint32_t pool_all, const uint64_t* wt, const uint64_t* kto, const uint64_t* sig,
                                 const uint64_t* mass, int64_t* match, double* dist) {
   uint32_t warp = (blockIdx.x * blockDim.x + threadIdx.x) >> 5, lane = threadIdx.x & 31;
@@ -635,7 +659,7 @@ __global__ void k_resolve_match(uint32_t K, const uint64_t* off, const uint32_t*
   uint64_t best_dw = ~0ull;
   uint32_t best_r = UINT32_MAX;
   if (state[k] == 2) {
-    for (uint64_t i = off[k] + lane; i < off[k + 1]; i += 32) {
+    for (uint64_t i = beg[k] + lane; i < beg[k] + cnt[k]; i += 32) {
       uint32_t r = cand[i];
       if (!pool_all && state[r] != 1) continue;
       uint64_t dw = wt[k] > wt[r] ? wt[k] - wt[r] : wt[r] - wt[k];
@@ -734,7 +758,7 @@ cudaError_t launch_sig_prof(uint32_t K, const uint64_t* kto, const uint32_t* typ
 cudaError_t launch_match_scan(uint32_t K, const uint64_t* kto, const uint64_t* sig, const uint64_t* mass,
                               const uint64_t* wt, photon_match_params p, uint32_t k_lo, uint32_t k_hi,
                               const MatchWs& mw, uint64_t* pairs, uint64_t pair_cap, uint64_t* n_pairs, DevErr* err,
-                              int num_sms, cudaStream_t s, bool prof_ready) {
+                              int num_sms, cudaStream_t s, bool prof_ready, bool fused) {
   cudaMemsetAsync(n_pairs, 0, 8, s);
   cudaMemsetAsync(mw.n_maybe, 0, 8, s);
   if (K == 0 || k_hi <= k_lo) return cudaGetLastError();
@@ -754,6 +778,20 @@ cudaError_t launch_match_scan(uint32_t K, const uint64_t* kto, const uint64_t* s
   const uint64_t j0 = filter_jobs_before(kb_lo), j1 = filter_jobs_before(kb_hi);
   if (j1 > j0) note_launch(), k_pair_filter<<<(unsigned)(j1 - j0), 256, 0, s>>>(a, j0, kb_lo, kb_hi);
   unsigned grid = (unsigned)num_sms * 8;
+  if (fused) {
+    // bucket the survivors by k into the pairs buffer (free in the fused path: close pairs go to cand segments)
+    const unsigned gb = (unsigned)umin64(ceil_div(mw.pair_cap, 256), (uint64_t)num_sms * 64);
+    cudaMemsetAsync(mw.cand_cnt, 0, sizeof(uint32_t) * K, s);
+    cudaMemsetAsync(mw.close_cnt, 0, sizeof(uint32_t) * K, s);
+    note_launch(), k_cand_count<<<gb, 256, 0, s>>>(mw.maybe, mw.pair_cap, mw.n_maybe, K, mw.cand_cnt, err);
+    note_launch(), k_cand_scan<<<1, 1024, 0, s>>>(mw.cand_cnt, K, mw.cand_off, mw.cand_cur);
+    note_launch(), k_pair_bucket<<<gb, 256, 0, s>>>(mw.maybe, mw.pair_cap, mw.n_maybe, K, mw.cand_off, mw.cand_cur,
+                                                    pairs);
+    a.maybe = pairs;
+    a.cand = mw.cand;
+    a.cbeg = mw.cand_off;
+    a.ccnt = mw.close_cnt;
+  }
   note_launch(), k_pair_exact<<<grid, 256, 0, s>>>(a, pairs, pair_cap, n_pairs);
   return cudaGetLastError();
 }
@@ -761,14 +799,17 @@ cudaError_t launch_match_scan(uint32_t K, const uint64_t* kto, const uint64_t* s
 cudaError_t launch_match_resolve(uint32_t K, const uint64_t* kto, const uint64_t* sig, const uint64_t* mass,
                                  const uint64_t* wt, photon_match_params p, const uint64_t* pairs, uint64_t n_pairs,
                                  const uint64_t* n_pairs_dev, const MatchWs& mw, int64_t* match, double* match_dist,
-                                 DevErr* err, int num_sms, cudaStream_t s) {
+                                 DevErr* err, int num_sms, cudaStream_t s, bool fused) {
   if (K == 0) return cudaSuccess;
-  cudaMemsetAsync(mw.cand_cnt, 0, sizeof(uint32_t) * K, s);
-  if (n_pairs) {
+  // candidate segments: fused -- written by k_pair_exact into the k-buckets (cand_off, close_cnt); else built here
+  // from the pair list (cand_off, cand_cnt)
+  const uint32_t* ccnt = fused ? mw.close_cnt : mw.cand_cnt;
+  if (!fused) cudaMemsetAsync(mw.cand_cnt, 0, sizeof(uint32_t) * K, s);
+  if (!fused && n_pairs) {
     note_launch(), k_cand_count<<<(unsigned)ceil_div(n_pairs, 256), 256, 0, s>>>(pairs, n_pairs, n_pairs_dev, K, mw.cand_cnt, err);
   }
-  note_launch(), k_cand_scan<<<1, 1024, 0, s>>>(mw.cand_cnt, K, mw.cand_off, mw.cand_cur);
-  if (n_pairs) {
+  if (!fused) note_launch(), k_cand_scan<<<1, 1024, 0, s>>>(mw.cand_cnt, K, mw.cand_off, mw.cand_cur);
+  if (!fused && n_pairs) {
     note_launch(), k_cand_scatter<<<(unsigned)ceil_div(n_pairs, 256), 256, 0, s>>>(pairs, n_pairs, n_pairs_dev, K, mw.cand_off,
                                                                     mw.cand_cur, mw.cand);
   }
@@ -781,20 +822,20 @@ cudaError_t launch_match_resolve(uint32_t K, const uint64_t* kto, const uint64_t
     unsigned grid = (unsigned)umin64((uint64_t)per_sm * num_sms, ceil_div((uint64_t)K * 32, 256));
     const uint64_t* off = mw.cand_off;
     const uint32_t* cand = mw.cand;
-    void* args[] = {(void*)&K, (void*)&off, (void*)&cand, (void*)&mw.state, (void*)&mw.cand_cur, (void*)&mw.ulist,
-                    (void*)&mw.rcnt, (void*)&mw.flag};
+    void* args[] = {(void*)&K, (void*)&off, (void*)&ccnt, (void*)&cand, (void*)&mw.state, (void*)&mw.cand_cur,
+                    (void*)&mw.ulist, (void*)&mw.rcnt, (void*)&mw.flag};
     note_launch();
     cudaError_t e = cudaLaunchCooperativeKernel((void*)k_resolve_coop, grid, 256, args, 0, s);
     if (e != cudaSuccess) return e;
   } else if (K <= 40960) {
     cudaFuncSetAttribute(k_resolve_states<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, 40960);
-    note_launch(), k_resolve_states<true><<<1, 1024, K, s>>>(K, mw.cand_off, mw.cand, mw.state, mw.cand_cur, mw.ulist,
+    note_launch(), k_resolve_states<true><<<1, 1024, K, s>>>(K, mw.cand_off, ccnt, mw.cand, mw.state, mw.cand_cur, mw.ulist,
                                                               mw.flag, p.pool_all_prior);
   } else {
-    note_launch(), k_resolve_states<false><<<1, 1024, 0, s>>>(K, mw.cand_off, mw.cand, mw.state, mw.cand_cur,
+    note_launch(), k_resolve_states<false><<<1, 1024, 0, s>>>(K, mw.cand_off, ccnt, mw.cand, mw.state, mw.cand_cur,
                                                                mw.ulist, mw.flag, p.pool_all_prior);
   }
-  note_launch(), k_resolve_match<<<(unsigned)ceil_div((uint64_t)K * 32, 256), 256, 0, s>>>(K, mw.cand_off, mw.cand, mw.state,
+  note_launch(), k_resolve_match<<<(unsigned)ceil_div((uint64_t)K * 32, 256), 256, 0, s>>>(K, mw.cand_off, ccnt, mw.cand, mw.state,
                                                                            p.pool_all_prior, wt, kto, sig, mass,
                                                                            match, match_dist);
   if (match_dist)
