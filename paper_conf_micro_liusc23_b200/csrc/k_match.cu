@@ -578,75 +578,39 @@ __global__ void __launch_bounds__(1024) k_resolve_states(uint32_t K, const uint6
   if (threadIdx.x == 0) flag[0] = rounds;
 }
 
-// The same fixed point over the whole GPU: a cooperative grid, one grid-wide barrier per round (rounds are few: the
-// longest chain of kernels blocked on undecided predecessors).  Each round visits the undecided list of the previous
-// round; a blocked kernel keeps its cursor.  Stale state reads only postpone a decision (states are monotone).
-__global__ void __launch_bounds__(256) k_resolve_coop(uint32_t K, const uint64_t* __restrict__ beg,
+// The same fixed point in ONE pass over the whole GPU, without barriers: warp j decides kernels j, j + nw, ... in
+// increasing order, each by the sequential rule (k is a representative iff none of its close predecessors is one),
+// waiting on a predecessor that is still undecided.  A predecessor r < k belongs to an earlier iteration of some
+// warp (or the same iteration of a warp with a smaller index), and the smallest undecided kernel never waits, so
+// with every warp resident (cooperative launch) the waits always end.  A kernel stops at its first representative.
+__global__ void __launch_bounds__(256) k_resolve_spin(uint32_t K, const uint64_t* __restrict__ beg,
                                                       const uint32_t* __restrict__ cnt,
                                                       const uint32_t* __restrict__ cand, uint8_t* state,
-                                                      uint32_t* cursor, uint32_t* ulist, uint32_t* rcnt,
                                                       uint32_t* flag) {
-  namespace cg = cooperative_groups;
-  cg::grid_group grid = cg::this_grid();
-  const uint64_t gt = grid.thread_rank(), gs = grid.size();
-  for (uint64_t k = gt; k < K; k += gs) {
-    state[k] = 0;
-    cursor[k] = 0;
-  }
-  for (uint64_t i = gt; i < (uint64_t)K + 2; i += gs) rcnt[i] = 0;
-  grid.sync();
-  volatile uint8_t* vs = state;
   const uint32_t lane = threadIdx.x & 31;
-  const uint64_t gw = gt >> 5, nw = gs >> 5;
-  uint32_t n = K;
-  const uint32_t* cur = nullptr;  // nullptr = identity (round 1 visits every kernel)
-  uint32_t* nxt = ulist;
-  uint32_t round = 0;
-  for (;;) {
-    // one warp per undecided kernel: 128 candidates (4 x 32 independent loads) per step, ballots decide
-    for (uint64_t q = gw; q < n; q += nw) {
-      const uint32_t k = cur ? cur[q] : (uint32_t)q;
-      const uint64_t o0 = beg[k], o1 = o0 + cnt[k];
-      uint64_t first_undec = o1;
-      bool rep_found = false;
-      for (uint64_t i0 = o0 + cursor[k]; i0 < o1; i0 += 128) {
-        uint32_t c4[4];
-#pragma unroll
-        for (int u = 0; u < 4; ++u) {
-          const uint64_t i = i0 + u * 32 + lane;
-          c4[u] = i < o1 ? cand[i] : UINT32_MAX;
-        }
-        uint8_t st[4];
-#pragma unroll
-        for (int u = 0; u < 4; ++u) st[u] = c4[u] != UINT32_MAX ? vs[c4[u]] : (uint8_t)2;
-        bool stop = false;
-#pragma unroll
-        for (int u = 0; u < 4; ++u) {
-          const unsigned rep = __ballot_sync(0xffffffffu, st[u] == 1);
-          const unsigned und = __ballot_sync(0xffffffffu, st[u] == 0);
-          if (rep) { rep_found = true; stop = true; break; }
-          if (und && first_undec == o1) first_undec = i0 + u * 32 + (__ffs(und) - 1);
-        }
-        if (stop) break;
+  const uint64_t gw = ((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const uint64_t nw = ((uint64_t)gridDim.x * blockDim.x) >> 5;
+  volatile uint8_t* vs = state;
+  for (uint64_t k = gw; k < K; k += nw) {
+    const uint64_t o0 = beg[k], o1 = o0 + cnt[k];
+    bool rep_found = false;
+    for (;;) {  // a sweep over all candidates: any representative decides at once; else wait while any is open
+      bool open = false;
+      for (uint64_t i0 = o0; i0 < o1; i0 += 32) {
+        const uint64_t i = i0 + lane;
+        const uint8_t st = i < o1 ? vs[cand[i]] : (uint8_t)2;
+        if (__ballot_sync(0xffffffffu, st == 1)) { rep_found = true; break; }
+        open |= __ballot_sync(0xffffffffu, st == 0) != 0;
       }
-      if (lane == 0) {
-        if (!rep_found && first_undec < o1) {  // blocked by an undecided predecessor: resume there next round
-          cursor[k] = (uint32_t)(first_undec - o0);
-          nxt[atomicAdd(&rcnt[round], 1u)] = k;
-        } else {
-          vs[k] = rep_found ? 2 : 1;
-        }
-      }
+      if (rep_found || !open) break;
+      __nanosleep(100);  // back off: many waiting warps poll L2
     }
-    grid.sync();
-    n = *(volatile uint32_t*)&rcnt[round];
-    ++round;
-    if (n == 0 || round > K) break;
-    cur = nxt;  // ping-pong between the two halves of ulist (the other half was fully read before the barrier)
-    nxt = (cur == ulist) ? ulist + K : ulist;
+    __syncwarp();
+    if (lane == 0) vs[k] = rep_found ? 2 : 1;
   }
-  if (gt == 0) flag[0] = round;
+  if (gw == 0 && lane == 0) flag[0] = 1;
 }
+
 
 // match[k] = argmin over eligible candidates of (|W_k - W_r|, r); match_dist exact -> fp64 (one warp per kernel)
 __global__ void k_resolve_match(uint32_t K, const uint64_t* beg, const uint32_t* cnt, const uint32_t* cand,
@@ -813,19 +777,19 @@ cudaError_t launch_match_resolve(uint32_t K, const uint64_t* kto, const uint64_t
     note_launch(), k_cand_scatter<<<(unsigned)ceil_div(n_pairs, 256), 256, 0, s>>>(pairs, n_pairs, n_pairs_dev, K, mw.cand_off,
                                                                     mw.cand_cur, mw.cand);
   }
-  if (!p.pool_all_prior && K > 2048) {  // large K: the whole GPU, one grid barrier per round
+  if (!p.pool_all_prior && K > 2048) {  // large K: the whole GPU, one pass (every warp resident: cooperative launch)
     static int per_sm = 0;
     if (!per_sm) {
-      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_resolve_coop, 256, 0);
+      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_resolve_spin, 256, 0);
       if (per_sm < 1) per_sm = 1;
     }
     unsigned grid = (unsigned)umin64((uint64_t)per_sm * num_sms, ceil_div((uint64_t)K * 32, 256));
+    cudaMemsetAsync(mw.state, 0, K, s);
     const uint64_t* off = mw.cand_off;
     const uint32_t* cand = mw.cand;
-    void* args[] = {(void*)&K, (void*)&off, (void*)&ccnt, (void*)&cand, (void*)&mw.state, (void*)&mw.cand_cur,
-                    (void*)&mw.ulist, (void*)&mw.rcnt, (void*)&mw.flag};
+    void* args[] = {(void*)&K, (void*)&off, (void*)&ccnt, (void*)&cand, (void*)&mw.state, (void*)&mw.flag};
     note_launch();
-    cudaError_t e = cudaLaunchCooperativeKernel((void*)k_resolve_coop, grid, 256, args, 0, s);
+    cudaError_t e = cudaLaunchCooperativeKernel((void*)k_resolve_spin, grid, 256, args, 0, s);
     if (e != cudaSuccess) return e;
   } else if (K <= 40960) {
     cudaFuncSetAttribute(k_resolve_states<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, 40960);
