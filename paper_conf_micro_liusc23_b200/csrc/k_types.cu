@@ -118,71 +118,98 @@ __device__ void emit_rows(const HashTable& ht, uint32_t k, const uint32_t* sorte
   }
 }
 
+// 32 < T_k <= 128: a register bitonic sort of 32E elements (E per lane, element i = lane * E + e) on a packed key
+// (~count) << 32 | key word 0 -- count desc, then key asc -- with the full-key compare (type_before) on ties.
+template <int E>
+__device__ __forceinline__ void warp_sort_reg(const HashTable& ht, uint64_t (&sk)[E], uint32_t (&sl)[E]) {
+  const uint32_t lane = threadIdx.x & 31;
+  auto before = [&](uint64_t ka, uint32_t sa, uint64_t kb, uint32_t sb) -> bool {  // a before b, padding last
+    if (sa == UINT32_MAX) return false;
+    if (sb == UINT32_MAX) return true;
+    if (ka != kb) return ka < kb;
+    return type_before(ht, sa, sb);
+  };
+  auto cswap = [&](int e, int f, uint32_t size) {  // in-lane pair (e < f)
+    const bool up = ((lane * E + e) & size) == 0;
+    const bool sw = up ? before(sk[f], sl[f], sk[e], sl[e]) : before(sk[e], sl[e], sk[f], sl[f]);
+    if (sw) {
+      const uint64_t tk = sk[e]; sk[e] = sk[f]; sk[f] = tk;
+      const uint32_t ts = sl[e]; sl[e] = sl[f]; sl[f] = ts;
+    }
+  };
+  for (uint32_t size = 2; size <= 32u * E; size <<= 1) {
+    for (uint32_t st = size >> 1; st > 0; st >>= 1) {
+      if (st >= (uint32_t)E) {
+        const uint32_t ls = st / E;
+        const bool lower = (lane & ls) == 0;
+#pragma unroll
+        for (int e = 0; e < E; ++e) {
+          const uint64_t ok = __shfl_xor_sync(0xffffffffu, sk[e], ls);
+          const uint32_t os = __shfl_xor_sync(0xffffffffu, sl[e], ls);
+          const bool up = ((lane * E + e) & size) == 0;
+          const bool mb = before(sk[e], sl[e], ok, os);
+          const bool keep = (lower == up) ? mb : !mb;
+          if (!keep && os != sl[e]) { sk[e] = ok; sl[e] = os; }
+        }
+      } else if (st == 1) {
+#pragma unroll
+        for (int e = 0; e < E; e += 2) cswap(e, e + 1, size);
+      } else {  // st == 2 (E == 4)
+        if (E == 4) { cswap(0, 2, size); cswap(1, 3, size); }
+      }
+    }
+  }
+}
+template <int E>
+__device__ __forceinline__ void sort_mid_reg(const HashTable& ht, uint64_t off, uint64_t n, const uint32_t* list,
+                                             const photon_types& out, uint32_t* canon, uint64_t Wk, uint32_t k) {
+  const uint32_t lane = threadIdx.x & 31;
+  uint64_t sk[E];
+  uint32_t sl[E];
+#pragma unroll
+  for (int e = 0; e < E; ++e) {
+    const uint32_t i = lane * E + e;
+    sl[e] = i < n ? list[off + i] : UINT32_MAX;
+    sk[e] = sl[e] != UINT32_MAX ? ((uint64_t)(~ht.count[sl[e]]) << 32) | ht.key[(uint64_t)sl[e] * 16] : ~0ull;
+  }
+  warp_sort_reg<E>(ht, sk, sl);
+#pragma unroll
+  for (int e = 0; e < E; ++e) {
+    const uint32_t r = lane * E + e, sl_ = sl[e];
+    if (r < n && off + r < out.capacity) {
+      const uint4* src = (const uint4*)(ht.key + (uint64_t)sl_ * 16);
+      uint4* dst = (uint4*)(out.type_key + (off + r) * 16);
+      dst[0] = src[0]; dst[1] = src[1]; dst[2] = src[2]; dst[3] = src[3];
+      out.type_count[off + r] = ht.count[sl_];
+      out.type_first_warp[off + r] = ht.first[sl_];
+      canon[sl_] = r;
+    }
+  }
+  const uint32_t first = __shfl_sync(0xffffffffu, sl[0], 0);
+  if (lane == 0) {
+    const uint64_t c0 = ht.count[first];
+    out.warp_sampling_ok[k] = (Wk > 0 && 100ull * c0 > 95ull * Wk) ? 1 : 0;  // L249 [P-15]
+  }
+}
+
 // Kernels with T_k <= 32 (almost all): one warp each, bitonic network over the first P = next_pow2(T_k) lanes with
-// shuffles; 32 < T_k <= 128: the same warp, a warp-private shared-memory bitonic sort.  Larger kernels are queued:
+// shuffles; 32 < T_k <= 128: the same warp, a register bitonic sort of 2 or 4 elements per lane.  Larger kernels are queued:
 // T_k <= SORT_SMEM_MAX at the front of cw.big (k_sort_mid, one CTA each), larger ones at the back (k_sort_large).
 __global__ void __launch_bounds__(256) k_sort_warp(HashTable ht, uint32_t K, const uint64_t* kto,
                                                    const uint32_t* list, const uint64_t* kwo,
                                                    const uint64_t* kernel_warps, photon_types out, uint32_t* canon,
                                                    uint32_t* big, uint32_t* nbig) {
-  const uint32_t lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
+  const uint32_t lane = threadIdx.x & 31;
   const uint32_t k = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   if (k >= K) return;
   const uint64_t off = kto[k], n = kto[k + 1] - off;
   const uint64_t Wk = kernel_warps ? kernel_warps[k] : (kwo[k + 1] - kwo[k]);
-  if (n > 32 && n <= WARP_SORT_MAX) {
-    // 32 < T_k <= 128: warp-private shared-memory bitonic sort; count and key words 0-3 staged in shared memory
-    __shared__ uint32_t s_slot[8][WARP_SORT_MAX], s_cnt[8][WARP_SORT_MAX];
-    __shared__ uint4 s_k0[8][WARP_SORT_MAX];
-    __shared__ uint16_t s_idx[8][WARP_SORT_MAX];
-    uint32_t P = 64;
-    while (P < n) P <<= 1;
-    for (uint32_t i = lane; i < P; i += 32) {
-      s_idx[wib][i] = (uint16_t)i;
-      if (i < n) {
-        uint32_t sl = list[off + i];
-        s_slot[wib][i] = sl;
-        s_cnt[wib][i] = ht.count[sl];
-        s_k0[wib][i] = *(const uint4*)(ht.key + (uint64_t)sl * 16);
-      }
-    }
-    __syncwarp();
-    auto before = [&](uint32_t a, uint32_t b) -> bool {  // element a before element b (padding last)
-      if (b >= n) return a < n;
-      if (a >= n) return false;
-      uint32_t ca = s_cnt[wib][a], cb = s_cnt[wib][b];
-      if (ca != cb) return ca > cb;
-      uint4 ka = s_k0[wib][a], kb = s_k0[wib][b];
-      if (ka.x != kb.x) return ka.x < kb.x;
-      if (ka.y != kb.y) return ka.y < kb.y;
-      if (ka.z != kb.z) return ka.z < kb.z;
-      if (ka.w != kb.w) return ka.w < kb.w;
-      return type_before(ht, s_slot[wib][a], s_slot[wib][b]);  // words 4.. (rare)
-    };
-    for (uint32_t size = 2; size <= P; size <<= 1) {
-      for (uint32_t stride = size >> 1; stride > 0; stride >>= 1) {
-        for (uint32_t t = lane; t < P / 2; t += 32) {
-          uint32_t i = 2 * stride * (t / stride) + (t % stride), j = i + stride;
-          bool up = ((i & size) == 0);
-          uint32_t a = s_idx[wib][i], b = s_idx[wib][j];
-          if (up ? before(b, a) : before(a, b)) { s_idx[wib][i] = (uint16_t)b; s_idx[wib][j] = (uint16_t)a; }
-        }
-        __syncwarp();
-      }
-    }
-    for (uint32_t r = lane; r < n && off + r < out.capacity; r += 32) {
-      uint32_t sl = s_slot[wib][s_idx[wib][r]];
-      const uint4* src = (const uint4*)(ht.key + (uint64_t)sl * 16);
-      uint4* dst = (uint4*)(out.type_key + (off + r) * 16);
-      dst[0] = src[0]; dst[1] = src[1]; dst[2] = src[2]; dst[3] = src[3];
-      out.type_count[off + r] = ht.count[sl];
-      out.type_first_warp[off + r] = ht.first[sl];
-      canon[sl] = r;
-    }
-    if (lane == 0) {
-      uint64_t c0 = s_cnt[wib][s_idx[wib][0]];
-      out.warp_sampling_ok[k] = (Wk > 0 && 100ull * c0 > 95ull * Wk) ? 1 : 0;  // L249 [P-15]
-    }
+  if (n > 32 && n <= 64) {
+    sort_mid_reg<2>(ht, off, n, list, out, canon, Wk, k);
+    return;
+  }
+  if (n > 64 && n <= WARP_SORT_MAX) {
+    sort_mid_reg<4>(ht, off, n, list, out, canon, Wk, k);
     return;
   }
   if (n > 32) {
