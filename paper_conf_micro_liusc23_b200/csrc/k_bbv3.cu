@@ -25,9 +25,11 @@
 //  * After the loop each lane sums its warp's pieces (owner column, then slot 0 of every later lane it spans) into
 //    16 key registers, carried across the chunks of a block; the worker's cells are cleared with 16-byte stores.
 //  * Fused: at the block's end the keys are hashed, grouped with __match_any_sync plus an exact 17-word check, and
-//    each distinct (kernel, key) of the block becomes one 80-byte entry (key, first warp, kernel, count) taken
-//    from the worker's run of the global entry pool (one atomic per ENT_BLK entries).  Each warp records its
-//    entry index (u32).  The entries are inserted into the global type table afterwards (k_types.cu).
+//    each distinct (kernel, key) of the block is looked up in the worker's direct-mapped cache of its recent
+//    entries (hash -> entry id): a hit that matches the entry's own key exactly adds the block's count to it,
+//    otherwise the key becomes a new 80-byte entry (key, first warp, kernel, count) from the worker's run of the
+//    global entry pool (one atomic per ENT_BLK entries).  Each warp records its entry index (u32).  The entries
+//    are inserted into the global type table afterwards (k_types.cu).
 #include "internal.h"
 
 namespace photon {
@@ -95,6 +97,7 @@ struct Args3 {
 };
 
 // per-worker scratch in shared memory
+constexpr int kEntCache = 128;
 struct WMisc {
   uint32_t rel[40];             // chunk-relative starts of the block's warps (rel[nw..] = block end), clamped
   uint32_t fwt[32];             // first-warp scatter table of the lane ranges
@@ -104,6 +107,10 @@ struct WMisc {
   uint32_t i_live, i_n;
   // the worker's current block of pool entries (fused)
   uint64_t e_next, e_end;
+  // direct-mapped cache of the worker's recent entries (hash -> entry id): a type seen again in a later block of
+  // the worker adds to its entry after an exact key check instead of opening a new one
+  uint64_t ch[kEntCache];
+  uint32_t ce[kEntCache];
 };
 constexpr uint32_t kWMiscBytes = (sizeof(WMisc) + 127) & ~127u;
 
@@ -171,6 +178,7 @@ __device__ __forceinline__ uint64_t hash16(uint32_t k, const uint32_t* p) {
 
 __device__ __forceinline__ void pool_init(WMisc* wm) {
   if ((threadIdx.x & 31) == 0) { wm->e_next = 0; wm->e_end = 0; }
+  for (int i = threadIdx.x & 31; i < kEntCache; i += 32) wm->ch[i] = 0ull;
   __syncwarp();
 }
 __device__ __forceinline__ void pool_flush(const Args3& a, WMisc* wm) {
@@ -196,7 +204,28 @@ __device__ void finalize_fused(const Args3& a, WMisc* wm, uint64_t w0, bool vali
   const unsigned eqm = __ballot_sync(0xffffffffu, eq);
   const bool is_l = valid && ((int)lane == leader || !eq);
   const uint32_t cnt = ((int)lane == leader) ? (uint32_t)__popc(peers & eqm & vmask) : 1u;
-  const unsigned lm = __ballot_sync(0xffffffffu, is_l);
+  // the worker's entry cache: an exact (kernel, key) match adds this block's count to the existing entry
+  uint32_t hit = UINT32_MAX;
+  const uint32_t cslot = (uint32_t)h & (kEntCache - 1);
+  if (is_l && wm->ch[cslot] == h) {
+    const uint32_t e = wm->ce[cslot];
+    if (e < a.ep.cap) {  // the exact check against the entry itself (written by this warp earlier)
+      TileEntry* d = a.ep.ent + e;
+      const uint4* kd = (const uint4*)d->key;
+      bool same = d->kernel == k;
+#pragma unroll
+      for (int q = 0; q < 4; ++q) {
+        const uint4 v = kd[q];
+        same &= v.x == p[4 * q] && v.y == p[4 * q + 1] && v.z == p[4 * q + 2] && v.w == p[4 * q + 3];
+      }
+      if (same) {
+        atomicAdd(&d->count, cnt);
+        hit = e;
+      }
+    }
+  }
+  const bool alloc = is_l && hit == UINT32_MAX;
+  const unsigned lm = __ballot_sync(0xffffffffu, alloc);
   const uint32_t nl = __popc(lm), rank = __popc(lm & ((1u << lane) - 1u));
   // entry ids: the rest of the worker's block, then a new block of ENT_BLK (one atomic per ENT_BLK entries)
   uint64_t e_next = wm->e_next, e_end = wm->e_end;
@@ -216,7 +245,7 @@ __device__ void finalize_fused(const Args3& a, WMisc* wm, uint64_t w0, bool vali
     id = e_next + rank;
     e_next += nl;
   }
-  if (is_l && id < a.ep.cap) {
+  if (alloc && id < a.ep.cap) {
     TileEntry* d = a.ep.ent + id;
     uint4* kd = (uint4*)d->key;
     kd[0] = make_uint4(p[0], p[1], p[2], p[3]);
@@ -227,8 +256,14 @@ __device__ void finalize_fused(const Args3& a, WMisc* wm, uint64_t w0, bool vali
     kd[4] = make_uint4((uint32_t)w, (uint32_t)(w >> 32), k, cnt);  // first warp, kernel, count
   }
   __syncwarp();
+  if (alloc) {  // remember the new entry: two leaders on one slot may leave its hash and id from different entries,
+                // which only costs a miss (every hit is checked against the entry's own key)
+    wm->ch[cslot] = h;
+    wm->ce[cslot] = (uint32_t)umin64(id, 0xFFFFFFFFull);
+  }
   if (lane == 0) { wm->e_next = e_next; wm->e_end = e_end; }
-  const uint32_t ent = (uint32_t)umin64(id, 0xFFFFFFFFull);
+  __syncwarp();
+  const uint32_t ent = alloc ? (uint32_t)umin64(id, 0xFFFFFFFFull) : hit;
   const uint32_t le = __shfl_sync(0xffffffffu, ent, leader);
   if (valid) a.ep.gid[w0 + lane] = (eq && (int)lane != leader) ? le : ent;
 }
