@@ -134,6 +134,12 @@ PHOTON_API int photon_bbv_build(photon_ctx *ctx, const photon_trace *trace, void
 PHOTON_API size_t photon_group_workspace_bytes(const photon_trace *trace, uint64_t type_capacity_hint);
 PHOTON_API int photon_warp_group(photon_ctx *ctx, const photon_trace *trace, const uint32_t *warp_bbv16 /*or NULL*/, void *ws,
                       size_t ws_bytes, photon_types *out, void *stream);
+/* The same call with its last step -- writing out->warp_type from the canonical ids -- issued on `remap_stream`
+ * (after an event wait on `stream`): everything but warp_type is complete in `stream` order when the call's work
+ * there is; warp_type is complete in `remap_stream` order.  Lets later per-type work (A3/A4) on `stream` overlap
+ * the per-warp write; the caller joins the streams before reading warp_type. */
+PHOTON_API int photon_warp_group2(photon_ctx *ctx, const photon_trace *trace, const uint32_t *warp_bbv16 /*or NULL*/,
+                                  void *ws, size_t ws_bytes, photon_types *out, void *stream, void *remap_stream);
 /* SYNCS the stream and returns kernel_type_off[K] (total types) in *total_types (HOST). */
 PHOTON_API int photon_types_total(photon_ctx *ctx, const photon_types *types, uint32_t n_kernels, uint64_t *total_types,
                        void *stream);

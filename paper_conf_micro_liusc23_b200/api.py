@@ -202,7 +202,8 @@ class Photon:
                           p("type_first_warp"), p("warp_sampling_ok"))
 
     def photon_warp_group(self, t: DeviceTrace, warp_bbv16=None, capacity_hint: int = 0, stream=None,
-                          check: bool = True, out: Optional[dict] = None) -> dict:
+                          check: bool = True, out: Optional[dict] = None, remap_stream=None) -> dict:
+        """remap_stream (optional): warp_type is written there (photon_warp_group2) -- join it before reading."""
         key = (t.n_kernels, t.n_warps)
         hint = max(capacity_hint, self._hint.get(key, 0))
         for _ in range(8):
@@ -212,9 +213,10 @@ class Photon:
             cap = min(max(t.n_warps, 1), ht_capacity(hint, t.n_warps))
             ty = out if self._types_fit(out, t.n_kernels, t.n_warps, cap) else self.alloc_types(t.n_kernels, t.n_warps, cap)
             tc = self.types_c(ty)
-            self._rc(self.L.photon_warp_group(self.ctx, ctypes.byref(ct),
-                                              None if warp_bbv16 is None else warp_bbv16.data_ptr(), ws.data_ptr(),
-                                              ws.numel(), ctypes.byref(tc), self.stream_ptr(stream)))
+            self._rc(self.L.photon_warp_group2(self.ctx, ctypes.byref(ct),
+                                               None if warp_bbv16 is None else warp_bbv16.data_ptr(), ws.data_ptr(),
+                                               ws.numel(), ctypes.byref(tc), self.stream_ptr(stream),
+                                               self.stream_ptr(remap_stream if remap_stream is not None else stream)))
             ty["_ws"] = ws
             if not check:
                 return ty
@@ -540,13 +542,19 @@ class Photon:
         """A1 -> A2 -> A3 -> A4 on one device (fused BBV + grouping pass, then canonical tables, signatures,
         match).  With check=False nothing synchronises (errors stay latched in the returned workspaces).  `out` (a
         previous result for the same trace) is reused instead of allocating new output tables."""
-        ty = self.photon_warp_group(t, None, capacity_hint, stream=stream, check=check, out=out)
+        # the per-warp warp_type write runs on a side stream, overlapping A3/A4 on the main one (joined below)
+        main = stream if stream is not None else self.torch.cuda.current_stream(self.device)
+        if getattr(self, "_side", None) is None:
+            self._side = self.torch.cuda.Stream(device=self.device)
+        side = self._side
+        ty = self.photon_warp_group(t, None, capacity_hint, stream=main, check=check, out=out, remap_stream=side)
         K = t.n_kernels
         ok = lambda k: out is not None and out.get(k) is not None and out[k].numel() == K
         mo = {"match": out["match"]} if ok("match") else None
         if mo is not None and want_dist and ok("match_dist"):
             mo["match_dist"] = out["match_dist"]
         m = self.photon_kernel_match(t.n_kernels, ty, t.warps_total, theta, n_cores, pool_all_prior, want_dist,
-                                     pair_capacity, stream=stream, check=check, out=mo)
+                                     pair_capacity, stream=main, check=check, out=mo)
+        main.wait_stream(side)
         ty.update(match=m["match"], match_dist=m.get("match_dist"), _mws=m["_ws"])
         return ty

@@ -21,6 +21,7 @@ struct photon_ctx {
   bool prof = false;
   std::vector<std::pair<cudaEvent_t, cudaEvent_t>> ev[PHOTON_PROF_N];
   size_t used[PHOTON_PROF_N] = {0};
+  cudaEvent_t fork = nullptr;  // photon_warp_group2: the remap's dependency on the main stream
 };
 
 namespace {
@@ -306,6 +307,7 @@ void photon_destroy(photon_ctx* ctx) {
   if (!ctx) return;
   for (auto& v : ctx->ev)
     for (auto& pr : v) { cudaEventDestroy(pr.first); cudaEventDestroy(pr.second); }
+  if (ctx->fork) cudaEventDestroy(ctx->fork);
   delete ctx;
 }
 
@@ -396,6 +398,11 @@ size_t photon_group_workspace_bytes(const photon_trace* t, uint64_t hint) {
 
 int photon_warp_group(photon_ctx* ctx, const photon_trace* t, const uint32_t* warp_bbv16, void* ws, size_t ws_bytes,
                       photon_types* out, void* stream) {
+  return photon_warp_group2(ctx, t, warp_bbv16, ws, ws_bytes, out, stream, stream);
+}
+
+int photon_warp_group2(photon_ctx* ctx, const photon_trace* t, const uint32_t* warp_bbv16, void* ws, size_t ws_bytes,
+                       photon_types* out, void* stream, void* remap_stream) {
   if (!ctx) return PHOTON_EINVAL;
   int rc = check_trace(ctx, t);
   if (rc) return rc;
@@ -434,7 +441,13 @@ int photon_warp_group(photon_ctx* ctx, const photon_trace* t, const uint32_t* wa
     CK(launch_entries_insert(g.ep, g.h.ht, err, ctx->num_sms, s), "insert");
     CK(launch_canonicalise(g.h.ht, t->n_kernels, t->kernel_warp_off, nullptr, *out, g.h.cw, err, ctx->num_sms, s),
        "canon");
-    CK(launch_remap_entries(g.ep, t->n_warps, g.h.cw.canon, out->warp_type, s), "remap");
+    cudaStream_t rs = (cudaStream_t)remap_stream;
+    if (rs != s) {  // fork: the per-warp write on its own stream, after the canonical ids exist
+      if (!ctx->fork) CK(cudaEventCreateWithFlags(&ctx->fork, cudaEventDisableTiming), "event");
+      CK(cudaEventRecord(ctx->fork, s), "event");
+      CK(cudaStreamWaitEvent(rs, ctx->fork, 0), "event");
+    }
+    CK(launch_remap_entries(g.ep, t->n_warps, g.h.cw.canon, out->warp_type, rs), "remap");
   }
   return PHOTON_OK;
 }
