@@ -32,19 +32,41 @@ constexpr int RBITS = 8;
 constexpr int RNB = 1 << RBITS;
 constexpr int REC_CHUNK = 4096;
 constexpr int JOB = 2048;       // records per warp job (one-pass multisplit)
-// the grouped copy holds retire (u64) and the duration retire - issue (u32); a duration >= kDurEsc is stored as
-// kDurEsc with the issue time in a side array (written only for those records)
+// The grouped copy: per record the retire time relative to its kernel's first retire (u32) and the duration
+// retire - issue (u32), 8 B/record; a relative retire or a duration >= kDurEsc is stored as kDurEsc with the exact
+// relative value in a side array (Yw: relative retire; Xw: relative issue, may be negative), written only for
+// those records.  Eq. 1's sums are shift-invariant over full windows and S_n, S_2n are durations, so the window
+// test and S_n need no absolute time.  (The radix path, B > 8192, uses base 0: absolute times, escaped >= 2^32.)
 constexpr uint32_t kDurEsc = 0xFFFFFFFFu;
-__device__ __forceinline__ void put_rec(uint64_t* Y, uint32_t* D, uint64_t* Xw, uint64_t dest, uint64_t x,
-                                        uint64_t y) {
-  Y[dest] = y;
+struct GCopy {
+  uint32_t* Y32;  // [R] relative retire, kDurEsc: in Yw
+  uint32_t* D;    // [R] duration, kDurEsc: issue in Xw
+  int64_t* Yw;    // [R] relative retire (escaped records only)
+  int64_t* Xw;    // [R] relative issue (escaped durations only)
+};
+__device__ __forceinline__ void put_rec(const GCopy& G, uint64_t dest, uint64_t x, uint64_t y, uint64_t base) {
+  const int64_t yr = (int64_t)(y - base);  // retire >= the kernel's first retire (validated order)
+  if ((uint64_t)yr < kDurEsc) {
+    G.Y32[dest] = (uint32_t)yr;
+  } else {
+    G.Y32[dest] = kDurEsc;
+    G.Yw[dest] = yr;
+  }
   const uint64_t d = y - x;
   if (d < kDurEsc) {
-    D[dest] = (uint32_t)d;
+    G.D[dest] = (uint32_t)d;
   } else {
-    D[dest] = kDurEsc;
-    Xw[dest] = x;
+    G.D[dest] = kDurEsc;
+    G.Xw[dest] = (int64_t)x - (int64_t)base;
   }
+}
+__device__ __forceinline__ int64_t g_y(const GCopy& G, uint64_t q) {
+  const uint32_t v = __ldg(G.Y32 + q);
+  return v != kDurEsc ? (int64_t)v : __ldg(G.Yw + q);
+}
+__device__ __forceinline__ int64_t g_x(const GCopy& G, uint64_t q, int64_t y) {
+  const uint32_t d = __ldg(G.D + q);
+  return d != kDurEsc ? y - (int64_t)d : __ldg(G.Xw + q);
 }
 constexpr int WT = 256;        // window threads
 constexpr int WPT = 8;         // positions per thread
@@ -290,12 +312,11 @@ __global__ void __launch_bounds__(RT) k_radix_down(const uint64_t* key, const ui
 }
 
 // ---- 3. gather + groups + work items -------------------------------------------------------------------------
-__global__ void k_gather(const uint32_t* idx, uint64_t n, const uint64_t* issue, const uint64_t* retire, uint64_t* Y,
-                         uint32_t* D, uint64_t* Xw) {
+__global__ void k_gather(const uint32_t* idx, uint64_t n, const uint64_t* issue, const uint64_t* retire, GCopy G) {
   uint64_t p = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
   if (p >= n) return;
   uint32_t i = idx[p];
-  put_rec(Y, D, Xw, p, issue[i], retire[i]);
+  put_rec(G, p, issue[i], retire[i], 0);
 }
 
 __global__ void k_set_u32(uint32_t* p, uint32_t v) { *p = v; }
@@ -550,7 +571,7 @@ __global__ void __launch_bounds__(HW * 32) k_job_hist(photon_timing t, JobMap jm
 }
 
 __global__ void __launch_bounds__(256, 3) k_job_scatter(photon_timing t, JobMap jm, uint64_t n_jobs, uint32_t* off,
-                                                     uint64_t* Y, uint32_t* D, uint64_t* Xw, DevErr* err) {
+                                                     GCopy G, DevErr* err) {
   __shared__ uint32_t run[8][kSmemBins];
   const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
   const uint32_t B = t.n_bb;
@@ -584,6 +605,7 @@ __global__ void __launch_bounds__(256, 3) k_job_scatter(photon_timing t, JobMap 
       }
     };
     load(cs, d, x, y);
+    const uint64_t kbase = a < e ? t.retire[a] : 0;  // the kernel's first retire: the copy's time base
     // retire[i - 1] of lane 0 in slot 0: the previous tile's last record (the job's first tile: one load)
     uint64_t carry = lane == 0 && cs > a && cs < ce ? t.retire[cs - 1] : 0;
     for (uint64_t i0 = cs; i0 < ce; i0 += 32 * TS) {
@@ -620,7 +642,7 @@ __global__ void __launch_bounds__(256, 3) k_job_scatter(photon_timing t, JobMap 
           if (dd != kNone && lane == lead) base = atomicAdd(&off[hb + (uint64_t)dd * nj + jl], (uint32_t)__popc(peers));
           base = __shfl_sync(0xffffffffu, base, lead);
         }
-        if (dd != kNone) put_rec(Y, D, Xw, base + __popc(peers & lt), x[u], y[u]);
+        if (dd != kNone) put_rec(G, base + __popc(peers & lt), x[u], y[u], kbase);
         __syncwarp();
       }
 #pragma unroll
@@ -748,11 +770,12 @@ __device__ __forceinline__ Sums shfl_xor_sums(const Sums& s, int m) {
 }
 
 struct WinArgs {
-  const uint64_t* X;  // issue times (D == nullptr), else the escape side array of the grouped copy
-  const uint64_t* Y;  // retire times
-  const uint32_t* D;  // grouped copy: durations (kDurEsc: issue in X), or nullptr
+  const uint64_t* X;  // raw streams (N1): issue times
+  const uint64_t* Y;  // raw streams (N1): retire times
+  const uint32_t* D;  // non-null: the positions are the grouped copy G (relative times), X / Y unused
+  GCopy G;
   const uint64_t* gstart;
-  const uint32_t* G;
+  const uint32_t* Gn;     // number of groups
   const uint64_t* list;   // compact run-major run list (k_runs_*)
   const uint32_t* total;  // its length
   uint32_t* ticket;       // global ticket counter (zeroed)
@@ -763,11 +786,12 @@ struct WinArgs {
   int64_t lim;     // fast path: shifted times must lie in (-lim, lim) (n * lim^2 < 2^61: int64 sums are exact)
 };
 
-// issue time of position q whose retire time is y
-__device__ __forceinline__ uint64_t win_x(const WinArgs& a, int64_t q, uint64_t y) {
-  if (!a.D) return __ldg(a.X + q);
-  const uint32_t d = __ldg(a.D + q);
-  return d != kDurEsc ? y - d : __ldg(a.X + q);
+// retire / issue time of position q (relative to the kernel's first retire for the grouped copy)
+__device__ __forceinline__ int64_t win_y(const WinArgs& a, int64_t q) {
+  return a.D ? g_y(a.G, q) : (int64_t)__ldg(a.Y + q);
+}
+__device__ __forceinline__ int64_t win_x(const WinArgs& a, int64_t q, int64_t y) {
+  return a.D ? g_x(a.G, q, y) : (int64_t)__ldg(a.X + q);
 }
 
 __device__ __forceinline__ void sums_sub(Sums& a, const Sums& b) {
@@ -842,30 +866,38 @@ __device__ bool window_run_fast(const WinArgs& a, uint32_t g, int64_t gs, int64_
                                 FSums* wpart, unsigned long long* best) {
   const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
   const int64_t n = a.n, base0 = P0 - 2 * n, span = P1 - base0;
-  const int64_t c = (int64_t)__ldg(a.Y + (base0 > gs ? base0 : gs));
+  const int64_t c = win_y(a, base0 > gs ? base0 : gs);
   bool ok = true;
   constexpr int FU = 8;  // loads in flight per thread (the fill is latency-bound otherwise)
   for (int64_t i0 = 0; i0 < span; i0 += WT * FU) {
-    uint64_t xv[FU], yv[FU];
+    uint32_t yv[FU], dv[FU];
 #pragma unroll
     for (int u = 0; u < FU; ++u) {
       const int64_t i = i0 + u * WT + tid, q = base0 + i;
       const bool in = i < span && q >= gs;
-      yv[u] = in ? __ldg(a.Y + q) : (uint64_t)c;
-      xv[u] = in ? (a.D ? (uint64_t)__ldg(a.D + q) : __ldg(a.X + q)) : (uint64_t)c;
-    }
-    if (a.D) {
-#pragma unroll
-      for (int u = 0; u < FU; ++u) {  // durations -> issue times (escaped ones from the side array)
-        const int64_t i = i0 + u * WT + tid, q = base0 + i;
-        if (i < span && q >= gs) xv[u] = xv[u] != kDurEsc ? yv[u] - xv[u] : __ldg(a.X + q);
+      if (a.D) {
+        yv[u] = in ? __ldg(a.G.Y32 + q) : 0u;
+        dv[u] = in ? __ldg(a.G.D + q) : 0u;
+      } else {
+        yv[u] = dv[u] = 0u;
       }
     }
 #pragma unroll
     for (int u = 0; u < FU; ++u) {
-      const int64_t i = i0 + u * WT + tid;
-      const int64_t x = (int64_t)xv[u] - c, y = (int64_t)yv[u] - c;  // positions < gs: (0, 0)
-      ok &= x > -a.lim && x < a.lim && y > -a.lim && y < a.lim;
+      const int64_t i = i0 + u * WT + tid, q = base0 + i;
+      int64_t x = c, y = c;  // positions < gs: (0, 0) after the shift
+      if (i < span && q >= gs) {
+        if (a.D) {
+          y = yv[u] != kDurEsc ? (int64_t)yv[u] : __ldg(a.G.Yw + q);
+          x = dv[u] != kDurEsc ? y - (int64_t)dv[u] : __ldg(a.G.Xw + q);
+        } else {
+          y = (int64_t)__ldg(a.Y + q);
+          x = (int64_t)__ldg(a.X + q);
+        }
+      }
+      x -= c;
+      y -= c;
+      ok &= x > -a.lim && y < a.lim;  // x <= y (validated), so both lie in (-lim, lim)
       if (i < span) ring[i] = make_int2((int)x, (int)y);
     }
   }
@@ -977,8 +1009,8 @@ __global__ void __launch_bounds__(WT, 2) k_window(WinArgs a) {
       const int64_t P0 = gs + 2 * n - 1 + (int64_t)r * RUN;
       const int64_t P1 = P0 + RUN < ge ? P0 + RUN : ge;
       if (a.ring && window_run_fast(a, g, gs, P0, P1, ring, fpart, &fbest)) continue;
-      auto X = [&](int64_t q) -> int64_t { return q >= gs ? (int64_t)win_x(a, q, __ldg(a.Y + q)) : 0; };
-      auto Yv = [&](int64_t q) -> int64_t { return q >= gs ? (int64_t)__ldg(a.Y + q) : 0; };
+      auto X = [&](int64_t q) -> int64_t { return q >= gs ? win_x(a, q, win_y(a, q)) : 0; };
+      auto Yv = [&](int64_t q) -> int64_t { return q >= gs ? win_y(a, q) : 0; };
       // base: windows ending at P0-1 ([P0-n, P0-1] and [P0-2n, P0-1]); positions < gs contribute 0
       Sums s;
       sums_zero(s);
@@ -1143,8 +1175,8 @@ __device__ uint64_t locate_record(const photon_timing& t, const JobMap& jm, cons
 }
 
 // group g -> (k, b): mode 0 (radix path) g = b*K + k; 1 (job path, B <= 256) g = k*B + b; 2 (compact) gkb[g]
-__global__ void k_finish(photon_timing t, JobMap jm, const uint32_t* cells, const uint32_t* idx, const uint64_t* Y,
-                         const uint32_t* D, const uint64_t* Xw, const uint32_t* G, const uint64_t* gfirst,
+__global__ void k_finish(photon_timing t, JobMap jm, const uint32_t* cells, const uint32_t* idx, GCopy C,
+                         const uint32_t* G, const uint64_t* gfirst,
                          const uint64_t* gstart, uint32_t n, int mode, const uint64_t* gkb, int64_t* first_stable,
                          uint64_t* dur) {
   const uint32_t lane = threadIdx.x & 31, ng = *G, K = t.n_kernels, B = t.n_bb;
@@ -1157,7 +1189,10 @@ __global__ void k_finish(photon_timing t, JobMap jm, const uint32_t* cells, cons
     else if (mode == 1) { k = g / B; b = g % B; }
     else { k = gkb[g] >> 16; b = gkb[g] & 0xFFFFu; }
     uint64_t s = 0;
-    for (uint64_t i = q + 1 - n + lane; i <= q; i += 32) s += D[i] != kDurEsc ? D[i] : Y[i] - Xw[i];
+    for (uint64_t i = q + 1 - n + lane; i <= q; i += 32) {
+      const uint32_t d = C.D[i];
+      s += d != kDurEsc ? (uint64_t)d : (uint64_t)(g_y(C, i) - C.Xw[i]);
+    }
     for (int o = 16; o > 0; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
     const uint64_t pos = mode == 0 ? idx[q] - t.kernel_rec_off[k]
                                    : locate_record(t, jm, cells, (uint32_t)k, (uint32_t)b, q, gstart[g]);
@@ -1326,7 +1361,7 @@ struct Layout {
                      // 0: LSD radix sort of composite keys (larger B)
   uint64_t* key0; uint64_t* key1;  // radix path only
   uint32_t* val0; uint32_t* val1;  // val0 = original record index of each sorted position (all paths)
-  uint64_t* Y; uint32_t* D; uint64_t* Xw;  // the grouped copy: retire, duration (kDurEsc: issue in Xw)
+  GCopy G;  // the grouped copy (8 B/record + escape side arrays)
   uint32_t* hist; uint32_t* bsum; uint32_t* misc;  // misc[0] = G, [1] = max runs, [2] = ticket, [4] = scan total
   uint64_t* gstart;  // [gcap+1]
   uint32_t* nruns;   // [gcap]
@@ -1355,7 +1390,8 @@ Layout make_layout(const photon_timing& t, void* base) {
     L.key0 = c.take<uint64_t>(R); L.key1 = c.take<uint64_t>(R);
     L.val0 = c.take<uint32_t>(R); L.val1 = c.take<uint32_t>(R);
   }
-  L.Y = c.take<uint64_t>(R); L.D = c.take<uint32_t>(R); L.Xw = c.take<uint64_t>(R);
+  L.G.Y32 = c.take<uint32_t>(R); L.G.D = c.take<uint32_t>(R); L.G.Yw = c.take<int64_t>(R);
+  L.G.Xw = c.take<int64_t>(R);
   // histogram cells: B * jobs; compact: sum_k B_k * jobs_k <= 2R + ... whenever no kernel has more than 2048
   // distinct BB ids (ECAPACITY otherwise)
   L.hn = L.mode == 1 ? (uint64_t)t.n_bb * L.n_jobs : (L.mode == 2 ? 2 * R + 65536 : (uint64_t)RNB * L.n_tiles);
@@ -1469,7 +1505,7 @@ cudaError_t launch_stable(const photon_timing& t, const uint64_t* kbb, photon_st
       // group starts first: kernels with > 256 local ids use the scanned cells as running offsets in the scatter
       note_launch(), k_job_gstart<<<(unsigned)umin64(ceil_div(L.gcap + 1, 256), (uint64_t)num_sms * 8), 256, 0, s>>>(
           L.hist, jm, L.goff, L.gkb, K, B, R, (uint64_t)B * L.n_jobs, L.gstart, L.misc + 0);
-      note_launch(), k_job_scatter<<<gj, 256, 0, s>>>(t, jm, L.n_jobs, L.hist, L.Y, L.D, L.Xw, err);
+      note_launch(), k_job_scatter<<<gj, 256, 0, s>>>(t, jm, L.n_jobs, L.hist, L.G, err);
       idx = nullptr;
       jmf = jm;
     } else {
@@ -1491,7 +1527,7 @@ cudaError_t launch_stable(const photon_timing& t, const uint64_t* kbb, photon_st
         uint32_t* tv = vin; vin = vout; vout = tv;
       }
       unsigned gR = (unsigned)ceil_div(R + 1, 256);
-      note_launch(), k_gather<<<gR, 256, 0, s>>>(vin, R, t.issue, t.retire, L.Y, L.D, L.Xw);
+      note_launch(), k_gather<<<gR, 256, 0, s>>>(vin, R, t.issue, t.retire, L.G);
       note_launch(), k_fill_gstart<<<gR, 256, 0, s>>>(kin, R, L.gcap, L.gstart);
       note_launch(), k_set_u32<<<1, 1, 0, s>>>(L.misc + 0, (uint32_t)L.gcap);
       idx = vin;
@@ -1500,13 +1536,13 @@ cudaError_t launch_stable(const photon_timing& t, const uint64_t* kbb, photon_st
     note_launch(), k_work_count<<<(unsigned)umin64(ceil_div(L.gcap, 256), (uint64_t)num_sms * 4), 256, 0, s>>>(
         L.gstart, L.misc + 0, 2 * p.window_n, L.nruns, L.gfirst, L.misc + 1);
     WinArgs wa{};
-    wa.X = L.Xw; wa.Y = L.Y; wa.D = L.D; wa.gstart = L.gstart; wa.G = L.misc + 0;
+    wa.X = nullptr; wa.Y = nullptr; wa.D = L.G.D; wa.G = L.G; wa.gstart = L.gstart; wa.Gn = L.misc + 0;
     wa.n = p.window_n; wa.dnum = p.delta_num; wa.dden = p.delta_den; wa.gfirst = L.gfirst;
     build_runlist(L.rl, L.misc + 0, L.nruns, L.misc, L.gcap, num_sms, wa, s);
     window_launch(wa, num_sms, s);
     // 5. outputs
     note_launch(), k_finish<<<(unsigned)umin64(ceil_div(L.gcap * 32, 256), (uint64_t)num_sms * 8), 256, 0, s>>>(
-        t, jmf, L.hist, idx, L.Y, L.D, L.Xw, L.misc + 0, L.gfirst, L.gstart, p.window_n, L.mode, L.gkb, first_stable,
+        t, jmf, L.hist, idx, L.G, L.misc + 0, L.gfirst, L.gstart, p.window_n, L.mode, L.gkb, first_stable,
         dur);
     unsigned gk = (unsigned)umin64(K, (uint64_t)num_sms * 8);
     note_launch(), k_switch<<<gk ? gk : 1, 256, 0, s>>>(first_stable, kbb, K, B, p.rate_num, p.rate_den, switch_at);
@@ -1547,7 +1583,7 @@ cudaError_t launch_warp_stable(const photon_timing& t, const uint8_t* ok, uint32
   note_launch(), k_warp_runs<<<(unsigned)ceil_div(K, 256), 256, 0, s>>>(t.kernel_rec_off, K, t.n_records, ok, 2 * n,
                                                                        nruns, gfirst, misc);
   WinArgs wa{};
-  wa.X = t.issue; wa.Y = t.retire; wa.D = nullptr; wa.gstart = t.kernel_rec_off; wa.G = misc + 0;
+  wa.X = t.issue; wa.Y = t.retire; wa.D = nullptr; wa.gstart = t.kernel_rec_off; wa.Gn = misc + 0;
   wa.n = n; wa.dnum = dnum; wa.dden = dden; wa.gfirst = gfirst;
   build_runlist(rl, misc + 0, nruns, misc, K, num_sms, wa, s);
   window_launch(wa, num_sms, s);
