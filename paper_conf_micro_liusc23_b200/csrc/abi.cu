@@ -9,6 +9,7 @@
 #include <vector>
 
 #include "internal.h"
+#include <nvtx3/nvToolsExt.h>
 
 using namespace photon;
 
@@ -25,6 +26,12 @@ struct photon_ctx {
 };
 
 namespace {
+
+// one NVTX range per C-ABI call (header-only NVTX3: no cost unless a tool such as nsys / ncu is attached)
+struct NvtxRange {
+  explicit NvtxRange(const char* name) { nvtxRangePushA(name); }
+  ~NvtxRange() { nvtxRangePop(); }
+};
 
 struct ProfScope {
   photon_ctx* c;
@@ -285,6 +292,7 @@ extern "C" {
 int photon_abi_version(void) { return PHOTON_ABI_VERSION; }
 
 int photon_create(photon_ctx** out, int cuda_device) {
+  NvtxRange nvtx_("photon_create");
   if (!out) return PHOTON_EINVAL;
   *out = nullptr;
   int n = 0;
@@ -312,6 +320,7 @@ void photon_destroy(photon_ctx* ctx) {
 }
 
 int photon_profile(photon_ctx* ctx, int enable) {
+  NvtxRange nvtx_("photon_profile");
   if (!ctx) return PHOTON_EINVAL;
   ctx->prof = enable != 0;
   for (auto& u : ctx->used) u = 0;
@@ -319,6 +328,7 @@ int photon_profile(photon_ctx* ctx, int enable) {
 }
 
 int photon_profile_read(photon_ctx* ctx, void* stream, double* ms, uint64_t* launches) {
+  NvtxRange nvtx_("photon_profile_read");
   if (!ctx || !ms || !launches) return PHOTON_EINVAL;
   CK(cudaStreamSynchronize((cudaStream_t)stream), "sync");
   for (int sec = 0; sec < PHOTON_PROF_N; ++sec) {
@@ -352,11 +362,13 @@ static int read_latch(photon_ctx* ctx, const void* ws, void* stream, int64_t* ba
 }
 
 int photon_check(photon_ctx* ctx, void* stream, int64_t* bad_index) {
+  NvtxRange nvtx_("photon_check");
   if (!ctx) return PHOTON_EINVAL;
   return read_latch(ctx, ctx->last_ws, stream, bad_index);
 }
 
 int photon_ws_status(photon_ctx* ctx, const void* ws, void* stream, int64_t* bad_index) {
+  NvtxRange nvtx_("photon_ws_status");
   if (!ctx) return PHOTON_EINVAL;
   return read_latch(ctx, ws, stream, bad_index);
 }
@@ -366,6 +378,7 @@ size_t photon_bbv_workspace_bytes(const photon_trace* t) { return t ? bbv_layout
 
 int photon_bbv_build(photon_ctx* ctx, const photon_trace* t, void* ws, size_t ws_bytes, uint32_t* warp_bbv16,
                      uint64_t* warp_insts, uint64_t* kernel_bb_insts, void* stream) {
+  NvtxRange nvtx_("photon_bbv_build");
   if (!ctx) return PHOTON_EINVAL;
   int rc = check_trace(ctx, t);
   if (rc) return rc;
@@ -398,11 +411,13 @@ size_t photon_group_workspace_bytes(const photon_trace* t, uint64_t hint) {
 
 int photon_warp_group(photon_ctx* ctx, const photon_trace* t, const uint32_t* warp_bbv16, void* ws, size_t ws_bytes,
                       photon_types* out, void* stream) {
+  NvtxRange nvtx_("photon_warp_group");
   return photon_warp_group2(ctx, t, warp_bbv16, ws, ws_bytes, out, stream, stream);
 }
 
 int photon_warp_group2(photon_ctx* ctx, const photon_trace* t, const uint32_t* warp_bbv16, void* ws, size_t ws_bytes,
                        photon_types* out, void* stream, void* remap_stream) {
+  NvtxRange nvtx_("photon_warp_group2");
   if (!ctx) return PHOTON_EINVAL;
   int rc = check_trace(ctx, t);
   if (rc) return rc;
@@ -453,6 +468,7 @@ int photon_warp_group2(photon_ctx* ctx, const photon_trace* t, const uint32_t* w
 }
 
 int photon_types_total(photon_ctx* ctx, const photon_types* types, uint32_t K, uint64_t* total, void* stream) {
+  NvtxRange nvtx_("photon_types_total");
   if (!ctx || !types || !total || !types->kernel_type_off) return PHOTON_EINVAL;
   CK(cudaStreamSynchronize((cudaStream_t)stream), "sync");
   CK(cudaMemcpy(total, types->kernel_type_off + K, 8, cudaMemcpyDeviceToHost), "read total");
@@ -467,6 +483,7 @@ size_t photon_match_workspace_bytes(uint32_t K, uint64_t T, uint64_t pair_cap) {
 int photon_kernel_match(photon_ctx* ctx, uint32_t K, const photon_types* types, const uint64_t* warps_total,
                         photon_match_params params, void* ws, size_t ws_bytes, int64_t* match, double* match_dist,
                         void* stream) {
+  NvtxRange nvtx_("photon_kernel_match");
   if (!ctx) return PHOTON_EINVAL;
   if (!types || !types->kernel_type_off || !types->type_key || !types->type_count || !warps_total || !match || !ws)
     return fail(ctx, PHOTON_EINVAL, "NULL argument");
@@ -539,6 +556,7 @@ size_t photon_group_full_workspace_bytes(const photon_trace* t) {
 
 int photon_warp_group_full(photon_ctx* ctx, const photon_trace* t, const uint32_t* warp_bbv16, void* ws,
                            size_t ws_bytes, photon_types* out, void* stream) {
+  NvtxRange nvtx_("photon_warp_group_full");
   if (!ctx) return PHOTON_EINVAL;
   int rc = check_trace(ctx, t);
   if (rc) return rc;
@@ -572,6 +590,7 @@ size_t photon_ingest_workspace_bytes(uint64_t n, uint64_t W) {
 
 int photon_ingest_tagged(photon_ctx* ctx, uint64_t n, uint64_t W, const uint32_t* warp, const uint16_t* bb, void* ws,
                          size_t ws_bytes, uint16_t* bb_out, uint64_t* warp_event_off, void* stream) {
+  NvtxRange nvtx_("photon_ingest_tagged");
   if (!ctx) return PHOTON_EINVAL;
   if ((n && (!warp || !bb || !bb_out)) || !warp_event_off || !ws) return fail(ctx, PHOTON_EINVAL, "NULL argument");
   if (W >= (1ull << 32) || n >= (1ull << 32)) return fail(ctx, PHOTON_EINVAL, "n and n_warps must be < 2^32");
@@ -600,6 +619,7 @@ size_t photon_pool_export_workspace_bytes(uint32_t K) {
 int photon_pool_export(photon_ctx* ctx, uint32_t K, const photon_types* types, const uint64_t* warps_total,
                        const int64_t* match, void* ws, size_t ws_bytes, photon_types* pool, uint64_t* pool_wt,
                        uint32_t* pool_kid, uint32_t* n_pool, void* stream) {
+  NvtxRange nvtx_("photon_pool_export");
   if (!ctx) return PHOTON_EINVAL;
   if (!types || !types->kernel_type_off || !types->type_key || !types->type_count || !warps_total || !match ||
       !pool || !pool->kernel_type_off || !pool->type_key || !pool->type_count || !pool_wt || !pool_kid || !n_pool ||
@@ -646,6 +666,7 @@ int photon_kernel_match_pooled(photon_ctx* ctx, uint32_t Kp, const photon_types*
                                uint64_t Tp, uint32_t K, const photon_types* types, const uint64_t* warps_total,
                                uint64_t T, photon_match_params params, void* ws, size_t ws_bytes, int64_t* match,
                                double* match_dist, void* stream) {
+  NvtxRange nvtx_("photon_kernel_match_pooled");
   if (!ctx) return PHOTON_EINVAL;
   if (!pool || !pool->kernel_type_off || (Kp && (!pool->type_key || !pool->type_count || !pool_wt)) || !types ||
       !types->kernel_type_off || !types->type_key || !types->type_count || !warps_total || !match || !ws)
@@ -671,6 +692,7 @@ int photon_kernel_match_pooled(photon_ctx* ctx, uint32_t Kp, const photon_types*
 
 int photon_match_stats(photon_ctx* ctx, uint32_t K, uint64_t T, const void* ws, size_t ws_bytes, uint64_t* stats,
                        void* stream) {
+  NvtxRange nvtx_("photon_match_stats");
   if (!ctx || !ws || !stats) return PHOTON_EINVAL;
   MatchLayout m = match_layout_fit(K, T, (void*)ws, ws_bytes);
   CK(cudaStreamSynchronize((cudaStream_t)stream), "sync");
@@ -689,6 +711,7 @@ int photon_match_stats(photon_ctx* ctx, uint32_t K, uint64_t T, const void* ws, 
 int photon_sig_build(photon_ctx* ctx, uint32_t K, const uint64_t* kto, const uint32_t* type_key,
                      const uint64_t* type_count, uint32_t k_lo, uint32_t k_hi, uint64_t* sig, uint64_t* mass,
                      void* ws, size_t ws_bytes, void* stream) {
+  NvtxRange nvtx_("photon_sig_build");
   if (!ctx) return PHOTON_EINVAL;
   if (!kto || !type_key || !type_count || !sig || !mass || k_hi > K || k_lo > k_hi || !ws)
     return fail(ctx, PHOTON_EINVAL, "bad sig_build arguments");
@@ -705,6 +728,7 @@ int photon_sig_build(photon_ctx* ctx, uint32_t K, const uint64_t* kto, const uin
 int photon_match_scan(photon_ctx* ctx, uint32_t K, const uint64_t* kto, const uint64_t* sig, const uint64_t* mass,
                       const uint64_t* warps_total, photon_match_params params, uint32_t k_lo, uint32_t k_hi, void* ws,
                       size_t ws_bytes, uint64_t* pairs, uint64_t pair_capacity, uint64_t* n_pairs, void* stream) {
+  NvtxRange nvtx_("photon_match_scan");
   if (!ctx) return PHOTON_EINVAL;
   if (!kto || !sig || !mass || !warps_total || !ws || !pairs || !n_pairs || k_hi > K || k_lo > k_hi || K == 0)
     return fail(ctx, PHOTON_EINVAL, "bad match_scan arguments");
@@ -730,6 +754,7 @@ int photon_match_resolve(photon_ctx* ctx, uint32_t K, const uint64_t* kto, const
                          const uint64_t* warps_total, photon_match_params params, const uint64_t* pairs,
                          uint64_t n_pairs, void* ws, size_t ws_bytes, int64_t* match, double* match_dist,
                          void* stream) {
+  NvtxRange nvtx_("photon_match_resolve");
   if (!ctx) return PHOTON_EINVAL;
   if (!kto || !sig || !mass || !warps_total || !ws || (n_pairs && !pairs) || !match || K == 0)
     return fail(ctx, PHOTON_EINVAL, "bad match_resolve arguments");
@@ -757,6 +782,7 @@ size_t photon_stable_workspace_bytes(const photon_timing* t) { return t ? stable
 
 int photon_bb_stable(photon_ctx* ctx, const photon_timing* t, const uint64_t* kbb, photon_stable_params p, void* ws,
                      size_t ws_bytes, int64_t* first_stable, uint64_t* dur, int64_t* switch_at, void* stream) {
+  NvtxRange nvtx_("photon_bb_stable");
   if (!ctx) return PHOTON_EINVAL;
   if (!t || !t->kernel_rec_off || (t->n_records && (!t->bb || !t->issue || !t->retire)) || !kbb || !first_stable ||
       !switch_at || !ws)
@@ -788,6 +814,7 @@ size_t photon_warp_stable_workspace_bytes(const photon_timing* t) {
 
 int photon_warp_stable(photon_ctx* ctx, const photon_timing* t, const uint8_t* ok, photon_warp_stable_params p,
                        void* ws, size_t ws_bytes, int64_t* switch_at, uint64_t* dur, void* stream) {
+  NvtxRange nvtx_("photon_warp_stable");
   if (!ctx) return PHOTON_EINVAL;
   if (!t || !t->kernel_rec_off || (t->n_records && (!t->issue || !t->retire)) || !switch_at || !ws)
     return fail(ctx, PHOTON_EINVAL, "NULL argument");
@@ -814,6 +841,7 @@ int photon_warp_stable(photon_ctx* ctx, const photon_timing* t, const uint8_t* o
 int photon_kernel_predict(photon_ctx* ctx, uint32_t K, const int64_t* match, const uint64_t* mass,
                           const uint64_t* full_insts, const uint64_t* full_cycles, void* ws, size_t ws_bytes,
                           uint64_t* pred_insts, uint64_t* pred_cycles, void* stream) {
+  NvtxRange nvtx_("photon_kernel_predict");
   if (!ctx) return PHOTON_EINVAL;
   if (!match || !mass || !full_insts || !full_cycles || !pred_insts || !pred_cycles || !ws || K == 0)
     return fail(ctx, PHOTON_EINVAL, "bad kernel_predict arguments");
@@ -838,6 +866,7 @@ size_t photon_bb_predict_workspace_bytes(const photon_trace* t) {
 
 int photon_bb_predict(photon_ctx* ctx, const photon_trace* t, const int64_t* first_stable, const uint64_t* dur,
                       void* ws, size_t ws_bytes, uint64_t* pred, uint32_t* unpred, void* stream) {
+  NvtxRange nvtx_("photon_bb_predict");
   if (!ctx) return PHOTON_EINVAL;
   int rc = check_trace(ctx, t);
   if (rc) return rc;
@@ -865,6 +894,7 @@ int photon_bb_predict(photon_ctx* ctx, const photon_trace* t, const int64_t* fir
 int photon_types_export(photon_ctx* ctx, uint32_t K_local, const photon_types* local, uint32_t kernel_base,
                         uint64_t warp_base, photon_type_row* rows, uint64_t row_capacity, uint64_t* n_rows,
                         void* stream) {
+  NvtxRange nvtx_("photon_types_export");
   if (!ctx) return PHOTON_EINVAL;
   if (!local || !rows || K_local == 0 || row_capacity == 0) return fail(ctx, PHOTON_EINVAL, "bad export arguments");
   CK(cudaSetDevice(ctx->device), "cudaSetDevice");
@@ -877,6 +907,7 @@ size_t photon_merge_workspace_bytes(uint64_t n_rows, uint32_t K) { return merge_
 
 int photon_types_merge(photon_ctx* ctx, const photon_type_row* rows, uint64_t n_rows, uint32_t K,
                        const uint64_t* kernel_warps, void* ws, size_t ws_bytes, photon_types* global, void* stream) {
+  NvtxRange nvtx_("photon_types_merge");
   if (!ctx) return PHOTON_EINVAL;
   if ((n_rows && !rows) || K == 0 || !kernel_warps || !ws || !global || !global->kernel_type_off ||
       !global->type_key || !global->type_count || !global->type_first_warp || !global->warp_sampling_ok)
@@ -896,6 +927,7 @@ int photon_types_merge(photon_ctx* ctx, const photon_type_row* rows, uint64_t n_
 int photon_types_remap(photon_ctx* ctx, uint32_t K_local, uint64_t W_local, const uint64_t* kernel_warp_off_local,
                        const photon_types* local, uint32_t kernel_base, uint64_t n_rows_merged, uint32_t K_global,
                        const void* merge_ws, size_t ws_bytes, uint32_t* warp_type_global, void* stream) {
+  NvtxRange nvtx_("photon_types_remap");
   if (!ctx) return PHOTON_EINVAL;
   if (!local || !kernel_warp_off_local || !merge_ws || !warp_type_global || K_local == 0)
     return fail(ctx, PHOTON_EINVAL, "bad remap arguments");

@@ -256,8 +256,10 @@ __device__ void finalize_fused(const Args3& a, WMisc* wm, uint64_t w0, bool vali
     kd[4] = make_uint4((uint32_t)w, (uint32_t)(w >> 32), k, cnt);  // first warp, kernel, count
   }
   __syncwarp();
-  if (alloc) {  // remember the new entry: two leaders on one slot may leave its hash and id from different entries,
-                // which only costs a miss (every hit is checked against the entry's own key)
+  // remember the new entries: one writer per slot (the lowest allocating lane mapping to it; every hit is checked
+  // against the entry's own key anyway)
+  const unsigned same_slot = __match_any_sync(0xffffffffu, alloc ? cslot : 0xFFFFFFFFu);
+  if (alloc && (int)lane == __ffs(same_slot) - 1) {
     wm->ch[cslot] = h;
     wm->ce[cslot] = (uint32_t)umin64(id, 0xFFFFFFFFull);
   }

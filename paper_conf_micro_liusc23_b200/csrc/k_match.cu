@@ -511,70 +511,56 @@ __global__ void k_pair_bucket(const uint64_t* pairs, uint64_t n_host, const uint
   }
 }
 
-// Fixed point of the launch-order rule: state 1 = representative, 2 = matched.  k decides once all its candidate
-// predecessors have decided (or one of them is a representative).  One CTA; monotone state (races benign).
-// Each kernel keeps a cursor into its candidate list: entries before it are decided non-representatives, so every
-// candidate is examined O(1) times plus once per round it blocks.  State lives in shared memory when K fits.
-template <bool SMEM>
-__global__ void __launch_bounds__(1024) k_resolve_states(uint32_t K, const uint64_t* beg, const uint32_t* cnt,
-                                                         const uint32_t* cand,
-                                                         uint8_t* state, uint32_t* cursor, uint32_t* ulist,
-                                                         uint32_t* flag, uint32_t pool_all) {
-  extern __shared__ uint8_t sstate[];
-  uint8_t* st = SMEM ? sstate : state;
-  for (uint32_t k = threadIdx.x; k < K; k += blockDim.x) {
-    st[k] = 0;
-    cursor[k] = 0;
+// Fixed point of the launch-order rule (small K, one CTA): state 1 = representative, 2 = matched, 0 = undecided.
+// Round-synchronous: every round reads the states of the previous round only (barrier), decides each undecided
+// kernel whose candidates allow it (a representative among them -> matched; none undecided -> representative),
+// and writes the decisions after a second barrier -- no thread reads a state another thread is writing.  The
+// result is the same fixed point (states are monotone); the rounds are at most the longest chain of undecided
+// predecessors.  pool_all: every prior kernel counts, so any candidate decides (matched) at once.
+constexpr uint32_t kResolveSmemK = 4096;
+__global__ void k_pool_all_states(uint32_t K, const uint32_t* cnt, uint8_t* state, uint32_t* flag) {
+  const uint32_t k = blockIdx.x * blockDim.x + threadIdx.x;
+  if (k < K) state[k] = cnt[k] > 0 ? 2 : 1;
+  if (k == 0) flag[0] = 1;
+}  // kernels per thread-owned slice: K <= 4 x 1024
+__global__ void __launch_bounds__(1024) k_resolve_rounds(uint32_t K, const uint64_t* beg, const uint32_t* cnt,
+                                                         const uint32_t* cand, uint8_t* state, uint32_t* flag,
+                                                         uint32_t pool_all) {
+  __shared__ uint8_t st[kResolveSmemK];
+  for (uint32_t k = threadIdx.x; k < K; k += blockDim.x) st[k] = pool_all ? (cnt[k] > 0 ? 2 : 1) : 0;
+  uint32_t rounds = 0;
+  if (!pool_all) {
+    for (;;) {
+      ++rounds;
+      __syncthreads();  // the previous round's decisions are visible
+      uint8_t dec[kResolveSmemK / 1024];
+      int open = 0;
+#pragma unroll
+      for (int j = 0; j < (int)(kResolveSmemK / 1024); ++j) {
+        const uint32_t k = threadIdx.x + j * 1024;
+        dec[j] = 0;
+        if (k >= K || st[k] != 0) continue;
+        const uint64_t o0 = beg[k], o1 = o0 + cnt[k];
+        bool rep = false, und = false;
+        for (uint64_t i = o0; i < o1 && !rep; ++i) {
+          const uint8_t s = st[cand[i]];
+          rep = s == 1;
+          und |= s == 0;
+        }
+        dec[j] = rep ? 2 : (und ? 0 : 1);
+        open |= dec[j] == 0;
+      }
+      const int any_open = __syncthreads_or(open);  // every read of this round is done
+#pragma unroll
+      for (int j = 0; j < (int)(kResolveSmemK / 1024); ++j) {
+        const uint32_t k = threadIdx.x + j * 1024;
+        if (k < K && dec[j] != 0) st[k] = dec[j];
+      }
+      if (!any_open) break;
+    }
   }
   __syncthreads();
-  if (pool_all) {
-    for (uint32_t k = threadIdx.x; k < K; k += blockDim.x) state[k] = cnt[k] > 0 ? 2 : 1;
-    if (threadIdx.x == 0) flag[0] = 1;
-    return;
-  }
-  volatile uint8_t* vs = st;
-  __shared__ uint32_t n_next;
-  uint32_t rounds = 0;
-  uint32_t n = K;           // round 1 visits every kernel; later rounds only the undecided list
-  uint32_t* cur = nullptr;  // current list (nullptr = identity)
-  uint32_t* nxt = ulist;
-  for (;;) {
-    ++rounds;
-    if (threadIdx.x == 0) n_next = 0;
-    __syncthreads();
-    for (uint32_t q = threadIdx.x; q < n; q += blockDim.x) {
-      const uint32_t k = cur ? cur[q] : q;
-      const uint64_t o0 = beg[k], o1 = o0 + cnt[k];
-      uint64_t first_undec = o1;
-      uint8_t res = 1;  // representative unless a candidate is one
-      // batches of 8 independent candidate loads (memory-level parallelism), then their states
-      for (uint64_t i0 = o0 + cursor[k]; i0 < o1 && res == 1; i0 += 8) {
-        uint32_t c8[8];
-#pragma unroll
-        for (int u = 0; u < 8; ++u) c8[u] = (i0 + u < o1) ? cand[i0 + u] : UINT32_MAX;
-#pragma unroll
-        for (int u = 0; u < 8; ++u) {
-          if (c8[u] == UINT32_MAX) break;
-          uint8_t s = vs[c8[u]];
-          if (s == 1) { res = 2; break; }
-          if (s == 0 && first_undec == o1) first_undec = i0 + u;
-        }
-      }
-      if (res == 1 && first_undec < o1) {  // blocked by an undecided predecessor: resume there next round
-        cursor[k] = (uint32_t)(first_undec - o0);
-        nxt[atomicAdd(&n_next, 1u)] = k;
-      } else {
-        vs[k] = res;
-      }
-    }
-    __syncthreads();
-    n = n_next;
-    if (n == 0) break;
-    cur = nxt;  // ping-pong between the two halves of ulist
-    nxt = (cur == ulist) ? ulist + K : ulist;
-  }
-  if (SMEM)
-    for (uint32_t k = threadIdx.x; k < K; k += blockDim.x) state[k] = st[k];
+  for (uint32_t k = threadIdx.x; k < K; k += blockDim.x) state[k] = st[k];
   if (threadIdx.x == 0) flag[0] = rounds;
 }
 
@@ -791,13 +777,11 @@ cudaError_t launch_match_resolve(uint32_t K, const uint64_t* kto, const uint64_t
     note_launch();
     cudaError_t e = cudaLaunchCooperativeKernel((void*)k_resolve_spin, grid, 256, args, 0, s);
     if (e != cudaSuccess) return e;
-  } else if (K <= 40960) {
-    cudaFuncSetAttribute(k_resolve_states<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, 40960);
-    note_launch(), k_resolve_states<true><<<1, 1024, K, s>>>(K, mw.cand_off, ccnt, mw.cand, mw.state, mw.cand_cur, mw.ulist,
-                                                              mw.flag, p.pool_all_prior);
-  } else {
-    note_launch(), k_resolve_states<false><<<1, 1024, 0, s>>>(K, mw.cand_off, ccnt, mw.cand, mw.state, mw.cand_cur,
-                                                               mw.ulist, mw.flag, p.pool_all_prior);
+  } else if (K <= kResolveSmemK) {
+    note_launch(), k_resolve_rounds<<<1, 1024, 0, s>>>(K, mw.cand_off, ccnt, mw.cand, mw.state, mw.flag,
+                                                       p.pool_all_prior);
+  } else {  // pool_all with a large K: every kernel with a candidate is matched
+    note_launch(), k_pool_all_states<<<(unsigned)ceil_div(K, 256), 256, 0, s>>>(K, ccnt, mw.state, mw.flag);
   }
   note_launch(), k_resolve_match<<<(unsigned)ceil_div((uint64_t)K * 32, 256), 256, 0, s>>>(K, mw.cand_off, ccnt, mw.cand, mw.state,
                                                                            p.pool_all_prior, wt, kto, sig, mass,

@@ -1,0 +1,29 @@
+"""compute-sanitizer as a repeatable target: memcheck over every C-ABI entry point on small seeded inputs, and
+racecheck / synccheck over the fused K1 pass, the chain, A5 and N2 (profiles/sanitize_run.py)."""
+import os
+import subprocess
+import sys
+
+import pytest
+
+pytestmark = [pytest.mark.gpu, pytest.mark.slow]
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def _run(tool, what):
+    cmd = ["compute-sanitizer", "--tool", tool, "--error-exitcode", "9", sys.executable,
+           os.path.join(ROOT, "profiles", "sanitize_run.py"), what]
+    p = subprocess.run(cmd, capture_output=True, text=True, timeout=1500, cwd=ROOT)
+    out = p.stdout + p.stderr
+    assert p.returncode == 0, out[-4000:]
+    assert "ERROR SUMMARY: 0 errors" in out or "SUMMARY: 0 hazards displayed (0 errors, 0 warnings)" in out, out[-4000:]
+    assert "sanitize run ok" in out
+
+
+def test_memcheck_all_entry_points():
+    _run("memcheck", "all")
+
+
+@pytest.mark.parametrize("tool", ["racecheck", "synccheck"])
+def test_shared_memory_races_k1_chain(tool):
+    _run(tool, "k1")
