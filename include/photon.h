@@ -294,13 +294,15 @@ PHOTON_API int photon_bb_predict(photon_ctx *ctx, const photon_trace *trace, con
  *   VERIFIED exactly: every member's event multiset is compared with its type's lowest warp's (equal sequences
  *   at once, else by event counts); a hash collision (probability ~2^-128 per pair) latches PHOTON_ERANGE with the
  *   warp index instead of a result.  ERANGE also for bb >= n_bb and bad offsets.
- *   ws >= photon_group_full_workspace_bytes(trace) (grows with W; the error latch is at its start).
+ *   ws >= photon_group_full_workspace_bytes(trace, hint): its hash table holds 2 x hint types (hint 0: 2 x W,
+ *   always enough); the call uses the largest table that fits ws_bytes and latches PHOTON_ECAPACITY if the
+ *   types outgrow it (the caller retries with a larger hint).  The error latch is at the workspace's start.
  * photon_ingest_tagged: n tagged events (warp[i] u32 < n_warps: the analysed-warp index, bb[i] u16), interleaved
  *   in any order (as a functional simulator retires them), to the CSR of photon_trace: bb_out[n] = the events
  *   stably sorted by warp (each warp keeps its events' stream order, L125) and warp_event_off[n_warps + 1].
  *   n < 2^32, n_warps < 2^32 (else EINVAL).  ERANGE (index = event): warp[i] >= n_warps.
  *   ws >= photon_ingest_workspace_bytes(n, n_warps). */
-PHOTON_API size_t photon_group_full_workspace_bytes(const photon_trace *trace);
+PHOTON_API size_t photon_group_full_workspace_bytes(const photon_trace *trace, uint64_t type_capacity_hint);
 PHOTON_API int photon_warp_group_full(photon_ctx *ctx, const photon_trace *trace, const uint32_t *warp_bbv16 /*[W][16]*/,
                                       void *ws, size_t ws_bytes, photon_types *out, void *stream);
 PHOTON_API size_t photon_ingest_workspace_bytes(uint64_t n_events, uint64_t n_warps);

@@ -102,7 +102,7 @@ _SIGS = [
     ("photon_bb_predict_workspace_bytes", c_size_t, [POINTER(Trace)]),
     ("photon_bb_predict", c_int, [c_void_p, POINTER(Trace), c_void_p, c_void_p, c_void_p, c_size_t, c_void_p,
                                   c_void_p, c_void_p]),
-    ("photon_group_full_workspace_bytes", c_size_t, [POINTER(Trace)]),
+    ("photon_group_full_workspace_bytes", c_size_t, [POINTER(Trace), c_uint64]),
     ("photon_warp_group_full", c_int, [c_void_p, POINTER(Trace), c_void_p, c_void_p, c_size_t, POINTER(Types),
                                        c_void_p]),
     ("photon_ingest_workspace_bytes", c_size_t, [c_uint64, c_uint64]),

@@ -289,15 +289,29 @@ class Photon:
         if warp_bbv16 is None:
             warp_bbv16 = self.photon_bbv_build(t, bbv16=True, insts=False, stream=stream, check=check)["warp_bbv16"]
         ct = t.c()
-        ws = self.workspace("group_full", self.L.photon_group_full_workspace_bytes(ctypes.byref(ct)))
         cap = max(t.n_warps, 1)
         ty = out if self._types_fit(out, t.n_kernels, t.n_warps, cap) else self.alloc_types(t.n_kernels, t.n_warps, cap)
-        self._rc(self.L.photon_warp_group_full(self.ctx, ctypes.byref(ct), warp_bbv16.data_ptr(), ws.data_ptr(),
-                                               ws.numel(), ctypes.byref(self.types_c(ty)), self.stream_ptr(stream)))
-        if check:
-            self.check(ws, stream)
-        ty["_ws"] = ws
-        return ty
+        # the hash table is sized from the types a checked call found before (a table for every warp otherwise)
+        key = ("full", t.n_kernels, t.n_warps)
+        hint = self._hint.get(key, 0)
+        for _ in range(8):
+            ws = self.workspace("group_full", self.L.photon_group_full_workspace_bytes(ctypes.byref(ct), hint))
+            self._rc(self.L.photon_warp_group_full(self.ctx, ctypes.byref(ct), warp_bbv16.data_ptr(), ws.data_ptr(),
+                                                   ws.numel(), ctypes.byref(self.types_c(ty)),
+                                                   self.stream_ptr(stream)))
+            ty["_ws"] = ws
+            if not check:
+                return ty
+            rc, bad = self.ws_status(ws, stream)
+            if rc == _lib.ECAPACITY and hint:
+                hint = 0  # the full-size table cannot overflow
+                continue
+            if rc != 0:
+                raise PhotonError(rc, self.L.photon_last_error(self.ctx).decode(), bad)
+            if key not in self._hint:
+                self._hint[key] = max(2 * self.photon_types_total(ty, t.n_kernels, stream), 512)
+            return ty
+        raise PhotonError(_lib.ECAPACITY, "full-BBV type table kept overflowing")
 
     def photon_ingest_tagged(self, warp, bb, n_warps: int, stream=None, check: bool = True) -> dict:
         """Interleaved (warp, bb) tagged events -> CSR by warp (stable): dict(bb, warp_event_off)."""

@@ -528,7 +528,14 @@ struct FullLayout {
   HtWs h;
   size_t bytes;
 };
-FullLayout full_layout(const photon_trace* t, void* base) {
+// the hash table: a power of two >= 2 x hint (>= 1024), or >= 2W without a hint (every warp its own type)
+uint64_t full_ht_cap(const photon_trace* t, uint64_t hint) {
+  const uint64_t h = hint ? (hint < t->n_warps ? hint : t->n_warps) : t->n_warps;
+  uint64_t cap = 1024;
+  while (cap < 2 * h) cap <<= 1;
+  return cap;
+}
+FullLayout full_layout(const photon_trace* t, void* base, uint64_t cap = 0) {
   Carver c(base);
   FullLayout L;
   const uint64_t W = t->n_warps + 1;
@@ -541,17 +548,16 @@ FullLayout full_layout(const photon_trace* t, void* base) {
   L.f.wslot = c.take<uint32_t>(W);
   L.f.nlist = c.take<uint32_t>(4);
   L.f.htab = c.take<ulonglong2>((uint64_t)t->n_bb + 1);
-  uint64_t cap = 1024;
-  while (cap < 2 * t->n_warps) cap <<= 1;  // groups <= W: load factor <= 1/2
+  if (!cap) cap = full_ht_cap(t, 0);
   carve_ht(c, cap, t->n_kernels, L.h);
   L.bytes = c.off + 256;
   return L;
 }
 }  // namespace
 
-size_t photon_group_full_workspace_bytes(const photon_trace* t) {
+size_t photon_group_full_workspace_bytes(const photon_trace* t, uint64_t type_capacity_hint) {
   if (!t) return 0;
-  return full_layout(t, nullptr).bytes;
+  return full_layout(t, nullptr, full_ht_cap(t, type_capacity_hint)).bytes;
 }
 
 int photon_warp_group_full(photon_ctx* ctx, const photon_trace* t, const uint32_t* warp_bbv16, void* ws,
@@ -566,9 +572,13 @@ int photon_warp_group_full(photon_ctx* ctx, const photon_trace* t, const uint32_
   if (t->n_warps >= (1ull << 32)) return fail(ctx, PHOTON_EINVAL, "n_warps must be < 2^32");
   if (!aligned(warp_bbv16, 16)) return fail(ctx, PHOTON_EINVAL, "warp_bbv16 must be 16-byte aligned");
   if (!aligned(out->type_key, 16)) return fail(ctx, PHOTON_EINVAL, "type_key must be 16-byte aligned");
-  const size_t need = photon_group_full_workspace_bytes(t);
+  // the largest table that fits the workspace (a hint-sized workspace gives a small table; ECAPACITY if it fills)
+  const size_t need = photon_group_full_workspace_bytes(t, 1);
   if (ws_bytes < need) return fail(ctx, PHOTON_EWORKSPACE, "workspace %zu < %zu bytes", ws_bytes, need);
-  FullLayout L = full_layout(t, ws);
+  uint64_t cap = 1024;
+  const uint64_t cap_max = full_ht_cap(t, 0);
+  while (cap < cap_max && full_layout(t, nullptr, cap * 2).bytes <= ws_bytes) cap <<= 1;
+  FullLayout L = full_layout(t, ws, cap);
   cudaStream_t s = (cudaStream_t)stream;
   CK(cudaSetDevice(ctx->device), "cudaSetDevice");
   ctx->last_ws = ws;

@@ -316,3 +316,22 @@ def test_chain_cuda_graph_replay_matches_oracle(ph, cfg):
     assert np.array_equal(_np(r["warp_type"], np.uint32), ref["warp_type"])
     assert np.array_equal(_np(r["warp_sampling_ok"], np.uint8), ref["warp_sampling_ok"])
     assert np.array_equal(_np(r["match"], np.int64), ref["match"])
+
+
+def test_group_full_table_hint_overflow_retry(ph):
+    # N2 sizes its hash table from the types a checked call found before on a trace of the same shape; a later
+    # trace of that shape with many more types overflows the small table (ECAPACITY) and the checked call retries
+    # with the full-size table -- both results equal the oracle
+    rs = np.random.default_rng(3)
+    few = [[[1, 2, 3] * 6 for _ in range(600)], [[4, 5] * 9 for _ in range(600)]]
+    many = [[list(rs.integers(0, 40, 18)) for _ in range(600)], [list(rs.integers(0, 40, 18)) for _ in range(600)]]
+    for kernels in (few, many):
+        tr = tg.trace_from_warps(kernels, bb_len=rs.integers(1, 9, 40).tolist())
+        d = _dev(ph, tr)
+        p16, _, _ = oracle.bbv(tr, want_kbb=False)
+        ref = oracle.group_full(tr, p16)
+        ty = ph.photon_warp_group_full(d)
+        T = int(ref["kernel_type_off"][-1])
+        assert np.array_equal(_np(ty["kernel_type_off"], np.uint64), ref["kernel_type_off"])
+        assert np.array_equal(_np(ty["warp_type"], np.uint32), ref["warp_type"])
+        assert np.array_equal(_np(ty["type_count"], np.uint64)[:T], ref["type_count"])
