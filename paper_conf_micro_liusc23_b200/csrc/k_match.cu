@@ -180,8 +180,10 @@ __host__ __device__ __forceinline__ uint64_t filter_jobs_before(uint64_t kb) {
 // word, give sum_j |q_k[j] - q_r[j]| with four VABSDIFF4.ACC per pair (the k-side words stay in registers for the
 // whole job); a sum >= thr8 proves D >= theta.  Fine level, only for pairs the coarse level keeps: the fp32
 // profile distance (bin-major shared tiles).  The k-block stays in shared memory for the job; the next r-block is
-// fetched into registers while the current one is scored.  Surviving pairs are appended with one atomic per warp.
+// fetched into registers while the current one is scored.  Survivors are collected in a shared list per job and
+// appended with one global atomic per CTA.
 constexpr int FTP = FT + 4;  // row stride (floats) of the bin-major profile tiles
+constexpr uint32_t kFiltBuf = 1024;  // survivors kept in shared memory per job
 __device__ __forceinline__ uint32_t sad4(uint32_t a, uint32_t b, uint32_t acc) { return __vsadu4(a, b) + acc; }
 __global__ void __launch_bounds__(256) k_pair_filter(ScanArgs a, uint64_t job0, uint32_t kb_lo, uint32_t kb_hi) {
   const uint64_t job = job0 + blockIdx.x;
@@ -195,11 +197,15 @@ __global__ void __launch_bounds__(256) k_pair_filter(ScanArgs a, uint64_t job0, 
   const uint32_t rb1 = rb0 + FR - 1 < kb ? rb0 + FR - 1 : kb;  // inclusive
 
   const uint32_t k0 = kb * FT;
-  __shared__ __align__(16) float pk[16][FTP], prb[2][16][FTP];
+  __shared__ __align__(16) float pk[16][FTP];
   __shared__ __align__(16) uint4 q8rb[2][FT];
   __shared__ uint64_t wk[FT], wrb[2][FT];
   __shared__ uint32_t okk[FT], okrb[2][FT];  // mass > 0 [P-19]
+  __shared__ uint64_t s_buf[kFiltBuf];       // the job's survivors
+  __shared__ uint32_t s_n;
+  __shared__ unsigned long long s_base;
   const int tid = threadIdx.x, lane = tid & 31;
+  if (tid == 0) s_n = 0;
   for (int i = tid; i < FT * 16; i += 256) {
     const int row = i >> 4, j = i & 15;
     const uint32_t k = k0 + row;
@@ -217,18 +223,12 @@ __global__ void __launch_bounds__(256) k_pair_filter(ScanArgs a, uint64_t job0, 
     const uint32_t k = k0 + i0 + u;
     qk[u] = k < a.K ? *(const uint4*)(a.prof8 + (uint64_t)k * 4) : make_uint4(0, 0, 0, 0);
   }
-  // register stage of one r-block: 4 fp32 profile values + one u8 word per thread, (wt, mass != 0) for tid < FT
-  float sv[4];
+  // register stage of one r-block: one u8 word per thread, (wt, mass != 0) for tid < FT (the fp32 r profiles are
+  // read from L1 / L2 by the fine check of the rare coarse survivors only)
   uint32_t sq = 0;
   uint64_t swr = 0;
   uint32_t sok = 0;
   auto fetch = [&](uint32_t rb) {
-#pragma unroll
-    for (int u = 0; u < 4; ++u) {
-      const int i = tid + u * 256, row = i >> 4, j = i & 15;
-      const uint32_t r = rb * FT + row;
-      sv[u] = r < a.K ? a.prof[(uint64_t)r * 16 + j] : 0.f;
-    }
     {
       const uint32_t r = rb * FT + (tid >> 2);
       sq = r < a.K ? a.prof8[(uint64_t)r * 4 + (tid & 3)] : 0u;
@@ -240,11 +240,6 @@ __global__ void __launch_bounds__(256) k_pair_filter(ScanArgs a, uint64_t job0, 
     }
   };
   auto store = [&](int buf) {
-#pragma unroll
-    for (int u = 0; u < 4; ++u) {
-      const int i = tid + u * 256;
-      prb[buf][i & 15][i >> 4] = sv[u];
-    }
     ((uint32_t*)q8rb[buf])[tid] = sq;
     if (tid < FT) { wrb[buf][tid] = swr; okrb[buf][tid] = sok; }
   };
@@ -254,7 +249,6 @@ __global__ void __launch_bounds__(256) k_pair_filter(ScanArgs a, uint64_t job0, 
   int cur = 0;
   for (uint32_t rb = rb0; rb <= rb1; ++rb, cur ^= 1) {
     if (rb < rb1) fetch(rb + 1);  // in flight while this block is scored
-    const float (*pr)[FTP] = prb[cur];
     const uint4* q8r = q8rb[cur];
     const uint64_t* wr = wrb[cur];
     const uint32_t* okr = okrb[cur];
@@ -281,33 +275,44 @@ __global__ void __launch_bounds__(256) k_pair_filter(ScanArgs a, uint64_t job0, 
     // fine level for the coarse survivors: fp32 profile distance
     for (uint32_t m = keep; m; m &= m - 1) {
       const int bit = __ffs(m) - 1, i = i0 + (bit >> 2), j = j0 + (bit & 3);
+      const float4* rp = (const float4*)(a.prof + (uint64_t)(r0 + j) * 16);  // r < K (eligible)
+      float pr[16];
+#pragma unroll
+      for (int q = 0; q < 4; ++q) {
+        const float4 v = __ldg(rp + q);
+        pr[4 * q] = v.x; pr[4 * q + 1] = v.y; pr[4 * q + 2] = v.z; pr[4 * q + 3] = v.w;
+      }
       float d = 0.f;
 #pragma unroll
-      for (int b = 0; b < 16; ++b) d += fabsf(pk[b][i] - pr[b][j]);
+      for (int b = 0; b < 16; ++b) d += fabsf(pk[b][i] - pr[b]);
       if (!(d < a.bound)) keep &= ~(1u << bit);
     }
-    // warp-aggregated append
-    const uint32_t cnt = __popc(keep);
-    uint32_t incl = cnt;
-    for (int o = 1; o < 32; o <<= 1) {
-      uint32_t y = __shfl_up_sync(0xffffffffu, incl, o);
-      if (lane >= o) incl += y;
-    }
-    const uint32_t total = __shfl_sync(0xffffffffu, incl, 31);
-    if (total) {
-      unsigned long long base = 0;
-      if (lane == 31) base = atomicAdd((unsigned long long*)a.n_maybe, (unsigned long long)total);
-      base = __shfl_sync(0xffffffffu, base, 31);
-      unsigned long long pos = base + (incl - cnt);
-      for (uint32_t m = keep; m; m &= m - 1, ++pos) {
-        const int bit = __ffs(m) - 1;
-        const uint32_t k = k0 + i0 + (bit >> 2), r = r0 + j0 + (bit & 3);
-        if (pos < a.cap) a.maybe[pos] = ((uint64_t)k << 32) | r;
+    // survivors go to the CTA's shared list (flushed to the global list once per job: no global atomic, whose
+    // latency would hold the whole CTA at the next barrier, inside the loop); a full list spills directly
+    for (uint32_t m = keep; m; m &= m - 1) {
+      const int bit = __ffs(m) - 1;
+      const uint32_t k = k0 + i0 + (bit >> 2), r = r0 + j0 + (bit & 3);
+      const uint64_t pr = ((uint64_t)k << 32) | r;
+      const uint32_t sp = atomicAdd(&s_n, 1u);
+      if (sp < kFiltBuf) {
+        s_buf[sp] = pr;
+      } else {
+        const unsigned long long pos = atomicAdd((unsigned long long*)a.n_maybe, 1ull);
+        if (pos < a.cap) a.maybe[pos] = pr;
         else latch(a.err, PHOTON_ECAPACITY, (int64_t)pos);
       }
     }
     if (rb < rb1) store(cur ^ 1);  // that buffer was last read before the previous barrier
     __syncthreads();
+  }
+  // flush the job's shared list: one global atomic per CTA
+  const uint32_t ns = s_n < kFiltBuf ? s_n : kFiltBuf;
+  if (tid == 0 && ns) s_base = atomicAdd((unsigned long long*)a.n_maybe, (unsigned long long)ns);
+  __syncthreads();
+  for (uint32_t i = tid; i < ns; i += 256) {
+    const unsigned long long pos = s_base + i;
+    if (pos < a.cap) a.maybe[pos] = s_buf[i];
+    else latch(a.err, PHOTON_ECAPACITY, (int64_t)pos);
   }
 }
 
