@@ -262,7 +262,14 @@ __global__ void __launch_bounds__(256) k_full_verify_seq(const uint32_t* __restr
     const uint64_t n = we - ws;
     bool seq = true;
     uint64_t i = lane;
-    for (; i + 96 < n; i += 128) {  // four load pairs in flight per lane
+    for (; i + 224 < n; i += 256) {  // eight load pairs in flight per lane
+      uint32_t x[8], y[8];
+#pragma unroll
+      for (int u = 0; u < 8; ++u) { x[u] = bb[ws + i + 32 * u]; y[u] = bb[rs + i + 32 * u]; }
+#pragma unroll
+      for (int u = 0; u < 8; ++u) seq &= x[u] == y[u];
+    }
+    for (; i + 96 < n; i += 128) {
       uint32_t x[4], y[4];
 #pragma unroll
       for (int u = 0; u < 4; ++u) { x[u] = bb[ws + i + 32 * u]; y[u] = bb[rs + i + 32 * u]; }
