@@ -869,6 +869,31 @@ __device__ bool window_run_fast(const WinArgs& a, uint32_t g, int64_t gs, int64_
   const int64_t c = win_y(a, base0 > gs ? base0 : gs);
   bool ok = true;
   constexpr int FU = 8;  // loads in flight per thread (the fill is latency-bound otherwise)
+  const uint32_t c32 = a.D ? __ldg(a.G.Y32 + (base0 > gs ? base0 : gs)) : kDurEsc;
+  if (c32 != kDurEsc) {
+    // the grouped copy without escapes (the usual case), in 32-bit arithmetic: retire times are non-decreasing
+    // along the group, so y' = Y32[q] - c32 >= 0 is exact in u32; x' = y' - D[q] lies in (-lim, y'] exactly when
+    // D[q] < y' + lim; an escaped record fails the test and the run takes the general path
+    const uint32_t lim32 = (uint32_t)a.lim;
+    for (int64_t i0 = 0; i0 < span; i0 += WT * FU) {
+      uint32_t yv[FU], dv[FU];
+#pragma unroll
+      for (int u = 0; u < FU; ++u) {
+        const int64_t i = i0 + u * WT + tid, q = base0 + i;
+        const bool in = i < span && q >= gs;
+        yv[u] = in ? __ldg(a.G.Y32 + q) : c32;
+        dv[u] = in ? __ldg(a.G.D + q) : 0u;
+      }
+#pragma unroll
+      for (int u = 0; u < FU; ++u) {
+        const int64_t i = i0 + u * WT + tid;
+        const uint32_t yr = yv[u] - c32;
+        ok &= yv[u] != kDurEsc && dv[u] != kDurEsc && yr < lim32 && dv[u] < yr + lim32;
+        if (i < span) ring[i] = make_int2((int)(yr - dv[u]), (int)yr);
+      }
+    }
+    if (!__syncthreads_and(ok)) return false;
+  } else {
   for (int64_t i0 = 0; i0 < span; i0 += WT * FU) {
     uint32_t yv[FU], dv[FU];
 #pragma unroll
@@ -902,6 +927,7 @@ __device__ bool window_run_fast(const WinArgs& a, uint32_t g, int64_t gs, int64_
     }
   }
   if (!__syncthreads_and(ok)) return false;
+  }
   // base: windows ending at P0 - 1 ([P0-n, P0-1] and [P0-2n, P0-1]); positions < gs are (0, 0)
   FSums s;
   fs_zero(s);

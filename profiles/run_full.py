@@ -13,5 +13,6 @@ ph = Photon(0)
 d = DeviceTrace.from_host(tg.Generator(cfg).trace(), ph.device)
 b16 = ph.photon_bbv_build(d, bbv16=True, insts=False)["warp_bbv16"]
 torch.cuda.synchronize()
-ph.photon_warp_group_full(d, b16)
+o = ph.photon_warp_group_full(d, b16)  # checked: learns the type-table hint
+ph.photon_warp_group_full(d, b16, check=False, out=o)  # the steady-state call (small table)
 torch.cuda.synchronize()
