@@ -200,6 +200,18 @@ PHOTON_API int photon_match_resolve(photon_ctx *ctx, uint32_t n_kernels, const u
                          const uint64_t *pairs, uint64_t n_pairs, void *ws, size_t ws_bytes, int64_t *match,
                          double *match_dist, void *stream);
 
+/* The chain A1 -> A2 -> A3 -> A4 in one call: photon_warp_group (fused, warp_bbv16 = NULL) into `out` with the
+ * group workspace `gws` (photon_group_workspace_bytes), then photon_kernel_match with the match workspace `mws`
+ * (photon_match_workspace_bytes(K, out->capacity, ...)) -- the same results and device errors (each workspace
+ * latches its own part's).  The library runs independent parts on two internal streams (the filter profiles,
+ * pair filter and bucketing beside the canonical sort; the warp_type write beside A3/A4) with event forks and
+ * joins: all work is ordered after earlier work on `stream`, and later work on `stream` sees every output.  The
+ * fork / join is captured with the rest when `stream` is being captured into a CUDA graph. */
+PHOTON_API int photon_analyse(photon_ctx *ctx, const photon_trace *trace, void *group_ws, size_t group_ws_bytes,
+                              photon_types *out, const uint64_t *warps_total /*[K]*/, photon_match_params params,
+                              void *match_ws, size_t match_ws_bytes, int64_t *match /*[K]*/,
+                              double *match_dist /*[K] or NULL*/, void *stream);
+
 /* ---- A5: per-BB stability test + BB-sampling switch (L208-210 Fig 7, L220-229 Eq. 1) -------------------
  * Timing stream: one record per retired BB execution of the detailed simulation, CSR by kernel, each kernel's
  * records sorted by retire time (ties keep input order) [P-18]; times are integer ticks < 2^40 [P-16].

@@ -80,6 +80,8 @@ _SIGS = [
     ("photon_warp_group", c_int, [c_void_p, POINTER(Trace), c_void_p, c_void_p, c_size_t, POINTER(Types), c_void_p]),
     ("photon_warp_group2", c_int, [c_void_p, POINTER(Trace), c_void_p, c_void_p, c_size_t, POINTER(Types), c_void_p,
                                    c_void_p]),
+    ("photon_analyse", c_int, [c_void_p, POINTER(Trace), c_void_p, c_size_t, POINTER(Types), c_void_p, MatchParams,
+                               c_void_p, c_size_t, c_void_p, c_void_p, c_void_p]),
     ("photon_types_total", c_int, [c_void_p, POINTER(Types), c_uint32, POINTER(c_uint64), c_void_p]),
     ("photon_match_workspace_bytes", c_size_t, [c_uint32, c_uint64, c_uint64]),
     ("photon_kernel_match", c_int, [c_void_p, c_uint32, POINTER(Types), c_void_p, MatchParams, c_void_p, c_size_t,

@@ -553,22 +553,48 @@ class Photon:
     # -- the benchmarked chain ---------------------------------------------------------------------------------
     def analyse(self, t: DeviceTrace, theta=(1, 20), n_cores=64, pool_all_prior=0, want_dist=False, stream=None,
                 check: bool = True, capacity_hint: int = 0, pair_capacity: int = 0, out: Optional[dict] = None) -> dict:
-        """A1 -> A2 -> A3 -> A4 on one device (fused BBV + grouping pass, then canonical tables, signatures,
-        match).  With check=False nothing synchronises (errors stay latched in the returned workspaces).  `out` (a
-        previous result for the same trace) is reused instead of allocating new output tables."""
-        # the per-warp warp_type write runs on a side stream, overlapping A3/A4 on the main one (joined below)
-        main = stream if stream is not None else self.torch.cuda.current_stream(self.device)
-        if getattr(self, "_side", None) is None:
-            self._side = self.torch.cuda.Stream(device=self.device)
-        side = self._side
-        ty = self.photon_warp_group(t, None, capacity_hint, stream=main, check=check, out=out, remap_stream=side)
-        K = t.n_kernels
+        """A1 -> A2 -> A3 -> A4 on one device in one call (photon_analyse: fused BBV + grouping pass, canonical
+        tables, signatures, match; the library overlaps the independent parts on its own streams).  With
+        check=False nothing synchronises (errors stay latched in the returned workspaces).  `out` (a previous result
+        for the same trace) is reused instead of allocating new output tables."""
+        K, W = t.n_kernels, t.n_warps
+        key = (K, W)
+        hint = max(capacity_hint, self._hint.get(key, 0))
+        pcap = max(pair_capacity or (16 * K + 65536), self._pcap.get(K, 0))
+        prm = self.match_params(theta, n_cores, pool_all_prior)
         ok = lambda k: out is not None and out.get(k) is not None and out[k].numel() == K
-        mo = {"match": out["match"]} if ok("match") else None
-        if mo is not None and want_dist and ok("match_dist"):
-            mo["match_dist"] = out["match_dist"]
-        m = self.photon_kernel_match(t.n_kernels, ty, t.warps_total, theta, n_cores, pool_all_prior, want_dist,
-                                     pair_capacity, stream=main, check=check, out=mo)
-        main.wait_stream(side)
-        ty.update(match=m["match"], match_dist=m.get("match_dist"), _mws=m["_ws"])
-        return ty
+        for _ in range(12):
+            ct = t.c()
+            gws = self.workspace("group", self.L.photon_group_workspace_bytes(ctypes.byref(ct), hint))
+            cap = min(max(W, 1), ht_capacity(hint, W))
+            ty = out if self._types_fit(out, K, W, cap) else self.alloc_types(K, W, cap)
+            mws = self.workspace("match", self.L.photon_match_workspace_bytes(K, ty["capacity"], pcap))
+            match = out["match"] if ok("match") else self.empty(K, "int64")
+            dist = None
+            if want_dist:
+                dist = out["match_dist"] if ok("match_dist") else self.empty(K, "float64")
+            tc = self.types_c(ty)
+            self._rc(self.L.photon_analyse(self.ctx, ctypes.byref(ct), gws.data_ptr(), gws.numel(), ctypes.byref(tc),
+                                           t.warps_total.data_ptr(), prm, mws.data_ptr(), mws.numel(),
+                                           match.data_ptr(), None if dist is None else dist.data_ptr(),
+                                           self.stream_ptr(stream)))
+            ty.update(match=match, match_dist=dist, _ws=gws, _mws=mws)
+            if not check:
+                return ty
+            rc, bad = self.ws_status(gws, stream)
+            if rc == _lib.ECAPACITY:  # the type table filled: a larger one
+                hint = max(2 * ht_capacity(hint, W), 1 << 12)
+                out = None
+                continue
+            if rc != 0:
+                raise PhotonError(rc, self.L.photon_last_error(self.ctx).decode(), bad)
+            rc, bad = self.ws_status(mws, stream)
+            if rc == _lib.ECAPACITY:  # the pair list filled: a larger one
+                pcap *= 4
+                continue
+            if rc != 0:
+                raise PhotonError(rc, self.L.photon_last_error(self.ctx).decode(), bad)
+            self._hint[key] = hint
+            self._pcap[K] = pcap
+            return ty
+        raise PhotonError(_lib.ECAPACITY, "type table or pair list kept overflowing")

@@ -23,6 +23,9 @@ struct photon_ctx {
   std::vector<std::pair<cudaEvent_t, cudaEvent_t>> ev[PHOTON_PROF_N];
   size_t used[PHOTON_PROF_N] = {0};
   cudaEvent_t fork = nullptr;  // photon_warp_group2: the remap's dependency on the main stream
+  // photon_analyse: two library streams and the events of its fork / join graph (created on first use)
+  cudaStream_t sa = nullptr, sb = nullptr;
+  cudaEvent_t aev[6] = {nullptr, nullptr, nullptr, nullptr, nullptr, nullptr};
 };
 
 namespace {
@@ -316,6 +319,10 @@ void photon_destroy(photon_ctx* ctx) {
   for (auto& v : ctx->ev)
     for (auto& pr : v) { cudaEventDestroy(pr.first); cudaEventDestroy(pr.second); }
   if (ctx->fork) cudaEventDestroy(ctx->fork);
+  for (auto& e : ctx->aev)
+    if (e) cudaEventDestroy(e);
+  if (ctx->sa) cudaStreamDestroy(ctx->sa);
+  if (ctx->sb) cudaStreamDestroy(ctx->sb);
   delete ctx;
 }
 
@@ -517,6 +524,95 @@ int photon_kernel_match(photon_ctx* ctx, uint32_t K, const photon_types* types, 
                             m.n_pairs, m.mw, match, match_dist, m.err, ctx->num_sms, s, /*fused=*/true),
        "resolve");
   }
+  return PHOTON_OK;
+}
+
+// ---- the whole chain in one call, its independent parts overlapped -------------------------------------------
+int photon_analyse(photon_ctx* ctx, const photon_trace* t, void* gws, size_t gws_bytes, photon_types* out,
+                   const uint64_t* warps_total, photon_match_params params, void* mws, size_t mws_bytes,
+                   int64_t* match, double* match_dist, void* stream) {
+  NvtxRange nvtx_("photon_analyse");
+  if (!ctx) return PHOTON_EINVAL;
+  int rc = check_trace(ctx, t);
+  if (rc) return rc;
+  if (!gws || !mws || !out || !warps_total || !match) return fail(ctx, PHOTON_EINVAL, "NULL argument");
+  if (!out->warp_type || !out->kernel_type_off || !out->type_key || !out->type_count || !out->type_first_warp ||
+      !out->warp_sampling_ok)
+    return fail(ctx, PHOTON_EINVAL, "NULL photon_types array");
+  if (!aligned(out->type_key, 16)) return fail(ctx, PHOTON_EINVAL, "type_key must be 16-byte aligned");
+  const uint32_t K = t->n_kernels;
+  if (K == 0) return fail(ctx, PHOTON_EINVAL, "K must be >= 1");
+  params = norm_params(params);
+  rc = check_match_params(ctx, params);
+  if (rc) return rc;
+  GroupWs g0 = group_layout(t, 0, nullptr, 0);
+  if (gws_bytes < g0.b.bytes + 256) return fail(ctx, PHOTON_EWORKSPACE, "group workspace too small");
+  GroupWs g = group_layout(t, 1, gws, gws_bytes);
+  if (g.bytes > gws_bytes) return fail(ctx, PHOTON_EWORKSPACE, "group workspace %zu < %zu bytes", gws_bytes, g.bytes);
+  const uint64_t T = out->capacity;
+  MatchLayout m0 = match_layout(K, T, 1024, nullptr);
+  if (mws_bytes < m0.bytes) return fail(ctx, PHOTON_EWORKSPACE, "match workspace %zu < %zu bytes", mws_bytes, m0.bytes);
+  MatchLayout m = match_layout_fit(K, T, mws, mws_bytes);
+  cudaStream_t s = (cudaStream_t)stream;
+  CK(cudaSetDevice(ctx->device), "cudaSetDevice");
+  if (!ctx->sa) {
+    CK(cudaStreamCreateWithFlags(&ctx->sa, cudaStreamNonBlocking), "stream");
+    CK(cudaStreamCreateWithFlags(&ctx->sb, cudaStreamNonBlocking), "stream");
+    for (auto& e : ctx->aev) CK(cudaEventCreateWithFlags(&e, cudaEventDisableTiming), "event");
+  }
+  cudaStream_t sa = ctx->sa, sb = ctx->sb;
+  cudaEvent_t e_lists = ctx->aev[0], e_sorted = ctx->aev[1], e_prof = ctx->aev[2], e_filt = ctx->aev[3],
+              e_remap = ctx->aev[4];
+  ctx->last_ws = gws;
+  TraceDev d = to_dev(t);
+  DevErr* err = g.b.err;
+  CK(cudaMemsetAsync(err, 0, sizeof(DevErr), s), "memset");
+  CK(cudaMemsetAsync(m.err, 0, sizeof(DevErr), s), "memset");
+  {
+    ProfScope ps(ctx, PHOTON_PROF_PREP, s);
+    CK(launch_ht_clear(g.h.ht, s), "ht_clear");
+    CK(cudaMemsetAsync(g.ep.count, 0, 8, s), "memset");
+    CK(launch_validate_offsets(d, err, s), "validate");
+    CK(launch_table_prep(d, g.b.tb, err, s), "table");
+  }
+  {
+    ProfScope ps(ctx, PHOTON_PROF_BBV_FUSED, s);
+    CK(launch_bbv3(d, g.b.tb, nullptr, nullptr, &g.ep, err, ctx->num_sms, s), "bbv_fused");
+  }
+  {
+    ProfScope ps(ctx, PHOTON_PROF_CANON, s);
+    CK(launch_entries_insert(g.ep, g.h.ht, err, ctx->num_sms, s), "insert");
+    CK(launch_canon_lists(g.h.ht, K, *out, g.h.cw, err, s), "canon");
+    // fork 1: the filter profiles, the pair filter and its bucketing need only the unsorted table and its lists
+    CK(cudaEventRecord(e_lists, s), "event");
+    CK(cudaStreamWaitEvent(sb, e_lists, 0), "event");
+    CK(launch_analyse_filter(K, out->kernel_type_off, g.h.cw.list, g.h.ht, m.mass, warps_total, params, m.mw, m.pairs,
+                             m.err, ctx->num_sms, sb, e_prof),
+       "filter");
+    CK(cudaEventRecord(e_filt, sb), "event");
+    CK(launch_canon_sort(g.h.ht, K, t->kernel_warp_off, nullptr, *out, g.h.cw, ctx->num_sms, s), "sort");
+    // fork 2: the per-warp warp_type write
+    CK(cudaEventRecord(e_sorted, s), "event");
+    CK(cudaStreamWaitEvent(sa, e_sorted, 0), "event");
+    CK(launch_remap_entries(g.ep, t->n_warps, g.h.cw.canon, out->warp_type, sa), "remap");
+    CK(cudaEventRecord(e_remap, sa), "event");
+  }
+  {
+    ProfScope ps(ctx, PHOTON_PROF_SCAN, s);
+    CK(cudaStreamWaitEvent(s, e_prof, 0), "event");  // 1/N
+    CK(launch_analyse_sigf(K, *out, m.sig, m.mw, s), "sigf");
+    CK(cudaStreamWaitEvent(s, e_filt, 0), "event");  // the bucketed survivors
+    CK(launch_analyse_exact(K, out->kernel_type_off, m.sig, m.mass, warps_total, params, m.mw, m.pairs,
+                            m.mw.pair_cap, m.n_pairs, m.err, ctx->num_sms, s),
+       "exact");
+  }
+  {
+    ProfScope ps(ctx, PHOTON_PROF_RESOLVE, s);
+    CK(launch_match_resolve(K, out->kernel_type_off, m.sig, m.mass, warps_total, params, m.pairs, m.mw.pair_cap,
+                            m.n_pairs, m.mw, match, match_dist, m.err, ctx->num_sms, s, /*fused=*/true),
+       "resolve");
+  }
+  CK(cudaStreamWaitEvent(s, e_remap, 0), "event");  // join: everything is ordered before later work on `stream`
   return PHOTON_OK;
 }
 

@@ -143,6 +143,61 @@ __global__ void k_sig_prof(uint32_t K, const uint64_t* __restrict__ kto, const u
   }
 }
 
+// photon_analyse's split of k_sig_prof, so the filter need not wait for the canonical sort:
+// k_prof_slots -- the filter profiles, 1/N and N from the UNSORTED type table (the per-kernel slot lists of the
+// canonicalisation; the bin sums are exact integers, so they equal the sorted rows' sums bit for bit);
+// k_sigf -- g and its fp32 copy g / N in the canonical row order, after the sort.
+__global__ void k_prof_slots(uint32_t K, const uint64_t* __restrict__ kto, const uint32_t* __restrict__ list,
+                             HashTable ht, uint64_t* __restrict__ mass, float* __restrict__ prof,
+                             double* __restrict__ invn, uint32_t* __restrict__ prof8, DevErr* err) {
+  const uint32_t k = (blockIdx.x * blockDim.x + threadIdx.x) >> 5, lane = threadIdx.x & 31;
+  if (k >= K) return;
+  const uint64_t r0 = kto[k], r1 = kto[k + 1];
+  uint64_t acc = 0;
+  bool over = false;
+  for (uint64_t r = r0 + (lane >> 4); r < r1; r += 2) {
+    const uint32_t sl = list[r];
+    const uint64_t g = (uint64_t)ht.count[sl] * (uint64_t)ht.key[(uint64_t)sl * 16 + (lane & 15)];
+    over |= g >= kMassLimit;
+    acc += g;
+    over |= acc >= kMassLimit;
+  }
+  const uint64_t bin = acc + __shfl_xor_sync(0xffffffffu, acc, 16);
+  uint64_t N = bin;
+  for (int o = 8; o > 0; o >>= 1) N += __shfl_xor_sync(0xffffffffu, N, o);
+  over = __any_sync(0xffffffffu, over) || N >= kMassLimit;
+  const double inv = N ? 1.0 / (double)N : 0.0;
+  const double P = N ? (double)bin / (double)N : 0.0;
+  uint32_t q = (uint32_t)rint(P * 255.0);
+  q = q > 255u ? 255u : q;
+  uint32_t w = q << (8 * (lane & 3));
+  w |= __shfl_xor_sync(0xffffffffu, w, 1);
+  w |= __shfl_xor_sync(0xffffffffu, w, 2);
+  if (lane < 16) {
+    prof[(uint64_t)k * 16 + lane] = (float)P;
+    if ((lane & 3) == 0) prof8[(uint64_t)k * 4 + (lane >> 2)] = w;
+    if (lane == 0) {
+      invn[k] = inv;
+      mass[k] = N;
+      if (over) latch(err, PHOTON_ERANGE, (int64_t)k);
+    }
+  }
+}
+__global__ void k_sigf(uint32_t K, const uint64_t* __restrict__ kto, const uint32_t* __restrict__ key,
+                       const uint64_t* __restrict__ count, const double* __restrict__ invn, uint64_t* __restrict__ sig,
+                       float* __restrict__ sigf) {
+  const uint32_t k = (blockIdx.x * blockDim.x + threadIdx.x) >> 5, lane = threadIdx.x & 31;
+  if (k >= K) return;
+  const uint64_t r0 = kto[k], r1 = kto[k + 1];
+  const double inv = invn[k];
+  for (uint64_t r = r0 + (lane >> 4); r < r1; r += 2) {
+    const uint64_t i = r * 16 + (lane & 15);
+    const uint64_t g = count[r] * (uint64_t)key[i];
+    sig[i] = g;
+    if (sigf) sigf[i] = (float)((double)g * inv);
+  }
+}
+
 // ---- pair filter: 64 x 64 tiles of (k, r < k) --------------------------------------------------------------
 constexpr int FT = 64;
 struct ScanArgs {
@@ -710,6 +765,47 @@ cudaError_t launch_sig_prof(uint32_t K, const uint64_t* kto, const uint32_t* typ
   return cudaGetLastError();
 }
 
+namespace {
+ScanArgs scan_args(uint32_t K, uint32_t k_lo, uint32_t k_hi, const uint64_t* kto, const uint64_t* sig,
+                   const uint64_t* mass, const uint64_t* wt, photon_match_params p, const MatchWs& mw, DevErr* err) {
+  ScanArgs a{};
+  a.K = K; a.k_lo = k_lo; a.k_hi = k_hi; a.kto = kto; a.sig = sig; a.mass = mass; a.wt = wt; a.prof = mw.prof; a.invn = mw.invn; a.prof8 = mw.prof8; a.sigf = mw.sigf;
+  a.p = p;
+  // rigorous margin: each |P_k - P_r| term carries <= 3 fp32 roundings of values in [0, 1] plus 16 additions
+  a.bound = (float)((double)p.theta_num / (double)p.theta_den) + 1e-5f;
+  // |q - 255 P| <= 1/2 + 2^-40 per value, so sum_j |q_k - q_r| <= 255 sum_j |P_k - P_r| + 16 + 2^-30 <= 255 D + 17:
+  // a pair with sum >= 255 theta + 17 has D >= theta
+  a.thr8 = (uint32_t)ceil(255.0 * (double)p.theta_num / (double)p.theta_den + 17.0);
+  a.maybe = mw.maybe; a.n_maybe = mw.n_maybe; a.cap = mw.pair_cap; a.err = err;
+  return a;
+}
+void launch_filter(const ScanArgs& a, cudaStream_t s) {
+  const uint32_t kb_hi = (uint32_t)ceil_div(a.k_hi, FT), kb_lo = a.k_lo / FT;
+  const uint64_t j0 = filter_jobs_before(kb_lo), j1 = filter_jobs_before(kb_hi);
+  if (j1 > j0) note_launch(), k_pair_filter<<<(unsigned)(j1 - j0), 256, 0, s>>>(a, j0, kb_lo, kb_hi);
+}
+// the fused path's survivors bucketed by k into `pairs` (free there: close pairs go to cand segments)
+void launch_bucket(uint32_t K, const MatchWs& mw, uint64_t* pairs, DevErr* err, int num_sms, cudaStream_t s) {
+  const unsigned gb = (unsigned)umin64(ceil_div(mw.pair_cap, 256), (uint64_t)num_sms * 64);
+  cudaMemsetAsync(mw.cand_cnt, 0, sizeof(uint32_t) * K, s);
+  cudaMemsetAsync(mw.close_cnt, 0, sizeof(uint32_t) * K, s);
+  note_launch(), k_cand_count<<<gb, 256, 0, s>>>(mw.maybe, mw.pair_cap, mw.n_maybe, K, mw.cand_cnt, err);
+  note_launch(), k_cand_scan<<<1, 1024, 0, s>>>(mw.cand_cnt, K, mw.cand_off, mw.cand_cur);
+  note_launch(), k_pair_bucket<<<gb, 256, 0, s>>>(mw.maybe, mw.pair_cap, mw.n_maybe, K, mw.cand_off, mw.cand_cur,
+                                                  pairs);
+}
+void launch_exact(ScanArgs a, bool fused, const MatchWs& mw, uint64_t* pairs, uint64_t pair_cap, uint64_t* n_pairs,
+                  int num_sms, cudaStream_t s) {
+  if (fused) {
+    a.maybe = pairs;
+    a.cand = mw.cand;
+    a.cbeg = mw.cand_off;
+    a.ccnt = mw.close_cnt;
+  }
+  note_launch(), k_pair_exact<<<(unsigned)num_sms * 8, 256, 0, s>>>(a, pairs, pair_cap, n_pairs);
+}
+}  // namespace
+
 cudaError_t launch_match_scan(uint32_t K, const uint64_t* kto, const uint64_t* sig, const uint64_t* mass,
                               const uint64_t* wt, photon_match_params p, uint32_t k_lo, uint32_t k_hi,
                               const MatchWs& mw, uint64_t* pairs, uint64_t pair_cap, uint64_t* n_pairs, DevErr* err,
@@ -720,34 +816,39 @@ cudaError_t launch_match_scan(uint32_t K, const uint64_t* kto, const uint64_t* s
   if (!prof_ready)
     note_launch(), k_prof<<<(unsigned)ceil_div((uint64_t)K * 32, 256), 256, 0, s>>>(K, kto, sig, mass, mw.prof,
                                                                                   mw.invn, mw.prof8, mw.sigf);
-  ScanArgs a{};
-  a.K = K; a.k_lo = k_lo; a.k_hi = k_hi; a.kto = kto; a.sig = sig; a.mass = mass; a.wt = wt; a.prof = mw.prof; a.invn = mw.invn; a.prof8 = mw.prof8; a.sigf = mw.sigf;
-  a.p = p;
-  // rigorous margin: each |P_k - P_r| term carries <= 3 fp32 roundings of values in [0, 1] plus 16 additions
-  a.bound = (float)((double)p.theta_num / (double)p.theta_den) + 1e-5f;
-  // |q - 255 P| <= 1/2 + 2^-40 per value, so sum_j |q_k - q_r| <= 255 sum_j |P_k - P_r| + 16 + 2^-30 <= 255 D + 17:
-  // a pair with sum >= 255 theta + 17 has D >= theta
-  a.thr8 = (uint32_t)ceil(255.0 * (double)p.theta_num / (double)p.theta_den + 17.0);
-  a.maybe = mw.maybe; a.n_maybe = mw.n_maybe; a.cap = mw.pair_cap; a.err = err;
-  const uint32_t kb_hi = (uint32_t)ceil_div(k_hi, FT), kb_lo = k_lo / FT;
-  const uint64_t j0 = filter_jobs_before(kb_lo), j1 = filter_jobs_before(kb_hi);
-  if (j1 > j0) note_launch(), k_pair_filter<<<(unsigned)(j1 - j0), 256, 0, s>>>(a, j0, kb_lo, kb_hi);
-  unsigned grid = (unsigned)num_sms * 8;
-  if (fused) {
-    // bucket the survivors by k into the pairs buffer (free in the fused path: close pairs go to cand segments)
-    const unsigned gb = (unsigned)umin64(ceil_div(mw.pair_cap, 256), (uint64_t)num_sms * 64);
-    cudaMemsetAsync(mw.cand_cnt, 0, sizeof(uint32_t) * K, s);
-    cudaMemsetAsync(mw.close_cnt, 0, sizeof(uint32_t) * K, s);
-    note_launch(), k_cand_count<<<gb, 256, 0, s>>>(mw.maybe, mw.pair_cap, mw.n_maybe, K, mw.cand_cnt, err);
-    note_launch(), k_cand_scan<<<1, 1024, 0, s>>>(mw.cand_cnt, K, mw.cand_off, mw.cand_cur);
-    note_launch(), k_pair_bucket<<<gb, 256, 0, s>>>(mw.maybe, mw.pair_cap, mw.n_maybe, K, mw.cand_off, mw.cand_cur,
-                                                    pairs);
-    a.maybe = pairs;
-    a.cand = mw.cand;
-    a.cbeg = mw.cand_off;
-    a.ccnt = mw.close_cnt;
-  }
-  note_launch(), k_pair_exact<<<grid, 256, 0, s>>>(a, pairs, pair_cap, n_pairs);
+  const ScanArgs a = scan_args(K, k_lo, k_hi, kto, sig, mass, wt, p, mw, err);
+  launch_filter(a, s);
+  if (fused) launch_bucket(K, mw, pairs, err, num_sms, s);
+  launch_exact(a, fused, mw, pairs, pair_cap, n_pairs, num_sms, s);
+  return cudaGetLastError();
+}
+
+// photon_analyse's split: A3 profiles + filter + bucketing from the unsorted table (stream sb), then -- after the
+// sort, on the main stream -- g / N in row order and the exact check
+cudaError_t launch_analyse_filter(uint32_t K, const uint64_t* kto, const uint32_t* list, const HashTable& ht,
+                                  uint64_t* mass, const uint64_t* wt, photon_match_params p, const MatchWs& mw,
+                                  uint64_t* pairs, DevErr* err, int num_sms, cudaStream_t sb, cudaEvent_t prof_done) {
+  cudaMemsetAsync(mw.n_maybe, 0, 8, sb);
+  note_launch(), k_prof_slots<<<(unsigned)ceil_div((uint64_t)K * 32, 256), 256, 0, sb>>>(K, kto, list, ht, mass,
+                                                                                       mw.prof, mw.invn, mw.prof8,
+                                                                                       err);
+  cudaEventRecord(prof_done, sb);
+  const ScanArgs a = scan_args(K, 0, K, kto, nullptr, mass, wt, p, mw, err);
+  launch_filter(a, sb);
+  launch_bucket(K, mw, pairs, err, num_sms, sb);
+  return cudaGetLastError();
+}
+cudaError_t launch_analyse_sigf(uint32_t K, const photon_types& types, uint64_t* sig, const MatchWs& mw,
+                                cudaStream_t s) {
+  note_launch(), k_sigf<<<(unsigned)ceil_div((uint64_t)K * 32, 256), 256, 0, s>>>(
+      K, types.kernel_type_off, types.type_key, types.type_count, mw.invn, sig, mw.sigf);
+  return cudaGetLastError();
+}
+cudaError_t launch_analyse_exact(uint32_t K, const uint64_t* kto, const uint64_t* sig, const uint64_t* mass,
+                                 const uint64_t* wt, photon_match_params p, const MatchWs& mw, uint64_t* pairs,
+                                 uint64_t pair_cap, uint64_t* n_pairs, DevErr* err, int num_sms, cudaStream_t s) {
+  cudaMemsetAsync(n_pairs, 0, 8, s);
+  launch_exact(scan_args(K, 0, K, kto, sig, mass, wt, p, mw, err), true, mw, pairs, pair_cap, n_pairs, num_sms, s);
   return cudaGetLastError();
 }
 
