@@ -15,6 +15,8 @@ def _run(tool, what):
            os.path.join(ROOT, "profiles", "sanitize_run.py"), what]
     p = subprocess.run(cmd, capture_output=True, text=True, timeout=1500, cwd=ROOT)
     out = p.stdout + p.stderr
+    if "closed on this pool" in out:  # the pool's operators have disabled compute-sanitizer (it left GPUs hung)
+        pytest.skip("compute-sanitizer is disabled on this GPU pool: " + out.strip().splitlines()[-1][:200])
     assert p.returncode == 0, out[-4000:]
     assert "ERROR SUMMARY: 0 errors" in out or "SUMMARY: 0 hazards displayed (0 errors, 0 warnings)" in out, out[-4000:]
     assert "sanitize run ok" in out
