@@ -50,7 +50,19 @@ constexpr int GRP = 4;              // workers sharing a row array (row stride G
 constexpr uint32_t ROWB = GRP * NCOL * 4;
 constexpr uint32_t ENT_BLK = 64;    // entries taken from the global pool at a time
 constexpr int SMEM_TBL_MAX = 4096;  // BB table entries kept in shared memory (else read through L1)
-constexpr uint32_t NARROW_QMAX = 9;
+#ifndef K1_PIN
+#define K1_PIN 1
+#endif
+#ifndef K1_VNX
+#define K1_VNX 1
+#endif
+#ifndef K1_PRMT
+#define K1_PRMT 0
+#endif
+#ifndef K1_QMAX
+#define K1_QMAX 11
+#endif
+constexpr uint32_t NARROW_QMAX = K1_QMAX;  // odd, <= 17 (divL)
 constexpr uint32_t kMarkN = 0x80000000u;  // neutral table: id in [B, P2)
 
 // Narrow: u16 cells, entry = (bin odd ? len << 16 : len) | (bin >> 1) << 10 (len < 1024); mark = bit 31.
@@ -97,7 +109,10 @@ struct Args3 {
 };
 
 // per-worker scratch in shared memory
-constexpr int kEntCache = 128;
+#ifndef K1_ENTCACHE
+#define K1_ENTCACHE 128
+#endif
+constexpr int kEntCache = K1_ENTCACHE;
 struct WMisc {
   uint32_t rel[40];             // chunk-relative starts of the block's warps (rel[nw..] = block end), clamped
   uint32_t fwt[32];             // first-warp scatter table of the lane ranges
@@ -114,6 +129,12 @@ struct WMisc {
 };
 constexpr uint32_t kWMiscBytes = (sizeof(WMisc) + 127) & ~127u;
 
+// x << s with s >= 64 giving 0 (PTX shl clamps the shift amount)
+__device__ __forceinline__ uint64_t shl64_clamp(uint64_t x, uint32_t s) {
+  uint64_t r;
+  asm("shl.b64 %0, %1, %2;" : "=l"(r) : "l"(x), "r"(s));
+  return r;
+}
 __device__ __forceinline__ void red_add(uint32_t saddr, uint32_t v) {
   // no "memory" clobber: cells are written only by these adds and read only after __syncwarp
   asm volatile("red.shared.add.u32 [%0], %1;" ::"r"(saddr), "r"(v));
@@ -284,9 +305,9 @@ __device__ __forceinline__ void clear_cells(uint32_t cw) {
 }
 
 // x / L for L = 8 Qe, Qe odd <= 17, x < 2^20: umulhi(x >> 3, ceil(2^32 / Qe))
-__device__ __forceinline__ uint32_t qinv_of(uint32_t Qe) {  // ceil(2^32 / Qe) for odd Qe <= 9
-  return Qe == 3u ? 0x55555556u : Qe == 5u ? 0x33333334u : Qe == 7u ? 0x24924925u : Qe == 9u ? 0x1C71C71Du : 0u;
-}
+__constant__ uint32_t kQinv[9] = {0u,          0x55555556u, 0x33333334u, 0x24924925u, 0x1C71C71Du,
+                                  0x1745D175u, 0x13B13B14u, 0x11111112u, 0x0F0F0F10u};  // Qe = 1, 3, ..., 17
+__device__ __forceinline__ uint32_t qinv_of(uint32_t Qe) { return kQinv[Qe >> 1]; }  // ceil(2^32 / Qe), odd Qe
 __device__ __forceinline__ uint32_t divL(uint32_t x, uint32_t Qe, uint32_t qinv) {
   return Qe == 1u ? (x >> 3) : __umulhi(x >> 3, qinv);
 }
@@ -521,9 +542,10 @@ __global__ void __launch_bounds__(WPC * 32, 1) k_bbv3(Args3 a) {
           nb2 = wm->rel[u + 2];
         }
         const uint32_t kn = (e - t0 * L + 7u) >> 3;
+        uint32_t tbr = tbase, m4r = mask4;
         auto look = [&](uint32_t x4) -> uint32_t {  // x4 = id * 4 (in the low bits, masked here)
-          if (GTBL) return __ldg(tbl_g + ((x4 & mask4) >> 2));
-          return lds_tbl((x4 & mask4) | tbase);  // the table is aligned to its size: one LOP3
+          if (GTBL) return __ldg(tbl_g + ((x4 & m4r) >> 2));
+          return lds_tbl((x4 & m4r) | tbr);  // the table is aligned to its size: one LOP3
         };
         // low halves: rotate left by 2 (one SHF; the wrapped bits fall outside mask4), high halves: shift right by 14
         auto lookup = [&](const uint4& v, uint32_t (&tv)[8]) {
@@ -536,24 +558,49 @@ __global__ void __launch_bounds__(WPC * 32, 1) k_bbv3(Args3 a) {
           tv[6] = look(__funnelshift_l(v.w, v.w, 2));
           tv[7] = look(v.w >> 14);
         };
+#if K1_PRMT
+        uint32_t cbx = __byte_perm(col, 0u, 0u), cby = __byte_perm(coln, 0u, 0u);  // column bytes, replicated
+#endif
         uint4 vnx = sb4[0];
         uint32_t tv[8];
         lookup(vnx, tv);
         for (uint32_t kk = 0; kk < kn; ++kk) {
+#if K1_PIN
+          asm volatile("" : "+r"(tbr), "+r"(m4r));  // keep the table base and mask live (no per-word remat)
+#endif
           const uint32_t p0 = (t0 * Qe + kk) * 8u;
           raw |= (vnx.x | vnx.y) | (vnx.z | vnx.w);
+#if K1_VNX
+          vnx = sb4[kk + 1];  // one word past the lane's range: always inside the allocation (unused at the end)
+#else
           vnx = sb4[kk + 1 < kn ? kk + 1 : kk];
+#endif
           if (MARK) orr |= (tv[0] | tv[1] | tv[2] | tv[3]) | (tv[4] | tv[5] | tv[6] | tv[7]);
           if (nb2 >= p0 + 8u) {  // at most one boundary (at nb) in the word: events j >= nb - p0 go to coln
             const uint32_t mcut = nb - p0;
+#if K1_PRMT
+            // the column bytes of the 8 events as two byte vectors (a worker's 64 columns share one 256-byte span,
+            // so a cell address is cw | column byte | row bits): one LOP3 per 4 events, one PRMT per event
+            const uint64_t bm = shl64_clamp(~0ull, mcut * 8u);  // bytes j >= mcut
+            const uint32_t cv0 = (cbx & ~(uint32_t)bm) | (cby & (uint32_t)bm);
+            const uint32_t cv1 = (cbx & ~(uint32_t)(bm >> 32)) | (cby & (uint32_t)(bm >> 32));
+#pragma unroll
+            for (int j = 0; j < 8; ++j)
+              red_add(__byte_perm(j < 4 ? cv0 : cv1, cw, 0x7650u + (j & 3)) | (tv[j] & M::ROFF), M::val(tv[j]));
+#else
 #pragma unroll
             for (int j = 0; j < 8; ++j) red_add(((uint32_t)j < mcut ? col : coln) | (tv[j] & M::ROFF), M::val(tv[j]));
+#endif
             if (nb <= p0 + 8u) {
               ++u;
               col = coln;
               coln = pcol(u + 1);
               nb = nb2;
               nb2 = wm->rel[u + 2];
+#if K1_PRMT
+              cbx = cby;
+              cby = __byte_perm(coln, 0u, 0u);
+#endif
             }
           } else {
             // several warp boundaries in the word (warps shorter than 8 events): event by event
@@ -573,6 +620,10 @@ __global__ void __launch_bounds__(WPC * 32, 1) k_bbv3(Args3 a) {
             coln = pcol(u + 1);
             nb = wm->rel[u + 1];
             nb2 = wm->rel[u + 2];
+#if K1_PRMT
+            cbx = __byte_perm(col, 0u, 0u);
+            cby = __byte_perm(coln, 0u, 0u);
+#endif
           }
           lookup(vnx, tv);
         }
@@ -843,7 +894,7 @@ Layout3 layout3(uint32_t P2, bool gtbl, int reserved) {
   const uint32_t A = M::ROWS * ROWB;  // row arrays aligned to their size (OR addressing)
   L.off_cells = up(L.off_tbl + tbl, A);
   L.off_stage = L.off_cells + (WPC / GRP) * A;
-  L.bytes = L.off_stage + WPC * NBUF * 32 * M::Q * 16;
+  L.bytes = L.off_stage + WPC * NBUF * 32 * M::Q * 16 + 16;  // + one word: the event loop reads a word ahead
   return L;
 }
 
