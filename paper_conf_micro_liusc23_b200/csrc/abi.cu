@@ -124,8 +124,8 @@ BbvWs bbv_layout(const photon_trace* t, void* base) {
 
 // Entry pool: one entry per distinct (kernel, key) of each 32-warp block -- at most W -- bounded by 8x the
 // type-table capacity (ECAPACITY beyond: the caller retries with a larger hint), plus room for every K1 worker's
-// partly used last block of 64 entries (<= 160 SMs x 16 workers).
-constexpr uint64_t kPoolSlack = 160ull * 16 * 64;
+// partly used last block of 64 entries (<= 160 SMs x 32 workers).
+constexpr uint64_t kPoolSlack = 160ull * 32 * 64;
 void carve_entries(Carver& c, uint64_t W, uint64_t cap, EntryPool& ep) {
   ep.cap = (W < 8 * cap ? W : 8 * cap) + kPoolSlack;
   ep.ent = c.take<TileEntry>(ep.cap);
