@@ -56,6 +56,59 @@ struct Carver {
   }
 };
 
+// ---- single-CTA exclusive scan of u32 counts into u64 offsets (1024 threads) ---------------------------------
+// off[i] = sum of cnt[0..i), off[n] = the total; zero[i] = 0 when zero != nullptr.  Tiles of 1024 x 8 counts: each
+// thread sums 8 consecutive counts in registers, one block scan of the thread sums per tile (two barriers), so a
+// K of 10^4 takes two tiles.  Returns the total (thread 0 only).
+__device__ __forceinline__ uint64_t cta_scan_counts(const uint32_t* __restrict__ cnt, uint32_t n, uint64_t* off,
+                                                    uint32_t* zero) {
+  constexpr int IT = 8;
+  __shared__ uint64_t s_ws[32];
+  const uint32_t tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
+  uint64_t carry = 0;  // identical in every thread
+  for (uint32_t base = 0; base < n; base += 1024u * IT) {
+    uint32_t v[IT];
+    const uint32_t i0 = base + tid * IT;
+    uint64_t sum = 0;
+#pragma unroll
+    for (int j = 0; j < IT; ++j) {
+      v[j] = i0 + j < n ? cnt[i0 + j] : 0u;
+      sum += v[j];
+    }
+    if (zero) {
+#pragma unroll
+      for (int j = 0; j < IT; ++j)
+        if (i0 + j < n) zero[i0 + j] = 0u;
+    }
+    uint64_t x = sum;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const uint64_t y = __shfl_up_sync(0xffffffffu, x, o);
+      if ((int)lane >= o) x += y;
+    }
+    if (lane == 31) s_ws[wid] = x;
+    __syncthreads();
+    uint64_t w = lane < (blockDim.x >> 5) ? s_ws[lane] : 0;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const uint64_t y = __shfl_up_sync(0xffffffffu, w, o);
+      if ((int)lane >= o) w += y;
+    }
+    const uint64_t wex = __shfl_sync(0xffffffffu, w, wid) - s_ws[wid];  // warps before this one
+    const uint64_t tot = __shfl_sync(0xffffffffu, w, 31);
+    __syncthreads();  // s_ws is rewritten by the next tile
+    uint64_t run = carry + wex + x - sum;
+#pragma unroll
+    for (int j = 0; j < IT; ++j) {
+      if (i0 + j < n) off[i0 + j] = run;
+      run += v[j];
+    }
+    carry += tot;
+  }
+  if (tid == 0) off[n] = carry;
+  return carry;
+}
+
 __host__ __device__ __forceinline__ uint64_t umin64(uint64_t a, uint64_t b) { return a < b ? a : b; }
 __host__ __device__ __forceinline__ uint64_t umax64(uint64_t a, uint64_t b) { return a > b ? a : b; }
 __host__ __device__ __forceinline__ uint64_t ceil_div(uint64_t a, uint64_t b) { return (a + b - 1) / b; }

@@ -515,38 +515,7 @@ __global__ void k_cand_count(const uint64_t* pairs, uint64_t n_host, const uint6
 }
 
 __global__ void __launch_bounds__(1024) k_cand_scan(const uint32_t* cnt, uint32_t K, uint64_t* off, uint32_t* cur) {
-  __shared__ uint64_t ws[32];
-  __shared__ uint64_t carry;
-  if (threadIdx.x == 0) carry = 0;
-  __syncthreads();
-  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
-  for (uint32_t base = 0; base < K; base += 1024) {
-    uint32_t k = base + threadIdx.x;
-    uint64_t v = k < K ? cnt[k] : 0;
-    if (k < K) cur[k] = 0;
-    uint64_t x = v;
-    for (int o = 1; o < 32; o <<= 1) {
-      uint64_t y = __shfl_up_sync(0xffffffffu, x, o);
-      if (lane >= o) x += y;
-    }
-    if (lane == 31) ws[wid] = x;
-    __syncthreads();
-    if (wid == 0) {
-      uint64_t s = ws[lane];
-      for (int o = 1; o < 32; o <<= 1) {
-        uint64_t y = __shfl_up_sync(0xffffffffu, s, o);
-        if (lane >= o) s += y;
-      }
-      ws[lane] = s;
-    }
-    __syncthreads();
-    uint64_t excl = carry + (wid ? ws[wid - 1] : 0) + x - v;
-    if (k < K) off[k] = excl;
-    __syncthreads();
-    if (threadIdx.x == 1023) carry = excl + v;
-    __syncthreads();
-  }
-  if (threadIdx.x == 0) off[K] = carry;
+  cta_scan_counts(cnt, K, off, cur);
 }
 
 __global__ void k_cand_scatter(const uint64_t* pairs, uint64_t n_host, const uint64_t* n_dev, uint32_t K,

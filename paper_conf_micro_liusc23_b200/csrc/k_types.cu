@@ -37,43 +37,8 @@ __global__ void k_count_types(HashTable ht, uint32_t K, uint32_t* tcount, DevErr
 // single CTA exclusive scan of tcount[K] -> kto[K+1]; also zeroes cursor and checks capacity
 __global__ void __launch_bounds__(1024) k_scan_types(const uint32_t* tcount, uint32_t K, uint64_t* kto,
                                                       uint32_t* cursor, uint64_t capacity, DevErr* err) {
-  __shared__ uint64_t warp_sums[32];
-  __shared__ uint64_t carry;
-  if (threadIdx.x == 0) carry = 0;
-  __syncthreads();
-  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
-  for (uint32_t base = 0; base < K; base += 1024) {
-    uint32_t k = base + threadIdx.x;
-    uint64_t v = k < K ? tcount[k] : 0;
-    if (k < K) cursor[k] = 0;
-    uint64_t x = v;
-#pragma unroll
-    for (int o = 1; o < 32; o <<= 1) {
-      uint64_t y = __shfl_up_sync(0xffffffffu, x, o);
-      if (lane >= o) x += y;
-    }
-    if (lane == 31) warp_sums[wid] = x;
-    __syncthreads();
-    if (wid == 0) {
-      uint64_t s = warp_sums[lane];
-#pragma unroll
-      for (int o = 1; o < 32; o <<= 1) {
-        uint64_t y = __shfl_up_sync(0xffffffffu, s, o);
-        if (lane >= o) s += y;
-      }
-      warp_sums[lane] = s;
-    }
-    __syncthreads();
-    uint64_t excl = carry + (wid ? warp_sums[wid - 1] : 0) + x - v;
-    if (k < K) kto[k] = excl;
-    __syncthreads();
-    if (threadIdx.x == 1023) carry = excl + v;
-    __syncthreads();
-  }
-  if (threadIdx.x == 0) {
-    kto[K] = carry;
-    if (carry > capacity) latch(err, PHOTON_ECAPACITY, (int64_t)carry);
-  }
+  const uint64_t total = cta_scan_counts(tcount, K, kto, cursor);
+  if (threadIdx.x == 0 && total > capacity) latch(err, PHOTON_ECAPACITY, (int64_t)total);
 }
 
 __global__ void k_scatter_types(HashTable ht, uint32_t K, const uint64_t* kto, uint32_t* cursor, uint32_t* list,
