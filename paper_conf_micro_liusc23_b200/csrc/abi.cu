@@ -224,6 +224,14 @@ MatchLayout match_layout(uint32_t K, uint64_t T, uint64_t pair_cap, void* base) 
   m.mw.ulist = c.take<uint32_t>(2ull * K + 2);
   m.mw.flag = c.take<uint32_t>(4);
   m.mw.rcnt = c.take<uint32_t>(K + 2);
+  {
+    const uint64_t NB = ((uint64_t)K + 63) / 64;
+    m.mw.border = c.take<uint32_t>(NB * 64 + 64);
+    m.mw.bfs = c.take<int>((uint64_t)K + 1);
+    m.mw.bandlo = c.take<uint32_t>(NB + 1);
+    m.mw.bjobs = c.take<uint32_t>(NB + 1);
+    m.mw.bjob_off = c.take<uint64_t>(NB + 1);
+  }
   m.mw.pair_cap = pair_cap;
   m.pairs = c.take<uint64_t>(pair_cap);
   m.n_pairs = c.take<uint64_t>(1);

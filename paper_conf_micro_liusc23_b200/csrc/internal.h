@@ -102,6 +102,11 @@ struct MatchWs {
   uint32_t* ulist;     // [2K] undecided-kernel lists (resolution rounds)
   uint32_t* flag;      // [4]
   uint32_t* rcnt;      // [K+2] undecided count of each resolution round
+  uint32_t* border;    // [NB * 64] band order: sorted position -> kernel (k_match.cu)
+  int* bfs;            // [K] the sorted projections
+  uint32_t* bandlo;    // [NB] first r-block of each k-block's band
+  uint32_t* bjobs;     // [NB] filter jobs of each k-block
+  uint64_t* bjob_off;  // [NB + 1]
   uint64_t pair_cap;
 };
 cudaError_t launch_sig_build(uint32_t K, const uint64_t* kto, const uint32_t* type_key, const uint64_t* type_count,

@@ -312,7 +312,10 @@ __device__ __forceinline__ uint32_t divL(uint32_t x, uint32_t Qe, uint32_t qinv)
   return Qe == 1u ? (x >> 3) : __umulhi(x >> 3, qinv);
 }
 
-constexpr uint64_t kAlpha = 48;  // per-warp cost of a block in event units (worker balance: events + kAlpha * warps)
+#ifndef K1_ALPHA
+#define K1_ALPHA 48
+#endif
+constexpr uint64_t kAlpha = K1_ALPHA;  // per-warp cost of a block in event units (worker balance: events + kAlpha * warps)
 
 template <bool WIDE, bool GTBL, bool MARK, bool FUSED>
 __global__ void __launch_bounds__(WPC * 32, 1) k_bbv3(Args3 a) {

@@ -221,11 +221,24 @@ struct ScanArgs {
   uint32_t* cand;
   const uint64_t* cbeg;
   uint32_t* ccnt;
+  // band order (single-GPU path): kernels sorted by the projection f (band_f); tiles of the sorted order whose f
+  // ranges differ by >= thr8 are never enumerated
+  const uint32_t* order;    // [NB * FT] sorted position -> kernel (>= K: padding)
+  const uint32_t* bandlo;   // [NB] first r-block that can hold a partner of k-block kb
+  const uint64_t* job_off;  // [NB + 1] jobs before k-block kb
 };
 
 // Jobs: one k-block (FT kernels) against a run of up to FR r-blocks (rb <= kb).  S(kb) = jobs before k-block kb
 //   = sum_{y=1..kb} ceil(y / FR) = FR q(q+1)/2 + rem (q+1), q = kb / FR, rem = kb % FR.
 constexpr int FR = 8;
+constexpr uint32_t kBandMaxK = 1u << 24;  // band-ordered filter up to this K (one-CTA sort and job scan)
+#ifndef PHOTON_BAND
+#define PHOTON_BAND 1
+#endif
+#ifndef PHOTON_FRB
+#define PHOTON_FRB 4
+#endif
+constexpr int FRB = PHOTON_FRB;  // r-blocks per band job (the band's tiles are few: short jobs keep the GPU full)
 __host__ __device__ __forceinline__ uint64_t filter_jobs_before(uint64_t kb) {
   const uint64_t q = kb / FR, rem = kb % FR;
   return FR * q * (q + 1) / 2 + rem * (q + 1);
@@ -240,34 +253,125 @@ __host__ __device__ __forceinline__ uint64_t filter_jobs_before(uint64_t kb) {
 constexpr int FTP = FT + 4;  // row stride (floats) of the bin-major profile tiles
 constexpr uint32_t kFiltBuf = 1024;  // survivors kept in shared memory per job
 __device__ __forceinline__ uint32_t sad4(uint32_t a, uint32_t b, uint32_t acc) { return __vsadu4(a, b) + acc; }
+
+// Band order.  f(k) = sum_{j < 8} q_k[j] - sum_{j >= 8} q_k[j] (u8 profile) satisfies |f(k) - f(r)| <=
+// sum_j |q_k[j] - q_r[j]|, so a pair with |f(k) - f(r)| >= thr8 fails the coarse test: with the kernels sorted by f,
+// only tiles near the diagonal of the sorted order can hold survivors (C5: ~1/5 of the pairs).
+__device__ __forceinline__ int band_f(uint4 q) {
+  return (int)(__vsadu4(q.x, 0u) + __vsadu4(q.y, 0u)) - (int)(__vsadu4(q.z, 0u) + __vsadu4(q.w, 0u));
+}
+constexpr int kBandOff = 2048;  // f + kBandOff in [0, 4096)
+// one CTA: counting sort of the kernels by f (order within equal f is immaterial), padding to whole tiles
+__global__ void __launch_bounds__(1024) k_band_sort(uint32_t K, const uint32_t* __restrict__ prof8, uint32_t n_pad,
+                                                    uint32_t* __restrict__ order, int* __restrict__ fsort) {
+  __shared__ uint32_t hist[4096];
+  __shared__ uint32_t wsum[32];
+  const uint32_t tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
+  for (uint32_t i = tid; i < 4096; i += 1024) hist[i] = 0u;
+  __syncthreads();
+  for (uint32_t k = tid; k < K; k += 1024) atomicAdd(&hist[band_f(*(const uint4*)(prof8 + 4ull * k)) + kBandOff], 1u);
+  __syncthreads();
+  // exclusive scan of hist: 4 bins per thread
+  uint32_t v[4], sum = 0;
+#pragma unroll
+  for (int j = 0; j < 4; ++j) { v[j] = hist[tid * 4 + j]; sum += v[j]; }
+  uint32_t x = sum;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const uint32_t y = __shfl_up_sync(0xffffffffu, x, o);
+    if ((int)lane >= o) x += y;
+  }
+  if (lane == 31) wsum[wid] = x;
+  __syncthreads();
+  uint32_t w = wsum[lane];
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const uint32_t y = __shfl_up_sync(0xffffffffu, w, o);
+    if ((int)lane >= o) w += y;
+  }
+  uint32_t run = __shfl_sync(0xffffffffu, w, wid) - wsum[wid] + x - sum;
+  __syncthreads();
+#pragma unroll
+  for (int j = 0; j < 4; ++j) { hist[tid * 4 + j] = run; run += v[j]; }
+  __syncthreads();
+  for (uint32_t k = tid; k < K; k += 1024) {
+    const int f = band_f(*(const uint4*)(prof8 + 4ull * k));
+    const uint32_t pos = atomicAdd(&hist[f + kBandOff], 1u);
+    order[pos] = k;
+    fsort[pos] = f;
+  }
+  for (uint32_t pos = K + tid; pos < n_pad; pos += 1024) order[pos] = UINT32_MAX;
+}
+// one CTA: per k-block the first r-block whose largest f is within thr8 of the k-block's smallest f, the job count
+// ceil((kb - rb_lo + 1) / FR), and the job prefix
+__global__ void __launch_bounds__(1024) k_band_jobs(uint32_t K, uint32_t NB, const int* __restrict__ fsort, int thr8,
+                                                    uint32_t* __restrict__ bandlo, uint32_t* __restrict__ job_cnt,
+                                                    uint64_t* __restrict__ job_off) {
+  for (uint32_t kb = threadIdx.x; kb < NB; kb += 1024) {
+    const int fmin = fsort[kb * FT];
+    uint32_t lo = 0, hi = kb;  // first rb with fmax(rb) > fmin - thr8 (rb = kb always qualifies)
+    while (lo < hi) {
+      const uint32_t mid = (lo + hi) >> 1;
+      const uint32_t last = mid * FT + FT - 1 < K ? mid * FT + FT - 1 : K - 1;
+      if (fsort[last] > fmin - thr8) hi = mid; else lo = mid + 1;
+    }
+    bandlo[kb] = lo;
+    job_cnt[kb] = (kb - lo) / FRB + 1;
+  }
+  __syncthreads();
+  cta_scan_counts(job_cnt, NB, job_off, nullptr);
+}
+
+template <bool BAND>
 __global__ void __launch_bounds__(256) k_pair_filter(ScanArgs a, uint64_t job0, uint32_t kb_lo, uint32_t kb_hi) {
   const uint64_t job = job0 + blockIdx.x;
-  uint32_t lo = kb_lo, hi = kb_hi - 1;  // last kb with filter_jobs_before(kb) <= job
-  while (lo < hi) {
-    const uint32_t mid = (lo + hi + 1) >> 1;
-    if (filter_jobs_before(mid) <= job) lo = mid; else hi = mid - 1;
+  uint32_t kb, rb0, rb1;
+  if constexpr (BAND) {
+    if (job >= a.job_off[kb_hi]) return;  // the grid is sized for every tile; the band needs fewer jobs
+    uint32_t lo = 0, hi = kb_hi - 1;  // last kb with job_off[kb] <= job
+    while (lo < hi) {
+      const uint32_t mid = (lo + hi + 1) >> 1;
+      if (a.job_off[mid] <= job) lo = mid; else hi = mid - 1;
+    }
+    kb = lo;
+    rb0 = a.bandlo[kb] + (uint32_t)(job - a.job_off[kb]) * FRB;
+    rb1 = rb0 + FRB - 1 < kb ? rb0 + FRB - 1 : kb;  // inclusive
+  } else {
+    uint32_t lo = kb_lo, hi = kb_hi - 1;  // last kb with filter_jobs_before(kb) <= job
+    while (lo < hi) {
+      const uint32_t mid = (lo + hi + 1) >> 1;
+      if (filter_jobs_before(mid) <= job) lo = mid; else hi = mid - 1;
+    }
+    kb = lo;
+    rb0 = (uint32_t)(job - filter_jobs_before(kb)) * FR;
+    rb1 = rb0 + FR - 1 < kb ? rb0 + FR - 1 : kb;  // inclusive
   }
-  const uint32_t kb = lo;
-  const uint32_t rb0 = (uint32_t)(job - filter_jobs_before(kb)) * FR;
-  const uint32_t rb1 = rb0 + FR - 1 < kb ? rb0 + FR - 1 : kb;  // inclusive
+  // tile row / column -> kernel (identity, or the band order; >= K: none)
+  auto kid_of = [&](uint32_t pos) -> uint32_t { return BAND ? a.order[pos] : pos; };
 
   const uint32_t k0 = kb * FT;
   __shared__ __align__(16) float pk[16][FTP];
   __shared__ __align__(16) uint4 q8rb[2][FT];
   __shared__ uint64_t wk[FT], wrb[2][FT];
   __shared__ uint32_t okk[FT], okrb[2][FT];  // mass > 0 [P-19]
-  __shared__ uint64_t s_buf[kFiltBuf];       // the job's survivors
+  __shared__ uint32_t kidk[FT], kidr[2][FT];  // the kernels of the tile rows / columns
+  // band order: the r-block's fp32 profiles staged too (its tiles are dense in coarse survivors); row stride 17
+  __shared__ float prs[BAND ? 2 : 1][BAND ? FT * 17 : 1];
+  constexpr uint32_t NBUF_S = BAND ? 2 * kFiltBuf : kFiltBuf;  // band jobs are dense in survivors
+  __shared__ uint64_t s_buf[NBUF_S];         // the job's survivors
   __shared__ uint32_t s_n;
   __shared__ unsigned long long s_base;
-  const int tid = threadIdx.x, lane = tid & 31;
+  const int tid = threadIdx.x;
   if (tid == 0) s_n = 0;
+  const uint32_t kpad = BAND ? (kb + 1) * FT : a.K;  // rows past K (identity) / padding (band) hold no kernel
   for (int i = tid; i < FT * 16; i += 256) {
     const int row = i >> 4, j = i & 15;
-    const uint32_t k = k0 + row;
+    const uint32_t k = k0 + row < kpad ? kid_of(k0 + row) : UINT32_MAX;
     pk[j][row] = k < a.K ? a.prof[(uint64_t)k * 16 + j] : 0.f;
   }
   if (tid < FT) {
-    const uint32_t k = k0 + tid;
+    const uint32_t k = k0 + tid < kpad ? kid_of(k0 + tid) : UINT32_MAX;
+    kidk[tid] = k;
     wk[tid] = k < a.K ? a.wt[k] : 0;
     okk[tid] = k < a.K && a.mass[k] != 0;
   }
@@ -275,28 +379,35 @@ __global__ void __launch_bounds__(256) k_pair_filter(ScanArgs a, uint64_t job0, 
   uint4 qk[4];  // u8 profiles of this thread's 4 k rows
 #pragma unroll
   for (int u = 0; u < 4; ++u) {
-    const uint32_t k = k0 + i0 + u;
+    const uint32_t k = k0 + i0 + u < kpad ? kid_of(k0 + i0 + u) : UINT32_MAX;
     qk[u] = k < a.K ? *(const uint4*)(a.prof8 + (uint64_t)k * 4) : make_uint4(0, 0, 0, 0);
   }
   // register stage of one r-block: one u8 word per thread, (wt, mass != 0) for tid < FT (the fp32 r profiles are
   // read from L1 / L2 by the fine check of the rare coarse survivors only)
   uint32_t sq = 0;
   uint64_t swr = 0;
-  uint32_t sok = 0;
+  uint32_t sok = 0, srid = 0;
+  float4 spf = make_float4(0.f, 0.f, 0.f, 0.f);
   auto fetch = [&](uint32_t rb) {
     {
-      const uint32_t r = rb * FT + (tid >> 2);
+      const uint32_t r = rb * FT + (tid >> 2) < kpad ? kid_of(rb * FT + (tid >> 2)) : UINT32_MAX;
       sq = r < a.K ? a.prof8[(uint64_t)r * 4 + (tid & 3)] : 0u;
+      if (BAND && r < a.K) spf = __ldg((const float4*)(a.prof + (uint64_t)r * 16) + (tid & 3));
     }
     if (tid < FT) {
-      const uint32_t r = rb * FT + tid;
+      const uint32_t r = rb * FT + tid < kpad ? kid_of(rb * FT + tid) : UINT32_MAX;
+      srid = r;
       swr = r < a.K ? a.wt[r] : 0;
       sok = r < a.K && a.mass[r] != 0;
     }
   };
   auto store = [&](int buf) {
     ((uint32_t*)q8rb[buf])[tid] = sq;
-    if (tid < FT) { wrb[buf][tid] = swr; okrb[buf][tid] = sok; }
+    if (BAND) {
+      float* d = &prs[BAND ? buf : 0][(tid >> 2) * 17 + (tid & 3) * 4];
+      d[0] = spf.x; d[1] = spf.y; d[2] = spf.z; d[3] = spf.w;
+    }
+    if (tid < FT) { wrb[buf][tid] = swr; okrb[buf][tid] = sok; kidr[buf][tid] = srid; }
   };
   fetch(rb0);
   store(0);
@@ -307,6 +418,7 @@ __global__ void __launch_bounds__(256) k_pair_filter(ScanArgs a, uint64_t job0, 
     const uint4* q8r = q8rb[cur];
     const uint64_t* wr = wrb[cur];
     const uint32_t* okr = okrb[cur];
+    const uint32_t* ridr = kidr[cur];
     const uint32_t r0 = rb * FT;
     // coarse level for all 16 pairs (four VABSDIFF4.ACC each); the per-pair eligibility rules only for survivors
     uint32_t keep = 0;  // bit 4u+v
@@ -321,21 +433,27 @@ __global__ void __launch_bounds__(256) k_pair_filter(ScanArgs a, uint64_t job0, 
     }
     for (uint32_t m = keep; m; m &= m - 1) {
       const int bit = __ffs(m) - 1, i = i0 + (bit >> 2), j = j0 + (bit & 3);
-      const uint32_t k = k0 + i, r = r0 + j;
       const uint64_t Wk = wk[i], Wr = wr[j];
-      const bool ok = okr[j] && r < k && k >= a.k_lo && k < a.k_hi && okk[i] &&
-                      (Wk == Wr || (Wk < Wr ? Wk : Wr) >= a.p.n_cores);  // [P-10]
+      // each unordered pair once: the identity order needs r < k; the band order takes the tile triangle (sorted
+      // position of the row > that of the column) and either launch order
+      const bool tri = BAND ? (rb < kb || j < i) : (r0 + j < k0 + i && k0 + i >= a.k_lo && k0 + i < a.k_hi);
+      const bool ok = okr[j] && tri && okk[i] && (Wk == Wr || (Wk < Wr ? Wk : Wr) >= a.p.n_cores);  // [P-10]
       if (!ok) keep &= ~(1u << bit);
     }
     // fine level for the coarse survivors: fp32 profile distance
     for (uint32_t m = keep; m; m &= m - 1) {
       const int bit = __ffs(m) - 1, i = i0 + (bit >> 2), j = j0 + (bit & 3);
-      const float4* rp = (const float4*)(a.prof + (uint64_t)(r0 + j) * 16);  // r < K (eligible)
       float pr[16];
+      if (BAND) {
 #pragma unroll
-      for (int q = 0; q < 4; ++q) {
-        const float4 v = __ldg(rp + q);
-        pr[4 * q] = v.x; pr[4 * q + 1] = v.y; pr[4 * q + 2] = v.z; pr[4 * q + 3] = v.w;
+        for (int b = 0; b < 16; ++b) pr[b] = prs[BAND ? cur : 0][j * 17 + b];
+      } else {
+        const float4* rp = (const float4*)(a.prof + (uint64_t)(r0 + j) * 16);  // r < K (eligible)
+#pragma unroll
+        for (int q = 0; q < 4; ++q) {
+          const float4 v = __ldg(rp + q);
+          pr[4 * q] = v.x; pr[4 * q + 1] = v.y; pr[4 * q + 2] = v.z; pr[4 * q + 3] = v.w;
+        }
       }
       float d = 0.f;
 #pragma unroll
@@ -346,10 +464,15 @@ __global__ void __launch_bounds__(256) k_pair_filter(ScanArgs a, uint64_t job0, 
     // latency would hold the whole CTA at the next barrier, inside the loop); a full list spills directly
     for (uint32_t m = keep; m; m &= m - 1) {
       const int bit = __ffs(m) - 1;
-      const uint32_t k = k0 + i0 + (bit >> 2), r = r0 + j0 + (bit & 3);
+      uint32_t k = k0 + i0 + (bit >> 2), r = r0 + j0 + (bit & 3);
+      if (BAND) {
+        const uint32_t x = kidk[i0 + (bit >> 2)], y = ridr[j0 + (bit & 3)];
+        k = x > y ? x : y;
+        r = x > y ? y : x;
+      }
       const uint64_t pr = ((uint64_t)k << 32) | r;
       const uint32_t sp = atomicAdd(&s_n, 1u);
-      if (sp < kFiltBuf) {
+      if (sp < NBUF_S) {
         s_buf[sp] = pr;
       } else {
         const unsigned long long pos = atomicAdd((unsigned long long*)a.n_maybe, 1ull);
@@ -361,7 +484,7 @@ __global__ void __launch_bounds__(256) k_pair_filter(ScanArgs a, uint64_t job0, 
     __syncthreads();
   }
   // flush the job's shared list: one global atomic per CTA
-  const uint32_t ns = s_n < kFiltBuf ? s_n : kFiltBuf;
+  const uint32_t ns = s_n < NBUF_S ? s_n : NBUF_S;
   if (tid == 0 && ns) s_base = atomicAdd((unsigned long long*)a.n_maybe, (unsigned long long)ns);
   __syncthreads();
   for (uint32_t i = tid; i < ns; i += 256) {
@@ -751,7 +874,20 @@ ScanArgs scan_args(uint32_t K, uint32_t k_lo, uint32_t k_hi, const uint64_t* kto
 void launch_filter(const ScanArgs& a, cudaStream_t s) {
   const uint32_t kb_hi = (uint32_t)ceil_div(a.k_hi, FT), kb_lo = a.k_lo / FT;
   const uint64_t j0 = filter_jobs_before(kb_lo), j1 = filter_jobs_before(kb_hi);
-  if (j1 > j0) note_launch(), k_pair_filter<<<(unsigned)(j1 - j0), 256, 0, s>>>(a, j0, kb_lo, kb_hi);
+  if (j1 > j0) note_launch(), k_pair_filter<false><<<(unsigned)(j1 - j0), 256, 0, s>>>(a, j0, kb_lo, kb_hi);
+}
+// the whole triangle through the band order: sort by f, the band's jobs, then the filter over those jobs only (the
+// grid is sized for every tile of the triangle; the jobs past the band's count return at once)
+void launch_filter_band(ScanArgs a, const MatchWs& mw, cudaStream_t s) {
+  const uint32_t K = a.K, NB = (uint32_t)ceil_div(K, FT);
+  if (NB == 0) return;
+  note_launch(), k_band_sort<<<1, 1024, 0, s>>>(K, a.prof8, NB * FT, mw.border, mw.bfs);
+  note_launch(), k_band_jobs<<<1, 1024, 0, s>>>(K, NB, mw.bfs, (int)a.thr8, mw.bandlo, mw.bjobs, mw.bjob_off);
+  a.order = mw.border;
+  a.bandlo = mw.bandlo;
+  a.job_off = mw.bjob_off;
+  const uint64_t jobs = (uint64_t)(NB / FRB) * (NB / FRB + 1) / 2 * FRB + (uint64_t)(NB % FRB) * (NB / FRB + 1);
+  note_launch(), k_pair_filter<true><<<(unsigned)jobs, 256, 0, s>>>(a, 0, 0, NB);
 }
 // the fused path's survivors bucketed by k into `pairs` (free there: close pairs go to cand segments)
 void launch_bucket(uint32_t K, const MatchWs& mw, uint64_t* pairs, DevErr* err, int num_sms, cudaStream_t s) {
@@ -803,7 +939,8 @@ cudaError_t launch_analyse_filter(uint32_t K, const uint64_t* kto, const uint32_
                                                                                        err);
   cudaEventRecord(prof_done, sb);
   const ScanArgs a = scan_args(K, 0, K, kto, nullptr, mass, wt, p, mw, err);
-  launch_filter(a, sb);
+  if (PHOTON_BAND && K <= kBandMaxK) launch_filter_band(a, mw, sb);  // f in [-2040, 2040]: the counting sort's 4096 bins
+  else launch_filter(a, sb);
   launch_bucket(K, mw, pairs, err, num_sms, sb);
   return cudaGetLastError();
 }
