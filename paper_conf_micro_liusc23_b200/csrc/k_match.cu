@@ -583,7 +583,7 @@ __device__ double group_dfp(const uint64_t* __restrict__ sig, const float* __res
 // The fp64 screen decides every pair whose distance is farther than its error bound from theta; the rest (ties
 // within ~1e-9) take the exact u128 sum.
 #ifndef PHOTON_XG
-#define PHOTON_XG 16  // lanes per pair (profiling builds may override)
+#define PHOTON_XG 8  // lanes per pair (profiling builds may override)
 #endif
 constexpr int XG = PHOTON_XG;
 __global__ void __launch_bounds__(256) k_pair_exact(ScanArgs a, uint64_t* pairs, uint64_t pair_cap,
