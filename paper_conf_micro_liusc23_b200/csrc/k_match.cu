@@ -226,6 +226,7 @@ struct ScanArgs {
   const uint32_t* order;    // [NB * FT] sorted position -> kernel (>= K: padding)
   const uint32_t* bandlo;   // [NB] first r-block that can hold a partner of k-block kb
   const uint64_t* job_off;  // [NB + 1] jobs before k-block kb
+  uint32_t* kcnt;           // survivors per k (the bucketing's counts), or nullptr
 };
 
 // Jobs: one k-block (FT kernels) against a run of up to FR r-blocks (rb <= kb).  S(kb) = jobs before k-block kb
@@ -262,8 +263,8 @@ __device__ __forceinline__ int band_f(uint4 q) {
 }
 constexpr int kBandOff = 2048;  // f + kBandOff in [0, 4096)
 // one CTA: counting sort of the kernels by f (order within equal f is immaterial), padding to whole tiles
-__global__ void __launch_bounds__(1024) k_band_sort(uint32_t K, const uint32_t* __restrict__ prof8, uint32_t n_pad,
-                                                    uint32_t* __restrict__ order, int* __restrict__ fsort) {
+__device__ __forceinline__ void band_sort_body(uint32_t K, const uint32_t* __restrict__ prof8, uint32_t n_pad,
+                                               uint32_t* __restrict__ order, int* __restrict__ fsort) {
   __shared__ uint32_t hist[4096];
   __shared__ uint32_t wsum[32];
   const uint32_t tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
@@ -302,11 +303,21 @@ __global__ void __launch_bounds__(1024) k_band_sort(uint32_t K, const uint32_t* 
   }
   for (uint32_t pos = K + tid; pos < n_pad; pos += 1024) order[pos] = UINT32_MAX;
 }
+__device__ void band_jobs(uint32_t K, uint32_t NB, const int* __restrict__ fsort, int thr8, uint32_t* bandlo,
+                          uint32_t* job_cnt, uint64_t* job_off);
+// the sort and the band's jobs in one CTA (fsort is written and read by the same block: ordered by the barrier)
+__global__ void __launch_bounds__(1024) k_band_sort_jobs(uint32_t K, const uint32_t* __restrict__ prof8,
+                                                         uint32_t NB, uint32_t* __restrict__ order, int* fsort,
+                                                         int thr8, uint32_t* bandlo, uint32_t* job_cnt,
+                                                         uint64_t* job_off) {
+  band_sort_body(K, prof8, NB * FT, order, fsort);
+  __syncthreads();
+  band_jobs(K, NB, fsort, thr8, bandlo, job_cnt, job_off);
+}
 // one CTA: per k-block the first r-block whose largest f is within thr8 of the k-block's smallest f, the job count
 // ceil((kb - rb_lo + 1) / FR), and the job prefix
-__global__ void __launch_bounds__(1024) k_band_jobs(uint32_t K, uint32_t NB, const int* __restrict__ fsort, int thr8,
-                                                    uint32_t* __restrict__ bandlo, uint32_t* __restrict__ job_cnt,
-                                                    uint64_t* __restrict__ job_off) {
+__device__ void band_jobs(uint32_t K, uint32_t NB, const int* __restrict__ fsort, int thr8, uint32_t* bandlo,
+                          uint32_t* job_cnt, uint64_t* job_off) {
   for (uint32_t kb = threadIdx.x; kb < NB; kb += 1024) {
     const int fmin = fsort[kb * FT];
     uint32_t lo = 0, hi = kb;  // first rb with fmax(rb) > fmin - thr8 (rb = kb always qualifies)
@@ -476,8 +487,12 @@ __global__ void __launch_bounds__(256) k_pair_filter(ScanArgs a, uint64_t job0, 
         s_buf[sp] = pr;
       } else {
         const unsigned long long pos = atomicAdd((unsigned long long*)a.n_maybe, 1ull);
-        if (pos < a.cap) a.maybe[pos] = pr;
-        else latch(a.err, PHOTON_ECAPACITY, (int64_t)pos);
+        if (pos < a.cap) {
+          a.maybe[pos] = pr;
+          if (a.kcnt) atomicAdd(&a.kcnt[k], 1u);
+        } else {
+          latch(a.err, PHOTON_ECAPACITY, (int64_t)pos);
+        }
       }
     }
     if (rb < rb1) store(cur ^ 1);  // that buffer was last read before the previous barrier
@@ -489,8 +504,12 @@ __global__ void __launch_bounds__(256) k_pair_filter(ScanArgs a, uint64_t job0, 
   __syncthreads();
   for (uint32_t i = tid; i < ns; i += 256) {
     const unsigned long long pos = s_base + i;
-    if (pos < a.cap) a.maybe[pos] = s_buf[i];
-    else latch(a.err, PHOTON_ECAPACITY, (int64_t)pos);
+    if (pos < a.cap) {
+      a.maybe[pos] = s_buf[i];
+      if (a.kcnt) atomicAdd(&a.kcnt[(uint32_t)(s_buf[i] >> 32)], 1u);
+    } else {
+      latch(a.err, PHOTON_ECAPACITY, (int64_t)pos);
+    }
   }
 }
 
@@ -881,8 +900,8 @@ void launch_filter(const ScanArgs& a, cudaStream_t s) {
 void launch_filter_band(ScanArgs a, const MatchWs& mw, cudaStream_t s) {
   const uint32_t K = a.K, NB = (uint32_t)ceil_div(K, FT);
   if (NB == 0) return;
-  note_launch(), k_band_sort<<<1, 1024, 0, s>>>(K, a.prof8, NB * FT, mw.border, mw.bfs);
-  note_launch(), k_band_jobs<<<1, 1024, 0, s>>>(K, NB, mw.bfs, (int)a.thr8, mw.bandlo, mw.bjobs, mw.bjob_off);
+  note_launch(), k_band_sort_jobs<<<1, 1024, 0, s>>>(K, a.prof8, NB, mw.border, mw.bfs, (int)a.thr8, mw.bandlo,
+                                                     mw.bjobs, mw.bjob_off);
   a.order = mw.border;
   a.bandlo = mw.bandlo;
   a.job_off = mw.bjob_off;
@@ -890,11 +909,14 @@ void launch_filter_band(ScanArgs a, const MatchWs& mw, cudaStream_t s) {
   note_launch(), k_pair_filter<true><<<(unsigned)jobs, 256, 0, s>>>(a, 0, 0, NB);
 }
 // the fused path's survivors bucketed by k into `pairs` (free there: close pairs go to cand segments)
-void launch_bucket(uint32_t K, const MatchWs& mw, uint64_t* pairs, DevErr* err, int num_sms, cudaStream_t s) {
+void launch_bucket(uint32_t K, const MatchWs& mw, uint64_t* pairs, DevErr* err, int num_sms, cudaStream_t s,
+                   bool counted = false) {
   const unsigned gb = (unsigned)umin64(ceil_div(mw.pair_cap, 256), (uint64_t)num_sms * 64);
-  cudaMemsetAsync(mw.cand_cnt, 0, sizeof(uint32_t) * K, s);
   cudaMemsetAsync(mw.close_cnt, 0, sizeof(uint32_t) * K, s);
-  note_launch(), k_cand_count<<<gb, 256, 0, s>>>(mw.maybe, mw.pair_cap, mw.n_maybe, K, mw.cand_cnt, err);
+  if (!counted) {  // else the filter counted its survivors per k
+    cudaMemsetAsync(mw.cand_cnt, 0, sizeof(uint32_t) * K, s);
+    note_launch(), k_cand_count<<<gb, 256, 0, s>>>(mw.maybe, mw.pair_cap, mw.n_maybe, K, mw.cand_cnt, err);
+  }
   note_launch(), k_cand_scan<<<1, 1024, 0, s>>>(mw.cand_cnt, K, mw.cand_off, mw.cand_cur);
   note_launch(), k_pair_bucket<<<gb, 256, 0, s>>>(mw.maybe, mw.pair_cap, mw.n_maybe, K, mw.cand_off, mw.cand_cur,
                                                   pairs);
@@ -938,10 +960,12 @@ cudaError_t launch_analyse_filter(uint32_t K, const uint64_t* kto, const uint32_
                                                                                        mw.prof, mw.invn, mw.prof8,
                                                                                        err);
   cudaEventRecord(prof_done, sb);
-  const ScanArgs a = scan_args(K, 0, K, kto, nullptr, mass, wt, p, mw, err);
+  ScanArgs a = scan_args(K, 0, K, kto, nullptr, mass, wt, p, mw, err);
+  a.kcnt = mw.cand_cnt;  // the filter counts its survivors per k (no separate count pass)
+  cudaMemsetAsync(mw.cand_cnt, 0, sizeof(uint32_t) * K, sb);
   if (PHOTON_BAND && K <= kBandMaxK) launch_filter_band(a, mw, sb);  // f in [-2040, 2040]: the counting sort's 4096 bins
   else launch_filter(a, sb);
-  launch_bucket(K, mw, pairs, err, num_sms, sb);
+  launch_bucket(K, mw, pairs, err, num_sms, sb, true);
   return cudaGetLastError();
 }
 cudaError_t launch_analyse_sigf(uint32_t K, const photon_types& types, uint64_t* sig, const MatchWs& mw,
