@@ -175,7 +175,7 @@ def run_reference(args):
     sample = f"kernels [0,{k1}) of {CONFIG_DESC.get(args.config)}: {tr.n_events} events, {tr.n_warps} warps"
     line = {"impl": "reference", "metric": METRIC, "value": value, "unit": "events/s", "n_gpus": args.gpus,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True,
-            "scaling": "weak", "vs_baseline": None, "dtype": "u16/u32/u64 integer (u128 exact compares)",
+            "scaling": "strong", "vs_baseline": None, "dtype": "u16/u32/u64 integer (u128 exact compares)",
             "data": "synthetic (tracegen, seeded)",
             "config": {"workload": CONFIG_DESC.get(args.config), "sample": sample, "theta": args.theta},
             "cpu_baseline": {"value": value, "unit": "events/s", "cores": 1, "kind": "oracle", "sample": sample},
