@@ -2,6 +2,7 @@
 #pragma once
 #include <cuda_runtime.h>
 #include <stdint.h>
+#include <cstdio>
 
 #include <atomic>
 
@@ -19,6 +20,28 @@ inline std::atomic<uint64_t>& launch_counter() {
   return n;
 }
 inline void note_launch() { launch_counter().fetch_add(1, std::memory_order_relaxed); }
+
+// ---- debug build (PHOTON_DEBUG=1, libphoton_debug.so): device-side bounds checks ------------------------------
+// compute-sanitizer is disabled on the GPU pool, so the debug library checks the accesses whose bounds are not
+// evident from the code (computed shared-memory cell / table / stage addresses, bucket cursors, scatter positions):
+// a failed check prints its site and traps, which the tests see as a CUDA error.  Compiled out otherwise.
+#ifndef PHOTON_DEBUG
+#define PHOTON_DEBUG 0
+#endif
+#if PHOTON_DEBUG
+#define PHOTON_DCHECK(cond, what, v)                                                                       \
+  do {                                                                                                     \
+    if (!(cond)) {                                                                                         \
+      printf("PHOTON_DCHECK failed: %s (%s:%d) value %llu\n", what, __FILE__, __LINE__,                    \
+             (unsigned long long)(v));                                                                     \
+      __trap();                                                                                            \
+    }                                                                                                      \
+  } while (0)
+#else
+#define PHOTON_DCHECK(cond, what, v) \
+  do {                               \
+  } while (0)
+#endif
 
 typedef unsigned __int128 u128;
 typedef __int128 i128;

@@ -347,6 +347,13 @@ __global__ void __launch_bounds__(WPC * 32, 1) k_bbv3(Args3 a) {
     return;
   }
   clear_cells<WIDE>(cw);
+  // every RED lands in this worker's 64 columns of its row array (debug build: checked)
+  auto red = [&](uint32_t ad, uint32_t v) {
+    PHOTON_DCHECK((ad - (cw - (wid % GRP) * NCOL * 4)) < ROWS * ROWB &&
+                      (((ad - (cw - (wid % GRP) * NCOL * 4)) & (ROWB - 1)) - (wid % GRP) * NCOL * 4) < NCOL * 4,
+                  "K1 cell address outside the worker's columns", ad);
+    red_add(ad, v);
+  };
   if (FUSED) pool_init(wm);
   if (lane == 0) {
     mbar_init(&wm->mbar[0], 1);
@@ -573,6 +580,7 @@ __global__ void __launch_bounds__(WPC * 32, 1) k_bbv3(Args3 a) {
 #endif
           const uint32_t p0 = (t0 * Qe + kk) * 8u;
           raw |= (vnx.x | vnx.y) | (vnx.z | vnx.w);
+          PHOTON_DCHECK(t0 * Qe + kk + 1u <= CW, "K1 stage read past the worker's buffer", t0 * Qe + kk + 1u);
 #if K1_VNX
           vnx = sb4[kk + 1];  // one word past the lane's range: always inside the allocation (unused at the end)
 #else
@@ -589,16 +597,17 @@ __global__ void __launch_bounds__(WPC * 32, 1) k_bbv3(Args3 a) {
             const uint32_t cv1 = (cbx & ~(uint32_t)(bm >> 32)) | (cby & (uint32_t)(bm >> 32));
 #pragma unroll
             for (int j = 0; j < 8; ++j)
-              red_add(__byte_perm(j < 4 ? cv0 : cv1, cw, 0x7650u + (j & 3)) | (tv[j] & M::ROFF), M::val(tv[j]));
+              red(__byte_perm(j < 4 ? cv0 : cv1, cw, 0x7650u + (j & 3)) | (tv[j] & M::ROFF), M::val(tv[j]));
 #else
 #pragma unroll
-            for (int j = 0; j < 8; ++j) red_add(((uint32_t)j < mcut ? col : coln) | (tv[j] & M::ROFF), M::val(tv[j]));
+            for (int j = 0; j < 8; ++j) red(((uint32_t)j < mcut ? col : coln) | (tv[j] & M::ROFF), M::val(tv[j]));
 #endif
             if (nb <= p0 + 8u) {
               ++u;
               col = coln;
               coln = pcol(u + 1);
               nb = nb2;
+              PHOTON_DCHECK(u + 2u < 40u, "K1 warp index past rel[]", u);
               nb2 = wm->rel[u + 2];
 #if K1_PRMT
               cbx = cby;
@@ -616,7 +625,7 @@ __global__ void __launch_bounds__(WPC * 32, 1) k_bbv3(Args3 a) {
               const uint32_t pos = p0 + j;
               const bool in = pos >= r && pos < e;
               while (in && pos >= wm->rel[u + 1] && u + 1 < nw) ++u;
-              red_add((in ? (u == myfw ? cw + t0 * 4u : pcol(u)) : scr) | (tv[j] & M::ROFF), M::val(tv[j]));
+              red((in ? (u == myfw ? cw + t0 * 4u : pcol(u)) : scr) | (tv[j] & M::ROFF), M::val(tv[j]));
             }
             while (p0 + 8u < e && wm->rel[u + 1] <= p0 + 8u && u + 1 < nw) ++u;  // the next word's warp
             col = u == myfw ? cw + t0 * 4u : pcol(u);

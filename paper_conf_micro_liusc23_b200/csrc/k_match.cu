@@ -630,7 +630,9 @@ __global__ void __launch_bounds__(256) k_pair_exact(ScanArgs a, uint64_t* pairs,
     if (act && close && (threadIdx.x & (XG - 1)) == 0) {
       const unsigned long long pos = atomicAdd((unsigned long long*)n_pairs, 1ull);
       if (a.cand) {  // fused path: the close r into k's segment of the k-bucketed survivors
-        a.cand[a.cbeg[k] + atomicAdd(&a.ccnt[k], 1u)] = r;
+        const uint64_t pos_c = a.cbeg[k] + atomicAdd(&a.ccnt[k], 1u);
+        PHOTON_DCHECK(pos_c < a.cbeg[k + 1], "close pair past k's candidate segment", k);
+        a.cand[pos_c] = r;
       } else if (pos < pair_cap) {
         pairs[pos] = pr;
       } else {
@@ -667,7 +669,9 @@ __global__ void k_cand_scatter(const uint64_t* pairs, uint64_t n_host, const uin
   if (i >= n) return;
   uint32_t k = (uint32_t)(pairs[i] >> 32), r = (uint32_t)pairs[i];
   if (k >= K || r >= k) return;
-  cand[off[k] + atomicAdd(&cur[k], 1u)] = r;
+  const uint64_t pos = off[k] + atomicAdd(&cur[k], 1u);
+  PHOTON_DCHECK(pos < off[k + 1], "candidate past k's segment", k);
+  cand[pos] = r;
 }
 
 // the filter survivors bucketed by k (stable order inside a bucket is immaterial): the exact check then visits
@@ -678,7 +682,11 @@ __global__ void k_pair_bucket(const uint64_t* pairs, uint64_t n_host, const uint
   for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x) {
     const uint64_t pr = pairs[i];
     const uint32_t k = (uint32_t)(pr >> 32);
-    if (k < K) out[off[k] + atomicAdd(&cur[k], 1u)] = pr;
+    if (k < K) {
+      const uint64_t pos = off[k] + atomicAdd(&cur[k], 1u);
+      PHOTON_DCHECK(pos < off[k + 1], "survivor past k's bucket", k);
+      out[pos] = pr;
+    }
   }
 }
 

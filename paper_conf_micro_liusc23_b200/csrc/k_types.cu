@@ -48,6 +48,7 @@ __global__ void k_scatter_types(HashTable ht, uint32_t K, const uint64_t* kto, u
   uint32_t k = ht.kern[i];
   if (k >= K) return;
   uint64_t pos = kto[k] + atomicAdd(&cursor[k], 1u);
+  PHOTON_DCHECK(pos < kto[k + 1], "type slot past its kernel's list", k);
   if (pos < capacity) list[pos] = (uint32_t)i;
 }
 
