@@ -591,7 +591,7 @@ int photon_analyse(photon_ctx* ctx, const photon_trace* t, void* gws, size_t gws
     ProfScope ps(ctx, PHOTON_PROF_CANON, s);
     CK(launch_entries_insert(g.ep, g.h.ht, err, ctx->num_sms, s), "insert");
     CK(launch_canon_lists(g.h.ht, K, *out, g.h.cw, err, s), "canon");
-    // fork 1: the filter profiles, the pair filter and its bucketing need only the unsorted table and its lists
+    // fork 1: the filter profiles, the pair filter and its candidate segments need only the unsorted table and its lists
     CK(cudaEventRecord(e_lists, s), "event");
     CK(cudaStreamWaitEvent(sb, e_lists, 0), "event");
     CK(launch_analyse_filter(K, out->kernel_type_off, g.h.cw.list, g.h.ht, m.mass, warps_total, params, m.mw, m.pairs,
@@ -609,7 +609,7 @@ int photon_analyse(photon_ctx* ctx, const photon_trace* t, void* gws, size_t gws
     ProfScope ps(ctx, PHOTON_PROF_SCAN, s);
     CK(cudaStreamWaitEvent(s, e_prof, 0), "event");  // 1/N
     CK(launch_analyse_sigf(K, *out, m.sig, m.mw, s), "sigf");
-    CK(cudaStreamWaitEvent(s, e_filt, 0), "event");  // the bucketed survivors
+    CK(cudaStreamWaitEvent(s, e_filt, 0), "event");  // the filter survivors and their segments
     CK(launch_analyse_exact(K, out->kernel_type_off, m.sig, m.mass, warps_total, params, m.mw, m.pairs,
                             m.mw.pair_cap, m.n_pairs, m.err, ctx->num_sms, s),
        "exact");

@@ -226,7 +226,7 @@ struct ScanArgs {
   const uint32_t* order;    // [NB * FT] sorted position -> kernel (>= K: padding)
   const uint32_t* bandlo;   // [NB] first r-block that can hold a partner of k-block kb
   const uint64_t* job_off;  // [NB + 1] jobs before k-block kb
-  uint32_t* kcnt;           // survivors per k (the bucketing's counts), or nullptr
+  uint32_t* kcnt;           // survivors per k (the sizes of the candidate segments), or nullptr
 };
 
 // Jobs: one k-block (FT kernels) against a run of up to FR r-blocks (rb <= kb).  S(kb) = jobs before k-block kb
@@ -629,7 +629,7 @@ __global__ void __launch_bounds__(256) k_pair_exact(ScanArgs a, uint64_t* pairs,
     }
     if (act && close && (threadIdx.x & (XG - 1)) == 0) {
       const unsigned long long pos = atomicAdd((unsigned long long*)n_pairs, 1ull);
-      if (a.cand) {  // fused path: the close r into k's segment of the k-bucketed survivors
+      if (a.cand) {  // fused path: the close r into k's candidate segment (sized by k's filter survivors)
         const uint64_t pos_c = a.cbeg[k] + atomicAdd(&a.ccnt[k], 1u);
         PHOTON_DCHECK(pos_c < a.cbeg[k + 1], "close pair past k's candidate segment", k);
         a.cand[pos_c] = r;
@@ -674,21 +674,6 @@ __global__ void k_cand_scatter(const uint64_t* pairs, uint64_t n_host, const uin
   cand[pos] = r;
 }
 
-// the filter survivors bucketed by k (stable order inside a bucket is immaterial): the exact check then visits
-// every candidate of one k back to back, so g_k stays in L1 for the run
-__global__ void k_pair_bucket(const uint64_t* pairs, uint64_t n_host, const uint64_t* n_dev, uint32_t K,
-                              const uint64_t* off, uint32_t* cur, uint64_t* out) {
-  uint64_t n = pair_count(n_host, n_dev);
-  for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x) {
-    const uint64_t pr = pairs[i];
-    const uint32_t k = (uint32_t)(pr >> 32);
-    if (k < K) {
-      const uint64_t pos = off[k] + atomicAdd(&cur[k], 1u);
-      PHOTON_DCHECK(pos < off[k + 1], "survivor past k's bucket", k);
-      out[pos] = pr;
-    }
-  }
-}
 
 // Fixed point of the launch-order rule (small K, one CTA): state 1 = representative, 2 = matched, 0 = undecided.
 // Round-synchronous: every round reads the states of the previous round only (barrier), decides each undecided
@@ -916,9 +901,9 @@ void launch_filter_band(ScanArgs a, const MatchWs& mw, cudaStream_t s) {
   const uint64_t jobs = (uint64_t)(NB / FRB) * (NB / FRB + 1) / 2 * FRB + (uint64_t)(NB % FRB) * (NB / FRB + 1);
   note_launch(), k_pair_filter<true><<<(unsigned)jobs, 256, 0, s>>>(a, 0, 0, NB);
 }
-// the fused path's survivors bucketed by k into `pairs` (free there: close pairs go to cand segments)
-void launch_bucket(uint32_t K, const MatchWs& mw, uint64_t* pairs, DevErr* err, int num_sms, cudaStream_t s,
-                   bool counted = false) {
+// the fused path's candidate segments: one per k, sized by k's filter survivors (the exact check writes the close
+// ones into it)
+void launch_segments(uint32_t K, const MatchWs& mw, DevErr* err, int num_sms, cudaStream_t s, bool counted = false) {
   const unsigned gb = (unsigned)umin64(ceil_div(mw.pair_cap, 256), (uint64_t)num_sms * 64);
   cudaMemsetAsync(mw.close_cnt, 0, sizeof(uint32_t) * K, s);
   if (!counted) {  // else the filter counted its survivors per k
@@ -926,14 +911,11 @@ void launch_bucket(uint32_t K, const MatchWs& mw, uint64_t* pairs, DevErr* err, 
     note_launch(), k_cand_count<<<gb, 256, 0, s>>>(mw.maybe, mw.pair_cap, mw.n_maybe, K, mw.cand_cnt, err);
   }
   note_launch(), k_cand_scan<<<1, 1024, 0, s>>>(mw.cand_cnt, K, mw.cand_off, mw.cand_cur);
-  note_launch(), k_pair_bucket<<<gb, 256, 0, s>>>(mw.maybe, mw.pair_cap, mw.n_maybe, K, mw.cand_off, mw.cand_cur,
-                                                  pairs);
 }
 void launch_exact(ScanArgs a, bool fused, const MatchWs& mw, uint64_t* pairs, uint64_t pair_cap, uint64_t* n_pairs,
                   int num_sms, cudaStream_t s) {
   if (fused) {
-    a.maybe = pairs;
-    a.cand = mw.cand;
+    a.cand = mw.cand;  // the survivors are checked in the filter's order (band tiles keep a k-block's pairs together)
     a.cbeg = mw.cand_off;
     a.ccnt = mw.close_cnt;
   }
@@ -953,12 +935,12 @@ cudaError_t launch_match_scan(uint32_t K, const uint64_t* kto, const uint64_t* s
                                                                                   mw.invn, mw.prof8, mw.sigf);
   const ScanArgs a = scan_args(K, k_lo, k_hi, kto, sig, mass, wt, p, mw, err);
   launch_filter(a, s);
-  if (fused) launch_bucket(K, mw, pairs, err, num_sms, s);
+  if (fused) launch_segments(K, mw, err, num_sms, s);
   launch_exact(a, fused, mw, pairs, pair_cap, n_pairs, num_sms, s);
   return cudaGetLastError();
 }
 
-// photon_analyse's split: A3 profiles + filter + bucketing from the unsorted table (stream sb), then -- after the
+// photon_analyse's split: A3 profiles + filter + candidate segments from the unsorted table (stream sb), then -- after the
 // sort, on the main stream -- g / N in row order and the exact check
 cudaError_t launch_analyse_filter(uint32_t K, const uint64_t* kto, const uint32_t* list, const HashTable& ht,
                                   uint64_t* mass, const uint64_t* wt, photon_match_params p, const MatchWs& mw,
@@ -973,7 +955,7 @@ cudaError_t launch_analyse_filter(uint32_t K, const uint64_t* kto, const uint32_
   cudaMemsetAsync(mw.cand_cnt, 0, sizeof(uint32_t) * K, sb);
   if (PHOTON_BAND && K <= kBandMaxK) launch_filter_band(a, mw, sb);  // f in [-2040, 2040]: the counting sort's 4096 bins
   else launch_filter(a, sb);
-  launch_bucket(K, mw, pairs, err, num_sms, sb, true);
+  launch_segments(K, mw, err, num_sms, sb, true);
   return cudaGetLastError();
 }
 cudaError_t launch_analyse_sigf(uint32_t K, const photon_types& types, uint64_t* sig, const MatchWs& mw,
@@ -995,7 +977,7 @@ cudaError_t launch_match_resolve(uint32_t K, const uint64_t* kto, const uint64_t
                                  const uint64_t* n_pairs_dev, const MatchWs& mw, int64_t* match, double* match_dist,
                                  DevErr* err, int num_sms, cudaStream_t s, bool fused) {
   if (K == 0) return cudaSuccess;
-  // candidate segments: fused -- written by k_pair_exact into the k-buckets (cand_off, close_cnt); else built here
+  // candidate segments: fused -- written by k_pair_exact into k's segment (cand_off, close_cnt); else built here
   // from the pair list (cand_off, cand_cnt)
   const uint32_t* ccnt = fused ? mw.close_cnt : mw.cand_cnt;
   if (!fused) cudaMemsetAsync(mw.cand_cnt, 0, sizeof(uint32_t) * K, s);
