@@ -262,15 +262,42 @@ __device__ __forceinline__ int band_f(uint4 q) {
   return (int)(__vsadu4(q.x, 0u) + __vsadu4(q.y, 0u)) - (int)(__vsadu4(q.z, 0u) + __vsadu4(q.w, 0u));
 }
 constexpr int kBandOff = 2048;  // f + kBandOff in [0, 4096)
-// one CTA: counting sort of the kernels by f (order within equal f is immaterial), padding to whole tiles
-__device__ __forceinline__ void band_sort_body(uint32_t K, const uint32_t* __restrict__ prof8, uint32_t n_pad,
-                                               uint32_t* __restrict__ order, int* __restrict__ fsort) {
+// One CTA: counting sort of the kernels by f (order within equal f is immaterial; padding to whole tiles), then per
+// k-block the first r-block whose largest f is within thr8 of the block's smallest f, the job count
+// ceil((kb - rb_lo + 1) / FRB) and the job prefix.  The projections are read once (8 kernels per thread in flight)
+// and kept, with the sorted ones, in shared memory when K fits (kBandSmemK), so the scatter and the binary searches
+// touch no global memory.
+constexpr uint32_t kBandSmemK = 16384;
+template <bool SM>
+__global__ void __launch_bounds__(1024) k_band_sort_jobs(uint32_t K, const uint32_t* __restrict__ prof8,
+                                                         uint32_t NB, uint32_t* __restrict__ order, int* fsort,
+                                                         int thr8, uint32_t* bandlo, uint32_t* job_cnt,
+                                                         uint64_t* job_off) {
+  extern __shared__ int sm_f[];  // SM: [K] f by kernel, [K] f by sorted position
   __shared__ uint32_t hist[4096];
   __shared__ uint32_t wsum[32];
   const uint32_t tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
+  int* fk = SM ? sm_f : nullptr;
+  int* fs = SM ? sm_f + K : fsort;
   for (uint32_t i = tid; i < 4096; i += 1024) hist[i] = 0u;
   __syncthreads();
-  for (uint32_t k = tid; k < K; k += 1024) atomicAdd(&hist[band_f(*(const uint4*)(prof8 + 4ull * k)) + kBandOff], 1u);
+  constexpr int IT = 8;
+  for (uint32_t base = 0; base < K; base += 1024u * IT) {
+    int f[IT];
+#pragma unroll
+    for (int u = 0; u < IT; ++u) {
+      const uint32_t k = base + u * 1024u + tid;
+      f[u] = k < K ? band_f(__ldg((const uint4*)(prof8 + 4ull * k))) : 0;
+    }
+#pragma unroll
+    for (int u = 0; u < IT; ++u) {
+      const uint32_t k = base + u * 1024u + tid;
+      if (k < K) {
+        atomicAdd(&hist[f[u] + kBandOff], 1u);
+        if (SM) fk[k] = f[u];
+      }
+    }
+  }
   __syncthreads();
   // exclusive scan of hist: 4 bins per thread
   uint32_t v[4], sum = 0;
@@ -296,35 +323,20 @@ __device__ __forceinline__ void band_sort_body(uint32_t K, const uint32_t* __res
   for (int j = 0; j < 4; ++j) { hist[tid * 4 + j] = run; run += v[j]; }
   __syncthreads();
   for (uint32_t k = tid; k < K; k += 1024) {
-    const int f = band_f(*(const uint4*)(prof8 + 4ull * k));
+    const int f = SM ? fk[k] : band_f(__ldg((const uint4*)(prof8 + 4ull * k)));
     const uint32_t pos = atomicAdd(&hist[f + kBandOff], 1u);
     order[pos] = k;
-    fsort[pos] = f;
+    fs[pos] = f;
   }
-  for (uint32_t pos = K + tid; pos < n_pad; pos += 1024) order[pos] = UINT32_MAX;
-}
-__device__ void band_jobs(uint32_t K, uint32_t NB, const int* __restrict__ fsort, int thr8, uint32_t* bandlo,
-                          uint32_t* job_cnt, uint64_t* job_off);
-// the sort and the band's jobs in one CTA (fsort is written and read by the same block: ordered by the barrier)
-__global__ void __launch_bounds__(1024) k_band_sort_jobs(uint32_t K, const uint32_t* __restrict__ prof8,
-                                                         uint32_t NB, uint32_t* __restrict__ order, int* fsort,
-                                                         int thr8, uint32_t* bandlo, uint32_t* job_cnt,
-                                                         uint64_t* job_off) {
-  band_sort_body(K, prof8, NB * FT, order, fsort);
-  __syncthreads();
-  band_jobs(K, NB, fsort, thr8, bandlo, job_cnt, job_off);
-}
-// one CTA: per k-block the first r-block whose largest f is within thr8 of the k-block's smallest f, the job count
-// ceil((kb - rb_lo + 1) / FR), and the job prefix
-__device__ void band_jobs(uint32_t K, uint32_t NB, const int* __restrict__ fsort, int thr8, uint32_t* bandlo,
-                          uint32_t* job_cnt, uint64_t* job_off) {
-  for (uint32_t kb = threadIdx.x; kb < NB; kb += 1024) {
-    const int fmin = fsort[kb * FT];
+  for (uint32_t pos = K + tid; pos < NB * FT; pos += 1024) order[pos] = UINT32_MAX;
+  __syncthreads();  // fs (shared or this block's global writes) complete
+  for (uint32_t kb = tid; kb < NB; kb += 1024) {
+    const int fmin = fs[kb * FT];
     uint32_t lo = 0, hi = kb;  // first rb with fmax(rb) > fmin - thr8 (rb = kb always qualifies)
     while (lo < hi) {
       const uint32_t mid = (lo + hi) >> 1;
       const uint32_t last = mid * FT + FT - 1 < K ? mid * FT + FT - 1 : K - 1;
-      if (fsort[last] > fmin - thr8) hi = mid; else lo = mid + 1;
+      if (fs[last] > fmin - thr8) hi = mid; else lo = mid + 1;
     }
     bandlo[kb] = lo;
     job_cnt[kb] = (kb - lo) / FRB + 1;
@@ -893,8 +905,15 @@ void launch_filter(const ScanArgs& a, cudaStream_t s) {
 void launch_filter_band(ScanArgs a, const MatchWs& mw, cudaStream_t s) {
   const uint32_t K = a.K, NB = (uint32_t)ceil_div(K, FT);
   if (NB == 0) return;
-  note_launch(), k_band_sort_jobs<<<1, 1024, 0, s>>>(K, a.prof8, NB, mw.border, mw.bfs, (int)a.thr8, mw.bandlo,
-                                                     mw.bjobs, mw.bjob_off);
+  if (K <= kBandSmemK) {
+    const int smem = (int)(2 * (size_t)K * sizeof(int));
+    cudaFuncSetAttribute(k_band_sort_jobs<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+    note_launch(), k_band_sort_jobs<true><<<1, 1024, smem, s>>>(K, a.prof8, NB, mw.border, mw.bfs, (int)a.thr8,
+                                                                 mw.bandlo, mw.bjobs, mw.bjob_off);
+  } else {
+    note_launch(), k_band_sort_jobs<false><<<1, 1024, 0, s>>>(K, a.prof8, NB, mw.border, mw.bfs, (int)a.thr8,
+                                                               mw.bandlo, mw.bjobs, mw.bjob_off);
+  }
   a.order = mw.border;
   a.bandlo = mw.bandlo;
   a.job_off = mw.bjob_off;
