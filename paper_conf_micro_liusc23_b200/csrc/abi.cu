@@ -569,7 +569,7 @@ int photon_analyse(photon_ctx* ctx, const photon_trace* t, void* gws, size_t gws
     for (auto& e : ctx->aev) CK(cudaEventCreateWithFlags(&e, cudaEventDisableTiming), "event");
   }
   cudaStream_t sa = ctx->sa, sb = ctx->sb;
-  cudaEvent_t e_lists = ctx->aev[0], e_sorted = ctx->aev[1], e_prof = ctx->aev[2], e_filt = ctx->aev[3],
+  cudaEvent_t e_lists = ctx->aev[0], e_sorted = ctx->aev[1], e_filt = ctx->aev[3],
               e_remap = ctx->aev[4];
   ctx->last_ws = gws;
   TraceDev d = to_dev(t);
@@ -595,10 +595,13 @@ int photon_analyse(photon_ctx* ctx, const photon_trace* t, void* gws, size_t gws
     CK(cudaEventRecord(e_lists, s), "event");
     CK(cudaStreamWaitEvent(sb, e_lists, 0), "event");
     CK(launch_analyse_filter(K, out->kernel_type_off, g.h.cw.list, g.h.ht, m.mass, warps_total, params, m.mw, m.pairs,
-                             m.err, ctx->num_sms, sb, e_prof),
+                             m.err, ctx->num_sms, sb),
        "filter");
     CK(cudaEventRecord(e_filt, sb), "event");
-    CK(launch_canon_sort(g.h.ht, K, t->kernel_warp_off, nullptr, *out, g.h.cw, ctx->num_sms, s), "sort");
+    // the canonical rows with A3 (g and g/N in row order, N summed by the sorting warp / CTA)
+    CK(launch_canon_sort(g.h.ht, K, t->kernel_warp_off, nullptr, *out, g.h.cw, ctx->num_sms, s,
+                         SigOut{m.sig, m.mw.sigf}),
+       "sort");
     // fork 2: the per-warp warp_type write
     CK(cudaEventRecord(e_sorted, s), "event");
     CK(cudaStreamWaitEvent(sa, e_sorted, 0), "event");
@@ -607,9 +610,7 @@ int photon_analyse(photon_ctx* ctx, const photon_trace* t, void* gws, size_t gws
   }
   {
     ProfScope ps(ctx, PHOTON_PROF_SCAN, s);
-    CK(cudaStreamWaitEvent(s, e_prof, 0), "event");  // 1/N
-    CK(launch_analyse_sigf(K, *out, m.sig, m.mw, s), "sigf");
-    CK(cudaStreamWaitEvent(s, e_filt, 0), "event");  // the filter survivors and their segments
+    CK(cudaStreamWaitEvent(s, e_filt, 0), "event");  // the filter survivors, their segments, mass and 1/N
     CK(launch_analyse_exact(K, out->kernel_type_off, m.sig, m.mass, warps_total, params, m.mw, m.pairs,
                             m.mw.pair_cap, m.n_pairs, m.err, ctx->num_sms, s),
        "exact");

@@ -146,7 +146,8 @@ __global__ void k_sig_prof(uint32_t K, const uint64_t* __restrict__ kto, const u
 // photon_analyse's split of k_sig_prof, so the filter need not wait for the canonical sort:
 // k_prof_slots -- the filter profiles, 1/N and N from the UNSORTED type table (the per-kernel slot lists of the
 // canonicalisation; the bin sums are exact integers, so they equal the sorted rows' sums bit for bit);
-// k_sigf -- g and its fp32 copy g / N in the canonical row order, after the sort.
+// g and its fp32 copy g / N in the canonical row order are written by the canonical sort itself (k_types.cu
+// emit_sig_row: the sorting warp / CTA sums N_k, the same exact integer).
 __global__ void k_prof_slots(uint32_t K, const uint64_t* __restrict__ kto, const uint32_t* __restrict__ list,
                              HashTable ht, uint64_t* __restrict__ mass, float* __restrict__ prof,
                              double* __restrict__ invn, uint32_t* __restrict__ prof8, DevErr* err) {
@@ -181,20 +182,6 @@ __global__ void k_prof_slots(uint32_t K, const uint64_t* __restrict__ kto, const
       mass[k] = N;
       if (over) latch(err, PHOTON_ERANGE, (int64_t)k);
     }
-  }
-}
-__global__ void k_sigf(uint32_t K, const uint64_t* __restrict__ kto, const uint32_t* __restrict__ key,
-                       const uint64_t* __restrict__ count, const double* __restrict__ invn, uint64_t* __restrict__ sig,
-                       float* __restrict__ sigf) {
-  const uint32_t k = (blockIdx.x * blockDim.x + threadIdx.x) >> 5, lane = threadIdx.x & 31;
-  if (k >= K) return;
-  const uint64_t r0 = kto[k], r1 = kto[k + 1];
-  const double inv = invn[k];
-  for (uint64_t r = r0 + (lane >> 4); r < r1; r += 2) {
-    const uint64_t i = r * 16 + (lane & 15);
-    const uint64_t g = count[r] * (uint64_t)key[i];
-    sig[i] = g;
-    if (sigf) sigf[i] = (float)((double)g * inv);
   }
 }
 
@@ -963,24 +950,17 @@ cudaError_t launch_match_scan(uint32_t K, const uint64_t* kto, const uint64_t* s
 // sort, on the main stream -- g / N in row order and the exact check
 cudaError_t launch_analyse_filter(uint32_t K, const uint64_t* kto, const uint32_t* list, const HashTable& ht,
                                   uint64_t* mass, const uint64_t* wt, photon_match_params p, const MatchWs& mw,
-                                  uint64_t* pairs, DevErr* err, int num_sms, cudaStream_t sb, cudaEvent_t prof_done) {
+                                  uint64_t* pairs, DevErr* err, int num_sms, cudaStream_t sb) {
   cudaMemsetAsync(mw.n_maybe, 0, 8, sb);
   note_launch(), k_prof_slots<<<(unsigned)ceil_div((uint64_t)K * 32, 256), 256, 0, sb>>>(K, kto, list, ht, mass,
                                                                                        mw.prof, mw.invn, mw.prof8,
                                                                                        err);
-  cudaEventRecord(prof_done, sb);
   ScanArgs a = scan_args(K, 0, K, kto, nullptr, mass, wt, p, mw, err);
   a.kcnt = mw.cand_cnt;  // the filter counts its survivors per k (no separate count pass)
   cudaMemsetAsync(mw.cand_cnt, 0, sizeof(uint32_t) * K, sb);
   if (PHOTON_BAND && K <= kBandMaxK) launch_filter_band(a, mw, sb);  // f in [-2040, 2040]: the counting sort's 4096 bins
   else launch_filter(a, sb);
   launch_segments(K, mw, err, num_sms, sb, true);
-  return cudaGetLastError();
-}
-cudaError_t launch_analyse_sigf(uint32_t K, const photon_types& types, uint64_t* sig, const MatchWs& mw,
-                                cudaStream_t s) {
-  note_launch(), k_sigf<<<(unsigned)ceil_div((uint64_t)K * 32, 256), 256, 0, s>>>(
-      K, types.kernel_type_off, types.type_key, types.type_count, mw.invn, sig, mw.sigf);
   return cudaGetLastError();
 }
 cudaError_t launch_analyse_exact(uint32_t K, const uint64_t* kto, const uint64_t* sig, const uint64_t* mass,

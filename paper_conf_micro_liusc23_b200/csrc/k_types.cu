@@ -67,8 +67,43 @@ __device__ __forceinline__ bool type_before(const HashTable& ht, uint32_t a, uin
   return ht.first[a] < ht.first[b];
 }
 
+// A3 of one row (Fig 5, L178 [P-5]): g = count * key word (u64), and g / N_k in fp32 through 1/N_k in fp64 (the
+// same arithmetic as k_sigf)
+__device__ __forceinline__ uint64_t key_sum(const uint4* kp) {
+  uint64_t t = 0;
+#pragma unroll
+  for (int q = 0; q < 4; ++q) {
+    const uint4 v = kp[q];
+    t += (uint64_t)v.x + v.y + v.z + v.w;
+  }
+  return t;
+}
+__device__ __forceinline__ void emit_sig_row(const SigOut& so, uint64_t row, uint64_t cnt, const uint4* kp,
+                                             double inv) {
+  ulonglong2* g2 = (ulonglong2*)(so.sig + row * 16);
+  float4* f4 = (float4*)(so.sigf + row * 16);
+#pragma unroll
+  for (int q = 0; q < 4; ++q) {
+    const uint4 v = kp[q];
+    const uint64_t a = cnt * v.x, b = cnt * v.y, c = cnt * v.z, d = cnt * v.w;
+    g2[2 * q] = make_ulonglong2(a, b);
+    g2[2 * q + 1] = make_ulonglong2(c, d);
+    f4[q] = make_float4((float)((double)a * inv), (float)((double)b * inv), (float)((double)c * inv),
+                        (float)((double)d * inv));
+  }
+}
+__device__ __forceinline__ uint64_t warp_sum_u64(uint64_t x) {
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) x += __shfl_xor_sync(0xffffffffu, x, o);
+  return x;
+}
+
 __device__ void emit_rows(const HashTable& ht, uint32_t k, const uint32_t* sorted, uint64_t n, uint64_t off,
-                          const photon_types& out, uint32_t* canon, uint64_t Wk) {
+                          const photon_types& out, uint32_t* canon, uint64_t Wk, const SigOut& so) {
+  __shared__ unsigned long long s_mass;
+  if (threadIdx.x == 0) s_mass = 0;
+  __syncthreads();
+  uint64_t part = 0;
   for (uint64_t r = threadIdx.x; r < n && off + r < out.capacity; r += blockDim.x) {
     uint32_t s = sorted[r];
     const uint4* src = (const uint4*)(ht.key + (uint64_t)s * 16);
@@ -77,10 +112,22 @@ __device__ void emit_rows(const HashTable& ht, uint32_t k, const uint32_t* sorte
     out.type_count[off + r] = ht.count[s];
     out.type_first_warp[off + r] = ht.first[s];
     canon[s] = (uint32_t)r;
+    if (so.sig) part += (uint64_t)ht.count[s] * key_sum(src);
   }
   if (threadIdx.x == 0) {
     uint64_t c0 = n ? ht.count[sorted[0]] : 0;
     out.warp_sampling_ok[k] = (Wk > 0 && 100ull * c0 > 95ull * Wk) ? 1 : 0;  // L249, strict [P-15]
+  }
+  if (so.sig) {
+    part = warp_sum_u64(part);
+    if ((threadIdx.x & 31) == 0) atomicAdd(&s_mass, (unsigned long long)part);
+    __syncthreads();
+    const uint64_t N = s_mass;
+    const double inv = N ? 1.0 / (double)N : 0.0;
+    for (uint64_t r = threadIdx.x; r < n && off + r < out.capacity; r += blockDim.x) {
+      const uint32_t s = sorted[r];
+      emit_sig_row(so, off + r, ht.count[s], (const uint4*)(ht.key + (uint64_t)s * 16), inv);
+    }
   }
 }
 
@@ -128,7 +175,8 @@ __device__ __forceinline__ void warp_sort_reg(const HashTable& ht, uint64_t (&sk
 }
 template <int E>
 __device__ __forceinline__ void sort_mid_reg(const HashTable& ht, uint64_t off, uint64_t n, const uint32_t* list,
-                                             const photon_types& out, uint32_t* canon, uint64_t Wk, uint32_t k) {
+                                             const photon_types& out, uint32_t* canon, uint64_t Wk, uint32_t k,
+                                             const SigOut& so) {
   const uint32_t lane = threadIdx.x & 31;
   uint64_t sk[E];
   uint32_t sl[E];
@@ -151,6 +199,23 @@ __device__ __forceinline__ void sort_mid_reg(const HashTable& ht, uint64_t off, 
       canon[sl_] = r;
     }
   }
+  if (so.sig) {
+    uint64_t part = 0;
+#pragma unroll
+    for (int e = 0; e < E; ++e) {
+      const uint32_t r = lane * E + e;
+      if (r < n && off + r < out.capacity)
+        part += (uint64_t)ht.count[sl[e]] * key_sum((const uint4*)(ht.key + (uint64_t)sl[e] * 16));
+    }
+    const uint64_t N = warp_sum_u64(part);
+    const double inv = N ? 1.0 / (double)N : 0.0;
+#pragma unroll
+    for (int e = 0; e < E; ++e) {
+      const uint32_t r = lane * E + e;
+      if (r < n && off + r < out.capacity)
+        emit_sig_row(so, off + r, ht.count[sl[e]], (const uint4*)(ht.key + (uint64_t)sl[e] * 16), inv);
+    }
+  }
   const uint32_t first = __shfl_sync(0xffffffffu, sl[0], 0);
   if (lane == 0) {
     const uint64_t c0 = ht.count[first];
@@ -164,18 +229,18 @@ __device__ __forceinline__ void sort_mid_reg(const HashTable& ht, uint64_t off, 
 __global__ void __launch_bounds__(256) k_sort_warp(HashTable ht, uint32_t K, const uint64_t* kto,
                                                    const uint32_t* list, const uint64_t* kwo,
                                                    const uint64_t* kernel_warps, photon_types out, uint32_t* canon,
-                                                   uint32_t* big, uint32_t* nbig) {
+                                                   uint32_t* big, uint32_t* nbig, SigOut so) {
   const uint32_t lane = threadIdx.x & 31;
   const uint32_t k = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   if (k >= K) return;
   const uint64_t off = kto[k], n = kto[k + 1] - off;
   const uint64_t Wk = kernel_warps ? kernel_warps[k] : (kwo[k + 1] - kwo[k]);
   if (n > 32 && n <= 64) {
-    sort_mid_reg<2>(ht, off, n, list, out, canon, Wk, k);
+    sort_mid_reg<2>(ht, off, n, list, out, canon, Wk, k, so);
     return;
   }
   if (n > 64 && n <= WARP_SORT_MAX) {
-    sort_mid_reg<4>(ht, off, n, list, out, canon, Wk, k);
+    sort_mid_reg<4>(ht, off, n, list, out, canon, Wk, k, so);
     return;
   }
   if (n > 32) {
@@ -220,13 +285,20 @@ __global__ void __launch_bounds__(256) k_sort_warp(HashTable ht, uint32_t K, con
       if (!keep) { mine = other; mc = oc; mk = ok; }
     }
   }
-  if (lane < n && off + lane < out.capacity) {
+  const bool row = lane < n && off + lane < out.capacity;
+  if (row) {
     const uint4* src = (const uint4*)(ht.key + (uint64_t)mine * 16);
     uint4* dst = (uint4*)(out.type_key + (off + lane) * 16);
     dst[0] = src[0]; dst[1] = src[1]; dst[2] = src[2]; dst[3] = src[3];
     out.type_count[off + lane] = ht.count[mine];
     out.type_first_warp[off + lane] = ht.first[mine];
     canon[mine] = lane;
+  }
+  if (so.sig) {
+    const uint4* kp = (const uint4*)(ht.key + (uint64_t)(row ? mine : 0u) * 16);
+    const uint64_t N = warp_sum_u64(row ? (uint64_t)mc * key_sum(kp) : 0ull);
+    const double inv = N ? 1.0 / (double)N : 0.0;
+    if (row) emit_sig_row(so, off + lane, mc, kp, inv);
   }
   uint32_t c0 = __shfl_sync(0xffffffffu, mine != UINT32_MAX ? mc : 0u, 0);
   if (lane == 0) out.warp_sampling_ok[k] = (Wk > 0 && 100ull * c0 > 95ull * Wk) ? 1 : 0;  // L249 [P-15]
@@ -236,7 +308,7 @@ __global__ void __launch_bounds__(256) k_sort_warp(HashTable ht, uint32_t K, con
 __global__ void __launch_bounds__(512) k_sort_mid(HashTable ht, uint32_t K, const uint64_t* kto,
                                                   const uint32_t* list, const uint64_t* kwo,
                                                   const uint64_t* kernel_warps, photon_types out, uint32_t* canon,
-                                                  const uint32_t* big, const uint32_t* nbig) {
+                                                  const uint32_t* big, const uint32_t* nbig, SigOut so) {
   __shared__ uint32_t sh[SORT_SMEM_MAX];
   const uint32_t nmid = nbig[0];
   for (uint32_t q = blockIdx.x; q < nmid; q += gridDim.x) {
@@ -260,7 +332,7 @@ __global__ void __launch_bounds__(512) k_sort_mid(HashTable ht, uint32_t K, cons
         __syncthreads();
       }
     }
-    emit_rows(ht, k, sh, n, off, out, canon, Wk);
+    emit_rows(ht, k, sh, n, off, out, canon, Wk, so);
     __syncthreads();
   }
 }
@@ -269,7 +341,8 @@ __global__ void __launch_bounds__(512) k_sort_mid(HashTable ht, uint32_t K, cons
 __global__ void __launch_bounds__(1024) k_sort_large(HashTable ht, uint32_t K, const uint64_t* kto,
                                                      const uint32_t* list, const uint64_t* kwo,
                                                      const uint64_t* kernel_warps, photon_types out, uint32_t* canon,
-                                                     uint32_t* scratch, const uint32_t* big, const uint32_t* nbig) {
+                                                     uint32_t* scratch, const uint32_t* big, const uint32_t* nbig,
+                                                     SigOut so) {
   const uint32_t nlarge = nbig[1];
   for (uint32_t q = 0; q < nlarge; ++q) {
     const uint32_t k = big[K - 1 - q];
@@ -292,7 +365,7 @@ __global__ void __launch_bounds__(1024) k_sort_large(HashTable ht, uint32_t K, c
         __syncthreads();
       }
     }
-    emit_rows(ht, k, scratch, n, off, out, canon, Wk);
+    emit_rows(ht, k, scratch, n, off, out, canon, Wk, so);
     __syncthreads();
   }
 }
@@ -478,14 +551,14 @@ cudaError_t launch_canon_lists(const HashTable& ht, uint32_t K, const photon_typ
   return cudaGetLastError();
 }
 cudaError_t launch_canon_sort(const HashTable& ht, uint32_t K, const uint64_t* kwo, const uint64_t* kernel_warps,
-                              const photon_types& out, const CanonWs& cw, int num_sms, cudaStream_t s) {
+                              const photon_types& out, const CanonWs& cw, int num_sms, cudaStream_t s, SigOut so) {
   cudaMemsetAsync(cw.nbig, 0, 8, s);
   note_launch(), k_sort_warp<<<(unsigned)ceil_div((uint64_t)K * 32, 256), 256, 0, s>>>(
-      ht, K, out.kernel_type_off, cw.list, kwo, kernel_warps, out, cw.canon, cw.big, cw.nbig);
+      ht, K, out.kernel_type_off, cw.list, kwo, kernel_warps, out, cw.canon, cw.big, cw.nbig, so);
   note_launch(), k_sort_mid<<<(unsigned)num_sms, 512, 0, s>>>(ht, K, out.kernel_type_off, cw.list, kwo, kernel_warps,
-                                                             out, cw.canon, cw.big, cw.nbig);
+                                                             out, cw.canon, cw.big, cw.nbig, so);
   note_launch(), k_sort_large<<<1, 1024, 0, s>>>(ht, K, out.kernel_type_off, cw.list, kwo, kernel_warps, out, cw.canon,
-                                                cw.scratch, cw.big, cw.nbig);
+                                                cw.scratch, cw.big, cw.nbig, so);
   return cudaGetLastError();
 }
 cudaError_t launch_canonicalise(const HashTable& ht, uint32_t K, const uint64_t* kwo, const uint64_t* kernel_warps,
