@@ -362,19 +362,18 @@ __global__ void __launch_bounds__(WPC * 32, 1) k_bbv3(Args3 a) {
   }
 
   const uint64_t W = a.W, E = a.E, E8 = E & ~7ull;
-  const uint64_t NB = (W + 31) >> 5;
   const uint32_t NWK = gridDim.x * WPC, gw = blockIdx.x * WPC + wid;
   const bool last_worker = gw + 1 == NWK;
-  // worker gw takes the blocks b whose cost(b) = start(b) + kAlpha * 32b lies in its 1/NWK share (the last worker:
-  // all remaining blocks, trailing empty warps included)
+  // worker gw takes the warps [w_lo, w_hi) whose cost(w) = start(w) + kAlpha * w lies in its 1/NWK share (the last
+  // worker: all remaining warps, trailing empty warps included), in blocks of up to 32 consecutive warps from w_lo.
+  // Warp-granular ranges (not whole 32-warp blocks) let a group of long warps -- VGG's fully connected layers,
+  // ~150K events per 32 warps -- spread over several workers.
   const uint64_t C = E + kAlpha * W;
   const uint64_t T_lo = (uint64_t)(((unsigned __int128)C * gw) / NWK);
   const uint64_t T_hi = (uint64_t)(((unsigned __int128)C * (gw + 1)) / NWK);
-  auto bcost = [&](uint64_t b) -> uint64_t { return a.weo[b << 5] + kAlpha * (b << 5); };
-  const uint64_t b_lo = search32(0, NB, bcost, T_lo);
-  auto in_range = [&](uint64_t b, uint64_t start_b) -> bool {
-    return b < NB && (last_worker || start_b + kAlpha * (b << 5) < T_hi);
-  };
+  auto wcost = [&](uint64_t w) -> uint64_t { return a.weo[w] + kAlpha * w; };
+  const uint64_t w_lo = gw == 0 ? 0 : search32(0, W, wcost, T_lo);
+  const uint64_t w_hi = last_worker ? W : search32(0, W, wcost, T_hi);
   auto clampE = [&](uint64_t x) -> uint64_t { return x < E ? x : E; };
 
   // ---- chunk issuer (lane 0): stages the worker's chunk sequence one chunk ahead.  State in shared memory except
@@ -383,18 +382,15 @@ __global__ void __launch_bounds__(WPC * 32, 1) k_bbv3(Args3 a) {
   if (lane == 0) {
     wm->i_live = 0;
     wm->i_n = 0;
-    if (b_lo < NB) {
-      const uint64_t st = a.weo[b_lo << 5];
-      if (in_range(b_lo, st)) {
-        const uint64_t s0 = clampE(st);
-        const uint64_t e_raw = a.weo[umin64((b_lo + 1) << 5, W)];
-        wm->i_live = 1;
-        wm->i_b = b_lo;
-        wm->i_cs = s0;
-        wm->i_te = umax64(clampE(e_raw), s0);
-        wm->i_pf = e_raw;  // raw end of block i_b (= raw start of the next block)
-        i_pf = a.weo[umin64((b_lo + 2) << 5, W)];
-      }
+    if (w_lo < w_hi) {
+      const uint64_t s0 = clampE(a.weo[w_lo]);
+      const uint64_t e_raw = a.weo[umin64(w_lo + 32, w_hi)];
+      wm->i_live = 1;
+      wm->i_b = w_lo;  // first warp of the issuer's block
+      wm->i_cs = s0;
+      wm->i_te = umax64(clampE(e_raw), s0);
+      wm->i_pf = e_raw;  // raw end of the block (= raw start of the next block)
+      i_pf = a.weo[umin64(w_lo + 64, w_hi)];
     }
   }
   auto issue = [&]() {  // lane 0 only
@@ -419,13 +415,13 @@ __global__ void __launch_bounds__(WPC * 32, 1) k_bbv3(Args3 a) {
     if (ce < te) {
       wm->i_cs = ce;
     } else {  // the next block starts where this one ends
-      const uint64_t nb_ = wm->i_b + 1;
-      if (nb_ < NB && in_range(nb_, wm->i_pf)) {
-        wm->i_b = nb_;
+      const uint64_t nw0 = wm->i_b + 32;
+      if (nw0 < w_hi) {
+        wm->i_b = nw0;
         wm->i_cs = te;
         wm->i_te = umax64(clampE(i_pf), te);
         wm->i_pf = i_pf;
-        i_pf = a.weo[umin64((nb_ + 2) << 5, W)];
+        i_pf = a.weo[umin64(nw0 + 64, w_hi)];
       } else {
         wm->i_live = 0;
       }
@@ -435,40 +431,38 @@ __global__ void __launch_bounds__(WPC * 32, 1) k_bbv3(Args3 a) {
   __syncwarp();
 
   // ---- per-block state (all lanes) ----
-  uint64_t b = b_lo;
-  uint64_t my_s = 0, blk_end = 0;  // weo[32b + lane], weo[min(32b + 32, W)] (raw)
-  if (b < NB) {
-    my_s = a.weo[umin64((b << 5) + lane, W)];
-    blk_end = a.weo[umin64((b + 1) << 5, W)];
+  uint64_t w0 = w_lo;              // first warp of the current block
+  uint64_t my_s = 0, blk_end = 0;  // weo[w0 + lane], weo[min(w0 + 32, w_hi)] (raw)
+  if (w0 < w_hi) {
+    my_s = a.weo[umin64(w0 + lane, w_hi)];
+    blk_end = a.weo[umin64(w0 + 32, w_hi)];
   }
-  // kernel of the block's first warp: last k with kwo[k] <= 32b
+  // kernel of the block's first warp: last k with kwo[k] <= w0
   uint32_t kb = 0;
-  if (b < NB && a.K > 1) {
+  if (w0 < w_hi && a.K > 1) {
     auto kf = [&](uint64_t kk) -> uint64_t { return a.kwo[kk]; };
-    kb = (uint32_t)(search32(1, a.K, kf, (b << 5) + 1) - 1);
+    kb = (uint32_t)(search32(1, a.K, kf, w0 + 1) - 1);
   }
   uint64_t kb1 = kb + 1 < a.K ? a.kwo[kb + 1] : ~0ull;  // first warp of the next kernel (prefetched)
   uint32_t n_done = 0;  // chunks consumed
   uint64_t prev_te = 0;
   uint32_t raw = 0, orr = 0;
 
-  while (b < NB) {
+  while (w0 < w_hi) {
     const uint64_t start_b = __shfl_sync(0xffffffffu, my_s, 0);
-    if (!in_range(b, start_b)) break;
-    const uint64_t w0 = b << 5;
-    const uint32_t nw = (uint32_t)umin64(32, W - w0);
+    const uint32_t nw = (uint32_t)umin64(32, w_hi - w0);
     // prefetch the next block's starts (used at its start)
     uint64_t nx_s = 0, nx_end = 0;
-    if (b + 1 < NB) {
-      nx_s = a.weo[umin64(((b + 1) << 5) + lane, W)];
-      nx_end = a.weo[umin64((b + 2) << 5, W)];
+    if (w0 + 32 < w_hi) {
+      nx_s = a.weo[umin64(w0 + 32 + lane, w_hi)];
+      nx_end = a.weo[umin64(w0 + 64, w_hi)];
     }
     // warp starts: lane u <= nw holds s_u; non-monotone offsets are latched and made monotone (memory safety)
     const uint64_t s_raw = lane < nw ? my_s : blk_end;
     const uint64_t s_next_raw = __shfl_down_sync(0xffffffffu, s_raw, 1);
     const bool bad = lane < nw && (lane + 1 < nw ? s_next_raw : blk_end) < s_raw;
     // the block's event range, exactly as the chunk issuer computes it: it starts where the previous block ended
-    const uint64_t ts = b == b_lo ? clampE(start_b) : prev_te;
+    const uint64_t ts = w0 == w_lo ? clampE(start_b) : prev_te;
     const uint64_t te = umax64(clampE(blk_end), ts);
     uint64_t s = umin64(umax64(clampE(s_raw), ts), te);
     if (__any_sync(0xffffffffu, bad)) {
@@ -721,7 +715,7 @@ __global__ void __launch_bounds__(WPC * 32, 1) k_bbv3(Args3 a) {
     // next block
     kb = __shfl_sync(0xffffffffu, k, nw - 1);
     kb1 = kb + 1 < a.K ? a.kwo[kb + 1] : ~0ull;  // consumed at the next block's end
-    ++b;
+    w0 += 32;
     my_s = nx_s;
     blk_end = nx_end;
   }
