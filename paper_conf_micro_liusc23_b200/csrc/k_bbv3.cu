@@ -109,6 +109,17 @@ struct Args3 {
 };
 
 // per-worker scratch in shared memory
+#ifndef K1_CTAG32
+#define K1_CTAG32 0
+#endif
+#if K1_CTAG32
+#define K1_TAG(h) ((uint32_t)((h) >> 32) | 1u)
+#else
+#define K1_TAG(h) (h)
+#endif
+#ifndef K1_CACHE2
+#define K1_CACHE2 1
+#endif
 #ifndef K1_ENTCACHE
 #define K1_ENTCACHE 128
 #endif
@@ -124,7 +135,11 @@ struct WMisc {
   uint64_t e_next, e_end;
   // direct-mapped cache of the worker's recent entries (hash -> entry id): a type seen again in a later block of
   // the worker adds to its entry after an exact key check instead of opening a new one
+#if K1_CTAG32
+  uint32_t ch[kEntCache];  // tag: high hash word | 1 (0 = empty; a false tag hit fails the exact key check)
+#else
   uint64_t ch[kEntCache];
+#endif
   uint32_t ce[kEntCache];
 };
 constexpr uint32_t kWMiscBytes = (sizeof(WMisc) + 127) & ~127u;
@@ -199,7 +214,7 @@ __device__ __forceinline__ uint64_t hash16(uint32_t k, const uint32_t* p) {
 
 __device__ __forceinline__ void pool_init(WMisc* wm) {
   if ((threadIdx.x & 31) == 0) { wm->e_next = 0; wm->e_end = 0; }
-  for (int i = threadIdx.x & 31; i < kEntCache; i += 32) wm->ch[i] = 0ull;
+  for (int i = threadIdx.x & 31; i < kEntCache; i += 32) wm->ch[i] = 0;
   __syncwarp();
 }
 __device__ __forceinline__ void pool_flush(const Args3& a, WMisc* wm) {
@@ -227,9 +242,17 @@ __device__ void finalize_fused(const Args3& a, WMisc* wm, uint64_t w0, bool vali
   const uint32_t cnt = ((int)lane == leader) ? (uint32_t)__popc(peers & eqm & vmask) : 1u;
   // the worker's entry cache: an exact (kernel, key) match adds this block's count to the existing entry
   uint32_t hit = UINT32_MAX;
+#if K1_CACHE2
+  // 2-way set-associative: set (h mod kEntCache/2), ways 2 set (most recent) and 2 set + 1
+  const uint32_t cslot = ((uint32_t)h & (kEntCache / 2 - 1)) * 2u;
+  const uint32_t cway = wm->ch[cslot] == K1_TAG(h) ? cslot : cslot + 1u;
+  if (is_l && wm->ch[cway] == K1_TAG(h)) {
+    const uint32_t e = wm->ce[cway];
+#else
   const uint32_t cslot = (uint32_t)h & (kEntCache - 1);
-  if (is_l && wm->ch[cslot] == h) {
+  if (is_l && wm->ch[cslot] == K1_TAG(h)) {
     const uint32_t e = wm->ce[cslot];
+#endif
     if (e < a.ep.cap) {  // the exact check against the entry itself (written by this warp earlier)
       TileEntry* d = a.ep.ent + e;
       const uint4* kd = (const uint4*)d->key;
@@ -281,7 +304,11 @@ __device__ void finalize_fused(const Args3& a, WMisc* wm, uint64_t w0, bool vali
   // against the entry's own key anyway)
   const unsigned same_slot = __match_any_sync(0xffffffffu, alloc ? cslot : 0xFFFFFFFFu);
   if (alloc && (int)lane == __ffs(same_slot) - 1) {
-    wm->ch[cslot] = h;
+#if K1_CACHE2
+    wm->ch[cslot + 1] = wm->ch[cslot];  // the previous most recent entry of the set moves to the second way
+    wm->ce[cslot + 1] = wm->ce[cslot];
+#endif
+    wm->ch[cslot] = K1_TAG(h);
     wm->ce[cslot] = (uint32_t)umin64(id, 0xFFFFFFFFull);
   }
   if (lane == 0) { wm->e_next = e_next; wm->e_end = e_end; }
