@@ -117,8 +117,8 @@ struct Args3 {
 #else
 #define K1_TAG(h) (h)
 #endif
-#ifndef K1_CACHE2
-#define K1_CACHE2 1
+#ifndef K1_CWAYS
+#define K1_CWAYS 2  // entry-cache associativity (1, 2 or 4)
 #endif
 #ifndef K1_ENTCACHE
 #define K1_ENTCACHE 128
@@ -242,17 +242,15 @@ __device__ void finalize_fused(const Args3& a, WMisc* wm, uint64_t w0, bool vali
   const uint32_t cnt = ((int)lane == leader) ? (uint32_t)__popc(peers & eqm & vmask) : 1u;
   // the worker's entry cache: an exact (kernel, key) match adds this block's count to the existing entry
   uint32_t hit = UINT32_MAX;
-#if K1_CACHE2
-  // 2-way set-associative: set (h mod kEntCache/2), ways 2 set (most recent) and 2 set + 1
-  const uint32_t cslot = ((uint32_t)h & (kEntCache / 2 - 1)) * 2u;
-  const uint32_t cway = wm->ch[cslot] == K1_TAG(h) ? cslot : cslot + 1u;
+  // K1_CWAYS-way set-associative: set (h mod kEntCache / ways) at cslot, most recent way first
+  constexpr uint32_t NWAY = K1_CWAYS;
+  const uint32_t cslot = ((uint32_t)h & (kEntCache / NWAY - 1)) * NWAY;
+  uint32_t cway = cslot;
+#pragma unroll
+  for (uint32_t q = NWAY - 1; q > 0; --q)
+    if (wm->ch[cslot + q] == K1_TAG(h)) cway = cslot + q;
   if (is_l && wm->ch[cway] == K1_TAG(h)) {
     const uint32_t e = wm->ce[cway];
-#else
-  const uint32_t cslot = (uint32_t)h & (kEntCache - 1);
-  if (is_l && wm->ch[cslot] == K1_TAG(h)) {
-    const uint32_t e = wm->ce[cslot];
-#endif
     if (e < a.ep.cap) {  // the exact check against the entry itself (written by this warp earlier)
       TileEntry* d = a.ep.ent + e;
       const uint4* kd = (const uint4*)d->key;
@@ -304,10 +302,11 @@ __device__ void finalize_fused(const Args3& a, WMisc* wm, uint64_t w0, bool vali
   // against the entry's own key anyway)
   const unsigned same_slot = __match_any_sync(0xffffffffu, alloc ? cslot : 0xFFFFFFFFu);
   if (alloc && (int)lane == __ffs(same_slot) - 1) {
-#if K1_CACHE2
-    wm->ch[cslot + 1] = wm->ch[cslot];  // the previous most recent entry of the set moves to the second way
-    wm->ce[cslot + 1] = wm->ce[cslot];
-#endif
+#pragma unroll
+    for (uint32_t q = NWAY - 1; q > 0; --q) {  // the set's entries move one way down
+      wm->ch[cslot + q] = wm->ch[cslot + q - 1];
+      wm->ce[cslot + q] = wm->ce[cslot + q - 1];
+    }
     wm->ch[cslot] = K1_TAG(h);
     wm->ce[cslot] = (uint32_t)umin64(id, 0xFFFFFFFFull);
   }
