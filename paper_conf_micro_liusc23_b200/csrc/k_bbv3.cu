@@ -117,6 +117,9 @@ struct Args3 {
 #else
 #define K1_TAG(h) (h)
 #endif
+#ifndef K1_NRANGE
+#define K1_NRANGE 1  // ranges per worker: worker g takes parts g, g + G, ... of a cost partition into G * K1_NRANGE
+#endif
 #ifndef K1_CWAYS
 #define K1_CWAYS 2  // entry-cache associativity (1, 2 or 4)
 #endif
@@ -130,7 +133,8 @@ struct WMisc {
   uint64_t mbar[2];
   // chunk issuer (lane 0)
   uint64_t i_b, i_cs, i_te, i_pf;
-  uint32_t i_live, i_n;
+  uint32_t i_live, i_n, i_ri;
+  uint64_t rlo[K1_NRANGE], rhi[K1_NRANGE];  // the worker's warp ranges (round-robin over the cost partition)
   // the worker's current block of pool entries (fused)
   uint64_t e_next, e_end;
   // direct-mapped cache of the worker's recent entries (hash -> entry id): a type seen again in a later block of
@@ -389,35 +393,48 @@ __global__ void __launch_bounds__(WPC * 32, 1) k_bbv3(Args3 a) {
 
   const uint64_t W = a.W, E = a.E, E8 = E & ~7ull;
   const uint32_t NWK = gridDim.x * WPC, gw = blockIdx.x * WPC + wid;
-  const bool last_worker = gw + 1 == NWK;
-  // worker gw takes the warps [w_lo, w_hi) whose cost(w) = start(w) + kAlpha * w lies in its 1/NWK share (the last
-  // worker: all remaining warps, trailing empty warps included), in blocks of up to 32 consecutive warps from w_lo.
-  // Warp-granular ranges (not whole 32-warp blocks) let a group of long warps -- VGG's fully connected layers,
-  // ~150K events per 32 warps -- spread over several workers.
+  // worker gw takes the warps whose cost(w) = start(w) + kAlpha * w lies in parts gw, gw + G, ... of a partition of
+  // the cost into G * K1_NRANGE equal parts (G workers; the last part: all remaining warps, trailing empty warps
+  // included), each in blocks of up to 32 consecutive warps from its first warp.  Warp-granular parts (not whole
+  // 32-warp blocks) let a group of long warps -- VGG's fully connected layers, ~150K events per 32 warps -- spread
+  // over several workers; several parts per worker average out regional cost differences.
   const uint64_t C = E + kAlpha * W;
-  const uint64_t T_lo = (uint64_t)(((unsigned __int128)C * gw) / NWK);
-  const uint64_t T_hi = (uint64_t)(((unsigned __int128)C * (gw + 1)) / NWK);
+  const uint64_t NP = (uint64_t)NWK * K1_NRANGE;
   auto wcost = [&](uint64_t w) -> uint64_t { return a.weo[w] + kAlpha * w; };
-  const uint64_t w_lo = gw == 0 ? 0 : search32(0, W, wcost, T_lo);
-  const uint64_t w_hi = last_worker ? W : search32(0, W, wcost, T_hi);
+  auto part_lo = [&](uint64_t j) -> uint64_t {
+    if (j == 0) return 0;
+    if (j >= NP) return W;
+    return search32(0, W, wcost, (uint64_t)(((unsigned __int128)C * j) / NP));
+  };
+#pragma unroll 1
+  for (int ri = 0; ri < K1_NRANGE; ++ri) {
+    const uint64_t j = (uint64_t)ri * NWK + gw;
+    const uint64_t lo = part_lo(j), hi = part_lo(j + 1);
+    if (lane == 0) { wm->rlo[ri] = lo; wm->rhi[ri] = hi; }
+  }
+  __syncwarp();
   auto clampE = [&](uint64_t x) -> uint64_t { return x < E ? x : E; };
 
   // ---- chunk issuer (lane 0): stages the worker's chunk sequence one chunk ahead.  State in shared memory except
   // the prefetched raw end of the block after the issuer's (a register, so its load is not waited on early).
   uint64_t i_pf = 0;
+  auto i_enter = [&](uint32_t ri) {  // lane 0: the first non-empty range from ri on (i_live = 0: none)
+    while (ri < K1_NRANGE && wm->rlo[ri] >= wm->rhi[ri]) ++ri;
+    wm->i_ri = ri;
+    wm->i_live = ri < K1_NRANGE ? 1u : 0u;
+    if (ri >= K1_NRANGE) return;
+    const uint64_t lo = wm->rlo[ri], hi = wm->rhi[ri];
+    const uint64_t s0 = clampE(a.weo[lo]);
+    const uint64_t e_raw = a.weo[umin64(lo + 32, hi)];
+    wm->i_b = lo;  // first warp of the issuer's block
+    wm->i_cs = s0;
+    wm->i_te = umax64(clampE(e_raw), s0);
+    wm->i_pf = e_raw;  // raw end of the block (= raw start of the next block)
+    i_pf = a.weo[umin64(lo + 64, hi)];
+  };
   if (lane == 0) {
-    wm->i_live = 0;
     wm->i_n = 0;
-    if (w_lo < w_hi) {
-      const uint64_t s0 = clampE(a.weo[w_lo]);
-      const uint64_t e_raw = a.weo[umin64(w_lo + 32, w_hi)];
-      wm->i_live = 1;
-      wm->i_b = w_lo;  // first warp of the issuer's block
-      wm->i_cs = s0;
-      wm->i_te = umax64(clampE(e_raw), s0);
-      wm->i_pf = e_raw;  // raw end of the block (= raw start of the next block)
-      i_pf = a.weo[umin64(w_lo + 64, w_hi)];
-    }
+    i_enter(0);
   }
   auto issue = [&]() {  // lane 0 only
     if (!wm->i_live) return;
@@ -442,53 +459,57 @@ __global__ void __launch_bounds__(WPC * 32, 1) k_bbv3(Args3 a) {
       wm->i_cs = ce;
     } else {  // the next block starts where this one ends
       const uint64_t nw0 = wm->i_b + 32;
-      if (nw0 < w_hi) {
+      const uint64_t rhi = wm->rhi[wm->i_ri];
+      if (nw0 < rhi) {
         wm->i_b = nw0;
         wm->i_cs = te;
         wm->i_te = umax64(clampE(i_pf), te);
         wm->i_pf = i_pf;
-        i_pf = a.weo[umin64(nw0 + 64, w_hi)];
+        i_pf = a.weo[umin64(nw0 + 64, rhi)];
       } else {
-        wm->i_live = 0;
+        i_enter(wm->i_ri + 1);
       }
     }
   };
   if (lane == 0) issue();
   __syncwarp();
 
+  uint32_t n_done = 0;  // chunks consumed
+  uint64_t prev_te = 0;
+  uint32_t raw = 0, orr = 0;
+#pragma unroll 1
+  for (int ri = 0; ri < K1_NRANGE; ++ri) {
+  const uint64_t r_lo = wm->rlo[ri], r_hi = wm->rhi[ri];
   // ---- per-block state (all lanes) ----
-  uint64_t w0 = w_lo;              // first warp of the current block
-  uint64_t my_s = 0, blk_end = 0;  // weo[w0 + lane], weo[min(w0 + 32, w_hi)] (raw)
-  if (w0 < w_hi) {
-    my_s = a.weo[umin64(w0 + lane, w_hi)];
-    blk_end = a.weo[umin64(w0 + 32, w_hi)];
+  uint64_t w0 = r_lo;              // first warp of the current block
+  uint64_t my_s = 0, blk_end = 0;  // weo[w0 + lane], weo[min(w0 + 32, r_hi)] (raw)
+  if (w0 < r_hi) {
+    my_s = a.weo[umin64(w0 + lane, r_hi)];
+    blk_end = a.weo[umin64(w0 + 32, r_hi)];
   }
   // kernel of the block's first warp: last k with kwo[k] <= w0
   uint32_t kb = 0;
-  if (w0 < w_hi && a.K > 1) {
+  if (w0 < r_hi && a.K > 1) {
     auto kf = [&](uint64_t kk) -> uint64_t { return a.kwo[kk]; };
     kb = (uint32_t)(search32(1, a.K, kf, w0 + 1) - 1);
   }
   uint64_t kb1 = kb + 1 < a.K ? a.kwo[kb + 1] : ~0ull;  // first warp of the next kernel (prefetched)
-  uint32_t n_done = 0;  // chunks consumed
-  uint64_t prev_te = 0;
-  uint32_t raw = 0, orr = 0;
 
-  while (w0 < w_hi) {
+  while (w0 < r_hi) {
     const uint64_t start_b = __shfl_sync(0xffffffffu, my_s, 0);
-    const uint32_t nw = (uint32_t)umin64(32, w_hi - w0);
+    const uint32_t nw = (uint32_t)umin64(32, r_hi - w0);
     // prefetch the next block's starts (used at its start)
     uint64_t nx_s = 0, nx_end = 0;
-    if (w0 + 32 < w_hi) {
-      nx_s = a.weo[umin64(w0 + 32 + lane, w_hi)];
-      nx_end = a.weo[umin64(w0 + 64, w_hi)];
+    if (w0 + 32 < r_hi) {
+      nx_s = a.weo[umin64(w0 + 32 + lane, r_hi)];
+      nx_end = a.weo[umin64(w0 + 64, r_hi)];
     }
     // warp starts: lane u <= nw holds s_u; non-monotone offsets are latched and made monotone (memory safety)
     const uint64_t s_raw = lane < nw ? my_s : blk_end;
     const uint64_t s_next_raw = __shfl_down_sync(0xffffffffu, s_raw, 1);
     const bool bad = lane < nw && (lane + 1 < nw ? s_next_raw : blk_end) < s_raw;
     // the block's event range, exactly as the chunk issuer computes it: it starts where the previous block ended
-    const uint64_t ts = w0 == w_lo ? clampE(start_b) : prev_te;
+    const uint64_t ts = w0 == r_lo ? clampE(start_b) : prev_te;
     const uint64_t te = umax64(clampE(blk_end), ts);
     uint64_t s = umin64(umax64(clampE(s_raw), ts), te);
     if (__any_sync(0xffffffffu, bad)) {
@@ -745,6 +766,7 @@ __global__ void __launch_bounds__(WPC * 32, 1) k_bbv3(Args3 a) {
     my_s = nx_s;
     blk_end = nx_end;
   }
+  }  // ranges
   if (FUSED) pool_flush(a, wm);
 }
 
