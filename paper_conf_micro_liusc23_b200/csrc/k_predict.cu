@@ -141,19 +141,30 @@ __global__ void __launch_bounds__(256) k_bb_predict_long(uint32_t B, const uint6
     const uint64_t* ds = dur + k * B;
     uint64_t lo = 0, hi = 0;
     uint32_t miss = 0;
-#pragma unroll 4
-    for (uint64_t i = s + lane; i < e; i += 32) {
-      const uint32_t bv = bb[i];
+    auto add = [&](uint32_t bv, uint64_t i) {
       if (bv >= B) {
         latch(err, PHOTON_ERANGE, (int64_t)i);
-        continue;
+        return;
       }
       const int64_t f = fs[bv];
       const uint64_t x = f >= 0 ? ds[bv] : 0ull;
       miss += f < 0 ? 1u : 0u;
       lo += x;
       hi += lo < x;
+    };
+    // 16-byte vectors of 8 ids over the aligned middle (eight independent table lookups per lane and load), the
+    // unaligned head and tail id by id
+    const bool vec = ((uintptr_t)bb & 15) == 0;
+    const uint64_t s8 = vec ? umin64((s + 7) & ~7ull, e) : e, e8 = vec ? umax64(e & ~7ull, s8) : e;
+    for (uint64_t i = s + lane; i < s8; i += 32) add(bb[i], i);
+#pragma unroll 2
+    for (uint64_t i = s8 + 8 * (uint64_t)lane; i < e8; i += 256) {
+      const uint4 v = __ldg(reinterpret_cast<const uint4*>(bb + i));
+      const uint32_t w4[4] = {v.x, v.y, v.z, v.w};
+#pragma unroll
+      for (int q = 0; q < 8; ++q) add((w4[q >> 1] >> ((q & 1) * 16)) & 0xFFFFu, i + q);
     }
+    for (uint64_t i = e8 + lane; i < e; i += 32) add(bb[i], i);
 #pragma unroll
     for (int o = 16; o > 0; o >>= 1) {
       const uint64_t ol = __shfl_xor_sync(0xffffffffu, lo, o), oh = __shfl_xor_sync(0xffffffffu, hi, o);
