@@ -1184,20 +1184,25 @@ __device__ uint64_t locate_record(const photon_timing& t, const JobMap& jm, cons
   }
   const unsigned hit = __ballot_sync(0xffffffffu, rank < incl && rank >= incl - cnt);
   const int owner = __ffs(hit) - 1;
-  uint64_t pos = ~0ull;
-  if ((int)lane == owner) {
-    uint32_t r = (uint32_t)(rank - (incl - cnt));
-    for (int u = 0; u < PER; ++u) {
-      const uint64_t i = l0 + u;
-      uint32_t x = t.bb[i];
-      if (x >= B) x = 0;
-      if (x == b) {
-        if (r == 0) { pos = i - a; break; }
-        --r;
-      }
-    }
+  if (owner < 0) return ~0ull;
+  // the owner's 64-record slice, two records per lane (one round of loads, no serial walk): the r-th match
+  const uint32_t r = (uint32_t)__shfl_sync(0xffffffffu, (uint32_t)(rank - (incl - cnt)), owner);
+  static_assert(PER == 64, "two records per lane");
+  const uint64_t i0 = cs + (uint64_t)owner * PER + 2 * lane;
+  uint32_t x0 = i0 < ce ? (uint32_t)t.bb[i0] : kNone, x1 = i0 + 1 < ce ? (uint32_t)t.bb[i0 + 1] : kNone;
+  if (x0 != kNone && x0 >= B) x0 = 0;
+  if (x1 != kNone && x1 >= B) x1 = 0;
+  const uint32_t m0 = x0 == b ? 1u : 0u, m1 = x1 == b ? 1u : 0u, c2 = m0 + m1;
+  uint32_t in2 = c2;
+  for (int o = 1; o < 32; o <<= 1) {
+    const uint32_t y = __shfl_up_sync(0xffffffffu, in2, o);
+    if ((int)lane >= o) in2 += y;
   }
-  return __shfl_sync(0xffffffffu, pos, owner < 0 ? 0 : owner);
+  const uint32_t ex2 = in2 - c2;  // matches before this lane's pair
+  uint64_t pos = ~0ull;
+  if (r >= ex2 && r < in2) pos = (r == ex2 && m0 ? i0 : i0 + 1) - a;
+  const unsigned ph = __ballot_sync(0xffffffffu, pos != ~0ull);
+  return __shfl_sync(0xffffffffu, pos, ph ? __ffs(ph) - 1 : 0);
 }
 
 // group g -> (k, b): mode 0 (radix path) g = b*K + k; 1 (job path, B <= 256) g = k*B + b; 2 (compact) gkb[g]
