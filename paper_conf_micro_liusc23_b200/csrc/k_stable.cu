@@ -1257,7 +1257,11 @@ __device__ __forceinline__ u128 block_sum_u128(u128 v, uint64_t* slo, uint64_t* 
 __global__ void __launch_bounds__(256) k_switch(const int64_t* first_stable, const uint64_t* kbb, uint32_t K,
                                                 uint32_t B, uint32_t rnum, uint32_t rden, int64_t* switch_at) {
   __shared__ uint64_t slo[8], shi[8];
+  __shared__ uint64_t s_t[256], s_w[256];
+  __shared__ uint32_t s_n;
+  __shared__ unsigned long long s_best;
   for (uint32_t k = blockIdx.x; k < K; k += gridDim.x) {
+    if (threadIdx.x == 0) s_best = ~0ull;
     const int64_t* fs = first_stable + (uint64_t)k * B;
     const uint64_t* w = kbb + (uint64_t)k * B;
     u128 t = 0, a = 0;
@@ -1268,7 +1272,31 @@ __global__ void __launch_bounds__(256) k_switch(const int64_t* first_stable, con
     const u128 total = block_sum_u128(t, slo, shi);
     const u128 all = block_sum_u128(a, slo, shi);
     int64_t ans = -1;
-    if (total > 0 && (u128)rden * all > (u128)rnum * total) {
+    // the stable BBs compacted (their t_b are distinct: one record each); with at most 256 of them, each one's
+    // acc(t_b) is summed over the compacted list in shared memory and the answer is the least qualifying t_b
+    if (threadIdx.x == 0) s_n = 0;
+    __syncthreads();
+    for (uint32_t b = threadIdx.x; b < B; b += blockDim.x)
+      if (fs[b] >= 0) {
+        const uint32_t j = atomicAdd(&s_n, 1u);
+        if (j < 256) { s_t[j] = (uint64_t)fs[b]; s_w[j] = w[b]; }
+      }
+    __syncthreads();
+    const uint32_t ns = s_n;
+    if (total > 0 && (u128)rden * all > (u128)rnum * total && ns <= 256) {
+      unsigned long long best = ~0ull;
+      if (threadIdx.x < ns) {
+        const uint64_t ti = s_t[threadIdx.x];
+        u128 acc = 0;
+        for (uint32_t j = 0; j < ns; ++j)
+          if (s_t[j] <= ti) acc += s_w[j];
+        if ((u128)rden * acc > (u128)rnum * total) best = ti;
+      }
+      for (int o = 16; o > 0; o >>= 1) best = umin64(best, __shfl_xor_sync(0xffffffffu, best, o));
+      if ((threadIdx.x & 31) == 0) atomicMin(&s_best, best);
+      __syncthreads();
+      ans = (int64_t)s_best;
+    } else if (total > 0 && (u128)rden * all > (u128)rnum * total) {
       uint64_t lo = 0, hi = 0xFFFFFFFFull;  // invariant: acc(hi) passes
       while (lo < hi) {
         uint64_t mid = (lo + hi) >> 1;
