@@ -412,17 +412,31 @@ __global__ void __launch_bounds__(256) k_presence(photon_timing t, const uint64_
     const uint32_t k = upper_idx(coff, t.n_kernels, job);
     const uint64_t a = umin64(t.kernel_rec_off[k], t.n_records), e = umin64(t.kernel_rec_off[k + 1], t.n_records);
     const uint64_t cs = a + (job - coff[k]) * JOB, ce = umin64(cs + JOB, e);
-    // lanes hitting the same bitmap word OR their bits together first (one shared atomic per distinct word: a
-    // kernel's few BB ids share words, and 32 same-address atomics would serialise)
-    for (uint64_t i0 = cs; i0 < ce; i0 += 32) {
-      const uint64_t i = i0 + lane;
-      uint32_t bb = i < ce ? (uint32_t)t.bb[i] : 0u;
-      if (bb >= t.n_bb) bb = 0;  // bad ids are latched by the scatter
-      const uint32_t w = i < ce ? bb >> 5 : kNone;
-      const unsigned peers = __match_any_sync(0xffffffffu, w);
-      const uint32_t v = __reduce_or_sync(peers, 1u << (bb & 31));
-      if (w != kNone && lane == __ffs(peers) - 1) atomicOr(&m[w], v);
+    // each lane ORs the bits of its run of records into a register while they stay in one bitmap word (a kernel's
+    // few BB ids share words) and flushes the word to shared memory when it changes: no warp collective per record;
+    // the aligned middle of the job as 16-byte vectors of 8 ids, the unaligned head and tail id by id
+    uint32_t cwd = kNone, cbits = 0;
+    auto put = [&](uint32_t id) {
+      if (id >= t.n_bb) id = 0;  // bad ids are latched by the scatter
+      const uint32_t wd = id >> 5;
+      if (wd != cwd) {
+        if (cbits) atomicOr(&m[cwd], cbits);
+        cwd = wd;
+        cbits = 0;
+      }
+      cbits |= 1u << (id & 31);
+    };
+    const bool vec = ((uintptr_t)t.bb & 15) == 0;
+    const uint64_t s8 = vec ? umin64((cs + 7) & ~7ull, ce) : ce, e8 = vec ? umax64(ce & ~7ull, s8) : ce;
+    for (uint64_t i = cs + lane; i < s8; i += 32) put(t.bb[i]);
+    for (uint64_t i = s8 + 8 * (uint64_t)lane; i < e8; i += 256) {
+      const uint4 v = __ldg(reinterpret_cast<const uint4*>(t.bb + i));
+      const uint32_t w4[4] = {v.x, v.y, v.z, v.w};
+#pragma unroll
+      for (int q = 0; q < 8; ++q) put((w4[q >> 1] >> ((q & 1) * 16)) & 0xFFFFu);
     }
+    for (uint64_t i = e8 + lane; i < ce; i += 32) put(t.bb[i]);
+    if (cbits) atomicOr(&m[cwd], cbits);
     __syncwarp();
     for (uint32_t w = lane; w < nw; w += 32) {
       const uint32_t v = m[w];
