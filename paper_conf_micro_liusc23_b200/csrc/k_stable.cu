@@ -549,6 +549,7 @@ __global__ void __launch_bounds__(HW * 32) k_job_hist(photon_timing t, JobMap jm
     }
     // lane-contiguous 8-id blocks from the aligned start: a lane counts at most 8 ids per 256-id step
     const uint64_t c0 = cs & ~7ull;
+    uint32_t cw_ = kNone, cb_ = 0, cl_ = 0;  // compact ids: the lane's cached bitmap word (index, bits, base)
     for (uint64_t i = c0 + lane * 8; i < ce; i += 256) {
       uint32_t w[4];
       if (vec && i + 8 <= t.n_records) {
@@ -565,7 +566,17 @@ __global__ void __launch_bounds__(HW * 32) k_job_hist(photon_timing t, JobMap jm
         const uint64_t q = i + j;
         uint32_t d = (w[j >> 1] >> ((j & 1) * 16)) & 0xFFFFu;
         if (q >= cs && q < ce) {
-          const uint32_t x = jm.lid(k, d < B ? d : 0u);  // bad ids count as bb 0 (latched by the scatter)
+          d = d < B ? d : 0u;  // bad ids count as bb 0 (latched by the scatter)
+          uint32_t x = d;
+          if (jm.compact) {  // local id: the lane keeps the last bitmap word's base and bits (a kernel's ids share
+                             // few words)
+            if ((d >> 5) != cw_) {
+              cw_ = d >> 5;
+              cb_ = jm.bits[(uint64_t)k * jm.nw + cw_];
+              cl_ = jm.lbase[(uint64_t)k * jm.nw + cw_];
+            }
+            x = cl_ + __popc(cb_ & ((1u << (d & 31)) - 1u));
+          }
           hb8[x * 32 + lane] += 1;
         }
       }
