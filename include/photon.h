@@ -204,7 +204,8 @@ PHOTON_API int photon_match_resolve(photon_ctx *ctx, uint32_t n_kernels, const u
  * group workspace `gws` (photon_group_workspace_bytes), then photon_kernel_match with the match workspace `mws`
  * (photon_match_workspace_bytes(K, out->capacity, ...)) -- the same results and device errors (each workspace
  * latches its own part's).  The library runs independent parts on two internal streams (the filter profiles,
- * pair filter and bucketing beside the canonical sort; the warp_type write beside A3/A4) with event forks and
+ * pair filter and its candidate segments beside the canonical sort, which also writes A3's g and g/N; the
+ * warp_type write beside A4) with event forks and
  * joins: all work is ordered after earlier work on `stream`, and later work on `stream` sees every output.  The
  * fork / join is captured with the rest when `stream` is being captured into a CUDA graph. */
 PHOTON_API int photon_analyse(photon_ctx *ctx, const photon_trace *trace, void *group_ws, size_t group_ws_bytes,
