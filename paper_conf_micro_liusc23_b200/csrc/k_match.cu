@@ -236,10 +236,9 @@ __host__ __device__ __forceinline__ uint64_t filter_jobs_before(uint64_t kb) {
 // word, give sum_j |q_k[j] - q_r[j]| with four VABSDIFF4.ACC per pair (the k-side words stay in registers for the
 // whole job); a sum >= thr8 proves D >= theta.  Fine level, only for pairs the coarse level keeps: the fp32
 // profile distance (bin-major shared tiles).  The k-block stays in shared memory for the job; the next r-block is
-// fetched into registers while the current one is scored.  Survivors are collected in a shared list per job and
-// appended with one global atomic per CTA.
+// fetched into registers while the current one is scored.  A tile's survivors are collected in a shared list of
+// tile-local (i, j) (it cannot overflow) and appended after the tile with one global atomic.
 constexpr int FTP = FT + 4;  // row stride (floats) of the bin-major profile tiles
-constexpr uint32_t kFiltBuf = 1024;  // survivors kept in shared memory per job
 __device__ __forceinline__ uint32_t sad4(uint32_t a, uint32_t b, uint32_t acc) { return __vsadu4(a, b) + acc; }
 
 // Band order.  f(k) = sum_{j < 8} q_k[j] - sum_{j >= 8} q_k[j] (u8 profile) satisfies |f(k) - f(r)| <=
@@ -367,8 +366,7 @@ __global__ void __launch_bounds__(256) k_pair_filter(ScanArgs a, uint64_t job0, 
   __shared__ uint32_t kidk[FT], kidr[2][FT];  // the kernels of the tile rows / columns
   // band order: the r-block's fp32 profiles staged too (its tiles are dense in coarse survivors); row stride 17
   __shared__ float prs[BAND ? 2 : 1][BAND ? FT * 17 : 1];
-  constexpr uint32_t NBUF_S = BAND ? 2 * kFiltBuf : kFiltBuf;  // band jobs are dense in survivors
-  __shared__ uint64_t s_buf[NBUF_S];         // the job's survivors
+  __shared__ uint16_t s_loc[FT * FT];       // the tile's survivors, tile-local (i, j)
   __shared__ uint32_t s_n;
   __shared__ unsigned long long s_base;
   const int tid = threadIdx.x;
@@ -470,45 +468,39 @@ __global__ void __launch_bounds__(256) k_pair_filter(ScanArgs a, uint64_t job0, 
       for (int b = 0; b < 16; ++b) d += fabsf(pk[b][i] - pr[b]);
       if (!(d < a.bound)) keep &= ~(1u << bit);
     }
-    // survivors go to the CTA's shared list (flushed to the global list once per job: no global atomic, whose
-    // latency would hold the whole CTA at the next barrier, inside the loop); a full list spills directly
+    // survivors of this tile go to a shared list as tile-local (i, j) (at most FT * FT, so it never overflows) and
+    // are flushed to the global list after the tile: one global atomic per tile with survivors
     for (uint32_t m = keep; m; m &= m - 1) {
       const int bit = __ffs(m) - 1;
-      uint32_t k = k0 + i0 + (bit >> 2), r = r0 + j0 + (bit & 3);
-      if (BAND) {
-        const uint32_t x = kidk[i0 + (bit >> 2)], y = ridr[j0 + (bit & 3)];
-        k = x > y ? x : y;
-        r = x > y ? y : x;
-      }
-      const uint64_t pr = ((uint64_t)k << 32) | r;
       const uint32_t sp = atomicAdd(&s_n, 1u);
-      if (sp < NBUF_S) {
-        s_buf[sp] = pr;
-      } else {
-        const unsigned long long pos = atomicAdd((unsigned long long*)a.n_maybe, 1ull);
+      s_loc[sp] = (uint16_t)((i0 + (bit >> 2)) * FT + j0 + (bit & 3));
+    }
+    __syncthreads();
+    const uint32_t ns = s_n;
+    if (ns) {
+      if (tid == 0) s_base = atomicAdd((unsigned long long*)a.n_maybe, (unsigned long long)ns);
+      __syncthreads();
+      for (uint32_t t = tid; t < ns; t += 256) {
+        const uint32_t ij = s_loc[t], i = ij / FT, j = ij % FT;
+        uint32_t k = k0 + i, r = r0 + j;
+        if (BAND) {
+          const uint32_t x = kidk[i], y = ridr[j];
+          k = x > y ? x : y;
+          r = x > y ? y : x;
+        }
+        const unsigned long long pos = s_base + t;
         if (pos < a.cap) {
-          a.maybe[pos] = pr;
+          a.maybe[pos] = ((uint64_t)k << 32) | r;
           if (a.kcnt) atomicAdd(&a.kcnt[k], 1u);
         } else {
           latch(a.err, PHOTON_ECAPACITY, (int64_t)pos);
         }
       }
+      __syncthreads();  // the list is read before it is reset
+      if (tid == 0) s_n = 0;
     }
     if (rb < rb1) store(cur ^ 1);  // that buffer was last read before the previous barrier
     __syncthreads();
-  }
-  // flush the job's shared list: one global atomic per CTA
-  const uint32_t ns = s_n < NBUF_S ? s_n : NBUF_S;
-  if (tid == 0 && ns) s_base = atomicAdd((unsigned long long*)a.n_maybe, (unsigned long long)ns);
-  __syncthreads();
-  for (uint32_t i = tid; i < ns; i += 256) {
-    const unsigned long long pos = s_base + i;
-    if (pos < a.cap) {
-      a.maybe[pos] = s_buf[i];
-      if (a.kcnt) atomicAdd(&a.kcnt[(uint32_t)(s_buf[i] >> 32)], 1u);
-    } else {
-      latch(a.err, PHOTON_ECAPACITY, (int64_t)pos);
-    }
   }
 }
 
