@@ -79,7 +79,7 @@ struct Carver {
   }
 };
 
-// ---- single-CTA exclusive scan of u32 counts into u64 offsets (1024 threads) ---------------------------------
+// ---- single-CTA exclusive scan of u32 counts into u64 offsets (any multiple of 32 threads) -------------------
 // off[i] = sum of cnt[0..i), off[n] = the total; zero[i] = 0 when zero != nullptr.  Tiles of 1024 x 8 counts: each
 // thread sums 8 consecutive counts in registers, one block scan of the thread sums per tile (two barriers), so a
 // K of 10^4 takes two tiles.  Returns the total (thread 0 only).
@@ -89,7 +89,7 @@ __device__ __forceinline__ uint64_t cta_scan_counts(const uint32_t* __restrict__
   __shared__ uint64_t s_ws[32];
   const uint32_t tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
   uint64_t carry = 0;  // identical in every thread
-  for (uint32_t base = 0; base < n; base += 1024u * IT) {
+  for (uint32_t base = 0; base < n; base += blockDim.x * IT) {
     uint32_t v[IT];
     const uint32_t i0 = base + tid * IT;
     uint64_t sum = 0;

@@ -214,6 +214,9 @@ struct ScanArgs {
   const uint32_t* bandlo;   // [NB] first r-block that can hold a partner of k-block kb
   const uint64_t* job_off;  // [NB + 1] jobs before k-block kb
   uint32_t* kcnt;           // survivors per k (the sizes of the candidate segments), or nullptr
+  uint32_t* ticket;         // with kcnt: the CTAs' completion counter; the last one scans kcnt into seg_off / seg_cur
+  uint64_t* seg_off;
+  uint32_t* seg_cur;
 };
 
 // Jobs: one k-block (FT kernels) against a run of up to FR r-blocks (rb <= kb).  S(kb) = jobs before k-block kb
@@ -332,11 +335,9 @@ __global__ void __launch_bounds__(1024) k_band_sort_jobs(uint32_t K, const uint3
 }
 
 template <bool BAND>
-__global__ void __launch_bounds__(256) k_pair_filter(ScanArgs a, uint64_t job0, uint32_t kb_lo, uint32_t kb_hi) {
-  const uint64_t job = job0 + blockIdx.x;
+__device__ void pair_filter_job(const ScanArgs& a, uint64_t job, uint32_t kb_lo, uint32_t kb_hi) {
   uint32_t kb, rb0, rb1;
   if constexpr (BAND) {
-    if (job >= a.job_off[kb_hi]) return;  // the grid is sized for every tile; the band needs fewer jobs
     uint32_t lo = 0, hi = kb_hi - 1;  // last kb with job_off[kb] <= job
     while (lo < hi) {
       const uint32_t mid = (lo + hi + 1) >> 1;
@@ -501,6 +502,24 @@ __global__ void __launch_bounds__(256) k_pair_filter(ScanArgs a, uint64_t job0, 
     }
     if (rb < rb1) store(cur ^ 1);  // that buffer was last read before the previous barrier
     __syncthreads();
+  }
+}
+
+template <bool BAND>
+__global__ void __launch_bounds__(256) k_pair_filter(ScanArgs a, uint64_t job0, uint32_t kb_lo, uint32_t kb_hi) {
+  const uint64_t job = job0 + blockIdx.x;
+  // band: the grid is sized for every tile of the triangle, the band needs fewer jobs
+  if (!BAND || job < a.job_off[kb_hi]) pair_filter_job<BAND>(a, job, kb_lo, kb_hi);
+  if (a.ticket) {  // the last CTA to finish scans the per-k survivor counts into the candidate segments
+    __shared__ bool s_last;
+    __threadfence();
+    __syncthreads();
+    if (threadIdx.x == 0) s_last = atomicAdd(a.ticket, 1u) + 1 == gridDim.x;
+    __syncthreads();
+    if (s_last) {
+      __threadfence();
+      cta_scan_counts(a.kcnt, a.K, a.seg_off, a.seg_cur);
+    }
   }
 }
 
@@ -904,10 +923,9 @@ void launch_filter_band(ScanArgs a, const MatchWs& mw, cudaStream_t s) {
 void launch_segments(uint32_t K, const MatchWs& mw, DevErr* err, int num_sms, cudaStream_t s, bool counted = false) {
   const unsigned gb = (unsigned)umin64(ceil_div(mw.pair_cap, 256), (uint64_t)num_sms * 64);
   cudaMemsetAsync(mw.close_cnt, 0, sizeof(uint32_t) * K, s);
-  if (!counted) {  // else the filter counted its survivors per k
-    cudaMemsetAsync(mw.cand_cnt, 0, sizeof(uint32_t) * K, s);
-    note_launch(), k_cand_count<<<gb, 256, 0, s>>>(mw.maybe, mw.pair_cap, mw.n_maybe, K, mw.cand_cnt, err);
-  }
+  if (counted) return;  // the filter counted its survivors per k and its last CTA scanned them
+  cudaMemsetAsync(mw.cand_cnt, 0, sizeof(uint32_t) * K, s);
+  note_launch(), k_cand_count<<<gb, 256, 0, s>>>(mw.maybe, mw.pair_cap, mw.n_maybe, K, mw.cand_cnt, err);
   note_launch(), k_cand_scan<<<1, 1024, 0, s>>>(mw.cand_cnt, K, mw.cand_off, mw.cand_cur);
 }
 void launch_exact(ScanArgs a, bool fused, const MatchWs& mw, uint64_t* pairs, uint64_t pair_cap, uint64_t* n_pairs,
@@ -948,8 +966,12 @@ cudaError_t launch_analyse_filter(uint32_t K, const uint64_t* kto, const uint32_
                                                                                        mw.prof, mw.invn, mw.prof8,
                                                                                        err);
   ScanArgs a = scan_args(K, 0, K, kto, nullptr, mass, wt, p, mw, err);
-  a.kcnt = mw.cand_cnt;  // the filter counts its survivors per k (no separate count pass)
+  a.kcnt = mw.cand_cnt;  // the filter counts its survivors per k (no separate count pass) and its last CTA scans
+  a.ticket = mw.flag + 2;  // the counts into the candidate segments (no separate scan launch)
+  a.seg_off = mw.cand_off;
+  a.seg_cur = mw.cand_cur;
   cudaMemsetAsync(mw.cand_cnt, 0, sizeof(uint32_t) * K, sb);
+  cudaMemsetAsync(mw.flag + 2, 0, sizeof(uint32_t), sb);
   if (PHOTON_BAND && K <= kBandMaxK) launch_filter_band(a, mw, sb);  // f in [-2040, 2040]: the counting sort's 4096 bins
   else launch_filter(a, sb);
   launch_segments(K, mw, err, num_sms, sb, true);
