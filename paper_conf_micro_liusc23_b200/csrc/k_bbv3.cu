@@ -25,7 +25,7 @@
 //  * After the loop each lane sums its warp's pieces (owner column, then slot 0 of every later lane it spans) into
 //    16 key registers, carried across the chunks of a block; the worker's cells are cleared with 16-byte stores.
 //  * Fused: at the block's end the keys are hashed, grouped with __match_any_sync plus an exact 17-word check, and
-//    each distinct (kernel, key) of the block is looked up in the worker's direct-mapped cache of its recent
+//    each distinct (kernel, key) of the block is looked up in the worker's 2-way set-associative cache of its recent
 //    entries (hash -> entry id): a hit that matches the entry's own key exactly adds the block's count to it,
 //    otherwise the key becomes a new 80-byte entry (key, first warp, kernel, count) from the worker's run of the
 //    global entry pool (one atomic per ENT_BLK entries).  Each warp records its entry index (u32).  The entries
@@ -55,9 +55,6 @@ constexpr int SMEM_TBL_MAX = 4096;  // BB table entries kept in shared memory (e
 #endif
 #ifndef K1_VNX
 #define K1_VNX 1
-#endif
-#ifndef K1_PRMT
-#define K1_PRMT 0
 #endif
 #ifndef K1_QMAX
 #define K1_QMAX 11
@@ -109,14 +106,6 @@ struct Args3 {
 };
 
 // per-worker scratch in shared memory
-#ifndef K1_CTAG32
-#define K1_CTAG32 0
-#endif
-#if K1_CTAG32
-#define K1_TAG(h) ((uint32_t)((h) >> 32) | 1u)
-#else
-#define K1_TAG(h) (h)
-#endif
 #ifndef K1_NRANGE
 #define K1_NRANGE 1  // ranges per worker: worker g takes parts g, g + G, ... of a cost partition into G * K1_NRANGE
 #endif
@@ -137,23 +126,13 @@ struct WMisc {
   uint64_t rlo[K1_NRANGE], rhi[K1_NRANGE];  // the worker's warp ranges (round-robin over the cost partition)
   // the worker's current block of pool entries (fused)
   uint64_t e_next, e_end;
-  // direct-mapped cache of the worker's recent entries (hash -> entry id): a type seen again in a later block of
-  // the worker adds to its entry after an exact key check instead of opening a new one
-#if K1_CTAG32
-  uint32_t ch[kEntCache];  // tag: high hash word | 1 (0 = empty; a false tag hit fails the exact key check)
-#else
+  // K1_CWAYS-way set-associative cache of the worker's recent entries (hash -> entry id): a type seen again in a
+  // later block of the worker adds to its entry after an exact key check instead of opening a new one
   uint64_t ch[kEntCache];
-#endif
   uint32_t ce[kEntCache];
 };
 constexpr uint32_t kWMiscBytes = (sizeof(WMisc) + 127) & ~127u;
 
-// x << s with s >= 64 giving 0 (PTX shl clamps the shift amount)
-__device__ __forceinline__ uint64_t shl64_clamp(uint64_t x, uint32_t s) {
-  uint64_t r;
-  asm("shl.b64 %0, %1, %2;" : "=l"(r) : "l"(x), "r"(s));
-  return r;
-}
 __device__ __forceinline__ void red_add(uint32_t saddr, uint32_t v) {
   // no "memory" clobber: cells are written only by these adds and read only after __syncwarp
   asm volatile("red.shared.add.u32 [%0], %1;" ::"r"(saddr), "r"(v));
@@ -252,8 +231,8 @@ __device__ void finalize_fused(const Args3& a, WMisc* wm, uint64_t w0, bool vali
   uint32_t cway = cslot;
 #pragma unroll
   for (uint32_t q = NWAY - 1; q > 0; --q)
-    if (wm->ch[cslot + q] == K1_TAG(h)) cway = cslot + q;
-  if (is_l && wm->ch[cway] == K1_TAG(h)) {
+    if (wm->ch[cslot + q] == h) cway = cslot + q;
+  if (is_l && wm->ch[cway] == h) {
     const uint32_t e = wm->ce[cway];
     if (e < a.ep.cap) {  // the exact check against the entry itself (written by this warp earlier)
       TileEntry* d = a.ep.ent + e;
@@ -311,7 +290,7 @@ __device__ void finalize_fused(const Args3& a, WMisc* wm, uint64_t w0, bool vali
       wm->ch[cslot + q] = wm->ch[cslot + q - 1];
       wm->ce[cslot + q] = wm->ce[cslot + q - 1];
     }
-    wm->ch[cslot] = K1_TAG(h);
+    wm->ch[cslot] = h;
     wm->ce[cslot] = (uint32_t)umin64(id, 0xFFFFFFFFull);
   }
   if (lane == 0) { wm->e_next = e_next; wm->e_end = e_end; }
@@ -609,9 +588,6 @@ __global__ void __launch_bounds__(WPC * 32, 1) k_bbv3(Args3 a) {
           tv[6] = look(__funnelshift_l(v.w, v.w, 2));
           tv[7] = look(v.w >> 14);
         };
-#if K1_PRMT
-        uint32_t cbx = __byte_perm(col, 0u, 0u), cby = __byte_perm(coln, 0u, 0u);  // column bytes, replicated
-#endif
         uint4 vnx = sb4[0];
         uint32_t tv[8];
         lookup(vnx, tv);
@@ -630,19 +606,8 @@ __global__ void __launch_bounds__(WPC * 32, 1) k_bbv3(Args3 a) {
           if (MARK) orr |= (tv[0] | tv[1] | tv[2] | tv[3]) | (tv[4] | tv[5] | tv[6] | tv[7]);
           if (nb2 >= p0 + 8u) {  // at most one boundary (at nb) in the word: events j >= nb - p0 go to coln
             const uint32_t mcut = nb - p0;
-#if K1_PRMT
-            // the column bytes of the 8 events as two byte vectors (a worker's 64 columns share one 256-byte span,
-            // so a cell address is cw | column byte | row bits): one LOP3 per 4 events, one PRMT per event
-            const uint64_t bm = shl64_clamp(~0ull, mcut * 8u);  // bytes j >= mcut
-            const uint32_t cv0 = (cbx & ~(uint32_t)bm) | (cby & (uint32_t)bm);
-            const uint32_t cv1 = (cbx & ~(uint32_t)(bm >> 32)) | (cby & (uint32_t)(bm >> 32));
-#pragma unroll
-            for (int j = 0; j < 8; ++j)
-              red(__byte_perm(j < 4 ? cv0 : cv1, cw, 0x7650u + (j & 3)) | (tv[j] & M::ROFF), M::val(tv[j]));
-#else
 #pragma unroll
             for (int j = 0; j < 8; ++j) red(((uint32_t)j < mcut ? col : coln) | (tv[j] & M::ROFF), M::val(tv[j]));
-#endif
             if (nb <= p0 + 8u) {
               ++u;
               col = coln;
@@ -650,10 +615,6 @@ __global__ void __launch_bounds__(WPC * 32, 1) k_bbv3(Args3 a) {
               nb = nb2;
               PHOTON_DCHECK(u + 2u < 40u, "K1 warp index past rel[]", u);
               nb2 = wm->rel[u + 2];
-#if K1_PRMT
-              cbx = cby;
-              cby = __byte_perm(coln, 0u, 0u);
-#endif
             }
           } else {
             // several warp boundaries in the word (warps shorter than 8 events): event by event
@@ -673,10 +634,6 @@ __global__ void __launch_bounds__(WPC * 32, 1) k_bbv3(Args3 a) {
             coln = pcol(u + 1);
             nb = wm->rel[u + 1];
             nb2 = wm->rel[u + 2];
-#if K1_PRMT
-            cbx = __byte_perm(col, 0u, 0u);
-            cby = __byte_perm(coln, 0u, 0u);
-#endif
           }
           lookup(vnx, tv);
         }
