@@ -615,7 +615,13 @@ __device__ double group_dfp(const uint64_t* __restrict__ sig, const float* __res
 #define PHOTON_XG 8  // lanes per pair (profiling builds may override)
 #endif
 constexpr int XG = PHOTON_XG;
-__global__ void __launch_bounds__(256) k_pair_exact(ScanArgs a, uint64_t* pairs, uint64_t pair_cap,
+#ifndef PHOTON_XGRID
+#define PHOTON_XGRID 5  // k_pair_exact CTAs per SM (grid-stride rounds; all resident)
+#endif
+#ifndef PHOTON_XMINB
+#define PHOTON_XMINB 5  // k_pair_exact: minimum resident CTAs per SM (a register cap without spills)
+#endif
+__global__ void __launch_bounds__(256, PHOTON_XMINB) k_pair_exact(ScanArgs a, uint64_t* pairs, uint64_t pair_cap,
                                                     uint64_t* n_pairs) {
   uint64_t n = *a.n_maybe;
   if (n > a.cap) n = a.cap;
@@ -935,7 +941,7 @@ void launch_exact(ScanArgs a, bool fused, const MatchWs& mw, uint64_t* pairs, ui
     a.cbeg = mw.cand_off;
     a.ccnt = mw.close_cnt;
   }
-  note_launch(), k_pair_exact<<<(unsigned)num_sms * 8, 256, 0, s>>>(a, pairs, pair_cap, n_pairs);
+  note_launch(), k_pair_exact<<<(unsigned)num_sms * PHOTON_XGRID, 256, 0, s>>>(a, pairs, pair_cap, n_pairs);
 }
 }  // namespace
 
