@@ -505,8 +505,16 @@ __device__ void pair_filter_job(const ScanArgs& a, uint64_t job, uint32_t kb_lo,
   }
 }
 
+#ifndef PHOTON_FMINB
+#define PHOTON_FMINB 0  // > 0: __launch_bounds__(256, PHOTON_FMINB)
+#endif
+#if PHOTON_FMINB > 0
+#define PHOTON_FMINB_LB __launch_bounds__(256, PHOTON_FMINB)
+#else
+#define PHOTON_FMINB_LB __launch_bounds__(256)
+#endif
 template <bool BAND>
-__global__ void __launch_bounds__(256) k_pair_filter(ScanArgs a, uint64_t job0, uint32_t kb_lo, uint32_t kb_hi) {
+__global__ void PHOTON_FMINB_LB k_pair_filter(ScanArgs a, uint64_t job0, uint32_t kb_lo, uint32_t kb_hi) {
   const uint64_t job = job0 + blockIdx.x;
   // band: the grid is sized for every tile of the triangle, the band needs fewer jobs
   if (!BAND || job < a.job_off[kb_hi]) pair_filter_job<BAND>(a, job, kb_lo, kb_hi);

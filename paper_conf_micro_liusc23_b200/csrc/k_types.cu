@@ -374,7 +374,15 @@ __global__ void __launch_bounds__(1024) k_sort_large(HashTable ht, uint32_t K, c
 // worker's entries are consecutive, so neighbours often share a key): equal (kernel, key) entries are grouped with
 // __match_any_sync on the hash plus an exact key check, their counts / first warps combined in shared memory, and
 // only each group's leader probes the table.  Unused entries (count 0) get no slot.
-__global__ void __launch_bounds__(256) k_entries_insert(EntryPool ep, HashTable ht, DevErr* err) {
+#ifndef PHOTON_IMINB
+#define PHOTON_IMINB 5  // > 0: __launch_bounds__(256, PHOTON_IMINB) (5: an 8-byte spill, measured -4 us on C5)
+#endif
+#if PHOTON_IMINB > 0
+#define PHOTON_IMINB_LB __launch_bounds__(256, PHOTON_IMINB)
+#else
+#define PHOTON_IMINB_LB __launch_bounds__(256)
+#endif
+__global__ void PHOTON_IMINB_LB k_entries_insert(EntryPool ep, HashTable ht, DevErr* err) {
   __shared__ uint32_t s_cnt[256];
   __shared__ unsigned long long s_first[256];
   const uint64_t n = umin64(*ep.count, ep.cap);
