@@ -241,7 +241,18 @@ def run_photon(args):
             os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(so.getsockname()[1]), RANK="0",
                               WORLD_SIZE="1")
             so.close()
-        dist.init_process_group("nccl", device_id=dev)
+        # NCCL's own prints at communicator creation (its version line when the environment sets NCCL_DEBUG=VERSION)
+        # go to stderr: stdout carries the one JSON line
+        sys.stdout.flush()
+        saved = os.dup(1)
+        os.dup2(2, 1)
+        try:
+            dist.init_process_group("nccl", device_id=dev)
+            dist.barrier()
+        finally:
+            sys.stdout.flush()
+            os.dup2(saved, 1)
+            os.close(saved)
     num, den = (int(x) for x in args.theta.split("/"))
     g = tg.Generator(args.config, args.seed)
     if sh:
