@@ -323,6 +323,9 @@ def test_match_many_kernels_synthetic(ph, K):
     gm = _np(m["match"], np.int64)
     assert (om >= 0).sum() > K // 4  # the clusters really produce matches
     assert np.array_equal(gm, om)
+    # without match_dist (the timed chain's setting) the same decisions
+    m2 = ph.photon_kernel_match(K, ty, to_device(wt, ph.device), (1, 20), 64, 0, want_dist=False)
+    assert np.array_equal(_np(m2["match"], np.int64), om)
     gd = _np(m["match_dist"], np.float64)
     fin = np.isfinite(od)
     assert np.array_equal(np.isfinite(gd), fin)
