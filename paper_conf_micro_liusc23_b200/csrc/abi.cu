@@ -569,8 +569,8 @@ int photon_analyse(photon_ctx* ctx, const photon_trace* t, void* gws, size_t gws
     for (auto& e : ctx->aev) CK(cudaEventCreateWithFlags(&e, cudaEventDisableTiming), "event");
   }
   cudaStream_t sa = ctx->sa, sb = ctx->sb;
-  cudaEvent_t e_lists = ctx->aev[0], e_sorted = ctx->aev[1], e_filt = ctx->aev[3],
-              e_remap = ctx->aev[4];
+  cudaEvent_t e_lists = ctx->aev[0], e_sorted = ctx->aev[1], e_prep = ctx->aev[2], e_filt = ctx->aev[3],
+              e_remap = ctx->aev[4], e_clear = ctx->aev[5];
   ctx->last_ws = gws;
   TraceDev d = to_dev(t);
   DevErr* err = g.b.err;
@@ -578,9 +578,14 @@ int photon_analyse(photon_ctx* ctx, const photon_trace* t, void* gws, size_t gws
   CK(cudaMemsetAsync(m.err, 0, sizeof(DevErr), s), "memset");
   {
     ProfScope ps(ctx, PHOTON_PROF_PREP, s);
-    CK(launch_ht_clear(g.h.ht, s), "ht_clear");
+    // fork 0: the type table's clear and the offsets check run beside K1 (K1 needs neither: it reads offsets
+    // defensively and the table is first written by the insertion, which joins them)
+    CK(cudaEventRecord(e_prep, s), "event");
+    CK(cudaStreamWaitEvent(sa, e_prep, 0), "event");
+    CK(launch_ht_clear(g.h.ht, sa), "ht_clear");
+    CK(launch_validate_offsets(d, err, sa), "validate");
+    CK(cudaEventRecord(e_clear, sa), "event");
     CK(cudaMemsetAsync(g.ep.count, 0, 8, s), "memset");
-    CK(launch_validate_offsets(d, err, s), "validate");
     CK(launch_table_prep(d, g.b.tb, err, s), "table");
   }
   {
@@ -589,6 +594,7 @@ int photon_analyse(photon_ctx* ctx, const photon_trace* t, void* gws, size_t gws
   }
   {
     ProfScope ps(ctx, PHOTON_PROF_CANON, s);
+    CK(cudaStreamWaitEvent(s, e_clear, 0), "event");  // join fork 0
     CK(launch_entries_insert(g.ep, g.h.ht, err, ctx->num_sms, s), "insert");
     CK(launch_canon_lists(g.h.ht, K, *out, g.h.cw, err, s), "canon");
     // fork 1: the filter profiles, the pair filter and its candidate segments need only the unsorted table and its lists
