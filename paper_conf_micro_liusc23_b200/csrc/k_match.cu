@@ -148,11 +148,27 @@ __global__ void k_sig_prof(uint32_t K, const uint64_t* __restrict__ kto, const u
 // canonicalisation; the bin sums are exact integers, so they equal the sorted rows' sums bit for bit);
 // g and its fp32 copy g / N in the canonical row order are written by the canonical sort itself (k_types.cu
 // emit_sig_row: the sorting warp / CTA sums N_k, the same exact integer).
+// zero (optional): the per-k counters the filter and the exact check fill next (kcnt, ccnt) and the survivor count
+// and filter ticket (n_maybe, ticket) -- zeroed here instead of by separate memset nodes
+struct SegZero {
+  uint32_t* kcnt;
+  uint32_t* ccnt;
+  uint64_t* n_maybe;
+  uint32_t* ticket;
+};
 __global__ void k_prof_slots(uint32_t K, const uint64_t* __restrict__ kto, const uint32_t* __restrict__ list,
                              HashTable ht, uint64_t* __restrict__ mass, float* __restrict__ prof,
-                             double* __restrict__ invn, uint32_t* __restrict__ prof8, DevErr* err) {
+                             double* __restrict__ invn, uint32_t* __restrict__ prof8, DevErr* err, SegZero z) {
   const uint32_t k = (blockIdx.x * blockDim.x + threadIdx.x) >> 5, lane = threadIdx.x & 31;
+  if (z.kcnt && blockIdx.x == 0 && threadIdx.x == 0) {
+    *z.n_maybe = 0;
+    *z.ticket = 0;
+  }
   if (k >= K) return;
+  if (z.kcnt && lane == 0) {
+    z.kcnt[k] = 0u;
+    z.ccnt[k] = 0u;
+  }
   const uint64_t r0 = kto[k], r1 = kto[k + 1];
   uint64_t acc = 0;
   bool over = false;
@@ -932,12 +948,11 @@ void launch_filter_band(ScanArgs a, const MatchWs& mw, cudaStream_t s) {
   const uint64_t jobs = (uint64_t)(NB / FRB) * (NB / FRB + 1) / 2 * FRB + (uint64_t)(NB % FRB) * (NB / FRB + 1);
   note_launch(), k_pair_filter<true><<<(unsigned)jobs, 256, 0, s>>>(a, 0, 0, NB);
 }
-// the fused path's candidate segments: one per k, sized by k's filter survivors (the exact check writes the close
-// ones into it)
-void launch_segments(uint32_t K, const MatchWs& mw, DevErr* err, int num_sms, cudaStream_t s, bool counted = false) {
+// the split path's candidate segments (fused = true): one per k, sized by k's filter survivors (the exact check
+// writes the close ones into it)
+void launch_segments(uint32_t K, const MatchWs& mw, DevErr* err, int num_sms, cudaStream_t s) {
   const unsigned gb = (unsigned)umin64(ceil_div(mw.pair_cap, 256), (uint64_t)num_sms * 64);
   cudaMemsetAsync(mw.close_cnt, 0, sizeof(uint32_t) * K, s);
-  if (counted) return;  // the filter counted its survivors per k and its last CTA scanned them
   cudaMemsetAsync(mw.cand_cnt, 0, sizeof(uint32_t) * K, s);
   note_launch(), k_cand_count<<<gb, 256, 0, s>>>(mw.maybe, mw.pair_cap, mw.n_maybe, K, mw.cand_cnt, err);
   note_launch(), k_cand_scan<<<1, 1024, 0, s>>>(mw.cand_cnt, K, mw.cand_off, mw.cand_cur);
@@ -975,21 +990,18 @@ cudaError_t launch_match_scan(uint32_t K, const uint64_t* kto, const uint64_t* s
 cudaError_t launch_analyse_filter(uint32_t K, const uint64_t* kto, const uint32_t* list, const HashTable& ht,
                                   uint64_t* mass, const uint64_t* wt, photon_match_params p, const MatchWs& mw,
                                   uint64_t* pairs, DevErr* err, int num_sms, cudaStream_t sb) {
-  cudaMemsetAsync(mw.n_maybe, 0, 8, sb);
+  const SegZero z{mw.cand_cnt, mw.close_cnt, mw.n_maybe, mw.flag + 2};
   note_launch(), k_prof_slots<<<(unsigned)ceil_div((uint64_t)K * 32, 256), 256, 0, sb>>>(K, kto, list, ht, mass,
                                                                                        mw.prof, mw.invn, mw.prof8,
-                                                                                       err);
+                                                                                       err, z);
   ScanArgs a = scan_args(K, 0, K, kto, nullptr, mass, wt, p, mw, err);
   a.kcnt = mw.cand_cnt;  // the filter counts its survivors per k (no separate count pass) and its last CTA scans
   a.ticket = mw.flag + 2;  // the counts into the candidate segments (no separate scan launch)
   a.seg_off = mw.cand_off;
   a.seg_cur = mw.cand_cur;
-  cudaMemsetAsync(mw.cand_cnt, 0, sizeof(uint32_t) * K, sb);
-  cudaMemsetAsync(mw.flag + 2, 0, sizeof(uint32_t), sb);
   if (PHOTON_BAND && K <= kBandMaxK) launch_filter_band(a, mw, sb);  // f in [-2040, 2040]: the counting sort's 4096 bins
   else launch_filter(a, sb);
-  launch_segments(K, mw, err, num_sms, sb, true);
-  return cudaGetLastError();
+  return cudaGetLastError();  // the candidate segments: counted and scanned by the filter, close_cnt zeroed above
 }
 cudaError_t launch_analyse_exact(uint32_t K, const uint64_t* kto, const uint64_t* sig, const uint64_t* mass,
                                  const uint64_t* wt, photon_match_params p, const MatchWs& mw, uint64_t* pairs,
