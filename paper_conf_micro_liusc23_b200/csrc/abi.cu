@@ -584,6 +584,10 @@ int photon_analyse(photon_ctx* ctx, const photon_trace* t, void* gws, size_t gws
     CK(cudaStreamWaitEvent(sa, e_prep, 0), "event");
     CK(launch_ht_clear(g.h.ht, sa), "ht_clear");
     CK(launch_validate_offsets(d, err, sa), "validate");
+    // the canonicalisation's and the resolution's per-call counters, zeroed here off the critical path
+    CK(cudaMemsetAsync(g.h.cw.tcount, 0, sizeof(uint32_t) * K, sa), "memset");
+    CK(cudaMemsetAsync(g.h.cw.nbig, 0, 8, sa), "memset");
+    CK(cudaMemsetAsync(m.mw.state, 0, K, sa), "memset");
     CK(cudaEventRecord(e_clear, sa), "event");
     CK(cudaMemsetAsync(g.ep.count, 0, 8, s), "memset");
     CK(launch_table_prep(d, g.b.tb, err, s), "table");
@@ -596,17 +600,17 @@ int photon_analyse(photon_ctx* ctx, const photon_trace* t, void* gws, size_t gws
     ProfScope ps(ctx, PHOTON_PROF_CANON, s);
     CK(cudaStreamWaitEvent(s, e_clear, 0), "event");  // join fork 0
     CK(launch_entries_insert(g.ep, g.h.ht, err, ctx->num_sms, s), "insert");
-    CK(launch_canon_lists(g.h.ht, K, *out, g.h.cw, err, s), "canon");
+    CK(launch_canon_lists(g.h.ht, K, *out, g.h.cw, err, s, /*zeroed=*/true), "canon");
     // fork 1: the filter profiles, the pair filter and its candidate segments need only the unsorted table and its lists
     CK(cudaEventRecord(e_lists, s), "event");
     CK(cudaStreamWaitEvent(sb, e_lists, 0), "event");
     CK(launch_analyse_filter(K, out->kernel_type_off, g.h.cw.list, g.h.ht, m.mass, warps_total, params, m.mw, m.pairs,
-                             m.err, ctx->num_sms, sb),
+                             m.n_pairs, m.err, ctx->num_sms, sb),
        "filter");
     CK(cudaEventRecord(e_filt, sb), "event");
     // the canonical rows with A3 (g and g/N in row order, N summed by the sorting warp / CTA)
     CK(launch_canon_sort(g.h.ht, K, t->kernel_warp_off, nullptr, *out, g.h.cw, ctx->num_sms, s,
-                         SigOut{m.sig, m.mw.sigf}),
+                         SigOut{m.sig, m.mw.sigf}, /*zeroed=*/true),
        "sort");
     // fork 2: the per-warp warp_type write
     CK(cudaEventRecord(e_sorted, s), "event");
@@ -624,7 +628,8 @@ int photon_analyse(photon_ctx* ctx, const photon_trace* t, void* gws, size_t gws
   {
     ProfScope ps(ctx, PHOTON_PROF_RESOLVE, s);
     CK(launch_match_resolve(K, out->kernel_type_off, m.sig, m.mass, warps_total, params, m.pairs, m.mw.pair_cap,
-                            m.n_pairs, m.mw, match, match_dist, m.err, ctx->num_sms, s, /*fused=*/true),
+                            m.n_pairs, m.mw, match, match_dist, m.err, ctx->num_sms, s, /*fused=*/true,
+                            /*zeroed=*/true),
        "resolve");
   }
   CK(cudaStreamWaitEvent(s, e_remap, 0), "event");  // join: everything is ordered before later work on `stream`

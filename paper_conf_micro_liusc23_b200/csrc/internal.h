@@ -118,13 +118,14 @@ cudaError_t launch_match_scan(uint32_t K, const uint64_t* kto, const uint64_t* s
 // photon_analyse: the match split around the canonical sort (k_match.cu)
 cudaError_t launch_analyse_filter(uint32_t K, const uint64_t* kto, const uint32_t* list, const HashTable& ht,
                                   uint64_t* mass, const uint64_t* wt, photon_match_params p, const MatchWs& mw,
-                                  uint64_t* pairs, DevErr* err, int num_sms, cudaStream_t sb);
+                                  uint64_t* pairs, uint64_t* n_pairs, DevErr* err, int num_sms, cudaStream_t sb);
 cudaError_t launch_analyse_exact(uint32_t K, const uint64_t* kto, const uint64_t* sig, const uint64_t* mass,
                                  const uint64_t* wt, photon_match_params p, const MatchWs& mw, uint64_t* pairs,
                                  uint64_t pair_cap, uint64_t* n_pairs, DevErr* err, int num_sms, cudaStream_t s);
 // the canonicalisation in two parts (photon_analyse overlaps work with the second)
+// zeroed: the caller zeroed the per-call counters (cw.tcount / cw.nbig / mw.state) earlier, off the critical path
 cudaError_t launch_canon_lists(const HashTable& ht, uint32_t K, const photon_types& out, const CanonWs& cw,
-                               DevErr* err, cudaStream_t s);
+                               DevErr* err, cudaStream_t s, bool zeroed = false);
 // A3 emitted with the rows (photon_analyse): sig = count * key (u64) and sigf = RN32(sig * RN64(1 / N_k)) in row
 // order, N_k summed by the sorting warp / CTA (nullptr: rows only)
 struct SigOut {
@@ -133,14 +134,14 @@ struct SigOut {
 };
 cudaError_t launch_canon_sort(const HashTable& ht, uint32_t K, const uint64_t* kwo, const uint64_t* kernel_warps,
                               const photon_types& out, const CanonWs& cw, int num_sms, cudaStream_t s,
-                              SigOut so = SigOut{nullptr, nullptr});
+                              SigOut so = SigOut{nullptr, nullptr}, bool zeroed = false);
 // the single-GPU fused A3: signatures + the filter profiles in one pass (launch_match_scan(prof_ready = true))
 cudaError_t launch_sig_prof(uint32_t K, const uint64_t* kto, const uint32_t* type_key, const uint64_t* type_count,
                             uint64_t* sig, uint64_t* mass, const MatchWs& mw, DevErr* err, cudaStream_t s);
 cudaError_t launch_match_resolve(uint32_t K, const uint64_t* kto, const uint64_t* sig, const uint64_t* mass,
                                  const uint64_t* wt, photon_match_params p, const uint64_t* pairs, uint64_t n_pairs,
                                  const uint64_t* n_pairs_dev, const MatchWs& mw, int64_t* match, double* match_dist,
-                                 DevErr* err, int num_sms, cudaStream_t s, bool fused = false);
+                                 DevErr* err, int num_sms, cudaStream_t s, bool fused = false, bool zeroed = false);
 
 // ---- A5 (k_stable.cu) -------------------------------------------------------------------------------------
 size_t stable_ws_bytes(const photon_timing& t);

@@ -155,6 +155,7 @@ struct SegZero {
   uint32_t* ccnt;
   uint64_t* n_maybe;
   uint32_t* ticket;
+  uint64_t* n_pairs;  // the exact check's close-pair count
 };
 __global__ void k_prof_slots(uint32_t K, const uint64_t* __restrict__ kto, const uint32_t* __restrict__ list,
                              HashTable ht, uint64_t* __restrict__ mass, float* __restrict__ prof,
@@ -163,6 +164,7 @@ __global__ void k_prof_slots(uint32_t K, const uint64_t* __restrict__ kto, const
   if (z.kcnt && blockIdx.x == 0 && threadIdx.x == 0) {
     *z.n_maybe = 0;
     *z.ticket = 0;
+    *z.n_pairs = 0;
   }
   if (k >= K) return;
   if (z.kcnt && lane == 0) {
@@ -989,8 +991,8 @@ cudaError_t launch_match_scan(uint32_t K, const uint64_t* kto, const uint64_t* s
 // sort, on the main stream -- g / N in row order and the exact check
 cudaError_t launch_analyse_filter(uint32_t K, const uint64_t* kto, const uint32_t* list, const HashTable& ht,
                                   uint64_t* mass, const uint64_t* wt, photon_match_params p, const MatchWs& mw,
-                                  uint64_t* pairs, DevErr* err, int num_sms, cudaStream_t sb) {
-  const SegZero z{mw.cand_cnt, mw.close_cnt, mw.n_maybe, mw.flag + 2};
+                                  uint64_t* pairs, uint64_t* n_pairs, DevErr* err, int num_sms, cudaStream_t sb) {
+  const SegZero z{mw.cand_cnt, mw.close_cnt, mw.n_maybe, mw.flag + 2, n_pairs};
   note_launch(), k_prof_slots<<<(unsigned)ceil_div((uint64_t)K * 32, 256), 256, 0, sb>>>(K, kto, list, ht, mass,
                                                                                        mw.prof, mw.invn, mw.prof8,
                                                                                        err, z);
@@ -1006,7 +1008,7 @@ cudaError_t launch_analyse_filter(uint32_t K, const uint64_t* kto, const uint32_
 cudaError_t launch_analyse_exact(uint32_t K, const uint64_t* kto, const uint64_t* sig, const uint64_t* mass,
                                  const uint64_t* wt, photon_match_params p, const MatchWs& mw, uint64_t* pairs,
                                  uint64_t pair_cap, uint64_t* n_pairs, DevErr* err, int num_sms, cudaStream_t s) {
-  cudaMemsetAsync(n_pairs, 0, 8, s);
+  // n_pairs was zeroed by k_prof_slots (launch_analyse_filter), which precedes this on the joined streams
   launch_exact(scan_args(K, 0, K, kto, sig, mass, wt, p, mw, err), true, mw, pairs, pair_cap, n_pairs, num_sms, s);
   return cudaGetLastError();
 }
@@ -1014,7 +1016,7 @@ cudaError_t launch_analyse_exact(uint32_t K, const uint64_t* kto, const uint64_t
 cudaError_t launch_match_resolve(uint32_t K, const uint64_t* kto, const uint64_t* sig, const uint64_t* mass,
                                  const uint64_t* wt, photon_match_params p, const uint64_t* pairs, uint64_t n_pairs,
                                  const uint64_t* n_pairs_dev, const MatchWs& mw, int64_t* match, double* match_dist,
-                                 DevErr* err, int num_sms, cudaStream_t s, bool fused) {
+                                 DevErr* err, int num_sms, cudaStream_t s, bool fused, bool zeroed) {
   if (K == 0) return cudaSuccess;
   // candidate segments: fused -- written by k_pair_exact into k's segment (cand_off, close_cnt); else built here
   // from the pair list (cand_off, cand_cnt)
@@ -1035,7 +1037,7 @@ cudaError_t launch_match_resolve(uint32_t K, const uint64_t* kto, const uint64_t
       if (per_sm < 1) per_sm = 1;
     }
     unsigned grid = (unsigned)umin64((uint64_t)per_sm * num_sms, ceil_div((uint64_t)K * 32, 256));
-    cudaMemsetAsync(mw.state, 0, K, s);
+    if (!zeroed) cudaMemsetAsync(mw.state, 0, K, s);
     const uint64_t* off = mw.cand_off;
     const uint32_t* cand = mw.cand;
     void* args[] = {(void*)&K, (void*)&off, (void*)&ccnt, (void*)&cand, (void*)&mw.state, (void*)&mw.flag};

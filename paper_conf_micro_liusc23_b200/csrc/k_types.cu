@@ -549,9 +549,9 @@ cudaError_t launch_ht_clear(const HashTable& ht, cudaStream_t s) {
 }
 
 cudaError_t launch_canon_lists(const HashTable& ht, uint32_t K, const photon_types& out, const CanonWs& cw,
-                               DevErr* err, cudaStream_t s) {
+                               DevErr* err, cudaStream_t s, bool zeroed) {
   uint64_t cap = ht.mask + 1;
-  cudaMemsetAsync(cw.tcount, 0, sizeof(uint32_t) * (K ? K : 1), s);
+  if (!zeroed) cudaMemsetAsync(cw.tcount, 0, sizeof(uint32_t) * (K ? K : 1), s);
   note_launch(), k_count_types<<<(unsigned)ceil_div(cap, 256), 256, 0, s>>>(ht, K, cw.tcount, err);
   note_launch(), k_scan_types<<<1, 1024, 0, s>>>(cw.tcount, K, out.kernel_type_off, cw.cursor, out.capacity, err);
   note_launch(), k_scatter_types<<<(unsigned)ceil_div(cap, 256), 256, 0, s>>>(ht, K, out.kernel_type_off, cw.cursor, cw.list,
@@ -559,8 +559,9 @@ cudaError_t launch_canon_lists(const HashTable& ht, uint32_t K, const photon_typ
   return cudaGetLastError();
 }
 cudaError_t launch_canon_sort(const HashTable& ht, uint32_t K, const uint64_t* kwo, const uint64_t* kernel_warps,
-                              const photon_types& out, const CanonWs& cw, int num_sms, cudaStream_t s, SigOut so) {
-  cudaMemsetAsync(cw.nbig, 0, 8, s);
+                              const photon_types& out, const CanonWs& cw, int num_sms, cudaStream_t s, SigOut so,
+                              bool zeroed) {
+  if (!zeroed) cudaMemsetAsync(cw.nbig, 0, 8, s);
   note_launch(), k_sort_warp<<<(unsigned)ceil_div((uint64_t)K * 32, 256), 256, 0, s>>>(
       ht, K, out.kernel_type_off, cw.list, kwo, kernel_warps, out, cw.canon, cw.big, cw.nbig, so);
   note_launch(), k_sort_mid<<<(unsigned)num_sms, 512, 0, s>>>(ht, K, out.kernel_type_off, cw.list, kwo, kernel_warps,
