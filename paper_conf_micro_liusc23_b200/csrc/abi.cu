@@ -575,7 +575,6 @@ int photon_analyse(photon_ctx* ctx, const photon_trace* t, void* gws, size_t gws
   TraceDev d = to_dev(t);
   DevErr* err = g.b.err;
   CK(cudaMemsetAsync(err, 0, sizeof(DevErr), s), "memset");
-  CK(cudaMemsetAsync(m.err, 0, sizeof(DevErr), s), "memset");
   {
     ProfScope ps(ctx, PHOTON_PROF_PREP, s);
     // fork 0: the type table's clear and the offsets check run beside K1 (K1 needs neither: it reads offsets
@@ -588,6 +587,7 @@ int photon_analyse(photon_ctx* ctx, const photon_trace* t, void* gws, size_t gws
     CK(cudaMemsetAsync(g.h.cw.tcount, 0, sizeof(uint32_t) * K, sa), "memset");
     CK(cudaMemsetAsync(g.h.cw.nbig, 0, 8, sa), "memset");
     CK(cudaMemsetAsync(m.mw.state, 0, K, sa), "memset");
+    CK(cudaMemsetAsync(m.err, 0, sizeof(DevErr), sa), "memset");  // the match part's error word (first latched after the join)
     CK(cudaEventRecord(e_clear, sa), "event");
     CK(cudaMemsetAsync(g.ep.count, 0, 8, s), "memset");
     CK(launch_table_prep(d, g.b.tb, err, s), "table");
