@@ -589,8 +589,7 @@ int photon_analyse(photon_ctx* ctx, const photon_trace* t, void* gws, size_t gws
     CK(cudaMemsetAsync(m.mw.state, 0, K, sa), "memset");
     CK(cudaMemsetAsync(m.err, 0, sizeof(DevErr), sa), "memset");  // the match part's error word (first latched after the join)
     CK(cudaEventRecord(e_clear, sa), "event");
-    CK(cudaMemsetAsync(g.ep.count, 0, 8, s), "memset");
-    CK(launch_table_prep(d, g.b.tb, err, s), "table");
+    CK(launch_table_prep(d, g.b.tb, err, s, g.ep.count), "table");  // also zeroes the entry pool's count
   }
   {
     ProfScope ps(ctx, PHOTON_PROF_BBV_FUSED, s);

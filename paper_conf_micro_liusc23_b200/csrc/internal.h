@@ -45,7 +45,8 @@ struct BbvTables {
   uint32_t* max_len;  // [1] max bb_len (device)
 };
 size_t bbv_table_bytes(uint32_t B);
-cudaError_t launch_table_prep(const TraceDev& t, const BbvTables& tb, DevErr* err, cudaStream_t s);
+cudaError_t launch_table_prep(const TraceDev& t, const BbvTables& tb, DevErr* err, cudaStream_t s,
+                              uint64_t* zero = nullptr);  // zero: a u64 the kernel also zeroes (optional)
 cudaError_t launch_validate_offsets(const TraceDev& t, DevErr* err, cudaStream_t s);
 // K1 (k_bbv3.cu): streaming BBV pass; fused with A2's per-worker de-duplication when ep != nullptr
 cudaError_t launch_bbv3(const TraceDev& t, const BbvTables& tb, uint32_t* warp_bbv16, uint64_t* warp_insts,

@@ -772,8 +772,9 @@ __global__ void __launch_bounds__(WPC * 32, 1) k_group3_from_bbv(Args3 a, const 
 // [B, P2) are marked.  max_len = max bb_len.
 __global__ void k_table_prep3(const uint32_t* __restrict__ bb_len, const uint8_t* __restrict__ bb_bin, uint32_t B,
                               uint32_t P2, uint32_t* __restrict__ tbl_n, uint32_t* __restrict__ tbl_w,
-                              uint32_t* __restrict__ tbl_x, uint32_t* max_len, DevErr* err) {
+                              uint32_t* __restrict__ tbl_x, uint32_t* max_len, DevErr* err, uint64_t* zero) {
   const uint32_t b = blockIdx.x * blockDim.x + threadIdx.x;
+  if (zero && b == 0) *zero = 0;  // the K1 entry pool's count (photon_analyse: one memset node fewer before K1)
   if (b >= P2) return;
   if (b >= B) {
     tbl_n[b] = kMarkN;
@@ -943,11 +944,11 @@ cudaError_t launch3_both(Args3 a, const BbvTables& tb, int num_sms, cudaStream_t
 
 size_t bbv_table_bytes(uint32_t B) { return (size_t)next_pow2_u32(B < 16 ? 16 : B) * 4 + 64; }
 
-cudaError_t launch_table_prep(const TraceDev& t, const BbvTables& tb, DevErr* err, cudaStream_t s) {
+cudaError_t launch_table_prep(const TraceDev& t, const BbvTables& tb, DevErr* err, cudaStream_t s, uint64_t* zero) {
   const uint32_t P2 = next_pow2_u32(t.B < 16 ? 16 : t.B);
   cudaMemsetAsync(tb.max_len, 0, 4, s);
   note_launch(), k_table_prep3<<<(P2 + 255) / 256, 256, 0, s>>>(t.bb_len, t.bb_bin, t.B, P2, tb.neutral, tb.narrow,
-                                                               tb.wide, tb.max_len, err);
+                                                               tb.wide, tb.max_len, err, zero);
   return cudaGetLastError();
 }
 
