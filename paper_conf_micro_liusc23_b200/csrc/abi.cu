@@ -603,8 +603,8 @@ int photon_analyse(photon_ctx* ctx, const photon_trace* t, void* gws, size_t gws
     // fork 1: the filter profiles, the pair filter and its candidate segments need only the unsorted table and its lists
     CK(cudaEventRecord(e_lists, s), "event");
     CK(cudaStreamWaitEvent(sb, e_lists, 0), "event");
-    CK(launch_analyse_filter(K, out->kernel_type_off, g.h.cw.list, g.h.ht, m.mass, warps_total, params, m.mw, m.pairs,
-                             m.n_pairs, m.err, ctx->num_sms, sb),
+    CK(launch_analyse_filter(K, out->kernel_type_off, g.h.cw.list, g.h.ht, m.mass, warps_total, params, m.mw,
+                             m.n_pairs, m.err, sb),
        "filter");
     CK(cudaEventRecord(e_filt, sb), "event");
     // the canonical rows with A3 (g and g/N in row order, N summed by the sorting warp / CTA)

@@ -119,7 +119,7 @@ cudaError_t launch_match_scan(uint32_t K, const uint64_t* kto, const uint64_t* s
 // photon_analyse: the match split around the canonical sort (k_match.cu)
 cudaError_t launch_analyse_filter(uint32_t K, const uint64_t* kto, const uint32_t* list, const HashTable& ht,
                                   uint64_t* mass, const uint64_t* wt, photon_match_params p, const MatchWs& mw,
-                                  uint64_t* pairs, uint64_t* n_pairs, DevErr* err, int num_sms, cudaStream_t sb);
+                                  uint64_t* n_pairs, DevErr* err, cudaStream_t sb);
 cudaError_t launch_analyse_exact(uint32_t K, const uint64_t* kto, const uint64_t* sig, const uint64_t* mass,
                                  const uint64_t* wt, photon_match_params p, const MatchWs& mw, uint64_t* pairs,
                                  uint64_t pair_cap, uint64_t* n_pairs, DevErr* err, int num_sms, cudaStream_t s);

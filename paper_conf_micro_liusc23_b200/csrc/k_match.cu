@@ -991,7 +991,7 @@ cudaError_t launch_match_scan(uint32_t K, const uint64_t* kto, const uint64_t* s
 // sort, on the main stream -- g / N in row order and the exact check
 cudaError_t launch_analyse_filter(uint32_t K, const uint64_t* kto, const uint32_t* list, const HashTable& ht,
                                   uint64_t* mass, const uint64_t* wt, photon_match_params p, const MatchWs& mw,
-                                  uint64_t* pairs, uint64_t* n_pairs, DevErr* err, int num_sms, cudaStream_t sb) {
+                                  uint64_t* n_pairs, DevErr* err, cudaStream_t sb) {
   const SegZero z{mw.cand_cnt, mw.close_cnt, mw.n_maybe, mw.flag + 2, n_pairs};
   note_launch(), k_prof_slots<<<(unsigned)ceil_div((uint64_t)K * 32, 256), 256, 0, sb>>>(K, kto, list, ht, mass,
                                                                                        mw.prof, mw.invn, mw.prof8,
